@@ -1,0 +1,247 @@
+"""Pins for oracle.ops (O2-O8) -- CPU only.  What fixes each value:
+library routines of torch CPU fp64 (F.conv2d, F.max_pool2d, autograd), closed
+forms, invariants and finite differences.  See DESIGN.md."""
+import numpy as np
+import pytest
+import torch
+import torch.nn.functional as F
+
+import synth
+from oracle import ops as O
+from oracle import plan as P
+
+torch.set_default_dtype(torch.float64)
+
+
+def _plan1(k, s, p, cin, cout, H, W, Oh, Ow, op="conv", N=1):
+    l = synth.conv(cin, cout, k, s, p) if op == "conv" else synth.maxpool(cin, k, s, p)
+    return P.plan([l], N, cin, H, W, Oh, Ow).layers[0]
+
+
+def _torch_split_conv(X, Wt, b, lp):
+    """pin-2 composition: per patch F.pad(p_i) + F.conv2d(padding=0), concatenated (Eq. 4-7).
+    Negative pads (k < s, R2) crop, which F.pad does."""
+    rows = []
+    for i in range(len(lp.Ih) - 1):
+        row = []
+        for j in range(len(lp.Iw) - 1):
+            xp = X[:, :, lp.Ih[i]:lp.Ih[i + 1], lp.Iw[j]:lp.Iw[j + 1]]
+            xp = F.pad(xp, (lp.pads_w[j][0], lp.pads_w[j][1], lp.pads_h[i][0], lp.pads_h[i][1]))
+            row.append(F.conv2d(xp, Wt, b, stride=(lp.sh, lp.sw)))
+        rows.append(torch.cat(row, 3))
+    return torch.cat(rows, 2)
+
+
+def _merged_conv(X, W, b, lp, relu=False):
+    Xp = O.split(X, lp.Ih, lp.Iw)
+    return O.merge(O.conv_fwd(Xp, W, b, lp, relu))
+
+
+GEOMS = [  # (k, s, p, H, W, Oh_count, Ow_count)
+    (3, 1, 1, 13, 11, 3, 2),
+    (3, 1, 1, 16, 16, 2, 2),
+    (7, 2, 3, 22, 18, 2, 3),
+    (3, 2, 1, 15, 12, 2, 2),
+    (1, 2, 0, 12, 14, 2, 3),   # k < s downsample (R2)
+    (5, 1, 2, 9, 10, 2, 2),
+]
+
+
+@pytest.mark.parametrize("k,s,p,H,W,nh,nw", GEOMS)
+def test_split_conv_equals_padded_patch_conv_pin2(k, s, p, H, W, nh, nw):
+    g = synth.rng(10 + k)
+    X = synth.uniform(g, (2, 3, H, W)).astype(np.float64)
+    Wt = synth.kaiming(g, 4, 3, k, k).astype(np.float64)
+    b = synth.uniform(g, (4,), -0.1, 0.1).astype(np.float64)
+    Ho, Wo = P.out_len(H, k, s, p, p), P.out_len(W, k, s, p, p)
+    lp = _plan1(k, s, p, 3, 4, H, W, P.boundaries_even(Ho, nh), P.boundaries_even(Wo, nw))
+    got = _merged_conv(X, Wt, b, lp)
+    ref = _torch_split_conv(torch.from_numpy(X), torch.from_numpy(Wt), torch.from_numpy(b), lp).numpy()
+    assert got.shape == ref.shape == (2, 4, Ho, Wo)
+    np.testing.assert_allclose(got, ref, rtol=1e-12, atol=1e-12)
+
+
+@pytest.mark.parametrize("k,s,p", [(3, 1, 1), (7, 2, 3), (1, 2, 0), (3, 2, 1)])
+def test_one_by_one_split_is_ordinary_conv_pin1(k, s, p):
+    """pin-1: with a single patch, p_0 = (p_b, p_e) and Eq. 6 is F.conv2d."""
+    g = synth.rng(20 + k)
+    X = synth.uniform(g, (2, 5, 17, 14)).astype(np.float64)
+    Wt = synth.kaiming(g, 6, 5, k, k).astype(np.float64)
+    b = synth.uniform(g, (6,), -0.1, 0.1).astype(np.float64)
+    Ho, Wo = P.out_len(17, k, s, p, p), P.out_len(14, k, s, p, p)
+    lp = _plan1(k, s, p, 5, 6, 17, 14, [0, Ho], [0, Wo])
+    got = _merged_conv(X, Wt, b, lp, relu=True)
+    ref = F.relu(F.conv2d(torch.from_numpy(X), torch.from_numpy(Wt), torch.from_numpy(b), stride=s, padding=p))
+    np.testing.assert_allclose(got, ref.numpy(), rtol=1e-12, atol=1e-12)
+
+
+def test_interior_outputs_equal_unsplit_pin4_and_independence_pin5():
+    g = synth.rng(3)
+    X = synth.uniform(g, (2, 4, 32, 32)).astype(np.float64)
+    Wt = synth.kaiming(g, 4, 4, 3, 3).astype(np.float64)
+    lp = _plan1(3, 1, 1, 4, 4, 32, 32, [0, 16, 32], [0, 16, 32])
+    got = _merged_conv(X, Wt, None, lp)
+    ref = F.conv2d(torch.from_numpy(X), torch.from_numpy(Wt), padding=1).numpy()
+    keep = np.ones(32, bool)
+    keep[[15, 16]] = False                                    # rows/cols whose window crosses a cut
+    np.testing.assert_allclose(got[:, :, keep][:, :, :, keep], ref[:, :, keep][:, :, :, keep], rtol=1e-13, atol=1e-13)
+    assert not np.allclose(got[:, :, 15], ref[:, :, 15])
+    # pin-5: perturbing patch (1,1)'s input leaves every other patch's output unchanged
+    X2 = X.copy()
+    X2[:, :, 16:, 16:] += synth.uniform(g, (2, 4, 16, 16)).astype(np.float64)
+    got2 = _merged_conv(X2, Wt, None, lp)
+    assert np.array_equal(got2[:, :, :16], got[:, :, :16]) and np.array_equal(got2[:, :, :, :16], got[:, :, :, :16])
+    assert not np.array_equal(got2[:, :, 16:, 16:], got[:, :, 16:, 16:])
+
+
+def test_all_ones_closed_form_pin6():
+    """pin-6 on the C1 geometry: Y = 16 v_h v_w (v = in-patch taps: 3 interior, 2 at a
+    patch edge) -> 144/96/64; dY = 1 gives dX with the same pattern and
+    dW[r,c] = N * sum_patches (P - [r != 1])(P - [c != 1]) -> 2048 / 1920 / 1800."""
+    X = np.ones((2, 16, 32, 32))
+    Wt = np.ones((16, 16, 3, 3))
+    lp = _plan1(3, 1, 1, 16, 16, 32, 32, [0, 16, 32], [0, 16, 32])
+    Y = _merged_conv(X, Wt, None, lp)
+    v = np.full(32, 3.0)
+    v[[0, 15, 16, 31]] = 2.0
+    assert np.array_equal(Y[0, 0], 16 * np.outer(v, v))
+    assert set(np.unique(Y)) == {64.0, 96.0, 144.0}
+    dYp = O.split(np.ones_like(Y), lp.Oh, lp.Ow)
+    dX = O.merge(O.conv_bwd_data(dYp, Wt, lp))
+    assert np.array_equal(dX[1, 3], 16 * np.outer(v, v))
+    dW, db = O.conv_bwd_filter(O.split(X, lp.Ih, lp.Iw), dYp, lp)
+    exp = np.array([[1800, 1920, 1800], [1920, 2048, 1920], [1800, 1920, 1800]], float)
+    assert np.array_equal(dW[5, 7], exp) and np.all(db == 2048)
+
+
+@pytest.mark.parametrize("k,s,p,H,W,nh,nw", GEOMS)
+def test_backward_equals_autograd_of_composition(k, s, p, H, W, nh, nw):
+    """dgrad / wgrad (a4, a5) equal torch autograd of the pin-2 composition (a library
+    routine), including the ReLU-output mask on dX and db = sum dY (R12)."""
+    g = synth.rng(30 + k + s)
+    X = synth.uniform(g, (2, 3, H, W)).astype(np.float64)
+    Wt = synth.kaiming(g, 4, 3, k, k).astype(np.float64)
+    b = synth.uniform(g, (4,), -0.1, 0.1).astype(np.float64)
+    Ho, Wo = P.out_len(H, k, s, p, p), P.out_len(W, k, s, p, p)
+    lp = _plan1(k, s, p, 3, 4, H, W, P.boundaries_even(Ho, nh), P.boundaries_even(Wo, nw))
+    G = synth.normal(g, (2, 4, Ho, Wo)).astype(np.float64)
+    Mask = synth.uniform(g, (2, 3, H, W)).astype(np.float64)  # plays "ReLU output" (positive part)
+    xt = torch.from_numpy(X).requires_grad_()
+    wt = torch.from_numpy(Wt).requires_grad_()
+    bt = torch.from_numpy(b).requires_grad_()
+    (_torch_split_conv(xt, wt, bt, lp) * torch.from_numpy(G)).sum().backward()
+    dYp = O.split(G, lp.Oh, lp.Ow)
+    dX = O.merge(O.conv_bwd_data(dYp, Wt, lp))
+    dXm = O.merge(O.conv_bwd_data(dYp, Wt, lp, O.split(Mask, lp.Ih, lp.Iw)))
+    dW, db = O.conv_bwd_filter(O.split(X, lp.Ih, lp.Iw), dYp, lp)
+    np.testing.assert_allclose(dX, xt.grad.numpy(), rtol=1e-12, atol=1e-12)
+    np.testing.assert_allclose(dXm, np.where(Mask > 0, xt.grad.numpy(), 0), rtol=1e-12, atol=1e-12)
+    np.testing.assert_allclose(dW, wt.grad.numpy(), rtol=1e-11, atol=1e-11)
+    np.testing.assert_allclose(db, bt.grad.numpy(), rtol=1e-12, atol=1e-12)
+
+
+def test_wgrad_linearity_pin10():
+    """pin-10: dW_split = sum over patches of dW of each padded-patch conv, computed
+    independently per patch by torch autograd (Eq. 6 is linear in the patches)."""
+    g = synth.rng(40)
+    X = synth.uniform(g, (1, 2, 10, 9)).astype(np.float64)
+    Wt = synth.kaiming(g, 3, 2, 3, 3).astype(np.float64)
+    lp = _plan1(3, 1, 1, 2, 3, 10, 9, [0, 3, 10], [0, 5, 9])
+    G = synth.normal(g, (1, 3, 10, 9)).astype(np.float64)
+    total = np.zeros_like(Wt)
+    for i in range(2):
+        for j in range(2):
+            wt = torch.from_numpy(Wt).requires_grad_()
+            xp = torch.from_numpy(X[:, :, lp.Ih[i]:lp.Ih[i + 1], lp.Iw[j]:lp.Iw[j + 1]])
+            xp = F.pad(xp, (*lp.pads_w[j], *lp.pads_h[i]))
+            gp = torch.from_numpy(G[:, :, lp.Oh[i]:lp.Oh[i + 1], lp.Ow[j]:lp.Ow[j + 1]])
+            (F.conv2d(xp, wt) * gp).sum().backward()
+            total += wt.grad.numpy()
+    dW, _ = O.conv_bwd_filter(O.split(X, lp.Ih, lp.Iw), O.split(G, lp.Oh, lp.Ow), lp)
+    np.testing.assert_allclose(dW, total, rtol=1e-12, atol=1e-12)
+
+
+def test_finite_differences_pin9():
+    """pin-9: central finite differences in fp64 on N=1, C 2->3, 6x6, boundaries
+    (0,3,6) x (0,2,6), loss = <Y, G> (brute force, no library)."""
+    g = synth.rng(9)
+    X = synth.uniform(g, (1, 2, 6, 6)).astype(np.float64)
+    Wt = synth.kaiming(g, 3, 2, 3, 3).astype(np.float64)
+    lp = _plan1(3, 1, 1, 2, 3, 6, 6, [0, 3, 6], [0, 2, 6])
+    G = synth.normal(g, (1, 3, 6, 6)).astype(np.float64)
+
+    def loss(x, w):
+        return float((_merged_conv(x, w, None, lp) * G).sum())
+
+    dYp = O.split(G, lp.Oh, lp.Ow)
+    dX = O.merge(O.conv_bwd_data(dYp, Wt, lp))
+    dW, _ = O.conv_bwd_filter(O.split(X, lp.Ih, lp.Iw), dYp, lp)
+    h = 1e-6
+    for idx in np.ndindex(X.shape):
+        e = np.zeros_like(X)
+        e[idx] = h
+        fd = (loss(X + e, Wt) - loss(X - e, Wt)) / (2 * h)
+        assert abs(fd - dX[idx]) < 1e-7
+    for idx in np.ndindex(Wt.shape):
+        e = np.zeros_like(Wt)
+        e[idx] = h
+        fd = (loss(X, Wt + e) - loss(X, Wt - e)) / (2 * h)
+        assert abs(fd - dW[idx]) < 1e-7
+
+
+# --------------------------------------------------------------------------- max-pool
+def test_pool_k_eq_s_is_natural_pin3():
+    """pin-3: with k = s and even boundaries the split pool is the unsplit F.max_pool2d,
+    values and indices (after the R8 mapping) bit-exact (P:128-130 + P:122)."""
+    g = synth.rng(50)
+    X = synth.uniform(g, (2, 3, 32, 24)).astype(np.float64)
+    X = np.maximum(X, 0)                                     # ReLU output: many all-zero windows (R9 ties)
+    lp = _plan1(2, 2, 0, 3, 3, 32, 24, [0, 8, 16], [0, 4, 12], op="maxpool")
+    Yp, Ap = O.pool_fwd(O.split(X, lp.Ih, lp.Iw), lp)
+    Y = O.merge(Yp)
+    idx = O.merge([[O.argmax_to_plane_index(Ap[i][j], lp, i, j) for j in range(2)] for i in range(2)])
+    ry, ri = F.max_pool2d(torch.from_numpy(X), 2, 2, return_indices=True)
+    assert np.array_equal(Y, ry.numpy()) and np.array_equal(idx, ri.numpy())
+
+
+def test_pool_padded_overlapping_per_patch():
+    """3x3 s2 p1 (ResNet) per patch == F.max_pool2d of the -inf-padded patch (R7, R9);
+    backward equals autograd of that composition (R10: overlapping windows accumulate)."""
+    g = synth.rng(51)
+    X = synth.uniform(g, (2, 3, 20, 18)).astype(np.float64)
+    Ho, Wo = P.out_len(20, 3, 2, 1, 1), P.out_len(18, 3, 2, 1, 1)
+    lp = _plan1(3, 2, 1, 3, 3, 20, 18, [0, 5, Ho], [0, 4, Wo], op="maxpool")
+    xt = torch.from_numpy(X).requires_grad_()
+    rows = []
+    for i in range(2):
+        row = []
+        for j in range(2):
+            xp = xt[:, :, lp.Ih[i]:lp.Ih[i + 1], lp.Iw[j]:lp.Iw[j + 1]]
+            xp = F.pad(xp, (*lp.pads_w[j], *lp.pads_h[i]), value=-np.inf)
+            row.append(F.max_pool2d(xp, 3, 2))
+        rows.append(torch.cat(row, 3))
+    ref = torch.cat(rows, 2)
+    G = synth.normal(g, tuple(ref.shape)).astype(np.float64)
+    (ref * torch.from_numpy(G)).sum().backward()
+    Yp, Ap = O.pool_fwd(O.split(X, lp.Ih, lp.Iw), lp)
+    assert np.array_equal(O.merge(Yp), ref.detach().numpy())
+    dX = O.merge(O.pool_bwd(O.split(G, lp.Oh, lp.Ow), Ap, lp))
+    np.testing.assert_allclose(dX, xt.grad.numpy(), rtol=1e-14, atol=1e-14)
+
+
+def test_pool_tie_break_first_max_r9():
+    X = np.zeros((1, 1, 2, 2))
+    _, A = O.pool_fwd_patch(X, 2, 2, 2, 2, (0, 0), (0, 0))
+    assert A[0, 0, 0, 0] == 0
+    X = np.array([[[[1.0, 3.0], [3.0, 2.0]]]])
+    _, A = O.pool_fwd_patch(X, 2, 2, 2, 2, (0, 0), (0, 0))
+    assert A[0, 0, 0, 0] == 1
+
+
+def test_split_merge_identity_pin8():
+    g = synth.rng(52)
+    X = synth.uniform(g, (2, 3, 13, 11)).astype(np.float64)
+    for Ih, Iw in [([0, 13], [0, 11]), ([0, 4, 9, 13], [0, 6, 11])]:
+        assert np.array_equal(O.merge(O.split(X, Ih, Iw)), X)
+    assert np.array_equal(O.offload_roundtrip(X), X)
+    assert np.array_equal(O.allreduce_sum([X, 2 * X]), 3 * X)

@@ -1,0 +1,262 @@
+/*
+ * splitcnn.h -- C ABI of the B200-native Split-CNN split window-operator library
+ * (libsplitcnn.so, sm_100a).
+ *
+ * Split-CNN (Jin & Hong, ASPLOS'19; /root/reference/PAPER.md, cited P:<line>)
+ * cuts the input of early CNN layers into spatial patches and runs every
+ * window operator (convolution, max-pool) on each patch independently with
+ * patch-local padding, so no window crosses a patch boundary:
+ *
+ *   I = ComputeInputSplitScheme(k, s, p, O)        Eq. 3, Eq. 1-2
+ *   X_0..X_{N-1} = Split_W(X, I)                   Eq. 4
+ *   p = ComputePadding(k, s, p, O, I)              Eq. 5
+ *   Y_n = Op(X_n, k, s, p_n)                       Eq. 6
+ *   Y = [Y_0..Y_{N-1}]_W                           Eq. 7
+ *   chained layers: O^m = I^{m+1}, no communication between patches
+ *   stochastic boundaries per minibatch
+ *
+ * CONVENTIONS (apply to every call)
+ *  - Every call returns splitcnn_status_t; nothing throws or exits.  On error
+ *    splitcnn_last_error() returns a thread-local message valid until the next
+ *    call on the same thread.
+ *  - Ownership: the caller owns every device / host buffer (PyTorch allocates
+ *    them).  The library owns only splitcnn_plan_t (host memory) and frees it in
+ *    splitcnn_plan_destroy().  Compute calls never allocate device memory; the
+ *    scratch they need is the caller's `ws` (size from splitcnn_workspace_size).
+ *  - Streams: every device call enqueues asynchronously on the given stream and
+ *    never synchronises.  CUDA launch errors map to SPLITCNN_ERR_CUDA.
+ *  - Levels: a plan over L layers has L+1 activation LEVELS; level m is the
+ *    input of layer m, level L the output of the last layer.  At each level the
+ *    activations of the split region live in PATCH BUFFERS: patch (i, j)
+ *    (row-major, i along H, j along W) is a contiguous [N][Hp_i][Wp_j][Cpad]
+ *    array (patch-major NHWC) at element offset
+ *        off(i, j) = N * Cpad * (bh[i] * W + (bh[i+1] - bh[i]) * bw[j])
+ *    from the level's base pointer, where bh / bw are the level's boundaries.
+ *    The whole level occupies N * H * W * Cpad elements.
+ *  - Channel padding: Cpad = C rounded up to a multiple of 8.  Padding channels
+ *    are written as zero by every producer and must be zero in inputs.
+ *  - Weights: [Cout][kh][kw][Cpad_in] in the compute dtype (padding channels
+ *    zero).  Bias: float32 [Cout].  Weight / bias gradients: float32, same
+ *    layouts.
+ *  - Full (unsplit) tensors: logical NCHW, physically NCHW (SPLITCNN_NCHW) or
+ *    NHWC with exactly C channels (SPLITCNN_NHWC).
+ *  - Sharding: every compute call takes a patch range [p0, p1) in row-major
+ *    patch index, so a rank computes only its patches.  The plan is global and
+ *    identical on every rank.  p1 = -1 means "all patches".
+ *  - Alignment: every device pointer must be 16-byte aligned
+ *    (SPLITCNN_ERR_ALIGNMENT otherwise).
+ */
+#ifndef SPLITCNN_H
+#define SPLITCNN_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define SPLITCNN_API __attribute__((visibility("default")))
+#else
+#define SPLITCNN_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st *splitcnn_stream_t; /* == cudaStream_t */
+typedef struct CUevent_st *splitcnn_event_t;   /* == cudaEvent_t  */
+
+typedef enum {
+    SPLITCNN_OK = 0,
+    SPLITCNN_ERR_INVALID_VALUE = 1,
+    SPLITCNN_ERR_ALIGNMENT = 2,
+    SPLITCNN_ERR_UNSUPPORTED = 3,
+    SPLITCNN_ERR_CUDA = 4,
+    SPLITCNN_ERR_OOM = 5
+} splitcnn_status_t;
+
+/* Storage / compute precision of activations and weights.
+ *  BF16: bf16 storage, fp32 accumulation (tcgen05 tensor cores where the shape allows).
+ *  FP32: fp32 storage, fp32-accurate arithmetic (FFMA).  Accumulation is fp32. */
+typedef enum { SPLITCNN_BF16 = 0, SPLITCNN_FP32 = 1 } splitcnn_dtype_t;
+
+typedef enum { SPLITCNN_OP_CONV = 0, SPLITCNN_OP_MAXPOOL = 1 } splitcnn_op_t;
+
+typedef enum { SPLITCNN_NCHW = 0, SPLITCNN_NHWC = 1 } splitcnn_layout_t;
+
+/* flags */
+#define SPLITCNN_FLAG_RELU 0x1u            /* conv_fwd: fuse ReLU into the epilogue */
+#define SPLITCNN_FLAG_POOL_RELU_MASK 0x2u  /* pool_fwd: record [max > 0] in argmax bit 7;
+                                              pool_bwd: multiply dX by that bit (the backward
+                                              of the ReLU feeding the pool)          */
+#define SPLITCNN_FLAG_FORCE_SIMT 0x100u    /* conv calls: use the CUDA-core kernels even where
+                                              the tcgen05 kernel applies (testing)          */
+
+/* One window-based layer Op(X, k, s, p).  Pads are the UNSPLIT layer's. */
+typedef struct {
+    int32_t op;          /* splitcnn_op_t */
+    int32_t kh, kw;      /* window */
+    int32_t sh, sw;      /* stride */
+    int32_t ph_b, ph_e;  /* padding along H: begin, end */
+    int32_t pw_b, pw_e;  /* padding along W */
+    int32_t cin, cout;   /* channels (cin == cout for MAXPOOL) */
+} splitcnn_layer_t;
+
+typedef struct splitcnn_plan_s *splitcnn_plan_t;
+
+#define SPLITCNN_MAX_SPLITS 32   /* patches per spatial dimension */
+
+/* Geometry of one activation level (all pointers point into plan-owned memory). */
+typedef struct {
+    int32_t N, C, Cpad, H, W;
+    int32_t n_h, n_w;         /* patch grid */
+    const int32_t *bh;        /* n_h + 1 boundaries along H (bh[0] = 0, bh[n_h] = H) */
+    const int32_t *bw;        /* n_w + 1 boundaries along W */
+    int64_t total_elems;      /* N * H * W * Cpad: elements of the level's patch buffers */
+} splitcnn_level_t;
+
+/* Geometry of one layer: per-patch pads (Eq. 5, P:139-141 with the R1 reading). */
+typedef struct {
+    splitcnn_layer_t layer;
+    int32_t n_h, n_w;
+    const int32_t *pad_h;     /* 2 * n_h: (begin, end) per patch row    */
+    const int32_t *pad_w;     /* 2 * n_w: (begin, end) per patch column */
+} splitcnn_layer_geom_t;
+
+/* ------------------------------------------------------------------ errors */
+SPLITCNN_API const char *splitcnn_last_error(void);
+SPLITCNN_API const char *splitcnn_status_string(splitcnn_status_t s);
+SPLITCNN_API const char *splitcnn_version(void);
+
+/* ------------------------------------------------------------------ boundaries (host) */
+/* "As evenly as possible": O[i] = floor(i * L / n), O[n] = L.
+ * O has n + 1 entries.  Errors: n < 1, n > L. */
+SPLITCNN_API splitcnn_status_t splitcnn_boundaries_even(int32_t L, int32_t n, int32_t *O);
+
+/* Stochastic splitting: one scheme per minibatch `step` and per spatial
+ * dimension.  s_0 = 0, s_i ~ DiscreteUniform(ceil((i-w)L/n), floor((i+w)L/n)) for i > 0.
+ * RNG: SplitMix64 with state0 = seed ^ (step * 0x9E3779B97F4A7C15); H draws
+ * first (i = 1..nh-1), then W; value = lo + next() % (hi - lo + 1); an empty range
+ * (lo > hi) takes floor(i L / n) without a draw.  Errors: omega outside [0, 0.5). */
+SPLITCNN_API splitcnn_status_t splitcnn_boundaries_random(int32_t Lh, int32_t nh, int32_t Lw, int32_t nw,
+                                             double omega, uint64_t seed, uint64_t step,
+                                             int32_t *O_h, int32_t *O_w);
+
+/* ------------------------------------------------------------------ plan (host) */
+/* Build the chained plan of a split region.  O_h (n_h + 1 entries) and O_w partition the
+ * LAST layer's output; each earlier layer's schemes follow backward:
+ * I_i = s * O_i (R2, within [lb, ub] of Eq. 1-2 whenever p_b <= k - s), pads from Eq. 5,
+ * and O^{m-1} = I^m.  Errors (SPLITCNN_ERR_INVALID_VALUE): O not strictly
+ * increasing, O[0] != 0, O[n] != output length, an empty patch at any level, output
+ * size <= 0, channel chain mismatch, n_h or n_w > SPLITCNN_MAX_SPLITS. */
+SPLITCNN_API splitcnn_status_t splitcnn_plan_create(const splitcnn_layer_t *layers, int32_t nlayers,
+                                       int32_t N, int32_t C, int32_t H, int32_t W,
+                                       const int32_t *O_h, int32_t n_h,
+                                       const int32_t *O_w, int32_t n_w,
+                                       splitcnn_plan_t *out);
+SPLITCNN_API splitcnn_status_t splitcnn_plan_destroy(splitcnn_plan_t plan);
+SPLITCNN_API splitcnn_status_t splitcnn_plan_num_layers(splitcnn_plan_t plan, int32_t *nlayers);
+SPLITCNN_API splitcnn_status_t splitcnn_plan_level(splitcnn_plan_t plan, int32_t level, splitcnn_level_t *out);
+SPLITCNN_API splitcnn_status_t splitcnn_plan_layer(splitcnn_plan_t plan, int32_t layer, splitcnn_layer_geom_t *out);
+
+/* Scratch bytes needed by a compute call (op: 0 = conv_fwd, 1 = conv_bwd_data,
+ * 2 = conv_bwd_filter); 0 when none is needed. */
+SPLITCNN_API splitcnn_status_t splitcnn_workspace_size(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                          int32_t op, size_t *bytes);
+
+/* ------------------------------------------------------------------ split / merge */
+/* Eq. 4: copy the full tensor x (level `level`'s N, C, H, W; layout x_layout) into
+ * the level's patch buffers (+ transpose to NHWC, + zero channel padding). */
+SPLITCNN_API splitcnn_status_t splitcnn_split(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                 const void *x, int32_t x_layout, void *patches,
+                                 int32_t p0, int32_t p1, splitcnn_stream_t stream);
+
+/* Eq. 7: concatenate the level's patch buffers into the full tensor y. */
+SPLITCNN_API splitcnn_status_t splitcnn_merge(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                 const void *patches, void *y, int32_t y_layout,
+                                 int32_t p0, int32_t p1, splitcnn_stream_t stream);
+
+/* ------------------------------------------------------------------ convolution */
+/* Forward, Eq. 6: for every patch in [p0, p1),
+ *   Y_p[n,oh,ow,co] = act(bias[co] + sum_{r,c,ci} X~_p[n, oh*sh - pt + r, ow*sw - pl + c, ci] W[co,r,c,ci])
+ * with X~_p the patch zero-padded by its own pads (pt, pl = the patch's begin pads).
+ * x: level `layer` patches; y: level `layer + 1` patches; bias nullable; flags: RELU.
+ * Errors: layer is not a conv. */
+SPLITCNN_API splitcnn_status_t splitcnn_conv_fwd(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                    const void *x, const void *w, const float *bias, void *y,
+                                    uint32_t flags, int32_t p0, int32_t p1, splitcnn_stream_t stream);
+
+/* Data gradient (adjoint of Eq. 6 within each patch):
+ *   dX_p[n,h,w,ci] = sum over co, r, c with oh = (h + pt - r)/sh integral and in range
+ *                    of dY_p[n,oh,ow,co] W[co,r,c,ci],   then * [relu_src > 0] if relu_src.
+ * dy: level layer+1; dx, relu_src (nullable): level `layer`.  ws: splitcnn_workspace_size(op=1). */
+SPLITCNN_API splitcnn_status_t splitcnn_conv_bwd_data(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                         const void *dy, const void *w, void *dx, const void *relu_src,
+                                         void *ws, size_t ws_bytes, uint32_t flags,
+                                         int32_t p0, int32_t p1, splitcnn_stream_t stream);
+
+/* Weight gradient summed over the patches [p0, p1) and the batch:
+ *   dW[co,r,c,ci] = beta * dW + sum_p sum_{n,oh,ow} dY_p[n,oh,ow,co] X~_p[n, oh*sh-pt+r, ow*sw-pl+c, ci]
+ *   db[co]        = beta * db + sum_p sum_{n,oh,ow} dY_p[n,oh,ow,co]          (db nullable)
+ * beta is 0 (overwrite) or 1 (accumulate).  The summation order is fixed (deterministic
+ * run to run).  ws: splitcnn_workspace_size(op=2); ERR_INVALID_VALUE if too small. */
+SPLITCNN_API splitcnn_status_t splitcnn_conv_bwd_filter(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                           const void *x, const void *dy, float *dw, float *db,
+                                           float beta, void *ws, size_t ws_bytes, uint32_t flags,
+                                           int32_t p0, int32_t p1, splitcnn_stream_t stream);
+
+/* ------------------------------------------------------------------ max-pool */
+/* Forward (Eq. 6 with Op = max-pool): the max over the in-patch window elements (padding
+ * is -inf) and its argmax as uint8 window-local index r*kw + c of the FIRST
+ * maximum in row-major window order (R8, R9).  With FLAG_POOL_RELU_MASK bit 7 of the
+ * argmax byte holds [max > 0].  x: level layer; y, argmax: level layer+1 ([N][Ho][Wo][Cpad]
+ * bytes per patch, same offsets as y).  Errors: kh * kw > 127. */
+SPLITCNN_API splitcnn_status_t splitcnn_pool_fwd(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                    const void *x, void *y, uint8_t *argmax, uint32_t flags,
+                                    int32_t p0, int32_t p1, splitcnn_stream_t stream);
+
+/* Backward: dX_p[argmax] += dY_p (summed in fp32 when windows overlap, R10); every element of
+ * dx is written (no memset needed).  With FLAG_POOL_RELU_MASK, dX is multiplied by bit 7. */
+SPLITCNN_API splitcnn_status_t splitcnn_pool_bwd(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                    const void *dy, const uint8_t *argmax, void *dx, uint32_t flags,
+                                    int32_t p0, int32_t p1, splitcnn_stream_t stream);
+
+/* ------------------------------------------------------------------ offload / prefetch */
+/* Patch-granular activation offload (HMMS): after `ready` (recorded by the caller
+ * on the compute stream after the buffer's last write, moment 1) copy patch `patch` of level
+ * `level` (its contiguous [N][Hp][Wp][Cpad] bytes) to host_pinned on mem_stream and record
+ * `done` (the caller makes the compute stream wait on `done` before freeing / overwriting,
+ * moment 2).  ready / done nullable.  host_pinned must be page-locked (ERR_INVALID_VALUE). */
+SPLITCNN_API splitcnn_status_t splitcnn_offload(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                   int32_t patch, const void *dev_patches, void *host_pinned,
+                                   splitcnn_event_t ready, splitcnn_stream_t mem_stream,
+                                   splitcnn_event_t done);
+/* Prefetch (moments 3-4): host_pinned -> the patch's device bytes on mem_stream after `ready`,
+ * then record `done` (the compute stream waits on it before the first backward use). */
+SPLITCNN_API splitcnn_status_t splitcnn_prefetch(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                    int32_t patch, const void *host_pinned, void *dev_patches,
+                                    splitcnn_event_t ready, splitcnn_stream_t mem_stream,
+                                    splitcnn_event_t done);
+/* Byte size / byte offset of one patch buffer at a level. */
+SPLITCNN_API splitcnn_status_t splitcnn_patch_bytes(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                       int32_t patch, size_t *offset, size_t *bytes);
+
+/* ------------------------------------------------------------------ offload planning (host) */
+/* Algorithm 1 and the reverse prefetch pass, SURVEY R15.
+ * Inputs, per serialized forward op t = 0..T-1: op_time_s[t] (profiled seconds),
+ * cand_bytes[t] = bytes of the TSO (patch buffer) that becomes offloadable at op t (0: none),
+ * bw_bytes_per_s = measured host-link bandwidth.
+ * Outputs: offload[t] = 1 if that TSO is offloaded; sync_at[t] = 1 if op t is an
+ * "end of offload" point (compute waits for all outstanding offloads, then frees them);
+ * for the backward list (op_time_bwd_s, need_bytes[t] = bytes first needed at backward op t),
+ * prefetch_start[t] = the backward op index at which the prefetch for need t starts (-1 none).
+ * The ratio cap: an offload is skipped if cumulative offloaded bytes would exceed
+ * sum(op_time) * bw. */
+SPLITCNN_API splitcnn_status_t splitcnn_offload_plan(int32_t T, const double *op_time_s, const int64_t *cand_bytes,
+                                        double bw_bytes_per_s, int32_t *offload, int32_t *sync_at);
+SPLITCNN_API splitcnn_status_t splitcnn_prefetch_plan(int32_t T, const double *op_time_bwd_s, const int64_t *need_bytes,
+                                         double bw_bytes_per_s, int32_t *prefetch_start);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SPLITCNN_H */

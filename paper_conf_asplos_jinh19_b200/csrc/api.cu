@@ -1,0 +1,338 @@
+// api.cu -- the extern "C" entry points of libsplitcnn (see include/splitcnn.h).
+// Argument validation, error plumbing and kernel dispatch; all arithmetic is in the kernels.
+#include <cstdio>
+#include <cstring>
+#include <string>
+
+#include "kernels.h"
+
+namespace splitcnn {
+
+static thread_local std::string g_last_error;
+
+void set_error(const std::string &msg) { g_last_error = msg; }
+
+splitcnn_status_t fail(splitcnn_status_t s, const std::string &msg) {
+    g_last_error = msg;
+    return s;
+}
+
+splitcnn_status_t check_launch(const char *what) {
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+    return SPLITCNN_OK;
+}
+
+}  // namespace splitcnn
+
+using namespace splitcnn;
+
+extern "C" const char *splitcnn_last_error(void) { return g_last_error.c_str(); }
+
+extern "C" const char *splitcnn_status_string(splitcnn_status_t s) {
+    switch (s) {
+        case SPLITCNN_OK: return "ok";
+        case SPLITCNN_ERR_INVALID_VALUE: return "invalid value";
+        case SPLITCNN_ERR_ALIGNMENT: return "misaligned pointer";
+        case SPLITCNN_ERR_UNSUPPORTED: return "unsupported";
+        case SPLITCNN_ERR_CUDA: return "CUDA error";
+        case SPLITCNN_ERR_OOM: return "out of memory";
+    }
+    return "unknown status";
+}
+
+extern "C" const char *splitcnn_version(void) { return "splitcnn-b200 0.1 (sm_100a)"; }
+
+namespace {
+
+bool aligned16(const void *p) { return ((uintptr_t)p & 15u) == 0; }
+
+splitcnn_status_t check_dtype(splitcnn_dtype_t dt) {
+    if (dt != SPLITCNN_BF16 && dt != SPLITCNN_FP32) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad dtype");
+    return SPLITCNN_OK;
+}
+
+splitcnn_status_t check_range(const splitcnn_plan_t plan, int level, int &p0, int &p1) {
+    const Level &L = plan->levels[level];
+    if (p1 < 0) p1 = L.npatch();
+    if (p0 < 0 || p0 > p1 || p1 > L.npatch()) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad patch range");
+    return SPLITCNN_OK;
+}
+
+splitcnn_status_t check_layer(const splitcnn_plan_t plan, int layer, int op) {
+    if (!plan) return fail(SPLITCNN_ERR_INVALID_VALUE, "null plan");
+    if (layer < 0 || layer >= (int)plan->layers.size()) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad layer index");
+    if (plan->layers[layer].L.op != op)
+        return fail(SPLITCNN_ERR_INVALID_VALUE, op == SPLITCNN_OP_CONV ? "layer is not a convolution" : "layer is not a max-pool");
+    return SPLITCNN_OK;
+}
+
+#define TRY(x)                                  \
+    do {                                        \
+        splitcnn_status_t _s = (x);             \
+        if (_s != SPLITCNN_OK) return _s;       \
+    } while (0)
+
+#define NEED_ALIGNED(p, name)                                                              \
+    do {                                                                                   \
+        if ((p) && !aligned16(p)) return fail(SPLITCNN_ERR_ALIGNMENT, name " must be 16-byte aligned"); \
+    } while (0)
+
+}  // namespace
+
+extern "C" splitcnn_status_t splitcnn_workspace_size(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                                     int32_t op, size_t *bytes) {
+    if (!bytes) return fail(SPLITCNN_ERR_INVALID_VALUE, "null bytes");
+    TRY(check_dtype(dtype));
+    TRY(check_layer(plan, layer, SPLITCNN_OP_CONV));
+    const Level &Li = plan->levels[layer], &Lo = plan->levels[layer + 1];
+    const LayerGeom &g = plan->layers[layer];
+    size_t b = 0;
+    if (op == 1) {
+        if (conv_tc_supported(1, dtype, Li, Lo, g)) b = conv_tc_ws_bytes(1, Li, Lo, g);
+    } else if (op == 2) {
+        b = wgrad_simt_ws_bytes(Li, Lo, g);
+        if (conv_tc_supported(2, dtype, Li, Lo, g)) b = std::max(b, conv_tc_ws_bytes(2, Li, Lo, g));
+    } else if (op != 0) {
+        return fail(SPLITCNN_ERR_INVALID_VALUE, "workspace_size: op must be 0, 1 or 2");
+    }
+    *bytes = b;
+    return SPLITCNN_OK;
+}
+
+extern "C" splitcnn_status_t splitcnn_split(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype, const void *x,
+                                            int32_t x_layout, void *patches, int32_t p0, int32_t p1,
+                                            splitcnn_stream_t stream) {
+    if (!plan || level < 0 || level >= (int)plan->levels.size()) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad level");
+    TRY(check_dtype(dtype));
+    if (!x || !patches) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    if (x_layout != SPLITCNN_NCHW && x_layout != SPLITCNN_NHWC) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad layout");
+    NEED_ALIGNED(x, "x");
+    NEED_ALIGNED(patches, "patches");
+    TRY(check_range(plan, level, p0, p1));
+    if (p1 == p0) return SPLITCNN_OK;
+    launch_split(dtype, plan->levels[level], x, x_layout, patches, p0, p1, (cudaStream_t)stream);
+    return check_launch("split");
+}
+
+extern "C" splitcnn_status_t splitcnn_merge(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                            const void *patches, void *y, int32_t y_layout, int32_t p0, int32_t p1,
+                                            splitcnn_stream_t stream) {
+    if (!plan || level < 0 || level >= (int)plan->levels.size()) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad level");
+    TRY(check_dtype(dtype));
+    if (!y || !patches) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    if (y_layout != SPLITCNN_NCHW && y_layout != SPLITCNN_NHWC) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad layout");
+    NEED_ALIGNED(y, "y");
+    NEED_ALIGNED(patches, "patches");
+    TRY(check_range(plan, level, p0, p1));
+    if (p1 == p0) return SPLITCNN_OK;
+    launch_merge(dtype, plan->levels[level], patches, y, y_layout, p0, p1, (cudaStream_t)stream);
+    return check_launch("merge");
+}
+
+extern "C" splitcnn_status_t splitcnn_conv_fwd(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype, const void *x,
+                                               const void *w, const float *bias, void *y, uint32_t flags, int32_t p0,
+                                               int32_t p1, splitcnn_stream_t stream) {
+    TRY(check_layer(plan, layer, SPLITCNN_OP_CONV));
+    TRY(check_dtype(dtype));
+    if (!x || !w || !y) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    NEED_ALIGNED(x, "x");
+    NEED_ALIGNED(w, "w");
+    NEED_ALIGNED(y, "y");
+    TRY(check_range(plan, layer, p0, p1));
+    if (p1 == p0) return SPLITCNN_OK;
+    const Level &Li = plan->levels[layer], &Lo = plan->levels[layer + 1];
+    const LayerGeom &g = plan->layers[layer];
+    const int relu = (flags & SPLITCNN_FLAG_RELU) ? 1 : 0;
+    if (!(flags & SPLITCNN_FLAG_FORCE_SIMT) && conv_tc_supported(0, dtype, Li, Lo, g)) {
+        TRY(launch_conv_fwd_tc(Li, Lo, g, x, w, bias, y, relu, p0, p1, (cudaStream_t)stream));
+    } else {
+        launch_conv_fwd_simt(dtype, Li, Lo, g, x, w, bias, y, relu, p0, p1, (cudaStream_t)stream);
+    }
+    return check_launch("conv_fwd");
+}
+
+extern "C" splitcnn_status_t splitcnn_conv_bwd_data(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                                    const void *dy, const void *w, void *dx, const void *relu_src,
+                                                    void *ws, size_t ws_bytes, uint32_t flags, int32_t p0, int32_t p1,
+                                                    splitcnn_stream_t stream) {
+    TRY(check_layer(plan, layer, SPLITCNN_OP_CONV));
+    TRY(check_dtype(dtype));
+    if (!dy || !w || !dx) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    NEED_ALIGNED(dy, "dy");
+    NEED_ALIGNED(w, "w");
+    NEED_ALIGNED(dx, "dx");
+    NEED_ALIGNED(relu_src, "relu_src");
+    NEED_ALIGNED(ws, "ws");
+    TRY(check_range(plan, layer, p0, p1));
+    if (p1 == p0) return SPLITCNN_OK;
+    const Level &Li = plan->levels[layer], &Lo = plan->levels[layer + 1];
+    const LayerGeom &g = plan->layers[layer];
+    if (!(flags & SPLITCNN_FLAG_FORCE_SIMT) && conv_tc_supported(1, dtype, Li, Lo, g)) {
+        const size_t need = conv_tc_ws_bytes(1, Li, Lo, g);
+        if (ws_bytes < need || (need && !ws)) return fail(SPLITCNN_ERR_INVALID_VALUE, "conv_bwd_data: workspace too small");
+        TRY(launch_conv_dgrad_tc(Li, Lo, g, dy, w, dx, relu_src, ws, p0, p1, (cudaStream_t)stream));
+    } else {
+        launch_conv_dgrad_simt(dtype, Li, Lo, g, dy, w, dx, relu_src, p0, p1, (cudaStream_t)stream);
+    }
+    return check_launch("conv_bwd_data");
+}
+
+extern "C" splitcnn_status_t splitcnn_conv_bwd_filter(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                                      const void *x, const void *dy, float *dw, float *db, float beta,
+                                                      void *ws, size_t ws_bytes, uint32_t flags, int32_t p0, int32_t p1,
+                                                      splitcnn_stream_t stream) {
+    TRY(check_layer(plan, layer, SPLITCNN_OP_CONV));
+    TRY(check_dtype(dtype));
+    if (!x || !dy || !dw) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    if (beta != 0.f && beta != 1.f) return fail(SPLITCNN_ERR_INVALID_VALUE, "beta must be 0 or 1");
+    NEED_ALIGNED(x, "x");
+    NEED_ALIGNED(dy, "dy");
+    NEED_ALIGNED(dw, "dw");
+    NEED_ALIGNED(ws, "ws");
+    TRY(check_range(plan, layer, p0, p1));
+    const Level &Li = plan->levels[layer], &Lo = plan->levels[layer + 1];
+    const LayerGeom &g = plan->layers[layer];
+    const bool tc = !(flags & SPLITCNN_FLAG_FORCE_SIMT) && conv_tc_supported(2, dtype, Li, Lo, g);
+    const size_t need = tc ? conv_tc_ws_bytes(2, Li, Lo, g) : wgrad_simt_ws_bytes(Li, Lo, g);
+    if (ws_bytes < need || !ws) return fail(SPLITCNN_ERR_INVALID_VALUE, "conv_bwd_filter: workspace too small");
+    if (tc) {
+        TRY(launch_conv_wgrad_tc(Li, Lo, g, x, dy, dw, db, beta, ws, p0, p1, (cudaStream_t)stream));
+    } else {
+        launch_conv_wgrad_simt(dtype, Li, Lo, g, x, dy, dw, db, beta, ws, p0, p1, (cudaStream_t)stream);
+    }
+    return check_launch("conv_bwd_filter");
+}
+
+extern "C" splitcnn_status_t splitcnn_pool_fwd(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype, const void *x,
+                                               void *y, uint8_t *argmax, uint32_t flags, int32_t p0, int32_t p1,
+                                               splitcnn_stream_t stream) {
+    TRY(check_layer(plan, layer, SPLITCNN_OP_MAXPOOL));
+    TRY(check_dtype(dtype));
+    if (!x || !y || !argmax) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    NEED_ALIGNED(x, "x");
+    NEED_ALIGNED(y, "y");
+    NEED_ALIGNED(argmax, "argmax");
+    TRY(check_range(plan, layer, p0, p1));
+    if (p1 == p0) return SPLITCNN_OK;
+    launch_pool_fwd(dtype, plan->levels[layer], plan->levels[layer + 1], plan->layers[layer], x, y, argmax,
+                    (flags & SPLITCNN_FLAG_POOL_RELU_MASK) ? 1 : 0, p0, p1, (cudaStream_t)stream);
+    return check_launch("pool_fwd");
+}
+
+extern "C" splitcnn_status_t splitcnn_pool_bwd(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype, const void *dy,
+                                               const uint8_t *argmax, void *dx, uint32_t flags, int32_t p0, int32_t p1,
+                                               splitcnn_stream_t stream) {
+    TRY(check_layer(plan, layer, SPLITCNN_OP_MAXPOOL));
+    TRY(check_dtype(dtype));
+    if (!dy || !dx || !argmax) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    NEED_ALIGNED(dy, "dy");
+    NEED_ALIGNED(dx, "dx");
+    NEED_ALIGNED(argmax, "argmax");
+    TRY(check_range(plan, layer, p0, p1));
+    if (p1 == p0) return SPLITCNN_OK;
+    launch_pool_bwd(dtype, plan->levels[layer], plan->levels[layer + 1], plan->layers[layer], dy, argmax, dx,
+                    (flags & SPLITCNN_FLAG_POOL_RELU_MASK) ? 1 : 0, p0, p1, (cudaStream_t)stream);
+    return check_launch("pool_bwd");
+}
+
+// ------------------------------------------------------------------ offload / prefetch
+extern "C" splitcnn_status_t splitcnn_patch_bytes(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                                  int32_t patch, size_t *offset, size_t *bytes) {
+    if (!plan || level < 0 || level >= (int)plan->levels.size()) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad level");
+    TRY(check_dtype(dtype));
+    const Level &L = plan->levels[level];
+    if (patch < 0 || patch >= L.npatch()) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad patch");
+    const size_t es = dtype == SPLITCNN_BF16 ? 2 : 4;
+    const int i = patch / L.nw(), j = patch % L.nw();
+    if (offset) *offset = (size_t)L.offset(i, j) * es;
+    if (bytes) *bytes = (size_t)L.patch_elems(i, j) * es;
+    return SPLITCNN_OK;
+}
+
+static splitcnn_status_t copy_patch(splitcnn_plan_t plan, int level, splitcnn_dtype_t dtype, int patch, const void *src,
+                                    void *dst, bool d2h, splitcnn_event_t ready, splitcnn_stream_t st,
+                                    splitcnn_event_t done) {
+    size_t off = 0, bytes = 0;
+    TRY(splitcnn_patch_bytes(plan, level, dtype, patch, &off, &bytes));
+    if (!src || !dst) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    const void *host = d2h ? dst : src;
+    cudaPointerAttributes attr;
+    if (cudaPointerGetAttributes(&attr, host) != cudaSuccess || attr.type != cudaMemoryTypeHost) {
+        cudaGetLastError();
+        return fail(SPLITCNN_ERR_INVALID_VALUE, "host buffer is not page-locked (pinned)");
+    }
+    cudaStream_t s = (cudaStream_t)st;
+    if (ready && cudaStreamWaitEvent(s, (cudaEvent_t)ready, 0) != cudaSuccess) return check_launch("offload: wait");
+    cudaError_t e;
+    if (d2h) e = cudaMemcpyAsync(dst, (const char *)src + off, bytes, cudaMemcpyDeviceToHost, s);
+    else e = cudaMemcpyAsync((char *)dst + off, src, bytes, cudaMemcpyHostToDevice, s);
+    if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("offload copy: ") + cudaGetErrorString(e));
+    if (done && cudaEventRecord((cudaEvent_t)done, s) != cudaSuccess) return check_launch("offload: record");
+    return SPLITCNN_OK;
+}
+
+extern "C" splitcnn_status_t splitcnn_offload(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype, int32_t patch,
+                                              const void *dev_patches, void *host_pinned, splitcnn_event_t ready,
+                                              splitcnn_stream_t mem_stream, splitcnn_event_t done) {
+    return copy_patch(plan, level, dtype, patch, dev_patches, host_pinned, true, ready, mem_stream, done);
+}
+
+extern "C" splitcnn_status_t splitcnn_prefetch(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype, int32_t patch,
+                                               const void *host_pinned, void *dev_patches, splitcnn_event_t ready,
+                                               splitcnn_stream_t mem_stream, splitcnn_event_t done) {
+    return copy_patch(plan, level, dtype, patch, host_pinned, dev_patches, false, ready, mem_stream, done);
+}
+
+// ------------------------------------------------------------------ Algorithm 1 + reverse
+extern "C" splitcnn_status_t splitcnn_offload_plan(int32_t T, const double *op_time_s, const int64_t *cand_bytes,
+                                                   double bw, int32_t *offload, int32_t *sync_at) {
+    if (T < 1 || !op_time_s || !cand_bytes || !offload || !sync_at || !(bw > 0))
+        return fail(SPLITCNN_ERR_INVALID_VALUE, "offload_plan: bad argument");
+    double cap = 0;  // theoretical limit: sum of t_op * BW
+    for (int t = 0; t < T; ++t) cap += op_time_s[t] * bw;
+    double balance = 0, offloaded = 0;
+    int pending = 0;
+    for (int t = 0; t < T; ++t) {
+        offload[t] = 0;
+        sync_at[t] = 0;
+        if (cand_bytes[t] > 0 && offloaded + (double)cand_bytes[t] <= cap) {  // ratio cap (R15)
+            offload[t] = 1;
+            ++pending;
+            balance -= (double)cand_bytes[t];  // loss = TSO size
+            offloaded += (double)cand_bytes[t];
+        }
+        balance += op_time_s[t] * bw;  // gain = t_op * BW
+        if (balance >= 0 || t == T - 1) {
+            if (pending) sync_at[t] = 1;  // end of offload for every TSO in TSO_to_free
+            pending = 0;
+            balance = 0;  // R15: no outstanding copy -> no carried capacity
+        }
+    }
+    return SPLITCNN_OK;
+}
+
+extern "C" splitcnn_status_t splitcnn_prefetch_plan(int32_t T, const double *op_time_s, const int64_t *need_bytes,
+                                                    double bw, int32_t *prefetch_start) {
+    if (T < 1 || !op_time_s || !need_bytes || !prefetch_start || !(bw > 0))
+        return fail(SPLITCNN_ERR_INVALID_VALUE, "prefetch_plan: bad argument");
+    double balance = 0;
+    std::vector<int> pend;
+    for (int t = 0; t < T; ++t) prefetch_start[t] = -1;
+    for (int t = T - 1; t >= 0; --t) {
+        if (!pend.empty()) {
+            balance += op_time_s[t] * bw;  // op t runs while the prefetch is in flight
+            if (balance >= 0) {
+                for (int u : pend) prefetch_start[u] = t;
+                pend.clear();
+                balance = 0;
+            }
+        }
+        if (need_bytes[t] > 0) {
+            pend.push_back(t);
+            balance -= (double)need_bytes[t];
+        }
+    }
+    for (int u : pend) prefetch_start[u] = 0;  // cannot be hidden: start at the first backward op
+    return SPLITCNN_OK;
+}

@@ -1,0 +1,304 @@
+// k_conv_simt.cu -- CUDA-core (FFMA, fp32 accumulate) split convolution kernels.
+//
+// These are the fp32-accurate path (SPLITCNN_FP32) and the general fallback for shapes the
+// tcgen05 kernel does not take.  Each pass is an implicit GEMM over ONE patch at a time
+// (grid.z = patch), reading the patch-major NHWC buffers directly; taps that fall outside the
+// patch read zero, which is exactly the patch-local padding of Eq. 6.
+//
+//   FWD   : M = N*Ho*Wo pixels, N = Cout, K = kh*kw*Cin_pad;  A = X~_p (gather), B = W^T
+//   DGRAD : M = N*Hp*Wp pixels, N = Cin_pad, K = kh*kw*Cout_pad; A = dY_p (strided gather), B = W
+//   WGRAD : M = Cout, N = kh*kw*Cin_pad, K = pixels of one chunk of one patch (split-K);
+//           partials -> workspace -> fixed-order reduction (deterministic)
+#include "common.cuh"
+#include "kernels.h"
+
+namespace splitcnn {
+
+enum { MODE_FWD = 0, MODE_DGRAD = 1, MODE_WGRAD = 2 };
+
+struct SimtArgs {
+    LevelDesc Li, Lo;
+    LayerDesc ly;
+    const void *x;        // FWD: X (level m); DGRAD: dY (level m+1); WGRAD: dY
+    const void *w;        // weights [Cout][kh][kw][Cin_pad]   (WGRAD: X, level m)
+    const float *bias;
+    void *y;              // FWD: Y (level m+1); DGRAD: dX (level m); WGRAD: float partials
+    const void *relu_src; // DGRAD mask (level m)
+    int Cout;             // true output channels of the layer
+    int relu;
+    int p0;
+    int cpp;              // WGRAD: chunks per patch
+};
+
+constexpr int BM = 64, BN = 64, BK = 8, NT = 256;
+
+template <typename T, int MODE>
+__global__ void __launch_bounds__(NT) conv_simt_kernel(SimtArgs a) {
+    __shared__ float As[2][BK][BM + 4];
+    __shared__ float Bs[2][BK][BN + 4];
+
+    const int tid = threadIdx.x;
+    const int zq = blockIdx.z;
+    const int q = a.p0 + (MODE == MODE_WGRAD ? zq / a.cpp : zq);
+    const PatchGeo gi = patch_geo(a.Li, q), go = patch_geo(a.Lo, q);
+    const int pt = a.ly.pad_h[2 * gi.i], pl = a.ly.pad_w[2 * gi.j];
+    const int kh = a.ly.kh, kw = a.ly.kw, sh = a.ly.sh, sw = a.ly.sw;
+    const int Cpi = a.Li.Cpad, Cpo = a.Lo.Cpad, N = a.Li.N;
+
+    int M, Ncols, Ktot, kbeg = 0;
+    if (MODE == MODE_FWD) { M = N * go.hp * go.wp; Ncols = Cpo; Ktot = kh * kw * Cpi; }
+    else if (MODE == MODE_DGRAD) { M = N * gi.hp * gi.wp; Ncols = Cpi; Ktot = kh * kw * Cpo; }
+    else {
+        M = a.Cout; Ncols = kh * kw * Cpi;
+        const int P = N * go.hp * go.wp;
+        const int chunk = (P + a.cpp - 1) / a.cpp;
+        kbeg = (zq % a.cpp) * chunk;
+        Ktot = min(P, kbeg + chunk);
+    }
+    const int m0 = blockIdx.x * BM, n0 = blockIdx.y * BN;
+    if (m0 >= M || n0 >= Ncols) {
+        if (MODE != MODE_WGRAD) return;
+    }
+
+    const T *X = (const T *)a.x;
+    const T *Wt = (const T *)a.w;
+
+    // element (row, k) of A and (k, col) of B
+    auto loadA = [&](int m, int k) -> float {
+        if (m >= M || k >= Ktot) return 0.f;
+        if (MODE == MODE_FWD) {
+            const int ci = k % Cpi, rc = k / Cpi, r = rc / kw, c = rc % kw;
+            const int ow = m % go.wp, t = m / go.wp, oh = t % go.hp, n = t / go.hp;
+            const int h = oh * sh - pt + r, w = ow * sw - pl + c;
+            if (h < 0 || h >= gi.hp || w < 0 || w >= gi.wp) return 0.f;
+            return to_f(X[gi.off + (((int64_t)n * gi.hp + h) * gi.wp + w) * Cpi + ci]);
+        } else if (MODE == MODE_DGRAD) {
+            const int co = k % Cpo, rc = k / Cpo, r = rc / kw, c = rc % kw;
+            const int w = m % gi.wp, t = m / gi.wp, h = t % gi.hp, n = t / gi.hp;
+            const int th = h + pt - r, tw = w + pl - c;
+            if (th < 0 || tw < 0 || th % sh || tw % sw) return 0.f;
+            const int oh = th / sh, ow = tw / sw;
+            if (oh >= go.hp || ow >= go.wp) return 0.f;
+            return to_f(X[go.off + (((int64_t)n * go.hp + oh) * go.wp + ow) * Cpo + co]);
+        } else {  // A(co, pixel) = dY
+            if (k < kbeg) return 0.f;
+            return to_f(X[go.off + (int64_t)k * Cpo + m]);
+        }
+    };
+    auto loadB = [&](int k, int col) -> float {
+        if (k >= Ktot || col >= Ncols) return 0.f;
+        if (MODE == MODE_FWD) {
+            if (col >= a.Cout) return 0.f;
+            return to_f(Wt[(int64_t)col * Ktot + k]);
+        } else if (MODE == MODE_DGRAD) {
+            const int co = k % Cpo, rc = k / Cpo;
+            if (co >= a.Cout) return 0.f;
+            return to_f(Wt[((int64_t)co * kh * kw + rc) * Cpi + col]);
+        } else {  // B(pixel, (r,c,ci)) = X~
+            if (k < kbeg) return 0.f;
+            const int ci = col % Cpi, rc = col / Cpi, r = rc / kw, c = rc % kw;
+            const int ow = k % go.wp, t = k / go.wp, oh = t % go.hp, n = t / go.hp;
+            const int h = oh * sh - pt + r, w = ow * sw - pl + c;
+            if (h < 0 || h >= gi.hp || w < 0 || w >= gi.wp) return 0.f;
+            return to_f(Wt[gi.off + (((int64_t)n * gi.hp + h) * gi.wp + w) * Cpi + ci]);
+        }
+    };
+    // lane mapping: make the memory-contiguous index lane-fastest
+    //   FWD:   A k-fast (ci contiguous), B k-fast (weights rows)
+    //   DGRAD: A k-fast (co contiguous), B col-fast (ci contiguous)
+    //   WGRAD: A row-fast (co contiguous), B col-fast (ci contiguous)
+    constexpr bool A_KFAST = (MODE != MODE_WGRAD);
+    constexpr bool B_KFAST = (MODE == MODE_FWD);
+
+    float ra[2], rb[2];
+    auto fetch = [&](int kt) {
+#pragma unroll
+        for (int s = 0; s < 2; ++s) {
+            const int e = tid + s * NT;
+            int mi, ki;
+            if (A_KFAST) { ki = e % BK; mi = e / BK; } else { mi = e % BM; ki = e / BM; }
+            ra[s] = loadA(m0 + mi, kt + ki);
+            int ni, kj;
+            if (B_KFAST) { kj = e % BK; ni = e / BK; } else { ni = e % BN; kj = e / BN; }
+            rb[s] = loadB(kt + kj, n0 + ni);
+        }
+    };
+    auto stash = [&](int buf) {
+#pragma unroll
+        for (int s = 0; s < 2; ++s) {
+            const int e = tid + s * NT;
+            int mi, ki;
+            if (A_KFAST) { ki = e % BK; mi = e / BK; } else { mi = e % BM; ki = e / BM; }
+            As[buf][ki][mi] = ra[s];
+            int ni, kj;
+            if (B_KFAST) { kj = e % BK; ni = e / BK; } else { ni = e % BN; kj = e / BN; }
+            Bs[buf][kj][ni] = rb[s];
+        }
+    };
+
+    float acc[4][4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = 0.f;
+    const int tx = tid % 16, ty = tid / 16;
+
+    const int kstart = (MODE == MODE_WGRAD) ? (kbeg / BK) * BK : 0;
+    int buf = 0;
+    if (m0 < M && n0 < Ncols && kstart < Ktot) {
+        fetch(kstart);
+        stash(0);
+        __syncthreads();
+        for (int kt = kstart; kt < Ktot; kt += BK) {
+            const bool more = kt + BK < Ktot;
+            if (more) fetch(kt + BK);
+#pragma unroll
+            for (int kk = 0; kk < BK; ++kk) {
+                float av[4], bv[4];
+#pragma unroll
+                for (int i = 0; i < 4; ++i) av[i] = As[buf][kk][ty * 4 + i];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) bv[j] = Bs[buf][kk][tx * 4 + j];
+#pragma unroll
+                for (int i = 0; i < 4; ++i)
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
+            }
+            if (more) {
+                stash(buf ^ 1);
+                __syncthreads();
+                buf ^= 1;
+            }
+        }
+    }
+
+    // epilogue
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        const int m = m0 + ty * 4 + i;
+        if (m >= M) continue;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const int col = n0 + tx * 4 + j;
+            if (col >= Ncols) continue;
+            float v = acc[i][j];
+            if (MODE == MODE_FWD) {
+                if (col < a.Cout) {
+                    if (a.bias) v += a.bias[col];
+                    if (a.relu) v = fmaxf(v, 0.f);
+                } else {
+                    v = 0.f;
+                }
+                ((T *)a.y)[go.off + (int64_t)m * Cpo + col] = from_f<T>(v);
+            } else if (MODE == MODE_DGRAD) {
+                const int64_t o = gi.off + (int64_t)m * Cpi + col;
+                if (a.relu_src && !(to_f(((const T *)a.relu_src)[o]) > 0.f)) v = 0.f;
+                ((T *)a.y)[o] = from_f<T>(v);
+            } else {
+                ((float *)a.y)[((int64_t)zq * M + m) * Ncols + col] = v;
+            }
+        }
+    }
+}
+
+// db partial per chunk: part_db[z][co] = sum over the chunk's pixels of dY[pixel][co]
+template <typename T>
+__global__ void __launch_bounds__(256) db_partial_kernel(LevelDesc Lo, const T *__restrict__ dY, float *__restrict__ part,
+                                                         int Cout, int p0, int cpp) {
+    const int zq = blockIdx.x;
+    const int q = p0 + zq / cpp;
+    const PatchGeo go = patch_geo(Lo, q);
+    const int P = Lo.N * go.hp * go.wp;
+    const int chunk = (P + cpp - 1) / cpp;
+    const int kb = (zq % cpp) * chunk, ke = min(P, kb + chunk);
+    for (int co = threadIdx.x; co < Cout; co += blockDim.x) {
+        float s = 0.f;
+        for (int k = kb; k < ke; ++k) s += to_f(dY[go.off + (int64_t)k * Lo.Cpad + co]);
+        part[(int64_t)zq * Cout + co] = s;
+    }
+}
+
+// dW[i] = beta * dW[i] + sum_z part[z][i]   (z ascending: fixed order)
+__global__ void __launch_bounds__(256) reduce_partials_kernel(const float *__restrict__ part, int Z, int64_t n,
+                                                              float *__restrict__ out, float beta) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        float s = 0.f;
+        for (int z = 0; z < Z; ++z) s += part[(int64_t)z * n + i];
+        out[i] = (beta != 0.f ? beta * out[i] : 0.f) + s;
+    }
+}
+
+static int64_t max_pixels(const Level &L, int p0, int p1) {
+    int64_t m = 0;
+    for (int q = p0; q < p1; ++q) {
+        int i = q / L.nw(), j = q % L.nw();
+        m = std::max<int64_t>(m, (int64_t)L.N * L.ph(i) * L.pw(j));
+    }
+    return m;
+}
+
+void launch_conv_fwd_simt(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *x,
+                          const void *w, const float *bias, void *y, int relu, int p0, int p1, cudaStream_t st) {
+    SimtArgs a{};
+    a.Li = make_level_desc(Li); a.Lo = make_level_desc(Lo); a.ly = make_layer_desc(g);
+    a.x = x; a.w = w; a.bias = bias; a.y = y; a.Cout = g.L.cout; a.relu = relu; a.p0 = p0;
+    dim3 grid((unsigned)((max_pixels(Lo, p0, p1) + BM - 1) / BM), (Lo.Cpad + BN - 1) / BN, p1 - p0);
+    if (dt == SPLITCNN_BF16) conv_simt_kernel<__nv_bfloat16, MODE_FWD><<<grid, NT, 0, st>>>(a);
+    else conv_simt_kernel<float, MODE_FWD><<<grid, NT, 0, st>>>(a);
+}
+
+void launch_conv_dgrad_simt(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy,
+                            const void *w, void *dx, const void *relu_src, int p0, int p1, cudaStream_t st) {
+    SimtArgs a{};
+    a.Li = make_level_desc(Li); a.Lo = make_level_desc(Lo); a.ly = make_layer_desc(g);
+    a.x = dy; a.w = w; a.y = dx; a.relu_src = relu_src; a.Cout = g.L.cout; a.p0 = p0;
+    dim3 grid((unsigned)((max_pixels(Li, p0, p1) + BM - 1) / BM), (Li.Cpad + BN - 1) / BN, p1 - p0);
+    if (dt == SPLITCNN_BF16) conv_simt_kernel<__nv_bfloat16, MODE_DGRAD><<<grid, NT, 0, st>>>(a);
+    else conv_simt_kernel<float, MODE_DGRAD><<<grid, NT, 0, st>>>(a);
+}
+
+// split-K chunking for the wgrad: a fixed function of the plan, so workspace_size agrees.
+int wgrad_simt_chunks_per_patch(const Level &Li, const Level &Lo, const LayerGeom &g, int npatch) {
+    const int tiles = ((g.L.cout + BM - 1) / BM) * ((g.L.kh * g.L.kw * Li.Cpad + BN - 1) / BN);
+    int cpp = (4 * 148 + tiles * npatch - 1) / (tiles * npatch);
+    int64_t minpix = INT64_MAX;
+    for (int i = 0; i < Lo.nh(); ++i)
+        for (int j = 0; j < Lo.nw(); ++j) minpix = std::min<int64_t>(minpix, (int64_t)Lo.N * Lo.ph(i) * Lo.pw(j));
+    cpp = std::max(1, std::min<int>(cpp, (int)std::max<int64_t>(1, minpix / 256)));
+    return std::min(cpp, 64);
+}
+
+size_t wgrad_simt_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g) {
+    const int np = Lo.nh() * Lo.nw();
+    const int cpp = wgrad_simt_chunks_per_patch(Li, Lo, g, np);
+    const int64_t Z = (int64_t)np * cpp;
+    const int64_t ncols = (int64_t)g.L.kh * g.L.kw * Li.Cpad;
+    return (size_t)(Z * g.L.cout * ncols + Z * g.L.cout) * sizeof(float);
+}
+
+void launch_conv_wgrad_simt(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *x,
+                            const void *dy, float *dw, float *db, float beta, void *ws, int p0, int p1, cudaStream_t st) {
+    const int np_all = Lo.nh() * Lo.nw();
+    const int cpp = wgrad_simt_chunks_per_patch(Li, Lo, g, np_all);
+    const int Z = (p1 - p0) * cpp;
+    const int ncols = g.L.kh * g.L.kw * Li.Cpad;
+    float *part = (float *)ws;
+    float *part_db = part + (int64_t)Z * g.L.cout * ncols;
+    SimtArgs a{};
+    a.Li = make_level_desc(Li); a.Lo = make_level_desc(Lo); a.ly = make_layer_desc(g);
+    a.x = dy; a.w = x; a.y = part; a.Cout = g.L.cout; a.p0 = p0; a.cpp = cpp;
+    dim3 grid((g.L.cout + BM - 1) / BM, (ncols + BN - 1) / BN, Z);
+    if (dt == SPLITCNN_BF16) conv_simt_kernel<__nv_bfloat16, MODE_WGRAD><<<grid, NT, 0, st>>>(a);
+    else conv_simt_kernel<float, MODE_WGRAD><<<grid, NT, 0, st>>>(a);
+    const int64_t n = (int64_t)g.L.cout * ncols;
+    reduce_partials_kernel<<<(unsigned)std::min<int64_t>((n + 255) / 256, 4096), 256, 0, st>>>(part, Z, n, dw, beta);
+    if (db) {
+        if (dt == SPLITCNN_BF16)
+            db_partial_kernel<__nv_bfloat16><<<Z, 256, 0, st>>>(make_level_desc(Lo), (const __nv_bfloat16 *)dy, part_db, g.L.cout, p0, cpp);
+        else
+            db_partial_kernel<float><<<Z, 256, 0, st>>>(make_level_desc(Lo), (const float *)dy, part_db, g.L.cout, p0, cpp);
+        reduce_partials_kernel<<<(g.L.cout + 255) / 256, 256, 0, st>>>(part_db, Z, g.L.cout, db, beta);
+    }
+}
+
+}  // namespace splitcnn

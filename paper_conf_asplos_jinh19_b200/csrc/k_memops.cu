@@ -1,0 +1,254 @@
+// k_memops.cu -- HBM-bound kernels of the split region:
+//   split  (Eq. 4)  full tensor  -> patch-major NHWC buffers (+ transpose, + channel pad)
+//   merge  (Eq. 7)  patch buffers -> full tensor
+//   max-pool forward / backward per patch (Eq. 6 with Op = max-pool)
+// One thread moves 8 channels (16 B in bf16) of one pixel; grid.y enumerates patches.
+#include "common.cuh"
+#include "kernels.h"
+
+namespace splitcnn {
+
+// ============================================================ split / merge
+template <typename T, bool NCHW>
+__global__ void __launch_bounds__(256) split_kernel(LevelDesc L, const T *__restrict__ x, T *__restrict__ P, int p0) {
+    const PatchGeo g = patch_geo(L, p0 + blockIdx.y);
+    const int G = L.Cpad / 8;
+    const int64_t units = (int64_t)L.N * g.hp * g.wp * G;
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < units; u += (int64_t)gridDim.x * blockDim.x) {
+        int n, h, w, cg;
+        if (NCHW) {  // pixel-fastest: coalesced reads of each channel plane
+            w = (int)(u % g.wp);
+            int64_t t = u / g.wp;
+            h = (int)(t % g.hp); t /= g.hp;
+            cg = (int)(t % G);
+            n = (int)(t / G);
+        } else {     // channel-fastest: coalesced 16 B reads and writes
+            cg = (int)(u % G);
+            int64_t t = u / G;
+            w = (int)(t % g.wp); t /= g.wp;
+            h = (int)(t % g.hp);
+            n = (int)(t / g.hp);
+        }
+        const int hg = g.h0 + h, wg = g.w0 + w, c0 = cg * 8;
+        float v[8];
+        if (NCHW) {
+#pragma unroll
+            for (int k = 0; k < 8; ++k)
+                v[k] = (c0 + k < L.C) ? to_f(x[(((int64_t)n * L.C + c0 + k) * L.H + hg) * L.W + wg]) : 0.f;
+        } else {
+            const T *src = x + (((int64_t)n * L.H + hg) * L.W + wg) * L.C + c0;
+            if ((L.C & 7) == 0) {
+                load8(src, v);
+            } else {
+#pragma unroll
+                for (int k = 0; k < 8; ++k) v[k] = (c0 + k < L.C) ? to_f(src[k]) : 0.f;
+            }
+        }
+        store8(P + g.off + (((int64_t)n * g.hp + h) * g.wp + w) * L.Cpad + c0, v);
+    }
+}
+
+template <typename T, bool NCHW>
+__global__ void __launch_bounds__(256) merge_kernel(LevelDesc L, const T *__restrict__ P, T *__restrict__ y, int p0) {
+    const PatchGeo g = patch_geo(L, p0 + blockIdx.y);
+    const int G = L.Cpad / 8;
+    const int64_t units = (int64_t)L.N * g.hp * g.wp * G;
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < units; u += (int64_t)gridDim.x * blockDim.x) {
+        int n, h, w, cg;
+        if (NCHW) {
+            w = (int)(u % g.wp);
+            int64_t t = u / g.wp;
+            h = (int)(t % g.hp); t /= g.hp;
+            cg = (int)(t % G);
+            n = (int)(t / G);
+        } else {
+            cg = (int)(u % G);
+            int64_t t = u / G;
+            w = (int)(t % g.wp); t /= g.wp;
+            h = (int)(t % g.hp);
+            n = (int)(t / g.hp);
+        }
+        const int hg = g.h0 + h, wg = g.w0 + w, c0 = cg * 8;
+        float v[8];
+        load8(P + g.off + (((int64_t)n * g.hp + h) * g.wp + w) * L.Cpad + c0, v);
+        if (NCHW) {
+#pragma unroll
+            for (int k = 0; k < 8; ++k)
+                if (c0 + k < L.C) y[(((int64_t)n * L.C + c0 + k) * L.H + hg) * L.W + wg] = from_f<T>(v[k]);
+        } else {
+            T *dst = y + (((int64_t)n * L.H + hg) * L.W + wg) * L.C + c0;
+            if ((L.C & 7) == 0) {
+                store8(dst, v);
+            } else {
+#pragma unroll
+                for (int k = 0; k < 8; ++k)
+                    if (c0 + k < L.C) dst[k] = from_f<T>(v[k]);
+            }
+        }
+    }
+}
+
+static int grid_x_for(int64_t units) {
+    int64_t b = (units + 255) / 256;
+    return (int)(b < 4096 ? (b < 1 ? 1 : b) : 4096);
+}
+
+static int64_t max_patch_units(const Level &L, int p0, int p1, int per_pixel) {
+    int64_t m = 0;
+    for (int q = p0; q < p1; ++q) {
+        int i = q / L.nw(), j = q % L.nw();
+        int64_t u = (int64_t)L.N * L.ph(i) * L.pw(j) * per_pixel;
+        if (u > m) m = u;
+    }
+    return m;
+}
+
+template <typename T>
+void launch_split_t(const Level &L, const void *x, int layout, void *P, int p0, int p1, cudaStream_t st) {
+    dim3 grid(grid_x_for(max_patch_units(L, p0, p1, L.Cpad / 8)), p1 - p0);
+    LevelDesc d = make_level_desc(L);
+    if (layout == SPLITCNN_NCHW)
+        split_kernel<T, true><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0);
+    else
+        split_kernel<T, false><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0);
+}
+
+template <typename T>
+void launch_merge_t(const Level &L, const void *P, void *y, int layout, int p0, int p1, cudaStream_t st) {
+    dim3 grid(grid_x_for(max_patch_units(L, p0, p1, L.Cpad / 8)), p1 - p0);
+    LevelDesc d = make_level_desc(L);
+    if (layout == SPLITCNN_NCHW)
+        merge_kernel<T, true><<<grid, 256, 0, st>>>(d, (const T *)P, (T *)y, p0);
+    else
+        merge_kernel<T, false><<<grid, 256, 0, st>>>(d, (const T *)P, (T *)y, p0);
+}
+
+void launch_split(splitcnn_dtype_t dt, const Level &L, const void *x, int layout, void *P, int p0, int p1, cudaStream_t st) {
+    if (dt == SPLITCNN_BF16) launch_split_t<__nv_bfloat16>(L, x, layout, P, p0, p1, st);
+    else launch_split_t<float>(L, x, layout, P, p0, p1, st);
+}
+void launch_merge(splitcnn_dtype_t dt, const Level &L, const void *P, void *y, int layout, int p0, int p1, cudaStream_t st) {
+    if (dt == SPLITCNN_BF16) launch_merge_t<__nv_bfloat16>(L, P, y, layout, p0, p1, st);
+    else launch_merge_t<float>(L, P, y, layout, p0, p1, st);
+}
+
+// ============================================================ max-pool
+// Forward: one thread = one output pixel x 8 channels.  The window max uses strict '>'
+// in row-major window order, so the argmax is the FIRST maximum (R9).  Padding is skipped (R7).
+template <typename T>
+__global__ void __launch_bounds__(256) pool_fwd_kernel(LevelDesc Li, LevelDesc Lo, LayerDesc ly, const T *__restrict__ X,
+                                                       T *__restrict__ Y, uint8_t *__restrict__ A, int p0, int relu_bit) {
+    const int q = p0 + blockIdx.y;
+    const PatchGeo gi = patch_geo(Li, q), go = patch_geo(Lo, q);
+    const int pt = ly.pad_h[2 * gi.i], pl = ly.pad_w[2 * gi.j];
+    const int G = Li.Cpad / 8;
+    const int64_t units = (int64_t)Lo.N * go.hp * go.wp * G;
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < units; u += (int64_t)gridDim.x * blockDim.x) {
+        const int cg = (int)(u % G);
+        int64_t t = u / G;
+        const int ow = (int)(t % go.wp); t /= go.wp;
+        const int oh = (int)(t % go.hp);
+        const int n = (int)(t / go.hp);
+        float best[8];
+        int arg[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) { best[k] = -INFINITY; arg[k] = -1; }
+        for (int r = 0; r < ly.kh; ++r) {
+            const int h = oh * ly.sh - pt + r;
+            if (h < 0 || h >= gi.hp) continue;
+            for (int c = 0; c < ly.kw; ++c) {
+                const int w = ow * ly.sw - pl + c;
+                if (w < 0 || w >= gi.wp) continue;
+                float v[8];
+                load8(X + gi.off + (((int64_t)n * gi.hp + h) * gi.wp + w) * Li.Cpad + cg * 8, v);
+                const int idx = r * ly.kw + c;
+#pragma unroll
+                for (int k = 0; k < 8; ++k)
+                    if (arg[k] < 0 || v[k] > best[k]) { best[k] = v[k]; arg[k] = idx; }
+            }
+        }
+        const int64_t o = go.off + (((int64_t)n * go.hp + oh) * go.wp + ow) * Lo.Cpad + cg * 8;
+        store8(Y + o, best);
+        uint32_t lo = 0, hi = 0;
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            uint32_t b = (uint32_t)(arg[k] & 0x7f) | ((relu_bit && best[k] > 0.f) ? 0x80u : 0u);
+            if (k < 4) lo |= b << (8 * k); else hi |= b << (8 * (k - 4));
+        }
+        *reinterpret_cast<uint2 *>(A + o) = make_uint2(lo, hi);
+    }
+}
+
+__device__ __forceinline__ int floordiv(int a, int b) { return (a >= 0) ? a / b : -((-a + b - 1) / b); }
+
+// Backward: gather form -- one thread = one INPUT pixel x 8 channels; it visits every window
+// that covers the pixel in (oh, ow) ascending order and adds dY where the argmax points at it.
+// Every dX element is written once (no memset, no atomics, deterministic order).
+template <typename T>
+__global__ void __launch_bounds__(256) pool_bwd_kernel(LevelDesc Li, LevelDesc Lo, LayerDesc ly, const T *__restrict__ dY,
+                                                       const uint8_t *__restrict__ A, T *__restrict__ dX, int p0, int relu_bit) {
+    const int q = p0 + blockIdx.y;
+    const PatchGeo gi = patch_geo(Li, q), go = patch_geo(Lo, q);
+    const int pt = ly.pad_h[2 * gi.i], pl = ly.pad_w[2 * gi.j];
+    const int G = Li.Cpad / 8;
+    const int64_t units = (int64_t)Li.N * gi.hp * gi.wp * G;
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < units; u += (int64_t)gridDim.x * blockDim.x) {
+        const int cg = (int)(u % G);
+        int64_t t = u / G;
+        const int w = (int)(t % gi.wp); t /= gi.wp;
+        const int h = (int)(t % gi.hp);
+        const int n = (int)(t / gi.hp);
+        int oh_lo = floordiv(h + pt - ly.kh, ly.sh) + 1, oh_hi = floordiv(h + pt, ly.sh);
+        int ow_lo = floordiv(w + pl - ly.kw, ly.sw) + 1, ow_hi = floordiv(w + pl, ly.sw);
+        if (oh_lo < 0) oh_lo = 0;
+        if (ow_lo < 0) ow_lo = 0;
+        if (oh_hi > go.hp - 1) oh_hi = go.hp - 1;
+        if (ow_hi > go.wp - 1) ow_hi = go.wp - 1;
+        float acc[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) acc[k] = 0.f;
+        for (int oh = oh_lo; oh <= oh_hi; ++oh)
+            for (int ow = ow_lo; ow <= ow_hi; ++ow) {
+                const int idx = (h - (oh * ly.sh - pt)) * ly.kw + (w - (ow * ly.sw - pl));
+                const int64_t o = go.off + (((int64_t)n * go.hp + oh) * go.wp + ow) * Lo.Cpad + cg * 8;
+                const uint2 a2 = __ldg(reinterpret_cast<const uint2 *>(A + o));
+                float g[8];
+                load8(dY + o, g);
+#pragma unroll
+                for (int k = 0; k < 8; ++k) {
+                    const uint32_t b = ((k < 4 ? a2.x : a2.y) >> (8 * (k & 3))) & 0xffu;
+                    const bool hit = (int)(b & 0x7fu) == idx && (!relu_bit || (b & 0x80u));
+                    acc[k] += hit ? g[k] : 0.f;
+                }
+            }
+        store8(dX + gi.off + (((int64_t)n * gi.hp + h) * gi.wp + w) * Li.Cpad + cg * 8, acc);
+    }
+}
+
+template <typename T>
+void launch_pool_fwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, void *y, uint8_t *a,
+                       int relu_bit, int p0, int p1, cudaStream_t st) {
+    dim3 grid(grid_x_for(max_patch_units(Lo, p0, p1, Lo.Cpad / 8)), p1 - p0);
+    pool_fwd_kernel<T><<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
+                                             (const T *)x, (T *)y, a, p0, relu_bit);
+}
+template <typename T>
+void launch_pool_bwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy, const uint8_t *a, void *dx,
+                       int relu_bit, int p0, int p1, cudaStream_t st) {
+    dim3 grid(grid_x_for(max_patch_units(Li, p0, p1, Li.Cpad / 8)), p1 - p0);
+    pool_bwd_kernel<T><<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
+                                             (const T *)dy, a, (T *)dx, p0, relu_bit);
+}
+
+void launch_pool_fwd(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, void *y,
+                     uint8_t *a, int relu_bit, int p0, int p1, cudaStream_t st) {
+    if (dt == SPLITCNN_BF16) launch_pool_fwd_t<__nv_bfloat16>(Li, Lo, g, x, y, a, relu_bit, p0, p1, st);
+    else launch_pool_fwd_t<float>(Li, Lo, g, x, y, a, relu_bit, p0, p1, st);
+}
+void launch_pool_bwd(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy,
+                     const uint8_t *a, void *dx, int relu_bit, int p0, int p1, cudaStream_t st) {
+    if (dt == SPLITCNN_BF16) launch_pool_bwd_t<__nv_bfloat16>(Li, Lo, g, dy, a, dx, relu_bit, p0, p1, st);
+    else launch_pool_bwd_t<float>(Li, Lo, g, dy, a, dx, relu_bit, p0, p1, st);
+}
+
+}  // namespace splitcnn

@@ -1,0 +1,36 @@
+// kernels.h -- launchers of the libsplitcnn kernels (library-private).
+#pragma once
+#include <cuda_runtime.h>
+
+#include "internal.h"
+
+namespace splitcnn {
+
+// k_memops.cu
+void launch_split(splitcnn_dtype_t dt, const Level &L, const void *x, int layout, void *P, int p0, int p1, cudaStream_t st);
+void launch_merge(splitcnn_dtype_t dt, const Level &L, const void *P, void *y, int layout, int p0, int p1, cudaStream_t st);
+void launch_pool_fwd(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, void *y,
+                     uint8_t *a, int relu_bit, int p0, int p1, cudaStream_t st);
+void launch_pool_bwd(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy,
+                     const uint8_t *a, void *dx, int relu_bit, int p0, int p1, cudaStream_t st);
+
+// k_conv_simt.cu
+void launch_conv_fwd_simt(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *x,
+                          const void *w, const float *bias, void *y, int relu, int p0, int p1, cudaStream_t st);
+void launch_conv_dgrad_simt(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy,
+                            const void *w, void *dx, const void *relu_src, int p0, int p1, cudaStream_t st);
+void launch_conv_wgrad_simt(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *x,
+                            const void *dy, float *dw, float *db, float beta, void *ws, int p0, int p1, cudaStream_t st);
+size_t wgrad_simt_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g);
+
+// k_conv_tc.cu (tcgen05); return false when the shape is not supported by the tensor-core path
+bool conv_tc_supported(int mode, splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g);
+size_t conv_tc_ws_bytes(int mode, const Level &Li, const Level &Lo, const LayerGeom &g);
+splitcnn_status_t launch_conv_fwd_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *w,
+                                     const float *bias, void *y, int relu, int p0, int p1, cudaStream_t st);
+splitcnn_status_t launch_conv_dgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy, const void *w,
+                                       void *dx, const void *relu_src, void *ws, int p0, int p1, cudaStream_t st);
+splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *dy,
+                                       float *dw, float *db, float beta, void *ws, int p0, int p1, cudaStream_t st);
+
+}  // namespace splitcnn

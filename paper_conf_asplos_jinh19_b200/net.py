@@ -1,0 +1,224 @@
+"""SplitNet -- executes a Split-CNN conv stack (split region + unsplit tail) through libsplitcnn.
+
+A step is one pass of the hot path: split (Eq. 4) -> per-patch conv / max-pool
+forward (Eq. 6) through the chained split region -> merge at the join (Eq. 7) -> the
+unsplit tail (a 1x1 "split", i.e. ordinary layers) -> backward in reverse order: pool backward,
+conv data gradient (ReLU mask fused), conv weight gradient summed over patches and batch.
+PyTorch only allocates device memory and provides the stream; every step runs in libsplitcnn.
+"""
+from __future__ import annotations
+
+import torch
+
+from . import splitcnn as sc
+from .plan import SplitPlan
+
+TORCH_DTYPE = {sc.BF16: torch.bfloat16, sc.FP32: torch.float32}
+
+
+def pack_weight(W_oihw: torch.Tensor, cpad_in: int, dtype) -> torch.Tensor:
+    """OIHW -> the library layout [Cout][kh][kw][Cpad_in] (zero channel padding); parameter setup."""
+    co, ci, kh, kw = W_oihw.shape
+    out = torch.zeros((co, kh, kw, cpad_in), dtype=dtype, device=W_oihw.device)
+    out[..., :ci] = W_oihw.permute(0, 2, 3, 1).to(dtype)
+    return out
+
+
+def unpack_grad(dW: torch.Tensor, cin: int) -> torch.Tensor:
+    """[Cout][kh][kw][Cpad_in] -> OIHW."""
+    return dW[..., :cin].permute(0, 3, 1, 2)
+
+
+class SplitNet:
+    def __init__(self, region: list[dict], tail: list[dict], N: int, C: int, H: int, W: int,
+                 split=(2, 2), mode: str = "even", omega: float = 0.2, seed: int = 0,
+                 dtype: int = sc.BF16, device="cuda", patch_range=None, force_simt: bool = False):
+        self.region_layers, self.tail_layers = region, tail
+        self.N, self.C, self.H, self.W = N, C, H, W
+        self.split, self.mode, self.omega, self.seed = split, mode, omega, seed
+        self.dtype, self.tdtype, self.device = dtype, TORCH_DTYPE[dtype], torch.device(device)
+        self.flags_extra = sc.FLAG_FORCE_SIMT if force_simt else 0
+        self.step_index = 0
+        self.region = self._make_region_plan(0)
+        self.patch_range = patch_range or (0, self.region.npatch)
+        L = self.region.levels[-1]
+        self.tail = SplitPlan(tail, N, L["C"], L["H"], L["W"], [0, _out_len(tail, L["H"], 0)],
+                              [0, _out_len(tail, L["W"], 1)]) if tail else None
+        self._alloc()
+
+    # ------------------------------------------------------------------ planning
+    def _region_output_hw(self):
+        h, w = self.H, self.W
+        for l in self.region_layers:
+            h = (h + l["ph_b"] + l["ph_e"] - l["kh"]) // l["sh"] + 1
+            w = (w + l["pw_b"] + l["pw_e"] - l["kw"]) // l["sw"] + 1
+        return h, w
+
+    def boundaries(self, step: int):
+        ho, wo = self._region_output_hw()
+        nh, nw = self.split
+        if self.mode == "random":                      # a new scheme per minibatch
+            return sc.splitcnn_boundaries_random(ho, nh, wo, nw, self.omega, self.seed, step)
+        return sc.splitcnn_boundaries_even(ho, nh), sc.splitcnn_boundaries_even(wo, nw)
+
+    def _make_region_plan(self, step: int) -> SplitPlan:
+        Oh, Ow = self.boundaries(step)
+        return SplitPlan(self.region_layers, self.N, self.C, self.H, self.W, Oh, Ow)
+
+    def replan(self, step: int):
+        """Stochastic splitting: redraw the boundaries; buffer sizes do not depend on them."""
+        if self.mode == "random":
+            self.region = self._make_region_plan(step)
+
+    # ------------------------------------------------------------------ buffers
+    def _stages(self):
+        st = [(self.region, m, l) for m, l in enumerate(self.region_layers)]
+        if self.tail:
+            st += [(self.tail, m, l) for m, l in enumerate(self.tail_layers)]
+        return st
+
+    def _alloc(self):
+        dev, td = self.device, self.tdtype
+        self.act_r = [torch.zeros(self.region.level_elems(m), dtype=td, device=dev)
+                      for m in range(self.region.nlayers + 1)]
+        self.act_t = ([torch.zeros(self.tail.level_elems(m), dtype=td, device=dev)
+                       for m in range(self.tail.nlayers + 1)] if self.tail else [])
+        self.argmax = {}
+        for plan, acts, key in ((self.region, self.act_r, "r"), (self.tail, self.act_t, "t")):
+            if plan is None:
+                continue
+            for m, l in enumerate(plan.layers):
+                if l["op"] == "maxpool":
+                    self.argmax[(key, m)] = torch.zeros(plan.level_elems(m + 1), dtype=torch.uint8, device=dev)
+        maxg = max([a.numel() for a in self.act_r + self.act_t])
+        self.grad = [torch.zeros(maxg, dtype=td, device=dev), torch.zeros(maxg, dtype=td, device=dev)]
+        ws = 0
+        for plan in (self.region, self.tail):
+            if plan is None:
+                continue
+            for m, l in enumerate(plan.layers):
+                if l["op"] == "conv":
+                    ws = max(ws, plan.workspace_size(m, self.dtype, 1), plan.workspace_size(m, self.dtype, 2))
+        self.ws = torch.zeros(max(ws, 16) // 4 + 4, dtype=torch.float32, device=dev)
+        self.ws_bytes = self.ws.numel() * 4
+        self.params, self.grads = {}, {}
+        for key, layers, plan in (("r", self.region_layers, self.region), ("t", self.tail_layers, self.tail)):
+            for m, l in enumerate(layers):
+                if l["op"] == "conv":
+                    cpad = plan.levels[m]["Cpad"]
+                    self.params[(key, m)] = (torch.zeros((l["cout"], l["kh"], l["kw"], cpad), dtype=td, device=dev),
+                                             torch.zeros(l["cout"], dtype=torch.float32, device=dev))
+                    self.grads[(key, m)] = (torch.zeros((l["cout"], l["kh"], l["kw"], cpad), dtype=torch.float32,
+                                                        device=dev),
+                                            torch.zeros(l["cout"], dtype=torch.float32, device=dev))
+
+    def set_params(self, params):
+        """params: list (region + tail order, convs only) of (W_oihw, b) torch/numpy arrays."""
+        it = iter(params)
+        for key, layers, plan in (("r", self.region_layers, self.region), ("t", self.tail_layers, self.tail)):
+            for m, l in enumerate(layers):
+                if l["op"] == "conv":
+                    W, b = next(it)
+                    W = torch.as_tensor(W).to(self.device)
+                    self.params[(key, m)][0].copy_(pack_weight(W, plan.levels[m]["Cpad"], self.tdtype))
+                    self.params[(key, m)][1].copy_(torch.as_tensor(b, dtype=torch.float32))
+
+    # ------------------------------------------------------------------ masks
+    def _masked(self, key: str, m: int) -> bool:
+        """Level m is the output of a conv with fused ReLU -> its gradient producer applies the mask."""
+        if key == "r":
+            return m > 0 and self.region_layers[m - 1]["op"] == "conv" and self.region_layers[m - 1].get("relu", True)
+        if m > 0:
+            return self.tail_layers[m - 1]["op"] == "conv" and self.tail_layers[m - 1].get("relu", True)
+        return self._masked("r", len(self.region_layers))
+
+    # ------------------------------------------------------------------ passes
+    def forward(self, x: torch.Tensor, stream=None):
+        """x: full NCHW tensor (dtype) on the device.  Returns the output level buffer."""
+        p0, p1 = self.patch_range
+        R, dt, fl = self.region.handle, self.dtype, self.flags_extra
+        sc.splitcnn_split(R, 0, dt, x, sc.NCHW, self.act_r[0], p0, p1, stream)
+        self._run_fwd("r", self.region, self.region_layers, self.act_r, p0, p1, stream)
+        if self.tail:
+            sc.splitcnn_merge(R, self.region.nlayers, dt, self.act_r[-1], self.act_t[0], sc.NHWC, p0, p1, stream)
+            self._run_fwd("t", self.tail, self.tail_layers, self.act_t, 0, 1, stream)
+            return self.act_t[-1]
+        return self.act_r[-1]
+
+    def _run_fwd(self, key, plan, layers, acts, p0, p1, stream):
+        for m, l in enumerate(layers):
+            if l["op"] == "conv":
+                W, b = self.params[(key, m)]
+                flags = (sc.FLAG_RELU if l.get("relu", True) else 0) | self.flags_extra
+                sc.splitcnn_conv_fwd(plan.handle, m, self.dtype, acts[m], W, b, acts[m + 1], flags, p0, p1, stream)
+            else:
+                flags = sc.FLAG_POOL_RELU_MASK if self._masked(key, m) else 0
+                sc.splitcnn_pool_fwd(plan.handle, m, self.dtype, acts[m], acts[m + 1], self.argmax[(key, m)], flags,
+                                     p0, p1, stream)
+
+    def backward(self, dy: torch.Tensor, stream=None, need_input_grad: bool = False):
+        """dy: gradient w.r.t. the output level buffer (same layout).  Fills self.grads."""
+        p0, p1 = self.patch_range
+        g = dy
+        if self.tail:
+            g = self._run_bwd("t", self.tail, self.tail_layers, self.act_t, g, 0, 1, stream, True)
+            gi = self.grad[0] if g is not self.grad[0] else self.grad[1]
+            sc.splitcnn_split(self.region.handle, self.region.nlayers, self.dtype, g, sc.NHWC, gi, p0, p1, stream)
+            g = gi
+        return self._run_bwd("r", self.region, self.region_layers, self.act_r, g, p0, p1, stream, need_input_grad)
+
+    def _run_bwd(self, key, plan, layers, acts, g, p0, p1, stream, need_input_grad):
+        for m in range(len(layers) - 1, -1, -1):
+            l = layers[m]
+            out = self.grad[0] if g is not self.grad[0] else self.grad[1]
+            last = (m == 0 and not need_input_grad)
+            if l["op"] == "conv":
+                W, _ = self.params[(key, m)]
+                dW, db = self.grads[(key, m)]
+                if not last:
+                    relu_src = acts[m] if self._masked(key, m) else None
+                    sc.splitcnn_conv_bwd_data(plan.handle, m, self.dtype, g, W, out, relu_src, self.ws, self.ws_bytes,
+                                              self.flags_extra, p0, p1, stream)
+                sc.splitcnn_conv_bwd_filter(plan.handle, m, self.dtype, acts[m], g, dW, db, 0.0, self.ws,
+                                            self.ws_bytes, self.flags_extra, p0, p1, stream)
+            else:
+                flags = sc.FLAG_POOL_RELU_MASK if self._masked(key, m) else 0
+                sc.splitcnn_pool_bwd(plan.handle, m, self.dtype, g, self.argmax[(key, m)], out, flags, p0, p1, stream)
+            if not last:
+                g = out
+        return g
+
+    def step(self, x, dy, stream=None):
+        self.replan(self.step_index)
+        self.forward(x, stream)
+        self.backward(dy, stream)
+        self.step_index += 1
+
+    # ------------------------------------------------------------------ accounting
+    def conv_flops(self) -> int:
+        """Algorithmic FLOPs of one fwd+bwd step: 2*N*Cout*Ho*Wo*Cin*kh*kw per pass;
+        fwd + wgrad for every conv, + dgrad for every conv except the first."""
+        total = 0
+        first = True
+        for plan, layers in ((self.region, self.region_layers), (self.tail, self.tail_layers)):
+            if plan is None:
+                continue
+            for m, l in enumerate(layers):
+                if l["op"] != "conv":
+                    continue
+                lo = plan.levels[m + 1]
+                f = 2 * lo["N"] * l["cout"] * lo["H"] * lo["W"] * l["cin"] * l["kh"] * l["kw"]
+                total += f * (2 if first else 3)
+                first = False
+        return total
+
+    def output_numel(self) -> int:
+        return (self.act_t[-1] if self.tail else self.act_r[-1]).numel()
+
+
+def _out_len(layers, L, dim):
+    for l in layers:
+        k, s = (l["kh"], l["sh"]) if dim == 0 else (l["kw"], l["sw"])
+        pb, pe = (l["ph_b"], l["ph_e"]) if dim == 0 else (l["pw_b"], l["pw_e"])
+        L = (L + pb + pe - k) // s + 1
+    return L

@@ -1,0 +1,99 @@
+"""Oracle composition of a whole split stack (region + unsplit tail), for the stack parity test.
+Composes oracle.ops only.  ``round_bf16`` emulates the bf16 STORAGE of every activation and
+gradient level (the exact inputs the bf16 GPU path feeds each op); arithmetic stays
+fp64."""
+from __future__ import annotations
+
+import numpy as np
+
+import synth
+from oracle import ops as O
+from oracle import plan as OP
+
+
+def _rnd(P, on):
+    if not on:
+        return P
+    return [[synth.to_bf16_f32(p.astype(np.float32)).astype(np.float64) for p in row] for row in P]
+
+
+def _masked(layers, m, prev_masked):
+    if m == 0:
+        return prev_masked
+    l = layers[m - 1]
+    return l["op"] == "conv" and l.get("relu", True)
+
+
+def run(region, tail, N, C, H, W, Oh, Ow, params, X, G, round_bf16=False):
+    """Returns (output NCHW, [dW OIHW per conv in order], [db per conv], pools) where pools maps
+    (key, m) -> (pool input patches, argmax patches) for the argmax-agreement check."""
+    rp = OP.plan(region, N, C, H, W, Oh, Ow)
+    Lr = rp.layers[-1]
+    tp = OP.plan(tail, N, region[-1]["cout"], Lr.H_out, Lr.W_out,
+                 [0, _out(tail, Lr.H_out, 0)], [0, _out(tail, Lr.W_out, 1)]) if tail else None
+    pit = iter(params)
+    prm = {}
+    for key, layers in (("r", region), ("t", tail)):
+        for m, l in enumerate(layers):
+            if l["op"] == "conv":
+                prm[(key, m)] = next(pit)
+
+    def fwd(key, plan, layers, P):
+        acts, args = [P], {}
+        for m, (l, lp) in enumerate(zip(layers, plan.layers)):
+            if l["op"] == "conv":
+                Wt, b = prm[(key, m)]
+                P = O.conv_fwd(P, Wt, b, lp, l.get("relu", True))
+            else:
+                P, args[m] = O.pool_fwd(P, lp)
+            P = _rnd(P, round_bf16)
+            acts.append(P)
+        return acts, args
+
+    def bwd(key, plan, layers, acts, args, g, first_masked, need_input):
+        grads = {}
+        for m in range(len(layers) - 1, -1, -1):
+            l, lp = layers[m], plan.layers[m]
+            msk = _masked(layers, m, first_masked)
+            last = m == 0 and not need_input
+            if l["op"] == "conv":
+                Wt, _ = prm[(key, m)]
+                grads[m] = O.conv_bwd_filter(acts[m], g, lp)
+                if not last:
+                    g = _rnd(O.conv_bwd_data(g, Wt, lp, acts[m] if msk else None), round_bf16)
+            else:
+                g = O.pool_bwd(g, args[m], lp)
+                if msk:
+                    g = O.relu_mask(g, acts[m])
+                g = _rnd(g, round_bf16)
+        return g, grads
+
+    pools = {}
+    acts_r, args_r = fwd("r", rp, region, _rnd(O.split(X, rp.layers[0].Ih, rp.layers[0].Iw), round_bf16))
+    out = O.merge(acts_r[-1])
+    pools.update({("r", m): (acts_r[m], a) for m, a in args_r.items()})
+    region_out_masked = _masked(region, len(region), False)
+    if tp is not None:
+        acts_t, args_t = fwd("t", tp, tail, [[out]])
+        pools.update({("t", m): (acts_t[m], a) for m, a in args_t.items()})
+        out = O.merge(acts_t[-1])
+        g, grads_t = bwd("t", tp, tail, acts_t, args_t, [[G]], region_out_masked, True)
+        g = O.split(O.merge(g), Lr.Oh, Lr.Ow)
+    else:
+        g, grads_t = O.split(G, Lr.Oh, Lr.Ow), {}
+    _, grads_r = bwd("r", rp, region, acts_r, args_r, g, False, False)
+    dWs, dbs = [], []
+    for key, layers, grads in (("r", region, grads_r), ("t", tail, grads_t)):
+        for m, l in enumerate(layers):
+            if l["op"] == "conv":
+                dWs.append(grads[m][0])
+                dbs.append(grads[m][1])
+    return out, dWs, dbs, pools
+
+
+def _out(layers, L, dim):
+    for l in layers:
+        k, s = (l["kh"], l["sh"]) if dim == 0 else (l["kw"], l["sw"])
+        pb, pe = (l["ph_b"], l["ph_e"]) if dim == 0 else (l["pw_b"], l["pw_e"])
+        L = (L + pb + pe - k) // s + 1
+    return L

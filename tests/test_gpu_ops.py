@@ -1,0 +1,267 @@
+"""GPU parity of every split operator against the CPU oracle, through the C ABI.
+
+Bars (BASELINE.json north_star): plan / boundaries / split / merge / pool values /
+argmax / k=s pool backward / offload BIT-EXACT; conv fwd / dgrad / wgrad normwise
+||y - y*||_inf / ||y*||_inf <= 1e-4 for FP32 (FFMA) and <= 2e-2 for BF16 inputs with fp32
+accumulation.  The oracle accumulates in fp64 on the exact (bf16-rounded) inputs the GPU sees.
+"""
+import numpy as np
+import pytest
+
+import synth
+from oracle import ops as O
+from oracle import plan as OP
+from tests.helpers import normwise, pack_level, unpack_level, w_lib_to_oihw, w_oihw_to_lib
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+TOL = {0: 2e-2, 1: 1e-4}   # BF16, FP32
+
+
+@pytest.fixture(scope="module")
+def sc():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import __graft_entry__
+    __graft_entry__.build()
+    from paper_conf_asplos_jinh19_b200 import splitcnn
+    return splitcnn
+
+
+def _td(sc, dtype):
+    return torch.bfloat16 if dtype == sc.BF16 else torch.float32
+
+
+def _dev(sc, a, dtype):
+    return torch.from_numpy(np.ascontiguousarray(a, dtype=np.float32)).to("cuda", _td(sc, dtype))
+
+
+def _host(t):
+    return t.float().cpu().numpy().astype(np.float64)
+
+
+def _round(a, dtype, sc):
+    return synth.to_bf16_f32(a).astype(np.float64) if dtype == sc.BF16 else a.astype(np.float32).astype(np.float64)
+
+
+def _make(sc, layers, N, C, H, W, nh, nw, seed):
+    L_h, L_w = H, W
+    for l in layers:
+        L_h = OP.out_len(L_h, l["kh"], l["sh"], l["ph_b"], l["ph_e"])
+        L_w = OP.out_len(L_w, l["kw"], l["sw"], l["pw_b"], l["pw_e"])
+    Oh, Ow = OP.boundaries_random(L_h, nh, L_w, nw, 0.3, seed, 0)
+    ref = OP.plan(layers, N, C, H, W, Oh, Ow)
+    from paper_conf_asplos_jinh19_b200.plan import SplitPlan
+    return ref, SplitPlan(layers, N, C, H, W, Oh, Ow)
+
+
+# (name, N, cin, cout, k, s, p, H, W, nh, nw, relu)
+CONV_CASES = [
+    ("C1", 2, 16, 16, 3, 1, 1, 32, 32, 2, 2, False),
+    ("ragged", 3, 13, 24, 3, 1, 1, 19, 23, 3, 2, True),
+    ("conv1_7x7s2", 2, 3, 16, 7, 2, 3, 30, 26, 2, 2, True),
+    ("3x3s2", 2, 16, 32, 3, 2, 1, 20, 18, 2, 3, True),
+    ("1x1s2_k<s", 2, 16, 32, 1, 2, 0, 14, 12, 2, 2, False),
+    ("vgg64", 4, 64, 64, 3, 1, 1, 32, 32, 2, 2, True),
+    ("vgg_first", 2, 3, 64, 3, 1, 1, 32, 28, 2, 2, True),
+    ("vgg128_256", 2, 128, 256, 3, 1, 1, 16, 16, 3, 3, True),
+    ("c5_7x7patch", 2, 256, 256, 3, 1, 1, 28, 28, 4, 4, True),
+]
+
+
+@pytest.mark.parametrize("case", CONV_CASES, ids=[c[0] for c in CONV_CASES])
+@pytest.mark.parametrize("mode", ["fp32", "bf16_tc", "bf16_simt"])
+def test_conv_parity(sc, case, mode):
+    name, N, cin, cout, k, s, p, H, W, nh, nw, relu = case
+    dtype = sc.FP32 if mode == "fp32" else sc.BF16
+    extra = sc.FLAG_FORCE_SIMT if mode == "bf16_simt" else 0
+    layers = [synth.conv(cin, cout, k, s, p, relu=relu)]
+    ref, pl = _make(sc, layers, N, cin, H, W, nh, nw, seed=sum(map(ord, name)))
+    lp = ref.layers[0]
+    lv0, lv1 = pl.levels
+    g = synth.rng(100 + len(name))
+    X = _round(synth.uniform(g, (N, cin, H, W)), dtype, sc)
+    Wt = _round(synth.kaiming(g, cout, cin, k, k), dtype, sc)
+    b = synth.uniform(g, (cout,), -0.1, 0.1).astype(np.float64)
+    Ho, Wo = lp.H_out, lp.W_out
+    G = _round(synth.normal(g, (N, cout, Ho, Wo)), dtype, sc)
+    M = _round(synth.uniform(g, (N, cin, H, W)), dtype, sc)     # ReLU-output stand-in for the mask
+
+    x = _dev(sc, pack_level(X, lv0), dtype)
+    w = _dev(sc, w_oihw_to_lib(Wt, lv0["Cpad"]), dtype)
+    bias = torch.from_numpy(b.astype(np.float32)).cuda()
+    y = torch.full((lv1["total_elems"],), 7.0, dtype=_td(sc, dtype), device="cuda")
+    flags = (sc.FLAG_RELU if relu else 0) | extra
+    sc.splitcnn_conv_fwd(pl.handle, 0, dtype, x, w, bias, y, flags)
+    Xp = O.split(X, lp.Ih, lp.Iw)
+    Yref = O.conv_fwd(Xp, Wt, b, lp, relu)
+    Ygot = unpack_level(_host(y), lv1, keep_pad=True)
+    err = max(normwise(Ygot[i][j][:, :cout], Yref[i][j]) for i in range(nh) for j in range(nw))
+    assert err <= TOL[dtype], f"fwd normwise {err}"
+    for row in Ygot:
+        for blk in row:
+            assert np.all(blk[:, cout:] == 0), "channel padding of Y must be zero"
+
+    dy = _dev(sc, pack_level(G, lv1), dtype)
+    mask = _dev(sc, pack_level(M, lv0), dtype)
+    dx = torch.full((lv0["total_elems"],), 7.0, dtype=_td(sc, dtype), device="cuda")
+    ws_b = max(pl.workspace_size(0, dtype, 1), pl.workspace_size(0, dtype, 2), 16)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    sc.splitcnn_conv_bwd_data(pl.handle, 0, dtype, dy, w, dx, mask, ws, ws_b, extra)
+    Gp = O.split(G, lp.Oh, lp.Ow)
+    dXref = O.conv_bwd_data(Gp, Wt, lp, O.split(M, lp.Ih, lp.Iw))
+    dXgot = unpack_level(_host(dx), lv0, keep_pad=True)
+    err = max(normwise(dXgot[i][j][:, :cin], dXref[i][j]) for i in range(nh) for j in range(nw))
+    assert err <= TOL[dtype], f"dgrad normwise {err}"
+    for row in dXgot:
+        for blk in row:
+            assert np.all(blk[:, cin:] == 0), "channel padding of dX must be zero"
+
+    dw = torch.full((cout, k, k, lv0["Cpad"]), 3.0, dtype=torch.float32, device="cuda")
+    db = torch.full((cout,), 3.0, dtype=torch.float32, device="cuda")
+    sc.splitcnn_conv_bwd_filter(pl.handle, 0, dtype, x, dy, dw, db, 0.0, ws, ws_b, extra)
+    dWref, dbref = O.conv_bwd_filter(Xp, Gp, lp)
+    dWgot = _host(dw)
+    assert normwise(w_lib_to_oihw(dWgot, cin), dWref) <= TOL[dtype]
+    assert normwise(_host(db), dbref) <= TOL[dtype]
+    if lv0["Cpad"] > cin:
+        assert np.all(dWgot[..., cin:] == 0)
+    # beta = 1 accumulates; the reduction order is fixed, so the result is exactly 2x
+    sc.splitcnn_conv_bwd_filter(pl.handle, 0, dtype, x, dy, dw, db, 1.0, ws, ws_b, extra)
+    np.testing.assert_array_equal(_host(dw), 2 * dWgot)
+    # determinism run to run
+    dw2 = torch.zeros_like(dw)
+    sc.splitcnn_conv_bwd_filter(pl.handle, 0, dtype, x, dy, dw2, None, 0.0, ws, ws_b, extra)
+    np.testing.assert_array_equal(_host(dw2), dWgot)
+
+
+def test_conv_patch_range_sharding(sc):
+    """Patches computed in two ranges [0,q) + [q,P) equal one call; wgrad partial sums add up."""
+    dtype = sc.BF16
+    layers = [synth.conv(64, 64, 3, 1, 1)]
+    ref, pl = _make(sc, layers, 2, 64, 32, 32, 2, 2, seed=5)
+    lv0, lv1 = pl.levels
+    g = synth.rng(5)
+    x = _dev(sc, pack_level(_round(synth.uniform(g, (2, 64, 32, 32)), dtype, sc), lv0), dtype)
+    w = _dev(sc, w_oihw_to_lib(_round(synth.kaiming(g, 64, 64, 3, 3), dtype, sc), lv0["Cpad"]), dtype)
+    y1 = torch.zeros(lv1["total_elems"], dtype=torch.bfloat16, device="cuda")
+    y2 = torch.zeros_like(y1)
+    sc.splitcnn_conv_fwd(pl.handle, 0, dtype, x, w, None, y1, sc.FLAG_RELU)
+    sc.splitcnn_conv_fwd(pl.handle, 0, dtype, x, w, None, y2, sc.FLAG_RELU, 0, 1)
+    sc.splitcnn_conv_fwd(pl.handle, 0, dtype, x, w, None, y2, sc.FLAG_RELU, 1, 4)
+    assert torch.equal(y1, y2)
+    ws_b = pl.workspace_size(0, dtype, 2)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    dw = torch.zeros((64, 3, 3, 64), dtype=torch.float32, device="cuda")
+    dwa = torch.zeros_like(dw)
+    dwb = torch.zeros_like(dw)
+    sc.splitcnn_conv_bwd_filter(pl.handle, 0, dtype, x, y1, dw, None, 0.0, ws, ws_b)
+    sc.splitcnn_conv_bwd_filter(pl.handle, 0, dtype, x, y1, dwa, None, 0.0, ws, ws_b, 0, 0, 2)
+    sc.splitcnn_conv_bwd_filter(pl.handle, 0, dtype, x, y1, dwb, None, 0.0, ws, ws_b, 0, 2, 4)
+    torch.testing.assert_close(dwa + dwb, dw, rtol=1e-5, atol=1e-5 * dw.abs().max().item())
+
+
+# --------------------------------------------------------------------------- split / merge
+@pytest.mark.parametrize("dtype_name", ["bf16", "fp32"])
+def test_split_merge_bit_exact(sc, dtype_name):
+    dtype = sc.BF16 if dtype_name == "bf16" else sc.FP32
+    for (N, C, H, W, nh, nw, seed) in [(2, 3, 32, 32, 2, 2, 0), (3, 13, 23, 17, 3, 2, 1), (2, 64, 28, 28, 4, 4, 2),
+                                       (1, 256, 56, 56, 8, 8, 3)]:
+        layers = [synth.conv(C, 8, 3, 1, 1)]
+        ref, pl = _make(sc, layers, N, C, H, W, nh, nw, seed)
+        lv0 = pl.levels[0]
+        g = synth.rng(seed)
+        X = _round(synth.uniform(g, (N, C, H, W)), dtype, sc)
+        xt = _dev(sc, X, dtype)
+        P = torch.full((lv0["total_elems"],), 5.0, dtype=_td(sc, dtype), device="cuda")
+        sc.splitcnn_split(pl.handle, 0, dtype, xt, sc.NCHW, P)
+        np.testing.assert_array_equal(_host(P), pack_level(X, lv0))
+        back = torch.zeros_like(xt)
+        sc.splitcnn_merge(pl.handle, 0, dtype, P, back, sc.NCHW)
+        assert torch.equal(back, xt)
+        # NHWC layout, and a partial patch range
+        xh = xt.permute(0, 2, 3, 1).contiguous()
+        P2 = torch.zeros_like(P)
+        npat = nh * nw
+        sc.splitcnn_split(pl.handle, 0, dtype, xh, sc.NHWC, P2, 0, npat // 2)
+        sc.splitcnn_split(pl.handle, 0, dtype, xh, sc.NHWC, P2, npat // 2, npat)
+        assert torch.equal(P2, P)
+        back2 = torch.zeros_like(xh)
+        sc.splitcnn_merge(pl.handle, 0, dtype, P2, back2, sc.NHWC)
+        assert torch.equal(back2, xh)
+
+
+# --------------------------------------------------------------------------- max-pool
+@pytest.mark.parametrize("dtype_name", ["bf16", "fp32"])
+@pytest.mark.parametrize("kind", ["2x2s2", "3x3s2p1"])
+def test_pool_parity(sc, dtype_name, kind):
+    dtype = sc.BF16 if dtype_name == "bf16" else sc.FP32
+    k, s, p = (2, 2, 0) if kind == "2x2s2" else (3, 2, 1)
+    N, C, H, W = 3, 24, 30, 22
+    layers = [synth.maxpool(C, k, s, p)]
+    ref, pl = _make(sc, layers, N, C, H, W, 3, 2, seed=11)
+    lp = ref.layers[0]
+    lv0, lv1 = pl.levels
+    g = synth.rng(11)
+    X = np.maximum(_round(synth.uniform(g, (N, C, H, W)), dtype, sc), 0)   # ReLU output: ties at 0 (R9)
+    X[:, :, ::3] = _round(synth.uniform(g, (N, C, (H + 2) // 3, W)), dtype, sc)
+    G = _round(synth.normal(g, (N, C, lp.H_out, lp.W_out)), dtype, sc)
+    x = _dev(sc, pack_level(X, lv0), dtype)
+    y = torch.zeros(lv1["total_elems"], dtype=_td(sc, dtype), device="cuda")
+    a = torch.zeros(lv1["total_elems"], dtype=torch.uint8, device="cuda")
+    sc.splitcnn_pool_fwd(pl.handle, 0, dtype, x, y, a, sc.FLAG_POOL_RELU_MASK)
+    Yref, Aref = O.pool_fwd(O.split(X, lp.Ih, lp.Iw), lp)
+    Ygot = unpack_level(_host(y), lv1)
+    Agot = unpack_level(a.cpu().numpy().astype(np.float64), lv1)
+    for i in range(3):
+        for j in range(2):
+            np.testing.assert_array_equal(Ygot[i][j], Yref[i][j])
+            np.testing.assert_array_equal(Agot[i][j].astype(np.int64) & 0x7F, Aref[i][j])
+            np.testing.assert_array_equal((Agot[i][j].astype(np.int64) >> 7) & 1, (Yref[i][j] > 0).astype(np.int64))
+    dy = _dev(sc, pack_level(G, lv1), dtype)
+    for flag in (0, sc.FLAG_POOL_RELU_MASK):
+        dx = torch.full((lv0["total_elems"],), 9.0, dtype=_td(sc, dtype), device="cuda")
+        sc.splitcnn_pool_bwd(pl.handle, 0, dtype, dy, a, dx, flag)
+        dXref = O.pool_bwd(O.split(G, lp.Oh, lp.Ow), Aref, lp)
+        if flag:
+            dXref = O.relu_mask(dXref, O.split(X, lp.Ih, lp.Iw))
+        dXgot = unpack_level(_host(dx), lv0)
+        for i in range(3):
+            for j in range(2):
+                if k == s:          # no overlap: a pure scatter, bit-exact
+                    np.testing.assert_array_equal(dXgot[i][j], dXref[i][j])
+                else:               # R10: overlapping windows accumulate in fp32
+                    assert normwise(dXgot[i][j], dXref[i][j]) <= (1e-6 if dtype == sc.FP32 else 1e-2)
+
+
+# --------------------------------------------------------------------------- offload / prefetch
+def test_offload_prefetch_roundtrip_bit_exact(sc):
+    dtype = sc.BF16
+    layers = [synth.conv(64, 64, 3, 1, 1)]
+    ref, pl = _make(sc, layers, 2, 64, 28, 28, 4, 4, seed=3)
+    lv0 = pl.levels[0]
+    x = torch.randn(lv0["total_elems"], device="cuda").to(torch.bfloat16)
+    keep = x.clone()
+    mem = torch.cuda.Stream()
+    ready = torch.cuda.Event()
+    ready.record()
+    hosts = []
+    for q in range(16):
+        off, nb = sc.splitcnn_patch_bytes(pl.handle, 0, dtype, q)
+        h = torch.empty(nb, dtype=torch.uint8, pin_memory=True)
+        done = torch.cuda.Event()
+        sc.splitcnn_offload(pl.handle, 0, dtype, q, x, h, ready, mem, done)
+        hosts.append((h, done))
+    for _, d in hosts:
+        torch.cuda.current_stream().wait_event(d)
+    x.zero_()
+    ready.record()
+    for q, (h, _) in enumerate(hosts):
+        d = torch.cuda.Event()
+        sc.splitcnn_prefetch(pl.handle, 0, dtype, q, h, x, ready, mem, d)
+        torch.cuda.current_stream().wait_event(d)
+    torch.cuda.synchronize()
+    assert torch.equal(x, keep)
+    with pytest.raises(sc.SplitCNNError, match="pinned"):
+        sc.splitcnn_offload(pl.handle, 0, dtype, 0, x, torch.empty(10 ** 6, dtype=torch.uint8), None, mem, None)

@@ -1,0 +1,350 @@
+"""bench.py -- VGG-19 Split-CNN fwd+bwd images/s on B200 (BASELINE.json metric).
+
+One STEP = one pass of the whole hot path over one synthetic batch: split ->
+per-patch conv(+bias+ReLU) / max-pool forward through the split region -> merge at the join ->
+unsplit tail -> backward (pool bwd, conv dgrad with fused ReLU mask, conv wgrad summed over
+patches and batch) [-> wgrad allreduce across ranks when N > 1].
+
+Default workload: C5 (VGG-19 224x224, global batch 256, 8x8 split at depth 50%).  Inputs are
+resident in HBM and far larger than L2 (126 MB), so no explicit L2 flush is needed.
+
+    python bench.py [--gpus N --steps K --warmup W --config C5|C2|C4 --impl ours|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "VGG-19 split-CNN fwd+bwd images/sec"
+UNIT = "images/s"
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d, "measured"
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled DURING the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index, self.rows, self.proc = index, [], None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.th = threading.Thread(target=self._read, daemon=True)
+            self.th.start()
+        except FileNotFoundError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        self.proc.wait()
+        self.th.join(timeout=2)
+        sm = [float(r[0]) for r in self.rows if r and r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if len(r) > 1 and r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in self.rows for k in range(4) if len(r) > 2 + k and r[2 + k] == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(sm)}
+
+
+# --------------------------------------------------------------------------- workloads
+def workload(name: str, N: int | None = None):
+    import synth
+    c = synth.vgg_config(name, N=N)
+    return c
+
+
+def make_inputs(c, dtype_t, device, world=1, rank=0):
+    """Seeded synthetic inputs: X ~ U[-1,1), W ~ Kaiming, b ~ U[-.1,.1), dY ~ N(0,1)."""
+    import torch
+    import synth
+    g = synth.rng(c["seed"])
+    params = [p for p in synth.layer_params(g, c["layers"] + c["tail"]) if p is not None]
+    gen = torch.Generator(device="cpu").manual_seed(c["seed"])
+    N = c["N"]
+    x = (torch.rand((N, 3, c["H"], c["W"]), generator=gen) * 2 - 1).to(dtype_t)
+    return params, x, gen
+
+
+# --------------------------------------------------------------------------- ours
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_asplos_jinh19_b200 import splitcnn as sc
+    from paper_conf_asplos_jinh19_b200.net import SplitNet
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.gpus != world:
+        world = max(world, 1)
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    c = workload(args.config)
+    dtype = sc.BF16 if args.dtype == "bf16" else sc.FP32
+    if world > 1:
+        from paper_conf_asplos_jinh19_b200.dist import DistSplitNet
+        net = DistSplitNet(c, world, rank, dtype)
+    else:
+        net = SplitNet(c["layers"], c["tail"], c["N"], 3, c["H"], c["W"], split=c["split"], mode=c["mode"],
+                       omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype)
+    params, x_host, gen = make_inputs(c, net.tdtype, "cuda")
+    net.set_params([(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params])
+    x = x_host.cuda()
+    out_numel = net.output_numel()
+    dy = torch.randn(out_numel, generator=gen).to(net.tdtype).cuda()
+    stream = torch.cuda.current_stream()
+
+    def step():
+        net.step(x, dy)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(args.warmup):
+        step()
+    barrier()
+    launches0 = sc.splitcnn_kernel_launches()
+    clocks = ClockSampler(local)
+    clocks.start()
+    net.timers = []
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier()
+    t0.record(stream)
+    for _ in range(args.steps):
+        step()
+    t1.record(stream)
+    barrier()
+    clk = clocks.stop()
+    launches = sc.splitcnn_kernel_launches() - launches0
+    ms = t0.elapsed_time(t1)
+    if world > 1:
+        tt = torch.tensor([ms], device="cuda")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ms = tt.item()
+    # per-kind device time from the events recorded around every library call
+    kinds = {}
+    for kind, e0, e1, work in net.timers:
+        k = kinds.setdefault(kind, [0.0, 0.0, 0])
+        k[0] += e0.elapsed_time(e1)
+        k[1] += work
+        k[2] += 1
+    net.timers = None
+    ms_step = ms / args.steps
+    global_batch = c["N"]
+    value = global_batch / (ms_step / 1e3)
+
+    # e2e: the same step through the public API with host buffers: pinned H2D of x and dY every
+    # step, D2H of the step's result (all weight / bias gradients) every step
+    xh = x_host.pin_memory()
+    dyh = dy.cpu().pin_memory()
+    grads = [t for pair in net.grads.values() for t in pair]
+    gh = [torch.empty(t.shape, dtype=t.dtype, pin_memory=True) for t in grads]
+    h2d = xh.numel() * xh.element_size() + dyh.numel() * dyh.element_size()
+    d2h = sum(t.numel() * t.element_size() for t in grads)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ke = max(1, min(args.steps, 10))
+    barrier()
+    e0.record(stream)
+    for _ in range(ke):
+        x.copy_(xh, non_blocking=True)
+        dy.copy_(dyh, non_blocking=True)
+        net.step(x, dy)
+        for t, h in zip(grads, gh):
+            h.copy_(t, non_blocking=True)
+    e1.record(stream)
+    barrier()
+    ms_e2e = e0.elapsed_time(e1) / ke
+    if world > 1:
+        tt = torch.tensor([ms_e2e], device="cuda")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ms_e2e = tt.item()
+
+    peaks, src = _peaks()
+    conv_ms = sum(kinds[k][0] for k in kinds if k.startswith("conv"))
+    conv_flop = sum(kinds[k][1] for k in kinds if k.startswith("conv"))
+    conv_launch_count = sum(kinds[k][2] for k in kinds if k.startswith("conv"))
+    achieved = conv_flop / (conv_ms / 1e3) / 1e12 if conv_ms > 0 else 0.0
+    peak = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])
+    if args.dtype == "fp32":
+        peak = 75.0     # FP32 SIMT nominal (App. B); fp32 path runs on FFMA
+    hbm_ms = sum(kinds[k][0] for k in kinds if not k.startswith("conv"))
+    hbm_bytes = sum(kinds[k][1] for k in kinds if not k.startswith("conv"))
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
+    if os.path.exists(tp):
+        traffic = json.load(open(tp)).get("conv_bytes_per_launch")
+    line = {
+        "metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True,
+        "scaling": "strong" if world > 1 else "weak", "vs_baseline": None,
+        "dtype": args.dtype, "data": "synthetic (seeded PCG64 / torch.Generator; random-init weights)",
+        "config": {"workload": f"{args.config}: {c['desc']}", "global_batch": global_batch,
+                   "image": [c["H"], c["W"]], "split": list(c["split"]), "split_mode": c["mode"],
+                   "split_convs": sum(1 for l in c["layers"] if l["op"] == "conv"),
+                   "parallelism": f"patch{world}" if world > 1 else "1gpu",
+                   "l2": "inputs/activations >> 126 MB L2 (no flush needed)"},
+        "e2e": {"value": round(global_batch / (ms_e2e / 1e3), 2), "unit": UNIT, "h2d_bytes_per_step": h2d,
+                "d2h_bytes_per_step": d2h},
+        "gpu_launches": launches,
+        "roofline": {"bound": "tensor", "kernel": "split conv (fwd+dgrad+wgrad, all layers)",
+                     "achieved": round(achieved, 2), "peak": peak, "unit": "TFLOP/s",
+                     "frac": round(achieved / peak, 4), "traffic": traffic,
+                     "peak_source": f"{src} bf16_tflops_sustained" if args.dtype == "bf16" else "nominal FP32 SIMT",
+                     "conv_share_of_step": round(conv_ms / max(ms, 1e-9), 4),
+                     "conv_launches_timed": conv_launch_count},
+        "hbm_ops": {"kinds": sorted(k for k in kinds if not k.startswith("conv")),
+                    "achieved_gbs": round(hbm_bytes / (hbm_ms / 1e3) / 1e9, 1) if hbm_ms > 0 else None,
+                    "peak_gbs": peaks["hbm_gbs"], "share_of_step": round(hbm_ms / max(ms, 1e-9), 4)},
+        "per_kind_ms_per_step": {k: round(v[0] / args.steps, 4) for k, v in kinds.items()},
+        "clocks": clk,
+    }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(args.config, budget_tiles=args.cpu_tiles)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+# --------------------------------------------------------------------------- oracle timing
+def oracle_sample_time(config: str, tiles: int):
+    """Time the ORACLE (as it stands) on a bounded sample of one step and scale to images/s.
+
+    Sample: 1 image; for every layer-op of the step (conv fwd / dgrad / wgrad, pool fwd / bwd) the
+    oracle runs on `tiles` output tiles, each 1/64 of the layer's output plane (region layers: one
+    of the plan's patches of a 8x8 even split of that level; tail layers: a 1/8 x 1/8 crop with the
+    layer's own padding).  Work is linear in output pixels, so time/image = sum over ops of
+    t(sample) * (output pixels of the op) / (sample output pixels)."""
+    import numpy as np
+    import synth
+    from oracle import ops as O
+    from oracle import plan as OP
+
+    c = workload(config, N=1)
+    g = synth.rng(c["seed"])
+    layers = c["layers"] + c["tail"]
+    params = synth.layer_params(g, layers)
+    H = c["H"]
+    total = 0.0
+    sample_px = 0
+    h = H
+    first_conv = True
+    for l, prm in zip(layers, params):
+        ho = OP.out_len(h, l["kh"], l["sh"], l["ph_b"], l["ph_e"])
+        # a tile = a patch of an 8x8 even split of this layer's output (>= 1 px)
+        n = min(8, ho)
+        Ob = OP.boundaries_even(ho, n)
+        lp = OP.plan([l], 1, l["cin"], h, h, Ob, Ob).layers[0]
+        t_layer = 0.0
+        px_s = 0
+        for t in range(tiles):
+            i, j = (t // n) % n, t % n
+            hp, wp = lp.Ih[i + 1] - lp.Ih[i], lp.Iw[j + 1] - lp.Iw[j]
+            X = g.uniform(-1, 1, (1, l["cin"], hp, wp))
+            if l["op"] == "conv":
+                W, b = prm
+                t0 = time.perf_counter()
+                Y = O.conv_fwd_patch(X, W, b, l["sh"], l["sw"], lp.pads_h[i], lp.pads_w[j], True)
+                if not first_conv:    # the step computes no input gradient for the first conv
+                    O.conv_bwd_data_patch(Y, W, hp, wp, l["sh"], l["sw"], lp.pads_h[i], lp.pads_w[j], X)
+                O.conv_bwd_filter_patch(X, Y, l["kh"], l["kw"], l["sh"], l["sw"], lp.pads_h[i], lp.pads_w[j])
+                t_layer += time.perf_counter() - t0
+            else:
+                t0 = time.perf_counter()
+                Y, A = O.pool_fwd_patch(X, l["kh"], l["kw"], l["sh"], l["sw"], lp.pads_h[i], lp.pads_w[j])
+                O.pool_bwd_patch(Y, A, hp, wp, l["kh"], l["kw"], l["sh"], l["sw"], lp.pads_h[i], lp.pads_w[j])
+                t_layer += time.perf_counter() - t0
+            px_s += (lp.Oh[i + 1] - lp.Oh[i]) * (lp.Ow[j + 1] - lp.Ow[j])
+        total += t_layer * (ho * ho) / px_s
+        first_conv = first_conv and l["op"] != "conv"
+        sample_px += px_s
+        h = ho
+    return total, f"1 image, {tiles} of 64 output tiles per layer-op (fwd+dgrad+wgrad / pool fwd+bwd), scaled by output pixels"
+
+
+def cpu_baseline(config: str, budget_tiles: int = 4):
+    import os as _os
+    t_img, sample = oracle_sample_time(config, budget_tiles)
+    cores = len(_os.sched_getaffinity(0))
+    return {"value": round(1.0 / t_img, 5), "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample,
+            "seconds_per_image_est": round(t_img, 2)}
+
+
+def run_reference(args):
+    """--impl reference: the oracle (test infrastructure) timed as it stands on the host cores."""
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    c = workload(args.config)
+    for _ in range(args.warmup):
+        oracle_sample_time(args.config, 1)
+    vals, t0 = [], time.perf_counter()
+    for _ in range(args.steps):
+        t_img, sample = oracle_sample_time(args.config, 1)
+        vals.append(t_img * c["N"])
+    ms_step = 1e3 * statistics.mean(vals)
+    value = c["N"] / (ms_step / 1e3)
+    cores = len(os.sched_getaffinity(0))
+    line = {"impl": "reference", "metric": METRIC, "value": round(value, 6), "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 1), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"{args.config}: {c['desc']}", "global_batch": c["N"]},
+            "cpu_baseline": {"kind": "oracle", "cores": cores, "sample": sample, "value": round(value, 6)},
+            "e2e": {"value": round(value, 6), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+            "wall_s": round(time.perf_counter() - t0, 1)}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C5", choices=["C2", "C4", "C5"])
+    ap.add_argument("--dtype", default="bf16", choices=["bf16", "fp32"])
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--cpu-tiles", type=int, default=12)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -126,6 +126,8 @@ typedef struct {
 SPLITCNN_API const char *splitcnn_last_error(void);
 SPLITCNN_API const char *splitcnn_status_string(splitcnn_status_t s);
 SPLITCNN_API const char *splitcnn_version(void);
+/* Total number of CUDA kernels this library has launched in the process (instrumentation). */
+SPLITCNN_API splitcnn_status_t splitcnn_kernel_launches(uint64_t *count);
 
 /* ------------------------------------------------------------------ boundaries (host) */
 /* "As evenly as possible": O[i] = floor(i * L / n), O[n] = L.

@@ -1,5 +1,6 @@
 // api.cu -- the extern "C" entry points of libsplitcnn (see include/splitcnn.h).
 // Argument validation, error plumbing and kernel dispatch; all arithmetic is in the kernels.
+#include <atomic>
 #include <cstdio>
 #include <cstring>
 #include <string>
@@ -9,6 +10,9 @@
 namespace splitcnn {
 
 static thread_local std::string g_last_error;
+static std::atomic<uint64_t> g_launches{0};
+
+void count_launch(int n) { g_launches.fetch_add((uint64_t)n, std::memory_order_relaxed); }
 
 void set_error(const std::string &msg) { g_last_error = msg; }
 
@@ -39,6 +43,12 @@ extern "C" const char *splitcnn_status_string(splitcnn_status_t s) {
         case SPLITCNN_ERR_OOM: return "out of memory";
     }
     return "unknown status";
+}
+
+extern "C" splitcnn_status_t splitcnn_kernel_launches(uint64_t *count) {
+    if (!count) return fail(SPLITCNN_ERR_INVALID_VALUE, "null count");
+    *count = g_launches.load(std::memory_order_relaxed);
+    return SPLITCNN_OK;
 }
 
 extern "C" const char *splitcnn_version(void) { return "splitcnn-b200 0.1 (sm_100a)"; }

@@ -67,3 +67,7 @@ splitcnn_status_t fail(splitcnn_status_t s, const std::string &msg);
 splitcnn_status_t check_launch(const char *what);
 
 }  // namespace splitcnn
+
+namespace splitcnn {
+void count_launch(int n = 1);  // every kernel launch of the library (splitcnn_kernel_launches)
+}

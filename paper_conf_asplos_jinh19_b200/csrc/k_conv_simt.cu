@@ -228,6 +228,21 @@ __global__ void __launch_bounds__(256) reduce_partials_kernel(const float *__res
     }
 }
 
+void launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, float *part, int cout, int p0, int p1,
+                        int cpp, cudaStream_t st) {
+    const int Z = (p1 - p0) * cpp;
+    if (dt == SPLITCNN_BF16)
+        db_partial_kernel<__nv_bfloat16><<<Z, 256, 0, st>>>(make_level_desc(Lo), (const __nv_bfloat16 *)dy, part, cout, p0, cpp);
+    else
+        db_partial_kernel<float><<<Z, 256, 0, st>>>(make_level_desc(Lo), (const float *)dy, part, cout, p0, cpp);
+    count_launch();
+}
+
+void launch_reduce(const float *part, int Z, int64_t n, float *out, float beta, cudaStream_t st) {
+    reduce_partials_kernel<<<(unsigned)std::min<int64_t>((n + 255) / 256, 4096), 256, 0, st>>>(part, Z, n, out, beta);
+    count_launch();
+}
+
 static int64_t max_pixels(const Level &L, int p0, int p1) {
     int64_t m = 0;
     for (int q = p0; q < p1; ++q) {
@@ -245,6 +260,7 @@ void launch_conv_fwd_simt(splitcnn_dtype_t dt, const Level &Li, const Level &Lo,
     dim3 grid((unsigned)((max_pixels(Lo, p0, p1) + BM - 1) / BM), (Lo.Cpad + BN - 1) / BN, p1 - p0);
     if (dt == SPLITCNN_BF16) conv_simt_kernel<__nv_bfloat16, MODE_FWD><<<grid, NT, 0, st>>>(a);
     else conv_simt_kernel<float, MODE_FWD><<<grid, NT, 0, st>>>(a);
+    count_launch();
 }
 
 void launch_conv_dgrad_simt(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy,
@@ -255,6 +271,7 @@ void launch_conv_dgrad_simt(splitcnn_dtype_t dt, const Level &Li, const Level &L
     dim3 grid((unsigned)((max_pixels(Li, p0, p1) + BM - 1) / BM), (Li.Cpad + BN - 1) / BN, p1 - p0);
     if (dt == SPLITCNN_BF16) conv_simt_kernel<__nv_bfloat16, MODE_DGRAD><<<grid, NT, 0, st>>>(a);
     else conv_simt_kernel<float, MODE_DGRAD><<<grid, NT, 0, st>>>(a);
+    count_launch();
 }
 
 // split-K chunking for the wgrad: a fixed function of the plan, so workspace_size agrees.
@@ -290,14 +307,15 @@ void launch_conv_wgrad_simt(splitcnn_dtype_t dt, const Level &Li, const Level &L
     dim3 grid((g.L.cout + BM - 1) / BM, (ncols + BN - 1) / BN, Z);
     if (dt == SPLITCNN_BF16) conv_simt_kernel<__nv_bfloat16, MODE_WGRAD><<<grid, NT, 0, st>>>(a);
     else conv_simt_kernel<float, MODE_WGRAD><<<grid, NT, 0, st>>>(a);
+    count_launch();
     const int64_t n = (int64_t)g.L.cout * ncols;
-    reduce_partials_kernel<<<(unsigned)std::min<int64_t>((n + 255) / 256, 4096), 256, 0, st>>>(part, Z, n, dw, beta);
+    { reduce_partials_kernel<<<(unsigned)std::min<int64_t>((n + 255) / 256, 4096), 256, 0, st>>>(part, Z, n, dw, beta); count_launch(); }
     if (db) {
         if (dt == SPLITCNN_BF16)
-            db_partial_kernel<__nv_bfloat16><<<Z, 256, 0, st>>>(make_level_desc(Lo), (const __nv_bfloat16 *)dy, part_db, g.L.cout, p0, cpp);
+            { db_partial_kernel<__nv_bfloat16><<<Z, 256, 0, st>>>(make_level_desc(Lo), (const __nv_bfloat16 *)dy, part_db, g.L.cout, p0, cpp); count_launch(); }
         else
-            db_partial_kernel<float><<<Z, 256, 0, st>>>(make_level_desc(Lo), (const float *)dy, part_db, g.L.cout, p0, cpp);
-        reduce_partials_kernel<<<(g.L.cout + 255) / 256, 256, 0, st>>>(part_db, Z, g.L.cout, db, beta);
+            { db_partial_kernel<float><<<Z, 256, 0, st>>>(make_level_desc(Lo), (const float *)dy, part_db, g.L.cout, p0, cpp); count_launch(); }
+        { reduce_partials_kernel<<<(g.L.cout + 255) / 256, 256, 0, st>>>(part_db, Z, g.L.cout, db, beta); count_launch(); }
     }
 }
 

@@ -1,13 +1,765 @@
-// k_conv_tc.cu -- tcgen05 implicit-GEMM split convolution (placeholder until the kernel lands).
+// k_conv_tc.cu -- tcgen05 implicit-GEMM split convolution for sm_100a (bf16 in, fp32 accumulate).
+//
+// One persistent, warp-specialised kernel serves the forward pass (Eq. 6) and the stride-1
+// data gradient (the forward mainloop on dY with spatially flipped, transposed weights and the
+// complementary per-patch pads k-1-p).  The patch-local zero padding of Split-CNN is folded into
+// the tile loads: every patch gets its OWN 4-D TMA tensor map whose extents are the patch
+// extents, so TMA's out-of-bounds zero fill IS the patch padding -- no window ever reads across a
+// patch boundary and the kernel has no boundary branches.
+//
+//   GEMM view (per patch):  M = output pixels (n, oh, ow) tiled as BNn x BH x BW boxes (<= 128 rows),
+//                           N = output channels (BN <= 256 per tile), K = taps x input channels.
+//   warp 0      TMA producer: per K step one 4-D box of the input patch at the tap's offset
+//               (element strides = conv stride) + one 2-D box of the weights, 128B/64B/32B swizzle
+//   warp 1      MMA issuer (one thread): tcgen05.mma 128 x BN x 16 into a TMEM accumulator;
+//               tcgen05.commit frees the smem stage / publishes the accumulator
+//   warps 2-5   epilogue: tcgen05.ld -> +bias, ReLU (fwd) or ReLU-mask (dgrad) -> bf16 -> global
+//   TMEM accumulators are double-buffered so the epilogue of tile t overlaps the mainloop of t+1.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <cstring>
+#include <mutex>
+#include <vector>
+
+#include "common.cuh"
 #include "kernels.h"
+#include "tc_ptx.cuh"
 
 namespace splitcnn {
-bool conv_tc_supported(int, splitcnn_dtype_t, const Level &, const Level &, const LayerGeom &) { return false; }
-size_t conv_tc_ws_bytes(int, const Level &, const Level &, const LayerGeom &) { return 0; }
-splitcnn_status_t launch_conv_fwd_tc(const Level &, const Level &, const LayerGeom &, const void *, const void *,
-                                     const float *, void *, int, int, int, cudaStream_t) { return fail(SPLITCNN_ERR_UNSUPPORTED, "tc"); }
-splitcnn_status_t launch_conv_dgrad_tc(const Level &, const Level &, const LayerGeom &, const void *, const void *,
-                                       void *, const void *, void *, int, int, cudaStream_t) { return fail(SPLITCNN_ERR_UNSUPPORTED, "tc"); }
-splitcnn_status_t launch_conv_wgrad_tc(const Level &, const Level &, const LayerGeom &, const void *, const void *,
-                                       float *, float *, float, void *, int, int, cudaStream_t) { return fail(SPLITCNN_ERR_UNSUPPORTED, "tc"); }
+
+constexpr int TC_MAXP = 64;  // patches per launch (tensor maps live in the kernel parameters)
+
+static bool wgrad_tc_ok(const Level &Li, const Level &Lo, const LayerGeom &g);
+size_t wgrad_tc_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g);
+
+struct TcConvParams {
+    CUtensorMap mapA[TC_MAXP];
+    CUtensorMap mapB;
+    int64_t out_off[TC_MAXP];
+    int tile_prefix[TC_MAXP + 1];
+    int out_h[TC_MAXP], out_w[TC_MAXP];
+    int pt[TC_MAXP], pl[TC_MAXP];
+    int nhb[TC_MAXP], nwb[TC_MAXP];
+    int npatch;
+    int N, BW, BH, BNn, rows_box, nnb, nco;
+    int kh, kw, s;
+    int cpadc;       // channels per A box (min(Cpad_A, 64))
+    int cchunks;     // 64-channel chunks per tap (Cpad_A >= 64)
+    int tps;         // taps per K step (Cpad_A < 64)
+    int ksteps;      // K steps per tile
+    int kchan;       // Cpad of the A side (K = taps * kchan)
+    int BN, Cout, Cpo;
+    int stages;
+    uint32_t tmem_cols;
+    uint32_t a_layout, a_sbo, a_lbo, a_chunk_bytes, a_tx_bytes, b_tx_bytes;
+    const float *bias;
+    __nv_bfloat16 *y;
+    const __nv_bfloat16 *relu_src;
+    int relu;
+};
+
+__device__ __forceinline__ void decode_tile(const TcConvParams &p, int t, int &ql, int &nb, int &hb, int &wb, int &cb) {
+    ql = 0;
+    while (t >= p.tile_prefix[ql + 1]) ++ql;
+    int idx = t - p.tile_prefix[ql];
+    cb = idx % p.nco;
+    idx /= p.nco;
+    wb = idx % p.nwb[ql];
+    idx /= p.nwb[ql];
+    hb = idx % p.nhb[ql];
+    nb = idx / p.nhb[ql];
+}
+
+__global__ void __launch_bounds__(192, 1) conv_tc_kernel(const __grid_constant__ TcConvParams p) {
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+    const int S = p.stages;
+    const uint32_t b_stage = (uint32_t)p.BN * 128u;
+    uint8_t *sA = smem;
+    uint8_t *sB = smem + (size_t)S * 16384;
+    uint64_t *full = (uint64_t *)(sB + (size_t)S * b_stage);
+    uint64_t *empty = full + S;
+    uint64_t *tfull = empty + S;
+    uint64_t *tempty = tfull + 2;
+    uint32_t *tmem_slot = (uint32_t *)(tempty + 2);
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (warp == 0 && lane == 0) {
+        for (int s = 0; s < S; ++s) {
+            tc::mbar_init(&full[s], 1);
+            tc::mbar_init(&empty[s], 1);
+        }
+        for (int a = 0; a < 2; ++a) {
+            tc::mbar_init(&tfull[a], 1);
+            tc::mbar_init(&tempty[a], 4);
+        }
+        tc::fence_barrier_init();
+    }
+    if (warp == 1) tc::tmem_alloc_dyn(tmem_slot, p.tmem_cols);
+    tc::tc_fence_before();
+    __syncthreads();
+    tc::tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+    const int total = p.tile_prefix[p.npatch];
+    const int KT = p.kh * p.kw;
+
+    if (warp == 0) {
+        if (lane == 0) {
+            // ================= TMA producer
+            for (int q = 0; q < p.npatch; ++q) tc::tma_prefetch_desc(&p.mapA[q]);
+            tc::tma_prefetch_desc(&p.mapB);
+            int stage = 0;
+            uint32_t ph = 0;
+            for (int t = blockIdx.x; t < total; t += gridDim.x) {
+                int ql, nb, hb, wb, cb;
+                decode_tile(p, t, ql, nb, hb, wb, cb);
+                const int wbase = wb * p.BW * p.s - p.pl[ql];
+                const int hbase = hb * p.BH * p.s - p.pt[ql];
+                const int n0 = nb * p.BNn, co0 = cb * p.BN;
+                for (int ks = 0; ks < p.ksteps; ++ks) {
+                    tc::mbar_wait(&empty[stage], ph ^ 1);
+                    tc::mbar_arrive_expect_tx(&full[stage], p.a_tx_bytes + p.b_tx_bytes);
+                    uint8_t *a = sA + (size_t)stage * 16384;
+                    uint8_t *b = sB + (size_t)stage * b_stage;
+                    if (p.tps > 1) {
+                        for (int j = 0; j < p.tps; ++j) {
+                            const int tap = min(ks * p.tps + j, KT - 1);  // past the last tap: weights are OOB zero
+                            const int r = tap / p.kw, c = tap - r * p.kw;
+                            tc::tma_load_4d(a + j * p.a_chunk_bytes, &p.mapA[ql], &full[stage], 0, wbase + c, hbase + r, n0);
+                        }
+                        tc::tma_load_2d(b, &p.mapB, &full[stage], ks * 64, co0);
+                    } else {
+                        const int tap = ks / p.cchunks, cc = ks - tap * p.cchunks;
+                        const int r = tap / p.kw, c = tap - r * p.kw;
+                        tc::tma_load_4d(a, &p.mapA[ql], &full[stage], cc * 64, wbase + c, hbase + r, n0);
+                        tc::tma_load_2d(b, &p.mapB, &full[stage], tap * p.kchan + cc * 64, co0);
+                    }
+                    if (++stage == S) { stage = 0; ph ^= 1; }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            // ================= MMA issuer
+            const uint32_t idesc = tc::idesc_bf16(128, p.BN);
+            int stage = 0, acc = 0;
+            uint32_t ph = 0, aph = 0;
+            for (int t = blockIdx.x; t < total; t += gridDim.x) {
+                tc::mbar_wait(&tempty[acc], aph ^ 1);
+                tc::tc_fence_after();
+                const uint32_t d = tmem_base + (uint32_t)(acc * p.BN);
+                for (int ks = 0; ks < p.ksteps; ++ks) {
+                    tc::mbar_wait(&full[stage], ph);
+                    tc::tc_fence_after();
+                    const uint32_t a_base = tc::smem_u32(sA + (size_t)stage * 16384);
+                    const uint32_t b_base = tc::smem_u32(sB + (size_t)stage * b_stage);
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const int k0 = 16 * j;
+                        const int chunk = k0 / p.cpadc;
+                        const uint32_t a_addr = a_base + chunk * p.a_chunk_bytes + (uint32_t)((k0 - chunk * p.cpadc) * 2);
+                        const uint64_t adesc = tc::smem_desc(a_addr, p.a_lbo, p.a_sbo, p.a_layout);
+                        const uint64_t bdesc = tc::smem_desc(b_base + 32u * j, 16, 1024, 2);
+                        tc::mma_bf16(d, adesc, bdesc, idesc, (ks | j) != 0);
+                    }
+                    tc::mma_commit(&empty[stage]);
+                    if (++stage == S) { stage = 0; ph ^= 1; }
+                }
+                tc::mma_commit(&tfull[acc]);
+                acc ^= 1;
+                if (acc == 0) aph ^= 1;
+            }
+        }
+    } else {
+        // ================= epilogue (warps 2..5 -> TMEM lane quadrants 2,3,0,1)
+        const int quad = warp & 3;
+        const int row = quad * 32 + lane;
+        const int wi = row % p.BW, hi = (row / p.BW) % p.BH, ni = row / (p.BW * p.BH);
+        int acc = 0;
+        uint32_t aph = 0;
+        for (int t = blockIdx.x; t < total; t += gridDim.x) {
+            int ql, nb, hb, wb, cb;
+            decode_tile(p, t, ql, nb, hb, wb, cb);
+            const int n = nb * p.BNn + ni, oh = hb * p.BH + hi, ow = wb * p.BW + wi;
+            const bool valid = row < p.rows_box && n < p.N && oh < p.out_h[ql] && ow < p.out_w[ql];
+            const int64_t base = p.out_off[ql] + (((int64_t)n * p.out_h[ql] + oh) * p.out_w[ql] + ow) * p.Cpo;
+            const int co0 = cb * p.BN;
+            tc::mbar_wait(&tfull[acc], aph);
+            tc::tc_fence_after();
+            const uint32_t tacc = tmem_base + (uint32_t)(acc * p.BN) + ((uint32_t)(quad * 32) << 16);
+            for (int cc = 0; cc < p.BN; cc += 16) {
+                float v[16];
+                tc::tmem_ld16(tacc + cc, v);
+                if (!valid) continue;
+#pragma unroll
+                for (int g = 0; g < 2; ++g) {
+                    const int co = co0 + cc + 8 * g;
+                    if (co >= p.Cpo) break;
+                    float o[8];
+#pragma unroll
+                    for (int e = 0; e < 8; ++e) {
+                        float x = v[8 * g + e];
+                        if (co + e < p.Cout) {
+                            if (p.bias) x += __ldg(p.bias + co + e);
+                            if (p.relu) x = fmaxf(x, 0.f);
+                        } else {
+                            x = 0.f;
+                        }
+                        o[e] = x;
+                    }
+                    if (p.relu_src) {
+                        float m[8];
+                        load8(p.relu_src + base + co, m);
+#pragma unroll
+                        for (int e = 0; e < 8; ++e) o[e] = (m[e] > 0.f) ? o[e] : 0.f;
+                    }
+                    store8(p.y + base + co, o);
+                }
+            }
+            tc::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(&tempty[acc]);
+            acc ^= 1;
+            if (acc == 0) aph ^= 1;
+        }
+    }
+    tc::tc_fence_before();
+    __syncthreads();
+    tc::tc_fence_after();
+    if (warp == 1) tc::tmem_dealloc(tmem_base, p.tmem_cols);
+}
+
+// dgrad weights: W'[ci][r'][c'][co] = W[co][kh-1-r'][kw-1-c'][ci], zero for co >= Cout
+__global__ void flip_weights_kernel(const __nv_bfloat16 *__restrict__ W, __nv_bfloat16 *__restrict__ Wt, int Cout,
+                                    int Cpad_in, int Cin, int kh, int kw, int Cpad_out) {
+    const int64_t n = (int64_t)Cin * kh * kw * Cpad_out;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const int co = (int)(i % Cpad_out);
+        int64_t t = i / Cpad_out;
+        const int c = (int)(t % kw);
+        t /= kw;
+        const int r = (int)(t % kh);
+        const int ci = (int)(t / kh);
+        Wt[i] = co < Cout ? W[(((int64_t)co * kh + (kh - 1 - r)) * kw + (kw - 1 - c)) * Cpad_in + ci] : __float2bfloat16(0.f);
+    }
+}
+
+// ============================================================ host side
+namespace {
+
+PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        cudaDriverEntryPointQueryResult q;
+        void *p = nullptr;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = (PFN_cuTensorMapEncodeTiled_v12000)p;
+    });
+    return fn;
+}
+
+int num_sms() {
+    static int n = 0;
+    if (!n) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        if (n <= 0) n = 148;
+    }
+    return n;
+}
+
+CUtensorMapSwizzle swz_for(int row_bytes) {
+    switch (row_bytes) {
+        case 128: return CU_TENSOR_MAP_SWIZZLE_128B;
+        case 64: return CU_TENSOR_MAP_SWIZZLE_64B;
+        case 32: return CU_TENSOR_MAP_SWIZZLE_32B;
+        default: return CU_TENSOR_MAP_SWIZZLE_NONE;
+    }
+}
+uint32_t layout_for(int row_bytes) {  // tcgen05 descriptor layout code
+    switch (row_bytes) {
+        case 128: return 2;
+        case 64: return 4;
+        case 32: return 6;
+        default: return 0;
+    }
+}
+
+struct TileShape {
+    int BW, BH, BNn;
+};
+
+// choose the pixel box (BW x BH x BNn <= 128 rows) minimising the number of tiles over the patches
+TileShape choose_tile(const std::vector<std::pair<int, int>> &ext, int N, int s) {
+    int maxh = 1, maxw = 1;
+    for (auto &e : ext) { maxh = std::max(maxh, e.first); maxw = std::max(maxw, e.second); }
+    TileShape best{1, 1, 1};
+    long best_tiles = -1;
+    const int wlim = std::min(std::min(maxw, 128), 256 / s), hlim = std::min(std::min(maxh, 128), 256 / s);
+    for (int bw = 1; bw <= wlim; ++bw) {
+        for (int bh = 1; bh <= hlim && bw * bh <= 128; ++bh) {
+            const int bn = std::min(std::min(128 / (bw * bh), N), 256);
+            long tiles = 0;
+            for (auto &e : ext)
+                tiles += (long)((N + bn - 1) / bn) * ((e.first + bh - 1) / bh) * ((e.second + bw - 1) / bw);
+            if (best_tiles < 0 || tiles < best_tiles || (tiles == best_tiles && bw > best.BW)) {
+                best_tiles = tiles;
+                best = {bw, bh, bn};
+            }
+        }
+    }
+    return best;
+}
+
+int round_up16(int x) { return (x + 15) / 16 * 16; }
+
+bool a_channels_ok(int cpad) { return cpad == 8 || cpad == 16 || cpad == 32 || cpad % 64 == 0; }
+
+// mode 0: forward (A = X at level m, out = level m+1); mode 1: dgrad (A = dY at level m+1, out = level m)
+splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const LayerGeom &g, const void *a_ptr,
+                            const void *w_ptr, int w_rows, const float *bias, void *y, const void *relu_src, int relu,
+                            int p0, int p1, cudaStream_t st) {
+    auto encode = get_encode();
+    if (!encode) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+    const int kh = g.L.kh, kw = g.L.kw, s = mode == 0 ? g.L.sh : 1;
+    const int cpad = La.Cpad;
+    const int cpadc = std::min(cpad, 64);
+    const int ncols_out = mode == 0 ? g.L.cout : g.L.cin;
+    const int BN = std::min(256, round_up16(ncols_out));
+    const int nco = (ncols_out + BN - 1) / BN;
+    const int N = La.N;
+    static bool attr_set = false;
+    for (int g0 = p0; g0 < p1; g0 += TC_MAXP) {
+        const int g1 = std::min(p1, g0 + TC_MAXP);
+        std::vector<std::pair<int, int>> ext;
+        for (int q = g0; q < g1; ++q) {
+            const int i = q / Lout.nw(), j = q % Lout.nw();
+            ext.push_back({Lout.ph(i), Lout.pw(j)});
+        }
+        const TileShape ts = choose_tile(ext, N, s);
+        static thread_local TcConvParams P;  // large; avoid the stack
+        std::memset(&P, 0, sizeof(P));
+        P.npatch = g1 - g0;
+        P.N = N; P.BW = ts.BW; P.BH = ts.BH; P.BNn = ts.BNn; P.rows_box = ts.BW * ts.BH * ts.BNn;
+        P.nnb = (N + ts.BNn - 1) / ts.BNn;
+        P.nco = nco;
+        P.kh = kh; P.kw = kw; P.s = s;
+        P.cpadc = cpadc;
+        P.kchan = cpad;
+        if (cpad >= 64) {
+            P.cchunks = cpad / 64; P.tps = 1; P.ksteps = kh * kw * P.cchunks;
+        } else {
+            P.cchunks = 1; P.tps = 64 / cpad; P.ksteps = (kh * kw + P.tps - 1) / P.tps;
+        }
+        P.BN = BN; P.Cout = ncols_out; P.Cpo = Lout.Cpad;
+        const int row_bytes = cpadc * 2;
+        P.a_layout = layout_for(row_bytes);
+        P.a_sbo = 8u * row_bytes;
+        P.a_chunk_bytes = 128u * row_bytes;
+        P.a_lbo = row_bytes == 16 ? P.a_chunk_bytes : 16u;
+        P.a_tx_bytes = (uint32_t)P.tps * P.rows_box * row_bytes;
+        P.b_tx_bytes = (uint32_t)BN * 128u;
+        const uint32_t stage_bytes = 16384u + P.b_tx_bytes;
+        P.stages = std::min<int>(8, (int)((200u * 1024u) / stage_bytes));
+        uint32_t cols = 32;
+        while (cols < 2u * BN) cols <<= 1;
+        P.tmem_cols = cols;
+        P.bias = bias;
+        P.y = (__nv_bfloat16 *)y;
+        P.relu_src = (const __nv_bfloat16 *)relu_src;
+        P.relu = relu;
+        int tiles = 0;
+        for (int q = g0; q < g1; ++q) {
+            const int ql = q - g0;
+            const int i = q / Lout.nw(), j = q % Lout.nw();
+            const int oh = Lout.ph(i), ow = Lout.pw(j);
+            P.out_h[ql] = oh; P.out_w[ql] = ow;
+            P.out_off[ql] = Lout.offset(i, j);
+            const int pt = g.pad_h[2 * i], pl = g.pad_w[2 * j];
+            P.pt[ql] = mode == 0 ? pt : kh - 1 - pt;
+            P.pl[ql] = mode == 0 ? pl : kw - 1 - pl;
+            P.nhb[ql] = (oh + ts.BH - 1) / ts.BH;
+            P.nwb[ql] = (ow + ts.BW - 1) / ts.BW;
+            P.tile_prefix[ql] = tiles;
+            tiles += P.nnb * P.nhb[ql] * P.nwb[ql] * nco;
+            // A map over the patch buffer: dims (C, W, H, N), TMA zero fill = patch padding
+            const int hp = La.ph(i), wp = La.pw(j);
+            void *base = (char *)a_ptr + La.offset(i, j) * 2;
+            cuuint64_t dims[4] = {(cuuint64_t)cpad, (cuuint64_t)wp, (cuuint64_t)hp, (cuuint64_t)N};
+            cuuint64_t strides[3] = {(cuuint64_t)cpad * 2, (cuuint64_t)wp * cpad * 2, (cuuint64_t)hp * wp * cpad * 2};
+            cuuint32_t box[4] = {(cuuint32_t)cpadc, (cuuint32_t)(ts.BW * s), (cuuint32_t)(ts.BH * s), (cuuint32_t)ts.BNn};
+            cuuint32_t es[4] = {1, (cuuint32_t)s, (cuuint32_t)s, 1};
+            CUresult r = encode(&P.mapA[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides, box, es,
+                                CU_TENSOR_MAP_INTERLEAVE_NONE, swz_for(row_bytes), CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+            if (r != CUDA_SUCCESS) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(A) failed");
+        }
+        P.tile_prefix[P.npatch] = tiles;
+        {
+            const int K = kh * kw * cpad;
+            cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)w_rows};
+            cuuint64_t strides[1] = {(cuuint64_t)K * 2};
+            cuuint32_t box[2] = {64, (cuuint32_t)BN};
+            cuuint32_t es[2] = {1, 1};
+            CUresult r = encode(&P.mapB, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(w_ptr), dims, strides, box,
+                                es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                                CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+            if (r != CUDA_SUCCESS) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(B) failed");
+        }
+        if (tiles == 0) continue;
+        const size_t smem = 1024 + (size_t)P.stages * stage_bytes + 256;
+        if (!attr_set) {
+            cudaFuncSetAttribute(conv_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+            attr_set = true;
+        }
+        const int grid = std::min(tiles, num_sms());
+        conv_tc_kernel<<<grid, 192, smem, st>>>(P);
+        count_launch();
+        {
+            cudaError_t e = cudaGetLastError();
+            if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("conv_tc_kernel: ") + cudaGetErrorString(e));
+        }
+    }
+    return SPLITCNN_OK;
+}
+
+}  // namespace
+
+bool conv_tc_supported(int mode, splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g) {
+    if (dt != SPLITCNN_BF16) return false;
+    if (g.L.sh != g.L.sw) return false;
+    if (Li.npatch() > 1024) return false;
+    if (mode == 0) {
+        if (!a_channels_ok(Li.Cpad)) return false;
+        if (g.L.sh > 2) return false;
+        return true;
+    }
+    if (mode == 1) {
+        if (g.L.sh != 1) return false;  // stride-2 dgrad: CUDA-core path (phase decomposition is future work)
+        if (!a_channels_ok(Lo.Cpad)) return false;
+        return true;
+    }
+    if (mode == 2) return wgrad_tc_ok(Li, Lo, g);
+    return false;
+}
+
+size_t conv_tc_ws_bytes(int mode, const Level &Li, const Level &Lo, const LayerGeom &g) {
+    if (mode == 2) return wgrad_tc_ws_bytes(Li, Lo, g);
+    if (mode == 1) return (size_t)g.L.cin * g.L.kh * g.L.kw * Lo.Cpad * 2 + 256;
+    return 0;
+}
+
+splitcnn_status_t launch_conv_fwd_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *w,
+                                     const float *bias, void *y, int relu, int p0, int p1, cudaStream_t st) {
+    return launch_tc(0, Li, Lo, g, x, w, g.L.cout, bias, y, nullptr, relu, p0, p1, st);
+}
+
+splitcnn_status_t launch_conv_dgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy, const void *w,
+                                       void *dx, const void *relu_src, void *ws, int p0, int p1, cudaStream_t st) {
+    const int64_t n = (int64_t)g.L.cin * g.L.kh * g.L.kw * Lo.Cpad;
+    flip_weights_kernel<<<(unsigned)std::min<int64_t>((n + 255) / 256, 2048), 256, 0, st>>>(
+        (const __nv_bfloat16 *)w, (__nv_bfloat16 *)ws, g.L.cout, Li.Cpad, g.L.cin, g.L.kh, g.L.kw, Lo.Cpad);
+    count_launch();
+    return launch_tc(1, Lo, Li, g, dy, ws, g.L.cin, nullptr, dx, relu_src, 0, p0, p1, st);
+}
+
+// ============================================================ weight gradient (tcgen05, MN-major)
+// dW[co][r][c][ci] = sum over pixels of dY[pix][co] * X~[pix shifted by (r, c)][ci]
+// GEMM per (co block of 128, tap, ci block): M = co, N = ci, K = pixels.  Both operands arrive from
+// TMA boxes whose rows are PIXELS and whose 128-byte rows hold 64 channels, i.e. MN-major SW128
+// tiles (an 8-pixel x 128 B atom; the next 64-channel block at LBO = 8 KB, the next 8 pixels at
+// SBO = 1 KB).  Split-K over pixel boxes of all patches in range; fp32 partial tiles go to the
+// workspace and a fixed-order reduction sums them (deterministic).
+constexpr int WG_ROWS = 64;  // pixels per K stage (4 MMAs of K = 16)
+
+struct TcWgradParams {
+    CUtensorMap mapDY[TC_MAXP];
+    CUtensorMap mapX[TC_MAXP];
+    int box_prefix[TC_MAXP + 1];
+    int pt[TC_MAXP], pl[TC_MAXP];
+    int nhb[TC_MAXP], nwb[TC_MAXP];
+    int npatch;
+    int BW, BH, BNn, rows_box;
+    int kh, kw, s;
+    int nco_blk, nci_blk, ntiles;   // tiles = nco_blk * taps * nci_blk
+    int BNc;                        // ci per tile (64..256)
+    int boxes_per_split, nsplit;
+    int Cout, Cpi;
+    int stages;
+    uint32_t tmem_cols;
+    float *part;                    // [nsplit][Cout][kh][kw][Cpi]
+};
+
+__global__ void __launch_bounds__(192, 1) wgrad_tc_kernel(const __grid_constant__ TcWgradParams p) {
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+    const int S = p.stages;
+    const uint32_t a_stage = 2u * WG_ROWS * 128u;                 // 128 co = two 64-channel blocks
+    const uint32_t b_stage = (uint32_t)(p.BNc / 64) * WG_ROWS * 128u;
+    uint8_t *sA = smem;
+    uint8_t *sB = smem + (size_t)S * a_stage;
+    uint64_t *full = (uint64_t *)(sB + (size_t)S * b_stage);
+    uint64_t *empty = full + S;
+    uint64_t *tfull = empty + S;
+    uint32_t *tmem_slot = (uint32_t *)(tfull + 1);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+    // rows >= rows_box of every stage are never written by TMA: zero them once so they add 0
+    {
+        uint4 *z = (uint4 *)smem;
+        const int n16 = (int)(((size_t)S * (a_stage + b_stage)) / 16);
+        for (int i = threadIdx.x; i < n16; i += blockDim.x) z[i] = make_uint4(0, 0, 0, 0);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    }
+    if (warp == 0 && lane == 0) {
+        for (int s = 0; s < S; ++s) {
+            tc::mbar_init(&full[s], 1);
+            tc::mbar_init(&empty[s], 1);
+        }
+        tc::mbar_init(&tfull[0], 1);
+        tc::fence_barrier_init();
+    }
+    if (warp == 1) tc::tmem_alloc_dyn(tmem_slot, p.tmem_cols);
+    tc::tc_fence_before();
+    __syncthreads();
+    tc::tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    // work item: z-major so CTAs running together share the same pixels (L2 reuse)
+    const int tile = blockIdx.x % p.ntiles, z = blockIdx.x / p.ntiles;
+    const int KT = p.kh * p.kw;
+    const int ci_blk = tile % p.nci_blk;
+    const int tap = (tile / p.nci_blk) % KT;
+    const int co_blk = tile / (p.nci_blk * KT);
+    const int r = tap / p.kw, c = tap - r * p.kw;
+    const int total_boxes = p.box_prefix[p.npatch];
+    const int b0 = z * p.boxes_per_split, b1 = min(total_boxes, b0 + p.boxes_per_split);
+
+    if (warp == 0) {
+        if (lane == 0) {
+            int stage = 0;
+            uint32_t ph = 0;
+            int ql = 0;
+            const uint32_t tx = (2u + (uint32_t)(p.BNc / 64)) * (uint32_t)p.rows_box * 128u;
+            for (int b = b0; b < b1; ++b) {
+                while (b >= p.box_prefix[ql + 1]) ++ql;
+                int idx = b - p.box_prefix[ql];
+                const int wb = idx % p.nwb[ql];
+                idx /= p.nwb[ql];
+                const int hb = idx % p.nhb[ql], nb = idx / p.nhb[ql];
+                const int ow0 = wb * p.BW, oh0 = hb * p.BH, n0 = nb * p.BNn;
+                tc::mbar_wait(&empty[stage], ph ^ 1);
+                tc::mbar_arrive_expect_tx(&full[stage], tx);
+                uint8_t *a = sA + (size_t)stage * a_stage;
+                uint8_t *bb = sB + (size_t)stage * b_stage;
+                for (int h = 0; h < 2; ++h)
+                    tc::tma_load_4d(a + h * WG_ROWS * 128, &p.mapDY[ql], &full[stage], co_blk * 128 + h * 64, ow0, oh0, n0);
+                for (int h = 0; h < p.BNc / 64; ++h)
+                    tc::tma_load_4d(bb + h * WG_ROWS * 128, &p.mapX[ql], &full[stage], ci_blk * p.BNc + h * 64,
+                                    ow0 * p.s - p.pl[ql] + c, oh0 * p.s - p.pt[ql] + r, n0);
+                if (++stage == S) { stage = 0; ph ^= 1; }
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            const uint32_t idesc = tc::idesc_bf16(128, p.BNc, 1, 1);
+            int stage = 0;
+            uint32_t ph = 0;
+            for (int b = b0; b < b1; ++b) {
+                tc::mbar_wait(&full[stage], ph);
+                tc::tc_fence_after();
+                const uint32_t a_base = tc::smem_u32(sA + (size_t)stage * a_stage);
+                const uint32_t b_base = tc::smem_u32(sB + (size_t)stage * b_stage);
+#pragma unroll
+                for (int j = 0; j < WG_ROWS / 16; ++j) {
+                    const uint64_t adesc = tc::smem_desc(a_base + 2048u * j, WG_ROWS * 128, 1024, 2);
+                    const uint64_t bdesc = tc::smem_desc(b_base + 2048u * j, WG_ROWS * 128, 1024, 2);
+                    tc::mma_bf16(tmem_base, adesc, bdesc, idesc, (b != b0 || j) ? 1u : 0u);
+                }
+                tc::mma_commit(&empty[stage]);
+                if (++stage == S) { stage = 0; ph ^= 1; }
+            }
+            tc::mma_commit(&tfull[0]);
+        }
+    } else {
+        const int quad = warp & 3;
+        const int co = co_blk * 128 + quad * 32 + lane;
+        const bool any = b1 > b0;
+        if (any) {
+            tc::mbar_wait(&tfull[0], 0);
+            tc::tc_fence_after();
+        }
+        const uint32_t tacc = tmem_base + ((uint32_t)(quad * 32) << 16);
+        float *dst = p.part + ((((int64_t)z * p.Cout + co) * KT + tap) * p.Cpi) + ci_blk * p.BNc;
+        for (int cc = 0; cc < p.BNc; cc += 16) {
+            float v[16];
+            if (any) {
+                tc::tmem_ld16(tacc + cc, v);
+            } else {
+#pragma unroll
+                for (int e = 0; e < 16; ++e) v[e] = 0.f;
+            }
+            if (co < p.Cout && ci_blk * p.BNc + cc < p.Cpi) {
+                float4 *d4 = reinterpret_cast<float4 *>(dst + cc);
+#pragma unroll
+                for (int e = 0; e < 4; ++e) d4[e] = make_float4(v[4 * e], v[4 * e + 1], v[4 * e + 2], v[4 * e + 3]);
+            }
+        }
+    }
+    tc::tc_fence_before();
+    __syncthreads();
+    tc::tc_fence_after();
+    if (warp == 1) tc::tmem_dealloc(tmem_base, p.tmem_cols);
+}
+
+namespace {
+
+struct WgradCfg {
+    TileShape ts;
+    int BNc, nco_blk, nci_blk, ntiles, total_boxes, nsplit, boxes_per_split;
+};
+
+WgradCfg wgrad_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, int p0, int p1) {
+    WgradCfg c{};
+    std::vector<std::pair<int, int>> ext;
+    for (int q = p0; q < p1; ++q) ext.push_back({Lo.ph(q / Lo.nw()), Lo.pw(q % Lo.nw())});
+    // pixel box of <= 64 rows (WG_ROWS) minimising the box count
+    TileShape best{1, 1, 1};
+    long best_n = -1;
+    const int N = Lo.N, s = g.L.sh;
+    int maxh = 1, maxw = 1;
+    for (auto &e : ext) { maxh = std::max(maxh, e.first); maxw = std::max(maxw, e.second); }
+    for (int bw = 1; bw <= std::min(std::min(maxw, WG_ROWS), 256 / s); ++bw)
+        for (int bh = 1; bh <= std::min(maxh, 256 / s) && bw * bh <= WG_ROWS; ++bh) {
+            const int bn = std::min(WG_ROWS / (bw * bh), N);
+            long n = 0;
+            for (auto &e : ext) n += (long)((N + bn - 1) / bn) * ((e.first + bh - 1) / bh) * ((e.second + bw - 1) / bw);
+            if (best_n < 0 || n < best_n || (n == best_n && bw > best.BW)) { best_n = n; best = {bw, bh, bn}; }
+        }
+    c.ts = best;
+    c.total_boxes = (int)best_n;
+    c.BNc = Li.Cpad % 256 == 0 ? 256 : (Li.Cpad % 128 == 0 ? 128 : 64);
+    c.nco_blk = (g.L.cout + 127) / 128;
+    c.nci_blk = Li.Cpad / c.BNc;
+    c.ntiles = c.nco_blk * g.L.kh * g.L.kw * c.nci_blk;
+    int Z = std::max(1, (2 * num_sms() + c.ntiles - 1) / c.ntiles);
+    Z = std::min(Z, std::max(1, c.total_boxes / 4));  // >= 4 boxes per split
+    Z = std::min(Z, 64);
+    c.boxes_per_split = (c.total_boxes + Z - 1) / Z;
+    c.nsplit = (c.total_boxes + c.boxes_per_split - 1) / c.boxes_per_split;
+    return c;
+}
+
+}  // namespace
+
+static bool wgrad_tc_ok(const Level &Li, const Level &Lo, const LayerGeom &g) {
+    return Li.Cpad % 64 == 0 && Lo.Cpad % 64 == 0 && g.L.sh == g.L.sw && g.L.sh <= 2;
+}
+
+size_t wgrad_tc_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g) {
+    // sized for the full patch range in groups of TC_MAXP patches (the largest group decides)
+    size_t best = 0;
+    const int np = Lo.npatch();
+    for (int g0 = 0; g0 < np; g0 += TC_MAXP) {
+        WgradCfg c = wgrad_cfg(Li, Lo, g, g0, std::min(np, g0 + TC_MAXP));
+        best = std::max(best, (size_t)c.nsplit * g.L.cout * g.L.kh * g.L.kw * Li.Cpad * sizeof(float));
+    }
+    // plus the db partials of the CUDA-core helper
+    return best + 64 * (size_t)g.L.cout * sizeof(float) * 64 + 256;
+}
+
+void launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, float *part, int cout, int p0, int p1,
+                        int cpp, cudaStream_t st);
+void launch_reduce(const float *part, int Z, int64_t n, float *out, float beta, cudaStream_t st);
+
+splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *dy,
+                                       float *dw, float *db, float beta, void *ws, int p0, int p1, cudaStream_t st) {
+    auto encode = get_encode();
+    if (!encode) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+    const int KT = g.L.kh * g.L.kw, s = g.L.sh;
+    const int64_t nW = (int64_t)g.L.cout * KT * Li.Cpad;
+    float *part = (float *)ws;
+    static bool attr_set = false;
+    bool first = true;
+    for (int g0 = p0; g0 < p1; g0 += TC_MAXP) {
+        const int g1 = std::min(p1, g0 + TC_MAXP);
+        WgradCfg c = wgrad_cfg(Li, Lo, g, g0, g1);
+        static thread_local TcWgradParams P;
+        std::memset(&P, 0, sizeof(P));
+        P.npatch = g1 - g0;
+        P.BW = c.ts.BW; P.BH = c.ts.BH; P.BNn = c.ts.BNn; P.rows_box = c.ts.BW * c.ts.BH * c.ts.BNn;
+        P.kh = g.L.kh; P.kw = g.L.kw; P.s = s;
+        P.nco_blk = c.nco_blk; P.nci_blk = c.nci_blk; P.ntiles = c.ntiles; P.BNc = c.BNc;
+        P.boxes_per_split = c.boxes_per_split; P.nsplit = c.nsplit;
+        P.Cout = g.L.cout; P.Cpi = Li.Cpad;
+        const uint32_t stage_bytes = 2u * WG_ROWS * 128u + (uint32_t)(c.BNc / 64) * WG_ROWS * 128u;
+        P.stages = std::min<int>(8, (int)((200u * 1024u) / stage_bytes));
+        uint32_t cols = 32;
+        while (cols < (uint32_t)c.BNc) cols <<= 1;
+        P.tmem_cols = cols;
+        P.part = part;
+        int boxes = 0;
+        for (int q = g0; q < g1; ++q) {
+            const int ql = q - g0, i = q / Lo.nw(), j = q % Lo.nw();
+            const int ho = Lo.ph(i), wo = Lo.pw(j), hp = Li.ph(i), wp = Li.pw(j);
+            P.pt[ql] = g.pad_h[2 * i];
+            P.pl[ql] = g.pad_w[2 * j];
+            P.nhb[ql] = (ho + c.ts.BH - 1) / c.ts.BH;
+            P.nwb[ql] = (wo + c.ts.BW - 1) / c.ts.BW;
+            P.box_prefix[ql] = boxes;
+            boxes += ((Lo.N + c.ts.BNn - 1) / c.ts.BNn) * P.nhb[ql] * P.nwb[ql];
+            {
+                const int C = Lo.Cpad;
+                void *base = (char *)dy + Lo.offset(i, j) * 2;
+                cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)wo, (cuuint64_t)ho, (cuuint64_t)Lo.N};
+                cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)wo * C * 2, (cuuint64_t)ho * wo * C * 2};
+                cuuint32_t box[4] = {64, (cuuint32_t)c.ts.BW, (cuuint32_t)c.ts.BH, (cuuint32_t)c.ts.BNn};
+                cuuint32_t es[4] = {1, 1, 1, 1};
+                if (encode(&P.mapDY[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides, box, es,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+                    return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(dY) failed");
+            }
+            {
+                const int C = Li.Cpad;
+                void *base = (char *)x + Li.offset(i, j) * 2;
+                cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)wp, (cuuint64_t)hp, (cuuint64_t)Li.N};
+                cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)wp * C * 2, (cuuint64_t)hp * wp * C * 2};
+                cuuint32_t box[4] = {64, (cuuint32_t)(c.ts.BW * s), (cuuint32_t)(c.ts.BH * s), (cuuint32_t)c.ts.BNn};
+                cuuint32_t es[4] = {1, (cuuint32_t)s, (cuuint32_t)s, 1};
+                if (encode(&P.mapX[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides, box, es,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+                    return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(X) failed");
+            }
+        }
+        P.box_prefix[P.npatch] = boxes;
+        const size_t smem = 1024 + (size_t)P.stages * stage_bytes + 256;
+        if (!attr_set) {
+            cudaFuncSetAttribute(wgrad_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+            attr_set = true;
+        }
+        wgrad_tc_kernel<<<c.ntiles * c.nsplit, 192, smem, st>>>(P);
+        count_launch();
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("wgrad_tc_kernel: ") + cudaGetErrorString(e));
+        // fixed-order sum of the split partials (and the previous groups' result) into dW
+        launch_reduce(part, c.nsplit, nW, dw, first ? beta : 1.f, st);
+        first = false;
+    }
+    if (db) {
+        const int np = p1 - p0;
+        const int cpp = std::max(1, std::min(64, (2 * num_sms() + np - 1) / np));
+        float *part_db = part + 0;  // the dW partials have been consumed by the reduction (stream order)
+        launch_db_partials(SPLITCNN_BF16, Lo, dy, part_db, g.L.cout, p0, p1, cpp, st);
+        launch_reduce(part_db, np * cpp, g.L.cout, db, beta, st);
+    }
+    return SPLITCNN_OK;
+}
+
 }  // namespace splitcnn

@@ -108,9 +108,9 @@ void launch_split_t(const Level &L, const void *x, int layout, void *P, int p0, 
     dim3 grid(grid_x_for(max_patch_units(L, p0, p1, L.Cpad / 8)), p1 - p0);
     LevelDesc d = make_level_desc(L);
     if (layout == SPLITCNN_NCHW)
-        split_kernel<T, true><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0);
+        { split_kernel<T, true><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0); count_launch(); }
     else
-        split_kernel<T, false><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0);
+        { split_kernel<T, false><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0); count_launch(); }
 }
 
 template <typename T>
@@ -118,9 +118,9 @@ void launch_merge_t(const Level &L, const void *P, void *y, int layout, int p0, 
     dim3 grid(grid_x_for(max_patch_units(L, p0, p1, L.Cpad / 8)), p1 - p0);
     LevelDesc d = make_level_desc(L);
     if (layout == SPLITCNN_NCHW)
-        merge_kernel<T, true><<<grid, 256, 0, st>>>(d, (const T *)P, (T *)y, p0);
+        { merge_kernel<T, true><<<grid, 256, 0, st>>>(d, (const T *)P, (T *)y, p0); count_launch(); }
     else
-        merge_kernel<T, false><<<grid, 256, 0, st>>>(d, (const T *)P, (T *)y, p0);
+        { merge_kernel<T, false><<<grid, 256, 0, st>>>(d, (const T *)P, (T *)y, p0); count_launch(); }
 }
 
 void launch_split(splitcnn_dtype_t dt, const Level &L, const void *x, int layout, void *P, int p0, int p1, cudaStream_t st) {
@@ -229,15 +229,15 @@ template <typename T>
 void launch_pool_fwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, void *y, uint8_t *a,
                        int relu_bit, int p0, int p1, cudaStream_t st) {
     dim3 grid(grid_x_for(max_patch_units(Lo, p0, p1, Lo.Cpad / 8)), p1 - p0);
-    pool_fwd_kernel<T><<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
-                                             (const T *)x, (T *)y, a, p0, relu_bit);
+    { pool_fwd_kernel<T><<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
+                                             (const T *)x, (T *)y, a, p0, relu_bit); count_launch(); }
 }
 template <typename T>
 void launch_pool_bwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy, const uint8_t *a, void *dx,
                        int relu_bit, int p0, int p1, cudaStream_t st) {
     dim3 grid(grid_x_for(max_patch_units(Li, p0, p1, Li.Cpad / 8)), p1 - p0);
-    pool_bwd_kernel<T><<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
-                                             (const T *)dy, a, (T *)dx, p0, relu_bit);
+    { pool_bwd_kernel<T><<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
+                                             (const T *)dy, a, (T *)dx, p0, relu_bit); count_launch(); }
 }
 
 void launch_pool_fwd(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, void *y,

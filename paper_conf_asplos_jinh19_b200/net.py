@@ -39,6 +39,7 @@ class SplitNet:
         self.dtype, self.tdtype, self.device = dtype, TORCH_DTYPE[dtype], torch.device(device)
         self.flags_extra = sc.FLAG_FORCE_SIMT if force_simt else 0
         self.step_index = 0
+        self.timers = None       # list -> every library call is bracketed by CUDA events (bench.py)
         self.region = self._make_region_plan(0)
         self.patch_range = patch_range or (0, self.region.npatch)
         L = self.region.levels[-1]
@@ -123,6 +124,27 @@ class SplitNet:
                     self.params[(key, m)][0].copy_(pack_weight(W, plan.levels[m]["Cpad"], self.tdtype))
                     self.params[(key, m)][1].copy_(torch.as_tensor(b, dtype=torch.float32))
 
+    # ------------------------------------------------------------------ instrumentation
+    def _call(self, kind: str, work: float, fn, *args):
+        """Run one library call; when self.timers is a list, bracket it with CUDA events on the
+        launching stream and record (kind, start, end, algorithmic work)."""
+        if self.timers is None:
+            return fn(*args)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        fn(*args)
+        e1.record()
+        self.timers.append((kind, e0, e1, work))
+
+    def _conv_work(self, plan, m, l):
+        lo = plan.levels[m + 1]
+        return 2.0 * lo["N"] * l["cout"] * lo["H"] * lo["W"] * l["cin"] * l["kh"] * l["kw"]
+
+    def _bytes(self, plan, m):
+        es = 2 if self.dtype == sc.BF16 else 4
+        li, lo = plan.levels[m], plan.levels[m + 1]
+        return es * li["N"] * li["C"] * li["H"] * li["W"], es * lo["N"] * lo["C"] * lo["H"] * lo["W"]
+
     # ------------------------------------------------------------------ masks
     def _masked(self, key: str, m: int) -> bool:
         """Level m is the output of a conv with fused ReLU -> its gradient producer applies the mask."""
@@ -137,10 +159,13 @@ class SplitNet:
         """x: full NCHW tensor (dtype) on the device.  Returns the output level buffer."""
         p0, p1 = self.patch_range
         R, dt, fl = self.region.handle, self.dtype, self.flags_extra
-        sc.splitcnn_split(R, 0, dt, x, sc.NCHW, self.act_r[0], p0, p1, stream)
+        b_in = 2 * self._bytes(self.region, 0)[0]
+        self._call("split", b_in, sc.splitcnn_split, R, 0, dt, x, sc.NCHW, self.act_r[0], p0, p1, stream)
         self._run_fwd("r", self.region, self.region_layers, self.act_r, p0, p1, stream)
         if self.tail:
-            sc.splitcnn_merge(R, self.region.nlayers, dt, self.act_r[-1], self.act_t[0], sc.NHWC, p0, p1, stream)
+            b_j = 2 * self._bytes(self.region, self.region.nlayers - 1)[1]
+            self._call("merge", b_j, sc.splitcnn_merge, R, self.region.nlayers, dt, self.act_r[-1], self.act_t[0],
+                       sc.NHWC, p0, p1, stream)
             self._run_fwd("t", self.tail, self.tail_layers, self.act_t, 0, 1, stream)
             return self.act_t[-1]
         return self.act_r[-1]
@@ -150,11 +175,14 @@ class SplitNet:
             if l["op"] == "conv":
                 W, b = self.params[(key, m)]
                 flags = (sc.FLAG_RELU if l.get("relu", True) else 0) | self.flags_extra
-                sc.splitcnn_conv_fwd(plan.handle, m, self.dtype, acts[m], W, b, acts[m + 1], flags, p0, p1, stream)
+                self._call("conv_fwd", self._conv_work(plan, m, l), sc.splitcnn_conv_fwd, plan.handle, m, self.dtype,
+                           acts[m], W, b, acts[m + 1], flags, p0, p1, stream)
             else:
                 flags = sc.FLAG_POOL_RELU_MASK if self._masked(key, m) else 0
-                sc.splitcnn_pool_fwd(plan.handle, m, self.dtype, acts[m], acts[m + 1], self.argmax[(key, m)], flags,
-                                     p0, p1, stream)
+                bi, bo = self._bytes(plan, m)
+                work = bi + bo + bo // (2 if self.dtype == sc.BF16 else 4)
+                self._call("pool_fwd", work, sc.splitcnn_pool_fwd, plan.handle, m, self.dtype, acts[m], acts[m + 1],
+                           self.argmax[(key, m)], flags, p0, p1, stream)
 
     def backward(self, dy: torch.Tensor, stream=None, need_input_grad: bool = False):
         """dy: gradient w.r.t. the output level buffer (same layout).  Fills self.grads."""
@@ -163,7 +191,9 @@ class SplitNet:
         if self.tail:
             g = self._run_bwd("t", self.tail, self.tail_layers, self.act_t, g, 0, 1, stream, True)
             gi = self.grad[0] if g is not self.grad[0] else self.grad[1]
-            sc.splitcnn_split(self.region.handle, self.region.nlayers, self.dtype, g, sc.NHWC, gi, p0, p1, stream)
+            b_j = 2 * self._bytes(self.region, self.region.nlayers - 1)[1]
+            self._call("split", b_j, sc.splitcnn_split, self.region.handle, self.region.nlayers, self.dtype, g,
+                       sc.NHWC, gi, p0, p1, stream)
             g = gi
         return self._run_bwd("r", self.region, self.region_layers, self.act_r, g, p0, p1, stream, need_input_grad)
 
@@ -175,15 +205,19 @@ class SplitNet:
             if l["op"] == "conv":
                 W, _ = self.params[(key, m)]
                 dW, db = self.grads[(key, m)]
+                work = self._conv_work(plan, m, l)
                 if not last:
                     relu_src = acts[m] if self._masked(key, m) else None
-                    sc.splitcnn_conv_bwd_data(plan.handle, m, self.dtype, g, W, out, relu_src, self.ws, self.ws_bytes,
-                                              self.flags_extra, p0, p1, stream)
-                sc.splitcnn_conv_bwd_filter(plan.handle, m, self.dtype, acts[m], g, dW, db, 0.0, self.ws,
-                                            self.ws_bytes, self.flags_extra, p0, p1, stream)
+                    self._call("conv_dgrad", work, sc.splitcnn_conv_bwd_data, plan.handle, m, self.dtype, g, W, out,
+                               relu_src, self.ws, self.ws_bytes, self.flags_extra, p0, p1, stream)
+                self._call("conv_wgrad", work, sc.splitcnn_conv_bwd_filter, plan.handle, m, self.dtype, acts[m], g, dW,
+                           db, 0.0, self.ws, self.ws_bytes, self.flags_extra, p0, p1, stream)
             else:
                 flags = sc.FLAG_POOL_RELU_MASK if self._masked(key, m) else 0
-                sc.splitcnn_pool_bwd(plan.handle, m, self.dtype, g, self.argmax[(key, m)], out, flags, p0, p1, stream)
+                bi, bo = self._bytes(plan, m)
+                work = bi + bo + bo // (2 if self.dtype == sc.BF16 else 4)
+                self._call("pool_bwd", work, sc.splitcnn_pool_bwd, plan.handle, m, self.dtype, g,
+                           self.argmax[(key, m)], out, flags, p0, p1, stream)
             if not last:
                 g = out
         return g

@@ -29,7 +29,7 @@ FLAG_FORCE_SIMT = 0x100
 MAX_SPLITS = 32
 
 EXPORTED = [
-    "splitcnn_last_error", "splitcnn_status_string", "splitcnn_version",
+    "splitcnn_last_error", "splitcnn_status_string", "splitcnn_version", "splitcnn_kernel_launches",
     "splitcnn_boundaries_even", "splitcnn_boundaries_random",
     "splitcnn_plan_create", "splitcnn_plan_destroy", "splitcnn_plan_num_layers", "splitcnn_plan_level",
     "splitcnn_plan_layer", "splitcnn_workspace_size",
@@ -72,6 +72,7 @@ def _sig(name, args, res=ctypes.c_int):
 _sig("splitcnn_last_error", [], ctypes.c_char_p)
 _sig("splitcnn_status_string", [ctypes.c_int], ctypes.c_char_p)
 _sig("splitcnn_version", [], ctypes.c_char_p)
+_sig("splitcnn_kernel_launches", [ctypes.POINTER(ctypes.c_uint64)])
 _sig("splitcnn_boundaries_even", [_i32, _i32, _pi32])
 _sig("splitcnn_boundaries_random", [_i32, _i32, _i32, _i32, _f64, _u64, _u64, _pi32, _pi32])
 _sig("splitcnn_plan_create", [ctypes.POINTER(Layer), _i32, _i32, _i32, _i32, _i32, _pi32, _i32, _pi32, _i32,
@@ -130,6 +131,12 @@ def _arr(vals, ctype=ctypes.c_int32):
 # ---------------------------------------------------------------- host calls
 def splitcnn_version() -> str:
     return _lib.splitcnn_version().decode()
+
+
+def splitcnn_kernel_launches() -> int:
+    n = ctypes.c_uint64()
+    _check(_lib.splitcnn_kernel_launches(ctypes.byref(n)))
+    return n.value
 
 
 def splitcnn_boundaries_even(L: int, n: int) -> list[int]:

@@ -66,6 +66,7 @@ def _run(sc, cfg_name, N, dtype, H=None, step=0, force_simt=False):
     # point, and fp32 vs fp64 accumulation may round a value to the neighbouring bf16 (R13, R9)
     flips = total = 0
     for (key, m), (xin, aref) in pools.items():
+        scale = max(float(np.abs(blk).max()) for row in xin for blk in row)
         plan = net.region if key == "r" else net.tail
         lv = plan.levels[m + 1]
         agot = unpack_level(net.argmax[(key, m)].cpu().numpy().astype(np.float64), lv)
@@ -83,7 +84,11 @@ def _run(sc, cfg_name, N, dtype, H=None, step=0, force_simt=False):
                         w = ow * lp["sw"] - lp["pads_w"][j][0] + a % lp["kw"]
                         return xin[i][j][n, ch, h, w]
                     v1, v2 = val(a_g[n, ch, oh, ow]), val(a_r[n, ch, oh, ow])
-                    assert bf and abs(v1 - v2) <= 2 ** -6 * max(abs(v1), abs(v2)), (key, m, v1, v2)
+                    # near-tie: within 2 bf16 ulps relative, or normwise (R13) within 2^-8 of the tensor's
+                    # max (values next to the ReLU kink round to 0 on one side and to a tiny positive
+                    # value on the other)
+                    tie = abs(v1 - v2) <= 2 ** -6 * max(abs(v1), abs(v2)) + 2 ** -8 * scale
+                    assert bf and tie, (key, m, v1, v2, scale)
     errs["argmax_flip_frac"] = flips / max(total, 1)
     return errs
 

@@ -153,12 +153,16 @@ def run_ours(args):
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         ms = tt.item()
     # per-kind device time from the events recorded around every library call
-    kinds = {}
-    for kind, e0, e1, work in net.timers:
+    kinds, per_layer = {}, {}
+    for kind, e0, e1, work, label in net.timers:
+        dt_ms = e0.elapsed_time(e1)
         k = kinds.setdefault(kind, [0.0, 0.0, 0])
-        k[0] += e0.elapsed_time(e1)
+        k[0] += dt_ms
         k[1] += work
         k[2] += 1
+        pl = per_layer.setdefault(f"{label}:{kind}", [0.0, 0.0])
+        pl[0] += dt_ms
+        pl[1] += work
     net.timers = None
     ms_step = ms / args.steps
     global_batch = c["N"]
@@ -229,6 +233,10 @@ def run_ours(args):
         "per_kind_ms_per_step": {k: round(v[0] / args.steps, 4) for k, v in kinds.items()},
         "clocks": clk,
     }
+    if args.per_layer:
+        line["per_layer"] = {k: {"ms": round(v[0] / args.steps, 4),
+                                 "tflops" if ":conv" in k else "gbs": round(v[1] / (v[0] / 1e3) / (1e12 if ":conv" in k else 1e9), 1)}
+                             for k, v in per_layer.items()}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(args.config, budget_tiles=args.cpu_tiles)
     if rank == 0:
@@ -337,6 +345,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--cpu-tiles", type=int, default=12)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--per-layer", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

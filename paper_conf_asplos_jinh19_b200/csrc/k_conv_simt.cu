@@ -201,23 +201,6 @@ __global__ void __launch_bounds__(NT) conv_simt_kernel(SimtArgs a) {
     }
 }
 
-// db partial per chunk: part_db[z][co] = sum over the chunk's pixels of dY[pixel][co]
-template <typename T>
-__global__ void __launch_bounds__(256) db_partial_kernel(LevelDesc Lo, const T *__restrict__ dY, float *__restrict__ part,
-                                                         int Cout, int p0, int cpp) {
-    const int zq = blockIdx.x;
-    const int q = p0 + zq / cpp;
-    const PatchGeo go = patch_geo(Lo, q);
-    const int P = Lo.N * go.hp * go.wp;
-    const int chunk = (P + cpp - 1) / cpp;
-    const int kb = (zq % cpp) * chunk, ke = min(P, kb + chunk);
-    for (int co = threadIdx.x; co < Cout; co += blockDim.x) {
-        float s = 0.f;
-        for (int k = kb; k < ke; ++k) s += to_f(dY[go.off + (int64_t)k * Lo.Cpad + co]);
-        part[(int64_t)zq * Cout + co] = s;
-    }
-}
-
 // dW[i] = beta * dW[i] + sum_z part[z][i]   (z ascending: fixed order)
 __global__ void __launch_bounds__(256) reduce_partials_kernel(const float *__restrict__ part, int Z, int64_t n,
                                                               float *__restrict__ out, float beta) {
@@ -228,14 +211,58 @@ __global__ void __launch_bounds__(256) reduce_partials_kernel(const float *__res
     }
 }
 
-void launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, float *part, int cout, int p0, int p1,
-                        int cpp, cudaStream_t st) {
-    const int Z = (p1 - p0) * cpp;
+// Column sums of the patch-buffer range [p0, p1) viewed as a [P pixels][Cpad] matrix (the patches of
+// a range are contiguous): block b sums rows [b*R, (b+1)*R) with 16-byte loads, reduces its pixel
+// lanes in shared memory in a fixed order and writes part[b][Cout].  Deterministic.
+template <typename T>
+__global__ void __launch_bounds__(256) colsum_kernel(const T *__restrict__ base, int64_t P, int Cpad, int Cout,
+                                                     int64_t R, float *__restrict__ part) {
+    __shared__ float red[256][8];
+    const int G = Cpad / 8;
+    const int lanes = 256 / G;
+    const int cg = threadIdx.x % G, pl = threadIdx.x / G;
+    float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    const int64_t r0 = blockIdx.x * R, r1 = min(P, r0 + R);
+    if (pl < lanes) {
+        for (int64_t r = r0 + pl; r < r1; r += lanes) {
+            float v[8];
+            load8(base + r * Cpad + cg * 8, v);
+#pragma unroll
+            for (int e = 0; e < 8; ++e) acc[e] += v[e];
+        }
+    }
+#pragma unroll
+    for (int e = 0; e < 8; ++e) red[threadIdx.x][e] = acc[e];
+    __syncthreads();
+    if (threadIdx.x < G) {
+        float s8[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        for (int l = 0; l < lanes; ++l)
+#pragma unroll
+            for (int e = 0; e < 8; ++e) s8[e] += red[l * G + threadIdx.x][e];
+#pragma unroll
+        for (int e = 0; e < 8; ++e)
+            if (threadIdx.x * 8 + e < Cout) part[(int64_t)blockIdx.x * Cout + threadIdx.x * 8 + e] = s8[e];
+    }
+}
+
+// returns the number of partial rows written
+int launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, float *part, int cout, int p0, int p1,
+                       cudaStream_t st) {
+    auto off = [&](int q) -> int64_t {
+        if (q >= Lo.npatch()) return Lo.total();
+        return Lo.offset(q / Lo.nw(), q % Lo.nw());
+    };
+    const int64_t e0 = off(p0), e1 = off(p1);
+    const int64_t P = (e1 - e0) / Lo.Cpad;
+    const int Z = 4 * 148;
+    const int64_t R = (P + Z - 1) / Z;
+    const int Zr = (int)((P + R - 1) / R);
     if (dt == SPLITCNN_BF16)
-        db_partial_kernel<__nv_bfloat16><<<Z, 256, 0, st>>>(make_level_desc(Lo), (const __nv_bfloat16 *)dy, part, cout, p0, cpp);
+        colsum_kernel<__nv_bfloat16><<<Zr, 256, 0, st>>>((const __nv_bfloat16 *)dy + e0, P, Lo.Cpad, cout, R, part);
     else
-        db_partial_kernel<float><<<Z, 256, 0, st>>>(make_level_desc(Lo), (const float *)dy, part, cout, p0, cpp);
+        colsum_kernel<float><<<Zr, 256, 0, st>>>((const float *)dy + e0, P, Lo.Cpad, cout, R, part);
     count_launch();
+    return Zr;
 }
 
 void launch_reduce(const float *part, int Z, int64_t n, float *out, float beta, cudaStream_t st) {
@@ -290,7 +317,7 @@ size_t wgrad_simt_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g)
     const int cpp = wgrad_simt_chunks_per_patch(Li, Lo, g, np);
     const int64_t Z = (int64_t)np * cpp;
     const int64_t ncols = (int64_t)g.L.kh * g.L.kw * Li.Cpad;
-    return (size_t)(Z * g.L.cout * ncols + Z * g.L.cout) * sizeof(float);
+    return (size_t)(Z * g.L.cout * ncols + 4 * 148 * g.L.cout) * sizeof(float);
 }
 
 void launch_conv_wgrad_simt(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *x,
@@ -311,11 +338,8 @@ void launch_conv_wgrad_simt(splitcnn_dtype_t dt, const Level &Li, const Level &L
     const int64_t n = (int64_t)g.L.cout * ncols;
     { reduce_partials_kernel<<<(unsigned)std::min<int64_t>((n + 255) / 256, 4096), 256, 0, st>>>(part, Z, n, dw, beta); count_launch(); }
     if (db) {
-        if (dt == SPLITCNN_BF16)
-            { db_partial_kernel<__nv_bfloat16><<<Z, 256, 0, st>>>(make_level_desc(Lo), (const __nv_bfloat16 *)dy, part_db, g.L.cout, p0, cpp); count_launch(); }
-        else
-            { db_partial_kernel<float><<<Z, 256, 0, st>>>(make_level_desc(Lo), (const float *)dy, part_db, g.L.cout, p0, cpp); count_launch(); }
-        { reduce_partials_kernel<<<(g.L.cout + 255) / 256, 256, 0, st>>>(part_db, Z, g.L.cout, db, beta); count_launch(); }
+        const int Zd = launch_db_partials(dt, Lo, dy, part_db, g.L.cout, p0, p1, st);
+        { reduce_partials_kernel<<<(g.L.cout + 255) / 256, 256, 0, st>>>(part_db, Zd, g.L.cout, db, beta); count_launch(); }
     }
 }
 

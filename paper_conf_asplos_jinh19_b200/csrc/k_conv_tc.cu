@@ -50,6 +50,7 @@ struct TcConvParams {
     int tps;         // taps per K step (Cpad_A < 64)
     int ksteps;      // K steps per tile
     int kchan;       // Cpad of the A side (K = taps * kchan)
+    int a3d;         // 8-channel A: 3-D maps with pixels merged into 128-byte-wide rows (coordinate 8*w)
     int BN, Cout, Cpo;
     int stages;
     uint32_t tmem_cols;
@@ -127,7 +128,10 @@ __global__ void __launch_bounds__(192, 1) conv_tc_kernel(const __grid_constant__
                         for (int j = 0; j < p.tps; ++j) {
                             const int tap = min(ks * p.tps + j, KT - 1);  // past the last tap: weights are OOB zero
                             const int r = tap / p.kw, c = tap - r * p.kw;
-                            tc::tma_load_4d(a + j * p.a_chunk_bytes, &p.mapA[ql], &full[stage], 0, wbase + c, hbase + r, n0);
+                            if (p.a3d)
+                                tc::tma_load_3d(a + j * p.a_chunk_bytes, &p.mapA[ql], &full[stage], 8 * (wbase + c), hbase + r, n0);
+                            else
+                                tc::tma_load_4d(a + j * p.a_chunk_bytes, &p.mapA[ql], &full[stage], 0, wbase + c, hbase + r, n0);
                         }
                         tc::tma_load_2d(b, &p.mapB, &full[stage], ks * 64, co0);
                     } else {
@@ -295,12 +299,12 @@ struct TileShape {
 };
 
 // choose the pixel box (BW x BH x BNn <= 128 rows) minimising the number of tiles over the patches
-TileShape choose_tile(const std::vector<std::pair<int, int>> &ext, int N, int s) {
+TileShape choose_tile(const std::vector<std::pair<int, int>> &ext, int N, int s, int bw_max = 128) {
     int maxh = 1, maxw = 1;
     for (auto &e : ext) { maxh = std::max(maxh, e.first); maxw = std::max(maxw, e.second); }
     TileShape best{1, 1, 1};
     long best_tiles = -1;
-    const int wlim = std::min(std::min(maxw, 128), 256 / s), hlim = std::min(std::min(maxh, 128), 256 / s);
+    const int wlim = std::min(std::min(std::min(maxw, 128), 256 / s), bw_max), hlim = std::min(std::min(maxh, 128), 256 / s);
     for (int bw = 1; bw <= wlim; ++bw) {
         for (int bh = 1; bh <= hlim && bw * bh <= 128; ++bh) {
             const int bn = std::min(std::min(128 / (bw * bh), N), 256);
@@ -341,7 +345,8 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             const int i = q / Lout.nw(), j = q % Lout.nw();
             ext.push_back({Lout.ph(i), Lout.pw(j)});
         }
-        const TileShape ts = choose_tile(ext, N, s);
+        const int a3d = (cpad == 8 && s == 1) ? 1 : 0;  // TMA rows of 16 B are slow: merge 8 pixels per row
+        const TileShape ts = choose_tile(ext, N, s, a3d ? 32 : 128);
         static thread_local TcConvParams P;  // large; avoid the stack
         std::memset(&P, 0, sizeof(P));
         P.npatch = g1 - g0;
@@ -351,6 +356,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.kh = kh; P.kw = kw; P.s = s;
         P.cpadc = cpadc;
         P.kchan = cpad;
+        P.a3d = a3d;
         if (cpad >= 64) {
             P.cchunks = cpad / 64; P.tps = 1; P.ksteps = kh * kw * P.cchunks;
         } else {
@@ -394,9 +400,20 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             cuuint64_t strides[3] = {(cuuint64_t)cpad * 2, (cuuint64_t)wp * cpad * 2, (cuuint64_t)hp * wp * cpad * 2};
             cuuint32_t box[4] = {(cuuint32_t)cpadc, (cuuint32_t)(ts.BW * s), (cuuint32_t)(ts.BH * s), (cuuint32_t)ts.BNn};
             cuuint32_t es[4] = {1, (cuuint32_t)s, (cuuint32_t)s, 1};
-            CUresult r = encode(&P.mapA[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides, box, es,
-                                CU_TENSOR_MAP_INTERLEAVE_NONE, swz_for(row_bytes), CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+            CUresult r;
+            if (a3d) {
+                cuuint64_t d3[3] = {(cuuint64_t)wp * 8, (cuuint64_t)hp, (cuuint64_t)N};
+                cuuint64_t s3[2] = {(cuuint64_t)wp * 16, (cuuint64_t)hp * wp * 16};
+                cuuint32_t b3[3] = {(cuuint32_t)(ts.BW * 8), (cuuint32_t)ts.BH, (cuuint32_t)ts.BNn};
+                cuuint32_t e3[3] = {1, 1, 1};
+                r = encode(&P.mapA[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, base, d3, s3, b3, e3,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+            } else {
+                r = encode(&P.mapA[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides, box, es,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, swz_for(row_bytes), CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+            }
             if (r != CUDA_SUCCESS) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(A) failed");
         }
         P.tile_prefix[P.npatch] = tiles;
@@ -470,12 +487,14 @@ splitcnn_status_t launch_conv_dgrad_tc(const Level &Li, const Level &Lo, const L
 
 // ============================================================ weight gradient (tcgen05, MN-major)
 // dW[co][r][c][ci] = sum over pixels of dY[pix][co] * X~[pix shifted by (r, c)][ci]
-// GEMM per (co block of 128, tap, ci block): M = co, N = ci, K = pixels.  Both operands arrive from
-// TMA boxes whose rows are PIXELS and whose 128-byte rows hold 64 channels, i.e. MN-major SW128
-// tiles (an 8-pixel x 128 B atom; the next 64-channel block at LBO = 8 KB, the next 8 pixels at
-// SBO = 1 KB).  Split-K over pixel boxes of all patches in range; fp32 partial tiles go to the
+// GEMM with M = co (a block of 128 = two 64-channel dY boxes), K = pixels, and N = a set of B BLOCKS:
+// each block is one TMA box of the input X at one tap's shift and one channel chunk of `cbox`
+// channels, so one accumulator tile can cover several taps and the dY tile is loaded once for all
+// of them.  Both operands are MN-major (pixels are rows): SW128 / SW64 / SW32 / no-swizzle for
+// cbox = 64 / 32 / 16 / 8.  Split-K over pixel boxes of all patches; fp32 partial tiles go to the
 // workspace and a fixed-order reduction sums them (deterministic).
-constexpr int WG_ROWS = 64;  // pixels per K stage (4 MMAs of K = 16)
+constexpr int WG_ROWS = 64;    // pixels per K stage (4 MMAs of K = 16)
+constexpr int WG_MAXBLK = 32;  // B blocks per tile
 
 struct TcWgradParams {
     CUtensorMap mapDY[TC_MAXP];
@@ -486,12 +505,18 @@ struct TcWgradParams {
     int npatch;
     int BW, BH, BNn, rows_box;
     int kh, kw, s;
-    int nco_blk, nci_blk, ntiles;   // tiles = nco_blk * taps * nci_blk
-    int BNc;                        // ci per tile (64..256)
+    int x3d;                        // X maps are 3-D (8-channel rows merged: coordinate 8*w)
+    int cbox;                       // channels per B block
+    int nchunk;                     // channel chunks per tap (Cpi / cbox)
+    int bpt;                        // real blocks per tile
+    int bpt_pad;                    // blocks per tile incl. zero blocks (N = bpt_pad * cbox, multiple of 16)
+    int nblocks;                    // KT * nchunk
+    int nco_blk, ntb, ntiles;       // tiles = nco_blk * ntb
     int boxes_per_split, nsplit;
     int Cout, Cpi;
     int stages;
     uint32_t tmem_cols;
+    uint32_t b_layout, b_lbo, b_sbo, b_kstep, b_box_bytes;
     float *part;                    // [nsplit][Cout][kh][kw][Cpi]
 };
 
@@ -499,20 +524,21 @@ __global__ void __launch_bounds__(192, 1) wgrad_tc_kernel(const __grid_constant_
     extern __shared__ uint8_t smem_raw[];
     uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     const int S = p.stages;
-    const uint32_t a_stage = 2u * WG_ROWS * 128u;                 // 128 co = two 64-channel blocks
-    const uint32_t b_stage = (uint32_t)(p.BNc / 64) * WG_ROWS * 128u;
+    const uint32_t a_stage = 2u * WG_ROWS * 128u;  // 128 co = two 64-channel blocks
+    const uint32_t b_stage = (uint32_t)p.bpt_pad * p.b_box_bytes;
+    const uint32_t b_stage_al = (b_stage + 1023u) & ~1023u;
     uint8_t *sA = smem;
     uint8_t *sB = smem + (size_t)S * a_stage;
-    uint64_t *full = (uint64_t *)(sB + (size_t)S * b_stage);
+    uint64_t *full = (uint64_t *)(sB + (size_t)S * b_stage_al);
     uint64_t *empty = full + S;
     uint64_t *tfull = empty + S;
     uint32_t *tmem_slot = (uint32_t *)(tfull + 1);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
-    // rows >= rows_box of every stage are never written by TMA: zero them once so they add 0
+    // rows >= rows_box and the zero blocks are never written by TMA: zero them once so they add 0
     {
         uint4 *z = (uint4 *)smem;
-        const int n16 = (int)(((size_t)S * (a_stage + b_stage)) / 16);
+        const int n16 = (int)(((size_t)S * (a_stage + b_stage_al)) / 16);
         for (int i = threadIdx.x; i < n16; i += blockDim.x) z[i] = make_uint4(0, 0, 0, 0);
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     }
@@ -532,11 +558,9 @@ __global__ void __launch_bounds__(192, 1) wgrad_tc_kernel(const __grid_constant_
 
     // work item: z-major so CTAs running together share the same pixels (L2 reuse)
     const int tile = blockIdx.x % p.ntiles, z = blockIdx.x / p.ntiles;
-    const int KT = p.kh * p.kw;
-    const int ci_blk = tile % p.nci_blk;
-    const int tap = (tile / p.nci_blk) % KT;
-    const int co_blk = tile / (p.nci_blk * KT);
-    const int r = tap / p.kw, c = tap - r * p.kw;
+    const int tb = tile % p.ntb, co_blk = tile / p.ntb;
+    const int blk0 = tb * p.bpt;
+    const int nblk = min(p.bpt, p.nblocks - blk0);
     const int total_boxes = p.box_prefix[p.npatch];
     const int b0 = z * p.boxes_per_split, b1 = min(total_boxes, b0 + p.boxes_per_split);
 
@@ -545,7 +569,7 @@ __global__ void __launch_bounds__(192, 1) wgrad_tc_kernel(const __grid_constant_
             int stage = 0;
             uint32_t ph = 0;
             int ql = 0;
-            const uint32_t tx = (2u + (uint32_t)(p.BNc / 64)) * (uint32_t)p.rows_box * 128u;
+            const uint32_t tx = 2u * (uint32_t)p.rows_box * 128u + (uint32_t)nblk * p.rows_box * p.cbox * 2u;
             for (int b = b0; b < b1; ++b) {
                 while (b >= p.box_prefix[ql + 1]) ++ql;
                 int idx = b - p.box_prefix[ql];
@@ -556,29 +580,36 @@ __global__ void __launch_bounds__(192, 1) wgrad_tc_kernel(const __grid_constant_
                 tc::mbar_wait(&empty[stage], ph ^ 1);
                 tc::mbar_arrive_expect_tx(&full[stage], tx);
                 uint8_t *a = sA + (size_t)stage * a_stage;
-                uint8_t *bb = sB + (size_t)stage * b_stage;
+                uint8_t *bb = sB + (size_t)stage * b_stage_al;
                 for (int h = 0; h < 2; ++h)
                     tc::tma_load_4d(a + h * WG_ROWS * 128, &p.mapDY[ql], &full[stage], co_blk * 128 + h * 64, ow0, oh0, n0);
-                for (int h = 0; h < p.BNc / 64; ++h)
-                    tc::tma_load_4d(bb + h * WG_ROWS * 128, &p.mapX[ql], &full[stage], ci_blk * p.BNc + h * 64,
-                                    ow0 * p.s - p.pl[ql] + c, oh0 * p.s - p.pt[ql] + r, n0);
+                for (int k = 0; k < nblk; ++k) {
+                    const int blk = blk0 + k;
+                    const int tap = blk / p.nchunk, ch = blk - tap * p.nchunk;
+                    const int r = tap / p.kw, c = tap - r * p.kw;
+                    const int wx = ow0 * p.s - p.pl[ql] + c, hx = oh0 * p.s - p.pt[ql] + r;
+                    if (p.x3d)
+                        tc::tma_load_3d(bb + k * p.b_box_bytes, &p.mapX[ql], &full[stage], 8 * wx, hx, n0);
+                    else
+                        tc::tma_load_4d(bb + k * p.b_box_bytes, &p.mapX[ql], &full[stage], ch * p.cbox, wx, hx, n0);
+                }
                 if (++stage == S) { stage = 0; ph ^= 1; }
             }
         }
     } else if (warp == 1) {
         if (lane == 0) {
-            const uint32_t idesc = tc::idesc_bf16(128, p.BNc, 1, 1);
+            const uint32_t idesc = tc::idesc_bf16(128, p.bpt_pad * p.cbox, 1, 1);
             int stage = 0;
             uint32_t ph = 0;
             for (int b = b0; b < b1; ++b) {
                 tc::mbar_wait(&full[stage], ph);
                 tc::tc_fence_after();
                 const uint32_t a_base = tc::smem_u32(sA + (size_t)stage * a_stage);
-                const uint32_t b_base = tc::smem_u32(sB + (size_t)stage * b_stage);
+                const uint32_t b_base = tc::smem_u32(sB + (size_t)stage * b_stage_al);
 #pragma unroll
                 for (int j = 0; j < WG_ROWS / 16; ++j) {
                     const uint64_t adesc = tc::smem_desc(a_base + 2048u * j, WG_ROWS * 128, 1024, 2);
-                    const uint64_t bdesc = tc::smem_desc(b_base + 2048u * j, WG_ROWS * 128, 1024, 2);
+                    const uint64_t bdesc = tc::smem_desc(b_base + p.b_kstep * j, p.b_lbo, p.b_sbo, p.b_layout);
                     tc::mma_bf16(tmem_base, adesc, bdesc, idesc, (b != b0 || j) ? 1u : 0u);
                 }
                 tc::mma_commit(&empty[stage]);
@@ -595,8 +626,9 @@ __global__ void __launch_bounds__(192, 1) wgrad_tc_kernel(const __grid_constant_
             tc::tc_fence_after();
         }
         const uint32_t tacc = tmem_base + ((uint32_t)(quad * 32) << 16);
-        float *dst = p.part + ((((int64_t)z * p.Cout + co) * KT + tap) * p.Cpi) + ci_blk * p.BNc;
-        for (int cc = 0; cc < p.BNc; cc += 16) {
+        const int KT = p.kh * p.kw;
+        const int ncols = nblk * p.cbox;
+        for (int cc = 0; cc < ncols; cc += 16) {
             float v[16];
             if (any) {
                 tc::tmem_ld16(tacc + cc, v);
@@ -604,10 +636,17 @@ __global__ void __launch_bounds__(192, 1) wgrad_tc_kernel(const __grid_constant_
 #pragma unroll
                 for (int e = 0; e < 16; ++e) v[e] = 0.f;
             }
-            if (co < p.Cout && ci_blk * p.BNc + cc < p.Cpi) {
-                float4 *d4 = reinterpret_cast<float4 *>(dst + cc);
+            if (co >= p.Cout) continue;
 #pragma unroll
-                for (int e = 0; e < 4; ++e) d4[e] = make_float4(v[4 * e], v[4 * e + 1], v[4 * e + 2], v[4 * e + 3]);
+            for (int g = 0; g < 2; ++g) {
+                const int col = cc + 8 * g;
+                if (col >= ncols) break;
+                const int blk = blk0 + col / p.cbox;
+                const int tap = blk / p.nchunk, ch = blk - tap * p.nchunk;
+                float *dst = p.part + ((((int64_t)z * p.Cout + co) * KT + tap) * p.Cpi) + ch * p.cbox + (col % p.cbox);
+                float4 *d4 = reinterpret_cast<float4 *>(dst);
+                d4[0] = make_float4(v[8 * g], v[8 * g + 1], v[8 * g + 2], v[8 * g + 3]);
+                d4[1] = make_float4(v[8 * g + 4], v[8 * g + 5], v[8 * g + 6], v[8 * g + 7]);
             }
         }
     }
@@ -621,20 +660,23 @@ namespace {
 
 struct WgradCfg {
     TileShape ts;
-    int BNc, nco_blk, nci_blk, ntiles, total_boxes, nsplit, boxes_per_split;
+    int x3d, cbox, nchunk, nblocks, bpt, bpt_pad, ntb, nco_blk, ntiles, total_boxes, nsplit, boxes_per_split;
 };
 
 WgradCfg wgrad_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, int p0, int p1) {
     WgradCfg c{};
+    const int N = Lo.N, s = g.L.sh, KT = g.L.kh * g.L.kw;
+    c.cbox = std::min(Li.Cpad, 64);
+    c.x3d = (c.cbox == 8 && s == 1) ? 1 : 0;
     std::vector<std::pair<int, int>> ext;
     for (int q = p0; q < p1; ++q) ext.push_back({Lo.ph(q / Lo.nw()), Lo.pw(q % Lo.nw())});
     // pixel box of <= 64 rows (WG_ROWS) minimising the box count
     TileShape best{1, 1, 1};
     long best_n = -1;
-    const int N = Lo.N, s = g.L.sh;
     int maxh = 1, maxw = 1;
     for (auto &e : ext) { maxh = std::max(maxh, e.first); maxw = std::max(maxw, e.second); }
-    for (int bw = 1; bw <= std::min(std::min(maxw, WG_ROWS), 256 / s); ++bw)
+    const int wlim = std::min(std::min(maxw, WG_ROWS), c.x3d ? 32 : 256 / s);
+    for (int bw = 1; bw <= wlim; ++bw)
         for (int bh = 1; bh <= std::min(maxh, 256 / s) && bw * bh <= WG_ROWS; ++bh) {
             const int bn = std::min(WG_ROWS / (bw * bh), N);
             long n = 0;
@@ -643,13 +685,18 @@ WgradCfg wgrad_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, int p0,
         }
     c.ts = best;
     c.total_boxes = (int)best_n;
-    c.BNc = Li.Cpad % 256 == 0 ? 256 : (Li.Cpad % 128 == 0 ? 128 : 64);
+    c.nchunk = Li.Cpad / c.cbox;
+    c.nblocks = KT * c.nchunk;
+    const int maxb = std::min(WG_MAXBLK, 256 / c.cbox);
+    c.ntb = (c.nblocks + maxb - 1) / maxb;
+    c.bpt = (c.nblocks + c.ntb - 1) / c.ntb;
+    c.bpt_pad = c.bpt;
+    while ((c.bpt_pad * c.cbox) % 16) ++c.bpt_pad;  // MMA N multiple of 16
     c.nco_blk = (g.L.cout + 127) / 128;
-    c.nci_blk = Li.Cpad / c.BNc;
-    c.ntiles = c.nco_blk * g.L.kh * g.L.kw * c.nci_blk;
+    c.ntiles = c.nco_blk * c.ntb;
     int Z = std::max(1, (2 * num_sms() + c.ntiles - 1) / c.ntiles);
     Z = std::min(Z, std::max(1, c.total_boxes / 4));  // >= 4 boxes per split
-    Z = std::min(Z, 64);
+    Z = std::min(Z, 128);
     c.boxes_per_split = (c.total_boxes + Z - 1) / Z;
     c.nsplit = (c.total_boxes + c.boxes_per_split - 1) / c.boxes_per_split;
     return c;
@@ -658,7 +705,7 @@ WgradCfg wgrad_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, int p0,
 }  // namespace
 
 static bool wgrad_tc_ok(const Level &Li, const Level &Lo, const LayerGeom &g) {
-    return Li.Cpad % 64 == 0 && Lo.Cpad % 64 == 0 && g.L.sh == g.L.sw && g.L.sh <= 2;
+    return a_channels_ok(Li.Cpad) && Lo.Cpad % 64 == 0 && g.L.sh == g.L.sw && g.L.sh <= 2;
 }
 
 size_t wgrad_tc_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g) {
@@ -669,12 +716,11 @@ size_t wgrad_tc_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g) {
         WgradCfg c = wgrad_cfg(Li, Lo, g, g0, std::min(np, g0 + TC_MAXP));
         best = std::max(best, (size_t)c.nsplit * g.L.cout * g.L.kh * g.L.kw * Li.Cpad * sizeof(float));
     }
-    // plus the db partials of the CUDA-core helper
-    return best + 64 * (size_t)g.L.cout * sizeof(float) * 64 + 256;
+    return std::max(best, (size_t)4 * 148 * g.L.cout * sizeof(float)) + 256;  // db partials reuse the space
 }
 
-void launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, float *part, int cout, int p0, int p1,
-                        int cpp, cudaStream_t st);
+int launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, float *part, int cout, int p0, int p1,
+                       cudaStream_t st);
 void launch_reduce(const float *part, int Z, int64_t n, float *out, float beta, cudaStream_t st);
 
 splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *dy,
@@ -694,13 +740,26 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
         P.npatch = g1 - g0;
         P.BW = c.ts.BW; P.BH = c.ts.BH; P.BNn = c.ts.BNn; P.rows_box = c.ts.BW * c.ts.BH * c.ts.BNn;
         P.kh = g.L.kh; P.kw = g.L.kw; P.s = s;
-        P.nco_blk = c.nco_blk; P.nci_blk = c.nci_blk; P.ntiles = c.ntiles; P.BNc = c.BNc;
+        P.x3d = c.x3d; P.cbox = c.cbox; P.nchunk = c.nchunk; P.bpt = c.bpt; P.bpt_pad = c.bpt_pad;
+        P.nblocks = c.nblocks; P.nco_blk = c.nco_blk; P.ntb = c.ntb; P.ntiles = c.ntiles;
         P.boxes_per_split = c.boxes_per_split; P.nsplit = c.nsplit;
         P.Cout = g.L.cout; P.Cpi = Li.Cpad;
-        const uint32_t stage_bytes = 2u * WG_ROWS * 128u + (uint32_t)(c.BNc / 64) * WG_ROWS * 128u;
+        const uint32_t row_bytes = (uint32_t)c.cbox * 2u;
+        P.b_box_bytes = WG_ROWS * row_bytes;
+        P.b_layout = layout_for((int)row_bytes);
+        if (row_bytes == 16) {        // no swizzle, MN-major: SBO = MN-block stride, LBO = 8-row K-group stride
+            P.b_sbo = P.b_box_bytes;
+            P.b_lbo = 128;
+        } else {                      // swizzled MN-major: LBO = MN-block stride, SBO = 8-row K-group stride
+            P.b_lbo = P.b_box_bytes;
+            P.b_sbo = 8u * row_bytes;
+        }
+        P.b_kstep = 16u * row_bytes;
+        const uint32_t b_stage_al = ((uint32_t)c.bpt_pad * P.b_box_bytes + 1023u) & ~1023u;
+        const uint32_t stage_bytes = 2u * WG_ROWS * 128u + b_stage_al;
         P.stages = std::min<int>(8, (int)((200u * 1024u) / stage_bytes));
         uint32_t cols = 32;
-        while (cols < (uint32_t)c.BNc) cols <<= 1;
+        while (cols < (uint32_t)(c.bpt_pad * c.cbox)) cols <<= 1;
         P.tmem_cols = cols;
         P.part = part;
         int boxes = 0;
@@ -728,14 +787,26 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
             {
                 const int C = Li.Cpad;
                 void *base = (char *)x + Li.offset(i, j) * 2;
-                cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)wp, (cuuint64_t)hp, (cuuint64_t)Li.N};
-                cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)wp * C * 2, (cuuint64_t)hp * wp * C * 2};
-                cuuint32_t box[4] = {64, (cuuint32_t)(c.ts.BW * s), (cuuint32_t)(c.ts.BH * s), (cuuint32_t)c.ts.BNn};
-                cuuint32_t es[4] = {1, (cuuint32_t)s, (cuuint32_t)s, 1};
-                if (encode(&P.mapX[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides, box, es,
-                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
-                    return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(X) failed");
+                CUresult r;
+                if (c.x3d) {  // 8-channel pixels merged into rows: dims (8*wp, hp, N), box (8*BW, BH, BNn)
+                    cuuint64_t dims[3] = {(cuuint64_t)wp * 8, (cuuint64_t)hp, (cuuint64_t)Li.N};
+                    cuuint64_t strides[2] = {(cuuint64_t)wp * 16, (cuuint64_t)hp * wp * 16};
+                    cuuint32_t box[3] = {(cuuint32_t)(c.ts.BW * 8), (cuuint32_t)c.ts.BH, (cuuint32_t)c.ts.BNn};
+                    cuuint32_t es[3] = {1, 1, 1};
+                    r = encode(&P.mapX[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, base, dims, strides, box, es,
+                               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                } else {
+                    cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)wp, (cuuint64_t)hp, (cuuint64_t)Li.N};
+                    cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)wp * C * 2, (cuuint64_t)hp * wp * C * 2};
+                    cuuint32_t box[4] = {(cuuint32_t)c.cbox, (cuuint32_t)(c.ts.BW * s), (cuuint32_t)(c.ts.BH * s),
+                                         (cuuint32_t)c.ts.BNn};
+                    cuuint32_t es[4] = {1, (cuuint32_t)s, (cuuint32_t)s, 1};
+                    r = encode(&P.mapX[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides, box, es,
+                               CU_TENSOR_MAP_INTERLEAVE_NONE, swz_for((int)row_bytes), CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                }
+                if (r != CUDA_SUCCESS) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(X) failed");
             }
         }
         P.box_prefix[P.npatch] = boxes;
@@ -753,11 +824,9 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
         first = false;
     }
     if (db) {
-        const int np = p1 - p0;
-        const int cpp = std::max(1, std::min(64, (2 * num_sms() + np - 1) / np));
-        float *part_db = part + 0;  // the dW partials have been consumed by the reduction (stream order)
-        launch_db_partials(SPLITCNN_BF16, Lo, dy, part_db, g.L.cout, p0, p1, cpp, st);
-        launch_reduce(part_db, np * cpp, g.L.cout, db, beta, st);
+        // the dW partials have been consumed by the reduction (stream order): reuse the space
+        const int Zd = launch_db_partials(SPLITCNN_BF16, Lo, dy, part, g.L.cout, p0, p1, st);
+        launch_reduce(part, Zd, g.L.cout, db, beta, st);
     }
     return SPLITCNN_OK;
 }

@@ -40,6 +40,7 @@ class SplitNet:
         self.flags_extra = sc.FLAG_FORCE_SIMT if force_simt else 0
         self.step_index = 0
         self.timers = None       # list -> every library call is bracketed by CUDA events (bench.py)
+        self._label = ""
         self.region = self._make_region_plan(0)
         self.patch_range = patch_range or (0, self.region.npatch)
         L = self.region.levels[-1]
@@ -134,7 +135,7 @@ class SplitNet:
         e0.record()
         fn(*args)
         e1.record()
-        self.timers.append((kind, e0, e1, work))
+        self.timers.append((kind, e0, e1, work, self._label))
 
     def _conv_work(self, plan, m, l):
         lo = plan.levels[m + 1]
@@ -172,6 +173,7 @@ class SplitNet:
 
     def _run_fwd(self, key, plan, layers, acts, p0, p1, stream):
         for m, l in enumerate(layers):
+            self._label = l.get("name", f"{key}{m}")
             if l["op"] == "conv":
                 W, b = self.params[(key, m)]
                 flags = (sc.FLAG_RELU if l.get("relu", True) else 0) | self.flags_extra
@@ -200,6 +202,7 @@ class SplitNet:
     def _run_bwd(self, key, plan, layers, acts, g, p0, p1, stream, need_input_grad):
         for m in range(len(layers) - 1, -1, -1):
             l = layers[m]
+            self._label = l.get("name", f"{key}{m}")
             out = self.grad[0] if g is not self.grad[0] else self.grad[1]
             last = (m == 0 and not need_input_grad)
             if l["op"] == "conv":

@@ -67,6 +67,11 @@ CONV_CASES = [
     ("vgg_first", 2, 3, 64, 3, 1, 1, 32, 28, 2, 2, True),
     ("vgg128_256", 2, 128, 256, 3, 1, 1, 16, 16, 3, 3, True),
     ("c5_7x7patch", 2, 256, 256, 3, 1, 1, 28, 28, 4, 4, True),
+    ("wg_c16", 2, 16, 64, 3, 1, 1, 20, 20, 2, 2, True),
+    ("wg_c32", 2, 32, 128, 3, 1, 1, 18, 22, 2, 3, True),
+    ("s2_c64", 2, 64, 128, 3, 2, 1, 28, 28, 2, 2, True),
+    ("7x7s2_c3_64", 2, 3, 64, 7, 2, 3, 30, 30, 2, 2, True),
+    ("c512", 1, 512, 512, 3, 1, 1, 14, 14, 2, 2, True),
 ]
 
 

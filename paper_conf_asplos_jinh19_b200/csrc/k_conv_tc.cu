@@ -36,6 +36,8 @@ size_t wgrad_tc_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g);
 
 struct TcConvParams {
     CUtensorMap mapA[TC_MAXP];
+    CUtensorMap mapY[TC_MAXP];   // output patch maps (TMA store of the staged tile)
+    CUtensorMap mapR[TC_MAXP];   // ReLU-mask source maps (dgrad), same geometry as the output
     CUtensorMap mapB;
     int64_t out_off[TC_MAXP];
     int tile_prefix[TC_MAXP + 1];
@@ -59,11 +61,22 @@ struct TcConvParams {
     __nv_bfloat16 *y;
     const __nv_bfloat16 *relu_src;
     int relu;
+    int tpp;          // tiles per patch when uniform (O(1) decode), else 0
+    int direct;       // 1: per-thread global stores (odd channel pads); 0: smem-staged TMA store
+    int ychunk;       // channels per output box (64, 32, 16 or 8)
+    uint32_t y_mask;  // swizzle mask of the staging tile (7 / 3 / 1 / 0)
+    uint32_t stage_off, bar_off;  // smem layout
 };
 
+static_assert(sizeof(TcConvParams) <= 32000, "kernel parameter space is 32 KB");
+
 __device__ __forceinline__ void decode_tile(const TcConvParams &p, int t, int &ql, int &nb, int &hb, int &wb, int &cb) {
-    ql = 0;
-    while (t >= p.tile_prefix[ql + 1]) ++ql;
+    if (p.tpp) {
+        ql = t / p.tpp;
+    } else {
+        ql = 0;
+        while (t >= p.tile_prefix[ql + 1]) ++ql;
+    }
     int idx = t - p.tile_prefix[ql];
     cb = idx % p.nco;
     idx /= p.nco;
@@ -73,18 +86,61 @@ __device__ __forceinline__ void decode_tile(const TcConvParams &p, int t, int &q
     nb = idx / p.nhb[ql];
 }
 
-__global__ void __launch_bounds__(192, 1) conv_tc_kernel(const __grid_constant__ TcConvParams p) {
+constexpr int CONV_THREADS = 64 + 256;  // producer warp, MMA warp, 8 epilogue warps (2 per TMEM lane quadrant)
+
+// 8 accumulator columns -> bf16x8 with the fused epilogue (bias, ReLU, or the dgrad ReLU mask)
+template <bool BIAS, bool RELU, bool MASK>
+__device__ __forceinline__ uint4 epi8(const uint32_t *r, const float *sb, int co, int Cout, uint4 m4) {
+    float o[8];
+#pragma unroll
+    for (int e = 0; e < 8; ++e) o[e] = __uint_as_float(r[e]);
+    if (co + 8 <= Cout) {
+        if (BIAS) {
+            const float4 b0 = *reinterpret_cast<const float4 *>(sb + co);
+            const float4 b1 = *reinterpret_cast<const float4 *>(sb + co + 4);
+            o[0] += b0.x; o[1] += b0.y; o[2] += b0.z; o[3] += b0.w;
+            o[4] += b1.x; o[5] += b1.y; o[6] += b1.z; o[7] += b1.w;
+        }
+    } else {
+#pragma unroll
+        for (int e = 0; e < 8; ++e) o[e] = (co + e < Cout) ? (BIAS ? o[e] + sb[co + e] : o[e]) : 0.f;
+    }
+    if (RELU) {
+#pragma unroll
+        for (int e = 0; e < 8; ++e) o[e] = fmaxf(o[e], 0.f);
+    }
+    if (MASK) {
+        const __nv_bfloat162 *mh = reinterpret_cast<const __nv_bfloat162 *>(&m4);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+            const float2 mf = __bfloat1622float2(mh[e]);
+            o[2 * e] = mf.x > 0.f ? o[2 * e] : 0.f;
+            o[2 * e + 1] = mf.y > 0.f ? o[2 * e + 1] : 0.f;
+        }
+    }
+    uint4 pk;
+    __nv_bfloat162 *h2 = reinterpret_cast<__nv_bfloat162 *>(&pk);
+#pragma unroll
+    for (int e = 0; e < 4; ++e) h2[e] = __floats2bfloat162_rn(o[2 * e], o[2 * e + 1]);
+    return pk;
+}
+
+template <bool BIAS, bool RELU, bool MASK>
+__global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_constant__ TcConvParams p) {
     extern __shared__ uint8_t smem_raw[];
     uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     const int S = p.stages;
     const uint32_t b_stage = (uint32_t)p.BN * 128u;
     uint8_t *sA = smem;
     uint8_t *sB = smem + (size_t)S * 16384;
-    uint64_t *full = (uint64_t *)(sB + (size_t)S * b_stage);
+    uint8_t *sY = smem + p.stage_off;  // output staging tile (1024-aligned)
+    uint64_t *full = (uint64_t *)(smem + p.bar_off);
     uint64_t *empty = full + S;
     uint64_t *tfull = empty + S;
     uint64_t *tempty = tfull + 2;
-    uint32_t *tmem_slot = (uint32_t *)(tempty + 2);
+    uint64_t *ybar = tempty + 2;
+    uint32_t *tmem_slot = (uint32_t *)(ybar + 1);
+    float *sbias = (float *)(smem + p.bar_off + 512);   // [Cout] bias (16-byte aligned)
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (warp == 0 && lane == 0) {
@@ -94,10 +150,13 @@ __global__ void __launch_bounds__(192, 1) conv_tc_kernel(const __grid_constant__
         }
         for (int a = 0; a < 2; ++a) {
             tc::mbar_init(&tfull[a], 1);
-            tc::mbar_init(&tempty[a], 4);
+            tc::mbar_init(&tempty[a], 8);
         }
+        tc::mbar_init(ybar, 1);
         tc::fence_barrier_init();
     }
+    if (BIAS)
+        for (int i = threadIdx.x; i < p.Cout; i += blockDim.x) sbias[i] = __ldg(p.bias + i);
     if (warp == 1) tc::tmem_alloc_dyn(tmem_slot, p.tmem_cols);
     tc::tc_fence_before();
     __syncthreads();
@@ -120,7 +179,7 @@ __global__ void __launch_bounds__(192, 1) conv_tc_kernel(const __grid_constant__
                 const int hbase = hb * p.BH * p.s - p.pt[ql];
                 const int n0 = nb * p.BNn, co0 = cb * p.BN;
                 for (int ks = 0; ks < p.ksteps; ++ks) {
-                    tc::mbar_wait(&empty[stage], ph ^ 1);
+                    tc::mbar_wait_sleep(&empty[stage], ph ^ 1);
                     tc::mbar_arrive_expect_tx(&full[stage], p.a_tx_bytes + p.b_tx_bytes);
                     uint8_t *a = sA + (size_t)stage * 16384;
                     uint8_t *b = sB + (size_t)stage * b_stage;
@@ -151,7 +210,7 @@ __global__ void __launch_bounds__(192, 1) conv_tc_kernel(const __grid_constant__
             int stage = 0, acc = 0;
             uint32_t ph = 0, aph = 0;
             for (int t = blockIdx.x; t < total; t += gridDim.x) {
-                tc::mbar_wait(&tempty[acc], aph ^ 1);
+                tc::mbar_wait_sleep(&tempty[acc], aph ^ 1);
                 tc::tc_fence_after();
                 const uint32_t d = tmem_base + (uint32_t)(acc * p.BN);
                 for (int ks = 0; ks < p.ksteps; ++ks) {
@@ -176,10 +235,85 @@ __global__ void __launch_bounds__(192, 1) conv_tc_kernel(const __grid_constant__
                 if (acc == 0) aph ^= 1;
             }
         }
+    } else if (!p.direct) {
+        // ================= epilogue: warps 2..9, TMEM lane quadrant = warp % 4, column half = (warp-2)/4;
+        // accumulator -> fused bias/ReLU/mask -> bf16 -> swizzled smem staging tile -> TMA store
+        const int quad = warp & 3;
+        const int half = (warp - 2) >> 2;
+        const int row = quad * 32 + lane;      // TMEM lane = tile row = staging row
+        const int etid = threadIdx.x - 64;     // 0..255
+        const uint32_t rowB = (uint32_t)p.ychunk * 2u;
+        const uint32_t chunk_bytes = 128u * rowB;
+        int acc = 0;
+        uint32_t aph = 0, yph = 0;
+        for (int t = blockIdx.x; t < total; t += gridDim.x) {
+            int ql, nb, hb, wb, cb;
+            decode_tile(p, t, ql, nb, hb, wb, cb);
+            const int co0 = cb * p.BN;
+            const int ow0 = wb * p.BW, oh0 = hb * p.BH, n0 = nb * p.BNn;
+            const int ncols = min(p.BN, p.Cpo - co0);       // channels this tile stores (multiple of ychunk)
+            const int nchunks = ncols / p.ychunk;
+            // the staging tile is free once the previous tile's TMA store has read it
+            if (etid == 0) tc::bulk_wait_read0();
+            tc::named_bar_sync(1, 256);
+            if (MASK) {  // ReLU-mask tile (same box as the output) into the staging tile
+                if (etid == 0) {
+                    tc::mbar_arrive_expect_tx(ybar, (uint32_t)nchunks * p.rows_box * rowB);
+                    for (int k = 0; k < nchunks; ++k)
+                        tc::tma_load_4d(sY + k * chunk_bytes, &p.mapR[ql], ybar, co0 + k * p.ychunk, ow0, oh0, n0);
+                }
+                tc::mbar_wait(ybar, yph);
+                yph ^= 1;
+            }
+            tc::mbar_wait(&tfull[acc], aph);
+            tc::tc_fence_after();
+            const uint32_t tacc = tmem_base + (uint32_t)(acc * p.BN) + ((uint32_t)(quad * 32) << 16);
+            // 16-column groups interleaved between the two column halves
+            for (int cc = 16 * half; cc < ncols; cc += 32) {
+                uint32_t r[16];
+                tc::tmem_ld16_nw(tacc + cc, r);
+                tc::tmem_wait_ld();
+#pragma unroll
+                for (int u = 0; u < 2; ++u) {
+                    const int c8 = cc + 8 * u;
+                    if (c8 >= ncols) break;
+                    const int k = c8 / p.ychunk;
+                    const uint32_t off = tc::swz((uint32_t)row * rowB + (uint32_t)(c8 - k * p.ychunk) * 2u, p.y_mask);
+                    uint4 *dst = reinterpret_cast<uint4 *>(sY + k * chunk_bytes + off);
+                    const uint4 m4 = MASK ? *dst : make_uint4(0, 0, 0, 0);
+                    *dst = epi8<BIAS, RELU, MASK>(r + 8 * u, sbias, co0 + c8, p.Cout, m4);
+                }
+            }
+            tc::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(&tempty[acc]);   // accumulator free: the MMA may proceed
+            tc::fence_proxy_async_smem();
+            tc::named_bar_sync(1, 256);
+            if (etid == 0) {
+                for (int k = 0; k < nchunks; ++k)
+                    tc::tma_store_4d(&p.mapY[ql], sY + k * chunk_bytes, co0 + k * p.ychunk, ow0, oh0, n0);
+                tc::bulk_commit();
+            }
+            acc ^= 1;
+            if (acc == 0) aph ^= 1;
+        }
+        if (etid == 0) tc::bulk_wait0();
     } else {
-        // ================= epilogue (warps 2..5 -> TMEM lane quadrants 2,3,0,1)
+        // ================= epilogue, direct per-thread stores (channel pads without a TMA box fit);
+        // warps 6..9 only keep the tempty arrival count
         const int quad = warp & 3;
         const int row = quad * 32 + lane;
+        if (warp >= 6) {
+            int acc = 0;
+            uint32_t aph = 0;
+            for (int t = blockIdx.x; t < total; t += gridDim.x) {
+                tc::mbar_wait(&tfull[acc], aph);
+                __syncwarp();
+                if (lane == 0) tc::mbar_arrive(&tempty[acc]);
+                acc ^= 1;
+                if (acc == 0) aph ^= 1;
+            }
+        } else {
         const int wi = row % p.BW, hi = (row / p.BW) % p.BH, ni = row / (p.BW * p.BH);
         int acc = 0;
         uint32_t aph = 0;
@@ -227,6 +361,7 @@ __global__ void __launch_bounds__(192, 1) conv_tc_kernel(const __grid_constant__
             if (lane == 0) tc::mbar_arrive(&tempty[acc]);
             acc ^= 1;
             if (acc == 0) aph ^= 1;
+        }
         }
     }
     tc::tc_fence_before();
@@ -337,7 +472,6 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
     const int BN = std::min(256, round_up16(ncols_out));
     const int nco = (ncols_out + BN - 1) / BN;
     const int N = La.N;
-    static bool attr_set = false;
     for (int g0 = p0; g0 < p1; g0 += TC_MAXP) {
         const int g1 = std::min(p1, g0 + TC_MAXP);
         std::vector<std::pair<int, int>> ext;
@@ -371,7 +505,15 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.a_tx_bytes = (uint32_t)P.tps * P.rows_box * row_bytes;
         P.b_tx_bytes = (uint32_t)BN * 128u;
         const uint32_t stage_bytes = 16384u + P.b_tx_bytes;
-        P.stages = std::min<int>(8, (int)((200u * 1024u) / stage_bytes));
+        // output staging for the TMA-store epilogue: channel box of min(64, Cpo), swizzle to match
+        const int ych = std::min(64, Lout.Cpad);
+        P.direct = !((ych == 8 || ych == 16 || ych == 32 || ych == 64) && Lout.Cpad % ych == 0);
+        P.ychunk = ych;
+        P.y_mask = ych == 64 ? 7u : ych == 32 ? 3u : ych == 16 ? 1u : 0u;
+        const uint32_t staging = P.direct ? 0u : (uint32_t)((BN + ych - 1) / ych) * 128u * (uint32_t)ych * 2u;
+        P.stages = std::min<int>(8, (int)((208u * 1024u - staging) / stage_bytes));
+        P.stage_off = (uint32_t)P.stages * stage_bytes;
+        P.bar_off = P.stage_off + ((staging + 1023u) & ~1023u);
         uint32_t cols = 32;
         while (cols < 2u * BN) cols <<= 1;
         P.tmem_cols = cols;
@@ -415,8 +557,30 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
                            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
             }
             if (r != CUDA_SUCCESS) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(A) failed");
+            if (!P.direct) {  // output (and ReLU-mask) maps over the output patch buffer
+                const int yc = Lout.Cpad;
+                cuuint64_t ydims[4] = {(cuuint64_t)yc, (cuuint64_t)ow, (cuuint64_t)oh, (cuuint64_t)N};
+                cuuint64_t ystr[3] = {(cuuint64_t)yc * 2, (cuuint64_t)ow * yc * 2, (cuuint64_t)oh * ow * yc * 2};
+                cuuint32_t ybox[4] = {(cuuint32_t)P.ychunk, (cuuint32_t)ts.BW, (cuuint32_t)ts.BH, (cuuint32_t)ts.BNn};
+                cuuint32_t yes[4] = {1, 1, 1, 1};
+                void *ybase = (char *)y + Lout.offset(i, j) * 2;
+                if (encode(&P.mapY[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, ybase, ydims, ystr, ybox, yes,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, swz_for(P.ychunk * 2), CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+                    return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(Y) failed");
+                if (relu_src) {
+                    void *rbase = (char *)relu_src + Lout.offset(i, j) * 2;
+                    if (encode(&P.mapR[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, rbase, ydims, ystr, ybox, yes,
+                               CU_TENSOR_MAP_INTERLEAVE_NONE, swz_for(P.ychunk * 2), CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+                        return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(R) failed");
+                }
+            }
         }
         P.tile_prefix[P.npatch] = tiles;
+        P.tpp = P.tile_prefix[1];
+        for (int ql = 1; ql < P.npatch; ++ql)
+            if (P.tile_prefix[ql + 1] - P.tile_prefix[ql] != P.tpp) P.tpp = 0;
         {
             const int K = kh * kw * cpad;
             cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)w_rows};
@@ -429,13 +593,27 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             if (r != CUDA_SUCCESS) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(B) failed");
         }
         if (tiles == 0) continue;
-        const size_t smem = 1024 + (size_t)P.stages * stage_bytes + 256;
-        if (!attr_set) {
-            cudaFuncSetAttribute(conv_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-            attr_set = true;
-        }
+        const size_t smem = 1024 + (size_t)P.bar_off + 512 + (bias ? 4 * (size_t)g.L.cout : 0) + 64;
         const int grid = std::min(tiles, num_sms());
-        conv_tc_kernel<<<grid, 192, smem, st>>>(P);
+        const int mode_bits = (bias ? 4 : 0) | (relu ? 2 : 0) | (relu_src ? 1 : 0);
+        auto launch = [&](auto kern) {
+            static bool set[8] = {false};
+            if (!set[mode_bits]) {
+                cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+                set[mode_bits] = true;
+            }
+            kern<<<grid, CONV_THREADS, smem, st>>>(P);
+        };
+        switch (mode_bits) {
+            case 0: launch(conv_tc_kernel<false, false, false>); break;
+            case 1: launch(conv_tc_kernel<false, false, true>); break;
+            case 2: launch(conv_tc_kernel<false, true, false>); break;
+            case 3: launch(conv_tc_kernel<false, true, true>); break;
+            case 4: launch(conv_tc_kernel<true, false, false>); break;
+            case 5: launch(conv_tc_kernel<true, false, true>); break;
+            case 6: launch(conv_tc_kernel<true, true, false>); break;
+            default: launch(conv_tc_kernel<true, true, true>); break;
+        }
         count_launch();
         {
             cudaError_t e = cudaGetLastError();

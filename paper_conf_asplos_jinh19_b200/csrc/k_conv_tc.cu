@@ -834,6 +834,141 @@ __global__ void __launch_bounds__(192, 1) wgrad_tc_kernel(const __grid_constant_
     if (warp == 1) tc::tmem_dealloc(tmem_base, p.tmem_cols);
 }
 
+// ------------------------------------------------------------ halo weight gradient (stride 1, 3 taps per row)
+// Same GEMM as above, but the kw taps of one kernel row r share ONE input box: the X tile for output
+// rows [h0, h0+BH) x 8 output columns is loaded with kw-1 halo columns (8+kw-1 pixels wide).  In the
+// MN-major SW128 layout a pixel is a 128-byte smem row, so the operand of tap (r, c) is the same tile
+// viewed c rows further on, and the kw taps are kw MN-blocks of ONE MMA with LBO = 128 B (N = kw*64).
+// The output-row K groups of 8 pixels sit Wp = 8+kw-1 rows apart (SBO = Wp*128 B).  The SW128 swizzle
+// is address-based, so any 128-byte row offset is a valid operand start (probed: scripts/umma_probe.cu).
+// Per stage: 2 dY boxes + 1 X box for BH*8 pixels (3 TMA ops vs 2+kw).
+struct TcWgHaloParams {
+    CUtensorMap mapDY[TC_MAXP];
+    CUtensorMap mapX[TC_MAXP];
+    int box_prefix[TC_MAXP + 1];
+    int pt[TC_MAXP], pl[TC_MAXP];
+    int nhb[TC_MAXP], nwb[TC_MAXP];
+    int npatch, BH, kh, kw;
+    int nco_blk, nchunk, ntiles, boxes_per_split, nsplit;
+    int Cout, Cpi, stages;
+    uint32_t tmem_cols;
+    float *part;  // [nsplit][Cout][kh][kw][Cpi]
+};
+
+__global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constant__ TcWgHaloParams p) {
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+    const int S = p.stages;
+    const int rows = p.BH * 8;                        // pixels per stage
+    const int Wp = 8 + p.kw - 1;
+    const uint32_t a_blk = (uint32_t)rows * 128u;     // one 64-channel dY block
+    const uint32_t a_stage = 2u * a_blk;
+    const uint32_t b_stage = ((uint32_t)Wp * p.BH * 128u + 1023u) & ~1023u;
+    uint8_t *sA = smem;
+    uint8_t *sB = smem + (size_t)S * a_stage;
+    uint64_t *full = (uint64_t *)(sB + (size_t)S * b_stage);
+    uint64_t *empty = full + S;
+    uint64_t *tfull = empty + S;
+    uint32_t *tmem_slot = (uint32_t *)(tfull + 1);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (warp == 0 && lane == 0) {
+        for (int s = 0; s < S; ++s) {
+            tc::mbar_init(&full[s], 1);
+            tc::mbar_init(&empty[s], 1);
+        }
+        tc::mbar_init(&tfull[0], 1);
+        tc::fence_barrier_init();
+    }
+    if (warp == 1) tc::tmem_alloc_dyn(tmem_slot, p.tmem_cols);
+    tc::tc_fence_before();
+    __syncthreads();
+    tc::tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    const int tile = blockIdx.x % p.ntiles, z = blockIdx.x / p.ntiles;
+    const int ch = tile % p.nchunk;
+    const int r = (tile / p.nchunk) % p.kh;
+    const int co_blk = tile / (p.nchunk * p.kh);
+    const int total_boxes = p.box_prefix[p.npatch];
+    const int b0 = z * p.boxes_per_split, b1 = min(total_boxes, b0 + p.boxes_per_split);
+    const int N = p.kw * 64;
+
+    if (warp == 0) {
+        if (lane == 0) {
+            int stage = 0, ql = 0;
+            uint32_t ph = 0;
+            const uint32_t tx = a_stage + (uint32_t)Wp * p.BH * 128u;
+            for (int b = b0; b < b1; ++b) {
+                while (b >= p.box_prefix[ql + 1]) ++ql;
+                int idx = b - p.box_prefix[ql];
+                const int wb = idx % p.nwb[ql];
+                idx /= p.nwb[ql];
+                const int hb = idx % p.nhb[ql], n = idx / p.nhb[ql];
+                const int ow0 = wb * 8, oh0 = hb * p.BH;
+                tc::mbar_wait_sleep(&empty[stage], ph ^ 1);
+                tc::mbar_arrive_expect_tx(&full[stage], tx);
+                uint8_t *a = sA + (size_t)stage * a_stage;
+                tc::tma_load_4d(a, &p.mapDY[ql], &full[stage], co_blk * 128, ow0, oh0, n);
+                tc::tma_load_4d(a + a_blk, &p.mapDY[ql], &full[stage], co_blk * 128 + 64, ow0, oh0, n);
+                tc::tma_load_4d(sB + (size_t)stage * b_stage, &p.mapX[ql], &full[stage], ch * 64, ow0 - p.pl[ql],
+                                oh0 - p.pt[ql] + r, n);
+                if (++stage == S) { stage = 0; ph ^= 1; }
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            const uint32_t idesc = tc::idesc_bf16(128, N, 1, 1);
+            int stage = 0;
+            uint32_t ph = 0;
+            for (int b = b0; b < b1; ++b) {
+                tc::mbar_wait(&full[stage], ph);
+                tc::tc_fence_after();
+                const uint32_t a_base = tc::smem_u32(sA + (size_t)stage * a_stage);
+                const uint32_t b_base = tc::smem_u32(sB + (size_t)stage * b_stage);
+                for (int j = 0; j < rows / 16; ++j) {
+                    // A: dY, MN-major: 8-pixel K groups at 1 KB, the second 64-co block at LBO = a_blk
+                    const uint64_t adesc = tc::smem_desc(a_base + 2048u * j, a_blk, 1024, 2);
+                    // B: X halo view, MN-major: tap c = MN block c at LBO = 128 B, K groups (output rows)
+                    //    at SBO = Wp rows; 16 pixels = 2 output rows
+                    const uint64_t bdesc = tc::smem_desc(b_base + (uint32_t)(2 * j * Wp) * 128u, 128, (uint32_t)Wp * 128u, 2);
+                    tc::mma_bf16(tmem_base, adesc, bdesc, idesc, (b != b0 || j) ? 1u : 0u);
+                }
+                tc::mma_commit(&empty[stage]);
+                if (++stage == S) { stage = 0; ph ^= 1; }
+            }
+            tc::mma_commit(&tfull[0]);
+        }
+    } else {
+        const int quad = warp & 3;
+        const int co = co_blk * 128 + quad * 32 + lane;
+        const bool any = b1 > b0;
+        if (any) {
+            tc::mbar_wait(&tfull[0], 0);
+            tc::tc_fence_after();
+        }
+        const uint32_t tacc = tmem_base + ((uint32_t)(quad * 32) << 16);
+        const int KT = p.kh * p.kw;
+        for (int cc = 0; cc < N; cc += 16) {
+            float v[16];
+            if (any) {
+                tc::tmem_ld16(tacc + cc, v);
+            } else {
+#pragma unroll
+                for (int e = 0; e < 16; ++e) v[e] = 0.f;
+            }
+            if (co >= p.Cout) continue;
+            const int c = cc / 64, ci = ch * 64 + (cc % 64);
+            float4 *d4 = reinterpret_cast<float4 *>(p.part + (((int64_t)z * p.Cout + co) * KT + r * p.kw + c) * p.Cpi + ci);
+#pragma unroll
+            for (int e = 0; e < 4; ++e) d4[e] = make_float4(v[4 * e], v[4 * e + 1], v[4 * e + 2], v[4 * e + 3]);
+        }
+    }
+    tc::tc_fence_before();
+    __syncthreads();
+    tc::tc_fence_after();
+    if (warp == 1) tc::tmem_dealloc(tmem_base, p.tmem_cols);
+}
+
 namespace {
 
 struct WgradCfg {
@@ -882,6 +1017,40 @@ WgradCfg wgrad_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, int p0,
 
 }  // namespace
 
+namespace {
+
+struct WgHaloCfg {
+    int BH, nco_blk, nchunk, ntiles, total_boxes, nsplit, boxes_per_split;
+};
+
+bool wgrad_halo_ok(const Level &Li, const Level &Lo, const LayerGeom &g) {
+    return g.L.sh == 1 && g.L.sw == 1 && g.L.kw >= 2 && g.L.kw <= 4 && Li.Cpad % 64 == 0 && Lo.Cpad % 64 == 0;
+}
+
+WgHaloCfg wgrad_halo_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, int p0, int p1) {
+    WgHaloCfg c{};
+    long best = -1;
+    for (int bh : {16, 8}) {
+        long n = 0;
+        for (int q = p0; q < p1; ++q)
+            n += (long)Lo.N * ((Lo.ph(q / Lo.nw()) + bh - 1) / bh) * ((Lo.pw(q % Lo.nw()) + 7) / 8);
+        // cost ~ boxes x (fixed per-box cost + pixels): prefer fewer, larger boxes unless they waste rows
+        const long cost = n * (bh * 8 + 192);
+        if (best < 0 || cost < best) { best = cost; c.BH = bh; c.total_boxes = (int)n; }
+    }
+    c.nco_blk = (g.L.cout + 127) / 128;
+    c.nchunk = Li.Cpad / 64;
+    c.ntiles = c.nco_blk * g.L.kh * c.nchunk;
+    int Z = std::max(1, (2 * num_sms() + c.ntiles - 1) / c.ntiles);
+    Z = std::min(Z, std::max(1, c.total_boxes / 4));
+    Z = std::min(Z, 128);
+    c.boxes_per_split = (c.total_boxes + Z - 1) / Z;
+    c.nsplit = (c.total_boxes + c.boxes_per_split - 1) / c.boxes_per_split;
+    return c;
+}
+
+}  // namespace
+
 static bool wgrad_tc_ok(const Level &Li, const Level &Lo, const LayerGeom &g) {
     return a_channels_ok(Li.Cpad) && Lo.Cpad % 64 == 0 && g.L.sh == g.L.sw && g.L.sh <= 2;
 }
@@ -893,6 +1062,10 @@ size_t wgrad_tc_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g) {
     for (int g0 = 0; g0 < np; g0 += TC_MAXP) {
         WgradCfg c = wgrad_cfg(Li, Lo, g, g0, std::min(np, g0 + TC_MAXP));
         best = std::max(best, (size_t)c.nsplit * g.L.cout * g.L.kh * g.L.kw * Li.Cpad * sizeof(float));
+        if (wgrad_halo_ok(Li, Lo, g)) {
+            WgHaloCfg h = wgrad_halo_cfg(Li, Lo, g, g0, std::min(np, g0 + TC_MAXP));
+            best = std::max(best, (size_t)h.nsplit * g.L.cout * g.L.kh * g.L.kw * Li.Cpad * sizeof(float));
+        }
     }
     return std::max(best, (size_t)4 * 148 * g.L.cout * sizeof(float)) + 256;  // db partials reuse the space
 }
@@ -910,8 +1083,78 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
     float *part = (float *)ws;
     static bool attr_set = false;
     bool first = true;
-    for (int g0 = p0; g0 < p1; g0 += TC_MAXP) {
-        const int g1 = std::min(p1, g0 + TC_MAXP);
+    int gend = p1;  // end of the patch range left for the generic kernel
+    if (wgrad_halo_ok(Li, Lo, g)) {
+        static bool halo_attr = false;
+        for (int g0 = p0; g0 < p1; g0 += TC_MAXP) {
+            const int g1 = std::min(p1, g0 + TC_MAXP);
+            WgHaloCfg c = wgrad_halo_cfg(Li, Lo, g, g0, g1);
+            static thread_local TcWgHaloParams P;
+            std::memset(&P, 0, sizeof(P));
+            P.npatch = g1 - g0;
+            P.BH = c.BH; P.kh = g.L.kh; P.kw = g.L.kw;
+            P.nco_blk = c.nco_blk; P.nchunk = c.nchunk; P.ntiles = c.ntiles;
+            P.boxes_per_split = c.boxes_per_split; P.nsplit = c.nsplit;
+            P.Cout = g.L.cout; P.Cpi = Li.Cpad;
+            const int Wp = 8 + g.L.kw - 1;
+            const uint32_t a_stage = 2u * c.BH * 8u * 128u;
+            const uint32_t b_stage = ((uint32_t)Wp * c.BH * 128u + 1023u) & ~1023u;
+            const uint32_t stage_bytes = a_stage + b_stage;
+            P.stages = std::min<int>(8, (int)((200u * 1024u) / stage_bytes));
+            P.tmem_cols = 256;
+            P.part = part;
+            int boxes = 0;
+            for (int q = g0; q < g1; ++q) {
+                const int ql = q - g0, i = q / Lo.nw(), j = q % Lo.nw();
+                const int ho = Lo.ph(i), wo = Lo.pw(j), hp = Li.ph(i), wp = Li.pw(j);
+                P.pt[ql] = g.pad_h[2 * i];
+                P.pl[ql] = g.pad_w[2 * j];
+                P.nhb[ql] = (ho + c.BH - 1) / c.BH;
+                P.nwb[ql] = (wo + 7) / 8;
+                P.box_prefix[ql] = boxes;
+                boxes += Lo.N * P.nhb[ql] * P.nwb[ql];
+                {
+                    const int C = Lo.Cpad;
+                    void *base = (char *)dy + Lo.offset(i, j) * 2;
+                    cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)wo, (cuuint64_t)ho, (cuuint64_t)Lo.N};
+                    cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)wo * C * 2, (cuuint64_t)ho * wo * C * 2};
+                    cuuint32_t box[4] = {64, 8, (cuuint32_t)c.BH, 1};
+                    cuuint32_t es[4] = {1, 1, 1, 1};
+                    if (encode(&P.mapDY[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides, box, es,
+                               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+                        return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(dY halo) failed");
+                }
+                {
+                    const int C = Li.Cpad;
+                    void *base = (char *)x + Li.offset(i, j) * 2;
+                    cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)wp, (cuuint64_t)hp, (cuuint64_t)Li.N};
+                    cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)wp * C * 2, (cuuint64_t)hp * wp * C * 2};
+                    cuuint32_t box[4] = {64, (cuuint32_t)Wp, (cuuint32_t)c.BH, 1};
+                    cuuint32_t es[4] = {1, 1, 1, 1};
+                    if (encode(&P.mapX[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides, box, es,
+                               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+                        return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(X halo) failed");
+                }
+            }
+            P.box_prefix[P.npatch] = boxes;
+            const size_t smem = 1024 + (size_t)P.stages * stage_bytes + 256;
+            if (!halo_attr) {
+                cudaFuncSetAttribute(wgrad_halo_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+                halo_attr = true;
+            }
+            wgrad_halo_kernel<<<c.ntiles * c.nsplit, 192, smem, st>>>(P);
+            count_launch();
+            cudaError_t e = cudaGetLastError();
+            if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("wgrad_halo_kernel: ") + cudaGetErrorString(e));
+            launch_reduce(part, c.nsplit, nW, dw, first ? beta : 1.f, st);
+            first = false;
+        }
+        gend = p0;  // done: skip the generic path below
+    }
+    for (int g0 = p0; g0 < gend; g0 += TC_MAXP) {
+        const int g1 = std::min(gend, g0 + TC_MAXP);
         WgradCfg c = wgrad_cfg(Li, Lo, g, g0, g1);
         static thread_local TcWgradParams P;
         std::memset(&P, 0, sizeof(P));

@@ -225,6 +225,42 @@ __global__ void __launch_bounds__(256) pool_bwd_kernel(LevelDesc Li, LevelDesc L
     }
 }
 
+// Backward for non-overlapping windows that tile the patch exactly (k = s, p = 0, hp = ho*s, wp = wo*s,
+// the VGG case): one thread per OUTPUT pixel x 8 channels reads dY + argmax once and writes the whole
+// k x k window (dY at the argmax, 0 elsewhere) -- every dX element written exactly once, coalesced.
+template <typename T>
+__global__ void __launch_bounds__(256) pool_bwd_scatter_kernel(LevelDesc Li, LevelDesc Lo, LayerDesc ly,
+                                                               const T *__restrict__ dY, const uint8_t *__restrict__ A,
+                                                               T *__restrict__ dX, int p0, int relu_bit) {
+    const int q = p0 + blockIdx.y;
+    const PatchGeo gi = patch_geo(Li, q), go = patch_geo(Lo, q);
+    const int G = Li.Cpad / 8;
+    const int64_t units = (int64_t)Lo.N * go.hp * go.wp * G;
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < units; u += (int64_t)gridDim.x * blockDim.x) {
+        const int cg = (int)(u % G);
+        int64_t t = u / G;
+        const int ow = (int)(t % go.wp); t /= go.wp;
+        const int oh = (int)(t % go.hp);
+        const int n = (int)(t / go.hp);
+        const int64_t o = go.off + (((int64_t)n * go.hp + oh) * go.wp + ow) * Lo.Cpad + cg * 8;
+        const uint2 a2 = __ldg(reinterpret_cast<const uint2 *>(A + o));
+        float g[8];
+        load8(dY + o, g);
+        for (int r = 0; r < ly.kh; ++r)
+            for (int c = 0; c < ly.kw; ++c) {
+                const int idx = r * ly.kw + c;
+                float v[8];
+#pragma unroll
+                for (int k = 0; k < 8; ++k) {
+                    const uint32_t b = ((k < 4 ? a2.x : a2.y) >> (8 * (k & 3))) & 0xffu;
+                    v[k] = ((int)(b & 0x7fu) == idx && (!relu_bit || (b & 0x80u))) ? g[k] : 0.f;
+                }
+                const int h = oh * ly.sh + r, w = ow * ly.sw + c;
+                store8(dX + gi.off + (((int64_t)n * gi.hp + h) * gi.wp + w) * Li.Cpad + cg * 8, v);
+            }
+    }
+}
+
 template <typename T>
 void launch_pool_fwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, void *y, uint8_t *a,
                        int relu_bit, int p0, int p1, cudaStream_t st) {
@@ -235,6 +271,18 @@ void launch_pool_fwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, con
 template <typename T>
 void launch_pool_bwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy, const uint8_t *a, void *dx,
                        int relu_bit, int p0, int p1, cudaStream_t st) {
+    bool exact = g.L.kh == g.L.sh && g.L.kw == g.L.sw;
+    for (size_t i = 0; exact && i < g.pad_h.size(); ++i) exact = g.pad_h[i] == 0;
+    for (size_t i = 0; exact && i < g.pad_w.size(); ++i) exact = g.pad_w[i] == 0;
+    for (int i = 0; exact && i < Li.nh(); ++i) exact = Li.ph(i) == Lo.ph(i) * g.L.sh;
+    for (int j = 0; exact && j < Li.nw(); ++j) exact = Li.pw(j) == Lo.pw(j) * g.L.sw;
+    if (exact) {
+        dim3 grid(grid_x_for(max_patch_units(Lo, p0, p1, Lo.Cpad / 8)), p1 - p0);
+        pool_bwd_scatter_kernel<T><<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
+                                                         (const T *)dy, a, (T *)dx, p0, relu_bit);
+        count_launch();
+        return;
+    }
     dim3 grid(grid_x_for(max_patch_units(Li, p0, p1, Li.Cpad / 8)), p1 - p0);
     { pool_bwd_kernel<T><<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
                                              (const T *)dy, a, (T *)dx, p0, relu_bit); count_launch(); }

@@ -172,7 +172,7 @@ def run_ours(args):
     # step, D2H of the step's result (all weight / bias gradients) every step
     xh = x_host.pin_memory()
     dyh = dy.cpu().pin_memory()
-    grads = [t for pair in net.grads.values() for t in pair]
+    grads = [net.grad_flat]
     gh = [torch.empty(t.shape, dtype=t.dtype, pin_memory=True) for t in grads]
     h2d = xh.numel() * xh.element_size() + dyh.numel() * dyh.element_size()
     d2h = sum(t.numel() * t.element_size() for t in grads)

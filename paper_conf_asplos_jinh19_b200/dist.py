@@ -1,0 +1,188 @@
+"""Patch-parallel Split-CNN across the GPUs of one node.
+
+Patches of a chained split region never communicate, so the region is sharded by contiguous
+PATCH ROWS: rank r owns patch range [p0, p1) and runs every region layer on it for the whole batch
+(weights replicated).  The unsplit tail runs BATCH-parallel, so at the join the region output is
+re-sharded (patch-sharded -> batch-sharded) and its gradient is sent back in backward.  The only
+reduction is the weight/bias-gradient sum (one NCCL all_reduce over one flat fp32 buffer,
+the wgrad allreduce of SURVEY 8(a) a10 / P:409-415).
+
+Join exchange without packing copies: in a patch buffer `[N][Hp][Wp][C]` the images of one batch
+shard are a CONTIGUOUS slice, and on the receiving side the same slice is a whole patch buffer of a
+plan built for the shard's batch size.  So every message is a plain view: (patch q, shard k) goes
+from the owner of q to rank k.  Messages between a pair of ranks are posted in ascending q on both
+sides, which fixes their matching order.
+"""
+from __future__ import annotations
+
+import torch
+import torch.distributed as dist
+
+from . import splitcnn as sc
+from .net import SplitNet, _out_len
+from .plan import SplitPlan
+
+
+# ------------------------------------------------------------------ pure index logic (CPU-testable)
+def patch_row_ranges(n_h: int, n_w: int, world: int):
+    """Contiguous blocks of patch rows per rank -> [(p0, p1)] in row-major patch index."""
+    if world > n_h:
+        raise ValueError(f"{world} ranks but only {n_h} patch rows to shard")
+    out = []
+    for r in range(world):
+        r0, r1 = (r * n_h) // world, ((r + 1) * n_h) // world
+        out.append((r0 * n_w, r1 * n_w))
+    return out
+
+
+def batch_ranges(N: int, world: int):
+    if N % world:
+        raise ValueError("global batch must divide across ranks")
+    b = N // world
+    return [(k * b, (k + 1) * b) for k in range(world)]
+
+
+def patch_geometry(level: dict):
+    """[(offset, elems_per_image)] of every patch buffer of a level (full batch)."""
+    N, Cp, W = level["N"], level["Cpad"], level["W"]
+    bh, bw = level["bh"], level["bw"]
+    out = []
+    for i in range(level["n_h"]):
+        hp = bh[i + 1] - bh[i]
+        for j in range(level["n_w"]):
+            wp = bw[j + 1] - bw[j]
+            out.append((N * Cp * (bh[i] * W + hp * bw[j]), hp * wp * Cp))
+    return out
+
+
+def join_messages(level_full: dict, level_shard: dict, owners, rank: int, world: int, nb: int):
+    """Messages of the forward join exchange seen from `rank`:
+    sends: (dst, patch, full-buffer offset, count); recvs: (src, patch, shard-buffer offset, count).
+    The backward exchange is the same list with the roles swapped."""
+    gf, gs = patch_geometry(level_full), patch_geometry(level_shard)
+    sends, recvs = [], []
+    for q, (off_f, per_img) in enumerate(gf):
+        owner = next(r for r, (a, b) in enumerate(owners) if a <= q < b)
+        cnt = nb * per_img
+        if owner == rank:
+            for k in range(world):
+                sends.append((k, q, off_f + k * cnt, cnt))
+        recvs.append((owner, q, gs[q][0], cnt))
+    return sends, recvs
+
+
+def exchange(src_flat: torch.Tensor, dst_flat: torch.Tensor, sends, recvs, rank: int):
+    """Post all sends / receives as tensor views (no packing); self-messages are local copies."""
+    ops = []
+    local = {}
+    for dst, q, off, cnt in sends:
+        if dst == rank:
+            local[q] = src_flat[off:off + cnt]
+        else:
+            ops.append(dist.P2POp(dist.isend, src_flat[off:off + cnt], dst))
+    for src, q, off, cnt in recvs:
+        if src == rank:
+            dst_flat[off:off + cnt].copy_(local[q])
+        else:
+            ops.append(dist.P2POp(dist.irecv, dst_flat[off:off + cnt], src))
+    if ops:
+        for w in dist.batch_isend_irecv(ops):
+            w.wait()
+
+
+def reverse(sends, recvs):
+    """Backward join exchange: every forward message travels back."""
+    rsends = [(src, q, off, cnt) for src, q, off, cnt in recvs]
+    rrecvs = [(dst, q, off, cnt) for dst, q, off, cnt in sends]
+    return rsends, rrecvs
+
+
+# ------------------------------------------------------------------ the distributed executor
+class DistSplitNet:
+    def __init__(self, c: dict, world: int, rank: int, dtype: int = sc.BF16, device="cuda"):
+        self.world, self.rank, self.dtype = world, rank, dtype
+        N, H, W = c["N"], c["H"], c["W"]
+        self.N = N
+        nb = N // world
+        self.nb = nb
+        # region: full batch, patch range of this rank
+        probe = SplitNet(c["layers"], [], 1, 3, H, W, split=c["split"], mode=c["mode"], omega=c.get("omega", 0.2),
+                         seed=c["seed"], dtype=dtype, device=device)
+        lv = probe.region.levels[0]
+        self.owners = patch_row_ranges(lv["n_h"], lv["n_w"], world)
+        del probe
+        self.region_net = SplitNet(c["layers"], [], N, 3, H, W, split=c["split"], mode=c["mode"],
+                                   omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype, device=device,
+                                   patch_range=self.owners[rank])
+        L = self.region_net.region.levels[-1]
+        self.C_join, self.H_join, self.W_join = L["C"], L["H"], L["W"]
+        tail = c["tail"]
+        last = c["layers"][-1]
+        self.tail_net = SplitNet(tail, [], nb, L["C"], L["H"], L["W"], split=(1, 1), dtype=dtype, device=device,
+                                 input_relu=last["op"] == "conv" and last.get("relu", True))
+        self.tdtype = self.region_net.tdtype
+        n_rg, n_tl = self.region_net.grad_numel(), self.tail_net.grad_numel()
+        self.grad_flat = torch.zeros(n_rg + n_tl, dtype=torch.float32, device=device)
+        self.region_net.bind_grads(self.grad_flat[:n_rg])
+        self.tail_net.bind_grads(self.grad_flat[n_rg:])
+        self._set_join_plan(0)
+        self.step_index = 0
+
+    @property
+    def timers(self):
+        return self.region_net.timers
+
+    @timers.setter
+    def timers(self, v):
+        self.region_net.timers = v
+        self.tail_net.timers = v
+
+    def _set_join_plan(self, step: int):
+        rn = self.region_net
+        Oh, Ow = rn.boundaries(step)
+        self.join_shard = SplitPlan(rn.region_layers, self.nb, 3, rn.H, rn.W, Oh, Ow)
+        self.staging = getattr(self, "staging", None)
+        n = self.join_shard.level_elems(self.join_shard.nlayers)
+        if self.staging is None or self.staging.numel() != n:
+            self.staging = torch.zeros(n, dtype=self.tdtype, device=rn.device)
+        lf = rn.region.levels[-1]
+        ls = self.join_shard.levels[-1]
+        self.msgs = join_messages(lf, ls, self.owners, self.rank, self.world, self.nb)
+
+    @property
+    def grads(self):
+        g = dict(self.region_net.grads)
+        g.update({("t", k[1]): v for k, v in self.tail_net.grads.items()})
+        return g
+
+    def set_params(self, params):
+        nr = sum(1 for l in self.region_net.region_layers if l["op"] == "conv")
+        self.region_net.set_params(params[:nr])
+        self.tail_net.set_params(params[nr:])
+
+    def output_numel(self) -> int:
+        return self.tail_net.output_numel()
+
+    def step(self, x, dy, stream=None):
+        rn, tn = self.region_net, self.tail_net
+        if rn.mode == "random":
+            rn.replan(self.step_index)
+            self._set_join_plan(self.step_index)
+        # region forward on this rank's patches (full batch)
+        rn.forward(x, stream)
+        # join: patch-sharded -> batch-sharded, merge into the tail's NHWC input
+        sends, recvs = self.msgs
+        exchange(rn.act_r[-1], self.staging, sends, recvs, self.rank)
+        Lj = self.join_shard.nlayers
+        sc.splitcnn_merge(self.join_shard.handle, Lj, self.dtype, self.staging, tn.act_r[0], sc.NHWC, 0, -1, stream)
+        tn._run_fwd("r", tn.region, tn.region_layers, tn.act_r, 0, 1, stream)
+        # tail backward (batch shard) down to the join gradient
+        g = tn.backward(dy, stream, need_input_grad=True)
+        sc.splitcnn_split(self.join_shard.handle, Lj, self.dtype, g, sc.NHWC, self.staging, 0, -1, stream)
+        rs, rr = reverse(sends, recvs)
+        g_region = rn.grad[0]
+        exchange(self.staging, g_region, rs, rr, self.rank)
+        rn.backward(g_region, stream)
+        # the wgrad allreduce (sum over ranks of the per-rank partial sums)
+        dist.all_reduce(self.grad_flat, op=dist.ReduceOp.SUM)
+        self.step_index += 1

@@ -32,12 +32,14 @@ def unpack_grad(dW: torch.Tensor, cin: int) -> torch.Tensor:
 class SplitNet:
     def __init__(self, region: list[dict], tail: list[dict], N: int, C: int, H: int, W: int,
                  split=(2, 2), mode: str = "even", omega: float = 0.2, seed: int = 0,
-                 dtype: int = sc.BF16, device="cuda", patch_range=None, force_simt: bool = False):
+                 dtype: int = sc.BF16, device="cuda", patch_range=None, force_simt: bool = False,
+                 grad_buffer: torch.Tensor | None = None, input_relu: bool = False):
         self.region_layers, self.tail_layers = region, tail
         self.N, self.C, self.H, self.W = N, C, H, W
         self.split, self.mode, self.omega, self.seed = split, mode, omega, seed
         self.dtype, self.tdtype, self.device = dtype, TORCH_DTYPE[dtype], torch.device(device)
         self.flags_extra = sc.FLAG_FORCE_SIMT if force_simt else 0
+        self.input_relu = input_relu   # level 0 is a ReLU output (e.g. a tail fed by a ReLU conv)
         self.step_index = 0
         self.timers = None       # list -> every library call is bracketed by CUDA events (bench.py)
         self._label = ""
@@ -46,7 +48,7 @@ class SplitNet:
         L = self.region.levels[-1]
         self.tail = SplitPlan(tail, N, L["C"], L["H"], L["W"], [0, _out_len(tail, L["H"], 0)],
                               [0, _out_len(tail, L["W"], 1)]) if tail else None
-        self._alloc()
+        self._alloc(grad_buffer)
 
     # ------------------------------------------------------------------ planning
     def _region_output_hw(self):
@@ -79,7 +81,16 @@ class SplitNet:
             st += [(self.tail, m, l) for m, l in enumerate(self.tail_layers)]
         return st
 
-    def _alloc(self):
+    def grad_numel(self) -> int:
+        """fp32 elements of all weight + bias gradients (for a caller-provided flat buffer)."""
+        n = 0
+        for layers, plan in ((self.region_layers, self.region), (self.tail_layers, self.tail)):
+            for m, l in enumerate(layers):
+                if l["op"] == "conv":
+                    n += l["cout"] * l["kh"] * l["kw"] * plan.levels[m]["Cpad"] + l["cout"]
+        return n
+
+    def _alloc(self, grad_buffer=None):
         dev, td = self.device, self.tdtype
         self.act_r = [torch.zeros(self.region.level_elems(m), dtype=td, device=dev)
                       for m in range(self.region.nlayers + 1)]
@@ -103,16 +114,30 @@ class SplitNet:
                     ws = max(ws, plan.workspace_size(m, self.dtype, 1), plan.workspace_size(m, self.dtype, 2))
         self.ws = torch.zeros(max(ws, 16) // 4 + 4, dtype=torch.float32, device=dev)
         self.ws_bytes = self.ws.numel() * 4
-        self.params, self.grads = {}, {}
+        self.params = {}
         for key, layers, plan in (("r", self.region_layers, self.region), ("t", self.tail_layers, self.tail)):
             for m, l in enumerate(layers):
                 if l["op"] == "conv":
                     cpad = plan.levels[m]["Cpad"]
                     self.params[(key, m)] = (torch.zeros((l["cout"], l["kh"], l["kw"], cpad), dtype=td, device=dev),
                                              torch.zeros(l["cout"], dtype=torch.float32, device=dev))
-                    self.grads[(key, m)] = (torch.zeros((l["cout"], l["kh"], l["kw"], cpad), dtype=torch.float32,
-                                                        device=dev),
-                                            torch.zeros(l["cout"], dtype=torch.float32, device=dev))
+        self.bind_grads(grad_buffer if grad_buffer is not None else
+                        torch.zeros(self.grad_numel(), dtype=torch.float32, device=dev))
+
+    def bind_grads(self, flat: torch.Tensor):
+        """All weight / bias gradients become views of one flat fp32 buffer (one allreduce per step)."""
+        self.grad_flat = flat
+        self.grads = {}
+        off = 0
+        for key, layers, plan in (("r", self.region_layers, self.region), ("t", self.tail_layers, self.tail)):
+            for m, l in enumerate(layers):
+                if l["op"] == "conv":
+                    cpad = plan.levels[m]["Cpad"]
+                    nw = l["cout"] * l["kh"] * l["kw"] * cpad
+                    dW = flat[off:off + nw].view(l["cout"], l["kh"], l["kw"], cpad)
+                    db = flat[off + nw:off + nw + l["cout"]]
+                    off += nw + l["cout"]
+                    self.grads[(key, m)] = (dW, db)
 
     def set_params(self, params):
         """params: list (region + tail order, convs only) of (W_oihw, b) torch/numpy arrays."""
@@ -150,18 +175,20 @@ class SplitNet:
     def _masked(self, key: str, m: int) -> bool:
         """Level m is the output of a conv with fused ReLU -> its gradient producer applies the mask."""
         if key == "r":
-            return m > 0 and self.region_layers[m - 1]["op"] == "conv" and self.region_layers[m - 1].get("relu", True)
+            if m == 0:
+                return self.input_relu
+            return self.region_layers[m - 1]["op"] == "conv" and self.region_layers[m - 1].get("relu", True)
         if m > 0:
             return self.tail_layers[m - 1]["op"] == "conv" and self.tail_layers[m - 1].get("relu", True)
         return self._masked("r", len(self.region_layers))
 
     # ------------------------------------------------------------------ passes
-    def forward(self, x: torch.Tensor, stream=None):
-        """x: full NCHW tensor (dtype) on the device.  Returns the output level buffer."""
+    def forward(self, x: torch.Tensor, stream=None, x_layout: int = sc.NCHW):
+        """x: full tensor (dtype) on the device, NCHW or NHWC.  Returns the output level buffer."""
         p0, p1 = self.patch_range
         R, dt, fl = self.region.handle, self.dtype, self.flags_extra
         b_in = 2 * self._bytes(self.region, 0)[0]
-        self._call("split", b_in, sc.splitcnn_split, R, 0, dt, x, sc.NCHW, self.act_r[0], p0, p1, stream)
+        self._call("split", b_in, sc.splitcnn_split, R, 0, dt, x, x_layout, self.act_r[0], p0, p1, stream)
         self._run_fwd("r", self.region, self.region_layers, self.act_r, p0, p1, stream)
         if self.tail:
             b_j = 2 * self._bytes(self.region, self.region.nlayers - 1)[1]

@@ -117,3 +117,31 @@ def test_c4_stochastic_stack_small(sc):
         assert max(errs.values()) <= 1e-4, errs
         errs = _run(sc, "C4", 1, sc.BF16, H=64, step=step)
         assert errs["out"] <= 2e-2 and errs["argmax_flip_frac"] < 1e-2, errs
+
+
+def test_dist_executor_world1_matches_single(sc):
+    """DistSplitNet (patch-row sharded region + join re-shard + batch-sharded tail + allreduce) at
+    world size 1 must reproduce SplitNet exactly (same kernels, same order)."""
+    import os
+    import torch.distributed as dist
+    from paper_conf_asplos_jinh19_b200.dist import DistSplitNet
+    from paper_conf_asplos_jinh19_b200.net import SplitNet
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    os.environ.setdefault("MASTER_PORT", "29533")
+    if not dist.is_initialized():
+        dist.init_process_group("nccl", rank=0, world_size=1)
+    c = synth.vgg_config("C5", N=2)
+    g = synth.rng(4)
+    params = [p for p in synth.layer_params(g, c["layers"] + c["tail"]) if p is not None]
+    tp = [(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params]
+    x = torch.from_numpy(synth.uniform(g, (2, 3, 224, 224))).to("cuda", torch.bfloat16)
+    single = SplitNet(c["layers"], c["tail"], 2, 3, 224, 224, split=c["split"], mode=c["mode"], seed=c["seed"])
+    single.set_params(tp)
+    dnet = DistSplitNet(c, 1, 0)
+    dnet.set_params(tp)
+    dy = torch.randn(single.output_numel(), generator=torch.Generator().manual_seed(0)).to("cuda", torch.bfloat16)
+    assert dnet.output_numel() == single.output_numel()
+    single.step(x, dy)
+    dnet.step(x, dy)
+    torch.cuda.synchronize()
+    assert torch.equal(single.grad_flat, dnet.grad_flat)

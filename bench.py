@@ -110,9 +110,15 @@ def run_ours(args):
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     c = workload(args.config)
     dtype = sc.BF16 if args.dtype == "bf16" else sc.FP32
+    use_offload = args.offload if args.offload is not None else (args.config == "C4")
     if world > 1:
         from paper_conf_asplos_jinh19_b200.dist import DistSplitNet
         net = DistSplitNet(c, world, rank, dtype)
+        use_offload = False
+    elif use_offload:
+        from paper_conf_asplos_jinh19_b200.offload import OffloadSplitNet
+        net = OffloadSplitNet(c["layers"], c["tail"], c["N"], 3, c["H"], c["W"], split=c["split"], mode=c["mode"],
+                              omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype)
     else:
         net = SplitNet(c["layers"], c["tail"], c["N"], 3, c["H"], c["W"], split=c["split"], mode=c["mode"],
                        omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype)
@@ -134,6 +140,34 @@ def run_ours(args):
     for _ in range(args.warmup):
         step()
     barrier()
+    offload_info = None
+    if use_offload:
+        # without offload first (same net, offload disabled): the degradation reference
+        net.offload_enabled = False
+        torch.cuda.reset_peak_memory_stats()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        barrier()
+        e0.record(stream)
+        for _ in range(args.steps):
+            step()
+        e1.record(stream)
+        barrier()
+        ms_plain = e0.elapsed_time(e1) / args.steps
+        peak_plain = torch.cuda.max_memory_allocated()
+        stats = net.profile_and_plan(x, dy, reps=20)
+        net.offload_enabled = True
+        for _ in range(2):
+            step()
+        barrier()
+        torch.cuda.reset_peak_memory_stats()
+        offload_info = {"plan": "Algorithm 1 + reverse pass (splitcnn_offload_plan / _prefetch_plan)",
+                        "host_link_gbs": round(stats["bw_bytes_per_s"] / 1e9, 1),
+                        "offloaded_levels": stats["offloaded_levels"],
+                        "offloaded_gb": round(stats["offloaded_bytes"] / 1e9, 3),
+                        "candidate_gb": round(stats["candidate_bytes"] / 1e9, 3),
+                        "cap_gb": round(stats["cap_bytes"] / 1e9, 3),
+                        "no_offload_ms_per_step": round(ms_plain, 3),
+                        "no_offload_peak_gb": round(peak_plain / 1e9, 2)}
     launches0 = sc.splitcnn_kernel_launches()
     clocks = ClockSampler(local)
     clocks.start()
@@ -166,6 +200,9 @@ def run_ours(args):
     net.timers = None
     ms_step = ms / args.steps
     global_batch = c["N"]
+    if offload_info is not None:
+        offload_info["offload_peak_gb"] = round(torch.cuda.max_memory_allocated() / 1e9, 2)
+        offload_info["degradation_pct"] = round(100 * (ms_step / offload_info["no_offload_ms_per_step"] - 1), 2)
     value = global_batch / (ms_step / 1e3)
 
     # e2e: the same step through the public API with host buffers: pinned H2D of x and dY every
@@ -233,6 +270,8 @@ def run_ours(args):
         "per_kind_ms_per_step": {k: round(v[0] / args.steps, 4) for k, v in kinds.items()},
         "clocks": clk,
     }
+    if offload_info is not None:
+        line["offload"] = offload_info
     if args.per_layer:
         line["per_layer"] = {k: {"ms": round(v[0] / args.steps, 4),
                                  "tflops" if ":conv" in k else "gbs": round(v[1] / (v[0] / 1e3) / (1e12 if ":conv" in k else 1e9), 1)}
@@ -346,6 +385,8 @@ def main():
     ap.add_argument("--cpu-tiles", type=int, default=12)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--per-layer", action="store_true")
+    ap.add_argument("--offload", dest="offload", action="store_true", default=None)
+    ap.add_argument("--no-offload", dest="offload", action="store_false")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

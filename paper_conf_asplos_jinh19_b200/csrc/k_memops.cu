@@ -3,6 +3,8 @@
 //   merge  (Eq. 7)  patch buffers -> full tensor
 //   max-pool forward / backward per patch (Eq. 6 with Op = max-pool)
 // One thread moves 8 channels (16 B in bf16) of one pixel; grid.y enumerates patches.
+#include <algorithm>
+
 #include "common.cuh"
 #include "kernels.h"
 
@@ -88,9 +90,13 @@ __global__ void __launch_bounds__(256) merge_kernel(LevelDesc L, const T *__rest
     }
 }
 
+// HBM-bound kernels: about 16 resident 256-thread blocks per SM over the whole launch (grid.y =
+// patches), each thread striding over several 8-channel units -- not one short-lived block per 256 units
+static int npatch_launch = 1;
 static int grid_x_for(int64_t units) {
     int64_t b = (units + 255) / 256;
-    return (int)(b < 4096 ? (b < 1 ? 1 : b) : 4096);
+    const int64_t cap = std::max<int64_t>(1, (148 * 16 + npatch_launch - 1) / npatch_launch);
+    return (int)std::max<int64_t>(1, std::min(b, cap));
 }
 
 static int64_t max_patch_units(const Level &L, int p0, int p1, int per_pixel) {
@@ -105,6 +111,7 @@ static int64_t max_patch_units(const Level &L, int p0, int p1, int per_pixel) {
 
 template <typename T>
 void launch_split_t(const Level &L, const void *x, int layout, void *P, int p0, int p1, cudaStream_t st) {
+    npatch_launch = p1 - p0;
     dim3 grid(grid_x_for(max_patch_units(L, p0, p1, L.Cpad / 8)), p1 - p0);
     LevelDesc d = make_level_desc(L);
     if (layout == SPLITCNN_NCHW)
@@ -115,6 +122,7 @@ void launch_split_t(const Level &L, const void *x, int layout, void *P, int p0, 
 
 template <typename T>
 void launch_merge_t(const Level &L, const void *P, void *y, int layout, int p0, int p1, cudaStream_t st) {
+    npatch_launch = p1 - p0;
     dim3 grid(grid_x_for(max_patch_units(L, p0, p1, L.Cpad / 8)), p1 - p0);
     LevelDesc d = make_level_desc(L);
     if (layout == SPLITCNN_NCHW)
@@ -264,6 +272,7 @@ __global__ void __launch_bounds__(256) pool_bwd_scatter_kernel(LevelDesc Li, Lev
 template <typename T>
 void launch_pool_fwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, void *y, uint8_t *a,
                        int relu_bit, int p0, int p1, cudaStream_t st) {
+    npatch_launch = p1 - p0;
     dim3 grid(grid_x_for(max_patch_units(Lo, p0, p1, Lo.Cpad / 8)), p1 - p0);
     { pool_fwd_kernel<T><<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
                                              (const T *)x, (T *)y, a, p0, relu_bit); count_launch(); }
@@ -277,12 +286,14 @@ void launch_pool_bwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, con
     for (int i = 0; exact && i < Li.nh(); ++i) exact = Li.ph(i) == Lo.ph(i) * g.L.sh;
     for (int j = 0; exact && j < Li.nw(); ++j) exact = Li.pw(j) == Lo.pw(j) * g.L.sw;
     if (exact) {
+        npatch_launch = p1 - p0;
         dim3 grid(grid_x_for(max_patch_units(Lo, p0, p1, Lo.Cpad / 8)), p1 - p0);
         pool_bwd_scatter_kernel<T><<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
                                                          (const T *)dy, a, (T *)dx, p0, relu_bit);
         count_launch();
         return;
     }
+    npatch_launch = p1 - p0;
     dim3 grid(grid_x_for(max_patch_units(Li, p0, p1, Li.Cpad / 8)), p1 - p0);
     { pool_bwd_kernel<T><<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
                                              (const T *)dy, a, (T *)dx, p0, relu_bit); count_launch(); }

@@ -198,9 +198,23 @@ class SplitNet:
             return self.act_t[-1]
         return self.act_r[-1]
 
+    # hooks (no-ops here; the offload executor overrides them)
+    def hook_before_fwd(self, key, m):
+        pass
+
+    def hook_after_fwd(self, key, m):
+        pass
+
+    def hook_before_bwd(self, key, m):
+        pass
+
+    def hook_after_bwd(self, key, m):
+        pass
+
     def _run_fwd(self, key, plan, layers, acts, p0, p1, stream):
         for m, l in enumerate(layers):
             self._label = l.get("name", f"{key}{m}")
+            self.hook_before_fwd(key, m)
             if l["op"] == "conv":
                 W, b = self.params[(key, m)]
                 flags = (sc.FLAG_RELU if l.get("relu", True) else 0) | self.flags_extra
@@ -212,6 +226,7 @@ class SplitNet:
                 work = bi + bo + bo // (2 if self.dtype == sc.BF16 else 4)
                 self._call("pool_fwd", work, sc.splitcnn_pool_fwd, plan.handle, m, self.dtype, acts[m], acts[m + 1],
                            self.argmax[(key, m)], flags, p0, p1, stream)
+            self.hook_after_fwd(key, m)
 
     def backward(self, dy: torch.Tensor, stream=None, need_input_grad: bool = False):
         """dy: gradient w.r.t. the output level buffer (same layout).  Fills self.grads."""
@@ -230,6 +245,7 @@ class SplitNet:
         for m in range(len(layers) - 1, -1, -1):
             l = layers[m]
             self._label = l.get("name", f"{key}{m}")
+            self.hook_before_bwd(key, m)
             out = self.grad[0] if g is not self.grad[0] else self.grad[1]
             last = (m == 0 and not need_input_grad)
             if l["op"] == "conv":
@@ -250,6 +266,7 @@ class SplitNet:
                            self.argmax[(key, m)], out, flags, p0, p1, stream)
             if not last:
                 g = out
+            self.hook_after_bwd(key, m)
         return g
 
     def step(self, x, dy, stream=None):

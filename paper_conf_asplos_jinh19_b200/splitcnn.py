@@ -258,9 +258,16 @@ def splitcnn_pool_bwd(plan, layer, dtype, dy, argmax, dx, flags=0, p0=0, p1=-1, 
 
 
 def _ev(e):
+    """cudaEvent_t of an int handle or a torch.cuda.Event.  torch creates the CUDA event lazily at the
+    first record(); an unrecorded torch event would be a NULL handle, so it is refused here."""
     if e is None:
         return None
-    return e if isinstance(e, int) else e.cuda_event
+    if isinstance(e, int):
+        return e
+    h = e.cuda_event
+    if not h:
+        raise ValueError("torch.cuda.Event has no CUDA handle yet (record it once before passing it)")
+    return h
 
 
 def splitcnn_offload(plan, level, dtype, patch, dev_patches, host_pinned, ready=None, mem_stream=None, done=None):

@@ -256,6 +256,7 @@ def test_offload_prefetch_roundtrip_bit_exact(sc):
         off, nb = sc.splitcnn_patch_bytes(pl.handle, 0, dtype, q)
         h = torch.empty(nb, dtype=torch.uint8, pin_memory=True)
         done = torch.cuda.Event()
+        done.record(mem)                       # creates the CUDA handle; the library re-records it
         sc.splitcnn_offload(pl.handle, 0, dtype, q, x, h, ready, mem, done)
         hosts.append((h, done))
     for _, d in hosts:
@@ -264,6 +265,7 @@ def test_offload_prefetch_roundtrip_bit_exact(sc):
     ready.record()
     for q, (h, _) in enumerate(hosts):
         d = torch.cuda.Event()
+        d.record(mem)
         sc.splitcnn_prefetch(pl.handle, 0, dtype, q, h, x, ready, mem, d)
         torch.cuda.current_stream().wait_event(d)
     torch.cuda.synchronize()

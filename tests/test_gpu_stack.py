@@ -145,3 +145,33 @@ def test_dist_executor_world1_matches_single(sc):
     dnet.step(x, dy)
     torch.cuda.synchronize()
     assert torch.equal(single.grad_flat, dnet.grad_flat)
+
+
+@pytest.mark.parametrize("bw", [1e15, 2e9])
+def test_offload_prefetch_executor_bitwise(sc, bw):
+    """Offload/prefetch driven by Algorithm 1 must not change a single bit of the
+    step's results; with an unbounded link every candidate is offloaded, with a slow one only what
+    the ratio cap allows.  Device memory of freed levels is returned to the allocator."""
+    from paper_conf_asplos_jinh19_b200.net import SplitNet
+    from paper_conf_asplos_jinh19_b200.offload import OffloadSplitNet
+    c = synth.vgg_config("C4", N=2)
+    H = 64
+    g = synth.rng(3)
+    params = [p for p in synth.layer_params(g, c["layers"] + c["tail"]) if p is not None]
+    tp = [(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params]
+    x = torch.from_numpy(synth.uniform(g, (2, 3, H, H))).to("cuda", torch.bfloat16)
+    kw = dict(split=c["split"], mode=c["mode"], omega=c["omega"], seed=c["seed"])
+    plain = SplitNet(c["layers"], c["tail"], 2, 3, H, H, **kw)
+    off = OffloadSplitNet(c["layers"], c["tail"], 2, 3, H, H, **kw)
+    plain.set_params(tp)
+    off.set_params(tp)
+    dy = torch.randn(plain.output_numel(), generator=torch.Generator().manual_seed(1)).to("cuda", torch.bfloat16)
+    stats = off.profile_and_plan(x, dy, reps=2, bw=bw)
+    assert stats["offloaded_bytes"] <= stats["cap_bytes"] + 1
+    if bw > 1e12:
+        assert stats["offloaded_bytes"] == stats["candidate_bytes"] > 0
+    for step in range(2):
+        plain.step(x, dy)
+        off.step(x, dy)
+        torch.cuda.synchronize()
+        assert torch.equal(plain.grad_flat, off.grad_flat)

@@ -19,6 +19,7 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <vector>
@@ -53,6 +54,10 @@ struct TcConvParams {
     int ksteps;      // K steps per tile
     int kchan;       // Cpad of the A side (K = taps * kchan)
     int a3d;         // 8-channel A: 3-D maps with pixels merged into 128-byte-wide rows (coordinate 8*w)
+    int halo;        // stride-1 halo mode: one A box per (channel chunk, kernel row) serves the kw column taps
+    int b3d;         // halo: the kw taps' weights arrive as one 3-D box
+    int Wp;          // halo: input box width = 8 + kw - 1
+    uint32_t a_stage;  // bytes per A stage (1024-aligned)
     int BN, Cout, Cpo;
     int stages;
     uint32_t tmem_cols;
@@ -130,9 +135,9 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
     extern __shared__ uint8_t smem_raw[];
     uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     const int S = p.stages;
-    const uint32_t b_stage = (uint32_t)p.BN * 128u;
+    const uint32_t b_stage = p.b_tx_bytes;   // BN x 128 B per tap box (kw boxes in halo mode)
     uint8_t *sA = smem;
-    uint8_t *sB = smem + (size_t)S * 16384;
+    uint8_t *sB = smem + (size_t)S * p.a_stage;
     uint8_t *sY = smem + p.stage_off;  // output staging tile (1024-aligned)
     uint64_t *full = (uint64_t *)(smem + p.bar_off);
     uint64_t *empty = full + S;
@@ -181,9 +186,18 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 for (int ks = 0; ks < p.ksteps; ++ks) {
                     tc::mbar_wait_sleep(&empty[stage], ph ^ 1);
                     tc::mbar_arrive_expect_tx(&full[stage], p.a_tx_bytes + p.b_tx_bytes);
-                    uint8_t *a = sA + (size_t)stage * 16384;
+                    uint8_t *a = sA + (size_t)stage * p.a_stage;
                     uint8_t *b = sB + (size_t)stage * b_stage;
-                    if (p.tps > 1) {
+                    if (p.halo) {
+                        const int cc = ks / p.kh, r = ks - cc * p.kh;
+                        tc::tma_load_4d(a, &p.mapA[ql], &full[stage], cc * 64, wbase, hbase + r, n0);
+                        if (p.b3d) {
+                            tc::tma_load_3d(b, &p.mapB, &full[stage], cc * 64, co0, r * p.kw);
+                        } else {
+                            for (int c = 0; c < p.kw; ++c)
+                                tc::tma_load_2d(b + c * p.BN * 128, &p.mapB, &full[stage], (r * p.kw + c) * p.kchan + cc * 64, co0);
+                        }
+                    } else if (p.tps > 1) {
                         for (int j = 0; j < p.tps; ++j) {
                             const int tap = min(ks * p.tps + j, KT - 1);  // past the last tap: weights are OOB zero
                             const int r = tap / p.kw, c = tap - r * p.kw;
@@ -216,8 +230,22 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 for (int ks = 0; ks < p.ksteps; ++ks) {
                     tc::mbar_wait(&full[stage], ph);
                     tc::tc_fence_after();
-                    const uint32_t a_base = tc::smem_u32(sA + (size_t)stage * 16384);
+                    const uint32_t a_base = tc::smem_u32(sA + (size_t)stage * p.a_stage);
                     const uint32_t b_base = tc::smem_u32(sB + (size_t)stage * b_stage);
+                    if (p.halo) {
+                        // tap c of this kernel row = the A tile viewed c pixel-rows further on (SW128 is
+                        // address-based, probed); 8-pixel M groups are Wp rows apart (SBO = Wp * 128 B)
+                        for (int c = 0; c < p.kw; ++c)
+#pragma unroll
+                            for (int j = 0; j < 4; ++j) {
+                                const uint64_t adesc = tc::smem_desc(a_base + 128u * c + 32u * j, 16, (uint32_t)p.Wp * 128u, 2);
+                                const uint64_t bdesc = tc::smem_desc(b_base + (uint32_t)(c * p.BN) * 128u + 32u * j, 16, 1024, 2);
+                                tc::mma_bf16(d, adesc, bdesc, idesc, (ks | c | j) != 0);
+                            }
+                        tc::mma_commit(&empty[stage]);
+                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        continue;
+                    }
 #pragma unroll
                     for (int j = 0; j < 4; ++j) {
                         const int k0 = 16 * j;
@@ -480,7 +508,18 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             ext.push_back({Lout.ph(i), Lout.pw(j)});
         }
         const int a3d = (cpad == 8 && s == 1) ? 1 : 0;  // TMA rows of 16 B are slow: merge 8 pixels per row
-        const TileShape ts = choose_tile(ext, N, s, a3d ? 32 : 128);
+        // halo mode for narrow outputs (per-tap TMA boxes cannot keep the MMA fed there)
+        const int halo = (s == 1 && cpad % 64 == 0 && BN <= 128 && kw >= 2 && kw <= 4 && !getenv("SPLITCNN_NO_HALO")) ? 1 : 0;
+        TileShape ts = choose_tile(ext, N, s, a3d ? 32 : 128);
+        if (halo) {  // 8 output columns per M group; BH x BNn groups (<= 16)
+            long best = -1;
+            for (int bh = 1; bh <= 16; ++bh)
+                for (int bn = 1; bh * bn <= 16 && bn <= N; ++bn) {
+                    long t = 0;
+                    for (auto &e : ext) t += (long)((N + bn - 1) / bn) * ((e.first + bh - 1) / bh) * ((e.second + 7) / 8);
+                    if (best < 0 || t < best || (t == best && bh * bn > ts.BH * ts.BNn)) { best = t; ts = {8, bh, bn}; }
+                }
+        }
         static thread_local TcConvParams P;  // large; avoid the stack
         std::memset(&P, 0, sizeof(P));
         P.npatch = g1 - g0;
@@ -491,6 +530,8 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.cpadc = cpadc;
         P.kchan = cpad;
         P.a3d = a3d;
+        P.halo = halo;
+        P.Wp = 8 + kw - 1;
         if (cpad >= 64) {
             P.cchunks = cpad / 64; P.tps = 1; P.ksteps = kh * kw * P.cchunks;
         } else {
@@ -504,7 +545,14 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.a_lbo = row_bytes == 16 ? P.a_chunk_bytes : 16u;
         P.a_tx_bytes = (uint32_t)P.tps * P.rows_box * row_bytes;
         P.b_tx_bytes = (uint32_t)BN * 128u;
-        const uint32_t stage_bytes = 16384u + P.b_tx_bytes;
+        P.a_stage = 16384u;
+        if (halo) {
+            P.ksteps = (cpad / 64) * kh;
+            P.a_tx_bytes = (uint32_t)P.Wp * ts.BH * ts.BNn * 128u;
+            P.a_stage = (P.a_tx_bytes + 1023u) & ~1023u;
+            P.b_tx_bytes = (uint32_t)kw * BN * 128u;
+        }
+        const uint32_t stage_bytes = P.a_stage + P.b_tx_bytes;
         // output staging for the TMA-store epilogue: channel box of min(64, Cpo), swizzle to match
         const int ych = std::min(64, Lout.Cpad);
         P.direct = !((ych == 8 || ych == 16 || ych == 32 || ych == 64) && Lout.Cpad % ych == 0);
@@ -542,6 +590,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             cuuint64_t strides[3] = {(cuuint64_t)cpad * 2, (cuuint64_t)wp * cpad * 2, (cuuint64_t)hp * wp * cpad * 2};
             cuuint32_t box[4] = {(cuuint32_t)cpadc, (cuuint32_t)(ts.BW * s), (cuuint32_t)(ts.BH * s), (cuuint32_t)ts.BNn};
             cuuint32_t es[4] = {1, (cuuint32_t)s, (cuuint32_t)s, 1};
+            if (halo) box[1] = (cuuint32_t)P.Wp;
             CUresult r;
             if (a3d) {
                 cuuint64_t d3[3] = {(cuuint64_t)wp * 8, (cuuint64_t)hp, (cuuint64_t)N};
@@ -587,9 +636,22 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             cuuint64_t strides[1] = {(cuuint64_t)K * 2};
             cuuint32_t box[2] = {64, (cuuint32_t)BN};
             cuuint32_t es[2] = {1, 1};
-            CUresult r = encode(&P.mapB, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(w_ptr), dims, strides, box,
-                                es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
-                                CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+            CUresult r = CUDA_ERROR_INVALID_VALUE;
+            P.b3d = 0;
+            if (halo) {  // (ci, co, tap) view of [Cout][taps][Cpad]: one box = the kw taps of a kernel row
+                cuuint64_t d3[3] = {(cuuint64_t)cpad, (cuuint64_t)w_rows, (cuuint64_t)(kh * kw)};
+                cuuint64_t s3[2] = {(cuuint64_t)K * 2, (cuuint64_t)cpad * 2};
+                cuuint32_t b3[3] = {64, (cuuint32_t)BN, (cuuint32_t)kw};
+                cuuint32_t e3[3] = {1, 1, 1};
+                r = encode(&P.mapB, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void *>(w_ptr), d3, s3, b3, e3,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                P.b3d = r == CUDA_SUCCESS;
+            }
+            if (r != CUDA_SUCCESS)
+                r = encode(&P.mapB, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(w_ptr), dims, strides, box, es,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
             if (r != CUDA_SUCCESS) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(B) failed");
         }
         if (tiles == 0) continue;
@@ -848,7 +910,7 @@ struct TcWgHaloParams {
     int box_prefix[TC_MAXP + 1];
     int pt[TC_MAXP], pl[TC_MAXP];
     int nhb[TC_MAXP], nwb[TC_MAXP];
-    int npatch, BH, kh, kw;
+    int npatch, BH, BNn, kh, kw;
     int nco_blk, nchunk, ntiles, boxes_per_split, nsplit;
     int Cout, Cpi, stages;
     uint32_t tmem_cols;
@@ -859,11 +921,13 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
     extern __shared__ uint8_t smem_raw[];
     uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     const int S = p.stages;
-    const int rows = p.BH * 8;                        // pixels per stage
+    // pixels per stage: BNn images x BH output rows x 8 output columns; for a FIXED kernel row r the X
+    // box has exactly BH rows per image, so the K groups (n, h) stay Wp rows apart across images too
+    const int rows = p.BNn * p.BH * 8;
     const int Wp = 8 + p.kw - 1;
     const uint32_t a_blk = (uint32_t)rows * 128u;     // one 64-channel dY block
     const uint32_t a_stage = 2u * a_blk;
-    const uint32_t b_stage = ((uint32_t)Wp * p.BH * 128u + 1023u) & ~1023u;
+    const uint32_t b_stage = ((uint32_t)Wp * p.BH * p.BNn * 128u + 1023u) & ~1023u;
     uint8_t *sA = smem;
     uint8_t *sB = smem + (size_t)S * a_stage;
     uint64_t *full = (uint64_t *)(sB + (size_t)S * b_stage);
@@ -897,13 +961,13 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
         if (lane == 0) {
             int stage = 0, ql = 0;
             uint32_t ph = 0;
-            const uint32_t tx = a_stage + (uint32_t)Wp * p.BH * 128u;
+            const uint32_t tx = a_stage + (uint32_t)Wp * p.BH * p.BNn * 128u;
             for (int b = b0; b < b1; ++b) {
                 while (b >= p.box_prefix[ql + 1]) ++ql;
                 int idx = b - p.box_prefix[ql];
                 const int wb = idx % p.nwb[ql];
                 idx /= p.nwb[ql];
-                const int hb = idx % p.nhb[ql], n = idx / p.nhb[ql];
+                const int hb = idx % p.nhb[ql], n = (idx / p.nhb[ql]) * p.BNn;
                 const int ow0 = wb * 8, oh0 = hb * p.BH;
                 tc::mbar_wait_sleep(&empty[stage], ph ^ 1);
                 tc::mbar_arrive_expect_tx(&full[stage], tx);
@@ -1020,7 +1084,7 @@ WgradCfg wgrad_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, int p0,
 namespace {
 
 struct WgHaloCfg {
-    int BH, nco_blk, nchunk, ntiles, total_boxes, nsplit, boxes_per_split;
+    int BH, BNn, nco_blk, nchunk, ntiles, total_boxes, nsplit, boxes_per_split;
 };
 
 bool wgrad_halo_ok(const Level &Li, const Level &Lo, const LayerGeom &g) {
@@ -1030,14 +1094,19 @@ bool wgrad_halo_ok(const Level &Li, const Level &Lo, const LayerGeom &g) {
 WgHaloCfg wgrad_halo_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, int p0, int p1) {
     WgHaloCfg c{};
     long best = -1;
-    for (int bh : {16, 8}) {
-        long n = 0;
-        for (int q = p0; q < p1; ++q)
-            n += (long)Lo.N * ((Lo.ph(q / Lo.nw()) + bh - 1) / bh) * ((Lo.pw(q % Lo.nw()) + 7) / 8);
-        // cost ~ boxes x (fixed per-box cost + pixels): prefer fewer, larger boxes unless they waste rows
-        const long cost = n * (bh * 8 + 192);
-        if (best < 0 || cost < best) { best = cost; c.BH = bh; c.total_boxes = (int)n; }
-    }
+    int maxh = 1;
+    for (int q = p0; q < p1; ++q) maxh = std::max(maxh, Lo.ph(q / Lo.nw()));
+    // BH x BNn x 8 pixels per stage (<= 128, a multiple of 16 for the K = 16 MMA steps)
+    for (int bh = 1; bh <= std::min(16, maxh); ++bh)
+        for (int bn = 1; bn * bh * 8 <= 128 && bn <= Lo.N; ++bn) {
+            if ((bh * bn) % 2) continue;
+            long n = 0;
+            for (int q = p0; q < p1; ++q)
+                n += (long)((Lo.N + bn - 1) / bn) * ((Lo.ph(q / Lo.nw()) + bh - 1) / bh) * ((Lo.pw(q % Lo.nw()) + 7) / 8);
+            // cost ~ boxes x (fixed per-box cost + MMA rows): fewer, fuller boxes win
+            const long cost = n * (bh * bn * 8 + 256);
+            if (best < 0 || cost < best) { best = cost; c.BH = bh; c.BNn = bn; c.total_boxes = (int)n; }
+        }
     c.nco_blk = (g.L.cout + 127) / 128;
     c.nchunk = Li.Cpad / 64;
     c.ntiles = c.nco_blk * g.L.kh * c.nchunk;
@@ -1092,13 +1161,13 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
             static thread_local TcWgHaloParams P;
             std::memset(&P, 0, sizeof(P));
             P.npatch = g1 - g0;
-            P.BH = c.BH; P.kh = g.L.kh; P.kw = g.L.kw;
+            P.BH = c.BH; P.BNn = c.BNn; P.kh = g.L.kh; P.kw = g.L.kw;
             P.nco_blk = c.nco_blk; P.nchunk = c.nchunk; P.ntiles = c.ntiles;
             P.boxes_per_split = c.boxes_per_split; P.nsplit = c.nsplit;
             P.Cout = g.L.cout; P.Cpi = Li.Cpad;
             const int Wp = 8 + g.L.kw - 1;
-            const uint32_t a_stage = 2u * c.BH * 8u * 128u;
-            const uint32_t b_stage = ((uint32_t)Wp * c.BH * 128u + 1023u) & ~1023u;
+            const uint32_t a_stage = 2u * c.BH * c.BNn * 8u * 128u;
+            const uint32_t b_stage = ((uint32_t)Wp * c.BH * c.BNn * 128u + 1023u) & ~1023u;
             const uint32_t stage_bytes = a_stage + b_stage;
             P.stages = std::min<int>(8, (int)((200u * 1024u) / stage_bytes));
             P.tmem_cols = 256;
@@ -1112,13 +1181,13 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
                 P.nhb[ql] = (ho + c.BH - 1) / c.BH;
                 P.nwb[ql] = (wo + 7) / 8;
                 P.box_prefix[ql] = boxes;
-                boxes += Lo.N * P.nhb[ql] * P.nwb[ql];
+                boxes += ((Lo.N + c.BNn - 1) / c.BNn) * P.nhb[ql] * P.nwb[ql];
                 {
                     const int C = Lo.Cpad;
                     void *base = (char *)dy + Lo.offset(i, j) * 2;
                     cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)wo, (cuuint64_t)ho, (cuuint64_t)Lo.N};
                     cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)wo * C * 2, (cuuint64_t)ho * wo * C * 2};
-                    cuuint32_t box[4] = {64, 8, (cuuint32_t)c.BH, 1};
+                    cuuint32_t box[4] = {64, 8, (cuuint32_t)c.BH, (cuuint32_t)c.BNn};
                     cuuint32_t es[4] = {1, 1, 1, 1};
                     if (encode(&P.mapDY[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides, box, es,
                                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -1130,7 +1199,7 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
                     void *base = (char *)x + Li.offset(i, j) * 2;
                     cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)wp, (cuuint64_t)hp, (cuuint64_t)Li.N};
                     cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)wp * C * 2, (cuuint64_t)hp * wp * C * 2};
-                    cuuint32_t box[4] = {64, (cuuint32_t)Wp, (cuuint32_t)c.BH, 1};
+                    cuuint32_t box[4] = {64, (cuuint32_t)Wp, (cuuint32_t)c.BH, (cuuint32_t)c.BNn};
                     cuuint32_t es[4] = {1, 1, 1, 1};
                     if (encode(&P.mapX[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides, box, es,
                                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,

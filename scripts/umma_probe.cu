@@ -27,7 +27,7 @@ __device__ __forceinline__ uint64_t desc(uint32_t saddr, uint32_t lbo, uint32_t 
 }
 
 // mode 0: A K-major (global A is [rowsA][64] with K contiguous); mode 1: A MN-major (global A is [rowsK][64 M... 128 M in 2 blocks])
-__global__ void probe(const __nv_bfloat16 *A, const __nv_bfloat16 *B, float *D, int mode, int off, int base_off) {
+__global__ void probe(const __nv_bfloat16 *A, const __nv_bfloat16 *B, float *D, int mode, int off, int base_off, int sbo_rows) {
     extern __shared__ __align__(1024) uint8_t smem[];
     uint8_t *sA = smem;                 // up to 2 x 32 KB
     uint8_t *sB = smem + 65536;         // 8 KB
@@ -70,7 +70,7 @@ __global__ void probe(const __nv_bfloat16 *A, const __nv_bfloat16 *B, float *D, 
         const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)mode << 15) | ((64u >> 3) << 17) | ((128u >> 4) << 24);
         for (int j = 0; j < 4; ++j) {
             uint64_t ad, bd;
-            if (mode == 0) ad = desc(s32(sA) + off * 128 + 32 * j, 16, 1024, 2, base_off);
+            if (mode == 0) ad = desc(s32(sA) + off * 128 + 32 * j, 16, sbo_rows * 128, 2, base_off);
             else ad = desc(s32(sA) + off * 128 + 2048 * j, 32768, 1024, 2, base_off);
             bd = desc(s32(sB) + 32 * j, 16, 1024, 2, 0);
             asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
@@ -115,7 +115,7 @@ int main() {
             for (int bo : {0, 1, 2, 3, 7}) {
                 if (bo && off == 0) continue;
                 cudaMemset(dD, 0, 128 * 64 * 4);
-                probe<<<1, 128, 80 * 1024>>>(dA, dB, dD, mode, off, bo);
+                probe<<<1, 128, 80 * 1024>>>(dA, dB, dD, mode, off, bo, 8);
                 cudaError_t e = cudaDeviceSynchronize();
                 if (e != cudaSuccess) { printf("mode %d off %d bo %d: CUDA error %s\n", mode, off, bo, cudaGetErrorString(e)); return 1; }
                 cudaMemcpy(hD.data(), dD, 128 * 64 * 4, cudaMemcpyDeviceToHost);
@@ -133,5 +133,23 @@ int main() {
                 printf("mode %s off %2d base_off %d : max|err| = %g %s\n", mode == 0 ? "K-major " : "MN-major", off, bo, maxerr,
                        maxerr < 1e-3 ? "MATCH" : "");
             }
+    // K-major A with 8-row M groups SBO = sbo rows apart (halo views): M row m -> A row (m/8)*sbo + m%8 + off
+    for (int sbo : {8, 9, 10, 12, 16})
+        for (int off : {0, 1, 2, 3}) {
+            cudaMemset(dD, 0, 128 * 64 * 4);
+            probe<<<1, 128, 80 * 1024>>>(dA, dB, dD, 0, off, 0, sbo);
+            cudaDeviceSynchronize();
+            cudaMemcpy(hD.data(), dD, 128 * 64 * 4, cudaMemcpyDeviceToHost);
+            double maxerr = 0;
+            for (int m = 0; m < 128; ++m)
+                for (int n = 0; n < 64; ++n) {
+                    const int row = (m / 8) * sbo + m % 8 + off;
+                    if (row >= 256) continue;
+                    double ref = 0;
+                    for (int k = 0; k < 64; ++k) ref += fA[row * 64 + k] * fB[n * 64 + k];
+                    maxerr = fmax(maxerr, fabs(ref - hD[m * 64 + n]));
+                }
+            printf("K-major SBO %2d rows off %d : max|err| = %g %s\n", sbo, off, maxerr, maxerr < 1e-3 ? "MATCH" : "");
+        }
     return 0;
 }

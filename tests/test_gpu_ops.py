@@ -72,6 +72,8 @@ CONV_CASES = [
     ("s2_c64", 2, 64, 128, 3, 2, 1, 28, 28, 2, 2, True),
     ("7x7s2_c3_64", 2, 3, 64, 7, 2, 3, 30, 30, 2, 2, True),
     ("c512", 1, 512, 512, 3, 1, 1, 14, 14, 2, 2, True),
+    ("halo_odd_n", 3, 64, 64, 3, 1, 1, 14, 14, 2, 2, True),
+    ("halo_uneven", 2, 128, 128, 3, 1, 1, 23, 19, 3, 2, True),
 ]
 
 

@@ -55,6 +55,7 @@ struct TcConvParams {
     int kchan;       // Cpad of the A side (K = taps * kchan)
     int a3d;         // 8-channel A: 3-D maps with pixels merged into 128-byte-wide rows (coordinate 8*w)
     int halo;        // stride-1 halo mode: one A box per (channel chunk, kernel row) serves the kw column taps
+    int halo8;       // 8-channel halo mode: ONE merged-row box per tile serves all taps (no-swizzle K-major A)
     int b3d;         // halo: the kw taps' weights arrive as one 3-D box
     int Wp;          // halo: input box width = 8 + kw - 1
     uint32_t a_stage;  // bytes per A stage (1024-aligned)
@@ -188,7 +189,12 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     tc::mbar_arrive_expect_tx(&full[stage], p.a_tx_bytes + p.b_tx_bytes);
                     uint8_t *a = sA + (size_t)stage * p.a_stage;
                     uint8_t *b = sB + (size_t)stage * b_stage;
-                    if (p.halo) {
+                    if (p.halo8) {
+                        // rows (h) x (8 + kw - 1) pixels x 8 channels; the weights' K = taps*8 in 64-wide boxes
+                        tc::tma_load_3d(a, &p.mapA[ql], &full[stage], 8 * wbase, hbase, n0);
+                        for (int kb = 0; kb * 64 < KT * 8; ++kb)
+                            tc::tma_load_2d(b + kb * p.BN * 128, &p.mapB, &full[stage], kb * 64, co0);
+                    } else if (p.halo) {
                         const int cc = ks / p.kh, r = ks - cc * p.kh;
                         tc::tma_load_4d(a, &p.mapA[ql], &full[stage], cc * 64, wbase, hbase + r, n0);
                         if (p.b3d) {
@@ -232,6 +238,23 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     tc::tc_fence_after();
                     const uint32_t a_base = tc::smem_u32(sA + (size_t)stage * p.a_stage);
                     const uint32_t b_base = tc::smem_u32(sB + (size_t)stage * b_stage);
+                    if (p.halo8) {
+                        // no-swizzle K-major A: a core matrix is 8 consecutive pixels x 16 B (8 channels);
+                        // M groups (output rows) are Wp pixels apart (SBO = Wp*16 B); each MMA covers the
+                        // K = 16 of two taps whose views differ by LBO = (pixel offset difference)*16 B
+                        const int npairs = (KT + 1) / 2;
+                        for (int pr = 0; pr < npairs; ++pr) {
+                            const int t0 = 2 * pr, t1 = 2 * pr + 1;
+                            const int o0 = (t0 / p.kw) * p.Wp + (t0 % p.kw);
+                            const int o1 = t1 < KT ? (t1 / p.kw) * p.Wp + (t1 % p.kw) : o0 + 1;
+                            const uint64_t adesc = tc::smem_desc(a_base + 16u * o0, 16u * (uint32_t)(o1 - o0), (uint32_t)p.Wp * 16u, 0);
+                            const uint64_t bdesc = tc::smem_desc(b_base + (uint32_t)((pr / 4) * p.BN) * 128u + 32u * (pr % 4), 16, 1024, 2);
+                            tc::mma_bf16(d, adesc, bdesc, idesc, (ks | pr) != 0);
+                        }
+                        tc::mma_commit(&empty[stage]);
+                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        continue;
+                    }
                     if (p.halo) {
                         // tap c of this kernel row = the A tile viewed c pixel-rows further on (SW128 is
                         // address-based, probed); 8-pixel M groups are Wp rows apart (SBO = Wp * 128 B)
@@ -510,8 +533,16 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         const int a3d = (cpad == 8 && s == 1) ? 1 : 0;  // TMA rows of 16 B are slow: merge 8 pixels per row
         // halo mode for narrow outputs (per-tap TMA boxes cannot keep the MMA fed there)
         const int halo = (s == 1 && cpad % 64 == 0 && BN <= 128 && kw >= 2 && kw <= 4 && !getenv("SPLITCNN_NO_HALO")) ? 1 : 0;
+        const int halo8 = (mode == 0 && cpad == 8 && s == 1 && kw <= 8 && kh * kw <= 16 && !getenv("SPLITCNN_NO_HALO")) ? 1 : 0;
         TileShape ts = choose_tile(ext, N, s, a3d ? 32 : 128);
-        if (halo) {  // 8 output columns per M group; BH x BNn groups (<= 16)
+        if (halo8) {  // 8 output columns x BH output rows, one image per tile
+            long best = -1;
+            for (int bh = 1; bh <= 16; ++bh) {
+                long t = 0;
+                for (auto &e : ext) t += (long)N * ((e.first + bh - 1) / bh) * ((e.second + 7) / 8);
+                if (best < 0 || t < best) { best = t; ts = {8, bh, 1}; }
+            }
+        } else if (halo) {  // 8 output columns per M group; BH x BNn groups (<= 16)
             long best = -1;
             for (int bh = 1; bh <= 16; ++bh)
                 for (int bn = 1; bh * bn <= 16 && bn <= N; ++bn) {
@@ -531,6 +562,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.kchan = cpad;
         P.a3d = a3d;
         P.halo = halo;
+        P.halo8 = halo8;
         P.Wp = 8 + kw - 1;
         if (cpad >= 64) {
             P.cchunks = cpad / 64; P.tps = 1; P.ksteps = kh * kw * P.cchunks;
@@ -546,7 +578,12 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.a_tx_bytes = (uint32_t)P.tps * P.rows_box * row_bytes;
         P.b_tx_bytes = (uint32_t)BN * 128u;
         P.a_stage = 16384u;
-        if (halo) {
+        if (halo8) {
+            P.ksteps = 1;
+            P.a_tx_bytes = (uint32_t)P.Wp * (ts.BH + kh - 1) * 16u;
+            P.a_stage = (P.a_tx_bytes + 1023u) & ~1023u;
+            P.b_tx_bytes = (uint32_t)((kh * kw * 8 + 63) / 64) * BN * 128u;
+        } else if (halo) {
             P.ksteps = (cpad / 64) * kh;
             P.a_tx_bytes = (uint32_t)P.Wp * ts.BH * ts.BNn * 128u;
             P.a_stage = (P.a_tx_bytes + 1023u) & ~1023u;
@@ -596,6 +633,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
                 cuuint64_t d3[3] = {(cuuint64_t)wp * 8, (cuuint64_t)hp, (cuuint64_t)N};
                 cuuint64_t s3[2] = {(cuuint64_t)wp * 16, (cuuint64_t)hp * wp * 16};
                 cuuint32_t b3[3] = {(cuuint32_t)(ts.BW * 8), (cuuint32_t)ts.BH, (cuuint32_t)ts.BNn};
+                if (halo8) { b3[0] = (cuuint32_t)(8 * P.Wp); b3[1] = (cuuint32_t)(ts.BH + kh - 1); b3[2] = 1; }
                 cuuint32_t e3[3] = {1, 1, 1};
                 r = encode(&P.mapA[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, base, d3, s3, b3, e3,
                            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -1033,6 +1071,142 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
     if (warp == 1) tc::tmem_dealloc(tmem_base, p.tmem_cols);
 }
 
+// ------------------------------------------------------------ narrow-input weight gradient (Cin_pad = 8)
+// dW[co][tap][ci] for an 8-channel input (VGG conv1_1, C = 3 padded to 8): per stage one dY tile
+// (BH output rows x 8 columns, MN-major SW128) and ONE X tile of (BH + kh - 1) rows x (8 + kw - 1)
+// pixels x 8 channels loaded with 16-byte pixel rows merged into 3-D rows.  In the no-swizzle
+// MN-major layout a core matrix is 8 pixels x 16 B, so the operand of tap t is the X tile viewed
+// o_t = r*Wp + c pixels further on; two taps form the two 8-channel MN blocks of one N = 16 MMA
+// (block stride SBO = (o_t1 - o_t0)*16 B, output-row K groups at LBO = Wp*16 B).
+struct TcWgNarrowParams {
+    CUtensorMap mapDY[TC_MAXP];
+    CUtensorMap mapX[TC_MAXP];
+    int box_prefix[TC_MAXP + 1];
+    int pt[TC_MAXP], pl[TC_MAXP];
+    int nhb[TC_MAXP], nwb[TC_MAXP];
+    int npatch, BH, kh, kw;
+    int nco_blk, boxes_per_split, nsplit;
+    int Cout, stages;
+    uint32_t tmem_cols;
+    float *part;  // [nsplit][Cout][kh][kw][8]
+};
+
+__global__ void __launch_bounds__(192, 1) wgrad_narrow_kernel(const __grid_constant__ TcWgNarrowParams p) {
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+    const int S = p.stages;
+    const int rows = p.BH * 8;
+    const int Wp = 8 + p.kw - 1, Hp = p.BH + p.kh - 1;
+    const int KT = p.kh * p.kw, npairs = (KT + 1) / 2;
+    const uint32_t a_blk = (uint32_t)rows * 128u;
+    const uint32_t a_stage = 2u * a_blk;
+    const uint32_t b_bytes = (uint32_t)Wp * Hp * 16u;
+    const uint32_t b_stage = (b_bytes + 1023u) & ~1023u;
+    uint8_t *sA = smem;
+    uint8_t *sB = smem + (size_t)S * a_stage;
+    uint64_t *full = (uint64_t *)(sB + (size_t)S * b_stage);
+    uint64_t *empty = full + S;
+    uint64_t *tfull = empty + S;
+    uint32_t *tmem_slot = (uint32_t *)(tfull + 1);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (warp == 0 && lane == 0) {
+        for (int s = 0; s < S; ++s) {
+            tc::mbar_init(&full[s], 1);
+            tc::mbar_init(&empty[s], 1);
+        }
+        tc::mbar_init(&tfull[0], 1);
+        tc::fence_barrier_init();
+    }
+    if (warp == 1) tc::tmem_alloc_dyn(tmem_slot, p.tmem_cols);
+    tc::tc_fence_before();
+    __syncthreads();
+    tc::tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+    const int co_blk = blockIdx.x % p.nco_blk, z = blockIdx.x / p.nco_blk;
+    const int total_boxes = p.box_prefix[p.npatch];
+    const int b0 = z * p.boxes_per_split, b1 = min(total_boxes, b0 + p.boxes_per_split);
+
+    if (warp == 0) {
+        if (lane == 0) {
+            int stage = 0, ql = 0;
+            uint32_t ph = 0;
+            for (int b = b0; b < b1; ++b) {
+                while (b >= p.box_prefix[ql + 1]) ++ql;
+                int idx = b - p.box_prefix[ql];
+                const int wb = idx % p.nwb[ql];
+                idx /= p.nwb[ql];
+                const int hb = idx % p.nhb[ql], n = idx / p.nhb[ql];
+                const int ow0 = wb * 8, oh0 = hb * p.BH;
+                tc::mbar_wait_sleep(&empty[stage], ph ^ 1);
+                tc::mbar_arrive_expect_tx(&full[stage], a_stage + b_bytes);
+                uint8_t *a = sA + (size_t)stage * a_stage;
+                tc::tma_load_4d(a, &p.mapDY[ql], &full[stage], co_blk * 128, ow0, oh0, n);
+                tc::tma_load_4d(a + a_blk, &p.mapDY[ql], &full[stage], co_blk * 128 + 64, ow0, oh0, n);
+                tc::tma_load_3d(sB + (size_t)stage * b_stage, &p.mapX[ql], &full[stage], 8 * (ow0 - p.pl[ql]),
+                                oh0 - p.pt[ql], n);
+                if (++stage == S) { stage = 0; ph ^= 1; }
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            const uint32_t idesc = tc::idesc_bf16(128, 16, 1, 1);
+            int stage = 0;
+            uint32_t ph = 0;
+            for (int b = b0; b < b1; ++b) {
+                tc::mbar_wait(&full[stage], ph);
+                tc::tc_fence_after();
+                const uint32_t a_base = tc::smem_u32(sA + (size_t)stage * a_stage);
+                const uint32_t b_base = tc::smem_u32(sB + (size_t)stage * b_stage);
+                for (int j = 0; j < rows / 16; ++j) {
+                    const uint64_t adesc = tc::smem_desc(a_base + 2048u * j, a_blk, 1024, 2);
+                    for (int pr = 0; pr < npairs; ++pr) {
+                        const int t0 = 2 * pr, t1 = 2 * pr + 1;
+                        const int o0 = (t0 / p.kw) * Wp + (t0 % p.kw);
+                        const int o1 = t1 < KT ? (t1 / p.kw) * Wp + (t1 % p.kw) : o0 + 1;
+                        const uint64_t bdesc = tc::smem_desc(b_base + (uint32_t)(2 * j * Wp + o0) * 16u, (uint32_t)Wp * 16u,
+                                                             (uint32_t)(o1 - o0) * 16u, 0);
+                        tc::mma_bf16(tmem_base + 16u * pr, adesc, bdesc, idesc, (b != b0 || j) ? 1u : 0u);
+                    }
+                }
+                tc::mma_commit(&empty[stage]);
+                if (++stage == S) { stage = 0; ph ^= 1; }
+            }
+            tc::mma_commit(&tfull[0]);
+        }
+    } else {
+        const int quad = warp & 3;
+        const int co = co_blk * 128 + quad * 32 + lane;
+        const bool any = b1 > b0;
+        if (any) {
+            tc::mbar_wait(&tfull[0], 0);
+            tc::tc_fence_after();
+        }
+        const uint32_t tacc = tmem_base + ((uint32_t)(quad * 32) << 16);
+        for (int pr = 0; pr < npairs; ++pr) {
+            float v[16];
+            if (any) {
+                tc::tmem_ld16(tacc + 16u * pr, v);
+            } else {
+#pragma unroll
+                for (int e = 0; e < 16; ++e) v[e] = 0.f;
+            }
+            if (co >= p.Cout) continue;
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const int tap = 2 * pr + h;
+                if (tap >= KT) break;
+                float4 *d4 = reinterpret_cast<float4 *>(p.part + (((int64_t)z * p.Cout + co) * KT + tap) * 8);
+                d4[0] = make_float4(v[8 * h], v[8 * h + 1], v[8 * h + 2], v[8 * h + 3]);
+                d4[1] = make_float4(v[8 * h + 4], v[8 * h + 5], v[8 * h + 6], v[8 * h + 7]);
+            }
+        }
+    }
+    tc::tc_fence_before();
+    __syncthreads();
+    tc::tc_fence_after();
+    if (warp == 1) tc::tmem_dealloc(tmem_base, p.tmem_cols);
+}
+
 namespace {
 
 struct WgradCfg {
@@ -1120,6 +1294,37 @@ WgHaloCfg wgrad_halo_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, i
 
 }  // namespace
 
+namespace {
+
+struct WgNarrowCfg {
+    int BH, nco_blk, total_boxes, nsplit, boxes_per_split;
+};
+
+bool wgrad_narrow_ok(const Level &Li, const Level &Lo, const LayerGeom &g) {
+    return Li.Cpad == 8 && g.L.sh == 1 && g.L.sw == 1 && g.L.kw <= 8 && g.L.kh * g.L.kw <= 16 && Lo.Cpad % 64 == 0;
+}
+
+WgNarrowCfg wgrad_narrow_cfg(const Level &Lo, const LayerGeom &g, int p0, int p1) {
+    WgNarrowCfg c{};
+    long best = -1;
+    for (int bh = 2; bh <= 16; bh += 2) {
+        long n = 0;
+        for (int q = p0; q < p1; ++q)
+            n += (long)Lo.N * ((Lo.ph(q / Lo.nw()) + bh - 1) / bh) * ((Lo.pw(q % Lo.nw()) + 7) / 8);
+        const long cost = n * (bh * 8 + 256);
+        if (best < 0 || cost < best) { best = cost; c.BH = bh; c.total_boxes = (int)n; }
+    }
+    c.nco_blk = (g.L.cout + 127) / 128;
+    int Z = std::max(1, (2 * num_sms() + c.nco_blk - 1) / c.nco_blk);
+    Z = std::min(Z, std::max(1, c.total_boxes / 4));
+    Z = std::min(Z, 296);
+    c.boxes_per_split = (c.total_boxes + Z - 1) / Z;
+    c.nsplit = (c.total_boxes + c.boxes_per_split - 1) / c.boxes_per_split;
+    return c;
+}
+
+}  // namespace
+
 static bool wgrad_tc_ok(const Level &Li, const Level &Lo, const LayerGeom &g) {
     return a_channels_ok(Li.Cpad) && Lo.Cpad % 64 == 0 && g.L.sh == g.L.sw && g.L.sh <= 2;
 }
@@ -1133,6 +1338,10 @@ size_t wgrad_tc_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g) {
         best = std::max(best, (size_t)c.nsplit * g.L.cout * g.L.kh * g.L.kw * Li.Cpad * sizeof(float));
         if (wgrad_halo_ok(Li, Lo, g)) {
             WgHaloCfg h = wgrad_halo_cfg(Li, Lo, g, g0, std::min(np, g0 + TC_MAXP));
+            best = std::max(best, (size_t)h.nsplit * g.L.cout * g.L.kh * g.L.kw * Li.Cpad * sizeof(float));
+        }
+        if (wgrad_narrow_ok(Li, Lo, g) && getenv("SPLITCNN_NARROW_WGRAD")) {
+            WgNarrowCfg h = wgrad_narrow_cfg(Lo, g, g0, std::min(np, g0 + TC_MAXP));
             best = std::max(best, (size_t)h.nsplit * g.L.cout * g.L.kh * g.L.kw * Li.Cpad * sizeof(float));
         }
     }
@@ -1153,7 +1362,76 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
     static bool attr_set = false;
     bool first = true;
     int gend = p1;  // end of the patch range left for the generic kernel
-    if (wgrad_halo_ok(Li, Lo, g)) {
+    // opt-in: correct, but slower than the generic multi-tap path on conv1_1 so far (many N = 16 MMAs)
+    if (wgrad_narrow_ok(Li, Lo, g) && getenv("SPLITCNN_NARROW_WGRAD")) {
+        static bool narrow_attr = false;
+        for (int g0 = p0; g0 < p1; g0 += TC_MAXP) {
+            const int g1 = std::min(p1, g0 + TC_MAXP);
+            WgNarrowCfg c = wgrad_narrow_cfg(Lo, g, g0, g1);
+            static thread_local TcWgNarrowParams P;
+            std::memset(&P, 0, sizeof(P));
+            P.npatch = g1 - g0;
+            P.BH = c.BH; P.kh = g.L.kh; P.kw = g.L.kw;
+            P.nco_blk = c.nco_blk; P.boxes_per_split = c.boxes_per_split; P.nsplit = c.nsplit;
+            P.Cout = g.L.cout;
+            const int Wp = 8 + g.L.kw - 1, Hp = c.BH + g.L.kh - 1;
+            const uint32_t a_stage = 2u * c.BH * 8u * 128u;
+            const uint32_t b_stage = ((uint32_t)Wp * Hp * 16u + 1023u) & ~1023u;
+            const uint32_t stage_bytes = a_stage + b_stage;
+            P.stages = std::min<int>(8, (int)((200u * 1024u) / stage_bytes));
+            uint32_t cols = 32;
+            while (cols < (uint32_t)(16 * ((g.L.kh * g.L.kw + 1) / 2))) cols <<= 1;
+            P.tmem_cols = cols;
+            P.part = part;
+            int boxes = 0;
+            for (int q = g0; q < g1; ++q) {
+                const int ql = q - g0, i = q / Lo.nw(), j = q % Lo.nw();
+                const int ho = Lo.ph(i), wo = Lo.pw(j), hp = Li.ph(i), wp = Li.pw(j);
+                P.pt[ql] = g.pad_h[2 * i];
+                P.pl[ql] = g.pad_w[2 * j];
+                P.nhb[ql] = (ho + c.BH - 1) / c.BH;
+                P.nwb[ql] = (wo + 7) / 8;
+                P.box_prefix[ql] = boxes;
+                boxes += Lo.N * P.nhb[ql] * P.nwb[ql];
+                {
+                    const int C = Lo.Cpad;
+                    void *base = (char *)dy + Lo.offset(i, j) * 2;
+                    cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)wo, (cuuint64_t)ho, (cuuint64_t)Lo.N};
+                    cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)wo * C * 2, (cuuint64_t)ho * wo * C * 2};
+                    cuuint32_t box[4] = {64, 8, (cuuint32_t)c.BH, 1};
+                    cuuint32_t es[4] = {1, 1, 1, 1};
+                    if (encode(&P.mapDY[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides, box, es,
+                               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+                        return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(dY narrow) failed");
+                }
+                {
+                    void *base = (char *)x + Li.offset(i, j) * 2;
+                    cuuint64_t d3[3] = {(cuuint64_t)wp * 8, (cuuint64_t)hp, (cuuint64_t)Li.N};
+                    cuuint64_t s3[2] = {(cuuint64_t)wp * 16, (cuuint64_t)hp * wp * 16};
+                    cuuint32_t b3[3] = {(cuuint32_t)(8 * Wp), (cuuint32_t)Hp, 1};
+                    cuuint32_t e3[3] = {1, 1, 1};
+                    if (encode(&P.mapX[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, base, d3, s3, b3, e3,
+                               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+                        return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(X narrow) failed");
+                }
+            }
+            P.box_prefix[P.npatch] = boxes;
+            const size_t smem = 1024 + (size_t)P.stages * stage_bytes + 256;
+            if (!narrow_attr) {
+                cudaFuncSetAttribute(wgrad_narrow_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+                narrow_attr = true;
+            }
+            wgrad_narrow_kernel<<<c.nco_blk * c.nsplit, 192, smem, st>>>(P);
+            count_launch();
+            cudaError_t e = cudaGetLastError();
+            if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("wgrad_narrow_kernel: ") + cudaGetErrorString(e));
+            launch_reduce(part, c.nsplit, nW, dw, first ? beta : 1.f, st);
+            first = false;
+        }
+        gend = p0;
+    } else if (wgrad_halo_ok(Li, Lo, g)) {
         static bool halo_attr = false;
         for (int g0 = p0; g0 < p1; g0 += TC_MAXP) {
             const int g1 = std::min(p1, g0 + TC_MAXP);

@@ -274,3 +274,24 @@ def test_offload_prefetch_roundtrip_bit_exact(sc):
     assert torch.equal(x, keep)
     with pytest.raises(sc.SplitCNNError, match="pinned"):
         sc.splitcnn_offload(pl.handle, 0, dtype, 0, x, torch.empty(10 ** 6, dtype=torch.uint8), None, mem, None)
+
+
+def test_narrow_wgrad_opt_in_parity(sc, monkeypatch):
+    """The opt-in 8-channel halo wgrad (SPLITCNN_NARROW_WGRAD) matches the oracle too."""
+    monkeypatch.setenv("SPLITCNN_NARROW_WGRAD", "1")
+    dtype = sc.BF16
+    layers = [synth.conv(3, 64, 3, 1, 1)]
+    ref, pl = _make(sc, layers, 2, 3, 30, 26, 2, 2, seed=17)
+    lp = ref.layers[0]
+    lv0, lv1 = pl.levels
+    g = synth.rng(17)
+    X = _round(synth.uniform(g, (2, 3, 30, 26)), dtype, sc)
+    G = _round(synth.normal(g, (2, 64, 30, 26)), dtype, sc)
+    x = _dev(sc, pack_level(X, lv0), dtype)
+    dy = _dev(sc, pack_level(G, lv1), dtype)
+    ws_b = pl.workspace_size(0, dtype, 2)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    dw = torch.zeros((64, 3, 3, 8), dtype=torch.float32, device="cuda")
+    sc.splitcnn_conv_bwd_filter(pl.handle, 0, dtype, x, dy, dw, None, 0.0, ws, ws_b)
+    dWref, _ = O.conv_bwd_filter(O.split(X, lp.Ih, lp.Iw), O.split(G, lp.Oh, lp.Ow), lp)
+    assert normwise(w_lib_to_oihw(_host(dw), 3), dWref) <= TOL[dtype]

@@ -59,6 +59,8 @@ struct TcConvParams {
     int b3d;         // halo: the kw taps' weights arrive as one 3-D box
     int Wp;          // halo: input box width = 8 + kw - 1
     uint32_t a_stage;  // bytes per A stage (1024-aligned)
+    int bres;          // halo: all weights resident in smem (loaded once per CTA)
+    uint32_t bres_off, bres_bytes;
     int BN, Cout, Cpo;
     int stages;
     uint32_t tmem_cols;
@@ -72,6 +74,10 @@ struct TcConvParams {
     int ychunk;       // channels per output box (64, 32, 16 or 8)
     uint32_t y_mask;  // swizzle mask of the staging tile (7 / 3 / 1 / 0)
     uint32_t stage_off, bar_off;  // smem layout
+    int ybufs;                    // staging buffers (2: the TMA store of tile t overlaps tile t+1)
+    int dbg;                      // experiments only (SPLITCNN_DBG): 1 no TMA store, 2 no MMA, 4 no loads, 8 no TMEM->smem
+    int egroups;                  // 2: two independent 4-warp epilogue groups, one per TMEM accumulator
+    uint32_t ybuf_bytes;
 };
 
 static_assert(sizeof(TcConvParams) <= 32000, "kernel parameter space is 32 KB");
@@ -145,7 +151,9 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
     uint64_t *tfull = empty + S;
     uint64_t *tempty = tfull + 2;
     uint64_t *ybar = tempty + 2;
-    uint32_t *tmem_slot = (uint32_t *)(ybar + 1);
+    uint64_t *wbar = ybar + 1;
+    uint32_t *tmem_slot = (uint32_t *)(wbar + 2);
+    uint8_t *sW = smem + p.bres_off;   // resident weights (bres)
     float *sbias = (float *)(smem + p.bar_off + 512);   // [Cout] bias (16-byte aligned)
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -156,9 +164,11 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
         }
         for (int a = 0; a < 2; ++a) {
             tc::mbar_init(&tfull[a], 1);
-            tc::mbar_init(&tempty[a], 8);
+            tc::mbar_init(&tempty[a], p.egroups == 2 ? 4 : 8);
         }
         tc::mbar_init(ybar, 1);
+        tc::mbar_init(wbar, 1);
+        tc::mbar_init(wbar + 1, 1);   // group 1's mask barrier
         tc::fence_barrier_init();
     }
     if (BIAS)
@@ -176,6 +186,20 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             // ================= TMA producer
             for (int q = 0; q < p.npatch; ++q) tc::tma_prefetch_desc(&p.mapA[q]);
             tc::tma_prefetch_desc(&p.mapB);
+            if (p.bres) {  // every (chunk, kernel row) weight box once, for all tiles of this CTA
+                tc::mbar_arrive_expect_tx(wbar, p.bres_bytes);
+                const int nchunk = p.kchan / 64;
+                for (int cc = 0; cc < nchunk; ++cc)
+                    for (int r = 0; r < p.kh; ++r) {
+                        uint8_t *dst = sW + (size_t)((cc * p.kh + r) * p.kw) * p.BN * 128;
+                        if (p.b3d) {
+                            tc::tma_load_3d(dst, &p.mapB, wbar, cc * 64, 0, r * p.kw);
+                        } else {
+                            for (int c = 0; c < p.kw; ++c)
+                                tc::tma_load_2d(dst + c * p.BN * 128, &p.mapB, wbar, (r * p.kw + c) * p.kchan + cc * 64, 0);
+                        }
+                    }
+            }
             int stage = 0;
             uint32_t ph = 0;
             for (int t = blockIdx.x; t < total; t += gridDim.x) {
@@ -184,8 +208,14 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 const int wbase = wb * p.BW * p.s - p.pl[ql];
                 const int hbase = hb * p.BH * p.s - p.pt[ql];
                 const int n0 = nb * p.BNn, co0 = cb * p.BN;
+                if (p.dbg & 16) continue;
                 for (int ks = 0; ks < p.ksteps; ++ks) {
                     tc::mbar_wait_sleep(&empty[stage], ph ^ 1);
+                    if (p.dbg & 4) {
+                        tc::mbar_arrive(&full[stage]);
+                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        continue;
+                    }
                     tc::mbar_arrive_expect_tx(&full[stage], p.a_tx_bytes + p.b_tx_bytes);
                     uint8_t *a = sA + (size_t)stage * p.a_stage;
                     uint8_t *b = sB + (size_t)stage * b_stage;
@@ -197,7 +227,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     } else if (p.halo) {
                         const int cc = ks / p.kh, r = ks - cc * p.kh;
                         tc::tma_load_4d(a, &p.mapA[ql], &full[stage], cc * 64, wbase, hbase + r, n0);
-                        if (p.b3d) {
+                        if (p.bres) {
+                        } else if (p.b3d) {
                             tc::tma_load_3d(b, &p.mapB, &full[stage], cc * 64, co0, r * p.kw);
                         } else {
                             for (int c = 0; c < p.kw; ++c)
@@ -224,68 +255,143 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             }
         }
     } else if (warp == 1) {
-        if (lane == 0) {
-            // ================= MMA issuer
+        {
+            // ================= MMA issuer: the whole warp runs the loop converged; elect.sync issues
             const uint32_t idesc = tc::idesc_bf16(128, p.BN);
             int stage = 0, acc = 0;
             uint32_t ph = 0, aph = 0;
+            if (p.bres) tc::mbar_wait(wbar, 0);
             for (int t = blockIdx.x; t < total; t += gridDim.x) {
                 tc::mbar_wait_sleep(&tempty[acc], aph ^ 1);
                 tc::tc_fence_after();
                 const uint32_t d = tmem_base + (uint32_t)(acc * p.BN);
                 for (int ks = 0; ks < p.ksteps; ++ks) {
-                    tc::mbar_wait(&full[stage], ph);
+                    if (!(p.dbg & 16)) tc::mbar_wait(&full[stage], ph);
                     tc::tc_fence_after();
                     const uint32_t a_base = tc::smem_u32(sA + (size_t)stage * p.a_stage);
                     const uint32_t b_base = tc::smem_u32(sB + (size_t)stage * b_stage);
+                    if (p.dbg & 2) {
+                        tc::mma_commit_ws(&empty[stage]);
+                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        continue;
+                    }
                     if (p.halo8) {
                         // no-swizzle K-major A: a core matrix is 8 consecutive pixels x 16 B (8 channels);
                         // M groups (output rows) are Wp pixels apart (SBO = Wp*16 B); each MMA covers the
                         // K = 16 of two taps whose views differ by LBO = (pixel offset difference)*16 B
                         const int npairs = (KT + 1) / 2;
+                        const uint64_t b0 = tc::smem_desc(b_base, 16, 1024, 2);
                         for (int pr = 0; pr < npairs; ++pr) {
                             const int t0 = 2 * pr, t1 = 2 * pr + 1;
                             const int o0 = (t0 / p.kw) * p.Wp + (t0 % p.kw);
                             const int o1 = t1 < KT ? (t1 / p.kw) * p.Wp + (t1 % p.kw) : o0 + 1;
                             const uint64_t adesc = tc::smem_desc(a_base + 16u * o0, 16u * (uint32_t)(o1 - o0), (uint32_t)p.Wp * 16u, 0);
-                            const uint64_t bdesc = tc::smem_desc(b_base + (uint32_t)((pr / 4) * p.BN) * 128u + 32u * (pr % 4), 16, 1024, 2);
-                            tc::mma_bf16(d, adesc, bdesc, idesc, (ks | pr) != 0);
+                            // descriptors are linear in the start address (field = addr >> 4)
+                            const uint64_t bdesc = b0 + (uint64_t)((((pr >> 2) * p.BN) * 128 + 32 * (pr & 3)) >> 4);
+                            tc::mma_bf16_ws(d, adesc, bdesc, idesc, (ks | pr) != 0);
                         }
-                        tc::mma_commit(&empty[stage]);
+                        tc::mma_commit_ws(&empty[stage]);
                         if (++stage == S) { stage = 0; ph ^= 1; }
                         continue;
                     }
                     if (p.halo) {
                         // tap c of this kernel row = the A tile viewed c pixel-rows further on (SW128 is
-                        // address-based, probed); 8-pixel M groups are Wp rows apart (SBO = Wp * 128 B)
-                        for (int c = 0; c < p.kw; ++c)
-#pragma unroll
-                            for (int j = 0; j < 4; ++j) {
-                                const uint64_t adesc = tc::smem_desc(a_base + 128u * c + 32u * j, 16, (uint32_t)p.Wp * 128u, 2);
-                                const uint64_t bdesc = tc::smem_desc(b_base + (uint32_t)(c * p.BN) * 128u + 32u * j, 16, 1024, 2);
-                                tc::mma_bf16(d, adesc, bdesc, idesc, (ks | c | j) != 0);
-                            }
-                        tc::mma_commit(&empty[stage]);
+                        // address-based, probed); 8-pixel M groups are Wp rows apart (SBO = Wp * 128 B).
+                        // Descriptors are linear in the start address: per-MMA descriptors are base + constant.
+                        const uint64_t a0 = tc::smem_desc(a_base, 16, (uint32_t)p.Wp * 128u, 2);
+                        const uint64_t b0 = p.bres ? tc::smem_desc(tc::smem_u32(sW) + (uint32_t)(ks * p.kw * p.BN) * 128u, 16, 1024, 2)
+                                                   : tc::smem_desc(b_base, 16, 1024, 2);
+                        const uint32_t bstep = (uint32_t)p.BN * 8u;   // BN*128 B >> 4
+                        for (int c = 0; c < p.kw; ++c) {
+                            const uint64_t ac = a0 + (uint64_t)(8 * c), bc = b0 + (uint64_t)(bstep * c);
+                            tc::mma_bf16_ws(d, ac, bc, idesc, (ks | c) != 0);
+                            tc::mma_bf16_ws(d, ac + 2, bc + 2, idesc, 1u);
+                            tc::mma_bf16_ws(d, ac + 4, bc + 4, idesc, 1u);
+                            tc::mma_bf16_ws(d, ac + 6, bc + 6, idesc, 1u);
+                        }
+                        if (!(p.dbg & 32)) tc::mma_commit_ws(&empty[stage]);
                         if (++stage == S) { stage = 0; ph ^= 1; }
                         continue;
                     }
+                    const uint64_t a0 = tc::smem_desc(a_base, p.a_lbo, p.a_sbo, p.a_layout);
+                    const uint64_t b0 = tc::smem_desc(b_base, 16, 1024, 2);
 #pragma unroll
                     for (int j = 0; j < 4; ++j) {
                         const int k0 = 16 * j;
                         const int chunk = k0 / p.cpadc;
-                        const uint32_t a_addr = a_base + chunk * p.a_chunk_bytes + (uint32_t)((k0 - chunk * p.cpadc) * 2);
-                        const uint64_t adesc = tc::smem_desc(a_addr, p.a_lbo, p.a_sbo, p.a_layout);
-                        const uint64_t bdesc = tc::smem_desc(b_base + 32u * j, 16, 1024, 2);
-                        tc::mma_bf16(d, adesc, bdesc, idesc, (ks | j) != 0);
+                        const uint32_t a_off = chunk * p.a_chunk_bytes + (uint32_t)((k0 - chunk * p.cpadc) * 2);
+                        tc::mma_bf16_ws(d, a0 + (uint64_t)(a_off >> 4), b0 + (uint64_t)(2 * j), idesc, (ks | j) != 0);
                     }
-                    tc::mma_commit(&empty[stage]);
+                    tc::mma_commit_ws(&empty[stage]);
                     if (++stage == S) { stage = 0; ph ^= 1; }
                 }
-                tc::mma_commit(&tfull[acc]);
+                tc::mma_commit_ws(&tfull[acc]);
                 acc ^= 1;
                 if (acc == 0) aph ^= 1;
             }
         }
+    } else if (!p.direct && p.egroups == 2) {
+        // ================= epilogue, two groups: warps 2..5 take even tiles (accumulator 0, staging 0),
+        // warps 6..9 odd tiles (accumulator 1, staging 1), so consecutive tiles' epilogues overlap
+        const int quad = warp & 3;
+        const int g = (warp - 2) >> 2;
+        const int row = quad * 32 + lane;
+        const int gtid = threadIdx.x - 64 - 128 * g;   // 0..127 within the group
+        const uint32_t rowB = (uint32_t)p.ychunk * 2u;
+        const uint32_t chunk_bytes = 128u * rowB;
+        uint8_t *sYb = sY + (size_t)g * p.ybuf_bytes;
+        uint64_t *mbar = g ? wbar + 1 : ybar;
+        uint32_t aph = 0, yph = 0;
+        for (int t = blockIdx.x + g * gridDim.x; t < total; t += 2 * gridDim.x) {
+            int ql, nb, hb, wb, cb;
+            decode_tile(p, t, ql, nb, hb, wb, cb);
+            const int co0 = cb * p.BN;
+            const int ow0 = wb * p.BW, oh0 = hb * p.BH, n0 = nb * p.BNn;
+            const int ncols = min(p.BN, p.Cpo - co0);
+            const int nchunks = ncols / p.ychunk;
+            if (gtid == 0) tc::bulk_wait_read0();      // this group's previous store has read the staging
+            tc::named_bar_sync(1 + g, 128);
+            if (MASK) {
+                if (gtid == 0) {
+                    tc::mbar_arrive_expect_tx(mbar, (uint32_t)nchunks * p.rows_box * rowB);
+                    for (int k = 0; k < nchunks; ++k)
+                        tc::tma_load_4d(sYb + k * chunk_bytes, &p.mapR[ql], mbar, co0 + k * p.ychunk, ow0, oh0, n0);
+                }
+                tc::mbar_wait(mbar, yph);
+                yph ^= 1;
+            }
+            tc::mbar_wait(&tfull[g], aph);
+            tc::tc_fence_after();
+            const uint32_t tacc = tmem_base + (uint32_t)(g * p.BN) + ((uint32_t)(quad * 32) << 16);
+            for (int cc = 0; cc < ((p.dbg & 8) ? 0 : ncols); cc += 32) {
+                uint32_t r[2][16];
+                tc::tmem_ld16_nw(tacc + cc, r[0]);
+                if (cc + 16 < ncols) tc::tmem_ld16_nw(tacc + cc + 16, r[1]);
+                tc::tmem_wait_ld();
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    const int c8 = cc + 8 * u;
+                    if (c8 >= ncols) break;
+                    const int k = c8 / p.ychunk;
+                    const uint32_t off = tc::swz((uint32_t)row * rowB + (uint32_t)(c8 - k * p.ychunk) * 2u, p.y_mask);
+                    uint4 *dst = reinterpret_cast<uint4 *>(sYb + k * chunk_bytes + off);
+                    const uint4 m4 = MASK ? *dst : make_uint4(0, 0, 0, 0);
+                    *dst = epi8<BIAS, RELU, MASK>(r[u >> 1] + 8 * (u & 1), sbias, co0 + c8, p.Cout, m4);
+                }
+            }
+            tc::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(&tempty[g]);
+            tc::fence_proxy_async_smem();
+            tc::named_bar_sync(1 + g, 128);
+            if (gtid == 0 && !(p.dbg & 1)) {
+                for (int k = 0; k < nchunks; ++k)
+                    tc::tma_store_4d(&p.mapY[ql], sYb + k * chunk_bytes, co0 + k * p.ychunk, ow0, oh0, n0);
+                tc::bulk_commit();
+            }
+            aph ^= 1;
+        }
+        if (gtid == 0) tc::bulk_wait0();
     } else if (!p.direct) {
         // ================= epilogue: warps 2..9, TMEM lane quadrant = warp % 4, column half = (warp-2)/4;
         // accumulator -> fused bias/ReLU/mask -> bf16 -> swizzled smem staging tile -> TMA store
@@ -295,7 +401,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
         const int etid = threadIdx.x - 64;     // 0..255
         const uint32_t rowB = (uint32_t)p.ychunk * 2u;
         const uint32_t chunk_bytes = 128u * rowB;
-        int acc = 0;
+        int acc = 0, yb = 0;
         uint32_t aph = 0, yph = 0;
         for (int t = blockIdx.x; t < total; t += gridDim.x) {
             int ql, nb, hb, wb, cb;
@@ -304,14 +410,18 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             const int ow0 = wb * p.BW, oh0 = hb * p.BH, n0 = nb * p.BNn;
             const int ncols = min(p.BN, p.Cpo - co0);       // channels this tile stores (multiple of ychunk)
             const int nchunks = ncols / p.ychunk;
-            // the staging tile is free once the previous tile's TMA store has read it
-            if (etid == 0) tc::bulk_wait_read0();
+            uint8_t *sYb = sY + (size_t)yb * p.ybuf_bytes;
+            // this staging buffer is free once the TMA store that last used it has read it
+            if (etid == 0) {
+                if (p.ybufs == 2) tc::bulk_wait_read1();
+                else tc::bulk_wait_read0();
+            }
             tc::named_bar_sync(1, 256);
             if (MASK) {  // ReLU-mask tile (same box as the output) into the staging tile
                 if (etid == 0) {
                     tc::mbar_arrive_expect_tx(ybar, (uint32_t)nchunks * p.rows_box * rowB);
                     for (int k = 0; k < nchunks; ++k)
-                        tc::tma_load_4d(sY + k * chunk_bytes, &p.mapR[ql], ybar, co0 + k * p.ychunk, ow0, oh0, n0);
+                        tc::tma_load_4d(sYb + k * chunk_bytes, &p.mapR[ql], ybar, co0 + k * p.ychunk, ow0, oh0, n0);
                 }
                 tc::mbar_wait(ybar, yph);
                 yph ^= 1;
@@ -330,7 +440,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     if (c8 >= ncols) break;
                     const int k = c8 / p.ychunk;
                     const uint32_t off = tc::swz((uint32_t)row * rowB + (uint32_t)(c8 - k * p.ychunk) * 2u, p.y_mask);
-                    uint4 *dst = reinterpret_cast<uint4 *>(sY + k * chunk_bytes + off);
+                    uint4 *dst = reinterpret_cast<uint4 *>(sYb + k * chunk_bytes + off);
                     const uint4 m4 = MASK ? *dst : make_uint4(0, 0, 0, 0);
                     *dst = epi8<BIAS, RELU, MASK>(r + 8 * u, sbias, co0 + c8, p.Cout, m4);
                 }
@@ -340,13 +450,14 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             if (lane == 0) tc::mbar_arrive(&tempty[acc]);   // accumulator free: the MMA may proceed
             tc::fence_proxy_async_smem();
             tc::named_bar_sync(1, 256);
-            if (etid == 0) {
+            if (etid == 0 && !(p.dbg & 1)) {
                 for (int k = 0; k < nchunks; ++k)
-                    tc::tma_store_4d(&p.mapY[ql], sY + k * chunk_bytes, co0 + k * p.ychunk, ow0, oh0, n0);
+                    tc::tma_store_4d(&p.mapY[ql], sYb + k * chunk_bytes, co0 + k * p.ychunk, ow0, oh0, n0);
                 tc::bulk_commit();
             }
             acc ^= 1;
             if (acc == 0) aph ^= 1;
+            if (p.ybufs == 2) yb ^= 1;
         }
         if (etid == 0) tc::bulk_wait0();
     } else {
@@ -563,6 +674,8 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.a3d = a3d;
         P.halo = halo;
         P.halo8 = halo8;
+        P.dbg = getenv("SPLITCNN_DBG") ? atoi(getenv("SPLITCNN_DBG")) : 0;
+        P.egroups = 1;
         P.Wp = 8 + kw - 1;
         if (cpad >= 64) {
             P.cchunks = cpad / 64; P.tps = 1; P.ksteps = kh * kw * P.cchunks;
@@ -578,6 +691,8 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.a_tx_bytes = (uint32_t)P.tps * P.rows_box * row_bytes;
         P.b_tx_bytes = (uint32_t)BN * 128u;
         P.a_stage = 16384u;
+        P.bres = 0;
+        P.bres_bytes = 0;
         if (halo8) {
             P.ksteps = 1;
             P.a_tx_bytes = (uint32_t)P.Wp * (ts.BH + kh - 1) * 16u;
@@ -588,6 +703,14 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             P.a_tx_bytes = (uint32_t)P.Wp * ts.BH * ts.BNn * 128u;
             P.a_stage = (P.a_tx_bytes + 1023u) & ~1023u;
             P.b_tx_bytes = (uint32_t)kw * BN * 128u;
+            // weights resident when they fit next to the staging tile and >= 2 A stages
+            const uint32_t wbytes = (uint32_t)(cpad / 64) * kh * kw * BN * 128u;
+            const uint32_t stg = (uint32_t)((BN + 63) / 64) * 128u * 128u;
+            if (nco == 1 && wbytes + stg + 2u * P.a_stage <= 200u * 1024u && !getenv("SPLITCNN_NO_BRES")) {
+                P.bres = 1;
+                P.bres_bytes = wbytes;
+                P.b_tx_bytes = 0;
+            }
         }
         const uint32_t stage_bytes = P.a_stage + P.b_tx_bytes;
         // output staging for the TMA-store epilogue: channel box of min(64, Cpo), swizzle to match
@@ -595,9 +718,14 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.direct = !((ych == 8 || ych == 16 || ych == 32 || ych == 64) && Lout.Cpad % ych == 0);
         P.ychunk = ych;
         P.y_mask = ych == 64 ? 7u : ych == 32 ? 3u : ych == 16 ? 1u : 0u;
-        const uint32_t staging = P.direct ? 0u : (uint32_t)((BN + ych - 1) / ych) * 128u * (uint32_t)ych * 2u;
-        P.stages = std::min<int>(8, (int)((208u * 1024u - staging) / stage_bytes));
-        P.stage_off = (uint32_t)P.stages * stage_bytes;
+        const uint32_t ybuf = P.direct ? 0u : (uint32_t)((BN + ych - 1) / ych) * 128u * (uint32_t)ych * 2u;
+        P.ybuf_bytes = (ybuf + 1023u) & ~1023u;
+        P.ybufs = (!P.direct && P.ybuf_bytes <= 32u * 1024u) ? 2 : 1;
+        P.egroups = (P.ybufs == 2 && !getenv("SPLITCNN_ONE_EPI")) ? 2 : 1;
+        const uint32_t staging = P.ybufs * P.ybuf_bytes;
+        P.stages = std::min<int>(8, (int)((208u * 1024u - staging - P.bres_bytes) / stage_bytes));
+        P.bres_off = (uint32_t)P.stages * stage_bytes;
+        P.stage_off = P.bres_off + ((P.bres_bytes + 1023u) & ~1023u);
         P.bar_off = P.stage_off + ((staging + 1023u) & ~1023u);
         uint32_t cols = 32;
         while (cols < 2u * BN) cols <<= 1;
@@ -875,7 +1003,7 @@ __global__ void __launch_bounds__(192, 1) wgrad_tc_kernel(const __grid_constant_
             }
         }
     } else if (warp == 1) {
-        if (lane == 0) {
+        {   // converged warp; elect.sync issues
             const uint32_t idesc = tc::idesc_bf16(128, p.bpt_pad * p.cbox, 1, 1);
             int stage = 0;
             uint32_t ph = 0;
@@ -884,16 +1012,16 @@ __global__ void __launch_bounds__(192, 1) wgrad_tc_kernel(const __grid_constant_
                 tc::tc_fence_after();
                 const uint32_t a_base = tc::smem_u32(sA + (size_t)stage * a_stage);
                 const uint32_t b_base = tc::smem_u32(sB + (size_t)stage * b_stage_al);
+                const uint64_t a0 = tc::smem_desc(a_base, WG_ROWS * 128, 1024, 2);
+                const uint64_t bd0 = tc::smem_desc(b_base, p.b_lbo, p.b_sbo, p.b_layout);
 #pragma unroll
-                for (int j = 0; j < WG_ROWS / 16; ++j) {
-                    const uint64_t adesc = tc::smem_desc(a_base + 2048u * j, WG_ROWS * 128, 1024, 2);
-                    const uint64_t bdesc = tc::smem_desc(b_base + p.b_kstep * j, p.b_lbo, p.b_sbo, p.b_layout);
-                    tc::mma_bf16(tmem_base, adesc, bdesc, idesc, (b != b0 || j) ? 1u : 0u);
-                }
-                tc::mma_commit(&empty[stage]);
+                for (int j = 0; j < WG_ROWS / 16; ++j)
+                    tc::mma_bf16_ws(tmem_base, a0 + (uint64_t)(128 * j), bd0 + (uint64_t)((p.b_kstep >> 4) * j), idesc,
+                                 (b != b0 || j) ? 1u : 0u);
+                tc::mma_commit_ws(&empty[stage]);
                 if (++stage == S) { stage = 0; ph ^= 1; }
             }
-            tc::mma_commit(&tfull[0]);
+            tc::mma_commit_ws(&tfull[0]);
         }
     } else {
         const int quad = warp & 3;
@@ -1018,7 +1146,7 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
             }
         }
     } else if (warp == 1) {
-        if (lane == 0) {
+        {   // converged warp; elect.sync issues
             const uint32_t idesc = tc::idesc_bf16(128, N, 1, 1);
             int stage = 0;
             uint32_t ph = 0;
@@ -1027,18 +1155,18 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
                 tc::tc_fence_after();
                 const uint32_t a_base = tc::smem_u32(sA + (size_t)stage * a_stage);
                 const uint32_t b_base = tc::smem_u32(sB + (size_t)stage * b_stage);
-                for (int j = 0; j < rows / 16; ++j) {
-                    // A: dY, MN-major: 8-pixel K groups at 1 KB, the second 64-co block at LBO = a_blk
-                    const uint64_t adesc = tc::smem_desc(a_base + 2048u * j, a_blk, 1024, 2);
-                    // B: X halo view, MN-major: tap c = MN block c at LBO = 128 B, K groups (output rows)
-                    //    at SBO = Wp rows; 16 pixels = 2 output rows
-                    const uint64_t bdesc = tc::smem_desc(b_base + (uint32_t)(2 * j * Wp) * 128u, 128, (uint32_t)Wp * 128u, 2);
-                    tc::mma_bf16(tmem_base, adesc, bdesc, idesc, (b != b0 || j) ? 1u : 0u);
-                }
-                tc::mma_commit(&empty[stage]);
+                // A: dY, MN-major: 8-pixel K groups at 1 KB, the second 64-co block at LBO = a_blk
+                // B: X halo view, MN-major: tap c = MN block c at LBO = 128 B, K groups (output rows)
+                //    at SBO = Wp rows; 16 pixels = 2 output rows.  Per-MMA descriptors = base + constant.
+                const uint64_t a0 = tc::smem_desc(a_base, a_blk, 1024, 2);
+                const uint64_t bd0 = tc::smem_desc(b_base, 128, (uint32_t)Wp * 128u, 2);
+                const uint64_t bstep = (uint64_t)(2 * Wp * 8);   // 2 rows of Wp pixels x 128 B, >> 4
+                for (int j = 0; j < rows / 16; ++j)
+                    tc::mma_bf16_ws(tmem_base, a0 + (uint64_t)(128 * j), bd0 + bstep * j, idesc, (b != b0 || j) ? 1u : 0u);
+                tc::mma_commit_ws(&empty[stage]);
                 if (++stage == S) { stage = 0; ph ^= 1; }
             }
-            tc::mma_commit(&tfull[0]);
+            tc::mma_commit_ws(&tfull[0]);
         }
     } else {
         const int quad = warp & 3;
@@ -1148,7 +1276,7 @@ __global__ void __launch_bounds__(192, 1) wgrad_narrow_kernel(const __grid_const
             }
         }
     } else if (warp == 1) {
-        if (lane == 0) {
+        {   // converged warp; elect.sync issues
             const uint32_t idesc = tc::idesc_bf16(128, 16, 1, 1);
             int stage = 0;
             uint32_t ph = 0;
@@ -1165,13 +1293,13 @@ __global__ void __launch_bounds__(192, 1) wgrad_narrow_kernel(const __grid_const
                         const int o1 = t1 < KT ? (t1 / p.kw) * Wp + (t1 % p.kw) : o0 + 1;
                         const uint64_t bdesc = tc::smem_desc(b_base + (uint32_t)(2 * j * Wp + o0) * 16u, (uint32_t)Wp * 16u,
                                                              (uint32_t)(o1 - o0) * 16u, 0);
-                        tc::mma_bf16(tmem_base + 16u * pr, adesc, bdesc, idesc, (b != b0 || j) ? 1u : 0u);
+                        tc::mma_bf16_ws(tmem_base + 16u * pr, adesc, bdesc, idesc, (b != b0 || j) ? 1u : 0u);
                     }
                 }
-                tc::mma_commit(&empty[stage]);
+                tc::mma_commit_ws(&empty[stage]);
                 if (++stage == S) { stage = 0; ph ^= 1; }
             }
-            tc::mma_commit(&tfull[0]);
+            tc::mma_commit_ws(&tfull[0]);
         }
     } else {
         const int quad = warp & 3;

@@ -16,8 +16,11 @@ class SplitPlan:
 
     def __del__(self):
         h = getattr(self, "handle", None)
-        if h:
-            sc.splitcnn_plan_destroy(h)
+        if h and sc is not None and getattr(sc, "splitcnn_plan_destroy", None) is not None:
+            try:
+                sc.splitcnn_plan_destroy(h)
+            except Exception:   # interpreter teardown
+                pass
             self.handle = None
 
     @property

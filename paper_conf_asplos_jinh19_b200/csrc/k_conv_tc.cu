@@ -705,8 +705,8 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             P.b_tx_bytes = (uint32_t)kw * BN * 128u;
             // weights resident when they fit next to the staging tile and >= 2 A stages
             const uint32_t wbytes = (uint32_t)(cpad / 64) * kh * kw * BN * 128u;
-            const uint32_t stg = (uint32_t)((BN + 63) / 64) * 128u * 128u;
-            if (nco == 1 && wbytes + stg + 2u * P.a_stage <= 200u * 1024u && !getenv("SPLITCNN_NO_BRES")) {
+            const uint32_t stg = (uint32_t)((BN + 63) / 64) * 128u * 128u;   // one staging buffer
+            if (nco == 1 && wbytes + stg + 2u * P.a_stage <= 206u * 1024u && !getenv("SPLITCNN_NO_BRES")) {
                 P.bres = 1;
                 P.bres_bytes = wbytes;
                 P.b_tx_bytes = 0;
@@ -721,9 +721,10 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         const uint32_t ybuf = P.direct ? 0u : (uint32_t)((BN + ych - 1) / ych) * 128u * (uint32_t)ych * 2u;
         P.ybuf_bytes = (ybuf + 1023u) & ~1023u;
         P.ybufs = (!P.direct && P.ybuf_bytes <= 32u * 1024u) ? 2 : 1;
+        if (P.bres && P.bres_bytes + 2u * P.ybuf_bytes + 2u * P.a_stage > 206u * 1024u) P.ybufs = 1;
         P.egroups = (P.ybufs == 2 && !getenv("SPLITCNN_ONE_EPI")) ? 2 : 1;
         const uint32_t staging = P.ybufs * P.ybuf_bytes;
-        P.stages = std::min<int>(8, (int)((208u * 1024u - staging - P.bres_bytes) / stage_bytes));
+        P.stages = std::min<int>(8, (int)((210u * 1024u - staging - P.bres_bytes) / stage_bytes));
         P.bres_off = (uint32_t)P.stages * stage_bytes;
         P.stage_off = P.bres_off + ((P.bres_bytes + 1023u) & ~1023u);
         P.bar_off = P.stage_off + ((staging + 1023u) & ~1023u);
@@ -1277,7 +1278,10 @@ __global__ void __launch_bounds__(192, 1) wgrad_narrow_kernel(const __grid_const
         }
     } else if (warp == 1) {
         {   // converged warp; elect.sync issues
-            const uint32_t idesc = tc::idesc_bf16(128, 16, 1, 1);
+            // per kernel row r: the kw column taps are kw 8-channel MN blocks of ONE MMA (consecutive
+            // pixels, SBO = 16 B); output-row K groups at LBO = Wp*16 B; N = kw*8 rounded up to 16
+            const int NR = ((p.kw * 8 + 15) / 16) * 16;
+            const uint32_t idesc = tc::idesc_bf16(128, NR, 1, 1);
             int stage = 0;
             uint32_t ph = 0;
             for (int b = b0; b < b1; ++b) {
@@ -1285,17 +1289,12 @@ __global__ void __launch_bounds__(192, 1) wgrad_narrow_kernel(const __grid_const
                 tc::tc_fence_after();
                 const uint32_t a_base = tc::smem_u32(sA + (size_t)stage * a_stage);
                 const uint32_t b_base = tc::smem_u32(sB + (size_t)stage * b_stage);
-                for (int j = 0; j < rows / 16; ++j) {
-                    const uint64_t adesc = tc::smem_desc(a_base + 2048u * j, a_blk, 1024, 2);
-                    for (int pr = 0; pr < npairs; ++pr) {
-                        const int t0 = 2 * pr, t1 = 2 * pr + 1;
-                        const int o0 = (t0 / p.kw) * Wp + (t0 % p.kw);
-                        const int o1 = t1 < KT ? (t1 / p.kw) * Wp + (t1 % p.kw) : o0 + 1;
-                        const uint64_t bdesc = tc::smem_desc(b_base + (uint32_t)(2 * j * Wp + o0) * 16u, (uint32_t)Wp * 16u,
-                                                             (uint32_t)(o1 - o0) * 16u, 0);
-                        tc::mma_bf16_ws(tmem_base + 16u * pr, adesc, bdesc, idesc, (b != b0 || j) ? 1u : 0u);
-                    }
-                }
+                const uint64_t a0 = tc::smem_desc(a_base, a_blk, 1024, 2);
+                const uint64_t bd0 = tc::smem_desc(b_base, (uint32_t)Wp * 16u, 16, 0);
+                for (int j = 0; j < rows / 16; ++j)
+                    for (int r = 0; r < p.kh; ++r)
+                        tc::mma_bf16_ws(tmem_base + (uint32_t)(r * NR), a0 + (uint64_t)(128 * j),
+                                        bd0 + (uint64_t)((2 * j + r) * Wp), idesc, (b != b0 || j) ? 1u : 0u);
                 tc::mma_commit_ws(&empty[stage]);
                 if (++stage == S) { stage = 0; ph ^= 1; }
             }
@@ -1310,24 +1309,26 @@ __global__ void __launch_bounds__(192, 1) wgrad_narrow_kernel(const __grid_const
             tc::tc_fence_after();
         }
         const uint32_t tacc = tmem_base + ((uint32_t)(quad * 32) << 16);
-        for (int pr = 0; pr < npairs; ++pr) {
-            float v[16];
-            if (any) {
-                tc::tmem_ld16(tacc + 16u * pr, v);
-            } else {
+        const int NR = ((p.kw * 8 + 15) / 16) * 16;
+        for (int r = 0; r < p.kh; ++r)
+            for (int cc = 0; cc < NR; cc += 16) {
+                float v[16];
+                if (any) {
+                    tc::tmem_ld16(tacc + (uint32_t)(r * NR + cc), v);
+                } else {
 #pragma unroll
-                for (int e = 0; e < 16; ++e) v[e] = 0.f;
-            }
-            if (co >= p.Cout) continue;
+                    for (int e = 0; e < 16; ++e) v[e] = 0.f;
+                }
+                if (co >= p.Cout) continue;
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                const int tap = 2 * pr + h;
-                if (tap >= KT) break;
-                float4 *d4 = reinterpret_cast<float4 *>(p.part + (((int64_t)z * p.Cout + co) * KT + tap) * 8);
-                d4[0] = make_float4(v[8 * h], v[8 * h + 1], v[8 * h + 2], v[8 * h + 3]);
-                d4[1] = make_float4(v[8 * h + 4], v[8 * h + 5], v[8 * h + 6], v[8 * h + 7]);
+                for (int h = 0; h < 2; ++h) {
+                    const int c = (cc >> 3) + h;          // column tap of this 8-channel block
+                    if (c >= p.kw) break;
+                    float4 *d4 = reinterpret_cast<float4 *>(p.part + (((int64_t)z * p.Cout + co) * KT + r * p.kw + c) * 8);
+                    d4[0] = make_float4(v[8 * h], v[8 * h + 1], v[8 * h + 2], v[8 * h + 3]);
+                    d4[1] = make_float4(v[8 * h + 4], v[8 * h + 5], v[8 * h + 6], v[8 * h + 7]);
+                }
             }
-        }
     }
     tc::tc_fence_before();
     __syncthreads();
@@ -1468,7 +1469,7 @@ size_t wgrad_tc_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g) {
             WgHaloCfg h = wgrad_halo_cfg(Li, Lo, g, g0, std::min(np, g0 + TC_MAXP));
             best = std::max(best, (size_t)h.nsplit * g.L.cout * g.L.kh * g.L.kw * Li.Cpad * sizeof(float));
         }
-        if (wgrad_narrow_ok(Li, Lo, g) && getenv("SPLITCNN_NARROW_WGRAD")) {
+        if (wgrad_narrow_ok(Li, Lo, g) && !getenv("SPLITCNN_NO_NARROW_WGRAD")) {
             WgNarrowCfg h = wgrad_narrow_cfg(Lo, g, g0, std::min(np, g0 + TC_MAXP));
             best = std::max(best, (size_t)h.nsplit * g.L.cout * g.L.kh * g.L.kw * Li.Cpad * sizeof(float));
         }
@@ -1490,8 +1491,7 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
     static bool attr_set = false;
     bool first = true;
     int gend = p1;  // end of the patch range left for the generic kernel
-    // opt-in: correct, but slower than the generic multi-tap path on conv1_1 so far (many N = 16 MMAs)
-    if (wgrad_narrow_ok(Li, Lo, g) && getenv("SPLITCNN_NARROW_WGRAD")) {
+    if (wgrad_narrow_ok(Li, Lo, g) && !getenv("SPLITCNN_NO_NARROW_WGRAD")) {
         static bool narrow_attr = false;
         for (int g0 = p0; g0 < p1; g0 += TC_MAXP) {
             const int g1 = std::min(p1, g0 + TC_MAXP);
@@ -1508,7 +1508,7 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
             const uint32_t stage_bytes = a_stage + b_stage;
             P.stages = std::min<int>(8, (int)((200u * 1024u) / stage_bytes));
             uint32_t cols = 32;
-            while (cols < (uint32_t)(16 * ((g.L.kh * g.L.kw + 1) / 2))) cols <<= 1;
+            while (cols < (uint32_t)(g.L.kh * (((g.L.kw * 8 + 15) / 16) * 16))) cols <<= 1;
             P.tmem_cols = cols;
             P.part = part;
             int boxes = 0;

@@ -77,10 +77,29 @@ struct TcConvParams {
     int ybufs;                    // staging buffers (2: the TMA store of tile t overlaps tile t+1)
     int dbg;                      // experiments only (SPLITCNN_DBG): 1 no TMA store, 2 no MMA, 4 no loads, 8 no TMEM->smem
     int egroups;                  // 2: two independent 4-warp epilogue groups, one per TMEM accumulator
+    int cta2;                     // 2-CTA MMA (cluster of 2, M = 256): each CTA owns one 128-row M box and N/2 of B
+    int BNh;                      // rows of B per CTA (BN / 2 in 2-CTA mode, else BN)
+    int total_m, total_pairs, m_tpp;
+    int m_prefix[TC_MAXP + 1];
     uint32_t ybuf_bytes;
 };
 
-static_assert(sizeof(TcConvParams) <= 32000, "kernel parameter space is 32 KB");
+static_assert(sizeof(TcConvParams) <= 32700, "kernel parameter space is 32 KB");
+
+// 2-CTA mode: M box index (across patches) -> patch, image block, row block, column block
+__device__ __forceinline__ void decode_mbox(const TcConvParams &p, int m, int &ql, int &nb, int &hb, int &wb) {
+    if (p.m_tpp) {
+        ql = m / p.m_tpp;
+    } else {
+        ql = 0;
+        while (m >= p.m_prefix[ql + 1]) ++ql;
+    }
+    int idx = m - p.m_prefix[ql];
+    wb = idx % p.nwb[ql];
+    idx /= p.nwb[ql];
+    hb = idx % p.nhb[ql];
+    nb = idx / p.nhb[ql];
+}
 
 __device__ __forceinline__ void decode_tile(const TcConvParams &p, int t, int &ql, int &nb, int &hb, int &wb, int &cb) {
     if (p.tpp) {
@@ -97,6 +116,23 @@ __device__ __forceinline__ void decode_tile(const TcConvParams &p, int t, int &q
     hb = idx % p.nhb[ql];
     nb = idx / p.nhb[ql];
 }
+
+// work item t of this CTA -> (patch, image block, row block, column block, co block); `valid` false for
+// the idle second half of an odd last pair
+__device__ __forceinline__ void get_tile(const TcConvParams &p, int t, uint32_t rank, int &ql, int &nb, int &hb, int &wb,
+                                         int &cb, bool &valid) {
+    if (p.cta2) {
+        cb = t % p.nco;
+        int m = 2 * (t / p.nco) + (int)rank;
+        valid = m < p.total_m;
+        m = min(m, p.total_m - 1);
+        decode_mbox(p, m, ql, nb, hb, wb);
+    } else {
+        decode_tile(p, t, ql, nb, hb, wb, cb);
+        valid = true;
+    }
+}
+
 
 constexpr int CONV_THREADS = 64 + 256;  // producer warp, MMA warp, 8 epilogue warps (2 per TMEM lane quadrant)
 
@@ -137,7 +173,7 @@ __device__ __forceinline__ uint4 epi8(const uint32_t *r, const float *sb, int co
     return pk;
 }
 
-template <bool BIAS, bool RELU, bool MASK>
+template <bool BIAS, bool RELU, bool MASK, bool CTA2>
 __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_constant__ TcConvParams p) {
     extern __shared__ uint8_t smem_raw[];
     uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -157,6 +193,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
     float *sbias = (float *)(smem + p.bar_off + 512);   // [Cout] bias (16-byte aligned)
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t rank = CTA2 ? tc::cluster_ctarank() : 0u;
+    const bool leader = rank == 0;
     if (warp == 0 && lane == 0) {
         for (int s = 0; s < S; ++s) {
             tc::mbar_init(&full[s], 1);
@@ -164,7 +202,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
         }
         for (int a = 0; a < 2; ++a) {
             tc::mbar_init(&tfull[a], 1);
-            tc::mbar_init(&tempty[a], p.egroups == 2 ? 4 : 8);
+            // the leader's accumulator-empty barrier hears both CTAs' epilogues in 2-CTA mode
+            tc::mbar_init(&tempty[a], (p.egroups == 2 ? 4 : 8) * (CTA2 ? 2 : 1));
         }
         tc::mbar_init(ybar, 1);
         tc::mbar_init(wbar, 1);
@@ -173,12 +212,18 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
     }
     if (BIAS)
         for (int i = threadIdx.x; i < p.Cout; i += blockDim.x) sbias[i] = __ldg(p.bias + i);
-    if (warp == 1) tc::tmem_alloc_dyn(tmem_slot, p.tmem_cols);
+    if (warp == 1) {
+        if (CTA2) tc::tmem_alloc2(tmem_slot, p.tmem_cols);
+        else tc::tmem_alloc_dyn(tmem_slot, p.tmem_cols);
+    }
     tc::tc_fence_before();
-    __syncthreads();
+    if (CTA2) tc::cluster_sync_all();
+    else __syncthreads();
     tc::tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
-    const int total = p.tile_prefix[p.npatch];
+    const int total = CTA2 ? p.total_pairs : p.tile_prefix[p.npatch];
+    const int tfirst = CTA2 ? (int)tc::cluster_id_x() : (int)blockIdx.x;
+    const int tstep = CTA2 ? (int)tc::nclusters_x() : (int)gridDim.x;
     const int KT = p.kh * p.kw;
 
     if (warp == 0) {
@@ -186,13 +231,23 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             // ================= TMA producer
             for (int q = 0; q < p.npatch; ++q) tc::tma_prefetch_desc(&p.mapA[q]);
             tc::tma_prefetch_desc(&p.mapB);
+            const uint32_t wbar_l = CTA2 ? tc::mapa_shared(wbar, 0) : 0u;
             if (p.bres) {  // every (chunk, kernel row) weight box once, for all tiles of this CTA
-                tc::mbar_arrive_expect_tx(wbar, p.bres_bytes);
+                const int rowB0 = (int)rank * p.BNh;  // 2-CTA: this CTA holds rows [rank*BN/2, +BN/2) of B
+                if (!CTA2) tc::mbar_arrive_expect_tx(wbar, p.bres_bytes);
+                else if (leader) tc::mbar_arrive_expect_tx(wbar, 2 * p.bres_bytes);
                 const int nchunk = p.kchan / 64;
                 for (int cc = 0; cc < nchunk; ++cc)
                     for (int r = 0; r < p.kh; ++r) {
-                        uint8_t *dst = sW + (size_t)((cc * p.kh + r) * p.kw) * p.BN * 128;
-                        if (p.b3d) {
+                        uint8_t *dst = sW + (size_t)((cc * p.kh + r) * p.kw) * p.BNh * 128;
+                        if (CTA2) {
+                            if (p.b3d) {
+                                tc::tma2_load_3d(dst, &p.mapB, wbar_l, cc * 64, rowB0, r * p.kw);
+                            } else {
+                                for (int c = 0; c < p.kw; ++c)
+                                    tc::tma2_load_2d(dst + c * p.BNh * 128, &p.mapB, wbar_l, (r * p.kw + c) * p.kchan + cc * 64, rowB0);
+                            }
+                        } else if (p.b3d) {
                             tc::tma_load_3d(dst, &p.mapB, wbar, cc * 64, 0, r * p.kw);
                         } else {
                             for (int c = 0; c < p.kw; ++c)
@@ -202,9 +257,10 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             }
             int stage = 0;
             uint32_t ph = 0;
-            for (int t = blockIdx.x; t < total; t += gridDim.x) {
+            for (int t = tfirst; t < total; t += tstep) {
                 int ql, nb, hb, wb, cb;
-                decode_tile(p, t, ql, nb, hb, wb, cb);
+                bool valid;
+                get_tile(p, t, rank, ql, nb, hb, wb, cb, valid);
                 const int wbase = wb * p.BW * p.s - p.pl[ql];
                 const int hbase = hb * p.BH * p.s - p.pt[ql];
                 const int n0 = nb * p.BNn, co0 = cb * p.BN;
@@ -216,9 +272,34 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                         if (++stage == S) { stage = 0; ph ^= 1; }
                         continue;
                     }
-                    tc::mbar_arrive_expect_tx(&full[stage], p.a_tx_bytes + p.b_tx_bytes);
                     uint8_t *a = sA + (size_t)stage * p.a_stage;
                     uint8_t *b = sB + (size_t)stage * b_stage;
+                    if (CTA2) {
+                        // both CTAs load their own A box and their half of B; bytes land on the leader's barrier
+                        const uint32_t fb = tc::mapa_shared(&full[stage], 0);
+                        if (leader) tc::mbar_arrive_expect_tx(&full[stage], 2 * (p.a_tx_bytes + p.b_tx_bytes));
+                        const int cor = co0 + (int)rank * p.BNh;
+                        if (p.halo) {
+                            const int cc = ks / p.kh, r = ks - cc * p.kh;
+                            tc::tma2_load_4d(a, &p.mapA[ql], fb, cc * 64, wbase, hbase + r, n0);
+                            if (!p.bres) {
+                                if (p.b3d) {
+                                    tc::tma2_load_3d(b, &p.mapB, fb, cc * 64, cor, r * p.kw);
+                                } else {
+                                    for (int c = 0; c < p.kw; ++c)
+                                        tc::tma2_load_2d(b + c * p.BNh * 128, &p.mapB, fb, (r * p.kw + c) * p.kchan + cc * 64, cor);
+                                }
+                            }
+                        } else {
+                            const int tap = ks / p.cchunks, cc = ks - tap * p.cchunks;
+                            const int r = tap / p.kw, c = tap - r * p.kw;
+                            tc::tma2_load_4d(a, &p.mapA[ql], fb, cc * 64, wbase + c, hbase + r, n0);
+                            tc::tma2_load_2d(b, &p.mapB, fb, tap * p.kchan + cc * 64, cor);
+                        }
+                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        continue;
+                    }
+                    tc::mbar_arrive_expect_tx(&full[stage], p.a_tx_bytes + p.b_tx_bytes);
                     if (p.halo8) {
                         // rows (h) x (8 + kw - 1) pixels x 8 channels; the weights' K = taps*8 in 64-wide boxes
                         tc::tma_load_3d(a, &p.mapA[ql], &full[stage], 8 * wbase, hbase, n0);
@@ -256,12 +337,13 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
         }
     } else if (warp == 1) {
         {
-            // ================= MMA issuer: the whole warp runs the loop converged; elect.sync issues
-            const uint32_t idesc = tc::idesc_bf16(128, p.BN);
+            // ================= MMA issuer: the whole warp runs the loop converged; elect.sync issues.
+            // In 2-CTA mode only the leader issues (M = 256 over the pair); the peer's warp 1 idles.
+            const uint32_t idesc = tc::idesc_bf16(CTA2 ? 256 : 128, p.BN);
             int stage = 0, acc = 0;
             uint32_t ph = 0, aph = 0;
-            if (p.bres) tc::mbar_wait(wbar, 0);
-            for (int t = blockIdx.x; t < total; t += gridDim.x) {
+            if (p.bres && leader) tc::mbar_wait(wbar, 0);
+            for (int t = leader ? tfirst : total; t < total; t += tstep) {
                 tc::mbar_wait_sleep(&tempty[acc], aph ^ 1);
                 tc::tc_fence_after();
                 const uint32_t d = tmem_base + (uint32_t)(acc * p.BN);
@@ -291,6 +373,31 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                             tc::mma_bf16_ws(d, adesc, bdesc, idesc, (ks | pr) != 0);
                         }
                         tc::mma_commit_ws(&empty[stage]);
+                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        continue;
+                    }
+                    if (p.halo && CTA2) {
+                        const uint64_t a0 = tc::smem_desc(a_base, 16, (uint32_t)p.Wp * 128u, 2);
+                        const uint64_t b0 = p.bres ? tc::smem_desc(tc::smem_u32(sW) + (uint32_t)(ks * p.kw * p.BNh) * 128u, 16, 1024, 2)
+                                                   : tc::smem_desc(b_base, 16, 1024, 2);
+                        const uint32_t bstep = (uint32_t)p.BNh * 8u;
+                        for (int c = 0; c < p.kw; ++c) {
+                            const uint64_t ac = a0 + (uint64_t)(8 * c), bc = b0 + (uint64_t)(bstep * c);
+                            tc::mma2_bf16_ws(d, ac, bc, idesc, (ks | c) != 0);
+                            tc::mma2_bf16_ws(d, ac + 2, bc + 2, idesc, 1u);
+                            tc::mma2_bf16_ws(d, ac + 4, bc + 4, idesc, 1u);
+                            tc::mma2_bf16_ws(d, ac + 6, bc + 6, idesc, 1u);
+                        }
+                        tc::mma2_commit_mc_ws(&empty[stage]);
+                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        continue;
+                    }
+                    if (CTA2) {
+                        const uint64_t a0 = tc::smem_desc(a_base, 16, 1024, 2);
+                        const uint64_t b0 = tc::smem_desc(b_base, 16, 1024, 2);
+#pragma unroll
+                        for (int j = 0; j < 4; ++j) tc::mma2_bf16_ws(d, a0 + (uint64_t)(2 * j), b0 + (uint64_t)(2 * j), idesc, (ks | j) != 0);
+                        tc::mma2_commit_mc_ws(&empty[stage]);
                         if (++stage == S) { stage = 0; ph ^= 1; }
                         continue;
                     }
@@ -325,7 +432,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     tc::mma_commit_ws(&empty[stage]);
                     if (++stage == S) { stage = 0; ph ^= 1; }
                 }
-                tc::mma_commit_ws(&tfull[acc]);
+                if (CTA2) tc::mma2_commit_mc_ws(&tfull[acc]);
+                else tc::mma_commit_ws(&tfull[acc]);
                 acc ^= 1;
                 if (acc == 0) aph ^= 1;
             }
@@ -342,16 +450,18 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
         uint8_t *sYb = sY + (size_t)g * p.ybuf_bytes;
         uint64_t *mbar = g ? wbar + 1 : ybar;
         uint32_t aph = 0, yph = 0;
-        for (int t = blockIdx.x + g * gridDim.x; t < total; t += 2 * gridDim.x) {
+        const uint32_t tempty_l = tc::mapa_shared(&tempty[g], 0);   // the leader's (own in 1-CTA mode)
+        for (int t = tfirst + g * tstep; t < total; t += 2 * tstep) {
             int ql, nb, hb, wb, cb;
-            decode_tile(p, t, ql, nb, hb, wb, cb);
+            bool valid;
+            get_tile(p, t, rank, ql, nb, hb, wb, cb, valid);
             const int co0 = cb * p.BN;
             const int ow0 = wb * p.BW, oh0 = hb * p.BH, n0 = nb * p.BNn;
             const int ncols = min(p.BN, p.Cpo - co0);
             const int nchunks = ncols / p.ychunk;
             if (gtid == 0) tc::bulk_wait_read0();      // this group's previous store has read the staging
             tc::named_bar_sync(1 + g, 128);
-            if (MASK) {
+            if (MASK && valid) {
                 if (gtid == 0) {
                     tc::mbar_arrive_expect_tx(mbar, (uint32_t)nchunks * p.rows_box * rowB);
                     for (int k = 0; k < nchunks; ++k)
@@ -381,10 +491,13 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             }
             tc::tc_fence_before();
             __syncwarp();
-            if (lane == 0) tc::mbar_arrive(&tempty[g]);
+            if (lane == 0) {
+                if (CTA2) tc::mbar_arrive_remote(tempty_l);
+                else tc::mbar_arrive(&tempty[g]);
+            }
             tc::fence_proxy_async_smem();
             tc::named_bar_sync(1 + g, 128);
-            if (gtid == 0 && !(p.dbg & 1)) {
+            if (gtid == 0 && valid && !(p.dbg & 1)) {
                 for (int k = 0; k < nchunks; ++k)
                     tc::tma_store_4d(&p.mapY[ql], sYb + k * chunk_bytes, co0 + k * p.ychunk, ow0, oh0, n0);
                 tc::bulk_commit();
@@ -403,9 +516,10 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
         const uint32_t chunk_bytes = 128u * rowB;
         int acc = 0, yb = 0;
         uint32_t aph = 0, yph = 0;
-        for (int t = blockIdx.x; t < total; t += gridDim.x) {
+        for (int t = tfirst; t < total; t += tstep) {
             int ql, nb, hb, wb, cb;
-            decode_tile(p, t, ql, nb, hb, wb, cb);
+            bool valid;
+            get_tile(p, t, rank, ql, nb, hb, wb, cb, valid);
             const int co0 = cb * p.BN;
             const int ow0 = wb * p.BW, oh0 = hb * p.BH, n0 = nb * p.BNn;
             const int ncols = min(p.BN, p.Cpo - co0);       // channels this tile stores (multiple of ychunk)
@@ -417,7 +531,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 else tc::bulk_wait_read0();
             }
             tc::named_bar_sync(1, 256);
-            if (MASK) {  // ReLU-mask tile (same box as the output) into the staging tile
+            if (MASK && valid) {  // ReLU-mask tile (same box as the output) into the staging tile
                 if (etid == 0) {
                     tc::mbar_arrive_expect_tx(ybar, (uint32_t)nchunks * p.rows_box * rowB);
                     for (int k = 0; k < nchunks; ++k)
@@ -447,10 +561,13 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             }
             tc::tc_fence_before();
             __syncwarp();
-            if (lane == 0) tc::mbar_arrive(&tempty[acc]);   // accumulator free: the MMA may proceed
+            if (lane == 0) {   // accumulator free: the MMA may proceed (the leader's barrier in 2-CTA mode)
+                if (CTA2) tc::mbar_arrive_remote(tc::mapa_shared(&tempty[acc], 0));
+                else tc::mbar_arrive(&tempty[acc]);
+            }
             tc::fence_proxy_async_smem();
             tc::named_bar_sync(1, 256);
-            if (etid == 0 && !(p.dbg & 1)) {
+            if (etid == 0 && valid && !(p.dbg & 1)) {
                 for (int k = 0; k < nchunks; ++k)
                     tc::tma_store_4d(&p.mapY[ql], sYb + k * chunk_bytes, co0 + k * p.ychunk, ow0, oh0, n0);
                 tc::bulk_commit();
@@ -527,9 +644,13 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
         }
     }
     tc::tc_fence_before();
-    __syncthreads();
+    if (CTA2) tc::cluster_sync_all();   // the peer's MMAs write this CTA's TMEM until the leader is done
+    else __syncthreads();
     tc::tc_fence_after();
-    if (warp == 1) tc::tmem_dealloc(tmem_base, p.tmem_cols);
+    if (warp == 1) {
+        if (CTA2) tc::tmem_dealloc2(tmem_base, p.tmem_cols);
+        else tc::tmem_dealloc(tmem_base, p.tmem_cols);
+    }
 }
 
 // dgrad weights: W'[ci][r'][c'][co] = W[co][kh-1-r'][kw-1-c'][ci], zero for co >= Cout
@@ -693,6 +814,17 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.a_stage = 16384u;
         P.bres = 0;
         P.bres_bytes = 0;
+        // 2-CTA pairs (M = 256): halves each CTA's shared-memory operand traffic per MMA (the 1-CTA
+        // kernel is bound by it at N <= 256); needs 64-channel SW128 A boxes and >= 32 output columns
+        {
+            const int ych0 = std::min(64, Lout.Cpad);
+            const bool tma_out = (ych0 == 8 || ych0 == 16 || ych0 == 32 || ych0 == 64) && Lout.Cpad % ych0 == 0;
+            long mb = 0;
+            for (auto &e : ext) mb += (long)P.nnb * ((e.first + ts.BH - 1) / ts.BH) * ((e.second + ts.BW - 1) / ts.BW);
+            P.cta2 = (cpad % 64 == 0 && !halo8 && !a3d && BN % 32 == 0 && tma_out && mb >= 2 && !getenv("SPLITCNN_NO_CTA2")) ? 1 : 0;
+        }
+        P.BNh = P.cta2 ? BN / 2 : BN;
+        if (P.cta2) P.b_tx_bytes = (uint32_t)P.BNh * 128u;
         if (halo8) {
             P.ksteps = 1;
             P.a_tx_bytes = (uint32_t)P.Wp * (ts.BH + kh - 1) * 16u;
@@ -702,9 +834,9 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             P.ksteps = (cpad / 64) * kh;
             P.a_tx_bytes = (uint32_t)P.Wp * ts.BH * ts.BNn * 128u;
             P.a_stage = (P.a_tx_bytes + 1023u) & ~1023u;
-            P.b_tx_bytes = (uint32_t)kw * BN * 128u;
+            P.b_tx_bytes = (uint32_t)kw * P.BNh * 128u;
             // weights resident when they fit next to the staging tile and >= 2 A stages
-            const uint32_t wbytes = (uint32_t)(cpad / 64) * kh * kw * BN * 128u;
+            const uint32_t wbytes = (uint32_t)(cpad / 64) * kh * kw * P.BNh * 128u;
             const uint32_t stg = (uint32_t)((BN + 63) / 64) * 128u * 128u;   // one staging buffer
             if (nco == 1 && wbytes + stg + 2u * P.a_stage <= 206u * 1024u && !getenv("SPLITCNN_NO_BRES")) {
                 P.bres = 1;
@@ -735,7 +867,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.y = (__nv_bfloat16 *)y;
         P.relu_src = (const __nv_bfloat16 *)relu_src;
         P.relu = relu;
-        int tiles = 0;
+        int tiles = 0, mboxes = 0;
         for (int q = g0; q < g1; ++q) {
             const int ql = q - g0;
             const int i = q / Lout.nw(), j = q % Lout.nw();
@@ -749,6 +881,8 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             P.nwb[ql] = (ow + ts.BW - 1) / ts.BW;
             P.tile_prefix[ql] = tiles;
             tiles += P.nnb * P.nhb[ql] * P.nwb[ql] * nco;
+            P.m_prefix[ql] = mboxes;
+            mboxes += P.nnb * P.nhb[ql] * P.nwb[ql];
             // A map over the patch buffer: dims (C, W, H, N), TMA zero fill = patch padding
             const int hp = La.ph(i), wp = La.pw(j);
             void *base = (char *)a_ptr + La.offset(i, j) * 2;
@@ -794,6 +928,12 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             }
         }
         P.tile_prefix[P.npatch] = tiles;
+        P.m_prefix[P.npatch] = mboxes;
+        P.total_m = mboxes;
+        P.total_pairs = ((mboxes + 1) / 2) * nco;
+        P.m_tpp = P.m_prefix[1];
+        for (int ql = 1; ql < P.npatch; ++ql)
+            if (P.m_prefix[ql + 1] - P.m_prefix[ql] != P.m_tpp) P.m_tpp = 0;
         P.tpp = P.tile_prefix[1];
         for (int ql = 1; ql < P.npatch; ++ql)
             if (P.tile_prefix[ql + 1] - P.tile_prefix[ql] != P.tpp) P.tpp = 0;
@@ -801,14 +941,14 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             const int K = kh * kw * cpad;
             cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)w_rows};
             cuuint64_t strides[1] = {(cuuint64_t)K * 2};
-            cuuint32_t box[2] = {64, (cuuint32_t)BN};
+            cuuint32_t box[2] = {64, (cuuint32_t)P.BNh};
             cuuint32_t es[2] = {1, 1};
             CUresult r = CUDA_ERROR_INVALID_VALUE;
             P.b3d = 0;
             if (halo) {  // (ci, co, tap) view of [Cout][taps][Cpad]: one box = the kw taps of a kernel row
                 cuuint64_t d3[3] = {(cuuint64_t)cpad, (cuuint64_t)w_rows, (cuuint64_t)(kh * kw)};
                 cuuint64_t s3[2] = {(cuuint64_t)K * 2, (cuuint64_t)cpad * 2};
-                cuuint32_t b3[3] = {64, (cuuint32_t)BN, (cuuint32_t)kw};
+                cuuint32_t b3[3] = {64, (cuuint32_t)P.BNh, (cuuint32_t)kw};
                 cuuint32_t e3[3] = {1, 1, 1};
                 r = encode(&P.mapB, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void *>(w_ptr), d3, s3, b3, e3,
                            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -823,25 +963,56 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         }
         if (tiles == 0) continue;
         const size_t smem = 1024 + (size_t)P.bar_off + 512 + (bias ? 4 * (size_t)g.L.cout : 0) + 64;
-        const int grid = std::min(tiles, num_sms());
+        const int grid = P.cta2 ? 2 * std::min(P.total_pairs, num_sms() / 2) : std::min(tiles, num_sms());
         const int mode_bits = (bias ? 4 : 0) | (relu ? 2 : 0) | (relu_src ? 1 : 0);
         auto launch = [&](auto kern) {
-            static bool set[8] = {false};
-            if (!set[mode_bits]) {
+            static bool set[16] = {false};
+            const int key = mode_bits + (P.cta2 ? 8 : 0);
+            if (!set[key]) {
                 cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-                set[mode_bits] = true;
+                set[key] = true;
             }
-            kern<<<grid, CONV_THREADS, smem, st>>>(P);
+            if (P.cta2) {
+                cudaLaunchConfig_t cfg = {};
+                cfg.gridDim = dim3((unsigned)grid);
+                cfg.blockDim = dim3(CONV_THREADS);
+                cfg.dynamicSmemBytes = smem;
+                cfg.stream = st;
+                cudaLaunchAttribute at[1];
+                at[0].id = cudaLaunchAttributeClusterDimension;
+                at[0].val.clusterDim.x = 2;
+                at[0].val.clusterDim.y = 1;
+                at[0].val.clusterDim.z = 1;
+                cfg.attrs = at;
+                cfg.numAttrs = 1;
+                cudaLaunchKernelEx(&cfg, kern, P);
+            } else {
+                kern<<<grid, CONV_THREADS, smem, st>>>(P);
+            }
         };
-        switch (mode_bits) {
-            case 0: launch(conv_tc_kernel<false, false, false>); break;
-            case 1: launch(conv_tc_kernel<false, false, true>); break;
-            case 2: launch(conv_tc_kernel<false, true, false>); break;
-            case 3: launch(conv_tc_kernel<false, true, true>); break;
-            case 4: launch(conv_tc_kernel<true, false, false>); break;
-            case 5: launch(conv_tc_kernel<true, false, true>); break;
-            case 6: launch(conv_tc_kernel<true, true, false>); break;
-            default: launch(conv_tc_kernel<true, true, true>); break;
+        // kernels holding cta_group::2 instructions must be launched as clusters: separate instantiations
+        if (P.cta2) {
+            switch (mode_bits) {
+                case 0: launch(conv_tc_kernel<false, false, false, true>); break;
+                case 1: launch(conv_tc_kernel<false, false, true, true>); break;
+                case 2: launch(conv_tc_kernel<false, true, false, true>); break;
+                case 3: launch(conv_tc_kernel<false, true, true, true>); break;
+                case 4: launch(conv_tc_kernel<true, false, false, true>); break;
+                case 5: launch(conv_tc_kernel<true, false, true, true>); break;
+                case 6: launch(conv_tc_kernel<true, true, false, true>); break;
+                default: launch(conv_tc_kernel<true, true, true, true>); break;
+            }
+        } else {
+            switch (mode_bits) {
+                case 0: launch(conv_tc_kernel<false, false, false, false>); break;
+                case 1: launch(conv_tc_kernel<false, false, true, false>); break;
+                case 2: launch(conv_tc_kernel<false, true, false, false>); break;
+                case 3: launch(conv_tc_kernel<false, true, true, false>); break;
+                case 4: launch(conv_tc_kernel<true, false, false, false>); break;
+                case 5: launch(conv_tc_kernel<true, false, true, false>); break;
+                case 6: launch(conv_tc_kernel<true, true, false, false>); break;
+                default: launch(conv_tc_kernel<true, true, true, false>); break;
+            }
         }
         count_launch();
         {

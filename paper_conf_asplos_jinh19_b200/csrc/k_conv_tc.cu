@@ -77,23 +77,32 @@ struct TcConvParams {
     int ybufs;                    // staging buffers (2: the TMA store of tile t overlaps tile t+1)
     int dbg;                      // experiments only (SPLITCNN_DBG): 1 no TMA store, 2 no MMA, 4 no loads, 8 no TMEM->smem
     int egroups;                  // 2: two independent 4-warp epilogue groups, one per TMEM accumulator
+    unsigned long long *trace;    // debug (SPLITCNN_TRACE): per-tile clock64 events of CTA 0
     int cta2;                     // 2-CTA MMA (cluster of 2, M = 256): each CTA owns one 128-row M box and N/2 of B
     int BNh;                      // rows of B per CTA (BN / 2 in 2-CTA mode, else BN)
     int total_m, total_pairs, m_tpp;
     int m_prefix[TC_MAXP + 1];
     uint32_t ybuf_bytes;
+    int uni;                      // every patch has the same tile grid: O(1) decode by fast division
+    tc::FastDiv fd_tpp, fd_mtpp, fd_nco, fd_nwb, fd_nhb;
+    int ysh;                      // log2(ychunk)
 };
 
 static_assert(sizeof(TcConvParams) <= 32700, "kernel parameter space is 32 KB");
 
 // 2-CTA mode: M box index (across patches) -> patch, image block, row block, column block
 __device__ __forceinline__ void decode_mbox(const TcConvParams &p, int m, int &ql, int &nb, int &hb, int &wb) {
-    if (p.m_tpp) {
-        ql = m / p.m_tpp;
-    } else {
-        ql = 0;
-        while (m >= p.m_prefix[ql + 1]) ++ql;
+    if (p.uni) {
+        uint32_t idx, r;
+        ql = (int)tc::fdivmod((uint32_t)m, p.fd_mtpp, idx);
+        idx = tc::fdivmod(idx, p.fd_nwb, r);
+        wb = (int)r;
+        nb = (int)tc::fdivmod(idx, p.fd_nhb, r);
+        hb = (int)r;
+        return;
     }
+    ql = 0;
+    while (m >= p.m_prefix[ql + 1]) ++ql;
     int idx = m - p.m_prefix[ql];
     wb = idx % p.nwb[ql];
     idx /= p.nwb[ql];
@@ -102,12 +111,19 @@ __device__ __forceinline__ void decode_mbox(const TcConvParams &p, int m, int &q
 }
 
 __device__ __forceinline__ void decode_tile(const TcConvParams &p, int t, int &ql, int &nb, int &hb, int &wb, int &cb) {
-    if (p.tpp) {
-        ql = t / p.tpp;
-    } else {
-        ql = 0;
-        while (t >= p.tile_prefix[ql + 1]) ++ql;
+    if (p.uni) {
+        uint32_t idx, r;
+        ql = (int)tc::fdivmod((uint32_t)t, p.fd_tpp, idx);
+        idx = tc::fdivmod(idx, p.fd_nco, r);
+        cb = (int)r;
+        idx = tc::fdivmod(idx, p.fd_nwb, r);
+        wb = (int)r;
+        nb = (int)tc::fdivmod(idx, p.fd_nhb, r);
+        hb = (int)r;
+        return;
     }
+    ql = 0;
+    while (t >= p.tile_prefix[ql + 1]) ++ql;
     int idx = t - p.tile_prefix[ql];
     cb = idx % p.nco;
     idx /= p.nco;
@@ -122,8 +138,10 @@ __device__ __forceinline__ void decode_tile(const TcConvParams &p, int t, int &q
 __device__ __forceinline__ void get_tile(const TcConvParams &p, int t, uint32_t rank, int &ql, int &nb, int &hb, int &wb,
                                          int &cb, bool &valid) {
     if (p.cta2) {
-        cb = t % p.nco;
-        int m = 2 * (t / p.nco) + (int)rank;
+        uint32_t r;
+        const int mp = (int)tc::fdivmod((uint32_t)t, p.fd_nco, r);
+        cb = (int)r;
+        int m = 2 * mp + (int)rank;
         valid = m < p.total_m;
         m = min(m, p.total_m - 1);
         decode_mbox(p, m, ql, nb, hb, wb);
@@ -173,10 +191,13 @@ __device__ __forceinline__ uint4 epi8(const uint32_t *r, const float *sb, int co
     return pk;
 }
 
+#define TC_TRACE(i, e) \
+    do { if (p.trace && blockIdx.x == 0 && (i) < 256) p.trace[(i) * 8 + (e)] = clock64(); } while (0)
+
 template <bool BIAS, bool RELU, bool MASK, bool CTA2>
 __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_constant__ TcConvParams p) {
     extern __shared__ uint8_t smem_raw[];
-    uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+    uint8_t *smem = smem_raw + ((1024u - (tc::smem_u32(smem_raw) & 1023u)) & 1023u);   // keeps the shared space
     const int S = p.stages;
     const uint32_t b_stage = p.b_tx_bytes;   // BN x 128 B per tap box (kw boxes in halo mode)
     uint8_t *sA = smem;
@@ -221,6 +242,11 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
     else __syncthreads();
     tc::tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
+    if (p.trace && threadIdx.x == 0 && blockIdx.x < 1000) {
+        unsigned long long g;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g));
+        p.trace[2048 + 2 * blockIdx.x] = g;
+    }
     const int total = CTA2 ? p.total_pairs : p.tile_prefix[p.npatch];
     const int tfirst = CTA2 ? (int)tc::cluster_id_x() : (int)blockIdx.x;
     const int tstep = CTA2 ? (int)tc::nclusters_x() : (int)gridDim.x;
@@ -232,7 +258,10 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             for (int q = 0; q < p.npatch; ++q) tc::tma_prefetch_desc(&p.mapA[q]);
             tc::tma_prefetch_desc(&p.mapB);
             const uint32_t wbar_l = CTA2 ? tc::mapa_shared(wbar, 0) : 0u;
-            if (p.bres) {  // every (chunk, kernel row) weight box once, for all tiles of this CTA
+            if (p.bres && p.halo8) {   // the K = taps x 8 filter in 64-wide boxes, once per CTA
+                tc::mbar_arrive_expect_tx(wbar, p.bres_bytes);
+                for (int kb = 0; kb * 64 < KT * 8; ++kb) tc::tma_load_2d(sW + kb * p.BN * 128, &p.mapB, wbar, kb * 64, 0);
+            } else if (p.bres) {  // every (chunk, kernel row) weight box once, for all tiles of this CTA
                 const int rowB0 = (int)rank * p.BNh;  // 2-CTA: this CTA holds rows [rank*BN/2, +BN/2) of B
                 if (!CTA2) tc::mbar_arrive_expect_tx(wbar, p.bres_bytes);
                 else if (leader) tc::mbar_arrive_expect_tx(wbar, 2 * p.bres_bytes);
@@ -255,9 +284,9 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                         }
                     }
             }
-            int stage = 0;
+            int stage = 0, it = 0;
             uint32_t ph = 0;
-            for (int t = tfirst; t < total; t += tstep) {
+            for (int t = tfirst; t < total; t += tstep, ++it) {
                 int ql, nb, hb, wb, cb;
                 bool valid;
                 get_tile(p, t, rank, ql, nb, hb, wb, cb, valid);
@@ -266,7 +295,9 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 const int n0 = nb * p.BNn, co0 = cb * p.BN;
                 if (p.dbg & 16) continue;
                 for (int ks = 0; ks < p.ksteps; ++ks) {
-                    tc::mbar_wait_sleep(&empty[stage], ph ^ 1);
+                    if (p.dbg & 64) tc::mbar_wait(&empty[stage], ph ^ 1);
+                    else tc::mbar_wait_sleep(&empty[stage], ph ^ 1);
+                    if (ks == 0) TC_TRACE(it, 6);
                     if (p.dbg & 4) {
                         tc::mbar_arrive(&full[stage]);
                         if (++stage == S) { stage = 0; ph ^= 1; }
@@ -303,8 +334,9 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     if (p.halo8) {
                         // rows (h) x (8 + kw - 1) pixels x 8 channels; the weights' K = taps*8 in 64-wide boxes
                         tc::tma_load_3d(a, &p.mapA[ql], &full[stage], 8 * wbase, hbase, n0);
-                        for (int kb = 0; kb * 64 < KT * 8; ++kb)
-                            tc::tma_load_2d(b + kb * p.BN * 128, &p.mapB, &full[stage], kb * 64, co0);
+                        if (!p.bres)
+                            for (int kb = 0; kb * 64 < KT * 8; ++kb)
+                                tc::tma_load_2d(b + kb * p.BN * 128, &p.mapB, &full[stage], kb * 64, co0);
                     } else if (p.halo) {
                         const int cc = ks / p.kh, r = ks - cc * p.kh;
                         tc::tma_load_4d(a, &p.mapA[ql], &full[stage], cc * 64, wbase, hbase + r, n0);
@@ -333,6 +365,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     }
                     if (++stage == S) { stage = 0; ph ^= 1; }
                 }
+                TC_TRACE(it, 7);
             }
         }
     } else if (warp == 1) {
@@ -340,15 +373,41 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             // ================= MMA issuer: the whole warp runs the loop converged; elect.sync issues.
             // In 2-CTA mode only the leader issues (M = 256 over the pair); the peer's warp 1 idles.
             const uint32_t idesc = tc::idesc_bf16(CTA2 ? 256 : 128, p.BN);
+            // halo8: per tap pair, the descriptor relative to the stage base (start address field 0)
+            uint64_t h8_adesc[8], h8_bdesc[8];
+            const int h8_npairs = p.halo8 ? (KT + 1) / 2 : 0;
+#pragma unroll
+            for (int pr = 0; pr < 8; ++pr) {
+                h8_adesc[pr] = h8_bdesc[pr] = 0;
+                if (pr < h8_npairs) {
+                    const int t0 = 2 * pr, t1 = 2 * pr + 1;
+                    const int o0 = (t0 / p.kw) * p.Wp + (t0 % p.kw);
+                    const int o1 = t1 < KT ? (t1 / p.kw) * p.Wp + (t1 % p.kw) : o0 + 1;
+                    h8_adesc[pr] = tc::smem_desc(0, 16u * (uint32_t)(o1 - o0), (uint32_t)p.Wp * 16u, 0) + (uint64_t)o0;
+                    h8_bdesc[pr] = tc::smem_desc(0, 16, 1024, 2) + (uint64_t)((((pr >> 2) * p.BN) * 128 + 32 * (pr & 3)) >> 4);
+                }
+            }
+            // generic path: start-address offset (>> 4) of the 4 K=16 slices of a K step
+            uint32_t g_aoff[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const int k0 = 16 * j;
+                const int chunk = k0 / p.cpadc;
+                g_aoff[j] = (chunk * p.a_chunk_bytes + (uint32_t)((k0 - chunk * p.cpadc) * 2)) >> 4;
+            }
             int stage = 0, acc = 0;
             uint32_t ph = 0, aph = 0;
             if (p.bres && leader) tc::mbar_wait(wbar, 0);
-            for (int t = leader ? tfirst : total; t < total; t += tstep) {
-                tc::mbar_wait_sleep(&tempty[acc], aph ^ 1);
+            int it = 0;
+            for (int t = leader ? tfirst : total; t < total; t += tstep, ++it) {
+                if (p.dbg & 64) tc::mbar_wait(&tempty[acc], aph ^ 1);
+                else tc::mbar_wait_sleep(&tempty[acc], aph ^ 1);
+                if (lane == 0) TC_TRACE(it, 0);
                 tc::tc_fence_after();
                 const uint32_t d = tmem_base + (uint32_t)(acc * p.BN);
                 for (int ks = 0; ks < p.ksteps; ++ks) {
                     if (!(p.dbg & 16)) tc::mbar_wait(&full[stage], ph);
+                    if (ks == 0 && lane == 0) TC_TRACE(it, 1);
                     tc::tc_fence_after();
                     const uint32_t a_base = tc::smem_u32(sA + (size_t)stage * p.a_stage);
                     const uint32_t b_base = tc::smem_u32(sB + (size_t)stage * b_stage);
@@ -360,17 +419,14 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     if (p.halo8) {
                         // no-swizzle K-major A: a core matrix is 8 consecutive pixels x 16 B (8 channels);
                         // M groups (output rows) are Wp pixels apart (SBO = Wp*16 B); each MMA covers the
-                        // K = 16 of two taps whose views differ by LBO = (pixel offset difference)*16 B
-                        const int npairs = (KT + 1) / 2;
-                        const uint64_t b0 = tc::smem_desc(b_base, 16, 1024, 2);
-                        for (int pr = 0; pr < npairs; ++pr) {
-                            const int t0 = 2 * pr, t1 = 2 * pr + 1;
-                            const int o0 = (t0 / p.kw) * p.Wp + (t0 % p.kw);
-                            const int o1 = t1 < KT ? (t1 / p.kw) * p.Wp + (t1 % p.kw) : o0 + 1;
-                            const uint64_t adesc = tc::smem_desc(a_base + 16u * o0, 16u * (uint32_t)(o1 - o0), (uint32_t)p.Wp * 16u, 0);
-                            // descriptors are linear in the start address (field = addr >> 4)
-                            const uint64_t bdesc = b0 + (uint64_t)((((pr >> 2) * p.BN) * 128 + 32 * (pr & 3)) >> 4);
-                            tc::mma_bf16_ws(d, adesc, bdesc, idesc, (ks | pr) != 0);
+                        // K = 16 of two taps whose views differ by LBO = (pixel offset difference)*16 B.
+                        // Descriptors are linear in the start address: tile-invariant parts precomputed.
+                        const uint64_t abase = (uint64_t)((a_base >> 4) & 0x3FFF);
+                        const uint64_t bbase = (uint64_t)(((p.bres ? tc::smem_u32(sW) : b_base) >> 4) & 0x3FFF);
+#pragma unroll
+                        for (int pr = 0; pr < 8; ++pr) {
+                            if (pr < h8_npairs)
+                                tc::mma_bf16_ws(d, h8_adesc[pr] + abase, h8_bdesc[pr] + bbase, idesc, (ks | pr) != 0);
                         }
                         tc::mma_commit_ws(&empty[stage]);
                         if (++stage == S) { stage = 0; ph ^= 1; }
@@ -423,17 +479,14 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     const uint64_t a0 = tc::smem_desc(a_base, p.a_lbo, p.a_sbo, p.a_layout);
                     const uint64_t b0 = tc::smem_desc(b_base, 16, 1024, 2);
 #pragma unroll
-                    for (int j = 0; j < 4; ++j) {
-                        const int k0 = 16 * j;
-                        const int chunk = k0 / p.cpadc;
-                        const uint32_t a_off = chunk * p.a_chunk_bytes + (uint32_t)((k0 - chunk * p.cpadc) * 2);
-                        tc::mma_bf16_ws(d, a0 + (uint64_t)(a_off >> 4), b0 + (uint64_t)(2 * j), idesc, (ks | j) != 0);
-                    }
+                    for (int j = 0; j < 4; ++j)
+                        tc::mma_bf16_ws(d, a0 + (uint64_t)g_aoff[j], b0 + (uint64_t)(2 * j), idesc, (ks | j) != 0);
                     tc::mma_commit_ws(&empty[stage]);
                     if (++stage == S) { stage = 0; ph ^= 1; }
                 }
                 if (CTA2) tc::mma2_commit_mc_ws(&tfull[acc]);
                 else tc::mma_commit_ws(&tfull[acc]);
+                if (lane == 0) TC_TRACE(it, 2);
                 acc ^= 1;
                 if (acc == 0) aph ^= 1;
             }
@@ -451,7 +504,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
         uint64_t *mbar = g ? wbar + 1 : ybar;
         uint32_t aph = 0, yph = 0;
         const uint32_t tempty_l = tc::mapa_shared(&tempty[g], 0);   // the leader's (own in 1-CTA mode)
-        for (int t = tfirst + g * tstep; t < total; t += 2 * tstep) {
+        int it = g;
+        for (int t = tfirst + g * tstep; t < total; t += 2 * tstep, it += 2) {
             int ql, nb, hb, wb, cb;
             bool valid;
             get_tile(p, t, rank, ql, nb, hb, wb, cb, valid);
@@ -471,6 +525,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 yph ^= 1;
             }
             tc::mbar_wait(&tfull[g], aph);
+            if (gtid == 0) TC_TRACE(it, 3);
             tc::tc_fence_after();
             const uint32_t tacc = tmem_base + (uint32_t)(g * p.BN) + ((uint32_t)(quad * 32) << 16);
             for (int cc = 0; cc < ((p.dbg & 8) ? 0 : ncols); cc += 32) {
@@ -482,8 +537,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 for (int u = 0; u < 4; ++u) {
                     const int c8 = cc + 8 * u;
                     if (c8 >= ncols) break;
-                    const int k = c8 / p.ychunk;
-                    const uint32_t off = tc::swz((uint32_t)row * rowB + (uint32_t)(c8 - k * p.ychunk) * 2u, p.y_mask);
+                    const int k = c8 >> p.ysh;
+                    const uint32_t off = tc::swz((uint32_t)row * rowB + (uint32_t)(c8 & (p.ychunk - 1)) * 2u, p.y_mask);
                     uint4 *dst = reinterpret_cast<uint4 *>(sYb + k * chunk_bytes + off);
                     const uint4 m4 = MASK ? *dst : make_uint4(0, 0, 0, 0);
                     *dst = epi8<BIAS, RELU, MASK>(r[u >> 1] + 8 * (u & 1), sbias, co0 + c8, p.Cout, m4);
@@ -495,6 +550,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 if (CTA2) tc::mbar_arrive_remote(tempty_l);
                 else tc::mbar_arrive(&tempty[g]);
             }
+            if (gtid == 0) TC_TRACE(it, 4);
             tc::fence_proxy_async_smem();
             tc::named_bar_sync(1 + g, 128);
             if (gtid == 0 && valid && !(p.dbg & 1)) {
@@ -502,6 +558,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     tc::tma_store_4d(&p.mapY[ql], sYb + k * chunk_bytes, co0 + k * p.ychunk, ow0, oh0, n0);
                 tc::bulk_commit();
             }
+            if (gtid == 0) TC_TRACE(it, 5);
             aph ^= 1;
         }
         if (gtid == 0) tc::bulk_wait0();
@@ -552,8 +609,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 for (int u = 0; u < 2; ++u) {
                     const int c8 = cc + 8 * u;
                     if (c8 >= ncols) break;
-                    const int k = c8 / p.ychunk;
-                    const uint32_t off = tc::swz((uint32_t)row * rowB + (uint32_t)(c8 - k * p.ychunk) * 2u, p.y_mask);
+                    const int k = c8 >> p.ysh;
+                    const uint32_t off = tc::swz((uint32_t)row * rowB + (uint32_t)(c8 & (p.ychunk - 1)) * 2u, p.y_mask);
                     uint4 *dst = reinterpret_cast<uint4 *>(sYb + k * chunk_bytes + off);
                     const uint4 m4 = MASK ? *dst : make_uint4(0, 0, 0, 0);
                     *dst = epi8<BIAS, RELU, MASK>(r + 8 * u, sbias, co0 + c8, p.Cout, m4);
@@ -642,6 +699,14 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             if (acc == 0) aph ^= 1;
         }
         }
+    }
+    if (p.trace && threadIdx.x == 64 && blockIdx.x < 1000) {
+        unsigned long long g;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g));
+        uint32_t smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        p.trace[2048 + 2 * blockIdx.x + 1] = g;
+        p.trace[3072 + blockIdx.x] = smid;
     }
     tc::tc_fence_before();
     if (CTA2) tc::cluster_sync_all();   // the peer's MMAs write this CTA's TMEM until the leader is done
@@ -830,6 +895,11 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             P.a_tx_bytes = (uint32_t)P.Wp * (ts.BH + kh - 1) * 16u;
             P.a_stage = (P.a_tx_bytes + 1023u) & ~1023u;
             P.b_tx_bytes = (uint32_t)((kh * kw * 8 + 63) / 64) * BN * 128u;
+            if (nco == 1 && !getenv("SPLITCNN_NO_BRES")) {   // the whole filter stays in smem (one load per CTA)
+                P.bres = 1;
+                P.bres_bytes = P.b_tx_bytes;
+                P.b_tx_bytes = 0;
+            }
         } else if (halo) {
             P.ksteps = (cpad / 64) * kh;
             P.a_tx_bytes = (uint32_t)P.Wp * ts.BH * ts.BNn * 128u;
@@ -934,6 +1004,15 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.m_tpp = P.m_prefix[1];
         for (int ql = 1; ql < P.npatch; ++ql)
             if (P.m_prefix[ql + 1] - P.m_prefix[ql] != P.m_tpp) P.m_tpp = 0;
+        P.uni = 1;
+        for (int ql = 1; ql < P.npatch; ++ql)
+            if (P.nhb[ql] != P.nhb[0] || P.nwb[ql] != P.nwb[0]) P.uni = 0;
+        P.fd_tpp = tc::make_fastdiv((uint32_t)std::max(1, P.tile_prefix[1]));
+        P.fd_mtpp = tc::make_fastdiv((uint32_t)std::max(1, P.m_prefix[1]));
+        P.fd_nco = tc::make_fastdiv((uint32_t)nco);
+        P.fd_nwb = tc::make_fastdiv((uint32_t)std::max(1, P.nwb[0]));
+        P.fd_nhb = tc::make_fastdiv((uint32_t)std::max(1, P.nhb[0]));
+        P.ysh = P.ychunk == 64 ? 6 : P.ychunk == 32 ? 5 : P.ychunk == 16 ? 4 : 3;
         P.tpp = P.tile_prefix[1];
         for (int ql = 1; ql < P.npatch; ++ql)
             if (P.tile_prefix[ql + 1] - P.tile_prefix[ql] != P.tpp) P.tpp = 0;
@@ -963,6 +1042,12 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         }
         if (tiles == 0) continue;
         const size_t smem = 1024 + (size_t)P.bar_off + 512 + (bias ? 4 * (size_t)g.L.cout : 0) + 64;
+        static unsigned long long *trace_buf = nullptr;
+        if (getenv("SPLITCNN_TRACE")) {
+            if (!trace_buf) cudaMalloc(&trace_buf, 4096 * sizeof(unsigned long long));
+            cudaMemsetAsync(trace_buf, 0, 4096 * sizeof(unsigned long long), st);
+            P.trace = trace_buf;
+        }
         const int grid = P.cta2 ? 2 * std::min(P.total_pairs, num_sms() / 2) : std::min(tiles, num_sms());
         const int mode_bits = (bias ? 4 : 0) | (relu ? 2 : 0) | (relu_src ? 1 : 0);
         auto launch = [&](auto kern) {
@@ -1018,6 +1103,34 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         {
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("conv_tc_kernel: ") + cudaGetErrorString(e));
+        }
+        if (P.trace) {   // debug: per-tile event times of CTA 0 relative to its first event
+            static unsigned long long h[4096];
+            cudaStreamSynchronize(st);
+            cudaMemcpy(h, P.trace, sizeof(h), cudaMemcpyDeviceToHost);
+            {
+                unsigned long long s0 = ~0ull, e1 = 0, smax = 0, emin = ~0ull;
+                for (int b = 0; b < std::min(grid, 1000); ++b) {
+                    const unsigned long long e = h[2048 + 2 * b + 1];
+                    s0 = std::min(s0, h[2048 + 2 * b]); smax = std::max(smax, h[2048 + 2 * b]);
+                    e1 = std::max(e1, e); emin = std::min(emin, e);
+                }
+                fprintf(stderr, "trace CTA (block smid end_us):");
+                for (int b = 0; b < std::min(grid, 1000); ++b)
+                    fprintf(stderr, " %d:%d:%.0f", b, (int)h[3072 + b], (h[2048 + 2 * b + 1] - s0) / 1e3);
+                fprintf(stderr, "\n");
+                fprintf(stderr, "trace CTAs: first start 0, last start %.1f us, first end %.1f us, last end %.1f us\n",
+                        (smax - s0) / 1e3, (emin - s0) / 1e3, (e1 - s0) / 1e3);
+            }
+            unsigned long long t0 = h[6];
+            fprintf(stderr, "trace tiles=%d grid=%d ksteps=%d BN=%d cta2=%d  [tile: prod_empty prod_done | mma_tempty mma_full mma_commit | epi_tfull epi_tempty epi_store]\n",
+                    tiles, grid, P.ksteps, P.BN, P.cta2);
+            for (int i = 0; i < 256; ++i) {
+                if (i == 12) i = 230;
+                const unsigned long long *r = h + i * 8;
+                auto d = [&](int e) { return r[e] ? (long long)(r[e] - t0) : -1LL; };
+                fprintf(stderr, "  %3d: %8lld %8lld | %8lld %8lld %8lld | %8lld %8lld %8lld\n", i, d(6), d(7), d(0), d(1), d(2), d(3), d(4), d(5));
+            }
         }
     }
     return SPLITCNN_OK;

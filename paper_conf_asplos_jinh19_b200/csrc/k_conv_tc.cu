@@ -84,7 +84,7 @@ struct TcConvParams {
     int m_prefix[TC_MAXP + 1];
     uint32_t ybuf_bytes;
     int uni;                      // every patch has the same tile grid: O(1) decode by fast division
-    tc::FastDiv fd_tpp, fd_mtpp, fd_nco, fd_nwb, fd_nhb;
+    FastDiv fd_tpp, fd_mtpp, fd_nco, fd_nwb, fd_nhb;
     int ysh;                      // log2(ychunk)
 };
 
@@ -94,10 +94,10 @@ static_assert(sizeof(TcConvParams) <= 32700, "kernel parameter space is 32 KB");
 __device__ __forceinline__ void decode_mbox(const TcConvParams &p, int m, int &ql, int &nb, int &hb, int &wb) {
     if (p.uni) {
         uint32_t idx, r;
-        ql = (int)tc::fdivmod((uint32_t)m, p.fd_mtpp, idx);
-        idx = tc::fdivmod(idx, p.fd_nwb, r);
+        ql = (int)fdivmod((uint32_t)m, p.fd_mtpp, idx);
+        idx = fdivmod(idx, p.fd_nwb, r);
         wb = (int)r;
-        nb = (int)tc::fdivmod(idx, p.fd_nhb, r);
+        nb = (int)fdivmod(idx, p.fd_nhb, r);
         hb = (int)r;
         return;
     }
@@ -113,12 +113,12 @@ __device__ __forceinline__ void decode_mbox(const TcConvParams &p, int m, int &q
 __device__ __forceinline__ void decode_tile(const TcConvParams &p, int t, int &ql, int &nb, int &hb, int &wb, int &cb) {
     if (p.uni) {
         uint32_t idx, r;
-        ql = (int)tc::fdivmod((uint32_t)t, p.fd_tpp, idx);
-        idx = tc::fdivmod(idx, p.fd_nco, r);
+        ql = (int)fdivmod((uint32_t)t, p.fd_tpp, idx);
+        idx = fdivmod(idx, p.fd_nco, r);
         cb = (int)r;
-        idx = tc::fdivmod(idx, p.fd_nwb, r);
+        idx = fdivmod(idx, p.fd_nwb, r);
         wb = (int)r;
-        nb = (int)tc::fdivmod(idx, p.fd_nhb, r);
+        nb = (int)fdivmod(idx, p.fd_nhb, r);
         hb = (int)r;
         return;
     }
@@ -139,7 +139,7 @@ __device__ __forceinline__ void get_tile(const TcConvParams &p, int t, uint32_t 
                                          int &cb, bool &valid) {
     if (p.cta2) {
         uint32_t r;
-        const int mp = (int)tc::fdivmod((uint32_t)t, p.fd_nco, r);
+        const int mp = (int)fdivmod((uint32_t)t, p.fd_nco, r);
         cb = (int)r;
         int m = 2 * mp + (int)rank;
         valid = m < p.total_m;
@@ -153,6 +153,38 @@ __device__ __forceinline__ void get_tile(const TcConvParams &p, int t, uint32_t 
 
 
 constexpr int CONV_THREADS = 64 + 256;  // producer warp, MMA warp, 8 epilogue warps (2 per TMEM lane quadrant)
+
+// 8 accumulator columns (all real channels) -> bf16x8: +bias, ReLU, dgrad ReLU mask
+template <bool BIAS, bool RELU, bool MASK>
+__device__ __forceinline__ uint4 epi8_full(const uint32_t *r, const float *sb, uint4 m4) {
+    float o[8];
+#pragma unroll
+    for (int e = 0; e < 8; ++e) o[e] = __uint_as_float(r[e]);
+    if (BIAS) {
+        const float4 b0 = *reinterpret_cast<const float4 *>(sb);
+        const float4 b1 = *reinterpret_cast<const float4 *>(sb + 4);
+        o[0] += b0.x; o[1] += b0.y; o[2] += b0.z; o[3] += b0.w;
+        o[4] += b1.x; o[5] += b1.y; o[6] += b1.z; o[7] += b1.w;
+    }
+    if (RELU) {
+#pragma unroll
+        for (int e = 0; e < 8; ++e) o[e] = fmaxf(o[e], 0.f);
+    }
+    if (MASK) {
+        const __nv_bfloat162 *mh = reinterpret_cast<const __nv_bfloat162 *>(&m4);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+            const float2 mf = __bfloat1622float2(mh[e]);
+            o[2 * e] = mf.x > 0.f ? o[2 * e] : 0.f;
+            o[2 * e + 1] = mf.y > 0.f ? o[2 * e + 1] : 0.f;
+        }
+    }
+    uint4 pk;
+    __nv_bfloat162 *h2 = reinterpret_cast<__nv_bfloat162 *>(&pk);
+#pragma unroll
+    for (int e = 0; e < 4; ++e) h2[e] = __floats2bfloat162_rn(o[2 * e], o[2 * e + 1]);
+    return pk;
+}
 
 // 8 accumulator columns -> bf16x8 with the fused epilogue (bias, ReLU, or the dgrad ReLU mask)
 template <bool BIAS, bool RELU, bool MASK>
@@ -528,7 +560,27 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             if (gtid == 0) TC_TRACE(it, 3);
             tc::tc_fence_after();
             const uint32_t tacc = tmem_base + (uint32_t)(g * p.BN) + ((uint32_t)(quad * 32) << 16);
-            for (int cc = 0; cc < ((p.dbg & 8) ? 0 : ncols); cc += 32) {
+            // fast path: whole 32-column groups of real channels inside one staging chunk (ychunk >= 32)
+            const bool fast = (ncols & 31) == 0 && co0 + ncols <= p.Cout && p.ychunk >= 32 && !(p.dbg & 8);
+            if (fast) {
+                const uint32_t rbase = (uint32_t)row * rowB;
+                const uint32_t rsw = ((rbase >> 7) & p.y_mask) << 4;
+                for (int cc = 0; cc < ncols; cc += 32) {
+                    uint32_t r2[2][16];
+                    tc::tmem_ld16_nw(tacc + cc, r2[0]);
+                    tc::tmem_ld16_nw(tacc + cc + 16, r2[1]);
+                    tc::tmem_wait_ld();
+                    uint8_t *cbase = sYb + (cc >> p.ysh) * chunk_bytes + rbase;
+                    const uint32_t cb0 = (uint32_t)(cc & (p.ychunk - 1)) * 2u;
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) {
+                        uint4 *dst = reinterpret_cast<uint4 *>(cbase + ((cb0 + 16u * u) ^ rsw));
+                        const uint4 m4 = MASK ? *dst : make_uint4(0, 0, 0, 0);
+                        *dst = epi8_full<BIAS, RELU, MASK>(r2[u >> 1] + 8 * (u & 1), sbias + co0 + cc + 8 * u, m4);
+                    }
+                }
+            }
+            for (int cc = 0; cc < ((p.dbg & 8) || fast ? 0 : ncols); cc += 32) {
                 uint32_t r[2][16];
                 tc::tmem_ld16_nw(tacc + cc, r[0]);
                 if (cc + 16 < ncols) tc::tmem_ld16_nw(tacc + cc + 16, r[1]);
@@ -1007,11 +1059,11 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.uni = 1;
         for (int ql = 1; ql < P.npatch; ++ql)
             if (P.nhb[ql] != P.nhb[0] || P.nwb[ql] != P.nwb[0]) P.uni = 0;
-        P.fd_tpp = tc::make_fastdiv((uint32_t)std::max(1, P.tile_prefix[1]));
-        P.fd_mtpp = tc::make_fastdiv((uint32_t)std::max(1, P.m_prefix[1]));
-        P.fd_nco = tc::make_fastdiv((uint32_t)nco);
-        P.fd_nwb = tc::make_fastdiv((uint32_t)std::max(1, P.nwb[0]));
-        P.fd_nhb = tc::make_fastdiv((uint32_t)std::max(1, P.nhb[0]));
+        P.fd_tpp = make_fastdiv((uint32_t)std::max(1, P.tile_prefix[1]));
+        P.fd_mtpp = make_fastdiv((uint32_t)std::max(1, P.m_prefix[1]));
+        P.fd_nco = make_fastdiv((uint32_t)nco);
+        P.fd_nwb = make_fastdiv((uint32_t)std::max(1, P.nwb[0]));
+        P.fd_nhb = make_fastdiv((uint32_t)std::max(1, P.nhb[0]));
         P.ysh = P.ychunk == 64 ? 6 : P.ychunk == 32 ? 5 : P.ychunk == 16 ? 4 : 3;
         P.tpp = P.tile_prefix[1];
         for (int ql = 1; ql < P.npatch; ++ql)

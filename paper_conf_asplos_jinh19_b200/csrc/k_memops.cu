@@ -11,26 +11,32 @@
 namespace splitcnn {
 
 // ============================================================ split / merge
+// Unit index u (< 2^31 per patch, checked on the host) -> coordinates by fast division; the
+// divisors are fixed per patch, so each thread builds its multipliers once.
+struct Dec3 {
+    FastDiv a, b, c;
+};
+__device__ __forceinline__ Dec3 make_dec3(uint32_t a, uint32_t b, uint32_t c) {
+    return {make_fastdiv(a), make_fastdiv(b), make_fastdiv(c)};
+}
+// u -> (x0 = u % a, x1 = (u / a) % b, x2 = (u / ab) % c, x3 = u / abc)
+__device__ __forceinline__ void dec3(uint32_t u, const Dec3 &d, int &x0, int &x1, int &x2, int &x3) {
+    uint32_t r;
+    u = fdivmod(u, d.a, r); x0 = (int)r;
+    u = fdivmod(u, d.b, r); x1 = (int)r;
+    u = fdivmod(u, d.c, r); x2 = (int)r;
+    x3 = (int)u;
+}
 template <typename T, bool NCHW>
 __global__ void __launch_bounds__(256) split_kernel(LevelDesc L, const T *__restrict__ x, T *__restrict__ P, int p0) {
     const PatchGeo g = patch_geo(L, p0 + blockIdx.y);
     const int G = L.Cpad / 8;
-    const int64_t units = (int64_t)L.N * g.hp * g.wp * G;
-    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < units; u += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t units = (uint32_t)L.N * g.hp * g.wp * G;
+    const Dec3 d = NCHW ? make_dec3(g.wp, g.hp, G) : make_dec3(G, g.wp, g.hp);
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < units; u += gridDim.x * blockDim.x) {
         int n, h, w, cg;
-        if (NCHW) {  // pixel-fastest: coalesced reads of each channel plane
-            w = (int)(u % g.wp);
-            int64_t t = u / g.wp;
-            h = (int)(t % g.hp); t /= g.hp;
-            cg = (int)(t % G);
-            n = (int)(t / G);
-        } else {     // channel-fastest: coalesced 16 B reads and writes
-            cg = (int)(u % G);
-            int64_t t = u / G;
-            w = (int)(t % g.wp); t /= g.wp;
-            h = (int)(t % g.hp);
-            n = (int)(t / g.hp);
-        }
+        if (NCHW) dec3(u, d, w, h, cg, n);   // pixel-fastest: coalesced reads of each channel plane
+        else dec3(u, d, cg, w, h, n);        // channel-fastest: coalesced 16 B reads and writes
         const int hg = g.h0 + h, wg = g.w0 + w, c0 = cg * 8;
         float v[8];
         if (NCHW) {
@@ -54,22 +60,12 @@ template <typename T, bool NCHW>
 __global__ void __launch_bounds__(256) merge_kernel(LevelDesc L, const T *__restrict__ P, T *__restrict__ y, int p0) {
     const PatchGeo g = patch_geo(L, p0 + blockIdx.y);
     const int G = L.Cpad / 8;
-    const int64_t units = (int64_t)L.N * g.hp * g.wp * G;
-    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < units; u += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t units = (uint32_t)L.N * g.hp * g.wp * G;
+    const Dec3 d = NCHW ? make_dec3(g.wp, g.hp, G) : make_dec3(G, g.wp, g.hp);
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < units; u += gridDim.x * blockDim.x) {
         int n, h, w, cg;
-        if (NCHW) {
-            w = (int)(u % g.wp);
-            int64_t t = u / g.wp;
-            h = (int)(t % g.hp); t /= g.hp;
-            cg = (int)(t % G);
-            n = (int)(t / G);
-        } else {
-            cg = (int)(u % G);
-            int64_t t = u / G;
-            w = (int)(t % g.wp); t /= g.wp;
-            h = (int)(t % g.hp);
-            n = (int)(t / g.hp);
-        }
+        if (NCHW) dec3(u, d, w, h, cg, n);   
+        else dec3(u, d, cg, w, h, n);        
         const int hg = g.h0 + h, wg = g.w0 + w, c0 = cg * 8;
         float v[8];
         load8(P + g.off + (((int64_t)n * g.hp + h) * g.wp + w) * L.Cpad + c0, v);
@@ -150,13 +146,11 @@ __global__ void __launch_bounds__(256) pool_fwd_kernel(LevelDesc Li, LevelDesc L
     const PatchGeo gi = patch_geo(Li, q), go = patch_geo(Lo, q);
     const int pt = ly.pad_h[2 * gi.i], pl = ly.pad_w[2 * gi.j];
     const int G = Li.Cpad / 8;
-    const int64_t units = (int64_t)Lo.N * go.hp * go.wp * G;
-    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < units; u += (int64_t)gridDim.x * blockDim.x) {
-        const int cg = (int)(u % G);
-        int64_t t = u / G;
-        const int ow = (int)(t % go.wp); t /= go.wp;
-        const int oh = (int)(t % go.hp);
-        const int n = (int)(t / go.hp);
+    const uint32_t units = (uint32_t)Lo.N * go.hp * go.wp * G;
+    const Dec3 d = make_dec3(G, go.wp, go.hp);
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < units; u += gridDim.x * blockDim.x) {
+        int cg, ow, oh, n;
+        dec3(u, d, cg, ow, oh, n);
         float best[8];
         int arg[8];
 #pragma unroll
@@ -199,13 +193,11 @@ __global__ void __launch_bounds__(256) pool_bwd_kernel(LevelDesc Li, LevelDesc L
     const PatchGeo gi = patch_geo(Li, q), go = patch_geo(Lo, q);
     const int pt = ly.pad_h[2 * gi.i], pl = ly.pad_w[2 * gi.j];
     const int G = Li.Cpad / 8;
-    const int64_t units = (int64_t)Li.N * gi.hp * gi.wp * G;
-    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < units; u += (int64_t)gridDim.x * blockDim.x) {
-        const int cg = (int)(u % G);
-        int64_t t = u / G;
-        const int w = (int)(t % gi.wp); t /= gi.wp;
-        const int h = (int)(t % gi.hp);
-        const int n = (int)(t / gi.hp);
+    const uint32_t units = (uint32_t)Li.N * gi.hp * gi.wp * G;
+    const Dec3 d = make_dec3(G, gi.wp, gi.hp);
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < units; u += gridDim.x * blockDim.x) {
+        int cg, w, h, n;
+        dec3(u, d, cg, w, h, n);
         int oh_lo = floordiv(h + pt - ly.kh, ly.sh) + 1, oh_hi = floordiv(h + pt, ly.sh);
         int ow_lo = floordiv(w + pl - ly.kw, ly.sw) + 1, ow_hi = floordiv(w + pl, ly.sw);
         if (oh_lo < 0) oh_lo = 0;
@@ -243,13 +235,11 @@ __global__ void __launch_bounds__(256) pool_bwd_scatter_kernel(LevelDesc Li, Lev
     const int q = p0 + blockIdx.y;
     const PatchGeo gi = patch_geo(Li, q), go = patch_geo(Lo, q);
     const int G = Li.Cpad / 8;
-    const int64_t units = (int64_t)Lo.N * go.hp * go.wp * G;
-    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < units; u += (int64_t)gridDim.x * blockDim.x) {
-        const int cg = (int)(u % G);
-        int64_t t = u / G;
-        const int ow = (int)(t % go.wp); t /= go.wp;
-        const int oh = (int)(t % go.hp);
-        const int n = (int)(t / go.hp);
+    const uint32_t units = (uint32_t)Lo.N * go.hp * go.wp * G;
+    const Dec3 d = make_dec3(G, go.wp, go.hp);
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < units; u += gridDim.x * blockDim.x) {
+        int cg, ow, oh, n;
+        dec3(u, d, cg, ow, oh, n);
         const int64_t o = go.off + (((int64_t)n * go.hp + oh) * go.wp + ow) * Lo.Cpad + cg * 8;
         const uint2 a2 = __ldg(reinterpret_cast<const uint2 *>(A + o));
         float g[8];

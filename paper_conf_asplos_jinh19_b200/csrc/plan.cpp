@@ -165,6 +165,14 @@ extern "C" splitcnn_status_t splitcnn_plan_create(const splitcnn_layer_t *layers
             }
         }
     }
+    // kernels index one patch's 8-channel units (N * h * w * Cpad / 8) in 32 bits
+    for (const auto &lv : p->levels)
+        for (int i = 0; i < lv.nh(); ++i)
+            for (int j = 0; j < lv.nw(); ++j)
+                if (lv.patch_elems(i, j) / 8 >= (int64_t)1 << 31) {
+                    delete p;
+                    return fail(SPLITCNN_ERR_UNSUPPORTED, "plan_create: a patch holds >= 2^34 elements");
+                }
     *out = p;
     return SPLITCNN_OK;
 }

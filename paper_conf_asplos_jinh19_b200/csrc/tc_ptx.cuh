@@ -11,25 +11,6 @@ __device__ __forceinline__ uint32_t smem_u32(const void *p) {
     return (uint32_t)__cvta_generic_to_shared(p);
 }
 
-// n / d and n % d for 0 <= n < 2^31 with a host-precomputed multiplier (round-up method)
-struct FastDiv {
-    uint32_t d, mul, shr;
-};
-__device__ __forceinline__ uint32_t fdiv(uint32_t n, const FastDiv &f) { return (__umulhi(n, f.mul) + n) >> f.shr; }
-__device__ __forceinline__ uint32_t fdivmod(uint32_t n, const FastDiv &f, uint32_t &rem) {
-    const uint32_t q = fdiv(n, f);
-    rem = n - q * f.d;
-    return q;
-}
-inline FastDiv make_fastdiv(uint32_t d) {
-    FastDiv f;
-    f.d = d;
-    uint32_t l = 0;
-    while ((1ull << l) < d) ++l;
-    f.shr = l;
-    f.mul = (uint32_t)(((1ull << 32) * ((1ull << l) - d)) / d + 1);
-    return f;
-}
 
 // ------------------------------------------------------------------ mbarrier
 __device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {

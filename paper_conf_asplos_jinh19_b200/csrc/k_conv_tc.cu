@@ -1420,9 +1420,14 @@ struct TcWgHaloParams {
     float *part;  // [nsplit][Cout][kh][kw][Cpi]
 };
 
+// CTA2: a cluster of 2 runs one tile of 256 output channels (each CTA: its own 128-channel dY block
+// as A) with cta_group::2 MMAs (M = 256); B is split by input channel -- each CTA loads 32 of the
+// chunk's 64 channels (SW64 rows of 64 B), so D column n < kw*32 is (tap n/32, ci n%32) of the
+// leader's half and n >= kw*32 the peer's.  Halves each CTA's smem operand traffic per MMA.
+template <bool CTA2>
 __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constant__ TcWgHaloParams p) {
     extern __shared__ uint8_t smem_raw[];
-    uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+    uint8_t *smem = smem_raw + ((1024u - (tc::smem_u32(smem_raw) & 1023u)) & 1023u);
     const int S = p.stages;
     // pixels per stage: BNn images x BH output rows x 8 output columns; for a FIXED kernel row r the X
     // box has exactly BH rows per image, so the K groups (n, h) stay Wp rows apart across images too
@@ -1430,7 +1435,9 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
     const int Wp = 8 + p.kw - 1;
     const uint32_t a_blk = (uint32_t)rows * 128u;     // one 64-channel dY block
     const uint32_t a_stage = 2u * a_blk;
-    const uint32_t b_stage = ((uint32_t)Wp * p.BH * p.BNn * 128u + 1023u) & ~1023u;
+    const uint32_t xrow = CTA2 ? 64u : 128u;            // bytes per X pixel row (32 or 64 channels)
+    const uint32_t b_bytes = (uint32_t)Wp * p.BH * p.BNn * xrow;
+    const uint32_t b_stage = (b_bytes + 1023u) & ~1023u;
     uint8_t *sA = smem;
     uint8_t *sB = smem + (size_t)S * a_stage;
     uint64_t *full = (uint64_t *)(sB + (size_t)S * b_stage);
@@ -1438,6 +1445,8 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
     uint64_t *tfull = empty + S;
     uint32_t *tmem_slot = (uint32_t *)(tfull + 1);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t rank = CTA2 ? tc::cluster_ctarank() : 0u;
+    const bool leader = rank == 0;
     if (warp == 0 && lane == 0) {
         for (int s = 0; s < S; ++s) {
             tc::mbar_init(&full[s], 1);
@@ -1446,16 +1455,22 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
         tc::mbar_init(&tfull[0], 1);
         tc::fence_barrier_init();
     }
-    if (warp == 1) tc::tmem_alloc_dyn(tmem_slot, p.tmem_cols);
+    if (warp == 1) {
+        if (CTA2) tc::tmem_alloc2(tmem_slot, p.tmem_cols);
+        else tc::tmem_alloc_dyn(tmem_slot, p.tmem_cols);
+    }
     tc::tc_fence_before();
-    __syncthreads();
+    if (CTA2) tc::cluster_sync_all();
+    else __syncthreads();
     tc::tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
 
-    const int tile = blockIdx.x % p.ntiles, z = blockIdx.x / p.ntiles;
+    // CTA2: work item = blockIdx.x / 2 over (co pair, kernel row, chunk) x split; ntiles counts pairs
+    const int item = CTA2 ? (int)(blockIdx.x >> 1) : (int)blockIdx.x;
+    const int tile = item % p.ntiles, z = item / p.ntiles;
     const int ch = tile % p.nchunk;
     const int r = (tile / p.nchunk) % p.kh;
-    const int co_blk = tile / (p.nchunk * p.kh);
+    const int co_blk = CTA2 ? 2 * (tile / (p.nchunk * p.kh)) + (int)rank : tile / (p.nchunk * p.kh);
     const int total_boxes = p.box_prefix[p.npatch];
     const int b0 = z * p.boxes_per_split, b1 = min(total_boxes, b0 + p.boxes_per_split);
     const int N = p.kw * 64;
@@ -1464,7 +1479,7 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
         if (lane == 0) {
             int stage = 0, ql = 0;
             uint32_t ph = 0;
-            const uint32_t tx = a_stage + (uint32_t)Wp * p.BH * p.BNn * 128u;
+            const uint32_t tx = a_stage + b_bytes;
             for (int b = b0; b < b1; ++b) {
                 while (b >= p.box_prefix[ql + 1]) ++ql;
                 int idx = b - p.box_prefix[ql];
@@ -1473,8 +1488,18 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
                 const int hb = idx % p.nhb[ql], n = (idx / p.nhb[ql]) * p.BNn;
                 const int ow0 = wb * 8, oh0 = hb * p.BH;
                 tc::mbar_wait_sleep(&empty[stage], ph ^ 1);
-                tc::mbar_arrive_expect_tx(&full[stage], tx);
                 uint8_t *a = sA + (size_t)stage * a_stage;
+                if (CTA2) {   // own dY block + own channel half of X; bytes land on the leader's barrier
+                    const uint32_t fb = tc::mapa_shared(&full[stage], 0);
+                    if (leader) tc::mbar_arrive_expect_tx(&full[stage], 2 * tx);
+                    tc::tma2_load_4d(a, &p.mapDY[ql], fb, co_blk * 128, ow0, oh0, n);
+                    tc::tma2_load_4d(a + a_blk, &p.mapDY[ql], fb, co_blk * 128 + 64, ow0, oh0, n);
+                    tc::tma2_load_4d(sB + (size_t)stage * b_stage, &p.mapX[ql], fb, ch * 64 + (int)rank * 32,
+                                     ow0 - p.pl[ql], oh0 - p.pt[ql] + r, n);
+                    if (++stage == S) { stage = 0; ph ^= 1; }
+                    continue;
+                }
+                tc::mbar_arrive_expect_tx(&full[stage], tx);
                 tc::tma_load_4d(a, &p.mapDY[ql], &full[stage], co_blk * 128, ow0, oh0, n);
                 tc::tma_load_4d(a + a_blk, &p.mapDY[ql], &full[stage], co_blk * 128 + 64, ow0, oh0, n);
                 tc::tma_load_4d(sB + (size_t)stage * b_stage, &p.mapX[ql], &full[stage], ch * 64, ow0 - p.pl[ql],
@@ -1484,10 +1509,10 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
         }
     } else if (warp == 1) {
         {   // converged warp; elect.sync issues
-            const uint32_t idesc = tc::idesc_bf16(128, N, 1, 1);
+            const uint32_t idesc = tc::idesc_bf16(CTA2 ? 256 : 128, N, 1, 1);
             int stage = 0;
             uint32_t ph = 0;
-            for (int b = b0; b < b1; ++b) {
+            for (int b = b0; b < (leader ? b1 : b0); ++b) {
                 tc::mbar_wait(&full[stage], ph);
                 tc::tc_fence_after();
                 const uint32_t a_base = tc::smem_u32(sA + (size_t)stage * a_stage);
@@ -1496,14 +1521,25 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
                 // B: X halo view, MN-major: tap c = MN block c at LBO = 128 B, K groups (output rows)
                 //    at SBO = Wp rows; 16 pixels = 2 output rows.  Per-MMA descriptors = base + constant.
                 const uint64_t a0 = tc::smem_desc(a_base, a_blk, 1024, 2);
-                const uint64_t bd0 = tc::smem_desc(b_base, 128, (uint32_t)Wp * 128u, 2);
-                const uint64_t bstep = (uint64_t)(2 * Wp * 8);   // 2 rows of Wp pixels x 128 B, >> 4
-                for (int j = 0; j < rows / 16; ++j)
-                    tc::mma_bf16_ws(tmem_base, a0 + (uint64_t)(128 * j), bd0 + bstep * j, idesc, (b != b0 || j) ? 1u : 0u);
-                tc::mma_commit_ws(&empty[stage]);
+                if (CTA2) {   // SW64 MN-major X: MN blocks of 32 channels, tap c = 1 row (64 B) further on
+                    const uint64_t bd0 = tc::smem_desc(b_base, 64, (uint32_t)Wp * 64u, 4);
+                    const uint64_t bstep = (uint64_t)(Wp * 8);   // 2 rows of Wp pixels x 64 B, >> 4
+                    for (int j = 0; j < rows / 16; ++j)
+                        tc::mma2_bf16_ws(tmem_base, a0 + (uint64_t)(128 * j), bd0 + bstep * j, idesc, (b != b0 || j) ? 1u : 0u);
+                    tc::mma2_commit_mc_ws(&empty[stage]);
+                } else {
+                    const uint64_t bd0 = tc::smem_desc(b_base, 128, (uint32_t)Wp * 128u, 2);
+                    const uint64_t bstep = (uint64_t)(2 * Wp * 8);   // 2 rows of Wp pixels x 128 B, >> 4
+                    for (int j = 0; j < rows / 16; ++j)
+                        tc::mma_bf16_ws(tmem_base, a0 + (uint64_t)(128 * j), bd0 + bstep * j, idesc, (b != b0 || j) ? 1u : 0u);
+                    tc::mma_commit_ws(&empty[stage]);
+                }
                 if (++stage == S) { stage = 0; ph ^= 1; }
             }
-            tc::mma_commit_ws(&tfull[0]);
+            if (leader) {
+                if (CTA2) tc::mma2_commit_mc_ws(&tfull[0]);
+                else tc::mma_commit_ws(&tfull[0]);
+            }
         }
     } else {
         const int quad = warp & 3;
@@ -1524,16 +1560,29 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
                 for (int e = 0; e < 16; ++e) v[e] = 0.f;
             }
             if (co >= p.Cout) continue;
-            const int c = cc / 64, ci = ch * 64 + (cc % 64);
+            // D column -> (tap, input channel); CTA2: the first kw*32 columns are the leader's channel half
+            int c, ci;
+            if (CTA2) {
+                const int hb = cc >= p.kw * 32 ? 1 : 0, n = cc - hb * p.kw * 32;
+                c = n >> 5;
+                ci = ch * 64 + hb * 32 + (n & 31);
+            } else {
+                c = cc / 64;
+                ci = ch * 64 + (cc % 64);
+            }
             float4 *d4 = reinterpret_cast<float4 *>(p.part + (((int64_t)z * p.Cout + co) * KT + r * p.kw + c) * p.Cpi + ci);
 #pragma unroll
             for (int e = 0; e < 4; ++e) d4[e] = make_float4(v[4 * e], v[4 * e + 1], v[4 * e + 2], v[4 * e + 3]);
         }
     }
     tc::tc_fence_before();
-    __syncthreads();
+    if (CTA2) tc::cluster_sync_all();
+    else __syncthreads();
     tc::tc_fence_after();
-    if (warp == 1) tc::tmem_dealloc(tmem_base, p.tmem_cols);
+    if (warp == 1) {
+        if (CTA2) tc::tmem_dealloc2(tmem_base, p.tmem_cols);
+        else tc::tmem_dealloc(tmem_base, p.tmem_cols);
+    }
 }
 
 // ------------------------------------------------------------ narrow-input weight gradient (Cin_pad = 8)
@@ -1907,9 +1956,12 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
             P.nco_blk = c.nco_blk; P.nchunk = c.nchunk; P.ntiles = c.ntiles;
             P.boxes_per_split = c.boxes_per_split; P.nsplit = c.nsplit;
             P.Cout = g.L.cout; P.Cpi = Li.Cpad;
+            // 2-CTA pairs of 128-channel output blocks when the channels pair up
+            const bool cta2 = g.L.cout % 256 == 0 && !getenv("SPLITCNN_NO_CTA2");
+            if (cta2) P.ntiles = c.ntiles / 2;
             const int Wp = 8 + g.L.kw - 1;
             const uint32_t a_stage = 2u * c.BH * c.BNn * 8u * 128u;
-            const uint32_t b_stage = ((uint32_t)Wp * c.BH * c.BNn * 128u + 1023u) & ~1023u;
+            const uint32_t b_stage = ((uint32_t)Wp * c.BH * c.BNn * (cta2 ? 64u : 128u) + 1023u) & ~1023u;
             const uint32_t stage_bytes = a_stage + b_stage;
             P.stages = std::min<int>(8, (int)((200u * 1024u) / stage_bytes));
             P.tmem_cols = 256;
@@ -1941,21 +1993,38 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
                     void *base = (char *)x + Li.offset(i, j) * 2;
                     cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)wp, (cuuint64_t)hp, (cuuint64_t)Li.N};
                     cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)wp * C * 2, (cuuint64_t)hp * wp * C * 2};
-                    cuuint32_t box[4] = {64, (cuuint32_t)Wp, (cuuint32_t)c.BH, (cuuint32_t)c.BNn};
+                    cuuint32_t box[4] = {cta2 ? 32u : 64u, (cuuint32_t)Wp, (cuuint32_t)c.BH, (cuuint32_t)c.BNn};
                     cuuint32_t es[4] = {1, 1, 1, 1};
                     if (encode(&P.mapX[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides, box, es,
-                               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+                               CU_TENSOR_MAP_INTERLEAVE_NONE, cta2 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B,
+                               CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
                         return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(X halo) failed");
                 }
             }
             P.box_prefix[P.npatch] = boxes;
             const size_t smem = 1024 + (size_t)P.stages * stage_bytes + 256;
             if (!halo_attr) {
-                cudaFuncSetAttribute(wgrad_halo_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+                cudaFuncSetAttribute(wgrad_halo_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+                cudaFuncSetAttribute(wgrad_halo_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
                 halo_attr = true;
             }
-            wgrad_halo_kernel<<<c.ntiles * c.nsplit, 192, smem, st>>>(P);
+            if (cta2) {
+                cudaLaunchConfig_t cfg = {};
+                cfg.gridDim = dim3((unsigned)(2 * P.ntiles * c.nsplit));
+                cfg.blockDim = dim3(192);
+                cfg.dynamicSmemBytes = smem;
+                cfg.stream = st;
+                cudaLaunchAttribute at[1];
+                at[0].id = cudaLaunchAttributeClusterDimension;
+                at[0].val.clusterDim.x = 2;
+                at[0].val.clusterDim.y = 1;
+                at[0].val.clusterDim.z = 1;
+                cfg.attrs = at;
+                cfg.numAttrs = 1;
+                cudaLaunchKernelEx(&cfg, wgrad_halo_kernel<true>, P);
+            } else {
+                wgrad_halo_kernel<false><<<c.ntiles * c.nsplit, 192, smem, st>>>(P);
+            }
             count_launch();
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("wgrad_halo_kernel: ") + cudaGetErrorString(e));

@@ -74,6 +74,7 @@ CONV_CASES = [
     ("c512", 1, 512, 512, 3, 1, 1, 14, 14, 2, 2, True),
     ("halo_odd_n", 3, 64, 64, 3, 1, 1, 14, 14, 2, 2, True),
     ("halo_uneven", 2, 128, 128, 3, 1, 1, 23, 19, 3, 2, True),
+    ("cta2_ragged", 3, 64, 256, 3, 1, 1, 21, 19, 3, 2, True),    # 2-CTA fwd + wgrad, odd M-box count
 ]
 
 

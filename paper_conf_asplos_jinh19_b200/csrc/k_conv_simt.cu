@@ -9,6 +9,9 @@
 //   DGRAD : M = N*Hp*Wp pixels, N = Cin_pad, K = kh*kw*Cout_pad; A = dY_p (strided gather), B = W
 //   WGRAD : M = Cout, N = kh*kw*Cin_pad, K = pixels of one chunk of one patch (split-K);
 //           partials -> workspace -> fixed-order reduction (deterministic)
+#include <algorithm>
+#include <type_traits>
+
 #include "common.cuh"
 #include "kernels.h"
 
@@ -201,13 +204,66 @@ __global__ void __launch_bounds__(NT) conv_simt_kernel(SimtArgs a) {
     }
 }
 
-// dW[i] = beta * dW[i] + sum_z part[z][i]   (z ascending: fixed order)
-__global__ void __launch_bounds__(256) reduce_partials_kernel(const float *__restrict__ part, int Z, int64_t n,
-                                                              float *__restrict__ out, float beta) {
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        float s = 0.f;
-        for (int z = 0; z < Z; ++z) s += part[(int64_t)z * n + i];
-        out[i] = (beta != 0.f ? beta * out[i] : 0.f) + s;
+// out[i] = beta * out[i] + sum_z part[z][i] for two segments (blockIdx.y: 0 = dW, 1 = db).  A block is
+// 32 column lanes x 8 z-slices: slice k sums z = k, k+8, ... in ascending order, then slice 0 adds the
+// 8 slice sums in ascending slice order -- a fixed summation tree independent of scheduling, so the
+// result is bitwise reproducible.  VEC = 4: each column lane owns 4 consecutive floats (n % 4 == 0).
+template <int VEC>
+__global__ void __launch_bounds__(256) reduce_partials_kernel(const float *__restrict__ part0, int64_t n0,
+                                                              float *__restrict__ out0, int Z0,
+                                                              const float *__restrict__ part1, int64_t n1,
+                                                              float *__restrict__ out1, int Z1, float beta) {
+    using V = typename std::conditional<VEC == 4, float4, float>::type;
+    const int Z = blockIdx.y ? Z1 : Z0;
+    const float *part = blockIdx.y ? part1 : part0;
+    float *out = blockIdx.y ? out1 : out0;
+    const int64_t nv = (blockIdx.y ? n1 : n0) / VEC;
+    const int64_t col = (int64_t)blockIdx.x * 32 + (threadIdx.x & 31);
+    const int zs = threadIdx.x >> 5;
+    __shared__ V red[8][32];
+    if ((int64_t)blockIdx.x * 32 >= nv) return;   // whole block idle (the shorter segment)
+    V s;
+    float *sf = reinterpret_cast<float *>(&s);
+#pragma unroll
+    for (int e = 0; e < VEC; ++e) sf[e] = 0.f;
+    if (col < nv) {
+        const V *pv = reinterpret_cast<const V *>(part) + col;
+        int z = zs;
+        for (; z + 24 < Z; z += 32) {   // 4 independent loads in flight, added in z order
+            const V a = __ldg(pv + (int64_t)z * nv), b = __ldg(pv + (int64_t)(z + 8) * nv);
+            const V c = __ldg(pv + (int64_t)(z + 16) * nv), d = __ldg(pv + (int64_t)(z + 24) * nv);
+            const float *af = reinterpret_cast<const float *>(&a), *bf = reinterpret_cast<const float *>(&b);
+            const float *cf = reinterpret_cast<const float *>(&c), *df = reinterpret_cast<const float *>(&d);
+#pragma unroll
+            for (int e = 0; e < VEC; ++e) sf[e] = (((sf[e] + af[e]) + bf[e]) + cf[e]) + df[e];
+        }
+        for (; z < Z; z += 8) {
+            const V a = __ldg(pv + (int64_t)z * nv);
+            const float *af = reinterpret_cast<const float *>(&a);
+#pragma unroll
+            for (int e = 0; e < VEC; ++e) sf[e] += af[e];
+        }
+    }
+    red[zs][threadIdx.x & 31] = s;
+    __syncthreads();
+    if (zs == 0 && col < nv) {
+        V t = red[0][threadIdx.x];
+        float *tf = reinterpret_cast<float *>(&t);
+#pragma unroll
+        for (int k = 1; k < 8; ++k) {
+            const V u = red[k][threadIdx.x];
+            const float *uf = reinterpret_cast<const float *>(&u);
+#pragma unroll
+            for (int e = 0; e < VEC; ++e) tf[e] += uf[e];
+        }
+        V *ov = reinterpret_cast<V *>(out) + col;
+        if (beta != 0.f) {
+            const V o = *ov;
+            const float *of = reinterpret_cast<const float *>(&o);
+#pragma unroll
+            for (int e = 0; e < VEC; ++e) tf[e] += beta * of[e];
+        }
+        *ov = t;
     }
 }
 
@@ -265,9 +321,20 @@ int launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, flo
     return Zr;
 }
 
-void launch_reduce(const float *part, int Z, int64_t n, float *out, float beta, cudaStream_t st) {
-    reduce_partials_kernel<<<(unsigned)std::min<int64_t>((n + 255) / 256, 4096), 256, 0, st>>>(part, Z, n, out, beta);
+void launch_reduce2(const float *part0, int64_t n0, float *out0, int Z0, const float *part1, int64_t n1, float *out1,
+                    int Z1, float beta, cudaStream_t st) {
+    if (!part1 || !out1) n1 = 0;
+    auto al16 = [](const void *q) { return ((uintptr_t)q & 15) == 0; };
+    const bool vec = n0 % 4 == 0 && n1 % 4 == 0 && al16(part0) && al16(out0) && (n1 == 0 || (al16(part1) && al16(out1)));
+    const int64_t cols = std::max(n0, n1) / (vec ? 4 : 1);
+    dim3 grid((unsigned)((cols + 31) / 32), n1 > 0 ? 2 : 1);
+    if (vec) reduce_partials_kernel<4><<<grid, 256, 0, st>>>(part0, n0, out0, Z0, part1, n1, out1, Z1, beta);
+    else reduce_partials_kernel<1><<<grid, 256, 0, st>>>(part0, n0, out0, Z0, part1, n1, out1, Z1, beta);
     count_launch();
+}
+
+void launch_reduce(const float *part, int Z, int64_t n, float *out, float beta, cudaStream_t st) {
+    launch_reduce2(part, n, out, Z, nullptr, 0, nullptr, 0, beta, st);
 }
 
 static int64_t max_pixels(const Level &L, int p0, int p1) {
@@ -336,10 +403,10 @@ void launch_conv_wgrad_simt(splitcnn_dtype_t dt, const Level &Li, const Level &L
     else conv_simt_kernel<float, MODE_WGRAD><<<grid, NT, 0, st>>>(a);
     count_launch();
     const int64_t n = (int64_t)g.L.cout * ncols;
-    { reduce_partials_kernel<<<(unsigned)std::min<int64_t>((n + 255) / 256, 4096), 256, 0, st>>>(part, Z, n, dw, beta); count_launch(); }
+    launch_reduce(part, Z, n, dw, beta, st);
     if (db) {
         const int Zd = launch_db_partials(dt, Lo, dy, part_db, g.L.cout, p0, p1, st);
-        { reduce_partials_kernel<<<(g.L.cout + 255) / 256, 256, 0, st>>>(part_db, Zd, g.L.cout, db, beta); count_launch(); }
+        launch_reduce(part_db, Zd, g.L.cout, db, beta, st);
     }
 }
 

@@ -414,7 +414,10 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 if (pr < h8_npairs) {
                     const int t0 = 2 * pr, t1 = 2 * pr + 1;
                     const int o0 = (t0 / p.kw) * p.Wp + (t0 % p.kw);
-                    const int o1 = t1 < KT ? (t1 / p.kw) * p.Wp + (t1 % p.kw) : o0 + 1;
+                    // a missing second tap (odd KT) re-reads tap t0's pixels (LBO = 0) against zero weights:
+                    // a view one pixel on would leave the loaded box for the tile's last row and multiply
+                    // stale shared memory (possibly NaN / Inf) by zero
+                    const int o1 = t1 < KT ? (t1 / p.kw) * p.Wp + (t1 % p.kw) : o0;
                     h8_adesc[pr] = tc::smem_desc(0, 16u * (uint32_t)(o1 - o0), (uint32_t)p.Wp * 16u, 0) + (uint64_t)o0;
                     h8_bdesc[pr] = tc::smem_desc(0, 16, 1024, 2) + (uint64_t)((((pr >> 2) * p.BN) * 128 + 32 * (pr & 3)) >> 4);
                 }
@@ -1843,23 +1846,35 @@ static bool wgrad_tc_ok(const Level &Li, const Level &Lo, const LayerGeom &g) {
     return a_channels_ok(Li.Cpad) && Lo.Cpad % 64 == 0 && g.L.sh == g.L.sw && g.L.sh <= 2;
 }
 
-size_t wgrad_tc_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g) {
-    // sized for the full patch range in groups of TC_MAXP patches (the largest group decides)
-    size_t best = 0;
-    const int np = Lo.npatch();
-    for (int g0 = 0; g0 < np; g0 += TC_MAXP) {
-        WgradCfg c = wgrad_cfg(Li, Lo, g, g0, std::min(np, g0 + TC_MAXP));
-        best = std::max(best, (size_t)c.nsplit * g.L.cout * g.L.kh * g.L.kw * Li.Cpad * sizeof(float));
-        if (wgrad_halo_ok(Li, Lo, g)) {
-            WgHaloCfg h = wgrad_halo_cfg(Li, Lo, g, g0, std::min(np, g0 + TC_MAXP));
-            best = std::max(best, (size_t)h.nsplit * g.L.cout * g.L.kh * g.L.kw * Li.Cpad * sizeof(float));
-        }
-        if (wgrad_narrow_ok(Li, Lo, g) && !getenv("SPLITCNN_NO_NARROW_WGRAD")) {
-            WgNarrowCfg h = wgrad_narrow_cfg(Lo, g, g0, std::min(np, g0 + TC_MAXP));
-            best = std::max(best, (size_t)h.nsplit * g.L.cout * g.L.kh * g.L.kw * Li.Cpad * sizeof(float));
-        }
+// which weight-gradient kernel takes a layer: 2 narrow (8-channel input), 1 halo, 0 generic
+static int wgrad_path(const Level &Li, const Level &Lo, const LayerGeom &g) {
+    if (wgrad_narrow_ok(Li, Lo, g) && !getenv("SPLITCNN_NO_NARROW_WGRAD")) return 2;
+    if (wgrad_halo_ok(Li, Lo, g)) return 1;
+    return 0;
+}
+
+// upper bound of the split count of ONE launch (any group of <= TC_MAXP patches): see the *_cfg Z caps
+static int wgrad_zbound(int path, const Level &Li, const LayerGeom &g) {
+    const int nco = (g.L.cout + 127) / 128;
+    int ntiles;
+    if (path == 2) return std::max(1, std::min(296, (2 * num_sms() + nco - 1) / nco));
+    if (path == 1) ntiles = nco * g.L.kh * (Li.Cpad / 64);
+    else {
+        const int cbox = std::min(Li.Cpad, 64), nblocks = g.L.kh * g.L.kw * (Li.Cpad / cbox);
+        const int maxb = std::min(WG_MAXBLK, 256 / cbox);
+        ntiles = nco * ((nblocks + maxb - 1) / maxb);
     }
-    return std::max(best, (size_t)4 * 148 * g.L.cout * sizeof(float)) + 256;  // db partials reuse the space
+    return std::max(1, std::min(128, (2 * num_sms() + ntiles - 1) / ntiles));
+}
+
+size_t wgrad_tc_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g) {
+    // every launch (group of <= TC_MAXP patches) of a call writes its split partials at its own z
+    // offset and ONE fixed-order reduction sums them all: [Zmax][dW]; the db column sums reuse the space
+    const int path = wgrad_path(Li, Lo, g);
+    const int64_t ngroups = (Lo.npatch() + TC_MAXP - 1) / TC_MAXP;
+    const int64_t zmax = ngroups * wgrad_zbound(path, Li, g);
+    const int64_t nW = (int64_t)g.L.cout * g.L.kh * g.L.kw * Li.Cpad;
+    return std::max((size_t)zmax * nW * sizeof(float), (size_t)4 * 148 * g.L.cout * sizeof(float)) + 256;
 }
 
 int launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, float *part, int cout, int p0, int p1,
@@ -1874,9 +1889,11 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
     const int64_t nW = (int64_t)g.L.cout * KT * Li.Cpad;
     float *part = (float *)ws;
     static bool attr_set = false;
-    bool first = true;
+    const int path = wgrad_path(Li, Lo, g);
+    const int64_t zcap = (int64_t)((Lo.npatch() + TC_MAXP - 1) / TC_MAXP) * wgrad_zbound(path, Li, g);
+    int zoff = 0;   // split partials written so far (all launches of this call)
     int gend = p1;  // end of the patch range left for the generic kernel
-    if (wgrad_narrow_ok(Li, Lo, g) && !getenv("SPLITCNN_NO_NARROW_WGRAD")) {
+    if (path == 2) {
         static bool narrow_attr = false;
         for (int g0 = p0; g0 < p1; g0 += TC_MAXP) {
             const int g1 = std::min(p1, g0 + TC_MAXP);
@@ -1895,7 +1912,7 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
             uint32_t cols = 32;
             while (cols < (uint32_t)(g.L.kh * (((g.L.kw * 8 + 15) / 16) * 16))) cols <<= 1;
             P.tmem_cols = cols;
-            P.part = part;
+            P.part = part + (int64_t)zoff * nW;
             int boxes = 0;
             for (int q = g0; q < g1; ++q) {
                 const int ql = q - g0, i = q / Lo.nw(), j = q % Lo.nw();
@@ -1940,11 +1957,10 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
             count_launch();
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("wgrad_narrow_kernel: ") + cudaGetErrorString(e));
-            launch_reduce(part, c.nsplit, nW, dw, first ? beta : 1.f, st);
-            first = false;
+            zoff += c.nsplit;
         }
         gend = p0;
-    } else if (wgrad_halo_ok(Li, Lo, g)) {
+    } else if (path == 1) {
         static bool halo_attr = false;
         for (int g0 = p0; g0 < p1; g0 += TC_MAXP) {
             const int g1 = std::min(p1, g0 + TC_MAXP);
@@ -1965,7 +1981,7 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
             const uint32_t stage_bytes = a_stage + b_stage;
             P.stages = std::min<int>(8, (int)((200u * 1024u) / stage_bytes));
             P.tmem_cols = 256;
-            P.part = part;
+            P.part = part + (int64_t)zoff * nW;
             int boxes = 0;
             for (int q = g0; q < g1; ++q) {
                 const int ql = q - g0, i = q / Lo.nw(), j = q % Lo.nw();
@@ -2028,8 +2044,7 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
             count_launch();
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("wgrad_halo_kernel: ") + cudaGetErrorString(e));
-            launch_reduce(part, c.nsplit, nW, dw, first ? beta : 1.f, st);
-            first = false;
+            zoff += c.nsplit;
         }
         gend = p0;  // done: skip the generic path below
     }
@@ -2062,7 +2077,7 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
         uint32_t cols = 32;
         while (cols < (uint32_t)(c.bpt_pad * c.cbox)) cols <<= 1;
         P.tmem_cols = cols;
-        P.part = part;
+        P.part = part + (int64_t)zoff * nW;
         int boxes = 0;
         for (int q = g0; q < g1; ++q) {
             const int ql = q - g0, i = q / Lo.nw(), j = q % Lo.nw();
@@ -2120,10 +2135,12 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
         count_launch();
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("wgrad_tc_kernel: ") + cudaGetErrorString(e));
-        // fixed-order sum of the split partials (and the previous groups' result) into dW
-        launch_reduce(part, c.nsplit, nW, dw, first ? beta : 1.f, st);
-        first = false;
+        zoff += c.nsplit;
     }
+    if (zoff > zcap) return fail(SPLITCNN_ERR_UNSUPPORTED, "wgrad split partials exceed the workspace bound");
+    // ONE fixed-order sum of every launch's split partials (z ascending) into dW: bitwise
+    // reproducible, and beta = 1 gives exactly 2x whatever the number of launches
+    launch_reduce(part, zoff, nW, dw, beta, st);
     if (db) {
         // the dW partials have been consumed by the reduction (stream order): reuse the space
         const int Zd = launch_db_partials(SPLITCNN_BF16, Lo, dy, part, g.L.cout, p0, p1, st);

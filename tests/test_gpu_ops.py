@@ -75,6 +75,8 @@ CONV_CASES = [
     ("halo_odd_n", 3, 64, 64, 3, 1, 1, 14, 14, 2, 2, True),
     ("halo_uneven", 2, 128, 128, 3, 1, 1, 23, 19, 3, 2, True),
     ("cta2_ragged", 3, 64, 256, 3, 1, 1, 21, 19, 3, 2, True),    # 2-CTA fwd + wgrad, odd M-box count
+    ("groups_81", 1, 64, 128, 3, 1, 1, 38, 36, 9, 9, True),      # > 64 patches: two launches per pass
+    ("narrow_groups_81", 1, 3, 64, 3, 1, 1, 38, 36, 9, 9, True),
 ]
 
 

@@ -472,13 +472,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                         const uint64_t b0 = p.bres ? tc::smem_desc(tc::smem_u32(sW) + (uint32_t)(ks * p.kw * p.BNh) * 128u, 16, 1024, 2)
                                                    : tc::smem_desc(b_base, 16, 1024, 2);
                         const uint32_t bstep = (uint32_t)p.BNh * 8u;
-                        for (int c = 0; c < p.kw; ++c) {
-                            const uint64_t ac = a0 + (uint64_t)(8 * c), bc = b0 + (uint64_t)(bstep * c);
-                            tc::mma2_bf16_ws(d, ac, bc, idesc, (ks | c) != 0);
-                            tc::mma2_bf16_ws(d, ac + 2, bc + 2, idesc, 1u);
-                            tc::mma2_bf16_ws(d, ac + 4, bc + 4, idesc, 1u);
-                            tc::mma2_bf16_ws(d, ac + 6, bc + 6, idesc, 1u);
-                        }
+                        for (int c = 0; c < p.kw; ++c)
+                            tc::mma2_bf16_x4_ws(d, a0 + (uint64_t)(8 * c), b0 + (uint64_t)(bstep * c), idesc, (ks | c) != 0);
                         tc::mma2_commit_mc_ws(&empty[stage]);
                         if (++stage == S) { stage = 0; ph ^= 1; }
                         continue;
@@ -486,8 +481,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     if (CTA2) {
                         const uint64_t a0 = tc::smem_desc(a_base, 16, 1024, 2);
                         const uint64_t b0 = tc::smem_desc(b_base, 16, 1024, 2);
-#pragma unroll
-                        for (int j = 0; j < 4; ++j) tc::mma2_bf16_ws(d, a0 + (uint64_t)(2 * j), b0 + (uint64_t)(2 * j), idesc, (ks | j) != 0);
+                        tc::mma2_bf16_x4_ws(d, a0, b0, idesc, ks != 0);
                         tc::mma2_commit_mc_ws(&empty[stage]);
                         if (++stage == S) { stage = 0; ph ^= 1; }
                         continue;
@@ -500,13 +494,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                         const uint64_t b0 = p.bres ? tc::smem_desc(tc::smem_u32(sW) + (uint32_t)(ks * p.kw * p.BN) * 128u, 16, 1024, 2)
                                                    : tc::smem_desc(b_base, 16, 1024, 2);
                         const uint32_t bstep = (uint32_t)p.BN * 8u;   // BN*128 B >> 4
-                        for (int c = 0; c < p.kw; ++c) {
-                            const uint64_t ac = a0 + (uint64_t)(8 * c), bc = b0 + (uint64_t)(bstep * c);
-                            tc::mma_bf16_ws(d, ac, bc, idesc, (ks | c) != 0);
-                            tc::mma_bf16_ws(d, ac + 2, bc + 2, idesc, 1u);
-                            tc::mma_bf16_ws(d, ac + 4, bc + 4, idesc, 1u);
-                            tc::mma_bf16_ws(d, ac + 6, bc + 6, idesc, 1u);
-                        }
+                        for (int c = 0; c < p.kw; ++c)
+                            tc::mma_bf16_x4_ws(d, a0 + (uint64_t)(8 * c), b0 + (uint64_t)(bstep * c), idesc, (ks | c) != 0);
                         if (!(p.dbg & 32)) tc::mma_commit_ws(&empty[stage]);
                         if (++stage == S) { stage = 0; ph ^= 1; }
                         continue;

@@ -1,6 +1,6 @@
 #!/bin/bash
 for L in ${TLAYERS:-conv1_1 conv1_2 conv4_2}; do
-SPLITCNN_TRACE=1 timeout 120 python - $L <<'PY' 2>&1 | grep -v "^  *[0-9]*:" | head -40
+SPLITCNN_TRACE=1 timeout 120 python - $L <<'PY' 2>&1 | grep -v "trace CTA (block" | head -${TLINES:-40}
 import os, sys, torch
 sys.argv = ["x", sys.argv[1]]
 sys.path.insert(0, os.getcwd())

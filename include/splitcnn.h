@@ -187,6 +187,27 @@ SPLITCNN_API splitcnn_status_t splitcnn_conv_fwd(splitcnn_plan_t plan, int32_t l
                                     const void *x, const void *w, const float *bias, void *y,
                                     uint32_t flags, int32_t p0, int32_t p1, splitcnn_stream_t stream);
 
+/* Fused forward of a conv (+bias, ReLU) `layer` and the 2x2 / stride-2 / unpadded max-pool
+ * `layer + 1` that follows it (ReLU in place): the tcgen05 epilogue pools the
+ * bf16-rounded conv outputs of each tile and writes ONLY the pool's output y_pool (level layer+2
+ * patches) and its argmax bytes (same layout as y_pool; window index r*2 + c of the first maximum,
+ * bit 7 = [max > 0], exactly as splitcnn_pool_fwd with FLAG_POOL_RELU_MASK).  The conv output
+ * (level layer+1) is never materialised: the backward pass needs only the argmax (pool_bwd with
+ * FLAG_POOL_RELU_MASK applies the ReLU mask).  Results are bitwise equal to conv_fwd followed by
+ * pool_fwd.  Patch-local pool windows never straddle a tile: the pool's I = 2*O (R2) makes every conv
+ * output patch extent even.  flags must hold RELU | POOL_RELU_MASK.
+ * Errors: ERR_UNSUPPORTED when the pair is not fusable (see splitcnn_conv_pool_supported; callers
+ * then run conv_fwd + pool_fwd). */
+SPLITCNN_API splitcnn_status_t splitcnn_conv_pool_fwd(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                         const void *x, const void *w, const float *bias, void *y_pool,
+                                         uint8_t *argmax, uint32_t flags, int32_t p0, int32_t p1,
+                                         splitcnn_stream_t stream);
+/* *supported = 1 when splitcnn_conv_pool_fwd takes (layer, layer + 1) for dtype: BF16, a conv on the
+ * tcgen05 path other than the 8-channel-input one, Cout a multiple of 16 equal to its channel pad,
+ * followed by a 2x2 / stride-2 max-pool with zero pads. */
+SPLITCNN_API splitcnn_status_t splitcnn_conv_pool_supported(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                               int32_t *supported);
+
 /* Data gradient (adjoint of Eq. 6 within each patch):
  *   dX_p[n,h,w,ci] = sum over co, r, c with oh = (h + pt - r)/sh integral and in range
  *                    of dY_p[n,oh,ow,co] W[co,r,c,ci],   then * [relu_src > 0] if relu_src.

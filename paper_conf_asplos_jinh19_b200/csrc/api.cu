@@ -162,6 +162,51 @@ extern "C" splitcnn_status_t splitcnn_conv_fwd(splitcnn_plan_t plan, int32_t lay
     return check_launch("conv_fwd");
 }
 
+// conv `layer` (+bias, ReLU) followed by a 2x2 / stride-2 / unpadded max-pool `layer + 1` whose
+// epilogue the tcgen05 kernel can take
+static bool conv_pool_fusable(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype) {
+    if (layer < 0 || layer + 1 >= (int)plan->layers.size()) return false;
+    const LayerGeom &g = plan->layers[layer], &q = plan->layers[layer + 1];
+    if (g.L.op != SPLITCNN_OP_CONV || q.L.op != SPLITCNN_OP_MAXPOOL) return false;
+    if (q.L.kh != 2 || q.L.kw != 2 || q.L.sh != 2 || q.L.sw != 2) return false;
+    for (int v : q.pad_h) if (v) return false;
+    for (int v : q.pad_w) if (v) return false;
+    const Level &Li = plan->levels[layer], &Lo = plan->levels[layer + 1];
+    if (!conv_tc_supported(0, dtype, Li, Lo, g)) return false;
+    if (Li.Cpad == 8 && g.L.sh == 1) return false;            // 8-channel halo path: no fused variant
+    if (g.L.cout != Lo.Cpad || g.L.cout % 16) return false;   // every stored channel is a real one
+    return true;
+}
+
+extern "C" splitcnn_status_t splitcnn_conv_pool_supported(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                                          int32_t *supported) {
+    if (!plan || !supported) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    TRY(check_dtype(dtype));
+    *supported = conv_pool_fusable(plan, layer, dtype) ? 1 : 0;
+    return SPLITCNN_OK;
+}
+
+extern "C" splitcnn_status_t splitcnn_conv_pool_fwd(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                                    const void *x, const void *w, const float *bias, void *y_pool,
+                                                    uint8_t *argmax, uint32_t flags, int32_t p0, int32_t p1,
+                                                    splitcnn_stream_t stream) {
+    TRY(check_layer(plan, layer, SPLITCNN_OP_CONV));
+    TRY(check_dtype(dtype));
+    if (!x || !w || !y_pool || !argmax) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    NEED_ALIGNED(x, "x");
+    NEED_ALIGNED(w, "w");
+    NEED_ALIGNED(y_pool, "y_pool");
+    NEED_ALIGNED(argmax, "argmax");
+    const uint32_t need = SPLITCNN_FLAG_RELU | SPLITCNN_FLAG_POOL_RELU_MASK;
+    if ((flags & need) != need || (flags & SPLITCNN_FLAG_FORCE_SIMT) || !conv_pool_fusable(plan, layer, dtype))
+        return fail(SPLITCNN_ERR_UNSUPPORTED, "conv_pool_fwd: not a fusable conv(+ReLU) -> 2x2/s2 max-pool pair");
+    TRY(check_range(plan, layer, p0, p1));
+    if (p1 == p0) return SPLITCNN_OK;
+    TRY(launch_conv_pool_fwd_tc(plan->levels[layer], plan->levels[layer + 1], plan->levels[layer + 2], plan->layers[layer],
+                                x, w, bias, y_pool, argmax, p0, p1, (cudaStream_t)stream));
+    return check_launch("conv_pool_fwd");
+}
+
 extern "C" splitcnn_status_t splitcnn_conv_bwd_data(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
                                                     const void *dy, const void *w, void *dx, const void *relu_src,
                                                     void *ws, size_t ws_bytes, uint32_t flags, int32_t p0, int32_t p1,

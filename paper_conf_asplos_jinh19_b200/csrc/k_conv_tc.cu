@@ -86,6 +86,10 @@ struct TcConvParams {
     int uni;                      // every patch has the same tile grid: O(1) decode by fast division
     FastDiv fd_tpp, fd_mtpp, fd_nco, fd_nwb, fd_nhb;
     int ysh;                      // log2(ychunk)
+    // fused 2x2 / stride-2 max-pool epilogue (POOL): pooled values + argmax bytes of level layer+2
+    __nv_bfloat16 *pool_y;
+    uint8_t *pool_a;
+    int64_t pool_off[TC_MAXP];
 };
 
 static_assert(sizeof(TcConvParams) <= 32700, "kernel parameter space is 32 KB");
@@ -223,10 +227,91 @@ __device__ __forceinline__ uint4 epi8(const uint32_t *r, const float *sb, int co
     return pk;
 }
 
+// Fused 2x2 / stride-2 max-pool of 16 accumulator columns (pool semantics of
+// pool_fwd_kernel: max over the window of the bf16-ROUNDED conv outputs, argmax = r*2 + c of the FIRST
+// maximum in window order, bit 7 = [max > 0]).  Rows are pixels (w fastest, BW a power of two, BH even),
+// so the window partners of row m are m^1 (c) and m^BW (r), both in the same warp: two shuffle rounds.
+// All lanes take part; `writer` (w and h even, pixel in range) stores 16 pooled values (32 B) and 16
+// argmax bytes (16 B).
+__device__ __forceinline__ void pool16(const float *v, int bw, bool writer, __nv_bfloat16 *yp, uint8_t *ap) {
+    float best[16];
+    uint32_t arg = 0;   // 2 bits per column
+#pragma unroll
+    for (int e = 0; e < 16; ++e) best[e] = __bfloat162float(__float2bfloat16_rn(v[e]));
+#pragma unroll
+    for (int e = 0; e < 16; ++e) {   // column partner: window index c = 1 (valid for even-w rows)
+        const float o = __shfl_xor_sync(0xffffffffu, best[e], 1);
+        if (o > best[e]) { best[e] = o; arg |= 1u << (2 * e); }
+    }
+    const uint32_t oarg = __shfl_xor_sync(0xffffffffu, arg, bw);
+#pragma unroll
+    for (int e = 0; e < 16; ++e) {   // row partner: window indices 2 + c (valid for even-h rows)
+        const float o = __shfl_xor_sync(0xffffffffu, best[e], bw);
+        if (o > best[e]) { best[e] = o; arg = (arg & ~(3u << (2 * e))) | ((2u + ((oarg >> (2 * e)) & 1u)) << (2 * e)); }
+    }
+    if (!writer) return;
+    uint4 pk[2];
+    __nv_bfloat162 *h2 = reinterpret_cast<__nv_bfloat162 *>(pk);
+#pragma unroll
+    for (int e = 0; e < 8; ++e) h2[e] = __floats2bfloat162_rn(best[2 * e], best[2 * e + 1]);
+    reinterpret_cast<uint4 *>(yp)[0] = pk[0];
+    reinterpret_cast<uint4 *>(yp)[1] = pk[1];
+    uint32_t ab[4] = {0, 0, 0, 0};
+#pragma unroll
+    for (int e = 0; e < 16; ++e)
+        ab[e >> 2] |= (((arg >> (2 * e)) & 3u) | (best[e] > 0.f ? 0x80u : 0u)) << (8 * (e & 3));
+    *reinterpret_cast<uint4 *>(ap) = make_uint4(ab[0], ab[1], ab[2], ab[3]);
+}
+
+// The same on 32 columns already packed as bf16x2 words w[16] (the conv epilogue's rounded values):
+// bf16x2 compares (__hgt2_mask) and bitwise selects, so a tie keeps the FIRST element bit for bit
+// (as pool_fwd_kernel's strict '>') and half the shuffles of the fp32 form.
+__device__ __forceinline__ uint32_t bsel(uint32_t m, uint32_t a, uint32_t b) { return (a & m) | (b & ~m); }
+__device__ __forceinline__ uint32_t hgt2(uint32_t a, uint32_t b) {
+    return __hgt2_mask(*reinterpret_cast<const __nv_bfloat162 *>(&a), *reinterpret_cast<const __nv_bfloat162 *>(&b));
+}
+__device__ __forceinline__ void pool32(const uint32_t *w, int bw, bool writer, __nv_bfloat16 *yp, uint8_t *ap) {
+    uint32_t best[16], cmask[16], amask[16];
+#pragma unroll
+    for (int e = 0; e < 16; ++e) {   // column partner (window index c = 1)
+        const uint32_t o = __shfl_xor_sync(0xffffffffu, w[e], 1);
+        cmask[e] = hgt2(o, w[e]);
+        best[e] = bsel(cmask[e], o, w[e]);
+    }
+#pragma unroll
+    for (int e = 0; e < 16; ++e) {   // row partner (window indices 2 + c)
+        const uint32_t o = __shfl_xor_sync(0xffffffffu, best[e], bw);
+        const uint32_t oc = __shfl_xor_sync(0xffffffffu, cmask[e], bw);
+        const uint32_t m = hgt2(o, best[e]);
+        best[e] = bsel(m, o, best[e]);
+        // per half: bit 1 = row index (m), bit 0 = column index of the winning row
+        amask[e] = (m & 0x00020002u) | (bsel(m, oc, cmask[e]) & 0x00010001u);
+    }
+    if (!writer) return;
+    uint4 *y4 = reinterpret_cast<uint4 *>(yp);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) y4[q] = make_uint4(best[4 * q], best[4 * q + 1], best[4 * q + 2], best[4 * q + 3]);
+    uint32_t ab[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+        uint32_t v = 0;
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const uint32_t wd = best[2 * q + h], am = amask[2 * q + h];
+            const uint32_t lo = (am & 3u) | ((wd & 0x7FFFu) ? 0x80u : 0u);            // element 2(2q+h)
+            const uint32_t hi = ((am >> 16) & 3u) | ((wd & 0x7FFF0000u) ? 0x80u : 0u); // element 2(2q+h)+1
+            v |= (lo | (hi << 8)) << (16 * h);
+        }
+        ab[q] = v;
+    }
+    reinterpret_cast<uint4 *>(ap)[0] = make_uint4(ab[0], ab[1], ab[2], ab[3]);
+    reinterpret_cast<uint4 *>(ap)[1] = make_uint4(ab[4], ab[5], ab[6], ab[7]);
+}
+
 #define TC_TRACE(i, e) \
     do { if (p.trace && blockIdx.x == 0 && (i) < 256) p.trace[(i) * 8 + (e)] = clock64(); } while (0)
 
-template <bool BIAS, bool RELU, bool MASK, bool CTA2>
+template <bool BIAS, bool RELU, bool MASK, bool CTA2, bool POOL = false>
 __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_constant__ TcConvParams p) {
     extern __shared__ uint8_t smem_raw[];
     uint8_t *smem = smem_raw + ((1024u - (tc::smem_u32(smem_raw) & 1023u)) & 1023u);   // keeps the shared space
@@ -537,6 +622,55 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             const int ow0 = wb * p.BW, oh0 = hb * p.BH, n0 = nb * p.BNn;
             const int ncols = min(p.BN, p.Cpo - co0);
             const int nchunks = ncols / p.ychunk;
+            if (POOL) {
+                // pooled outputs straight from registers: no staging tile, no store of the conv output
+                tc::mbar_wait(&tfull[g], aph);
+                if (gtid == 0) TC_TRACE(it, 3);
+                tc::tc_fence_after();
+                const uint32_t tacc = tmem_base + (uint32_t)(g * p.BN) + ((uint32_t)(quad * 32) << 16);
+                const int wi = row & (p.BW - 1), hi = (row / p.BW) % p.BH, ni = row / (p.BW * p.BH);
+                const int n = n0 + ni, ph = (oh0 + hi) >> 1, pw = (ow0 + wi) >> 1;
+                const int poh = p.out_h[ql] >> 1, pow_ = p.out_w[ql] >> 1;
+                const bool writer = valid && !(wi & 1) && !(hi & 1) && row < p.rows_box && n < p.N && ph < poh && pw < pow_;
+                const int64_t pix = p.pool_off[ql] + (((int64_t)n * poh + ph) * pow_ + pw) * p.Cpo + co0;
+                for (int cc = 0; cc < ncols; cc += 32) {   // ncols % 16 == 0; two loads in flight
+                    uint32_t r2[2][16];
+                    tc::tmem_ld16_nw(tacc + cc, r2[0]);
+                    if (cc + 16 < ncols) tc::tmem_ld16_nw(tacc + cc + 16, r2[1]);
+                    tc::tmem_wait_ld();
+                    if (cc + 32 <= ncols) {   // 32 columns: bias/ReLU/round as the stored-conv epilogue, pool packed
+                        uint4 pk[4];
+#pragma unroll
+                        for (int u = 0; u < 4; ++u)
+                            pk[u] = epi8_full<BIAS, RELU, false>(r2[u >> 1] + 8 * (u & 1), sbias + co0 + cc + 8 * u,
+                                                                 make_uint4(0, 0, 0, 0));
+                        pool32(reinterpret_cast<const uint32_t *>(pk), p.BW, writer, p.pool_y + pix + cc, p.pool_a + pix + cc);
+                        continue;
+                    }
+#pragma unroll
+                    for (int hh = 0; hh < 2; ++hh) {
+                        if (cc + 16 * hh >= ncols) break;
+                        float v[16];
+#pragma unroll
+                        for (int e = 0; e < 16; ++e) {
+                            float o = __uint_as_float(r2[hh][e]);
+                            if (BIAS) o += sbias[co0 + cc + 16 * hh + e];
+                            if (RELU) o = fmaxf(o, 0.f);
+                            v[e] = o;
+                        }
+                        pool16(v, p.BW, writer, p.pool_y + pix + cc + 16 * hh, p.pool_a + pix + cc + 16 * hh);
+                    }
+                }
+                tc::tc_fence_before();
+                __syncwarp();
+                if (lane == 0) {
+                    if (CTA2) tc::mbar_arrive_remote(tempty_l);
+                    else tc::mbar_arrive(&tempty[g]);
+                }
+                if (gtid == 0) TC_TRACE(it, 4);
+                aph ^= 1;
+                continue;
+            }
             if (gtid == 0) tc::bulk_wait_read0();      // this group's previous store has read the staging
             tc::named_bar_sync(1 + g, 128);
             if (MASK && valid) {
@@ -626,6 +760,37 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             const int ncols = min(p.BN, p.Cpo - co0);       // channels this tile stores (multiple of ychunk)
             const int nchunks = ncols / p.ychunk;
             uint8_t *sYb = sY + (size_t)yb * p.ybuf_bytes;
+            if (POOL) {   // fused max-pool: 16-column groups interleaved between the two column halves
+                tc::mbar_wait(&tfull[acc], aph);
+                tc::tc_fence_after();
+                const uint32_t tacc = tmem_base + (uint32_t)(acc * p.BN) + ((uint32_t)(quad * 32) << 16);
+                const int wi = row & (p.BW - 1), hi = (row / p.BW) % p.BH, ni = row / (p.BW * p.BH);
+                const int n = n0 + ni, ph = (oh0 + hi) >> 1, pw = (ow0 + wi) >> 1;
+                const int poh = p.out_h[ql] >> 1, pow_ = p.out_w[ql] >> 1;
+                const bool writer = valid && !(wi & 1) && !(hi & 1) && row < p.rows_box && n < p.N && ph < poh && pw < pow_;
+                const int64_t pix = p.pool_off[ql] + (((int64_t)n * poh + ph) * pow_ + pw) * p.Cpo + co0;
+                for (int cc = 16 * half; cc < ncols; cc += 32) {
+                    float v[16];
+                    tc::tmem_ld16(tacc + cc, v);
+#pragma unroll
+                    for (int e = 0; e < 16; ++e) {
+                        float o = v[e];
+                        if (BIAS) o += sbias[co0 + cc + e];
+                        if (RELU) o = fmaxf(o, 0.f);
+                        v[e] = o;
+                    }
+                    pool16(v, p.BW, writer, p.pool_y + pix + cc, p.pool_a + pix + cc);
+                }
+                tc::tc_fence_before();
+                __syncwarp();
+                if (lane == 0) {
+                    if (CTA2) tc::mbar_arrive_remote(tc::mapa_shared(&tempty[acc], 0));
+                    else tc::mbar_arrive(&tempty[acc]);
+                }
+                acc ^= 1;
+                if (acc == 0) aph ^= 1;
+                continue;
+            }
             // this staging buffer is free once the TMA store that last used it has read it
             if (etid == 0) {
                 if (p.ybufs == 2) tc::bulk_wait_read1();
@@ -847,14 +1012,39 @@ TileShape choose_tile(const std::vector<std::pair<int, int>> &ext, int N, int s,
     return best;
 }
 
+// tile shape for the fused-pool forward: BW a power of two <= 16 (window partners m^1, m^BW inside a
+// warp) and BH even (tiles start at even rows: no 2x2 window straddles a tile)
+TileShape choose_tile_pool(const std::vector<std::pair<int, int>> &ext, int N) {
+    TileShape best{2, 2, 1};
+    long best_tiles = -1;
+    for (int bw = 2; bw <= 16; bw *= 2)
+        for (int bh = 2; bw * bh <= 128; bh += 2) {
+            const int bn = std::min(128 / (bw * bh), N);
+            long tiles = 0;
+            for (auto &e : ext) tiles += (long)((N + bn - 1) / bn) * ((e.first + bh - 1) / bh) * ((e.second + bw - 1) / bw);
+            if (best_tiles < 0 || tiles < best_tiles || (tiles == best_tiles && bw > best.BW)) {
+                best_tiles = tiles;
+                best = {bw, bh, bn};
+            }
+        }
+    return best;
+}
+
 int round_up16(int x) { return (x + 15) / 16 * 16; }
 
 bool a_channels_ok(int cpad) { return cpad == 8 || cpad == 16 || cpad == 32 || cpad % 64 == 0; }
 
 // mode 0: forward (A = X at level m, out = level m+1); mode 1: dgrad (A = dY at level m+1, out = level m)
+// fused max-pool target of the forward pass (level layer+2 values + argmax bytes), or none
+struct PoolFuse {
+    void *y = nullptr;
+    uint8_t *a = nullptr;
+    const Level *Lp = nullptr;
+};
+
 splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const LayerGeom &g, const void *a_ptr,
                             const void *w_ptr, int w_rows, const float *bias, void *y, const void *relu_src, int relu,
-                            int p0, int p1, cudaStream_t st) {
+                            int p0, int p1, cudaStream_t st, const PoolFuse *pool = nullptr) {
     auto encode = get_encode();
     if (!encode) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
     const int kh = g.L.kh, kw = g.L.kw, s = mode == 0 ? g.L.sh : 1;
@@ -875,7 +1065,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         // halo mode for narrow outputs (per-tap TMA boxes cannot keep the MMA fed there)
         const int halo = (s == 1 && cpad % 64 == 0 && BN <= 128 && kw >= 2 && kw <= 4 && !getenv("SPLITCNN_NO_HALO")) ? 1 : 0;
         const int halo8 = (mode == 0 && cpad == 8 && s == 1 && kw <= 8 && kh * kw <= 16 && !getenv("SPLITCNN_NO_HALO")) ? 1 : 0;
-        TileShape ts = choose_tile(ext, N, s, a3d ? 32 : 128);
+        TileShape ts = pool ? choose_tile_pool(ext, N) : choose_tile(ext, N, s, a3d ? 32 : 128);
         if (halo8) {  // 8 output columns x BH output rows, one image per tile
             long best = -1;
             for (int bh = 1; bh <= 16; ++bh) {
@@ -885,7 +1075,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             }
         } else if (halo) {  // 8 output columns per M group; BH x BNn groups (<= 16)
             long best = -1;
-            for (int bh = 1; bh <= 16; ++bh)
+            for (int bh = pool ? 2 : 1; bh <= 16; bh += pool ? 2 : 1)   // fused pool: whole 2x2 windows per tile
                 for (int bn = 1; bh * bn <= 16 && bn <= N; ++bn) {
                     long t = 0;
                     for (auto &e : ext) t += (long)((N + bn - 1) / bn) * ((e.first + bh - 1) / bh) * ((e.second + 7) / 8);
@@ -981,6 +1171,12 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.y = (__nv_bfloat16 *)y;
         P.relu_src = (const __nv_bfloat16 *)relu_src;
         P.relu = relu;
+        if (pool) {
+            if (halo8 || P.direct || P.Cout != P.Cpo || P.Cout % 16 || (ts.BW & (ts.BW - 1)) || ts.BW > 16 || ts.BH % 2)
+                return fail(SPLITCNN_ERR_UNSUPPORTED, "conv_pool_fwd: geometry not fusable");
+            P.pool_y = (__nv_bfloat16 *)pool->y;
+            P.pool_a = pool->a;
+        }
         int tiles = 0, mboxes = 0;
         for (int q = g0; q < g1; ++q) {
             const int ql = q - g0;
@@ -988,6 +1184,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             const int oh = Lout.ph(i), ow = Lout.pw(j);
             P.out_h[ql] = oh; P.out_w[ql] = ow;
             P.out_off[ql] = Lout.offset(i, j);
+            if (pool) P.pool_off[ql] = pool->Lp->offset(i, j);
             const int pt = g.pad_h[2 * i], pl = g.pad_w[2 * j];
             P.pt[ql] = mode == 0 ? pt : kh - 1 - pt;
             P.pl[ql] = mode == 0 ? pl : kw - 1 - pl;
@@ -1021,7 +1218,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
                            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
             }
             if (r != CUDA_SUCCESS) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(A) failed");
-            if (!P.direct) {  // output (and ReLU-mask) maps over the output patch buffer
+            if (!P.direct && !pool) {  // output (and ReLU-mask) maps over the output patch buffer
                 const int yc = Lout.Cpad;
                 cuuint64_t ydims[4] = {(cuuint64_t)yc, (cuuint64_t)ow, (cuuint64_t)oh, (cuuint64_t)N};
                 cuuint64_t ystr[3] = {(cuuint64_t)yc * 2, (cuuint64_t)ow * yc * 2, (cuuint64_t)oh * ow * yc * 2};
@@ -1120,7 +1317,39 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             }
         };
         // kernels holding cta_group::2 instructions must be launched as clusters: separate instantiations
-        if (P.cta2) {
+        if (pool) {
+            const int key = 16 + (bias ? 1 : 0) + (P.cta2 ? 2 : 0);
+            auto launch_pool = [&](auto kern) {
+                static bool set[4] = {false};
+                if (!set[key - 16]) {
+                    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+                    set[key - 16] = true;
+                }
+                if (P.cta2) {
+                    cudaLaunchConfig_t cfg = {};
+                    cfg.gridDim = dim3((unsigned)grid);
+                    cfg.blockDim = dim3(CONV_THREADS);
+                    cfg.dynamicSmemBytes = smem;
+                    cfg.stream = st;
+                    cudaLaunchAttribute at[1];
+                    at[0].id = cudaLaunchAttributeClusterDimension;
+                    at[0].val.clusterDim.x = 2;
+                    at[0].val.clusterDim.y = 1;
+                    at[0].val.clusterDim.z = 1;
+                    cfg.attrs = at;
+                    cfg.numAttrs = 1;
+                    cudaLaunchKernelEx(&cfg, kern, P);
+                } else {
+                    kern<<<grid, CONV_THREADS, smem, st>>>(P);
+                }
+            };
+            switch (key) {
+                case 16: launch_pool(conv_tc_kernel<false, true, false, false, true>); break;
+                case 17: launch_pool(conv_tc_kernel<true, true, false, false, true>); break;
+                case 18: launch_pool(conv_tc_kernel<false, true, false, true, true>); break;
+                default: launch_pool(conv_tc_kernel<true, true, false, true, true>); break;
+            }
+        } else if (P.cta2) {
             switch (mode_bits) {
                 case 0: launch(conv_tc_kernel<false, false, false, true>); break;
                 case 1: launch(conv_tc_kernel<false, false, true, true>); break;
@@ -1209,6 +1438,16 @@ size_t conv_tc_ws_bytes(int mode, const Level &Li, const Level &Lo, const LayerG
 splitcnn_status_t launch_conv_fwd_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *w,
                                      const float *bias, void *y, int relu, int p0, int p1, cudaStream_t st) {
     return launch_tc(0, Li, Lo, g, x, w, g.L.cout, bias, y, nullptr, relu, p0, p1, st);
+}
+
+splitcnn_status_t launch_conv_pool_fwd_tc(const Level &Li, const Level &Lo, const Level &Lp, const LayerGeom &g,
+                                          const void *x, const void *w, const float *bias, void *y_pool, uint8_t *argmax,
+                                          int p0, int p1, cudaStream_t st) {
+    PoolFuse pf;
+    pf.y = y_pool;
+    pf.a = argmax;
+    pf.Lp = &Lp;
+    return launch_tc(0, Li, Lo, g, x, w, g.L.cout, bias, nullptr, nullptr, 1, p0, p1, st, &pf);
 }
 
 splitcnn_status_t launch_conv_dgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy, const void *w,

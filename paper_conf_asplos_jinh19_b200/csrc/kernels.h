@@ -28,6 +28,9 @@ bool conv_tc_supported(int mode, splitcnn_dtype_t dt, const Level &Li, const Lev
 size_t conv_tc_ws_bytes(int mode, const Level &Li, const Level &Lo, const LayerGeom &g);
 splitcnn_status_t launch_conv_fwd_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *w,
                                      const float *bias, void *y, int relu, int p0, int p1, cudaStream_t st);
+splitcnn_status_t launch_conv_pool_fwd_tc(const Level &Li, const Level &Lo, const Level &Lp, const LayerGeom &g,
+                                          const void *x, const void *w, const float *bias, void *y_pool, uint8_t *argmax,
+                                          int p0, int p1, cudaStream_t st);
 splitcnn_status_t launch_conv_dgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy, const void *w,
                                        void *dx, const void *relu_src, void *ws, int p0, int p1, cudaStream_t st);
 splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *dy,

@@ -33,13 +33,14 @@ class SplitNet:
     def __init__(self, region: list[dict], tail: list[dict], N: int, C: int, H: int, W: int,
                  split=(2, 2), mode: str = "even", omega: float = 0.2, seed: int = 0,
                  dtype: int = sc.BF16, device="cuda", patch_range=None, force_simt: bool = False,
-                 grad_buffer: torch.Tensor | None = None, input_relu: bool = False):
+                 grad_buffer: torch.Tensor | None = None, input_relu: bool = False, fuse_pool: bool = True):
         self.region_layers, self.tail_layers = region, tail
         self.N, self.C, self.H, self.W = N, C, H, W
         self.split, self.mode, self.omega, self.seed = split, mode, omega, seed
         self.dtype, self.tdtype, self.device = dtype, TORCH_DTYPE[dtype], torch.device(device)
         self.flags_extra = sc.FLAG_FORCE_SIMT if force_simt else 0
         self.input_relu = input_relu   # level 0 is a ReLU output (e.g. a tail fed by a ReLU conv)
+        self.fuse_pool = fuse_pool and dtype == sc.BF16 and not force_simt
         self.step_index = 0
         self.timers = None       # list -> every library call is bracketed by CUDA events (bench.py)
         self._label = ""
@@ -90,11 +91,28 @@ class SplitNet:
                     n += l["cout"] * l["kh"] * l["kw"] * plan.levels[m]["Cpad"] + l["cout"]
         return n
 
+    def _fusable(self, key: str, plan, layers, m: int) -> bool:
+        """conv m (+ReLU) and the 2x2/s2 max-pool m+1 run as ONE fused call (conv_pool_fwd)."""
+        return (self.fuse_pool and m + 1 < len(layers) and layers[m]["op"] == "conv" and layers[m].get("relu", True)
+                and layers[m + 1]["op"] == "maxpool"
+                and sc.splitcnn_conv_pool_supported(plan.handle, m, self.dtype))
+
     def _alloc(self, grad_buffer=None):
         dev, td = self.device, self.tdtype
-        self.act_r = [torch.zeros(self.region.level_elems(m), dtype=td, device=dev)
+        # the conv output of a fused conv -> pool pair is never materialised (the pool's argmax
+        # carries everything the backward pass needs): its level gets no buffer
+        self.fused = set()
+        for key, plan, layers in (("r", self.region, self.region_layers), ("t", self.tail, self.tail_layers)):
+            if plan is None:
+                continue
+            for m in range(len(layers)):
+                if self._fusable(key, plan, layers, m):
+                    self.fused.add((key, m))
+        skip_r = {m + 1 for k, m in self.fused if k == "r"}
+        skip_t = {m + 1 for k, m in self.fused if k == "t"}
+        self.act_r = [torch.zeros(0 if m in skip_r else self.region.level_elems(m), dtype=td, device=dev)
                       for m in range(self.region.nlayers + 1)]
-        self.act_t = ([torch.zeros(self.tail.level_elems(m), dtype=td, device=dev)
+        self.act_t = ([torch.zeros(0 if m in skip_t else self.tail.level_elems(m), dtype=td, device=dev)
                        for m in range(self.tail.nlayers + 1)] if self.tail else [])
         self.argmax = {}
         for plan, acts, key in ((self.region, self.act_r, "r"), (self.tail, self.act_t, "t")):
@@ -103,7 +121,8 @@ class SplitNet:
             for m, l in enumerate(plan.layers):
                 if l["op"] == "maxpool":
                     self.argmax[(key, m)] = torch.zeros(plan.level_elems(m + 1), dtype=torch.uint8, device=dev)
-        maxg = max([a.numel() for a in self.act_r + self.act_t])
+        maxg = max([self.region.level_elems(m) for m in range(self.region.nlayers + 1)] +
+                   ([self.tail.level_elems(m) for m in range(self.tail.nlayers + 1)] if self.tail else []))
         self.grad = [torch.zeros(maxg, dtype=td, device=dev), torch.zeros(maxg, dtype=td, device=dev)]
         ws = 0
         for plan in (self.region, self.tail):
@@ -212,9 +231,21 @@ class SplitNet:
         pass
 
     def _run_fwd(self, key, plan, layers, acts, p0, p1, stream):
+        skip = False
         for m, l in enumerate(layers):
+            if skip:          # the pool half of a fused pair
+                skip = False
+                continue
             self._label = l.get("name", f"{key}{m}")
             self.hook_before_fwd(key, m)
+            if (key, m) in self.fused:
+                W, b = self.params[(key, m)]
+                self._call("conv_fwd", self._conv_work(plan, m, l), sc.splitcnn_conv_pool_fwd, plan.handle, m,
+                           self.dtype, acts[m], W, b, acts[m + 2], self.argmax[(key, m + 1)],
+                           sc.FLAG_RELU | sc.FLAG_POOL_RELU_MASK | self.flags_extra, p0, p1, stream)
+                self.hook_after_fwd(key, m)
+                skip = True
+                continue
             if l["op"] == "conv":
                 W, b = self.params[(key, m)]
                 flags = (sc.FLAG_RELU if l.get("relu", True) else 0) | self.flags_extra

@@ -44,6 +44,7 @@ class OffloadSplitNet(SplitNet):
     """SplitNet whose split-region activations are offloaded / prefetched per Algorithm 1."""
 
     def __init__(self, *args, offload: bool = True, **kw):
+        kw.setdefault("fuse_pool", False)   # the planner walks the unfused op list (one op per layer)
         super().__init__(*args, **kw)
         self.offload_enabled = offload
         L = self.region.nlayers

@@ -298,3 +298,50 @@ def test_narrow_wgrad_opt_in_parity(sc, monkeypatch):
     sc.splitcnn_conv_bwd_filter(pl.handle, 0, dtype, x, dy, dw, None, 0.0, ws, ws_b)
     dWref, _ = O.conv_bwd_filter(O.split(X, lp.Ih, lp.Iw), O.split(G, lp.Oh, lp.Ow), lp)
     assert normwise(w_lib_to_oihw(_host(dw), 3), dWref) <= TOL[dtype]
+
+
+# (name, N, cin, cout, H, W, nh, nw): conv3x3 s1 p1 (+bias, ReLU) -> max-pool 2x2 s2, stochastic boundaries
+POOL_FUSE_CASES = [
+    ("c2_like", 4, 64, 64, 32, 32, 2, 2),          # halo path, 16x16 patches
+    ("ragged", 3, 64, 128, 36, 28, 3, 2),          # uneven patches (even extents by R2)
+    ("generic_bn256", 2, 128, 256, 24, 20, 2, 2),  # non-halo (BN > 128) tile chooser, 2-CTA
+    ("tail_like", 2, 256, 512, 28, 28, 1, 1),      # unsplit tail (1x1 split), Cout 512
+]
+
+
+@pytest.mark.parametrize("case", POOL_FUSE_CASES, ids=[c[0] for c in POOL_FUSE_CASES])
+def test_conv_pool_fused_matches_unfused_and_oracle(sc, case):
+    """f1: conv(+bias, ReLU) -> max-pool fused in the tcgen05 epilogue equals conv_fwd + pool_fwd BITWISE
+    (values and argmax bytes incl. the ReLU bit), and the oracle's pooled values within the bf16 bar."""
+    name, N, cin, cout, H, W, nh, nw = case
+    dtype = sc.BF16
+    layers = [synth.conv(cin, cout, 3, 1, 1, relu=True), synth.maxpool(cout)]
+    ref, pl = _make(sc, layers, N, cin, H, W, nh, nw, seed=sum(map(ord, name)))
+    assert sc.splitcnn_conv_pool_supported(pl.handle, 0, dtype)
+    lv0, lv1, lv2 = pl.levels
+    g = synth.rng(7 + len(name))
+    X = _round(synth.uniform(g, (N, cin, H, W)), dtype, sc)
+    Wt = _round(synth.kaiming(g, cout, cin, 3, 3), dtype, sc)
+    b = synth.uniform(g, (cout,), -0.1, 0.1).astype(np.float64)
+    x = _dev(sc, pack_level(X, lv0), dtype)
+    w = _dev(sc, w_oihw_to_lib(Wt, lv0["Cpad"]), dtype)
+    bias = torch.from_numpy(b.astype(np.float32)).cuda()
+    y1 = torch.zeros(lv1["total_elems"], dtype=torch.bfloat16, device="cuda")
+    yp = torch.full((lv2["total_elems"],), 7.0, dtype=torch.bfloat16, device="cuda")
+    ap = torch.full((lv2["total_elems"],), 0x55, dtype=torch.uint8, device="cuda")
+    sc.splitcnn_conv_fwd(pl.handle, 0, dtype, x, w, bias, y1, sc.FLAG_RELU)
+    sc.splitcnn_pool_fwd(pl.handle, 1, dtype, y1, yp, ap, sc.FLAG_POOL_RELU_MASK)
+    yf = torch.full_like(yp, -3.0)
+    af = torch.full_like(ap, 0xAA)
+    sc.splitcnn_conv_pool_fwd(pl.handle, 0, dtype, x, w, bias, yf, af)
+    torch.cuda.synchronize()
+    assert torch.equal(yf, yp), "fused pooled values differ from conv_fwd + pool_fwd"
+    assert torch.equal(af, ap), "fused argmax bytes differ from conv_fwd + pool_fwd"
+    # and the oracle: conv (fp64) -> bf16 rounding -> pool
+    lp0, lp1 = ref.layers
+    Y = O.conv_fwd(O.split(X, lp0.Ih, lp0.Iw), Wt, b, lp0, True)
+    Y = [[synth.to_bf16_f32(y.astype(np.float32)).astype(np.float64) for y in row] for row in Y]
+    P, _ = O.pool_fwd(Y, lp1)
+    got = unpack_level(_host(yf), lv2)
+    err = max(normwise(got[i][j], P[i][j]) for i in range(nh) for j in range(nw))
+    assert err <= TOL[dtype], err

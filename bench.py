@@ -86,7 +86,10 @@ def make_inputs(c, dtype_t, device, world=1, rank=0):
     import torch
     import synth
     g = synth.rng(c["seed"])
-    params = [p for p in synth.layer_params(g, c["layers"] + c["tail"]) if p is not None]
+    if c.get("resnet"):
+        params = synth.resnet_params(g, c["layers"], c["blocks"])
+    else:
+        params = [p for p in synth.layer_params(g, c["layers"] + c["tail"]) if p is not None]
     gen = torch.Generator(device="cpu").manual_seed(c["seed"])
     N = c["N"]
     x = (torch.rand((N, 3, c["H"], c["W"]), generator=gen) * 2 - 1).to(dtype_t)
@@ -111,7 +114,13 @@ def run_ours(args):
     c = workload(args.config)
     dtype = sc.BF16 if args.dtype == "bf16" else sc.FP32
     use_offload = args.offload if args.offload is not None else (args.config == "C4")
-    if world > 1:
+    if c.get("resnet"):
+        from paper_conf_asplos_jinh19_b200.resnet import ResSplitNet
+        if world > 1:
+            raise SystemExit("C3 runs on one GPU (the ResNet stack is not patch-sharded here)")
+        net = ResSplitNet(c["layers"], c["blocks"], c["N"], 3, c["H"], c["W"], split=c["split"], dtype=dtype)
+        use_offload = False
+    elif world > 1:
         from paper_conf_asplos_jinh19_b200.dist import DistSplitNet
         net = DistSplitNet(c, world, rank, dtype)
         use_offload = False
@@ -302,12 +311,17 @@ def oracle_sample_time(config: str, tiles: int):
     g = synth.rng(c["seed"])
     layers = c["layers"] + c["tail"]
     params = synth.layer_params(g, layers)
-    H = c["H"]
+    ops, h = [], c["H"]
+    for m, (l, prm) in enumerate(zip(layers, params)):
+        ops.append((l, prm, h))
+        for b in c.get("blocks", ()):      # ResNet: the 1x1 downsample reads the block input
+            if b["a"] == m and b["ds"] is not None:
+                ops.append((b["ds"], synth.layer_params(g, [b["ds"]])[0], h))
+        h = OP.out_len(h, l["kh"], l["sh"], l["ph_b"], l["ph_e"])
     total = 0.0
     sample_px = 0
-    h = H
     first_conv = True
-    for l, prm in zip(layers, params):
+    for l, prm, h in ops:
         ho = OP.out_len(h, l["kh"], l["sh"], l["ph_b"], l["ph_e"])
         # a tile = a patch of an 8x8 even split of this layer's output (>= 1 px)
         n = min(8, ho)
@@ -336,7 +350,6 @@ def oracle_sample_time(config: str, tiles: int):
         total += t_layer * (ho * ho) / px_s
         first_conv = first_conv and l["op"] != "conv"
         sample_px += px_s
-        h = ho
     return total, f"1 image, {tiles} of 64 output tiles per layer-op (fwd+dgrad+wgrad / pool fwd+bwd), scaled by output pixels"
 
 
@@ -379,7 +392,7 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="C5", choices=["C2", "C4", "C5"])
+    ap.add_argument("--config", default="C5", choices=["C2", "C3", "C4", "C5"])
     ap.add_argument("--dtype", default="bf16", choices=["bf16", "fp32"])
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--cpu-tiles", type=int, default=12)

@@ -243,6 +243,20 @@ SPLITCNN_API splitcnn_status_t splitcnn_pool_bwd(splitcnn_plan_t plan, int32_t l
                                     const void *dy, const uint8_t *argmax, void *dx, uint32_t flags,
                                     int32_t p0, int32_t p1, splitcnn_stream_t stream);
 
+/* ------------------------------------------------------------------ residual add */
+/* Pointwise add on the patch buffers of one level (ResNet residual join; the add is split-
+ * invariant, so a shortcut and its sibling branch share the level's I and O).  Acts on
+ * the contiguous element span of patches [p0, p1) of `level` (patches of a level are stored back
+ * to back).  a, b, y, mask: level buffers (same layout); y may alias a or b.
+ *   mask == NULL: y = a + b, then max(., 0) with FLAG_RELU            (forward join)
+ *   mask != NULL: y = (a + b) * [mask > 0]                          (backward: sum of a fork's
+ *                 two gradient contributions times the ReLU mask of the block output mask)
+ * Arithmetic in fp32, one rounding to the storage type.  Errors: null a/b/y, misalignment,
+ * FLAG_RELU together with a mask. */
+SPLITCNN_API splitcnn_status_t splitcnn_add(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                const void *a, const void *b, void *y, const void *mask, uint32_t flags,
+                                int32_t p0, int32_t p1, splitcnn_stream_t stream);
+
 /* ------------------------------------------------------------------ offload / prefetch */
 /* Patch-granular activation offload (HMMS): after `ready` (recorded by the caller
  * on the compute stream after the buffer's last write, moment 1) copy patch `patch` of level

@@ -182,6 +182,13 @@ def pool_bwd(dYp, Ap, lp: LayerPlan):
              for j in C] for i in R]
 
 
+def residual_add(Ap, Bp, relu=False):
+    """Residual join of a ResNet basic block, per patch: Y_p = A_p + B_p (then ReLU).  The add is
+    pointwise, so the shortcut shares its sibling's split scheme (summation)."""
+    out = [[Ap[i][j] + Bp[i][j] for j in range(len(row))] for i, row in enumerate(Ap)]
+    return [[np.maximum(y, 0.0) for y in row] for row in out] if relu else out
+
+
 def relu_mask(dXp, Mp):
     """ReLU backward: keep the gradient where the ReLU output is > 0."""
     return [[np.where(Mp[i][j] > 0, dXp[i][j], 0.0) for j in range(len(row))]

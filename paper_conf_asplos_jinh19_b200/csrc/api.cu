@@ -291,6 +291,30 @@ extern "C" splitcnn_status_t splitcnn_pool_bwd(splitcnn_plan_t plan, int32_t lay
     return check_launch("pool_bwd");
 }
 
+// ------------------------------------------------------------------ residual add
+extern "C" splitcnn_status_t splitcnn_add(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype, const void *a,
+                                          const void *b, void *y, const void *mask, uint32_t flags, int32_t p0,
+                                          int32_t p1, splitcnn_stream_t stream) {
+    if (!plan || level < 0 || level >= (int)plan->levels.size()) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad level");
+    TRY(check_dtype(dtype));
+    if (!a || !b || !y) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    if (mask && (flags & SPLITCNN_FLAG_RELU)) return fail(SPLITCNN_ERR_INVALID_VALUE, "FLAG_RELU with a mask");
+    NEED_ALIGNED(a, "a");
+    NEED_ALIGNED(b, "b");
+    NEED_ALIGNED(y, "y");
+    NEED_ALIGNED(mask, "mask");
+    TRY(check_range(plan, level, p0, p1));
+    if (p1 == p0) return SPLITCNN_OK;
+    const Level &L = plan->levels[level];
+    auto off = [&](int p) { return p == L.npatch() ? L.total() : L.offset(p / L.nw(), p % L.nw()); };
+    const int64_t o0 = off(p0), n = off(p1) - o0;
+    const size_t es = dtype == SPLITCNN_BF16 ? 2 : 4;
+    auto at = [&](const void *p) { return p ? (const void *)((const char *)p + o0 * es) : nullptr; };
+    launch_add(dtype, at(a), at(b), (void *)at(y), at(mask), (flags & SPLITCNN_FLAG_RELU) ? 1 : 0, n,
+               (cudaStream_t)stream);
+    return check_launch("add");
+}
+
 // ------------------------------------------------------------------ offload / prefetch
 extern "C" splitcnn_status_t splitcnn_patch_bytes(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
                                                   int32_t patch, size_t *offset, size_t *bytes) {

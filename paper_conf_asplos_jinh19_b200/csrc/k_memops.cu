@@ -289,6 +289,51 @@ void launch_pool_bwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, con
                                              (const T *)dy, a, (T *)dx, p0, relu_bit); count_launch(); }
 }
 
+// ============================================================ residual add (ResNet blocks)
+// Pointwise over the contiguous element range of patches [p0, p1) of one level (patch buffers of
+// a level are laid out back to back, so the range is one flat span):
+//   forward   y = a + b            (RELU: y = max(a + b, 0))
+//   backward  y = (a + b) * [m > 0] (m = the block's ReLU output; sums the two gradient
+//                                    contributions of a fork and applies its ReLU mask once)
+// One thread = 8 elements (16 B of bf16); y may alias a or b (each element is read, then written,
+// by the same thread).  fp32 sum, one rounding to T.
+template <typename T, bool RELU, bool MASK>
+__global__ void __launch_bounds__(256) add_kernel(const T *a, const T *b, T *y, const T *__restrict__ m, int64_t n8) {
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n8; u += (int64_t)gridDim.x * blockDim.x) {
+        float va[8], vb[8], vm[8];
+        load8(a + u * 8, va);
+        load8(b + u * 8, vb);
+        if (MASK) load8(m + u * 8, vm);
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            float s = va[k] + vb[k];
+            if (RELU) s = fmaxf(s, 0.f);
+            if (MASK) s = vm[k] > 0.f ? s : 0.f;
+            va[k] = s;
+        }
+        store8(y + u * 8, va);
+    }
+}
+
+template <typename T>
+void launch_add_t(const void *a, const void *b, void *y, const void *m, int relu, int64_t n, cudaStream_t st) {
+    const int64_t n8 = n / 8;
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n8 + 255) / 256, 148 * 8));
+    if (m)
+        add_kernel<T, false, true><<<grid, 256, 0, st>>>((const T *)a, (const T *)b, (T *)y, (const T *)m, n8);
+    else if (relu)
+        add_kernel<T, true, false><<<grid, 256, 0, st>>>((const T *)a, (const T *)b, (T *)y, nullptr, n8);
+    else
+        add_kernel<T, false, false><<<grid, 256, 0, st>>>((const T *)a, (const T *)b, (T *)y, nullptr, n8);
+    count_launch();
+}
+
+void launch_add(splitcnn_dtype_t dt, const void *a, const void *b, void *y, const void *m, int relu, int64_t n,
+                cudaStream_t st) {
+    if (dt == SPLITCNN_BF16) launch_add_t<__nv_bfloat16>(a, b, y, m, relu, n, st);
+    else launch_add_t<float>(a, b, y, m, relu, n, st);
+}
+
 void launch_pool_fwd(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, void *y,
                      uint8_t *a, int relu_bit, int p0, int p1, cudaStream_t st) {
     if (dt == SPLITCNN_BF16) launch_pool_fwd_t<__nv_bfloat16>(Li, Lo, g, x, y, a, relu_bit, p0, p1, st);

@@ -13,6 +13,8 @@ void launch_pool_fwd(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, cons
                      uint8_t *a, int relu_bit, int p0, int p1, cudaStream_t st);
 void launch_pool_bwd(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy,
                      const uint8_t *a, void *dx, int relu_bit, int p0, int p1, cudaStream_t st);
+void launch_add(splitcnn_dtype_t dt, const void *a, const void *b, void *y, const void *m, int relu, int64_t n,
+                cudaStream_t st);
 
 // k_conv_simt.cu
 void launch_conv_fwd_simt(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *x,

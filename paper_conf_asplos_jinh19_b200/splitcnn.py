@@ -35,7 +35,7 @@ EXPORTED = [
     "splitcnn_plan_layer", "splitcnn_workspace_size",
     "splitcnn_split", "splitcnn_merge",
     "splitcnn_conv_fwd", "splitcnn_conv_bwd_data", "splitcnn_conv_bwd_filter",
-    "splitcnn_pool_fwd", "splitcnn_pool_bwd", "splitcnn_conv_pool_fwd", "splitcnn_conv_pool_supported",
+    "splitcnn_pool_fwd", "splitcnn_pool_bwd", "splitcnn_conv_pool_fwd", "splitcnn_conv_pool_supported", "splitcnn_add",
     "splitcnn_offload", "splitcnn_prefetch", "splitcnn_patch_bytes",
     "splitcnn_offload_plan", "splitcnn_prefetch_plan",
 ]
@@ -90,6 +90,7 @@ _sig("splitcnn_conv_bwd_filter", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _
 _sig("splitcnn_pool_fwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
 _sig("splitcnn_pool_bwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
 _sig("splitcnn_conv_pool_fwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
+_sig("splitcnn_add", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
 _sig("splitcnn_conv_pool_supported", [_vp, _i32, ctypes.c_int, _pi32])
 _sig("splitcnn_offload", [_vp, _i32, ctypes.c_int, _i32, _vp, _vp, _vp, _vp, _vp])
 _sig("splitcnn_prefetch", [_vp, _i32, ctypes.c_int, _i32, _vp, _vp, _vp, _vp, _vp])
@@ -257,6 +258,11 @@ def splitcnn_pool_fwd(plan, layer, dtype, x, y, argmax, flags=0, p0=0, p1=-1, st
 def splitcnn_pool_bwd(plan, layer, dtype, dy, argmax, dx, flags=0, p0=0, p1=-1, stream=None):
     _check(_lib.splitcnn_pool_bwd(plan, layer, dtype, _ptr(dy), _ptr(argmax), _ptr(dx), flags, p0, p1,
                                   _stream(stream)))
+
+
+def splitcnn_add(plan, level, dtype, a, b, y, mask=None, flags=0, p0=0, p1=-1, stream=None):
+    _check(_lib.splitcnn_add(plan, level, dtype, _ptr(a), _ptr(b), _ptr(y), _ptr(mask), flags, p0, p1,
+                             _stream(stream)))
 
 
 def splitcnn_conv_pool_fwd(plan, layer, dtype, x, w, bias, y_pool, argmax, flags=FLAG_RELU | FLAG_POOL_RELU_MASK,

@@ -50,6 +50,25 @@ def resnet18_split_stack():
     return L
 
 
+def resnet18_blocks(w1: int = 64, w2: int = 128):
+    """The same stack as ``resnet18_split_stack`` with its residual structure (BN-free; P:203
+    residual adds): ``chain`` is the main branch as one layer chain (every block's second conv has
+    no ReLU of its own -- the ReLU follows the add), ``blocks`` lists per basic block the chain
+    index of its first conv and its shortcut (None = identity, else the 1x1 s2 downsample conv)."""
+    L = [conv(3, w1, k=7, s=2, p=3, name="conv1"), maxpool(w1, k=3, s=2, p=1, name="maxpool")]
+    blocks = []
+    c = w1
+    for stage, (w, s0) in enumerate(((w1, 1), (w2, 2)), start=1):
+        for b in range(2):
+            s = s0 if b == 0 else 1
+            ds = conv(c, w, k=1, s=s, p=0, relu=False, name=f"layer{stage}_{b}_ds") if (s != 1 or c != w) else None
+            blocks.append(dict(a=len(L), ds=ds))
+            L.append(conv(c, w, s=s, name=f"layer{stage}_{b}_a"))
+            L.append(conv(w, w, relu=False, name=f"layer{stage}_{b}_b"))
+            c = w
+    return L, blocks
+
+
 def split_region(layers, depth_convs: int, include_next_pool: bool):
     """First ``depth_convs`` convolutions (plus interleaved pools, plus the pool right
     after the last split conv when ``include_next_pool``) -> (region, tail)."""
@@ -73,6 +92,8 @@ CONFIGS = {
     "C2": dict(name="C2", desc="VGG-19 conv stack, CIFAR-shaped 32x32, N=128, 2x2 split, depth 50%",
                N=128, H=32, W=32, split=(2, 2), mode="even", depth=8, pool_inside=True,
                dtype="bf16", seed=1),
+    "C3": dict(name="C3", desc="ResNet-18 224x224 (BN-free split stack conv1..layer2), N=256, 2x2 split",
+               N=256, H=224, W=224, split=(2, 2), mode="even", dtype="bf16", seed=2, resnet=True),
     "C4": dict(name="C4", desc="VGG-19 224x224, N=512, stochastic 4x4 split at depth 75%, offload",
                N=512, H=224, W=224, split=(4, 4), mode="random", omega=0.2, depth=12,
                pool_inside=False, dtype="bf16", seed=3),
@@ -85,6 +106,12 @@ CONFIGS = {
 def vgg_config(name: str, N: int | None = None):
     """Region/tail layer lists of a VGG config, optionally at a reduced batch ``N``."""
     c = dict(CONFIGS[name])
+    if c.get("resnet"):
+        c["layers"], c["blocks"] = resnet18_blocks()
+        c["tail"], c["C"] = [], 3
+        if N is not None:
+            c["N"] = N
+        return c
     region, tail = split_region(vgg19_layers(), c["depth"], c["pool_inside"])
     c["layers"], c["tail"] = region, tail
     c["C"] = 3
@@ -118,6 +145,13 @@ def to_bf16_f32(a: np.ndarray) -> np.ndarray:
     u = a.view(np.uint32).astype(np.uint64)
     r = ((u + 0x7FFF + ((u >> 16) & 1)) >> 16) << 16
     return r.astype(np.uint32).view(np.float32)
+
+
+def resnet_params(g: np.random.Generator, chain, blocks, dtype=np.float32):
+    """(W, b) per conv of the chain in order, then per downsample conv in block order."""
+    ps = [p for p in layer_params(g, chain, dtype) if p is not None]
+    ps += [p for p in layer_params(g, [b["ds"] for b in blocks if b["ds"] is not None], dtype)]
+    return ps
 
 
 def layer_params(g: np.random.Generator, layers, dtype=np.float32):

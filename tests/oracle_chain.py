@@ -97,3 +97,93 @@ def _out(layers, L, dim):
         pb, pe = (l["ph_b"], l["ph_e"]) if dim == 0 else (l["pw_b"], l["pw_e"])
         L = (L + pb + pe - k) // s + 1
     return L
+
+
+def run_resnet(chain, blocks, N, C, H, W, Oh, Ow, params, X, G, round_bf16=False):
+    """Oracle composition of the BN-free ResNet split stack (synth.resnet18_blocks): the main
+    chain with a residual join after every block's second conv, the 1x1 downsample on its own
+    one-layer plan sharing the block's output partition.  G is the gradient of the merged output.
+    Returns (output NCHW, dWs, dbs) with dWs/dbs in synth.resnet_params order (chain convs, then
+    downsample convs)."""
+    rp = OP.plan(chain, N, C, H, W, Oh, Ow)
+    nconv = sum(1 for l in chain if l["op"] == "conv")
+    pit = iter(params)
+    prm = {m: next(pit) for m, l in enumerate(chain) if l["op"] == "conv"}
+    ds = {}
+    for k, b in enumerate(blocks):
+        if b["ds"] is not None:
+            lo = rp.layers[b["a"] + 1]
+            li = rp.layers[b["a"]]
+            dp = OP.plan([b["ds"]], N, b["ds"]["cin"], li.H_in, li.W_in, lo.Oh, lo.Ow).layers[0]
+            assert dp.Ih == li.Ih and dp.Iw == li.Iw
+            ds[k] = (dp, next(pit))
+    at = {b["a"]: k for k, b in enumerate(blocks)}
+    block_out = {b["a"] + 2 for b in blocks}
+    rnd = lambda P: _rnd(P, round_bf16)
+    # forward
+    acts = [rnd(O.split(X, rp.layers[0].Ih, rp.layers[0].Iw))]
+    args, sc_out = {}, {}
+    m = 0
+    while m < len(chain):
+        l, lp = chain[m], rp.layers[m]
+        if m in at:
+            k = at[m]
+            Wa, ba = prm[m]
+            Wb, bb = prm[m + 1]
+            h = rnd(O.conv_fwd(acts[m], Wa, ba, lp, True))
+            z = rnd(O.conv_fwd(h, Wb, bb, rp.layers[m + 1], False))
+            if k in ds:
+                dp, (Wd, bd) = ds[k]
+                s = sc_out[k] = rnd(O.conv_fwd(acts[m], Wd, bd, dp, False))
+            else:
+                s = acts[m]
+            acts += [h, rnd(O.residual_add(z, s, relu=True))]
+            m += 2
+            continue
+        if l["op"] == "conv":
+            Wt, b = prm[m]
+            acts.append(rnd(O.conv_fwd(acts[m], Wt, b, lp, l.get("relu", True))))
+        else:
+            P, args[m] = O.pool_fwd(acts[m], lp)
+            acts.append(rnd(P))
+        m += 1
+    out = O.merge(acts[-1])
+    # backward
+    grads, gds = {}, {}
+    g = rnd(O.relu_mask(O.split(G, rp.layers[-1].Oh, rp.layers[-1].Ow), acts[-1]))
+    m = len(chain) - 1
+    while m >= 0:
+        a = m - 1
+        if a in at:
+            k = at[a]
+            Wa, _ = prm[a]
+            Wb, _ = prm[a + 1]
+            grads[a + 1] = O.conv_bwd_filter(acts[a + 1], g, rp.layers[a + 1])
+            gh = rnd(O.conv_bwd_data(g, Wb, rp.layers[a + 1], acts[a + 1]))
+            grads[a] = O.conv_bwd_filter(acts[a], gh, rp.layers[a])
+            gx = rnd(O.conv_bwd_data(gh, Wa, rp.layers[a]))
+            if k in ds:
+                dp, (Wd, _) = ds[k]
+                gds[k] = O.conv_bwd_filter(acts[a], g, dp)
+                gs = rnd(O.conv_bwd_data(g, Wd, dp))
+            else:
+                gs = g
+            gsum = O.residual_add(gx, gs)
+            g = rnd(O.relu_mask(gsum, acts[a]) if a in block_out else gsum)
+            m = a - 1
+            continue
+        l, lp = chain[m], rp.layers[m]
+        if l["op"] == "conv":
+            grads[m] = O.conv_bwd_filter(acts[m], g, lp)
+            if m > 0:
+                g = rnd(O.conv_bwd_data(g, prm[m][0], lp, acts[m] if _masked(chain, m, False) else None))
+        else:
+            g = O.pool_bwd(g, args[m], lp)
+            if _masked(chain, m, False):
+                g = O.relu_mask(g, acts[m])
+            g = rnd(g)
+        m -= 1
+    dWs = [grads[m][0] for m in sorted(grads)] + [gds[k][0] for k in sorted(gds)]
+    dbs = [grads[m][1] for m in sorted(grads)] + [gds[k][1] for k in sorted(gds)]
+    assert len(dWs) == nconv + len(ds)
+    return out, dWs, dbs

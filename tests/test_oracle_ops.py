@@ -245,3 +245,85 @@ def test_split_merge_identity_pin8():
         assert np.array_equal(O.merge(O.split(X, Ih, Iw)), X)
     assert np.array_equal(O.offload_roundtrip(X), X)
     assert np.array_equal(O.allreduce_sum([X, 2 * X]), 3 * X)
+
+
+# --------------------------------------------------------------------------- ResNet split stack
+def _torch_resnet(chain, blocks, X, params):
+    """Unsplit BN-free ResNet stack in torch fp64 (library routines), for the 1x1-split pin."""
+    import torch
+    import torch.nn.functional as F
+    x = torch.tensor(X, requires_grad=True)
+    ps = [(torch.tensor(W, requires_grad=True), torch.tensor(b, requires_grad=True)) for W, b in params]
+    nconv = sum(1 for l in chain if l["op"] == "conv")
+    cidx = {m: i for i, m in enumerate(m for m, l in enumerate(chain) if l["op"] == "conv")}
+    dsi = {k: nconv + i for i, k in enumerate(k for k, b in enumerate(blocks) if b["ds"] is not None)}
+    at = {b["a"]: k for k, b in enumerate(blocks)}
+
+    def conv(h, l, p):
+        return F.conv2d(h, p[0], p[1], stride=l["sh"], padding=l["ph_b"])
+
+    h, m = x, 0
+    while m < len(chain):
+        l = chain[m]
+        if m in at:
+            k = at[m]
+            t = F.relu(conv(h, l, ps[cidx[m]]))
+            z = conv(t, chain[m + 1], ps[cidx[m + 1]])
+            s = conv(h, blocks[k]["ds"], ps[dsi[k]]) if k in dsi else h
+            h = F.relu(z + s)
+            m += 2
+            continue
+        if l["op"] == "conv":
+            h = conv(h, l, ps[cidx[m]])
+            if l.get("relu", True):
+                h = F.relu(h)
+        else:
+            h = F.max_pool2d(h, l["kh"], l["sh"], l["ph_b"])
+        m += 1
+    return h, x, ps
+
+
+def test_resnet_stack_1x1_split_equals_unsplit_torch():
+    """pin-1 for the ResNet composition (residual joins, 1x1 s2 downsample, 3x3 s2 p1 pool):
+    a 1x1 split reduces to the unsplit network; forward and all weight gradients vs torch fp64
+    autograd (loss = <Y, G>)."""
+    import torch
+    from tests import oracle_chain
+    chain, blocks = synth.resnet18_blocks(8, 16)
+    g = synth.rng(7)
+    N, H = 2, 32
+    X = synth.uniform(g, (N, 3, H, H)).astype(np.float64)
+    params = [(W.astype(np.float64), b.astype(np.float64)) for W, b in synth.resnet_params(g, chain, blocks)]
+    Y, x, ps = _torch_resnet(chain, blocks, X, params)
+    G = synth.normal(g, tuple(Y.shape)).astype(np.float64)
+    (Y * torch.tensor(G)).sum().backward()
+    out, dWs, dbs = oracle_chain.run_resnet(chain, blocks, N, 3, H, H, [0, Y.shape[2]], [0, Y.shape[3]],
+                                            params, X, G)
+    assert np.abs(out - Y.detach().numpy()).max() < 1e-12
+    assert len(dWs) == len(ps)
+    for (Wt, bt), dW, db in zip(ps, dWs, dbs):
+        assert np.abs(dW - Wt.grad.numpy()).max() < 1e-10 * max(1.0, np.abs(dW).max())
+        assert np.abs(db - bt.grad.numpy()).max() < 1e-10 * max(1.0, np.abs(db).max())
+
+
+def test_resnet_stack_split_patch_independence_and_interior():
+    """The 2x2-split ResNet stack keeps patches independent: perturbing the input of one
+    patch leaves every other patch's output bitwise unchanged, and the split output differs from
+    the unsplit one (Split-CNN changes the result)."""
+    from tests import oracle_chain
+    chain, blocks = synth.resnet18_blocks(8, 16)
+    g = synth.rng(8)
+    N, H = 1, 32
+    X = synth.uniform(g, (N, 3, H, H)).astype(np.float64)
+    params = [(W.astype(np.float64), b.astype(np.float64)) for W, b in synth.resnet_params(g, chain, blocks)]
+    G = np.zeros((N, 16, 4, 4))
+    O2 = [0, 2, 4]
+    out, _, _ = oracle_chain.run_resnet(chain, blocks, N, 3, H, H, O2, O2, params, X, G)
+    X2 = X.copy()
+    X2[:, :, :16, :16] += 0.5          # patch (0, 0) at the input (I = 8 * O at the input level)
+    out2, _, _ = oracle_chain.run_resnet(chain, blocks, N, 3, H, H, O2, O2, params, X2, G)
+    assert not np.array_equal(out[:, :, :2, :2], out2[:, :, :2, :2])
+    assert np.array_equal(out[:, :, 2:, :], out2[:, :, 2:, :])
+    assert np.array_equal(out[:, :, :, 2:], out2[:, :, :, 2:])
+    full, _, _ = oracle_chain.run_resnet(chain, blocks, N, 3, H, H, [0, 4], [0, 4], params, X, G)
+    assert not np.allclose(full, out)

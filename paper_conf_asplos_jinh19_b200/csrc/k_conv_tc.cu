@@ -929,16 +929,37 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
 
 // dgrad weights: W'[ci][r'][c'][co] = W[co][kh-1-r'][kw-1-c'][ci], zero for co >= Cout
 __global__ void flip_weights_kernel(const __nv_bfloat16 *__restrict__ W, __nv_bfloat16 *__restrict__ Wt, int Cout,
-                                    int Cpad_in, int Cin, int kh, int kw, int Cpad_out) {
-    const int64_t n = (int64_t)Cin * kh * kw * Cpad_out;
+                                    int Cpad_in, int Cin, int kh, int kw, int Cpad_out, int r0h, int r0w, int step,
+                                    int nth, int ntw) {
+    // Wt[ci][j][l][co] = W[co][r0h + step*(nth-1-j)][r0w + step*(ntw-1-l)][ci]   (stride-1 dgrad: r0 = 0,
+    // step = 1, nt = k -- the 180-degree flip; stride-s phase (rho_h, rho_w): the taps r = r0 (mod s))
+    const int64_t n = (int64_t)Cin * nth * ntw * Cpad_out;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const int co = (int)(i % Cpad_out);
         int64_t t = i / Cpad_out;
-        const int c = (int)(t % kw);
-        t /= kw;
-        const int r = (int)(t % kh);
-        const int ci = (int)(t / kh);
-        Wt[i] = co < Cout ? W[(((int64_t)co * kh + (kh - 1 - r)) * kw + (kw - 1 - c)) * Cpad_in + ci] : __float2bfloat16(0.f);
+        const int c = (int)(t % ntw);
+        t /= ntw;
+        const int r = (int)(t % nth);
+        const int ci = (int)(t / nth);
+        const int rr = r0h + step * (nth - 1 - r), cc = r0w + step * (ntw - 1 - c);
+        Wt[i] = co < Cout ? W[(((int64_t)co * kh + rr) * kw + cc) * Cpad_in + ci] : __float2bfloat16(0.f);
+    }
+}
+
+// Stride-s dgrad, zero phases: dX elements of phase (rh, rw) that no tap reaches (k < s) are zero.
+__global__ void zero_phase_kernel(__nv_bfloat16 *__restrict__ dx, LevelDesc L, int S, int rh, int rw, int p0) {
+    const PatchGeo g = patch_geo(L, p0 + blockIdx.y);
+    const int hq = (g.hp - rh + S - 1) / S, wq = (g.wp - rw + S - 1) / S, G = L.Cpad / 8;
+    const int64_t units = (int64_t)L.N * hq * wq * G;
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < units; u += (int64_t)gridDim.x * blockDim.x) {
+        const int cg = (int)(u % G);
+        int64_t t = u / G;
+        const int w = (int)(t % wq);
+        t /= wq;
+        const int h = (int)(t % hq);
+        const int n = (int)(t / hq);
+        *reinterpret_cast<uint4 *>(dx + g.off + (((int64_t)n * g.hp + h * S + rh) * g.wp + w * S + rw) * L.Cpad + cg * 8) =
+            make_uint4(0, 0, 0, 0);
     }
 }
 
@@ -1036,6 +1057,13 @@ bool a_channels_ok(int cpad) { return cpad == 8 || cpad == 16 || cpad == 32 || c
 
 // mode 0: forward (A = X at level m, out = level m+1); mode 1: dgrad (A = dY at level m+1, out = level m)
 // fused max-pool target of the forward pass (level layer+2 values + argmax bytes), or none
+// Stride-S data gradient by output phase: dX[S*t + rho] = sum over the taps r = r0 (mod S) -- a
+// stride-1 correlation of dY with the (kh' x kw') sub-filter, written through a tensor map that
+// views the dX patch at element stride S from (rho_h, rho_w).
+struct Phase {
+    int S, rh, rw, kh, kw, pt, pl;
+};
+
 struct PoolFuse {
     void *y = nullptr;
     uint8_t *a = nullptr;
@@ -1044,10 +1072,13 @@ struct PoolFuse {
 
 splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const LayerGeom &g, const void *a_ptr,
                             const void *w_ptr, int w_rows, const float *bias, void *y, const void *relu_src, int relu,
-                            int p0, int p1, cudaStream_t st, const PoolFuse *pool = nullptr) {
+                            int p0, int p1, cudaStream_t st, const PoolFuse *pool = nullptr, const Phase *ph = nullptr) {
     auto encode = get_encode();
     if (!encode) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
-    const int kh = g.L.kh, kw = g.L.kw, s = mode == 0 ? g.L.sh : 1;
+    const int kh = ph ? ph->kh : g.L.kh, kw = ph ? ph->kw : g.L.kw, s = mode == 0 ? g.L.sh : 1;
+    const int PS = ph ? ph->S : 1, prh = ph ? ph->rh : 0, prw = ph ? ph->rw : 0;
+    auto out_ext_h = [&](int i) { return (Lout.ph(i) - prh + PS - 1) / PS; };
+    auto out_ext_w = [&](int j) { return (Lout.pw(j) - prw + PS - 1) / PS; };
     const int cpad = La.Cpad;
     const int cpadc = std::min(cpad, 64);
     const int ncols_out = mode == 0 ? g.L.cout : g.L.cin;
@@ -1059,7 +1090,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         std::vector<std::pair<int, int>> ext;
         for (int q = g0; q < g1; ++q) {
             const int i = q / Lout.nw(), j = q % Lout.nw();
-            ext.push_back({Lout.ph(i), Lout.pw(j)});
+            ext.push_back({out_ext_h(i), out_ext_w(j)});
         }
         const int a3d = (cpad == 8 && s == 1) ? 1 : 0;  // TMA rows of 16 B are slow: merge 8 pixels per row
         // halo mode for narrow outputs (per-tap TMA boxes cannot keep the MMA fed there)
@@ -1163,6 +1194,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.ybufs = (!P.direct && P.ybuf_bytes <= 32u * 1024u) ? 2 : 1;
         if (P.bres && P.bres_bytes + 2u * P.ybuf_bytes + 2u * P.a_stage > 206u * 1024u) P.ybufs = 1;
         P.egroups = (P.ybufs == 2 && !getenv("SPLITCNN_ONE_EPI")) ? 2 : 1;
+        if (ph && P.direct) return fail(SPLITCNN_ERR_UNSUPPORTED, "phase dgrad needs a TMA-store output");
         const uint32_t staging = P.ybufs * P.ybuf_bytes;
         P.stages = std::min<int>(8, (int)((210u * 1024u - staging - P.bres_bytes) / stage_bytes));
         P.bres_off = (uint32_t)P.stages * stage_bytes;
@@ -1185,13 +1217,13 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         for (int q = g0; q < g1; ++q) {
             const int ql = q - g0;
             const int i = q / Lout.nw(), j = q % Lout.nw();
-            const int oh = Lout.ph(i), ow = Lout.pw(j);
+            const int oh = out_ext_h(i), ow = out_ext_w(j);
             P.out_h[ql] = oh; P.out_w[ql] = ow;
             P.out_off[ql] = Lout.offset(i, j);
             if (pool) P.pool_off[ql] = pool->Lp->offset(i, j);
             const int pt = g.pad_h[2 * i], pl = g.pad_w[2 * j];
-            P.pt[ql] = mode == 0 ? pt : kh - 1 - pt;
-            P.pl[ql] = mode == 0 ? pl : kw - 1 - pl;
+            P.pt[ql] = ph ? ph->pt : mode == 0 ? pt : kh - 1 - pt;
+            P.pl[ql] = ph ? ph->pl : mode == 0 ? pl : kw - 1 - pl;
             P.nhb[ql] = (oh + ts.BH - 1) / ts.BH;
             P.nwb[ql] = (ow + ts.BW - 1) / ts.BW;
             P.tile_prefix[ql] = tiles;
@@ -1224,17 +1256,20 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             if (r != CUDA_SUCCESS) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(A) failed");
             if (!P.direct && !pool) {  // output (and ReLU-mask) maps over the output patch buffer
                 const int yc = Lout.Cpad;
+                // phase view (S > 1): pixel (h, w) of the view is pixel (S*h + rho_h, S*w + rho_w) of the patch
+                const int fh = Lout.ph(i), fw = Lout.pw(j);
                 cuuint64_t ydims[4] = {(cuuint64_t)yc, (cuuint64_t)ow, (cuuint64_t)oh, (cuuint64_t)N};
-                cuuint64_t ystr[3] = {(cuuint64_t)yc * 2, (cuuint64_t)ow * yc * 2, (cuuint64_t)oh * ow * yc * 2};
+                cuuint64_t ystr[3] = {(cuuint64_t)yc * 2 * PS, (cuuint64_t)fw * yc * 2 * PS, (cuuint64_t)fh * fw * yc * 2};
                 cuuint32_t ybox[4] = {(cuuint32_t)P.ychunk, (cuuint32_t)ts.BW, (cuuint32_t)ts.BH, (cuuint32_t)ts.BNn};
                 cuuint32_t yes[4] = {1, 1, 1, 1};
-                void *ybase = (char *)y + Lout.offset(i, j) * 2;
+                const int64_t yoff = Lout.offset(i, j) + ((int64_t)prh * fw + prw) * yc;
+                void *ybase = (char *)y + yoff * 2;
                 if (encode(&P.mapY[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, ybase, ydims, ystr, ybox, yes,
                            CU_TENSOR_MAP_INTERLEAVE_NONE, swz_for(P.ychunk * 2), CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
                     return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(Y) failed");
                 if (relu_src) {
-                    void *rbase = (char *)relu_src + Lout.offset(i, j) * 2;
+                    void *rbase = (char *)relu_src + yoff * 2;
                     if (encode(&P.mapR[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, rbase, ydims, ystr, ybox, yes,
                                CU_TENSOR_MAP_INTERLEAVE_NONE, swz_for(P.ychunk * 2), CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
@@ -1425,8 +1460,15 @@ bool conv_tc_supported(int mode, splitcnn_dtype_t dt, const Level &Li, const Lev
         return true;
     }
     if (mode == 1) {
-        if (g.L.sh != 1) return false;  // stride-2 dgrad: CUDA-core path (phase decomposition is future work)
         if (!a_channels_ok(Lo.Cpad)) return false;
+        if (g.L.sh == 1) return true;
+        // stride S > 1: phase decomposition -- one begin pad per dimension, every patch at least S
+        // pixels wide (no empty phase view), TMA-store output channels
+        if (g.L.sh > 2 || !(Li.Cpad == 8 || Li.Cpad == 16 || Li.Cpad == 32 || Li.Cpad % 64 == 0)) return false;
+        for (int i = 0; i < Li.nh(); ++i)
+            if (g.pad_h[2 * i] != g.pad_h[0] || Li.ph(i) < g.L.sh) return false;
+        for (int j = 0; j < Li.nw(); ++j)
+            if (g.pad_w[2 * j] != g.pad_w[0] || Li.pw(j) < g.L.sw) return false;
         return true;
     }
     if (mode == 2) return wgrad_tc_ok(Li, Lo, g);
@@ -1435,7 +1477,7 @@ bool conv_tc_supported(int mode, splitcnn_dtype_t dt, const Level &Li, const Lev
 
 size_t conv_tc_ws_bytes(int mode, const Level &Li, const Level &Lo, const LayerGeom &g) {
     if (mode == 2) return wgrad_tc_ws_bytes(Li, Lo, g);
-    if (mode == 1) return (size_t)g.L.cin * g.L.kh * g.L.kw * Lo.Cpad * 2 + 256;
+    if (mode == 1) return (size_t)g.L.cin * g.L.kh * g.L.kw * Lo.Cpad * 2 + 256 + (size_t)g.L.sh * g.L.sw * 1024;
     return 0;
 }
 
@@ -1456,11 +1498,42 @@ splitcnn_status_t launch_conv_pool_fwd_tc(const Level &Li, const Level &Lo, cons
 
 splitcnn_status_t launch_conv_dgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy, const void *w,
                                        void *dx, const void *relu_src, void *ws, int p0, int p1, cudaStream_t st) {
-    const int64_t n = (int64_t)g.L.cin * g.L.kh * g.L.kw * Lo.Cpad;
-    flip_weights_kernel<<<(unsigned)std::min<int64_t>((n + 255) / 256, 2048), 256, 0, st>>>(
-        (const __nv_bfloat16 *)w, (__nv_bfloat16 *)ws, g.L.cout, Li.Cpad, g.L.cin, g.L.kh, g.L.kw, Lo.Cpad);
-    count_launch();
-    return launch_tc(1, Lo, Li, g, dy, ws, g.L.cin, nullptr, dx, relu_src, 0, p0, p1, st);
+    const int S = g.L.sh, kh = g.L.kh, kw = g.L.kw;
+    if (S == 1) {
+        const int64_t n = (int64_t)g.L.cin * kh * kw * Lo.Cpad;
+        flip_weights_kernel<<<(unsigned)std::min<int64_t>((n + 255) / 256, 2048), 256, 0, st>>>(
+            (const __nv_bfloat16 *)w, (__nv_bfloat16 *)ws, g.L.cout, Li.Cpad, g.L.cin, kh, kw, Lo.Cpad, 0, 0, 1, kh, kw);
+        count_launch();
+        return launch_tc(1, Lo, Li, g, dy, ws, g.L.cin, nullptr, dx, relu_src, 0, p0, p1, st);
+    }
+    // stride S: S*S output phases, each a stride-1 correlation with the taps r = (rho + p_b) (mod S)
+    // (every patch of a plan shares its begin pad under R2, checked in conv_tc_supported)
+    const int pbh = g.pad_h[0], pbw = g.pad_w[0];
+    char *wsp = (char *)ws;
+    for (int rh = 0; rh < S; ++rh)
+        for (int rw = 0; rw < S; ++rw) {
+            const int r0h = ((rh + pbh) % S + S) % S, r0w = ((rw + pbw) % S + S) % S;
+            const int nth = r0h < kh ? (kh - r0h + S - 1) / S : 0, ntw = r0w < kw ? (kw - r0w + S - 1) / S : 0;
+            if (nth == 0 || ntw == 0) {
+                LevelDesc d = make_level_desc(Li);
+                dim3 grid((unsigned)std::max(1, std::min(2048, 148 * 8 / std::max(1, p1 - p0))), (unsigned)(p1 - p0));
+                zero_phase_kernel<<<grid, 256, 0, st>>>((__nv_bfloat16 *)dx, d, S, rh, rw, p0);
+                count_launch();
+                continue;
+            }
+            const int ch = (rh + pbh - r0h) / S, cw = (rw + pbw - r0w) / S;
+            const int64_t n = (int64_t)g.L.cin * nth * ntw * Lo.Cpad;
+            flip_weights_kernel<<<(unsigned)std::min<int64_t>((n + 255) / 256, 2048), 256, 0, st>>>(
+                (const __nv_bfloat16 *)w, (__nv_bfloat16 *)wsp, g.L.cout, Li.Cpad, g.L.cin, kh, kw, Lo.Cpad, r0h, r0w, S,
+                nth, ntw);
+            count_launch();
+            Phase ph{S, rh, rw, nth, ntw, nth - 1 - ch, ntw - 1 - cw};
+            const splitcnn_status_t r = launch_tc(1, Lo, Li, g, dy, wsp, g.L.cin, nullptr, dx, relu_src, 0, p0, p1, st,
+                                                  nullptr, &ph);
+            if (r != SPLITCNN_OK) return r;
+            wsp += ((n * 2 + 1023) / 1024) * 1024;
+        }
+    return SPLITCNN_OK;
 }
 
 // ============================================================ weight gradient (tcgen05, MN-major)

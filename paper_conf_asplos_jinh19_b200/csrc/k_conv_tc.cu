@@ -2219,7 +2219,30 @@ size_t wgrad_tc_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g) {
     const int64_t ngroups = (Lo.npatch() + TC_MAXP - 1) / TC_MAXP;
     const int64_t zmax = ngroups * wgrad_zbound(path, Li, g);
     const int64_t nW = (int64_t)g.L.cout * g.L.kh * g.L.kw * Li.Cpad;
-    return std::max((size_t)zmax * nW * sizeof(float), (size_t)4 * 148 * g.L.cout * sizeof(float)) + 256;
+    // + a separate region for the db column-sum partials (computed concurrently, see launch_conv_wgrad_tc)
+    const size_t dbp = (((size_t)4 * 148 * g.L.cout * sizeof(float)) + 255) & ~(size_t)255;
+    return (((size_t)zmax * nW * sizeof(float) + 255) & ~(size_t)255) + dbp + 256;
+}
+
+// Library-owned side stream per device (fork/join through events, so the caller's stream semantics are
+// kept, and CUDA-graph capture records the fork as a parallel branch).
+struct SideStream {
+    cudaStream_t s = nullptr;
+    cudaEvent_t fork = nullptr, join = nullptr;
+};
+static SideStream &side_stream() {
+    static SideStream ss[16];
+    static std::mutex mu;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> lk(mu);
+    SideStream &r = ss[dev & 15];
+    if (!r.s) {
+        cudaStreamCreateWithFlags(&r.s, cudaStreamNonBlocking);
+        cudaEventCreateWithFlags(&r.fork, cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&r.join, cudaEventDisableTiming);
+    }
+    return r;
 }
 
 int launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, float *part, int cout, int p0, int p1,
@@ -2238,6 +2261,23 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
     const int64_t zcap = (int64_t)((Lo.npatch() + TC_MAXP - 1) / TC_MAXP) * wgrad_zbound(path, Li, g);
     int zoff = 0;   // split partials written so far (all launches of this call)
     int gend = p1;  // end of the patch range left for the generic kernel
+    // db = column sums of dY: HBM-bound, while the wgrad GEMM is not -- run it concurrently on a side
+    // stream (forked after dY's producer, joined before this call returns), into its own partial region
+    float *part_db = (float *)((char *)ws + ((((size_t)zcap * nW * sizeof(float)) + 255) & ~(size_t)255));
+    SideStream *ss = nullptr;
+    if (db) {
+        ss = &side_stream();
+        cudaEventRecord(ss->fork, st);
+        cudaStreamWaitEvent(ss->s, ss->fork, 0);
+    }
+    bool db_launched = false;
+    auto launch_db = [&]() {
+        if (!db || db_launched) return;
+        db_launched = true;
+        const int Zd = launch_db_partials(SPLITCNN_BF16, Lo, dy, part_db, g.L.cout, p0, p1, ss->s);
+        launch_reduce(part_db, Zd, g.L.cout, db, beta, ss->s);
+        cudaEventRecord(ss->join, ss->s);
+    };
     if (path == 2) {
         static bool narrow_attr = false;
         for (int g0 = p0; g0 < p1; g0 += TC_MAXP) {
@@ -2300,6 +2340,7 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
             }
             wgrad_narrow_kernel<<<c.nco_blk * c.nsplit, 192, smem, st>>>(P);
             count_launch();
+            launch_db();
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("wgrad_narrow_kernel: ") + cudaGetErrorString(e));
             zoff += c.nsplit;
@@ -2387,6 +2428,7 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
                 wgrad_halo_kernel<false><<<c.ntiles * c.nsplit, 192, smem, st>>>(P);
             }
             count_launch();
+            launch_db();
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("wgrad_halo_kernel: ") + cudaGetErrorString(e));
             zoff += c.nsplit;
@@ -2478,6 +2520,7 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
         }
         wgrad_tc_kernel<<<c.ntiles * c.nsplit, 192, smem, st>>>(P);
         count_launch();
+        launch_db();
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("wgrad_tc_kernel: ") + cudaGetErrorString(e));
         zoff += c.nsplit;
@@ -2487,9 +2530,10 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
     // reproducible, and beta = 1 gives exactly 2x whatever the number of launches
     launch_reduce(part, zoff, nW, dw, beta, st);
     if (db) {
-        // the dW partials have been consumed by the reduction (stream order): reuse the space
-        const int Zd = launch_db_partials(SPLITCNN_BF16, Lo, dy, part, g.L.cout, p0, p1, st);
-        launch_reduce(part, Zd, g.L.cout, db, beta, st);
+        launch_db();                              // (no GEMM launch when the range is empty)
+        cudaStreamWaitEvent(st, ss->join, 0);     // join: db is complete in the caller's stream order
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("db column sums: ") + cudaGetErrorString(e));
     }
     return SPLITCNN_OK;
 }

@@ -1961,7 +1961,9 @@ __global__ void __launch_bounds__(192, 1) wgrad_narrow_kernel(const __grid_const
     const int Wp = 8 + p.kw - 1, Hp = p.BH + p.kh - 1;
     const int KT = p.kh * p.kw, npairs = (KT + 1) / 2;
     const uint32_t a_blk = (uint32_t)rows * 128u;
-    const uint32_t a_stage = 2u * a_blk;
+    // Cout <= 64: one dY channel block per stage; the MMA's upper 64 rows then read the next stage's
+    // bytes and produce accumulator rows for channels >= Cout, which are never stored
+    const uint32_t a_stage = (p.Cout <= 64 ? 1u : 2u) * a_blk;
     const uint32_t b_bytes = (uint32_t)Wp * Hp * 16u;
     const uint32_t b_stage = (b_bytes + 1023u) & ~1023u;
     uint8_t *sA = smem;
@@ -2000,10 +2002,11 @@ __global__ void __launch_bounds__(192, 1) wgrad_narrow_kernel(const __grid_const
                 const int hb = idx % p.nhb[ql], n = idx / p.nhb[ql];
                 const int ow0 = wb * 8, oh0 = hb * p.BH;
                 tc::mbar_wait_sleep(&empty[stage], ph ^ 1);
-                tc::mbar_arrive_expect_tx(&full[stage], a_stage + b_bytes);
+                const bool hi = co_blk * 128 + 64 < p.Cout;     // upper 64-channel block has real channels
+                tc::mbar_arrive_expect_tx(&full[stage], (hi ? 2u : 1u) * a_blk + b_bytes);
                 uint8_t *a = sA + (size_t)stage * a_stage;
                 tc::tma_load_4d(a, &p.mapDY[ql], &full[stage], co_blk * 128, ow0, oh0, n);
-                tc::tma_load_4d(a + a_blk, &p.mapDY[ql], &full[stage], co_blk * 128 + 64, ow0, oh0, n);
+                if (hi) tc::tma_load_4d(a + a_blk, &p.mapDY[ql], &full[stage], co_blk * 128 + 64, ow0, oh0, n);
                 tc::tma_load_3d(sB + (size_t)stage * b_stage, &p.mapX[ql], &full[stage], 8 * (ow0 - p.pl[ql]),
                                 oh0 - p.pt[ql], n);
                 if (++stage == S) { stage = 0; ph ^= 1; }
@@ -2290,10 +2293,13 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
             P.nco_blk = c.nco_blk; P.boxes_per_split = c.boxes_per_split; P.nsplit = c.nsplit;
             P.Cout = g.L.cout;
             const int Wp = 8 + g.L.kw - 1, Hp = c.BH + g.L.kh - 1;
-            const uint32_t a_stage = 2u * c.BH * 8u * 128u;
+            const uint32_t a_stage = (g.L.cout <= 64 ? 1u : 2u) * c.BH * 8u * 128u;
             const uint32_t b_stage = ((uint32_t)Wp * Hp * 16u + 1023u) & ~1023u;
             const uint32_t stage_bytes = a_stage + b_stage;
-            P.stages = std::min<int>(8, (int)((200u * 1024u) / stage_bytes));
+            // two co-resident CTAs per SM (grid = 2 x SMs) hide each other's TMA latency when the
+            // stages fit in half the shared memory
+            const uint32_t budget = (4u * stage_bytes <= 100u * 1024u) ? 100u * 1024u : 200u * 1024u;
+            P.stages = std::min<int>(8, (int)(budget / stage_bytes));
             uint32_t cols = 32;
             while (cols < (uint32_t)(g.L.kh * (((g.L.kw * 8 + 15) / 16) * 16))) cols <<= 1;
             P.tmem_cols = cols;

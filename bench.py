@@ -92,7 +92,7 @@ def make_inputs(c, dtype_t, device, world=1, rank=0):
         params = [p for p in synth.layer_params(g, c["layers"] + c["tail"]) if p is not None]
     gen = torch.Generator(device="cpu").manual_seed(c["seed"])
     N = c["N"]
-    x = (torch.rand((N, 3, c["H"], c["W"]), generator=gen) * 2 - 1).to(dtype_t)
+    x = (torch.rand((N, c.get("C", 3), c["H"], c["W"]), generator=gen) * 2 - 1).to(dtype_t)
     return params, x, gen
 
 
@@ -112,6 +112,8 @@ def run_ours(args):
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     c = workload(args.config)
+    if args.dtype is None:
+        args.dtype = c.get("dtype", "bf16")
     dtype = sc.BF16 if args.dtype == "bf16" else sc.FP32
     use_offload = args.offload if args.offload is not None else (args.config == "C4")
     if c.get("resnet"):
@@ -129,8 +131,9 @@ def run_ours(args):
         net = OffloadSplitNet(c["layers"], c["tail"], c["N"], 3, c["H"], c["W"], split=c["split"], mode=c["mode"],
                               omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype)
     else:
-        net = SplitNet(c["layers"], c["tail"], c["N"], 3, c["H"], c["W"], split=c["split"], mode=c["mode"],
+        net = SplitNet(c["layers"], c["tail"], c["N"], c.get("C", 3), c["H"], c["W"], split=c["split"], mode=c["mode"],
                        omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype)
+    net.input_grad = args.config == "C1"      # C1 = one layer's fwd + dgrad + wgrad
     params, x_host, gen = make_inputs(c, net.tdtype, "cuda")
     net.set_params([(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params])
     x = x_host.cuda()
@@ -320,7 +323,7 @@ def oracle_sample_time(config: str, tiles: int):
         h = OP.out_len(h, l["kh"], l["sh"], l["ph_b"], l["ph_e"])
     total = 0.0
     sample_px = 0
-    first_conv = True
+    first_conv = config != "C1"     # C1 times its dgrad too
     for l, prm, h in ops:
         ho = OP.out_len(h, l["kh"], l["sh"], l["ph_b"], l["ph_e"])
         # a tile = a patch of an 8x8 even split of this layer's output (>= 1 px)
@@ -392,8 +395,8 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="C5", choices=["C2", "C3", "C4", "C5"])
-    ap.add_argument("--dtype", default="bf16", choices=["bf16", "fp32"])
+    ap.add_argument("--config", default="C5", choices=["C1", "C2", "C3", "C4", "C5"])
+    ap.add_argument("--dtype", default=None, choices=["bf16", "fp32"])
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--cpu-tiles", type=int, default=12)
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -81,7 +81,14 @@ typedef enum { SPLITCNN_BF16 = 0, SPLITCNN_FP32 = 1 } splitcnn_dtype_t;
 
 typedef enum { SPLITCNN_OP_CONV = 0, SPLITCNN_OP_MAXPOOL = 1 } splitcnn_op_t;
 
-typedef enum { SPLITCNN_NCHW = 0, SPLITCNN_NHWC = 1 } splitcnn_layout_t;
+typedef enum {
+    SPLITCNN_NCHW = 0,
+    SPLITCNN_NHWC = 1,
+    /* split only: NCHW full tensor of C/4 channels and 2H x 2W pixels read space-to-depth by 2:
+     * level channel 4c + 2*ph + pw of pixel (h, w) = x[n, c, 2h + ph, 2w + pw].  A stride-2 conv on the
+     * full tensor equals a stride-1 conv on this level with regrouped weights (the ResNet stem). */
+    SPLITCNN_NCHW_S2D = 2
+} splitcnn_layout_t;
 
 /* flags */
 #define SPLITCNN_FLAG_RELU 0x1u            /* conv_fwd: fuse ReLU into the epilogue */
@@ -167,7 +174,8 @@ SPLITCNN_API splitcnn_status_t splitcnn_workspace_size(splitcnn_plan_t plan, int
 
 /* ------------------------------------------------------------------ split / merge */
 /* Eq. 4: copy the full tensor x (level `level`'s N, C, H, W; layout x_layout) into
- * the level's patch buffers (+ transpose to NHWC, + zero channel padding). */
+ * the level's patch buffers (+ transpose to NHWC, + zero channel padding).  SPLITCNN_NCHW_S2D needs
+ * C % 4 == 0 and even patch boundaries are implied (x is N x C/4 x 2H x 2W). */
 SPLITCNN_API splitcnn_status_t splitcnn_split(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
                                  const void *x, int32_t x_layout, void *patches,
                                  int32_t p0, int32_t p1, splitcnn_stream_t stream);

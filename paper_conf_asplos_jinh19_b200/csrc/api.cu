@@ -116,7 +116,10 @@ extern "C" splitcnn_status_t splitcnn_split(splitcnn_plan_t plan, int32_t level,
     if (!plan || level < 0 || level >= (int)plan->levels.size()) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad level");
     TRY(check_dtype(dtype));
     if (!x || !patches) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
-    if (x_layout != SPLITCNN_NCHW && x_layout != SPLITCNN_NHWC) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad layout");
+    if (x_layout != SPLITCNN_NCHW && x_layout != SPLITCNN_NHWC && x_layout != SPLITCNN_NCHW_S2D)
+        return fail(SPLITCNN_ERR_INVALID_VALUE, "bad layout");
+    if (x_layout == SPLITCNN_NCHW_S2D && plan->levels[level].C % 4)
+        return fail(SPLITCNN_ERR_INVALID_VALUE, "space-to-depth split needs C % 4 == 0");
     NEED_ALIGNED(x, "x");
     NEED_ALIGNED(patches, "patches");
     TRY(check_range(plan, level, p0, p1));

@@ -27,7 +27,7 @@ __device__ __forceinline__ void dec3(uint32_t u, const Dec3 &d, int &x0, int &x1
     u = fdivmod(u, d.c, r); x2 = (int)r;
     x3 = (int)u;
 }
-template <typename T, bool NCHW>
+template <typename T, bool NCHW, bool S2D = false>
 __global__ void __launch_bounds__(256) split_kernel(LevelDesc L, const T *__restrict__ x, T *__restrict__ P, int p0) {
     const PatchGeo g = patch_geo(L, p0 + blockIdx.y);
     const int G = L.Cpad / 8;
@@ -39,7 +39,15 @@ __global__ void __launch_bounds__(256) split_kernel(LevelDesc L, const T *__rest
         else dec3(u, d, cg, w, h, n);        // channel-fastest: coalesced 16 B reads and writes
         const int hg = g.h0 + h, wg = g.w0 + w, c0 = cg * 8;
         float v[8];
-        if (NCHW) {
+        if (S2D) {   // level channel 4c + 2ph + pw of (hg, wg) = x[n, c, 2hg + ph, 2wg + pw]
+            const int C4 = L.C >> 2, H2 = 2 * L.H, W2 = 2 * L.W;
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+                const int cc = c0 + k;
+                v[k] = (cc < L.C) ? to_f(x[(((int64_t)n * C4 + (cc >> 2)) * H2 + 2 * hg + ((cc >> 1) & 1)) * W2 + 2 * wg + (cc & 1)])
+                                  : 0.f;
+            }
+        } else if (NCHW) {
 #pragma unroll
             for (int k = 0; k < 8; ++k)
                 v[k] = (c0 + k < L.C) ? to_f(x[(((int64_t)n * L.C + c0 + k) * L.H + hg) * L.W + wg]) : 0.f;
@@ -110,7 +118,9 @@ void launch_split_t(const Level &L, const void *x, int layout, void *P, int p0, 
     npatch_launch = p1 - p0;
     dim3 grid(grid_x_for(max_patch_units(L, p0, p1, L.Cpad / 8)), p1 - p0);
     LevelDesc d = make_level_desc(L);
-    if (layout == SPLITCNN_NCHW)
+    if (layout == SPLITCNN_NCHW_S2D)
+        { split_kernel<T, true, true><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0); count_launch(); }
+    else if (layout == SPLITCNN_NCHW)
         { split_kernel<T, true><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0); count_launch(); }
     else
         { split_kernel<T, false><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0); count_launch(); }

@@ -42,6 +42,7 @@ class SplitNet:
         self.input_relu = input_relu   # level 0 is a ReLU output (e.g. a tail fed by a ReLU conv)
         self.fuse_pool = fuse_pool and dtype == sc.BF16 and not force_simt
         self.step_index = 0
+        self.input_grad = False  # step(): also compute dX of the first layer (C1's single-layer pass)
         self.timers = None       # list -> every library call is bracketed by CUDA events (bench.py)
         self._label = ""
         self.region = self._make_region_plan(0)
@@ -303,7 +304,7 @@ class SplitNet:
     def step(self, x, dy, stream=None):
         self.replan(self.step_index)
         self.forward(x, stream)
-        self.backward(dy, stream)
+        self.backward(dy, stream, need_input_grad=self.input_grad)
         self.step_index += 1
 
     # ------------------------------------------------------------------ accounting
@@ -320,7 +321,7 @@ class SplitNet:
                     continue
                 lo = plan.levels[m + 1]
                 f = 2 * lo["N"] * l["cout"] * lo["H"] * lo["W"] * l["cin"] * l["kh"] * l["kw"]
-                total += f * (2 if first else 3)
+                total += f * (2 if first and not self.input_grad else 3)
                 first = False
         return total
 

@@ -24,11 +24,59 @@ from .net import SplitNet, pack_weight
 from .plan import SplitPlan
 
 
+def s2d_stem_layer(l: dict) -> dict:
+    """The 7x7 s2 p3 stem on C channels as the equivalent 4x4 s1 conv on the space-to-depth(2) input
+    (4C channels, H/2 x W/2): out[t] = sum_{q, phi} Xs2d[t + q - 2][phi] * W[2q + phi - 1] (tap -1 is
+    zero), i.e. begin pad 2, end pad 1 -- and under R2 the same patch-local pads (2, k - s - p_b = 1)."""
+    return dict(op="conv", kh=4, kw=4, sh=1, sw=1, ph_b=2, ph_e=1, pw_b=2, pw_e=1, cin=4 * l["cin"],
+                cout=l["cout"], relu=l.get("relu", True), name=l.get("name", "conv1"))
+
+
+def s2d_stem_weight(W: torch.Tensor) -> torch.Tensor:
+    """OIHW [Co][C][7][7] -> OIHW [Co][4C][4][4]: W''[o][4c + 2ph + pw][qh][qw] = W[o][c][2qh+ph-1][2qw+pw-1]."""
+    co, c, kh, kw = W.shape
+    out = torch.zeros((co, 4 * c, 4, 4), dtype=W.dtype, device=W.device)
+    for qh in range(4):
+        for ph in range(2):
+            r = 2 * qh + ph - 1
+            if not 0 <= r < kh:
+                continue
+            for qw in range(4):
+                for pw in range(2):
+                    s = 2 * qw + pw - 1
+                    if 0 <= s < kw:
+                        out[:, 2 * ph + pw::4, qh, qw] = W[:, :, r, s]
+    return out
+
+
+def s2d_stem_grad(dWp: torch.Tensor, cin: int) -> torch.Tensor:
+    """Packed stem gradient [Co][4][4][Cpad >= 4*cin] -> OIHW [Co][cin][7][7] (adjoint of s2d_stem_weight;
+    the zero tap's gradient is dropped)."""
+    co = dWp.shape[0]
+    out = torch.zeros((co, cin, 7, 7), dtype=dWp.dtype, device=dWp.device)
+    for r in range(7):
+        qh, ph = (r + 1) // 2, (r + 1) % 2
+        for s_ in range(7):
+            qw, pw = (s_ + 1) // 2, (s_ + 1) % 2
+            out[:, :, r, s_] = dWp[:, qh, qw, 2 * ph + pw:4 * cin:4]
+    return out
+
+
 class ResSplitNet(SplitNet):
     def __init__(self, chain: list[dict], blocks: list[dict], N: int, C: int, H: int, W: int, split=(2, 2),
-                 dtype: int = sc.BF16, device="cuda", force_simt: bool = False, **kw):
+                 dtype: int = sc.BF16, device="cuda", force_simt: bool = False, s2d_stem: bool | None = None, **kw):
         self.blocks = blocks
         self.block_at = {b["a"]: k for k, b in enumerate(blocks)}
+        st = chain[0]
+        ok = (st["op"] == "conv" and st["kh"] == st["kw"] == 7 and st["sh"] == st["sw"] == 2 and st["ph_b"] == 3
+              and H % 2 == 0 and W % 2 == 0 and dtype == sc.BF16 and not force_simt)
+        # the stride-2 stem on a 3-channel input is a poor tensor-core shape (8-channel padded, strided
+        # TMA rows); read space-to-depth it is a stride-1 4x4 conv on 12 (pad 16) channels, same sums
+        self.s2d = ok if s2d_stem is None else (s2d_stem and ok)
+        self.stem_cin = st["cin"]
+        if self.s2d:
+            chain = [s2d_stem_layer(st)] + list(chain[1:])
+            C, H, W = 4 * C, H // 2, W // 2
         super().__init__(chain, [], N, C, H, W, split=split, mode="even", dtype=dtype, device=device,
                          force_simt=force_simt, fuse_pool=False, **kw)
 
@@ -94,11 +142,22 @@ class ResSplitNet(SplitNet):
                 self._ds_params[k] = (
                     torch.zeros((l["cout"], l["kh"], l["kw"], p.levels[0]["Cpad"]), dtype=self.tdtype, device=self.device),
                     torch.zeros(l["cout"], dtype=torch.float32, device=self.device))
+        if self.s2d:
+            W0, b0 = params[0]
+            params = [(s2d_stem_weight(torch.as_tensor(W0)), b0)] + params[1:]
         super().set_params(params[:nchain])
         for (k, l, p), (W, b) in zip(self._ds_layers(), params[nchain:]):
             W = torch.as_tensor(W).to(self.device)
             self._ds_params[k][0].copy_(pack_weight(W, p.levels[0]["Cpad"], self.tdtype))
             self._ds_params[k][1].copy_(torch.as_tensor(b, dtype=torch.float32))
+
+    def grad_oihw(self, key) -> torch.Tensor:
+        """Weight gradient of conv `key` in OIHW (the stem's s2d gradient mapped back to 7x7)."""
+        dW = self.grads[key][0]
+        if key == ("r", 0) and self.s2d:
+            return s2d_stem_grad(dW, self.stem_cin)
+        l = self.region_layers[key[1]] if key[0] == "r" else self.blocks[key[1]]["ds"]
+        return dW[..., :l["cin"]].permute(0, 3, 1, 2)
 
     def _masked(self, key: str, m: int) -> bool:
         """ReLU mask of level m: conv outputs with their own ReLU, and block outputs (ReLU after the add)."""
@@ -112,6 +171,8 @@ class ResSplitNet(SplitNet):
         R, dt, fl = self.region.handle, self.dtype, self.flags_extra
         acts = self.act_r
         self._label = "input"
+        if self.s2d:
+            x_layout = sc.NCHW_S2D
         self._call("split", 2 * self._bytes(self.region, 0)[0], sc.splitcnn_split, R, 0, dt, x, x_layout, acts[0],
                    p0, p1, stream)
         m = 0

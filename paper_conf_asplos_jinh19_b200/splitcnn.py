@@ -22,7 +22,7 @@ _lib = ctypes.CDLL(LIB_PATH)
 OK, ERR_INVALID_VALUE, ERR_ALIGNMENT, ERR_UNSUPPORTED, ERR_CUDA, ERR_OOM = range(6)
 BF16, FP32 = 0, 1
 OP_CONV, OP_MAXPOOL = 0, 1
-NCHW, NHWC = 0, 1
+NCHW, NHWC, NCHW_S2D = 0, 1, 2
 FLAG_RELU = 0x1
 FLAG_POOL_RELU_MASK = 0x2
 FLAG_FORCE_SIMT = 0x100

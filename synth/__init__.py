@@ -87,7 +87,7 @@ def split_region(layers, depth_convs: int, include_next_pool: bool):
 # --------------------------------------------------------------------------- BASELINE.json configs
 CONFIGS = {
     "C1": dict(name="C1", desc="single split conv3x3 layer, N=2, C=16->16, 32x32, 2x2 split, fp32",
-               layers=[conv(16, 16, relu=False, name="conv")], tail=[], N=2, C=3, H=32, W=32,
+               layers=[conv(16, 16, relu=False, name="conv")], tail=[], N=2, C=16, H=32, W=32,
                split=(2, 2), mode="even", dtype="fp32", seed=0),
     "C2": dict(name="C2", desc="VGG-19 conv stack, CIFAR-shaped 32x32, N=128, 2x2 split, depth 50%",
                N=128, H=32, W=32, split=(2, 2), mode="even", depth=8, pool_inside=True,
@@ -106,6 +106,10 @@ CONFIGS = {
 def vgg_config(name: str, N: int | None = None):
     """Region/tail layer lists of a VGG config, optionally at a reduced batch ``N``."""
     c = dict(CONFIGS[name])
+    if "layers" in c:                      # C1: one explicit layer, no VGG region/tail split
+        if N is not None:
+            c["N"] = N
+        return c
     if c.get("resnet"):
         c["layers"], c["blocks"] = resnet18_blocks()
         c["tail"], c["C"] = [], 3

@@ -22,10 +22,12 @@ def sc():
     return splitcnn
 
 
-def _run(sc, dtype, N=2, H=64, widths=(64, 128), split=(2, 2), seed=2):
+def _run(sc, dtype, N=2, H=64, widths=(64, 128), split=(2, 2), seed=2, s2d=None):
     from paper_conf_asplos_jinh19_b200.resnet import ResSplitNet
     chain, blocks = synth.resnet18_blocks(*widths)
-    net = ResSplitNet(chain, blocks, N, 3, H, H, split=split, dtype=dtype)
+    net = ResSplitNet(chain, blocks, N, 3, H, H, split=split, dtype=dtype, s2d_stem=s2d)
+    if s2d is not None:
+        assert net.s2d == s2d
     g = synth.rng(seed)
     bf = dtype == sc.BF16
     X = synth.uniform(g, (N, 3, H, H))
@@ -50,9 +52,8 @@ def _run(sc, dtype, N=2, H=64, widths=(64, 128), split=(2, 2), seed=2):
     got = out.float().cpu().numpy().reshape(N, L["H"], L["W"], L["C"]).transpose(0, 3, 1, 2)
     errs = {"out": normwise(got, ref_out)}
     keys = [("r", m) for m, l in enumerate(chain) if l["op"] == "conv"] + [("ds", k) for k in sorted(net.ds_plans)]
-    cins = [l["cin"] for l in chain if l["op"] == "conv"] + [blocks[k]["ds"]["cin"] for k in sorted(net.ds_plans)]
-    for i, (key, cin) in enumerate(zip(keys, cins)):
-        dW = w_lib_to_oihw(net.grads[key][0].cpu().numpy(), cin)
+    for i, key in enumerate(keys):
+        dW = net.grad_oihw(key).double().cpu().numpy()
         errs[f"dW{i}"] = normwise(dW, dWs[i])
         errs[f"db{i}"] = normwise(net.grads[key][1].cpu().numpy(), dbs[i])
     # the block outputs are the merged output of the last level; also check level 2 (pool output)
@@ -77,6 +78,52 @@ def test_resnet_stack_bf16(sc):
     errs = _run(sc, sc.BF16)
     assert errs["out"] <= 2e-2, errs
     assert max(errs.values()) <= 1e-1, errs
+
+
+def test_resnet_stack_bf16_strided_stem(sc):
+    """The same stack with the stem run as the plain 7x7 s2 conv (no space-to-depth): same bounds."""
+    errs = _run(sc, sc.BF16, s2d=False)
+    assert errs["out"] <= 2e-2, errs
+    assert max(errs.values()) <= 1e-1, errs
+
+
+def test_s2d_stem_conv_matches_oracle_per_op(sc):
+    """Space-to-depth stem (split layout NCHW_S2D + 4x4 s1 conv on 12 channels) vs the oracle's 7x7 s2
+    p3 split conv, forward and weight gradient, bf16 within 2e-2 (same products, other order)."""
+    from oracle import ops as O
+    from oracle import plan as OP
+    from paper_conf_asplos_jinh19_b200.plan import SplitPlan
+    from paper_conf_asplos_jinh19_b200.resnet import s2d_stem_layer, s2d_stem_weight, s2d_stem_grad
+    g = synth.rng(11)
+    N, H, cout = 2, 60, 64
+    l = synth.conv(3, cout, k=7, s=2, p=3)
+    X = synth.to_bf16_f32(synth.uniform(g, (N, 3, H, H)))
+    Wt = synth.to_bf16_f32(synth.kaiming(g, cout, 3, 7, 7))
+    b = synth.uniform(g, (cout,), -0.1, 0.1)
+    G = synth.to_bf16_f32(synth.normal(g, (N, cout, 30, 30)))
+    Oh = [0, 11, 30]
+    ref = OP.plan([l], N, 3, H, H, Oh, Oh).layers[0]
+    pl = SplitPlan([s2d_stem_layer(l)], N, 12, H // 2, H // 2, Oh, Oh)
+    lv0, lv1 = pl.levels
+    assert lv0["bh"] == [v // 2 for v in ref.Ih]
+    x = torch.from_numpy(X).to("cuda", torch.bfloat16)
+    xp = torch.empty(lv0["total_elems"], dtype=torch.bfloat16, device="cuda")
+    sc.splitcnn_split(pl.handle, 0, sc.BF16, x, sc.NCHW_S2D, xp)
+    from paper_conf_asplos_jinh19_b200.net import pack_weight
+    w = pack_weight(s2d_stem_weight(torch.from_numpy(Wt)).cuda(), lv0["Cpad"], torch.bfloat16)
+    y = torch.empty(lv1["total_elems"], dtype=torch.bfloat16, device="cuda")
+    sc.splitcnn_conv_fwd(pl.handle, 0, sc.BF16, xp, w, torch.from_numpy(b).cuda(), y, 0)
+    Yref = O.conv_fwd(O.split(X.astype(np.float64), ref.Ih, ref.Iw), Wt.astype(np.float64), b.astype(np.float64), ref)
+    from tests.helpers import pack_level
+    got = unpack_level(y.float().cpu().numpy(), lv1)
+    assert max(normwise(got[i][j], Yref[i][j]) for i in range(2) for j in range(2)) <= 2e-2
+    dy = torch.from_numpy(pack_level(G.astype(np.float64), lv1).astype(np.float32)).to("cuda", torch.bfloat16)
+    ws_b = max(pl.workspace_size(0, sc.BF16, 2), 16)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    dw = torch.zeros((cout, 4, 4, lv0["Cpad"]), dtype=torch.float32, device="cuda")
+    sc.splitcnn_conv_bwd_filter(pl.handle, 0, sc.BF16, xp, dy, dw, None, 0.0, ws, ws_b)
+    dWref, _ = O.conv_bwd_filter(O.split(X.astype(np.float64), ref.Ih, ref.Iw), O.split(G.astype(np.float64), Oh, Oh), ref)
+    assert normwise(s2d_stem_grad(dw, 3).double().cpu().numpy(), dWref) <= 2e-2
 
 
 def test_resnet_stack_ragged_fp32(sc):

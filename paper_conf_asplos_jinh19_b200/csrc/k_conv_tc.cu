@@ -1782,7 +1782,9 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
     const int rows = p.BNn * p.BH * 8;
     const int Wp = 8 + p.kw - 1;
     const uint32_t a_blk = (uint32_t)rows * 128u;     // one 64-channel dY block
-    const uint32_t a_stage = 2u * a_blk;
+    // Cout <= 64: the upper dY block is all out of bounds -- not loaded, and not even given space (the
+    // MMA's rows 64..127 read the next stage's bytes; those accumulator rows are never stored)
+    const uint32_t a_stage = (p.Cout <= 64 ? 1u : 2u) * a_blk;
     const uint32_t xrow = CTA2 ? 64u : 128u;            // bytes per X pixel row (32 or 64 channels)
     const uint32_t b_bytes = (uint32_t)Wp * p.BH * p.BNn * xrow;
     const uint32_t b_stage = (b_bytes + 1023u) & ~1023u;
@@ -1827,7 +1829,8 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
         if (lane == 0) {
             int stage = 0, ql = 0;
             uint32_t ph = 0;
-            const uint32_t tx = a_stage + b_bytes;
+            const bool hi = p.Cout > 64;
+            const uint32_t tx = (hi ? 2u : 1u) * a_blk + b_bytes;
             for (int b = b0; b < b1; ++b) {
                 while (b >= p.box_prefix[ql + 1]) ++ql;
                 int idx = b - p.box_prefix[ql];
@@ -1849,7 +1852,7 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
                 }
                 tc::mbar_arrive_expect_tx(&full[stage], tx);
                 tc::tma_load_4d(a, &p.mapDY[ql], &full[stage], co_blk * 128, ow0, oh0, n);
-                tc::tma_load_4d(a + a_blk, &p.mapDY[ql], &full[stage], co_blk * 128 + 64, ow0, oh0, n);
+                if (hi) tc::tma_load_4d(a + a_blk, &p.mapDY[ql], &full[stage], co_blk * 128 + 64, ow0, oh0, n);
                 tc::tma_load_4d(sB + (size_t)stage * b_stage, &p.mapX[ql], &full[stage], ch * 64, ow0 - p.pl[ql],
                                 oh0 - p.pt[ql] + r, n);
                 if (++stage == S) { stage = 0; ph ^= 1; }
@@ -2368,7 +2371,7 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
             const bool cta2 = g.L.cout % 256 == 0 && !getenv("SPLITCNN_NO_CTA2");
             if (cta2) P.ntiles = c.ntiles / 2;
             const int Wp = 8 + g.L.kw - 1;
-            const uint32_t a_stage = 2u * c.BH * c.BNn * 8u * 128u;
+            const uint32_t a_stage = (g.L.cout <= 64 ? 1u : 2u) * c.BH * c.BNn * 8u * 128u;
             const uint32_t b_stage = ((uint32_t)Wp * c.BH * c.BNn * (cta2 ? 64u : 128u) + 1023u) & ~1023u;
             const uint32_t stage_bytes = a_stage + b_stage;
             P.stages = std::min<int>(8, (int)((200u * 1024u) / stage_bytes));

@@ -247,25 +247,41 @@ __global__ void __launch_bounds__(256) pool_bwd_scatter_kernel(LevelDesc Li, Lev
     const int G = Li.Cpad / 8;
     const uint32_t units = (uint32_t)Lo.N * go.hp * go.wp * G;
     const Dec3 d = make_dec3(G, go.wp, go.hp);
-    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < units; u += gridDim.x * blockDim.x) {
-        int cg, ow, oh, n;
-        dec3(u, d, cg, ow, oh, n);
-        const int64_t o = go.off + (((int64_t)n * go.hp + oh) * go.wp + ow) * Lo.Cpad + cg * 8;
-        const uint2 a2 = __ldg(reinterpret_cast<const uint2 *>(A + o));
-        float g[8];
-        load8(dY + o, g);
-        for (int r = 0; r < ly.kh; ++r)
-            for (int c = 0; c < ly.kw; ++c) {
-                const int idx = r * ly.kw + c;
-                float v[8];
+    const uint32_t stride = gridDim.x * blockDim.x;
+    // two units per iteration: both units' dY + argmax loads are in flight before the first store
+    for (uint32_t u0 = blockIdx.x * blockDim.x + threadIdx.x; u0 < units; u0 += 2 * stride) {
+        int64_t o[2];
+        uint2 a2[2];
+        float g[2][8];
+        int oh[2], ow[2], n[2], cg[2];
+        bool ok[2];
 #pragma unroll
-                for (int k = 0; k < 8; ++k) {
-                    const uint32_t b = ((k < 4 ? a2.x : a2.y) >> (8 * (k & 3))) & 0xffu;
-                    v[k] = ((int)(b & 0x7fu) == idx && (!relu_bit || (b & 0x80u))) ? g[k] : 0.f;
-                }
-                const int h = oh * ly.sh + r, w = ow * ly.sw + c;
-                store8(dX + gi.off + (((int64_t)n * gi.hp + h) * gi.wp + w) * Li.Cpad + cg * 8, v);
+        for (int k = 0; k < 2; ++k) {
+            const uint32_t u = u0 + k * stride;
+            ok[k] = u < units;
+            dec3(ok[k] ? u : u0, d, cg[k], ow[k], oh[k], n[k]);
+            o[k] = go.off + (((int64_t)n[k] * go.hp + oh[k]) * go.wp + ow[k]) * Lo.Cpad + cg[k] * 8;
+            if (ok[k]) {
+                a2[k] = __ldg(reinterpret_cast<const uint2 *>(A + o[k]));
+                load8(dY + o[k], g[k]);
             }
+        }
+#pragma unroll
+        for (int k = 0; k < 2; ++k) {
+            if (!ok[k]) continue;
+            for (int r = 0; r < ly.kh; ++r)
+                for (int c = 0; c < ly.kw; ++c) {
+                    const int idx = r * ly.kw + c;
+                    float v[8];
+#pragma unroll
+                    for (int e = 0; e < 8; ++e) {
+                        const uint32_t b = ((e < 4 ? a2[k].x : a2[k].y) >> (8 * (e & 3))) & 0xffu;
+                        v[e] = ((int)(b & 0x7fu) == idx && (!relu_bit || (b & 0x80u))) ? g[k][e] : 0.f;
+                    }
+                    const int h = oh[k] * ly.sh + r, w = ow[k] * ly.sw + c;
+                    store8(dX + gi.off + (((int64_t)n[k] * gi.hp + h) * gi.wp + w) * Li.Cpad + cg[k] * 8, v);
+                }
+        }
     }
 }
 

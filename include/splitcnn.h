@@ -265,6 +265,39 @@ SPLITCNN_API splitcnn_status_t splitcnn_add(splitcnn_plan_t plan, int32_t level,
                                 const void *a, const void *b, void *y, const void *mask, uint32_t flags,
                                 int32_t p0, int32_t p1, splitcnn_stream_t stream);
 
+/* ------------------------------------------------------------------ batch normalisation */
+/* Whole-tensor BN on a split level.  BN is not a window operator, so
+ * Split-CNN keeps it unsplit: its statistics are those of the LOGICAL tensor over all patches,
+ * images and pixels (= unsplit training-mode BN), assembled from per-patch partial sums.  Every call
+ * acts on the contiguous span of patches [p0, p1) of `level`; under patch sharding each rank passes
+ * its span and the caller sums the [2][C] partial sums across ranks (a 2C-float allreduce) before
+ * bn_fwd / bn_bwd.  fp32 partials per block, one fixed-order fp64 sum per channel: bitwise
+ * reproducible.  ws: scratch of splitcnn_bn_workspace_size bytes (caller-owned).
+ *   bn_stats      sums[0][c] = sum x, sums[1][c] = sum x^2
+ *   bn_fwd        mean = sums0/count, var = sums1/count - mean^2 (biased), mean_invstd[0][c] = mean,
+ *                 mean_invstd[1][c] = 1/sqrt(var + eps); y = gamma*(x-mean)*invstd + beta (FLAG_RELU:
+ *                 then max(., 0)); y may alias x.  count = N*H*W of the logical tensor.
+ *   bn_bwd_sums   g = dy*[y > 0] (y = the ReLU output; NULL: g = dy), xhat = (x-mean)*invstd;
+ *                 t[0][c] = sum g (= dbeta), t[1][c] = sum g*xhat (= dgamma)
+ *   bn_bwd        dx = gamma*invstd*(g - t0/count - xhat*t1/count); dx may alias dy.
+ * Channel padding (c >= C) of y / dx is written as zero.  Errors: null pointers, Cpad > 2048. */
+SPLITCNN_API splitcnn_status_t splitcnn_bn_workspace_size(splitcnn_plan_t plan, int32_t level, size_t *bytes);
+SPLITCNN_API splitcnn_status_t splitcnn_bn_stats(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                     const void *x, float *sums, void *ws, size_t ws_bytes,
+                                     int32_t p0, int32_t p1, splitcnn_stream_t stream);
+SPLITCNN_API splitcnn_status_t splitcnn_bn_fwd(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                   const void *x, const float *sums, double count, const float *gamma,
+                                   const float *beta, float eps, float *mean_invstd, void *y, uint32_t flags,
+                                   int32_t p0, int32_t p1, splitcnn_stream_t stream);
+SPLITCNN_API splitcnn_status_t splitcnn_bn_bwd_sums(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                        const void *dy, const void *x, const void *y, const float *mean_invstd,
+                                        float *t, void *ws, size_t ws_bytes, int32_t p0, int32_t p1,
+                                        splitcnn_stream_t stream);
+SPLITCNN_API splitcnn_status_t splitcnn_bn_bwd(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                   const void *dy, const void *x, const void *y, const float *mean_invstd,
+                                   const float *gamma, const float *t, double count, void *dx,
+                                   int32_t p0, int32_t p1, splitcnn_stream_t stream);
+
 /* ------------------------------------------------------------------ offload / prefetch */
 /* Patch-granular activation offload (HMMS): after `ready` (recorded by the caller
  * on the compute stream after the buffer's last write, moment 1) copy patch `patch` of level

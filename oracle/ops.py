@@ -189,6 +189,41 @@ def residual_add(Ap, Bp, relu=False):
     return [[np.maximum(y, 0.0) for y in row] for row in out] if relu else out
 
 
+def batch_norm(Xp, gamma, beta, eps=1e-5, relu=False):
+    """Whole-tensor BN on a split level (R11; BN is not a window op, so Split-CNN keeps it
+    unsplit): per-channel mean and biased variance over the LOGICAL tensor (all patches, images and
+    pixels), y = gamma*(x-mean)/sqrt(var+eps) + beta, then ReLU.  Returns (Yp, mean, invstd)."""
+    X = merge(Xp)
+    mean = X.mean(axis=(0, 2, 3))
+    var = ((X - mean[None, :, None, None]) ** 2).mean(axis=(0, 2, 3))
+    invstd = 1.0 / np.sqrt(var + eps)
+    Y = (X - mean[None, :, None, None]) * (gamma * invstd)[None, :, None, None] + beta[None, :, None, None]
+    if relu:
+        Y = np.maximum(Y, 0.0)
+    return _resplit(Y, Xp), mean, invstd
+
+
+def batch_norm_bwd(dYp, Xp, Yp, gamma, mean, invstd, relu=False):
+    """Adjoint of batch_norm (training mode): with g = dY*[Y>0] (ReLU) and xhat = (x-mean)*invstd,
+    dgamma = sum g*xhat, dbeta = sum g, dX = gamma*invstd*(g - mean(g) - xhat*mean(g*xhat))."""
+    dY, X = merge(dYp), merge(Xp)
+    g = np.where(merge(Yp) > 0, dY, 0.0) if relu else dY
+    xh = (X - mean[None, :, None, None]) * invstd[None, :, None, None]
+    M = X.shape[0] * X.shape[2] * X.shape[3]
+    dbeta = g.sum(axis=(0, 2, 3))
+    dgamma = (g * xh).sum(axis=(0, 2, 3))
+    dX = (gamma * invstd)[None, :, None, None] * (g - dbeta[None, :, None, None] / M
+                                                 - xh * dgamma[None, :, None, None] / M)
+    return _resplit(dX, Xp), dgamma, dbeta
+
+
+def _resplit(Y, like):
+    """Cut a full tensor along the partition of the patch list ``like`` (layout glue)."""
+    hs = np.cumsum([0] + [row[0].shape[2] for row in like])
+    ws = np.cumsum([0] + [p.shape[3] for p in like[0]])
+    return [[Y[:, :, hs[i]:hs[i + 1], ws[j]:ws[j + 1]] for j in range(len(like[0]))] for i in range(len(like))]
+
+
 def relu_mask(dXp, Mp):
     """ReLU backward: keep the gradient where the ReLU output is > 0."""
     return [[np.where(Mp[i][j] > 0, dXp[i][j], 0.0) for j in range(len(row))]

@@ -318,6 +318,102 @@ extern "C" splitcnn_status_t splitcnn_add(splitcnn_plan_t plan, int32_t level, s
     return check_launch("add");
 }
 
+// ------------------------------------------------------------------ batch normalisation
+namespace {
+splitcnn_status_t bn_span(splitcnn_plan_t plan, int level, splitcnn_dtype_t dtype, int &p0, int &p1, int64_t &o0,
+                          int64_t &n) {
+    if (!plan || level < 0 || level >= (int)plan->levels.size()) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad level");
+    TRY(check_dtype(dtype));
+    TRY(check_range(plan, level, p0, p1));
+    const Level &L = plan->levels[level];
+    if (L.Cpad > 2048) return fail(SPLITCNN_ERR_UNSUPPORTED, "bn: Cpad > 2048");
+    auto off = [&](int p) { return p == L.npatch() ? L.total() : L.offset(p / L.nw(), p % L.nw()); };
+    o0 = off(p0);
+    n = off(p1) - o0;
+    return SPLITCNN_OK;
+}
+const void *at_(const void *p, int64_t o, splitcnn_dtype_t dt) {
+    return p ? (const void *)((const char *)p + o * (dt == SPLITCNN_BF16 ? 2 : 4)) : nullptr;
+}
+}  // namespace
+
+extern "C" splitcnn_status_t splitcnn_bn_workspace_size(splitcnn_plan_t plan, int32_t level, size_t *bytes) {
+    if (!plan || level < 0 || level >= (int)plan->levels.size() || !bytes)
+        return fail(SPLITCNN_ERR_INVALID_VALUE, "bad argument");
+    *bytes = bn_ws_bytes(plan->levels[level].C);
+    return SPLITCNN_OK;
+}
+
+extern "C" splitcnn_status_t splitcnn_bn_stats(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                               const void *x, float *sums, void *ws, size_t ws_bytes, int32_t p0,
+                                               int32_t p1, splitcnn_stream_t stream) {
+    int64_t o0, n;
+    TRY(bn_span(plan, level, dtype, p0, p1, o0, n));
+    if (!x || !sums || !ws) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    NEED_ALIGNED(x, "x");
+    const Level &L = plan->levels[level];
+    if (ws_bytes < bn_ws_bytes(L.C)) return fail(SPLITCNN_ERR_INVALID_VALUE, "bn_stats: workspace too small");
+    if (n == 0) return cudaMemsetAsync(sums, 0, 2 * L.C * sizeof(float), (cudaStream_t)stream) == cudaSuccess
+                           ? SPLITCNN_OK : fail(SPLITCNN_ERR_CUDA, "memset");
+    launch_bn_reduce(dtype, 0, at_(x, o0, dtype), nullptr, nullptr, nullptr, n / L.Cpad, L.Cpad, L.C, (float *)ws, sums,
+                     (cudaStream_t)stream);
+    return check_launch("bn_stats");
+}
+
+extern "C" splitcnn_status_t splitcnn_bn_fwd(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                             const void *x, const float *sums, double count, const float *gamma,
+                                             const float *beta, float eps, float *mean_invstd, void *y,
+                                             uint32_t flags, int32_t p0, int32_t p1, splitcnn_stream_t stream) {
+    int64_t o0, n;
+    TRY(bn_span(plan, level, dtype, p0, p1, o0, n));
+    if (!x || !sums || !gamma || !beta || !mean_invstd || !y) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    if (!(count > 0)) return fail(SPLITCNN_ERR_INVALID_VALUE, "bn_fwd: count must be > 0");
+    NEED_ALIGNED(x, "x");
+    NEED_ALIGNED(y, "y");
+    const Level &L = plan->levels[level];
+    launch_bn_fwd(dtype, at_(x, o0, dtype), sums, count, gamma, beta, eps, mean_invstd, (void *)at_(y, o0, dtype),
+                  (flags & SPLITCNN_FLAG_RELU) ? 1 : 0, n, L.Cpad, L.C, (cudaStream_t)stream);
+    return check_launch("bn_fwd");
+}
+
+extern "C" splitcnn_status_t splitcnn_bn_bwd_sums(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                                  const void *dy, const void *x, const void *y,
+                                                  const float *mean_invstd, float *t, void *ws, size_t ws_bytes,
+                                                  int32_t p0, int32_t p1, splitcnn_stream_t stream) {
+    int64_t o0, n;
+    TRY(bn_span(plan, level, dtype, p0, p1, o0, n));
+    if (!dy || !x || !mean_invstd || !t || !ws) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    NEED_ALIGNED(dy, "dy");
+    NEED_ALIGNED(x, "x");
+    NEED_ALIGNED(y, "y");
+    const Level &L = plan->levels[level];
+    if (ws_bytes < bn_ws_bytes(L.C)) return fail(SPLITCNN_ERR_INVALID_VALUE, "bn_bwd_sums: workspace too small");
+    if (n == 0) return cudaMemsetAsync(t, 0, 2 * L.C * sizeof(float), (cudaStream_t)stream) == cudaSuccess
+                           ? SPLITCNN_OK : fail(SPLITCNN_ERR_CUDA, "memset");
+    launch_bn_reduce(dtype, 1, at_(x, o0, dtype), at_(dy, o0, dtype), at_(y, o0, dtype), mean_invstd, n / L.Cpad,
+                     L.Cpad, L.C, (float *)ws, t, (cudaStream_t)stream);
+    return check_launch("bn_bwd_sums");
+}
+
+extern "C" splitcnn_status_t splitcnn_bn_bwd(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                             const void *dy, const void *x, const void *y, const float *mean_invstd,
+                                             const float *gamma, const float *t, double count, void *dx, int32_t p0,
+                                             int32_t p1, splitcnn_stream_t stream) {
+    int64_t o0, n;
+    TRY(bn_span(plan, level, dtype, p0, p1, o0, n));
+    if (!dy || !x || !mean_invstd || !gamma || !t || !dx) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    if (!(count > 0)) return fail(SPLITCNN_ERR_INVALID_VALUE, "bn_bwd: count must be > 0");
+    NEED_ALIGNED(dy, "dy");
+    NEED_ALIGNED(x, "x");
+    NEED_ALIGNED(y, "y");
+    NEED_ALIGNED(dx, "dx");
+    if (n == 0) return SPLITCNN_OK;
+    const Level &L = plan->levels[level];
+    launch_bn_bwd(dtype, at_(dy, o0, dtype), at_(x, o0, dtype), at_(y, o0, dtype), mean_invstd, gamma, t, count,
+                  (void *)at_(dx, o0, dtype), n, L.Cpad, L.C, (cudaStream_t)stream);
+    return check_launch("bn_bwd");
+}
+
 // ------------------------------------------------------------------ offload / prefetch
 extern "C" splitcnn_status_t splitcnn_patch_bytes(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
                                                   int32_t patch, size_t *offset, size_t *bytes) {

@@ -16,6 +16,17 @@ void launch_pool_bwd(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, cons
 void launch_add(splitcnn_dtype_t dt, const void *a, const void *b, void *y, const void *m, int relu, int64_t n,
                 cudaStream_t st);
 
+// k_bn.cu
+size_t bn_ws_bytes(int C);
+void launch_bn_reduce(splitcnn_dtype_t dt, int mode, const void *x, const void *dy, const void *y, const float *mi,
+                      int64_t P, int Cpad, int C, float *part, float *sums, cudaStream_t st);
+void launch_bn_fwd(splitcnn_dtype_t dt, const void *x, const float *sums, double count, const float *gamma,
+                   const float *beta, float eps, float *mi, void *y, int relu, int64_t n, int Cpad, int C,
+                   cudaStream_t st);
+void launch_bn_bwd(splitcnn_dtype_t dt, const void *dy, const void *x, const void *y, const float *mi,
+                   const float *gamma, const float *t, double count, void *dx, int64_t n, int Cpad, int C,
+                   cudaStream_t st);
+
 // k_conv_simt.cu
 void launch_conv_fwd_simt(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *x,
                           const void *w, const float *bias, void *y, int relu, int p0, int p1, cudaStream_t st);

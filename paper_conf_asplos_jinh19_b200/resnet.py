@@ -317,3 +317,241 @@ class ResSplitNet(SplitNet):
 
     def output_numel(self) -> int:
         return self.out.numel()
+
+
+class ResBNSplitNet(ResSplitNet):
+    """ResNet-18 split stack WITH batch normalisation: every conv (stem, the
+    two of each block, the downsample) is conv (no bias) -> whole-tensor BN -> (ReLU), i.e.
+        h = ReLU(BN_a(conv_a(x))),  y = ReLU(BN_b(conv_b(h)) + shortcut(x)),  shortcut = x | BN_ds(ds(x)).
+    BN statistics are over the logical tensor (all patches) via splitcnn_bn_stats / _bn_fwd; conv
+    outputs z are kept (BN backward needs them), BN(+ReLU) outputs live in separate level buffers.
+    One GPU (no stats allreduce here; under patch sharding the [2][C] sums would be all-reduced)."""
+
+    def __init__(self, *a, eps: float = 1e-5, **kw):
+        self.eps = eps
+        super().__init__(*a, **kw)
+
+    def _bn_keys(self):
+        keys = [("r", m) for m, l in enumerate(self.region_layers) if l["op"] == "conv"]
+        return keys + [("ds", k) for k in sorted(self.ds_plans)]
+
+    def _bn_level(self, key):
+        """(plan, level index, logical count) of the conv output that BN `key` normalises."""
+        if key[0] == "r":
+            P, lv = self.region, key[1] + 1
+        else:
+            P, lv = self.ds_plans[key[1]], 1
+        L = P.levels[lv]
+        return P, lv, float(L["N"] * L["H"] * L["W"])
+
+    def _alloc(self, grad_buffer=None):
+        super()._alloc(grad_buffer)
+        dev, td = self.device, self.tdtype
+        R = self.region
+        # post-BN activations of every region conv output level (the conv output z stays in act_r)
+        self.bn_out = {m + 1: torch.zeros(R.level_elems(m + 1), dtype=td, device=dev)
+                       for m, l in enumerate(self.region_layers) if l["op"] == "conv"}
+        self.ds_bn = {k: torch.zeros_like(v) for k, v in self.ds_out.items()}
+        self.bn_sums, self.bn_mi, self.bn_gamma, self.bn_beta = {}, {}, {}, {}
+        ws = 0
+        for key in self._bn_keys():
+            P, lv, _ = self._bn_level(key)
+            C = P.levels[lv]["C"]
+            self.bn_sums[key] = torch.zeros(2 * C, dtype=torch.float32, device=dev)
+            self.bn_mi[key] = torch.zeros(2 * C, dtype=torch.float32, device=dev)
+            self.bn_gamma[key] = torch.ones(C, dtype=torch.float32, device=dev)
+            self.bn_beta[key] = torch.zeros(C, dtype=torch.float32, device=dev)
+            ws = max(ws, sc.splitcnn_bn_workspace_size(P.handle, lv))
+        self.bn_ws = torch.zeros(ws // 4 + 4, dtype=torch.float32, device=dev)
+        self.bn_ws_bytes = self.bn_ws.numel() * 4
+
+    def grad_numel(self) -> int:
+        n = super().grad_numel()
+        for key in self._bn_keys():
+            P, lv, _ = self._bn_level(key)
+            n += 2 * P.levels[lv]["C"]
+        return n
+
+    def bind_grads(self, flat: torch.Tensor):
+        super().bind_grads(flat)
+        off = super().grad_numel()
+        self.bn_grads = {}
+        for key in self._bn_keys():
+            P, lv, _ = self._bn_level(key)
+            C = P.levels[lv]["C"]
+            self.bn_grads[key] = flat[off:off + 2 * C]     # [dbeta; dgamma] = the bn_bwd_sums layout
+            off += 2 * C
+
+    def set_bn_params(self, bn_params):
+        """bn_params: (gamma, beta) per conv in _bn_keys() order (chain convs, then downsamples)."""
+        for key, (gm, bt) in zip(self._bn_keys(), bn_params):
+            self.bn_gamma[key].copy_(torch.as_tensor(gm, dtype=torch.float32))
+            self.bn_beta[key].copy_(torch.as_tensor(bt, dtype=torch.float32))
+
+    def _inp(self, m):
+        """The tensor layer m reads: the BN(+ReLU) output for a conv output level, else the level itself."""
+        return self.bn_out.get(m, self.act_r[m]) if m > 0 else self.act_r[0]
+
+    # ------------------------------------------------------------------ BN helpers
+    def _bn_fwd(self, key, z, y, relu, stream):
+        P, lv, cnt = self._bn_level(key)
+        p0, p1 = self.patch_range if key[0] == "r" else (0, P.npatch)
+        nb = z.numel() * z.element_size()
+        self._call("bn", nb, sc.splitcnn_bn_stats, P.handle, lv, self.dtype, z, self.bn_sums[key], self.bn_ws,
+                   self.bn_ws_bytes, p0, p1, stream)
+        self._call("bn", 2 * nb, sc.splitcnn_bn_fwd, P.handle, lv, self.dtype, z, self.bn_sums[key], cnt,
+                   self.bn_gamma[key], self.bn_beta[key], self.eps, self.bn_mi[key], y,
+                   sc.FLAG_RELU if relu else 0, p0, p1, stream)
+
+    def _bn_bwd(self, key, g, z, y_mask, out, stream):
+        """out = dL/dz from g = dL/d(BN output) (y_mask: the BN+ReLU output, or None)."""
+        P, lv, cnt = self._bn_level(key)
+        p0, p1 = self.patch_range if key[0] == "r" else (0, P.npatch)
+        nb = z.numel() * z.element_size()
+        t = self.bn_grads[key]
+        self._call("bn", (3 if y_mask is not None else 2) * nb, sc.splitcnn_bn_bwd_sums, P.handle, lv, self.dtype, g,
+                   z, y_mask, self.bn_mi[key], t, self.bn_ws, self.bn_ws_bytes, p0, p1, stream)
+        self._call("bn", (4 if y_mask is not None else 3) * nb, sc.splitcnn_bn_bwd, P.handle, lv, self.dtype, g, z,
+                   y_mask, self.bn_mi[key], self.bn_gamma[key], t, cnt, out, p0, p1, stream)
+
+    # ------------------------------------------------------------------ passes
+    def forward(self, x: torch.Tensor, stream=None, x_layout: int = sc.NCHW):
+        p0, p1 = self.patch_range
+        R, dt, fl = self.region.handle, self.dtype, self.flags_extra
+        acts, L = self.act_r, self.region_layers
+        self._label = "input"
+        self._call("split", 2 * self._bytes(self.region, 0)[0], sc.splitcnn_split, R, 0, dt, x,
+                   sc.NCHW_S2D if self.s2d else x_layout, acts[0], p0, p1, stream)
+
+        def conv(m, relu):
+            W, _ = self.params[("r", m)]
+            self._label = L[m]["name"]
+            self._call("conv_fwd", self._conv_work(self.region, m, L[m]), sc.splitcnn_conv_fwd, R, m, dt, self._inp(m),
+                       W, None, acts[m + 1], fl, p0, p1, stream)
+            self._bn_fwd(("r", m), acts[m + 1], self.bn_out[m + 1], relu, stream)
+
+        m = 0
+        while m < len(L):
+            if m in self.block_at:
+                k = self.block_at[m]
+                conv(m, True)
+                conv(m + 1, False)
+                if k in self.ds_plans:
+                    P, lds = self.ds_plans[k], self.blocks[k]["ds"]
+                    W, _ = self._ds_params[k]
+                    self._label = lds["name"]
+                    self._call("conv_fwd", self._conv_work(P, 0, lds), sc.splitcnn_conv_fwd, P.handle, 0, dt,
+                               self._inp(m), W, None, self.ds_out[k], fl, 0, P.npatch, stream)
+                    self._bn_fwd(("ds", k), self.ds_out[k], self.ds_bn[k], False, stream)
+                    s = self.ds_bn[k]
+                else:
+                    s = self._inp(m)
+                self._label = f"{L[m]['name'][:-2]}_add"
+                y = self.bn_out[m + 2]
+                self._call("add", 3 * y.numel() * y.element_size(), sc.splitcnn_add, R, m + 2, dt, y, s, y, None,
+                           sc.FLAG_RELU, p0, p1, stream)
+                m += 2
+                continue
+            if L[m]["op"] == "conv":
+                conv(m, True)
+            else:
+                self._label = L[m]["name"]
+                bi, bo = self._bytes(self.region, m)
+                self._call("pool_fwd", bi + bo + bo // (2 if dt == sc.BF16 else 4), sc.splitcnn_pool_fwd, R, m, dt,
+                           self._inp(m), acts[m + 1], self.argmax[("r", m)], sc.FLAG_POOL_RELU_MASK, p0, p1, stream)
+            m += 1
+        nl = self.region.nlayers
+        self._label = "output"
+        self._call("merge", 2 * self._bytes(self.region, nl - 1)[1], sc.splitcnn_merge, R, nl, dt, self._inp(nl),
+                   self.out, sc.NHWC, p0, p1, stream)
+        return self.out
+
+    def backward(self, dy: torch.Tensor, stream=None, need_input_grad: bool = False):
+        p0, p1 = self.patch_range
+        R, dt, fl = self.region.handle, self.dtype, self.flags_extra
+        acts, L = self.act_r, self.region_layers
+        nl = self.region.nlayers
+        g = self.grad[0]
+        self._label = "output"
+        self._call("split", 2 * self._bytes(self.region, nl - 1)[1], sc.splitcnn_split, R, nl, dt, dy, sc.NHWC, g,
+                   p0, p1, stream)
+        nb = self._bytes(self.region, nl - 1)[1]
+        self._call("add", 3 * nb, sc.splitcnn_add, R, nl, dt, g, self.zeros, g, self._inp(nl), 0, p0, p1, stream)
+
+        def conv_bwd(m, gz, want_dx):
+            """conv m backward from gz = dL/dz_m: wgrad, and dgrad into a free buffer (unmasked)."""
+            W, _ = self.params[("r", m)]
+            dW, _ = self.grads[("r", m)]
+            wk = self._conv_work(self.region, m, L[m])
+            self._label = L[m]["name"]
+            out = None
+            if want_dx:
+                out = self._free(gz, *busy)
+                self._call("conv_dgrad", wk, sc.splitcnn_conv_bwd_data, R, m, dt, gz, W, out, None, self.ws,
+                           self.ws_bytes, fl, p0, p1, stream)
+            self._call("conv_wgrad", wk, sc.splitcnn_conv_bwd_filter, R, m, dt, self._inp(m), gz, dW, None, 0.0,
+                       self.ws, self.ws_bytes, fl, p0, p1, stream)
+            return out
+
+        busy = []
+        m = nl - 1
+        while m >= 0:
+            a = m - 1
+            if a in self.block_at:
+                k = self.block_at[a]
+                gz = g                                           # dL/d(BN_b out + shortcut), masked
+                busy = [gz]
+                gzb = self._free(gz)
+                self._label = L[a + 1]["name"]
+                self._bn_bwd(("r", a + 1), gz, acts[a + 2], None, gzb, stream)
+                busy = [gz, gzb]
+                gh = conv_bwd(a + 1, gzb, True)                  # dL/dh (h = BN_a+ReLU output), unmasked
+                busy = [gz, gh]
+                gza = gzb                                        # gzb is consumed: reuse its buffer
+                self._label = L[a]["name"]
+                self._bn_bwd(("r", a), gh, acts[a + 1], self.bn_out[a + 1], gza, stream)
+                busy = [gz, gza]
+                gx = conv_bwd(a, gza, True)
+                busy = [gz, gx]
+                if k in self.ds_plans:
+                    P, lds = self.ds_plans[k], self.blocks[k]["ds"]
+                    W, _ = self._ds_params[k]
+                    dW, _ = self.grads[("ds", k)]
+                    gzd = self._free(gz, gx)
+                    self._label = lds["name"]
+                    self._bn_bwd(("ds", k), gz, self.ds_out[k], None, gzd, stream)
+                    gs = self._free(gz, gx, gzd)
+                    wk = self._conv_work(P, 0, lds)
+                    self._call("conv_dgrad", wk, sc.splitcnn_conv_bwd_data, P.handle, 0, dt, gzd, W, gs, None, self.ws,
+                               self.ws_bytes, fl, 0, P.npatch, stream)
+                    self._call("conv_wgrad", wk, sc.splitcnn_conv_bwd_filter, P.handle, 0, dt, self._inp(a), gzd, dW,
+                               None, 0.0, self.ws, self.ws_bytes, fl, 0, P.npatch, stream)
+                else:
+                    gs = gz
+                mask = self._inp(a) if a in self.block_out else None
+                self._label = f"{L[a]['name'][:-2]}_add"
+                nb = self._bytes(self.region, a)[0]
+                self._call("add", (4 if mask is not None else 3) * nb, sc.splitcnn_add, R, a, dt, gx, gs, gx, mask, 0,
+                           p0, p1, stream)
+                g = gx
+                m = a - 1
+                continue
+            l = L[m]
+            busy = [g]
+            if l["op"] == "conv":                                # the stem: g = dL/d(BN+ReLU out), masked
+                gz = self._free(g)
+                self._label = l["name"]
+                self._bn_bwd(("r", m), g, acts[m + 1], None, gz, stream)
+                busy = [gz]
+                last = m == 0 and not need_input_grad
+                out = conv_bwd(m, gz, not last)
+                g = out if out is not None else gz
+            else:
+                out = self._free(g)
+                self._label = l["name"]
+                bi, bo = self._bytes(self.region, m)
+                self._call("pool_bwd", bi + bo + bo // (2 if dt == sc.BF16 else 4), sc.splitcnn_pool_bwd, R, m, dt, g,
+                           self.argmax[("r", m)], out, sc.FLAG_POOL_RELU_MASK, p0, p1, stream)
+                g = out
+            m -= 1
+        return g

@@ -36,6 +36,7 @@ EXPORTED = [
     "splitcnn_split", "splitcnn_merge",
     "splitcnn_conv_fwd", "splitcnn_conv_bwd_data", "splitcnn_conv_bwd_filter",
     "splitcnn_pool_fwd", "splitcnn_pool_bwd", "splitcnn_conv_pool_fwd", "splitcnn_conv_pool_supported", "splitcnn_add",
+    "splitcnn_bn_workspace_size", "splitcnn_bn_stats", "splitcnn_bn_fwd", "splitcnn_bn_bwd_sums", "splitcnn_bn_bwd",
     "splitcnn_offload", "splitcnn_prefetch", "splitcnn_patch_bytes",
     "splitcnn_offload_plan", "splitcnn_prefetch_plan",
 ]
@@ -90,6 +91,11 @@ _sig("splitcnn_conv_bwd_filter", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _
 _sig("splitcnn_pool_fwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
 _sig("splitcnn_pool_bwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
 _sig("splitcnn_conv_pool_fwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
+_sig("splitcnn_bn_workspace_size", [_vp, _i32, ctypes.POINTER(_sz)])
+_sig("splitcnn_bn_stats", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _sz, _i32, _i32, _vp])
+_sig("splitcnn_bn_fwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _f64, _vp, _vp, _f32, _vp, _vp, _u32, _i32, _i32, _vp])
+_sig("splitcnn_bn_bwd_sums", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _vp, _vp, _sz, _i32, _i32, _vp])
+_sig("splitcnn_bn_bwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _vp, _vp, _f64, _vp, _i32, _i32, _vp])
 _sig("splitcnn_add", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
 _sig("splitcnn_conv_pool_supported", [_vp, _i32, ctypes.c_int, _pi32])
 _sig("splitcnn_offload", [_vp, _i32, ctypes.c_int, _i32, _vp, _vp, _vp, _vp, _vp])
@@ -263,6 +269,32 @@ def splitcnn_pool_bwd(plan, layer, dtype, dy, argmax, dx, flags=0, p0=0, p1=-1, 
 def splitcnn_add(plan, level, dtype, a, b, y, mask=None, flags=0, p0=0, p1=-1, stream=None):
     _check(_lib.splitcnn_add(plan, level, dtype, _ptr(a), _ptr(b), _ptr(y), _ptr(mask), flags, p0, p1,
                              _stream(stream)))
+
+
+def splitcnn_bn_workspace_size(plan, level) -> int:
+    out = _sz(0)
+    _check(_lib.splitcnn_bn_workspace_size(plan, level, ctypes.byref(out)))
+    return out.value
+
+
+def splitcnn_bn_stats(plan, level, dtype, x, sums, ws, ws_bytes, p0=0, p1=-1, stream=None):
+    _check(_lib.splitcnn_bn_stats(plan, level, dtype, _ptr(x), _ptr(sums), _ptr(ws), ws_bytes, p0, p1, _stream(stream)))
+
+
+def splitcnn_bn_fwd(plan, level, dtype, x, sums, count, gamma, beta, eps, mean_invstd, y, flags=0, p0=0, p1=-1,
+                    stream=None):
+    _check(_lib.splitcnn_bn_fwd(plan, level, dtype, _ptr(x), _ptr(sums), float(count), _ptr(gamma), _ptr(beta),
+                                float(eps), _ptr(mean_invstd), _ptr(y), flags, p0, p1, _stream(stream)))
+
+
+def splitcnn_bn_bwd_sums(plan, level, dtype, dy, x, y, mean_invstd, t, ws, ws_bytes, p0=0, p1=-1, stream=None):
+    _check(_lib.splitcnn_bn_bwd_sums(plan, level, dtype, _ptr(dy), _ptr(x), _ptr(y), _ptr(mean_invstd), _ptr(t),
+                                     _ptr(ws), ws_bytes, p0, p1, _stream(stream)))
+
+
+def splitcnn_bn_bwd(plan, level, dtype, dy, x, y, mean_invstd, gamma, t, count, dx, p0=0, p1=-1, stream=None):
+    _check(_lib.splitcnn_bn_bwd(plan, level, dtype, _ptr(dy), _ptr(x), _ptr(y), _ptr(mean_invstd), _ptr(gamma),
+                                _ptr(t), float(count), _ptr(dx), p0, p1, _stream(stream)))
 
 
 def splitcnn_conv_pool_fwd(plan, layer, dtype, x, w, bias, y_pool, argmax, flags=FLAG_RELU | FLAG_POOL_RELU_MASK,

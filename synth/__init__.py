@@ -158,6 +158,11 @@ def resnet_params(g: np.random.Generator, chain, blocks, dtype=np.float32):
     return ps
 
 
+def bn_params(g: np.random.Generator, channels, dtype=np.float32):
+    """(gamma, beta) per BN: gamma ~ U[0.5, 1.5), beta ~ U[-0.1, 0.1) (so the affine part is exercised)."""
+    return [(uniform(g, (c,), 0.5, 1.5, dtype), uniform(g, (c,), -0.1, 0.1, dtype)) for c in channels]
+
+
 def layer_params(g: np.random.Generator, layers, dtype=np.float32):
     """(W, b) per conv layer in order, None for pools.  W is OIHW, b is [Cout]."""
     out = []

@@ -187,3 +187,99 @@ def run_resnet(chain, blocks, N, C, H, W, Oh, Ow, params, X, G, round_bf16=False
     dbs = [grads[m][1] for m in sorted(grads)] + [gds[k][1] for k in sorted(gds)]
     assert len(dWs) == nconv + len(ds)
     return out, dWs, dbs
+
+
+def run_resnet_bn(chain, blocks, N, C, H, W, Oh, Ow, params, bn, X, G, round_bf16=False, eps=1e-5):
+    """Oracle composition of the ResNet split stack WITH whole-tensor BN (R11): conv (no bias) -> BN
+    -> ReLU; y = ReLU(BN_b(conv_b(h)) + shortcut), shortcut = x | BN_ds(ds(x)).  ``params`` = (W, _)
+    per conv (biases unused), ``bn`` = (gamma, beta) per conv, both in synth.resnet_params order.
+    Returns (output NCHW, dWs, dgammas, dbetas)."""
+    rp = OP.plan(chain, N, C, H, W, Oh, Ow)
+    conv_ms = [m for m, l in enumerate(chain) if l["op"] == "conv"]
+    prm = {m: params[i][0] for i, m in enumerate(conv_ms)}
+    bnp = {("r", m): bn[i] for i, m in enumerate(conv_ms)}
+    ds, i = {}, len(conv_ms)
+    for k, b in enumerate(blocks):
+        if b["ds"] is not None:
+            lo, li = rp.layers[b["a"] + 1], rp.layers[b["a"]]
+            dp = OP.plan([b["ds"]], N, b["ds"]["cin"], li.H_in, li.W_in, lo.Oh, lo.Ow).layers[0]
+            ds[k] = (dp, params[i][0])
+            bnp[("ds", k)] = bn[i]
+            i += 1
+    at = {b["a"]: k for k, b in enumerate(blocks)}
+    block_out = {b["a"] + 2 for b in blocks}
+    rnd = lambda P: _rnd(P, round_bf16)
+    zero = lambda Wt: np.zeros(Wt.shape[0])
+    st = {}   # key -> (z, y, mean, invstd, relu)
+
+    def cbn(key, Xp, Wt, lp, relu):
+        z = rnd(O.conv_fwd(Xp, Wt, zero(Wt), lp, False))
+        y, mean, inv = O.batch_norm(z, *bnp[key], eps=eps, relu=relu)
+        y = rnd(y)
+        st[key] = (z, y, mean, inv, relu)
+        return y
+
+    inp = {0: rnd(O.split(X, rp.layers[0].Ih, rp.layers[0].Iw))}
+    args = {}
+    m = 0
+    while m < len(chain):
+        l, lp = chain[m], rp.layers[m]
+        if m in at:
+            k = at[m]
+            h = cbn(("r", m), inp[m], prm[m], lp, True)
+            inp[m + 1] = h
+            zb = cbn(("r", m + 1), h, prm[m + 1], rp.layers[m + 1], False)
+            s = cbn(("ds", k), inp[m], ds[k][1], ds[k][0], False) if k in ds else inp[m]
+            inp[m + 2] = rnd(O.residual_add(zb, s, relu=True))
+            m += 2
+            continue
+        if l["op"] == "conv":
+            inp[m + 1] = cbn(("r", m), inp[m], prm[m], lp, True)
+        else:
+            P, args[m] = O.pool_fwd(inp[m], lp)
+            inp[m + 1] = rnd(P)
+        m += 1
+    nl = len(chain)
+    out = O.merge(inp[nl])
+    grads, bgrads = {}, {}
+
+    def bn_bwd(key, g):
+        z, y, mean, inv, relu = st[key]
+        dz, dgm, dbt = O.batch_norm_bwd(g, z, y, bnp[key][0], mean, inv, relu=False)
+        bgrads[key] = (dgm, dbt)
+        return rnd(dz)
+
+    g = rnd(O.relu_mask(O.split(G, rp.layers[-1].Oh, rp.layers[-1].Ow), inp[nl]))
+    m = nl - 1
+    while m >= 0:
+        a = m - 1
+        if a in at:
+            k = at[a]
+            gzb = bn_bwd(("r", a + 1), g)
+            grads[("r", a + 1)] = O.conv_bwd_filter(inp[a + 1], gzb, rp.layers[a + 1])[0]
+            gh = O.conv_bwd_data(gzb, prm[a + 1], rp.layers[a + 1])
+            gh = rnd(O.relu_mask(gh, inp[a + 1]))               # ReLU of BN_a (applied inside BN bwd on the GPU)
+            gza = bn_bwd(("r", a), gh)
+            grads[("r", a)] = O.conv_bwd_filter(inp[a], gza, rp.layers[a])[0]
+            gx = rnd(O.conv_bwd_data(gza, prm[a], rp.layers[a]))
+            if k in ds:
+                dp, Wd = ds[k]
+                gzd = bn_bwd(("ds", k), g)
+                grads[("ds", k)] = O.conv_bwd_filter(inp[a], gzd, dp)[0]
+                gs = rnd(O.conv_bwd_data(gzd, Wd, dp))
+            else:
+                gs = g
+            gsum = O.residual_add(gx, gs)
+            g = rnd(O.relu_mask(gsum, inp[a]) if a in block_out else gsum)
+            m = a - 1
+            continue
+        l, lp = chain[m], rp.layers[m]
+        if l["op"] == "conv":
+            gz = bn_bwd(("r", m), g)
+            grads[("r", m)] = O.conv_bwd_filter(inp[m], gz, lp)[0]
+        else:
+            g = O.pool_bwd(g, args[m], lp)
+            g = rnd(O.relu_mask(g, inp[m]))                     # the stem's BN+ReLU output feeds the pool
+        m -= 1
+    keys = [("r", m) for m in conv_ms] + [("ds", k) for k in sorted(ds)]
+    return out, [grads[k] for k in keys], [bgrads[k][0] for k in keys], [bgrads[k][1] for k in keys]

@@ -1,0 +1,136 @@
+"""Whole-tensor batch normalisation on split levels (R11) through the C ABI, against
+oracle.ops.batch_norm / batch_norm_bwd; and the BN ResNet split stack (ResBNSplitNet) against
+tests/oracle_chain.run_resnet_bn."""
+import numpy as np
+import pytest
+
+import synth
+from oracle import ops as O
+from tests import oracle_chain
+from tests.helpers import normwise, pack_level, unpack_level
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def sc():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import __graft_entry__
+    __graft_entry__.build()
+    from paper_conf_asplos_jinh19_b200 import splitcnn
+    return splitcnn
+
+
+@pytest.mark.parametrize("dtype_name", ["fp32", "bf16"])
+@pytest.mark.parametrize("C", [13, 64])
+def test_bn_ops_parity(sc, dtype_name, C):
+    """stats / fwd(+ReLU) / bwd sums / bwd on a level with uneven 3x2 patches; also sharded halves
+    (p0..q + q..P partial sums add up to the full sums)."""
+    from paper_conf_asplos_jinh19_b200.plan import SplitPlan
+    dtype = sc.FP32 if dtype_name == "fp32" else sc.BF16
+    td = torch.float32 if dtype == sc.FP32 else torch.bfloat16
+    rnd = (lambda a: a.astype(np.float32).astype(np.float64)) if dtype == sc.FP32 else \
+        (lambda a: synth.to_bf16_f32(a.astype(np.float32)).astype(np.float64))
+    N, H, W = 3, 11, 9
+    l = synth.conv(C, C, 1, 1, 0)
+    pl = SplitPlan([l], N, C, H, W, [0, 3, 7, 11], [0, 5, 9])
+    lv = pl.levels[0]
+    g = synth.rng(20 + C)
+    X = rnd(synth.normal(g, (N, C, H, W)) * 1.5 + 0.3)
+    G = rnd(synth.normal(g, (N, C, H, W)))
+    gm = synth.uniform(g, (C,), 0.5, 1.5).astype(np.float64)
+    bt = synth.uniform(g, (C,), -0.1, 0.1).astype(np.float64)
+    Ih, Iw = [0, 3, 7, 11], [0, 5, 9]
+    Xp, Gp = O.split(X, Ih, Iw), O.split(G, Ih, Iw)
+    Yr, mean, inv = O.batch_norm(Xp, gm, bt, relu=True)
+    dXr, dgr, dbr = O.batch_norm_bwd(Gp, Xp, Yr, gm, mean, inv, relu=True)
+
+    dev = lambda a: torch.from_numpy(pack_level(a, lv).astype(np.float32)).to("cuda", td)
+    x, dy = dev(X), dev(G)
+    f32 = lambda a: torch.from_numpy(np.asarray(a, np.float32)).cuda()
+    gamma, beta = f32(gm), f32(bt)
+    ws_b = sc.splitcnn_bn_workspace_size(pl.handle, 0)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    sums = torch.zeros(2 * C, device="cuda")
+    half = torch.zeros(2 * C, device="cuda")
+    sc.splitcnn_bn_stats(pl.handle, 0, dtype, x, sums, ws, ws_b)
+    sc.splitcnn_bn_stats(pl.handle, 0, dtype, x, half, ws, ws_b, 0, 2)
+    rest = torch.zeros(2 * C, device="cuda")
+    sc.splitcnn_bn_stats(pl.handle, 0, dtype, x, rest, ws, ws_b, 2, 6)
+    torch.testing.assert_close(half + rest, sums, rtol=1e-5, atol=1e-3)
+    Xf = O.merge(Xp)
+    ref_s = np.concatenate([Xf.sum(axis=(0, 2, 3)), (Xf ** 2).sum(axis=(0, 2, 3))])
+    assert normwise(sums.double().cpu().numpy(), ref_s) < 1e-5
+    mi = torch.zeros(2 * C, device="cuda")
+    y = torch.full_like(x, 7.0)
+    cnt = float(N * H * W)
+    sc.splitcnn_bn_fwd(pl.handle, 0, dtype, x, sums, cnt, gamma, beta, 1e-5, mi, y, sc.FLAG_RELU)
+    tol = 1e-4 if dtype == sc.FP32 else 2e-2
+    Yg = unpack_level(y.float().cpu().numpy(), lv, keep_pad=True)
+    for i in range(3):
+        for j in range(2):
+            assert normwise(Yg[i][j][:, :C], Yr[i][j]) <= tol
+            assert np.all(Yg[i][j][:, C:] == 0)
+    t = torch.zeros(2 * C, device="cuda")
+    sc.splitcnn_bn_bwd_sums(pl.handle, 0, dtype, dy, x, y, mi, t, ws, ws_b)
+    assert normwise(t[C:].double().cpu().numpy(), dgr) <= tol
+    assert normwise(t[:C].double().cpu().numpy(), dbr) <= tol
+    dx = torch.full_like(x, 7.0)
+    sc.splitcnn_bn_bwd(pl.handle, 0, dtype, dy, x, y, mi, gamma, t, cnt, dx)
+    dXg = unpack_level(dx.float().cpu().numpy(), lv)
+    assert max(normwise(dXg[i][j], dXr[i][j]) for i in range(3) for j in range(2)) <= tol
+
+
+def _run_stack(sc, dtype, N=2, H=64, seed=6):
+    from paper_conf_asplos_jinh19_b200.resnet import ResBNSplitNet
+    chain, blocks = synth.resnet18_blocks(64, 128)
+    net = ResBNSplitNet(chain, blocks, N, 3, H, H, split=(2, 2), dtype=dtype)
+    g = synth.rng(seed)
+    bf = dtype == sc.BF16
+    X = synth.uniform(g, (N, 3, H, H))
+    params = synth.resnet_params(g, chain, blocks)
+    bn = synth.bn_params(g, [W.shape[0] for W, _ in params])
+    if bf:
+        X = synth.to_bf16_f32(X)
+        params = [(synth.to_bf16_f32(Wt), b) for Wt, b in params]
+    net.set_params([(torch.from_numpy(Wt), torch.from_numpy(b)) for Wt, b in params])
+    net.set_bn_params(bn)
+    L = net.region.levels[-1]
+    G = synth.normal(g, (N, L["C"], L["H"], L["W"]))
+    if bf:
+        G = synth.to_bf16_f32(G)
+    x = torch.from_numpy(X).to("cuda", net.tdtype)
+    dy = torch.from_numpy(np.ascontiguousarray(G.transpose(0, 2, 3, 1))).reshape(-1).to("cuda", net.tdtype)
+    out = net.forward(x)
+    net.backward(dy)
+    torch.cuda.synchronize()
+    Oh, Ow = net.boundaries(0)
+    ref_out, dWs, dgs, dbs = oracle_chain.run_resnet_bn(
+        chain, blocks, N, 3, H, H, Oh, Ow, [(W.astype(np.float64), b.astype(np.float64)) for W, b in params],
+        [(gm.astype(np.float64), bt.astype(np.float64)) for gm, bt in bn], X.astype(np.float64), G.astype(np.float64),
+        round_bf16=bf)
+    got = out.float().cpu().numpy().reshape(N, L["H"], L["W"], L["C"]).transpose(0, 3, 1, 2)
+    errs = {"out": normwise(got, ref_out)}
+    for i, key in enumerate(net._bn_keys()):
+        errs[f"dW{i}"] = normwise(net.grad_oihw(key).double().cpu().numpy(), dWs[i])
+        C = len(dgs[i])
+        t = net.bn_grads[key].double().cpu().numpy()
+        errs[f"dgamma{i}"] = normwise(t[C:], dgs[i])
+        errs[f"dbeta{i}"] = normwise(t[:C], dbs[i])
+    return errs
+
+
+def test_resnet_bn_stack_fp32(sc):
+    """The BN ResNet split stack end to end in fp32: output, every dW, dgamma, dbeta within 1e-4."""
+    errs = _run_stack(sc, sc.FP32)
+    assert max(errs.values()) <= 1e-4, errs
+
+
+def test_resnet_bn_stack_bf16(sc):
+    """bf16 (tensor cores, s2d stem): forward output within 2e-2; gradients to the whole-stack
+    regression bound of test_gpu_resnet (ReLU-kink / pool near-tie routing at small K)."""
+    errs = _run_stack(sc, sc.BF16)
+    assert errs["out"] <= 2e-2, errs
+    assert max(errs.values()) <= 1e-1, errs

@@ -327,3 +327,72 @@ def test_resnet_stack_split_patch_independence_and_interior():
     assert np.array_equal(out[:, :, :, 2:], out2[:, :, :, 2:])
     full, _, _ = oracle_chain.run_resnet(chain, blocks, N, 3, H, H, [0, 4], [0, 4], params, X, G)
     assert not np.allclose(full, out)
+
+
+def _torch_resnet_bn(chain, blocks, X, params, bn, eps=1e-5):
+    import torch
+    import torch.nn.functional as F
+    x = torch.tensor(X, requires_grad=True)
+    ws = [torch.tensor(W, requires_grad=True) for W, _ in params]
+    bns = [(torch.tensor(gm, requires_grad=True), torch.tensor(bt, requires_grad=True)) for gm, bt in bn]
+    conv_ms = [m for m, l in enumerate(chain) if l["op"] == "conv"]
+    ci = {m: i for i, m in enumerate(conv_ms)}
+    dsi = {k: len(conv_ms) + i for i, k in enumerate(k for k, b in enumerate(blocks) if b["ds"] is not None)}
+    at = {b["a"]: k for k, b in enumerate(blocks)}
+
+    def cbn(h, l, i, relu):
+        z = F.conv2d(h, ws[i], None, stride=l["sh"], padding=l["ph_b"])
+        y = F.batch_norm(z, None, None, bns[i][0], bns[i][1], training=True, eps=eps)
+        return F.relu(y) if relu else y
+
+    h, m = x, 0
+    while m < len(chain):
+        l = chain[m]
+        if m in at:
+            k = at[m]
+            t = cbn(h, l, ci[m], True)
+            zb = cbn(t, chain[m + 1], ci[m + 1], False)
+            s = cbn(h, blocks[k]["ds"], dsi[k], False) if k in dsi else h
+            h = F.relu(zb + s)
+            m += 2
+            continue
+        h = cbn(h, l, ci[m], True) if l["op"] == "conv" else F.max_pool2d(h, l["kh"], l["sh"], l["ph_b"])
+        m += 1
+    return h, ws, bns
+
+
+def test_resnet_bn_stack_1x1_split_equals_unsplit_torch():
+    """pin-1 for the BN ResNet composition (R11: BN statistics over the logical tensor): a 1x1 split
+    reduces to the unsplit network with training-mode F.batch_norm; forward, every dW, dgamma, dbeta
+    vs torch fp64 autograd."""
+    import torch
+    from tests import oracle_chain
+    chain, blocks = synth.resnet18_blocks(8, 16)
+    g = synth.rng(9)
+    N, H = 2, 32
+    X = synth.uniform(g, (N, 3, H, H)).astype(np.float64)
+    params = [(W.astype(np.float64), b.astype(np.float64)) for W, b in synth.resnet_params(g, chain, blocks)]
+    chans = [W.shape[0] for W, _ in params]
+    bn = [(gm.astype(np.float64), bt.astype(np.float64)) for gm, bt in synth.bn_params(g, chans)]
+    Y, ws, bns = _torch_resnet_bn(chain, blocks, X, params, bn)
+    G = synth.normal(g, tuple(Y.shape)).astype(np.float64)
+    (Y * torch.tensor(G)).sum().backward()
+    out, dWs, dgs, dbs = oracle_chain.run_resnet_bn(chain, blocks, N, 3, H, H, [0, Y.shape[2]], [0, Y.shape[3]],
+                                                    params, bn, X, G)
+    assert np.abs(out - Y.detach().numpy()).max() < 1e-11
+    for w, dW in zip(ws, dWs):
+        assert np.abs(dW - w.grad.numpy()).max() < 1e-9 * max(1.0, np.abs(dW).max())
+    for (gm, bt), dg, db in zip(bns, dgs, dbs):
+        assert np.abs(dg - gm.grad.numpy()).max() < 1e-9 * max(1.0, np.abs(dg).max())
+        assert np.abs(db - bt.grad.numpy()).max() < 1e-9 * max(1.0, np.abs(db).max())
+
+
+def test_batch_norm_split_invariant():
+    """R11: whole-tensor BN on patches equals BN of the merged tensor cut the same way (a split never
+    changes BN, unlike the window ops), for uneven patches."""
+    g = synth.rng(10)
+    X = synth.normal(g, (2, 5, 9, 7)).astype(np.float64)
+    gm, bt = synth.uniform(g, (5,), 0.5, 1.5).astype(np.float64), synth.uniform(g, (5,), -0.1, 0.1).astype(np.float64)
+    P1, _, _ = O.batch_norm(O.split(X, [0, 9], [0, 7]), gm, bt, relu=True)
+    P2, _, _ = O.batch_norm(O.split(X, [0, 2, 9], [0, 4, 5, 7]), gm, bt, relu=True)
+    assert np.array_equal(O.merge(P1), O.merge(P2))

@@ -117,10 +117,11 @@ def run_ours(args):
     dtype = sc.BF16 if args.dtype == "bf16" else sc.FP32
     use_offload = args.offload if args.offload is not None else (args.config == "C4")
     if c.get("resnet"):
-        from paper_conf_asplos_jinh19_b200.resnet import ResSplitNet
+        from paper_conf_asplos_jinh19_b200.resnet import ResBNSplitNet, ResSplitNet
         if world > 1:
             raise SystemExit("C3 runs on one GPU (the ResNet stack is not patch-sharded here)")
-        net = ResSplitNet(c["layers"], c["blocks"], c["N"], 3, c["H"], c["W"], split=c["split"], dtype=dtype)
+        cls = ResBNSplitNet if args.bn else ResSplitNet
+        net = cls(c["layers"], c["blocks"], c["N"], 3, c["H"], c["W"], split=c["split"], dtype=dtype)
         use_offload = False
     elif world > 1:
         from paper_conf_asplos_jinh19_b200.dist import DistSplitNet
@@ -136,6 +137,9 @@ def run_ours(args):
     net.input_grad = args.config == "C1"      # C1 = one layer's fwd + dgrad + wgrad
     params, x_host, gen = make_inputs(c, net.tdtype, "cuda")
     net.set_params([(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params])
+    if getattr(net, "set_bn_params", None) is not None:
+        import synth
+        net.set_bn_params(synth.bn_params(synth.rng(c["seed"] + 100), [W.shape[0] for W, _ in params]))
     x = x_host.cuda()
     out_numel = net.output_numel()
     dy = torch.randn(out_numel, generator=gen).to(net.tdtype).cuda()
@@ -262,7 +266,8 @@ def run_ours(args):
         "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True,
         "scaling": "strong" if world > 1 else "weak", "vs_baseline": None,
         "dtype": args.dtype, "data": "synthetic (seeded PCG64 / torch.Generator; random-init weights)",
-        "config": {"workload": f"{args.config}: {c['desc']}", "global_batch": global_batch,
+        "config": {"workload": f"{args.config}: {c['desc']}" + (" + whole-tensor BN" if args.bn else ""),
+                   "global_batch": global_batch,
                    "image": [c["H"], c["W"]], "split": list(c["split"]), "split_mode": c["mode"],
                    "split_convs": sum(1 for l in c["layers"] if l["op"] == "conv"),
                    "parallelism": f"patch{world}" if world > 1 else "1gpu",
@@ -401,6 +406,7 @@ def main():
     ap.add_argument("--cpu-tiles", type=int, default=12)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--per-layer", action="store_true")
+    ap.add_argument("--bn", action="store_true", help="C3 with whole-tensor BN after every conv (R11, f2)")
     ap.add_argument("--offload", dest="offload", action="store_true", default=None)
     ap.add_argument("--no-offload", dest="offload", action="store_false")
     args = ap.parse_args()

@@ -82,13 +82,17 @@ __global__ void __launch_bounds__(BN_THREADS) bn_reduce_kernel(const T *__restri
     }
 }
 
-// out[k][c] = sum over z ascending of part[z][k][c], accumulated in fp64 (2C columns, one thread each)
+// out[i] = sum over z of part[z][i] (i < 2C) in fp64: one warp per column, lane l sums z = l, l+32, ...
+// in order, then a fixed xor-tree across lanes -- the same order every run (bitwise reproducible)
 __global__ void bn_sum_partials_kernel(const float *__restrict__ part, int Z, int C, float *__restrict__ out) {
-    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    const int i = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    const int lane = threadIdx.x & 31;
     if (i >= 2 * C) return;
     double s = 0.0;
-    for (int z = 0; z < Z; ++z) s += (double)part[(int64_t)z * 2 * C + i];
-    out[i] = (float)s;
+    for (int z = lane; z < Z; z += 32) s += (double)__ldg(part + (int64_t)z * 2 * C + i);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (lane == 0) out[i] = (float)s;
 }
 
 // mean_invstd[0][c] = mean, [1][c] = 1/sqrt(var + eps)  (fp64 arithmetic on the fp32 sums)
@@ -171,7 +175,7 @@ static void bn_reduce_t(int mode, const void *x, const void *dy, const void *y, 
     else
         bn_reduce_kernel<T, 1><<<Z, BN_THREADS, 0, st>>>((const T *)x, (const T *)dy, (const T *)y, mi, P, Cpad, C, R,
                                                          part);
-    bn_sum_partials_kernel<<<(2 * C + 127) / 128, 128, 0, st>>>(part, Z, C, sums);
+    bn_sum_partials_kernel<<<(2 * C + 7) / 8, 256, 0, st>>>(part, Z, C, sums);
     count_launch(2);
 }
 

@@ -184,20 +184,55 @@ def run_ours(args):
                         "cap_gb": round(stats["cap_bytes"] / 1e9, 3),
                         "no_offload_ms_per_step": round(ms_plain, 3),
                         "no_offload_peak_gb": round(peak_plain / 1e9, 2)}
+    use_graph = args.graph if args.graph is not None else (args.config in ("C1", "C2") and world == 1)
+    graph = None
+    if use_graph:
+        # small configs are launch-bound: capture one whole step (every library call enqueues on the
+        # current stream, the db side stream joins back) and replay it; the plan is static (even split)
+        side = torch.cuda.Stream()
+        side.wait_stream(stream)
+        with torch.cuda.stream(side):
+            step()
+        stream.wait_stream(side)
+        torch.cuda.synchronize()
+        graph = torch.cuda.CUDAGraph()
+        l0 = sc.splitcnn_kernel_launches()
+        with torch.cuda.graph(graph):
+            step()
+        launches_per_step = sc.splitcnn_kernel_launches() - l0
+        torch.cuda.synchronize()
+        for _ in range(3):
+            graph.replay()
+        step = graph.replay                   # noqa: F811 (the timed step is the graph replay)
     launches0 = sc.splitcnn_kernel_launches()
     clocks = ClockSampler(local)
     clocks.start()
-    net.timers = []
+    net.timers = None if graph else []
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    flush_l2 = c["H"] < 224          # small working sets: flush L2 between timed steps, time each step
+    if flush_l2:
+        l2buf = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")     # 256 MB > 126 MB L2
+        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     barrier()
     t0.record(stream)
-    for _ in range(args.steps):
+    for i in range(args.steps):
+        if flush_l2:
+            l2buf.zero_()
+            evs[i][0].record(stream)
         step()
+        if flush_l2:
+            evs[i][1].record(stream)
     t1.record(stream)
     barrier()
     clk = clocks.stop()
-    launches = sc.splitcnn_kernel_launches() - launches0
-    ms = t0.elapsed_time(t1)
+    launches = (launches_per_step * args.steps) if graph else sc.splitcnn_kernel_launches() - launches0
+    ms = sum(a.elapsed_time(b) for a, b in evs) if flush_l2 else t0.elapsed_time(t1)
+    if graph:
+        # per-kind breakdown (roofline) from an eager pass with events around every call
+        net.timers = []
+        for _ in range(args.steps):
+            net.step(x, dy)
+        torch.cuda.synchronize()
     if world > 1:
         tt = torch.tensor([ms], device="cuda")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
@@ -236,7 +271,7 @@ def run_ours(args):
     for _ in range(ke):
         x.copy_(xh, non_blocking=True)
         dy.copy_(dyh, non_blocking=True)
-        net.step(x, dy)
+        step()
         for t, h in zip(grads, gh):
             h.copy_(t, non_blocking=True)
     e1.record(stream)
@@ -271,7 +306,9 @@ def run_ours(args):
                    "image": [c["H"], c["W"]], "split": list(c["split"]), "split_mode": c["mode"],
                    "split_convs": sum(1 for l in c["layers"] if l["op"] == "conv"),
                    "parallelism": f"patch{world}" if world > 1 else "1gpu",
-                   "l2": "inputs/activations >> 126 MB L2 (no flush needed)"},
+                   "l2": "inputs/activations >> 126 MB L2 (no flush needed)" if c["H"] >= 224 else
+                         "L2 flushed (256 MB write) before every timed step; each step timed by its own events",
+                   "cuda_graph": bool(graph)},
         "e2e": {"value": round(global_batch / (ms_e2e / 1e3), 2), "unit": UNIT, "h2d_bytes_per_step": h2d,
                 "d2h_bytes_per_step": d2h},
         "gpu_launches": launches,
@@ -406,6 +443,9 @@ def main():
     ap.add_argument("--cpu-tiles", type=int, default=12)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--per-layer", action="store_true")
+    ap.add_argument("--graph", dest="graph", action="store_true", default=None,
+                    help="time CUDA-graph replays of the step (default for C1, C2)")
+    ap.add_argument("--no-graph", dest="graph", action="store_false")
     ap.add_argument("--bn", action="store_true", help="C3 with whole-tensor BN after every conv (R11, f2)")
     ap.add_argument("--offload", dest="offload", action="store_true", default=None)
     ap.add_argument("--no-offload", dest="offload", action="store_false")

@@ -133,7 +133,7 @@ def run_ours(args):
                               omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype)
     else:
         net = SplitNet(c["layers"], c["tail"], c["N"], c.get("C", 3), c["H"], c["W"], split=c["split"], mode=c["mode"],
-                       omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype)
+                       omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype, static_pool=args.static_pool)
     net.input_grad = args.config == "C1"      # C1 = one layer's fwd + dgrad + wgrad
     params, x_host, gen = make_inputs(c, net.tdtype, "cuda")
     net.set_params([(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params])
@@ -326,6 +326,11 @@ def run_ours(args):
     }
     if offload_info is not None:
         line["offload"] = offload_info
+    line["memory"] = {"peak_allocated_gb": round(torch.cuda.max_memory_allocated() / 1e9, 3),
+                      "static_pool": bool(getattr(net, "static_pool", False))}
+    if getattr(net, "static_pool", False):
+        line["memory"]["pool_gb"] = round(net.pool_bytes / 1e9, 3)
+        line["memory"]["tso_sum_gb"] = round(net.pool_naive_bytes / 1e9, 3)
     if args.per_layer:
         line["per_layer"] = {k: {"ms": round(v[0] / args.steps, 4),
                                  "tflops" if ":conv" in k else "gbs": round(v[1] / (v[0] / 1e3) / (1e12 if ":conv" in k else 1e9), 1)}
@@ -446,6 +451,8 @@ def main():
     ap.add_argument("--graph", dest="graph", action="store_true", default=None,
                     help="time CUDA-graph replays of the step (default for C1, C2)")
     ap.add_argument("--no-graph", dest="graph", action="store_false")
+    ap.add_argument("--static-pool", action="store_true",
+                    help="HMMS static memory plan: all activations / gradients in one first-fit arena (f3)")
     ap.add_argument("--bn", action="store_true", help="C3 with whole-tensor BN after every conv (R11, f2)")
     ap.add_argument("--offload", dest="offload", action="store_true", default=None)
     ap.add_argument("--no-offload", dest="offload", action="store_false")

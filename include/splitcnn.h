@@ -334,6 +334,19 @@ SPLITCNN_API splitcnn_status_t splitcnn_offload_plan(int32_t T, const double *op
 SPLITCNN_API splitcnn_status_t splitcnn_prefetch_plan(int32_t T, const double *op_time_bwd_s, const int64_t *need_bytes,
                                          double bw_bytes_per_s, int32_t *prefetch_start);
 
+/* ------------------------------------------------------------------ static memory planning */
+/* HMMS static memory planning (§4.4): first-fit placement of n tensor storage
+ * objects (TSOs) in ONE contiguous pool, walking the serialized op list.  TSO i occupies
+ * ceil(bytes[i] / align) * align bytes from op first_use[i] through op last_use[i] inclusive.  At op
+ * t, TSOs whose last use is < t are released first (free neighbours coalesce), then the TSOs first
+ * used at t are placed, in index order, at the lowest offset of a free hole they fit in; the pool
+ * grows at its end otherwise.  Outputs: offsets[i] (multiples of align; 0 for empty TSOs) and
+ * *pool_bytes = the high-water mark.  Host-only, O(n * holes).  Errors: null pointers, align not a
+ * power of two, negative size, last_use < first_use. */
+SPLITCNN_API splitcnn_status_t splitcnn_memplan(int32_t n, const int64_t *bytes, const int32_t *first_use,
+                                    const int32_t *last_use, int64_t align, int64_t *offsets,
+                                    int64_t *pool_bytes);
+
 #ifdef __cplusplus
 }
 #endif

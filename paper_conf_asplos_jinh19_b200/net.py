@@ -33,7 +33,8 @@ class SplitNet:
     def __init__(self, region: list[dict], tail: list[dict], N: int, C: int, H: int, W: int,
                  split=(2, 2), mode: str = "even", omega: float = 0.2, seed: int = 0,
                  dtype: int = sc.BF16, device="cuda", patch_range=None, force_simt: bool = False,
-                 grad_buffer: torch.Tensor | None = None, input_relu: bool = False, fuse_pool: bool = True):
+                 grad_buffer: torch.Tensor | None = None, input_relu: bool = False, fuse_pool: bool = True,
+                 static_pool: bool = False):
         self.region_layers, self.tail_layers = region, tail
         self.N, self.C, self.H, self.W = N, C, H, W
         self.split, self.mode, self.omega, self.seed = split, mode, omega, seed
@@ -42,6 +43,7 @@ class SplitNet:
         self.input_relu = input_relu   # level 0 is a ReLU output (e.g. a tail fed by a ReLU conv)
         self.fuse_pool = fuse_pool and dtype == sc.BF16 and not force_simt
         self.step_index = 0
+        self.static_pool = static_pool   # HMMS static memory plan: one arena, first-fit offsets
         self.input_grad = False  # step(): also compute dX of the first layer (C1's single-layer pass)
         self.timers = None       # list -> every library call is bracketed by CUDA events (bench.py)
         self._label = ""
@@ -111,20 +113,24 @@ class SplitNet:
                     self.fused.add((key, m))
         skip_r = {m + 1 for k, m in self.fused if k == "r"}
         skip_t = {m + 1 for k, m in self.fused if k == "t"}
-        self.act_r = [torch.zeros(0 if m in skip_r else self.region.level_elems(m), dtype=td, device=dev)
-                      for m in range(self.region.nlayers + 1)]
-        self.act_t = ([torch.zeros(0 if m in skip_t else self.tail.level_elems(m), dtype=td, device=dev)
-                       for m in range(self.tail.nlayers + 1)] if self.tail else [])
-        self.argmax = {}
-        for plan, acts, key in ((self.region, self.act_r, "r"), (self.tail, self.act_t, "t")):
-            if plan is None:
-                continue
-            for m, l in enumerate(plan.layers):
-                if l["op"] == "maxpool":
-                    self.argmax[(key, m)] = torch.zeros(plan.level_elems(m + 1), dtype=torch.uint8, device=dev)
-        maxg = max([self.region.level_elems(m) for m in range(self.region.nlayers + 1)] +
-                   ([self.tail.level_elems(m) for m in range(self.tail.nlayers + 1)] if self.tail else []))
-        self.grad = [torch.zeros(maxg, dtype=td, device=dev), torch.zeros(maxg, dtype=td, device=dev)]
+        if self.static_pool:
+            self._alloc_static()      # activations, argmax bytes and gradients: views of one planned arena
+        else:
+            self.act_r = [torch.zeros(0 if m in skip_r else self.region.level_elems(m), dtype=td, device=dev)
+                          for m in range(self.region.nlayers + 1)]
+            self.act_t = ([torch.zeros(0 if m in skip_t else self.tail.level_elems(m), dtype=td, device=dev)
+                           for m in range(self.tail.nlayers + 1)] if self.tail else [])
+            self.argmax = {}
+            for plan, key in ((self.region, "r"), (self.tail, "t")):
+                if plan is None:
+                    continue
+                for m, l in enumerate(plan.layers):
+                    if l["op"] == "maxpool":
+                        self.argmax[(key, m)] = torch.zeros(plan.level_elems(m + 1), dtype=torch.uint8, device=dev)
+            maxg = max([self.region.level_elems(m) for m in range(self.region.nlayers + 1)] +
+                       ([self.tail.level_elems(m) for m in range(self.tail.nlayers + 1)] if self.tail else []))
+            self.gbuf = None
+            self.grad = [torch.zeros(maxg, dtype=td, device=dev), torch.zeros(maxg, dtype=td, device=dev)]
         ws = 0
         for plan in (self.region, self.tail):
             if plan is None:
@@ -143,6 +149,93 @@ class SplitNet:
                                              torch.zeros(l["cout"], dtype=torch.float32, device=dev))
         self.bind_grads(grad_buffer if grad_buffer is not None else
                         torch.zeros(self.grad_numel(), dtype=torch.float32, device=dev))
+
+    # ------------------------------------------------------------------ HMMS static memory plan
+    def _tso_schedule(self):
+        """Serialized op list of one step (forward ops in topological order, then the backward
+        ops in reverse) as the TSOs each op touches: [(op, [tso names])].  TSOs: ('a', key, m)
+        activation level, ('am', key, m) argmax bytes, ('g', key, m) gradient of level m."""
+        ops = [("split", [("a", "r", 0)])]
+        for key, layers in (("r", self.region_layers), ("t", self.tail_layers)):
+            if key == "t":
+                if not self.tail:
+                    break
+                ops.append(("merge", [("a", "r", len(self.region_layers)), ("a", "t", 0)]))
+            skip = False
+            for m, l in enumerate(layers):
+                if skip:
+                    skip = False
+                    continue
+                if (key, m) in self.fused:
+                    ops.append((f"{key}{m}+pool", [("a", key, m), ("a", key, m + 2), ("am", key, m + 1)]))
+                    skip = True
+                elif l["op"] == "conv":
+                    ops.append((f"{key}{m}", [("a", key, m), ("a", key, m + 1)]))
+                else:
+                    ops.append((f"{key}{m}", [("a", key, m), ("a", key, m + 1), ("am", key, m)]))
+        out_key = ("a", "t", len(self.tail_layers)) if self.tail else ("a", "r", len(self.region_layers))
+        for key, layers in (("t", self.tail_layers), ("r", self.region_layers)):
+            if key == "t" and not self.tail:
+                continue
+            for m in range(len(layers) - 1, -1, -1):
+                top = m == len(layers) - 1 and (key == "t" or not self.tail)
+                gin = [] if top else [("g", key, m + 1)]          # the step's dY is the caller's
+                last = key == "r" and m == 0 and not self.input_grad
+                gout = [] if last else [("g", key, m)]
+                if layers[m]["op"] == "conv":
+                    ops.append((f"{key}{m}'", gin + [("a", key, m)] + gout))
+                else:
+                    ops.append((f"{key}{m}'", gin + [("am", key, m)] + gout))
+            if key == "t":
+                ops.append(("join'", [("g", "t", 0), ("g", "r", len(self.region_layers))]))
+        ops.append(("end", [out_key]))                    # the step's output stays readable
+        return ops
+
+    def _tso_bytes(self, name):
+        kind, key, m = name
+        plan = self.region if key == "r" else self.tail
+        es = 2 if self.dtype == sc.BF16 else 4
+        if kind == "am":
+            return plan.level_elems(m + 1)
+        if kind == "a" and (key, m - 1) in self.fused:
+            return 0                                       # a fused pair's conv output is never stored
+        return plan.level_elems(m) * es
+
+    def _alloc_static(self):
+        """Place every activation, argmax and gradient TSO of the step in ONE device arena with the
+        library's first-fit static planner (splitcnn_memplan): each lives only from the op
+        that first touches it to the op that last does, so backward gradients reuse the space of
+        activations whose last use has passed."""
+        sched = self._tso_schedule()
+        names, first, last = [], {}, {}
+        for t, (_, ts) in enumerate(sched):
+            for n in ts:
+                if n not in first:
+                    first[n] = t
+                    names.append(n)
+                last[n] = t
+        nbytes = [self._tso_bytes(n) for n in names]
+        offs, pool = sc.splitcnn_memplan(nbytes, [first[n] for n in names], [last[n] for n in names], 1024)
+        self.arena = torch.empty(max(pool, 1024), dtype=torch.uint8, device=self.device)
+        self.pool_bytes = pool
+        self.pool_naive_bytes = sum(nbytes)
+        td = self.tdtype
+        views = {}
+        for n, o, b in zip(names, offs, nbytes):
+            v = self.arena[o:o + b]
+            views[n] = v if n[0] == "am" else v.view(td)
+        empty = torch.zeros(0, dtype=td, device=self.device)
+        self.act_r = [views.get(("a", "r", m), empty) for m in range(self.region.nlayers + 1)]
+        self.act_t = ([views.get(("a", "t", m), empty) for m in range(self.tail.nlayers + 1)] if self.tail else [])
+        self.argmax = {(n[1], n[2]): v for n, v in views.items() if n[0] == "am"}
+        self.gbuf = {(n[1], n[2]): v for n, v in views.items() if n[0] == "g"}
+        self.grad = None
+
+    def _gout(self, key, m, g):
+        """Buffer for the gradient of level m: its planned TSO, or the ping-pong buffer g is not."""
+        if self.gbuf is not None:
+            return self.gbuf[(key, m)]
+        return self.grad[0] if g is not self.grad[0] else self.grad[1]
 
     def bind_grads(self, flat: torch.Tensor):
         """All weight / bias gradients become views of one flat fp32 buffer (one allreduce per step)."""
@@ -266,7 +359,7 @@ class SplitNet:
         g = dy
         if self.tail:
             g = self._run_bwd("t", self.tail, self.tail_layers, self.act_t, g, 0, 1, stream, True)
-            gi = self.grad[0] if g is not self.grad[0] else self.grad[1]
+            gi = self._gout("r", self.region.nlayers, g)
             b_j = 2 * self._bytes(self.region, self.region.nlayers - 1)[1]
             self._call("split", b_j, sc.splitcnn_split, self.region.handle, self.region.nlayers, self.dtype, g,
                        sc.NHWC, gi, p0, p1, stream)
@@ -278,8 +371,8 @@ class SplitNet:
             l = layers[m]
             self._label = l.get("name", f"{key}{m}")
             self.hook_before_bwd(key, m)
-            out = self.grad[0] if g is not self.grad[0] else self.grad[1]
-            last = (m == 0 and not need_input_grad)
+            last = (m == 0 and not need_input_grad) and key == "r"
+            out = None if (last and self.gbuf is not None) else self._gout(key, m, g)
             if l["op"] == "conv":
                 W, _ = self.params[(key, m)]
                 dW, db = self.grads[(key, m)]

@@ -38,7 +38,7 @@ EXPORTED = [
     "splitcnn_pool_fwd", "splitcnn_pool_bwd", "splitcnn_conv_pool_fwd", "splitcnn_conv_pool_supported", "splitcnn_add",
     "splitcnn_bn_workspace_size", "splitcnn_bn_stats", "splitcnn_bn_fwd", "splitcnn_bn_bwd_sums", "splitcnn_bn_bwd",
     "splitcnn_offload", "splitcnn_prefetch", "splitcnn_patch_bytes",
-    "splitcnn_offload_plan", "splitcnn_prefetch_plan",
+    "splitcnn_offload_plan", "splitcnn_prefetch_plan", "splitcnn_memplan",
 ]
 
 
@@ -102,6 +102,7 @@ _sig("splitcnn_offload", [_vp, _i32, ctypes.c_int, _i32, _vp, _vp, _vp, _vp, _vp
 _sig("splitcnn_prefetch", [_vp, _i32, ctypes.c_int, _i32, _vp, _vp, _vp, _vp, _vp])
 _sig("splitcnn_patch_bytes", [_vp, _i32, ctypes.c_int, _i32, ctypes.POINTER(_sz), ctypes.POINTER(_sz)])
 _sig("splitcnn_offload_plan", [_i32, ctypes.POINTER(_f64), ctypes.POINTER(_i64), _f64, _pi32, _pi32])
+_sig("splitcnn_memplan", [_i32, ctypes.POINTER(_i64), _pi32, _pi32, _i64, ctypes.POINTER(_i64), ctypes.POINTER(_i64)])
 _sig("splitcnn_prefetch_plan", [_i32, ctypes.POINTER(_f64), ctypes.POINTER(_i64), _f64, _pi32])
 
 
@@ -330,3 +331,13 @@ def splitcnn_offload(plan, level, dtype, patch, dev_patches, host_pinned, ready=
 def splitcnn_prefetch(plan, level, dtype, patch, host_pinned, dev_patches, ready=None, mem_stream=None, done=None):
     _check(_lib.splitcnn_prefetch(plan, level, dtype, patch, _ptr(host_pinned), _ptr(dev_patches), _ev(ready),
                                   _stream(mem_stream), _ev(done)))
+
+
+def splitcnn_memplan(nbytes, first_use, last_use, align=256):
+    """HMMS static first-fit plan: returns (offsets, pool_bytes)."""
+    n = len(nbytes)
+    off = (ctypes.c_int64 * max(n, 1))()
+    pool = ctypes.c_int64(0)
+    _check(_lib.splitcnn_memplan(n, _arr(nbytes, ctypes.c_int64), _arr(first_use), _arr(last_use), align, off,
+                                 ctypes.byref(pool)))
+    return [off[i] for i in range(n)], pool.value

@@ -176,3 +176,78 @@ def test_offload_plan_all_fit():
     assert off == [1, 0, 1, 0, 1] and sync == [1, 0, 1, 0, 1]
     off, sync = OO.offload_plan([1.0] * 4, [150, 0, 0, 0], 100.0)
     assert off == [1, 0, 0, 0] and sync == [0, 1, 0, 0]
+
+
+# --------------------------------------------------------------------------- HMMS static memory planning
+def test_memplan_worked_example(sc):
+    """P:287 first fit, worked by hand: A(100B, ops 0-1), B(200B, 0-3), C(50B, 1-2), D(300B, 2-3),
+    align 64 -> A@0, B@128, C@384 (no hole at op 1), A freed before op 2 but D(320) does not fit its
+    128-byte hole -> D@448; pool 768."""
+    off, pool = sc.splitcnn_memplan([100, 200, 50, 300], [0, 0, 1, 2], [1, 3, 2, 3], 64)
+    assert off == [0, 128, 384, 448] and pool == 768
+    from oracle.memplan import first_fit
+    assert first_fit([100, 200, 50, 300], [0, 0, 1, 2], [1, 3, 2, 3], 64) == (off, pool)
+
+
+def test_memplan_reuses_freed_space(sc):
+    """A chain of producer -> consumer tensors (each alive for two ops) needs only two slots."""
+    n = 10
+    off, pool = sc.splitcnn_memplan([1000] * n, list(range(n)), [i + 1 for i in range(n)], 256)
+    assert pool == 2 * 1024
+    assert set(off) == {0, 1024}
+
+
+def test_memplan_matches_oracle_random(sc):
+    """Library planner == oracle first fit on random TSO tables; both satisfy the invariants."""
+    import random
+    from oracle.memplan import check_plan, first_fit
+    rnd = random.Random(5)
+    for _ in range(200):
+        n = rnd.randint(0, 25)
+        T = rnd.randint(1, 30)
+        fu = [rnd.randrange(T) for _ in range(n)]
+        lu = [f + rnd.randrange(T - f) for f in fu]
+        nb = [rnd.choice([0, 1, 100, 256, 1000, 4096, 70000]) for _ in range(n)]
+        al = rnd.choice([1, 16, 256])
+        off, pool = sc.splitcnn_memplan(nb, fu, lu, al)
+        assert (off, pool) == first_fit(nb, fu, lu, al)
+        check_plan(nb, fu, lu, off, pool, al)
+
+
+def test_memplan_errors(sc):
+    with pytest.raises(sc.SplitCNNError):
+        sc.splitcnn_memplan([10], [3], [2], 64)
+    with pytest.raises(sc.SplitCNNError):
+        sc.splitcnn_memplan([10], [0], [0], 48)
+
+
+@pytest.mark.parametrize("cfg", ["C2", "C4", "C5"])
+def test_static_pool_plan_of_a_step(sc, cfg):
+    """f3: the SplitNet step's TSO table (activations, argmax bytes, per-level gradients over the
+    serialized fwd + reverse bwd op list) planned by splitcnn_memplan is a valid plan (oracle
+    invariants: no two live TSOs overlap) and smaller than the non-planned layout (every activation
+    kept + two max-size gradient buffers)."""
+    from oracle.memplan import check_plan
+    from paper_conf_asplos_jinh19_b200.net import SplitNet
+    c = synth.vgg_config(cfg)
+    net = SplitNet(c["layers"], c["tail"], c["N"], 3, c["H"], c["W"], split=c["split"], mode=c["mode"],
+                   seed=c["seed"], device="meta", static_pool=True)
+    sched = net._tso_schedule()
+    names, first, last = [], {}, {}
+    for t, (_, ts) in enumerate(sched):
+        for n in ts:
+            first.setdefault(n, t)
+            names.append(n) if n not in names else None
+            last[n] = t
+    nb = [net._tso_bytes(n) for n in names]
+    off, pool = sc.splitcnn_memplan(nb, [first[n] for n in names], [last[n] for n in names], 1024)
+    assert pool == net.pool_bytes
+    check_plan(nb, [first[n] for n in names], [last[n] for n in names], off, pool, 1024)
+    acts = sum(b for n, b in zip(names, nb) if n[0] in ("a", "am"))
+    maxg = max(b for n, b in zip(names, nb) if n[0] == "g")
+    assert pool < acts + 2 * maxg
+    # gradient TSOs exist only in the backward part of the op list (op names ending in "'")
+    bwd0 = min(t for t, (op, _) in enumerate(sched) if op.endswith("'"))
+    for n in names:
+        if n[0] == "g":
+            assert first[n] >= bwd0

@@ -203,3 +203,35 @@ def test_step_bitwise_reproducible(sc):
             continue
         bad = [i for i, (a, b) in enumerate(zip(cur, ref)) if not torch.equal(a, b)]
         assert not bad, f"non-reproducible buffers (activation levels / grads = last): {bad}"
+
+
+@pytest.mark.parametrize("cfg,N,H", [("C5", 16, 224), ("C2", 8, 32), ("C4", 2, 64)])
+def test_static_pool_step_bitwise(sc, cfg, N, H):
+    """f3 (HMMS static memory planning): the step run with every activation / argmax /
+    gradient buffer placed in one first-fit planned arena gives bitwise the same outputs and
+    gradients as the default executor, in less device memory."""
+    from paper_conf_asplos_jinh19_b200.net import SplitNet
+    c = synth.vgg_config(cfg, N=N)
+    g = synth.rng(c["seed"])
+    params = [p for p in synth.layer_params(g, c["layers"] + c["tail"]) if p is not None]
+    tp = [(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params]
+    x = torch.from_numpy(synth.uniform(g, (N, 3, H, H))).to("cuda", torch.bfloat16)
+    kw = dict(split=c["split"], mode=c["mode"], omega=c.get("omega", 0.2), seed=c["seed"])
+    torch.cuda.synchronize()
+    m0 = torch.cuda.memory_allocated()
+    plain = SplitNet(c["layers"], c["tail"], N, 3, H, H, **kw)
+    m1 = torch.cuda.memory_allocated()
+    stat = SplitNet(c["layers"], c["tail"], N, 3, H, H, static_pool=True, **kw)
+    m2 = torch.cuda.memory_allocated()
+    assert m2 - m1 < m1 - m0, (m1 - m0, m2 - m1)
+    plain.set_params(tp)
+    stat.set_params(tp)
+    dy = torch.randn(plain.output_numel(), generator=torch.Generator().manual_seed(2)).to("cuda", torch.bfloat16)
+    for _ in range(2):
+        plain.step(x, dy)
+        stat.step(x, dy)
+        torch.cuda.synchronize()
+        out_p = plain.act_t[-1] if plain.tail else plain.act_r[-1]
+        out_s = stat.act_t[-1] if stat.tail else stat.act_r[-1]
+        assert torch.equal(out_p, out_s)
+        assert torch.equal(plain.grad_flat, stat.grad_flat)

@@ -125,6 +125,15 @@ def _ptr(t) -> int | None:
     return t.data_ptr()
 
 
+def _f32(t) -> int | None:
+    """float* argument: a torch tensor must be float32 (the C side reads / writes fp32)."""
+    if t is not None and not isinstance(t, int) and getattr(t, "dtype", None) is not None:
+        import torch
+        if t.dtype != torch.float32:
+            raise TypeError(f"expected a float32 tensor, got {t.dtype}")
+    return _ptr(t)
+
+
 def _stream(stream):
     if stream is None:
         import torch
@@ -279,23 +288,23 @@ def splitcnn_bn_workspace_size(plan, level) -> int:
 
 
 def splitcnn_bn_stats(plan, level, dtype, x, sums, ws, ws_bytes, p0=0, p1=-1, stream=None):
-    _check(_lib.splitcnn_bn_stats(plan, level, dtype, _ptr(x), _ptr(sums), _ptr(ws), ws_bytes, p0, p1, _stream(stream)))
+    _check(_lib.splitcnn_bn_stats(plan, level, dtype, _ptr(x), _f32(sums), _ptr(ws), ws_bytes, p0, p1, _stream(stream)))
 
 
 def splitcnn_bn_fwd(plan, level, dtype, x, sums, count, gamma, beta, eps, mean_invstd, y, flags=0, p0=0, p1=-1,
                     stream=None):
-    _check(_lib.splitcnn_bn_fwd(plan, level, dtype, _ptr(x), _ptr(sums), float(count), _ptr(gamma), _ptr(beta),
-                                float(eps), _ptr(mean_invstd), _ptr(y), flags, p0, p1, _stream(stream)))
+    _check(_lib.splitcnn_bn_fwd(plan, level, dtype, _ptr(x), _f32(sums), float(count), _f32(gamma), _f32(beta),
+                                float(eps), _f32(mean_invstd), _ptr(y), flags, p0, p1, _stream(stream)))
 
 
 def splitcnn_bn_bwd_sums(plan, level, dtype, dy, x, y, mean_invstd, t, ws, ws_bytes, p0=0, p1=-1, stream=None):
-    _check(_lib.splitcnn_bn_bwd_sums(plan, level, dtype, _ptr(dy), _ptr(x), _ptr(y), _ptr(mean_invstd), _ptr(t),
+    _check(_lib.splitcnn_bn_bwd_sums(plan, level, dtype, _ptr(dy), _ptr(x), _ptr(y), _f32(mean_invstd), _f32(t),
                                      _ptr(ws), ws_bytes, p0, p1, _stream(stream)))
 
 
 def splitcnn_bn_bwd(plan, level, dtype, dy, x, y, mean_invstd, gamma, t, count, dx, p0=0, p1=-1, stream=None):
-    _check(_lib.splitcnn_bn_bwd(plan, level, dtype, _ptr(dy), _ptr(x), _ptr(y), _ptr(mean_invstd), _ptr(gamma),
-                                _ptr(t), float(count), _ptr(dx), p0, p1, _stream(stream)))
+    _check(_lib.splitcnn_bn_bwd(plan, level, dtype, _ptr(dy), _ptr(x), _ptr(y), _f32(mean_invstd), _f32(gamma),
+                                _f32(t), float(count), _ptr(dx), p0, p1, _stream(stream)))
 
 
 def splitcnn_conv_pool_fwd(plan, layer, dtype, x, w, bias, y_pool, argmax, flags=FLAG_RELU | FLAG_POOL_RELU_MASK,

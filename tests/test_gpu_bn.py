@@ -53,17 +53,17 @@ def test_bn_ops_parity(sc, dtype_name, C):
     gamma, beta = f32(gm), f32(bt)
     ws_b = sc.splitcnn_bn_workspace_size(pl.handle, 0)
     ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
-    sums = torch.zeros(2 * C, device="cuda")
-    half = torch.zeros(2 * C, device="cuda")
+    sums = torch.zeros(2 * C, dtype=torch.float32, device="cuda")
+    half = torch.zeros(2 * C, dtype=torch.float32, device="cuda")
     sc.splitcnn_bn_stats(pl.handle, 0, dtype, x, sums, ws, ws_b)
     sc.splitcnn_bn_stats(pl.handle, 0, dtype, x, half, ws, ws_b, 0, 2)
-    rest = torch.zeros(2 * C, device="cuda")
+    rest = torch.zeros(2 * C, dtype=torch.float32, device="cuda")
     sc.splitcnn_bn_stats(pl.handle, 0, dtype, x, rest, ws, ws_b, 2, 6)
     torch.testing.assert_close(half + rest, sums, rtol=1e-5, atol=1e-3)
     Xf = O.merge(Xp)
     ref_s = np.concatenate([Xf.sum(axis=(0, 2, 3)), (Xf ** 2).sum(axis=(0, 2, 3))])
     assert normwise(sums.double().cpu().numpy(), ref_s) < 1e-5
-    mi = torch.zeros(2 * C, device="cuda")
+    mi = torch.zeros(2 * C, dtype=torch.float32, device="cuda")
     y = torch.full_like(x, 7.0)
     cnt = float(N * H * W)
     sc.splitcnn_bn_fwd(pl.handle, 0, dtype, x, sums, cnt, gamma, beta, 1e-5, mi, y, sc.FLAG_RELU)
@@ -73,7 +73,7 @@ def test_bn_ops_parity(sc, dtype_name, C):
         for j in range(2):
             assert normwise(Yg[i][j][:, :C], Yr[i][j]) <= tol
             assert np.all(Yg[i][j][:, C:] == 0)
-    t = torch.zeros(2 * C, device="cuda")
+    t = torch.zeros(2 * C, dtype=torch.float32, device="cuda")
     sc.splitcnn_bn_bwd_sums(pl.handle, 0, dtype, dy, x, y, mi, t, ws, ws_b)
     assert normwise(t[C:].double().cpu().numpy(), dgr) <= tol
     assert normwise(t[:C].double().cpu().numpy(), dbr) <= tol

@@ -235,3 +235,46 @@ def test_static_pool_step_bitwise(sc, cfg, N, H):
         out_s = stat.act_t[-1] if stat.tail else stat.act_r[-1]
         assert torch.equal(out_p, out_s)
         assert torch.equal(plain.grad_flat, stat.grad_flat)
+
+
+def test_autograd_module_matches_executor(sc):
+    """SplitStack (torch.nn front end): y, every weight / bias gradient bitwise equal to the executor's
+    step; x.grad of a single split conv (C1 shape, fp32) equal to the oracle's data gradient."""
+    from oracle import ops as O
+    from oracle import plan as OP
+    from paper_conf_asplos_jinh19_b200.autograd import SplitStack
+    from paper_conf_asplos_jinh19_b200.net import SplitNet
+    c = synth.vgg_config("C2", N=2)
+    g = synth.rng(1)
+    params = [p for p in synth.layer_params(g, c["layers"] + c["tail"]) if p is not None]
+    tp = [(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params]
+    x = torch.from_numpy(synth.uniform(g, (2, 3, 32, 32))).to("cuda", torch.bfloat16)
+    mod = SplitStack(c["layers"], c["tail"], 2, 3, 32, 32, split=c["split"])
+    mod.set_params(tp)
+    ref = SplitNet(c["layers"], c["tail"], 2, 3, 32, 32, split=c["split"])
+    ref.set_params(tp)
+    y = mod(x)
+    gy = torch.randn(y.shape, generator=torch.Generator().manual_seed(3)).to("cuda", torch.bfloat16)
+    y.backward(gy)
+    ref.step(x, gy)
+    torch.cuda.synchronize()
+    assert torch.equal(y, ref.act_t[-1])
+    for key in mod.keys:
+        assert torch.equal(mod.weight(key).grad.float(), ref.grads[key][0].to(torch.bfloat16).float()), key
+        assert torch.equal(getattr(mod, f"b{mod.keys.index(key)}").grad, ref.grads[key][1]), key
+    # input gradient, C1: one 3x3 16->16 split conv, fp32
+    l = synth.conv(16, 16, relu=False)
+    one = SplitStack([l], [], 2, 16, 32, 32, split=(2, 2), dtype=sc.FP32)
+    g1 = synth.rng(0)
+    X = synth.uniform(g1, (2, 16, 32, 32))
+    Wt, b = synth.layer_params(g1, [l])[0]
+    one.set_params([(torch.from_numpy(Wt), torch.from_numpy(b))])
+    xt = torch.from_numpy(X).cuda().requires_grad_(True)
+    yo = one(xt)
+    G = synth.normal(g1, (2, 16, 32, 32))
+    lv = one.net.region.levels[1]
+    from tests.helpers import pack_level
+    yo.backward(torch.from_numpy(pack_level(G.astype(np.float64), lv).astype(np.float32)).cuda())
+    pl = OP.plan([l], 2, 16, 32, 32, [0, 16, 32], [0, 16, 32]).layers[0]
+    dXr = O.merge(O.conv_bwd_data(O.split(G.astype(np.float64), pl.Oh, pl.Ow), Wt.astype(np.float64), pl))
+    assert normwise(xt.grad.double().cpu().numpy(), dXr) <= 1e-4

@@ -207,7 +207,7 @@ def run_ours(args):
     launches0 = sc.splitcnn_kernel_launches()
     clocks = ClockSampler(local)
     clocks.start()
-    net.timers = None if graph else []
+    net.timers = None             # the timed steps carry no per-call events (breakdown: separate pass below)
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     flush_l2 = c["H"] < 224          # small working sets: flush L2 between timed steps, time each step
     if flush_l2:
@@ -227,12 +227,11 @@ def run_ours(args):
     clk = clocks.stop()
     launches = (launches_per_step * args.steps) if graph else sc.splitcnn_kernel_launches() - launches0
     ms = sum(a.elapsed_time(b) for a, b in evs) if flush_l2 else t0.elapsed_time(t1)
-    if graph:
-        # per-kind breakdown (roofline) from an eager pass with events around every call
-        net.timers = []
-        for _ in range(args.steps):
-            net.step(x, dy)
-        torch.cuda.synchronize()
+    # per-kind breakdown (roofline) from an eager pass with CUDA events around every library call
+    net.timers = []
+    for _ in range(args.steps):
+        net.step(x, dy)
+    barrier()
     if world > 1:
         tt = torch.tensor([ms], device="cuda")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
@@ -256,24 +255,35 @@ def run_ours(args):
         offload_info["degradation_pct"] = round(100 * (ms_step / offload_info["no_offload_ms_per_step"] - 1), 2)
     value = global_batch / (ms_step / 1e3)
 
-    # e2e: the same step through the public API with host buffers: pinned H2D of x and dY every
-    # step, D2H of the step's result (all weight / bias gradients) every step
+    # e2e: the same step through the public API with host buffers: every step copies its inputs (x, dY)
+    # from pinned host memory and reads back its result (all weight / bias gradients) -- through
+    # HostPipeline, which overlaps step i+1's H2D and step i's D2H with compute (double buffers, events)
+    from paper_conf_asplos_jinh19_b200.pipeline import HostPipeline
     xh = x_host.pin_memory()
     dyh = dy.cpu().pin_memory()
-    grads = [net.grad_flat]
-    gh = [torch.empty(t.shape, dtype=t.dtype, pin_memory=True) for t in grads]
+    gh = torch.empty(net.grad_flat.shape, dtype=net.grad_flat.dtype, pin_memory=True)
     h2d = xh.numel() * xh.element_size() + dyh.numel() * dyh.element_size()
-    d2h = sum(t.numel() * t.element_size() for t in grads)
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    d2h = gh.numel() * gh.element_size()
     ke = max(1, min(args.steps, 10))
+    if graph is None:
+        pipe = HostPipeline(net, x, dy.numel())
+        for _ in range(2):
+            pipe.submit(xh, dyh, gh)
+        pipe.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     barrier()
     e0.record(stream)
     for _ in range(ke):
-        x.copy_(xh, non_blocking=True)
-        dy.copy_(dyh, non_blocking=True)
-        step()
-        for t, h in zip(grads, gh):
-            h.copy_(t, non_blocking=True)
+        if graph is None:
+            pipe.submit(xh, dyh, gh)
+        else:       # graph-captured step: its input / output buffers are fixed, copies on the same stream
+            x.copy_(xh, non_blocking=True)
+            dy.copy_(dyh, non_blocking=True)
+            step()
+            gh.copy_(net.grad_flat, non_blocking=True)
+    if graph is None:
+        pipe.d2h.synchronize()
+        stream.wait_stream(pipe.d2h)
     e1.record(stream)
     barrier()
     ms_e2e = e0.elapsed_time(e1) / ke

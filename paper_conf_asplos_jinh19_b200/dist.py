@@ -122,9 +122,7 @@ class DistSplitNet:
                                  input_relu=last["op"] == "conv" and last.get("relu", True))
         self.tdtype = self.region_net.tdtype
         n_rg, n_tl = self.region_net.grad_numel(), self.tail_net.grad_numel()
-        self.grad_flat = torch.zeros(n_rg + n_tl, dtype=torch.float32, device=device)
-        self.region_net.bind_grads(self.grad_flat[:n_rg])
-        self.tail_net.bind_grads(self.grad_flat[n_rg:])
+        self.bind_grads(torch.zeros(n_rg + n_tl, dtype=torch.float32, device=device))
         self._set_join_plan(0)
         self.step_index = 0
 
@@ -136,6 +134,13 @@ class DistSplitNet:
     def timers(self, v):
         self.region_net.timers = v
         self.tail_net.timers = v
+
+    def bind_grads(self, flat: torch.Tensor):
+        """All region + tail weight / bias gradients as views of one flat fp32 buffer (one allreduce)."""
+        n_rg = self.region_net.grad_numel()
+        self.grad_flat = flat
+        self.region_net.bind_grads(flat[:n_rg])
+        self.tail_net.bind_grads(flat[n_rg:])
 
     def _set_join_plan(self, step: int):
         rn = self.region_net

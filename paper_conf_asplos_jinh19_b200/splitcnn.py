@@ -250,7 +250,7 @@ def splitcnn_merge(plan, level, dtype, patches, y, y_layout, p0=0, p1=-1, stream
 
 
 def splitcnn_conv_fwd(plan, layer, dtype, x, w, bias, y, flags=0, p0=0, p1=-1, stream=None):
-    _check(_lib.splitcnn_conv_fwd(plan, layer, dtype, _ptr(x), _ptr(w), _ptr(bias), _ptr(y), flags, p0, p1,
+    _check(_lib.splitcnn_conv_fwd(plan, layer, dtype, _ptr(x), _ptr(w), _f32(bias), _ptr(y), flags, p0, p1,
                                   _stream(stream)))
 
 
@@ -262,7 +262,7 @@ def splitcnn_conv_bwd_data(plan, layer, dtype, dy, w, dx, relu_src=None, ws=None
 
 def splitcnn_conv_bwd_filter(plan, layer, dtype, x, dy, dw, db=None, beta=0.0, ws=None, ws_bytes=0, flags=0, p0=0,
                              p1=-1, stream=None):
-    _check(_lib.splitcnn_conv_bwd_filter(plan, layer, dtype, _ptr(x), _ptr(dy), _ptr(dw), _ptr(db), float(beta),
+    _check(_lib.splitcnn_conv_bwd_filter(plan, layer, dtype, _ptr(x), _ptr(dy), _f32(dw), _f32(db), float(beta),
                                          _ptr(ws), ws_bytes, flags, p0, p1, _stream(stream)))
 
 
@@ -309,7 +309,7 @@ def splitcnn_bn_bwd(plan, level, dtype, dy, x, y, mean_invstd, gamma, t, count, 
 
 def splitcnn_conv_pool_fwd(plan, layer, dtype, x, w, bias, y_pool, argmax, flags=FLAG_RELU | FLAG_POOL_RELU_MASK,
                            p0=0, p1=-1, stream=None):
-    _check(_lib.splitcnn_conv_pool_fwd(plan, layer, dtype, _ptr(x), _ptr(w), _ptr(bias), _ptr(y_pool), _ptr(argmax),
+    _check(_lib.splitcnn_conv_pool_fwd(plan, layer, dtype, _ptr(x), _ptr(w), _f32(bias), _ptr(y_pool), _ptr(argmax),
                                        flags, p0, p1, _stream(stream)))
 
 

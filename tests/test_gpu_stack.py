@@ -278,3 +278,32 @@ def test_autograd_module_matches_executor(sc):
     pl = OP.plan([l], 2, 16, 32, 32, [0, 16, 32], [0, 16, 32]).layers[0]
     dXr = O.merge(O.conv_bwd_data(O.split(G.astype(np.float64), pl.Oh, pl.Ow), Wt.astype(np.float64), pl))
     assert normwise(xt.grad.double().cpu().numpy(), dXr) <= 1e-4
+
+
+def test_host_pipeline_bitwise(sc):
+    """HostPipeline (overlapped H2D of step i+1 / D2H of step i): per-step host gradients equal a plain
+    synchronous loop of copy -> step -> copy back, for three different batches."""
+    from paper_conf_asplos_jinh19_b200.net import SplitNet
+    from paper_conf_asplos_jinh19_b200.pipeline import HostPipeline
+    c = synth.vgg_config("C2", N=4)
+    g = synth.rng(1)
+    params = [p for p in synth.layer_params(g, c["layers"] + c["tail"]) if p is not None]
+    tp = [(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params]
+    a = SplitNet(c["layers"], c["tail"], 4, 3, 32, 32, split=c["split"])
+    b = SplitNet(c["layers"], c["tail"], 4, 3, 32, 32, split=c["split"])
+    a.set_params(tp)
+    b.set_params(tp)
+    xs = [torch.from_numpy(synth.uniform(g, (4, 3, 32, 32))).to(torch.bfloat16).pin_memory() for _ in range(3)]
+    dys = [torch.randn(a.output_numel(), generator=torch.Generator().manual_seed(i)).to(torch.bfloat16).pin_memory()
+           for i in range(3)]
+    ref = []
+    for xh, dyh in zip(xs, dys):
+        a.step(xh.cuda(), dyh.cuda())
+        ref.append(a.grad_flat.cpu())
+    pipe = HostPipeline(b, xs[0].cuda(), a.output_numel())
+    outs = [torch.empty(b.grad_flat.shape, dtype=torch.float32).pin_memory() for _ in range(3)]
+    for xh, dyh, o in zip(xs, dys, outs):
+        pipe.submit(xh, dyh, o)
+    pipe.synchronize()
+    for r, o in zip(ref, outs):
+        assert torch.equal(r, o)

@@ -461,8 +461,9 @@ def main():
     ap.add_argument("--graph", dest="graph", action="store_true", default=None,
                     help="time CUDA-graph replays of the step (default for C1, C2)")
     ap.add_argument("--no-graph", dest="graph", action="store_false")
-    ap.add_argument("--static-pool", action="store_true",
-                    help="HMMS static memory plan: all activations / gradients in one first-fit arena (f3)")
+    ap.add_argument("--static-pool", dest="static_pool", action="store_true", default=True,
+                    help="HMMS static memory plan: all activations / gradients in one first-fit arena (f3; default)")
+    ap.add_argument("--no-static-pool", dest="static_pool", action="store_false")
     ap.add_argument("--bn", action="store_true", help="C3 with whole-tensor BN after every conv (R11, f2)")
     ap.add_argument("--offload", dest="offload", action="store_true", default=None)
     ap.add_argument("--no-offload", dest="offload", action="store_false")

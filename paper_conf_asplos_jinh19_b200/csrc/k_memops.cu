@@ -4,6 +4,7 @@
 //   max-pool forward / backward per patch (Eq. 6 with Op = max-pool)
 // One thread moves 8 channels (16 B in bf16) of one pixel; grid.y enumerates patches.
 #include <algorithm>
+#include <cstdlib>
 
 #include "common.cuh"
 #include "kernels.h"
@@ -285,6 +286,68 @@ __global__ void __launch_bounds__(256) pool_bwd_scatter_kernel(LevelDesc Li, Lev
     }
 }
 
+// Backward for 3x3 / stride-2 windows (ResNet's max-pool, any pads): one thread = a 2x2 block of
+// input pixels (padded rows 2a+1, 2a+2 and columns 2b+1, 2b+2) x 8 channels.  Those four pixels are
+// covered exactly by the windows (a|a+1, b|b+1); the thread loads each of them once (instead of once
+// per covered pixel, 9 loads for 4 pixels in the gather form) and sums in the gather kernel's order
+// (oh ascending, then ow) -> bitwise the same dX.
+template <typename T>
+__global__ void __launch_bounds__(256) pool_bwd_k3s2_kernel(LevelDesc Li, LevelDesc Lo, LayerDesc ly,
+                                                            const T *__restrict__ dY, const uint8_t *__restrict__ A,
+                                                            T *__restrict__ dX, int p0, int relu_bit) {
+    const int q = p0 + blockIdx.y;
+    const PatchGeo gi = patch_geo(Li, q), go = patch_geo(Lo, q);
+    const int pt = ly.pad_h[2 * gi.i], pl = ly.pad_w[2 * gi.j];
+    const int a_lo = floordiv(pt - 1, 2), a_hi = floordiv(gi.hp + pt - 2, 2);
+    const int b_lo = floordiv(pl - 1, 2), b_hi = floordiv(gi.wp + pl - 2, 2);
+    const int na = a_hi - a_lo + 1, nb = b_hi - b_lo + 1;
+    const int G = Li.Cpad / 8;
+    if (na <= 0 || nb <= 0) return;
+    const uint32_t units = (uint32_t)Li.N * na * nb * G;
+    const Dec3 d = make_dec3(G, nb, na);
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < units; u += gridDim.x * blockDim.x) {
+        int cg, bi, ai, n;
+        dec3(u, d, cg, bi, ai, n);
+        const int a = a_lo + ai, b = b_lo + bi;
+        uint2 am[4];
+        float g[4][8];
+        bool in[4];
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {            // t = 2*(oh - a) + (ow - b)
+            const int oh = a + (t >> 1), ow = b + (t & 1);
+            in[t] = oh >= 0 && oh < go.hp && ow >= 0 && ow < go.wp;
+            if (in[t]) {
+                const int64_t o = go.off + (((int64_t)n * go.hp + oh) * go.wp + ow) * Lo.Cpad + cg * 8;
+                am[t] = __ldg(reinterpret_cast<const uint2 *>(A + o));
+                load8(dY + o, g[t]);
+            }
+        }
+#pragma unroll
+        for (int py = 0; py < 2; ++py)
+#pragma unroll
+            for (int px = 0; px < 2; ++px) {
+                const int h = 2 * a + 1 + py - pt, w = 2 * b + 1 + px - pl;
+                if (h < 0 || h >= gi.hp || w < 0 || w >= gi.wp) continue;
+                float acc[8];
+#pragma unroll
+                for (int k = 0; k < 8; ++k) acc[k] = 0.f;
+#pragma unroll
+                for (int t = 0; t < 4; ++t) {
+                    const int dh = t >> 1, dw = t & 1;
+                    if (!in[t] || (dh && !py) || (dw && !px)) continue;   // window (a+dh, b+dw) covers the pixel?
+                    const int idx = (1 + py - 2 * dh) * 3 + (1 + px - 2 * dw);
+#pragma unroll
+                    for (int k = 0; k < 8; ++k) {
+                        const uint32_t bt = ((k < 4 ? am[t].x : am[t].y) >> (8 * (k & 3))) & 0xffu;
+                        const bool hit = (int)(bt & 0x7fu) == idx && (!relu_bit || (bt & 0x80u));
+                        acc[k] += hit ? g[t][k] : 0.f;
+                    }
+                }
+                store8(dX + gi.off + (((int64_t)n * gi.hp + h) * gi.wp + w) * Li.Cpad + cg * 8, acc);
+            }
+    }
+}
+
 template <typename T>
 void launch_pool_fwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, void *y, uint8_t *a,
                        int relu_bit, int p0, int p1, cudaStream_t st) {
@@ -311,6 +374,13 @@ void launch_pool_bwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, con
     }
     npatch_launch = p1 - p0;
     dim3 grid(grid_x_for(max_patch_units(Li, p0, p1, Li.Cpad / 8)), p1 - p0);
+    if (g.L.kh == 3 && g.L.kw == 3 && g.L.sh == 2 && g.L.sw == 2 && !getenv("SPLITCNN_POOL_GATHER")) {
+        dim3 g4((unsigned)std::max(1, (int)grid.x / 4 + 1), p1 - p0);
+        pool_bwd_k3s2_kernel<T><<<g4, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
+                                                    (const T *)dy, a, (T *)dx, p0, relu_bit);
+        count_launch();
+        return;
+    }
     { pool_bwd_kernel<T><<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
                                              (const T *)dy, a, (T *)dx, p0, relu_bit); count_launch(); }
 }

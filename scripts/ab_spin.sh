@@ -1,0 +1,6 @@
+#!/bin/bash
+mkdir -p gpurun_out
+for L in conv1_1 conv1_2 conv2_1 conv4_2; do
+  timeout 120 python scripts/layer_bench.py $L C5 >> gpurun_out/ab_spin.txt 2>&1
+  SPLITCNN_DBG=256 timeout 120 python scripts/layer_bench.py $L C5 | sed 's/^/SPIN /' >> gpurun_out/ab_spin.txt 2>&1
+done

@@ -2082,6 +2082,23 @@ struct WgradCfg {
     int x3d, cbox, nchunk, nblocks, bpt, bpt_pad, ntb, nco_blk, ntiles, total_boxes, nsplit, boxes_per_split;
 };
 
+// Split-K count of a weight-gradient launch: enough splits to occupy the SMs, but not more than pays
+// for the fp32 partials they write and the reduction reads back (2 * Z * |dW| * 4 bytes of HBM):
+// minimise  waves * (boxes per split) * (MMA time per box)  +  partial traffic / HBM bandwidth.
+static int choose_splits(long total_boxes, int ntiles, double box_flops, double dw_elems, int zcap) {
+    const double sm_flops = 8192.0 * 1.8e9, hbm = 6.0e12;
+    int bestZ = 1;
+    double best = -1.0;
+    for (int Z = 1; Z <= zcap; ++Z) {
+        const long bps = (total_boxes + Z - 1) / Z;
+        const long nsplit = (total_boxes + bps - 1) / bps;
+        const long waves = ((long)ntiles * nsplit + num_sms() - 1) / num_sms();
+        const double t = (double)waves * bps * box_flops / sm_flops + 2.0 * nsplit * dw_elems * 4.0 / hbm;
+        if (best < 0 || t < best * 0.98) { best = t; bestZ = Z; }
+    }
+    return bestZ;
+}
+
 WgradCfg wgrad_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, int p0, int p1) {
     WgradCfg c{};
     const int N = Lo.N, s = g.L.sh, KT = g.L.kh * g.L.kw;
@@ -2116,6 +2133,9 @@ WgradCfg wgrad_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, int p0,
     int Z = std::max(1, (2 * num_sms() + c.ntiles - 1) / c.ntiles);
     Z = std::min(Z, std::max(1, c.total_boxes / 4));  // >= 4 boxes per split
     Z = std::min(Z, 128);
+    if (!getenv("SPLITCNN_ZMAX"))
+        Z = choose_splits(c.total_boxes, c.ntiles, 2.0 * 128 * c.bpt_pad * c.cbox * c.ts.BW * c.ts.BH * c.ts.BNn,
+                          (double)g.L.cout * KT * Li.Cpad, Z);
     c.boxes_per_split = (c.total_boxes + Z - 1) / Z;
     c.nsplit = (c.total_boxes + c.boxes_per_split - 1) / c.boxes_per_split;
     return c;
@@ -2155,6 +2175,9 @@ WgHaloCfg wgrad_halo_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, i
     int Z = std::max(1, (2 * num_sms() + c.ntiles - 1) / c.ntiles);
     Z = std::min(Z, std::max(1, c.total_boxes / 4));
     Z = std::min(Z, 128);
+    if (!getenv("SPLITCNN_ZMAX"))
+        Z = choose_splits(c.total_boxes, c.ntiles, 2.0 * 128 * g.L.kw * 64 * c.BH * c.BNn * 8,
+                          (double)g.L.cout * g.L.kh * g.L.kw * Li.Cpad, Z);
     c.boxes_per_split = (c.total_boxes + Z - 1) / Z;
     c.nsplit = (c.total_boxes + c.boxes_per_split - 1) / c.boxes_per_split;
     return c;

@@ -44,7 +44,8 @@ class OffloadSplitNet(SplitNet):
     """SplitNet whose split-region activations are offloaded / prefetched per Algorithm 1."""
 
     def __init__(self, *args, offload: bool = True, **kw):
-        kw.setdefault("fuse_pool", False)   # the planner walks the unfused op list (one op per layer)
+        # fused conv -> pool pairs are ONE forward op of the planner's serialized list (their conv
+        # output level is never materialised); the backward list stays one op per layer
         super().__init__(*args, **kw)
         self.offload_enabled = offload
         L = self.region.nlayers
@@ -59,14 +60,19 @@ class OffloadSplitNet(SplitNet):
         self.stats = {}
 
     # ------------------------------------------------------------------ op indexing
-    def _fwd_ops(self):
+    def _all_ops(self):
         ops = [("r", m) for m in range(len(self.region_layers))]
         if self.tail:
             ops += [("t", m) for m in range(len(self.tail_layers))]
         return ops
 
+    def _fwd_ops(self):
+        """Serialized forward ops: a fused conv -> pool pair (key, m) is one op (its pool half m+1 skipped)."""
+        skip = {(k, m + 1) for k, m in self.fused}
+        return [op for op in self._all_ops() if op not in skip]
+
     def _bwd_ops(self):
-        return list(reversed(self._fwd_ops()))
+        return list(reversed(self._all_ops()))
 
     # ------------------------------------------------------------------ profiling + planning
     def profile_and_plan(self, x, dy, reps: int = 20, bw: float | None = None):
@@ -91,9 +97,9 @@ class OffloadSplitNet(SplitNet):
             d[label] = d.get(label, 0.0) + e0.elapsed_time(e1) / 1e3 / reps
         self.timers = None
         self.offload_enabled = saved
-        names = [(self.region_layers if k == "r" else self.tail_layers)[m].get("name", f"{k}{m}") for k, m in ops]
-        op_t = [fwd_t.get(n, 0.0) for n in names]
-        op_bt = [bwd_t.get(n, 0.0) for n in reversed(names)]
+        nm = lambda k, m: (self.region_layers if k == "r" else self.tail_layers)[m].get("name", f"{k}{m}")
+        op_t = [fwd_t.get(nm(k, m), 0.0) for k, m in ops]
+        op_bt = [bwd_t.get(nm(k, m), 0.0) for k, m in self._bwd_ops()]
         if bw is None:
             d2h, h2d = measure_host_bandwidth()
             bw = min(d2h, h2d)
@@ -145,6 +151,8 @@ class OffloadSplitNet(SplitNet):
     def hook_before_fwd(self, key, m):
         if key == "r":
             self._ensure(m + 1)      # allocate a level right before the op that produces it
+            if (key, m) in self.fused:
+                self._ensure(m + 2)  # a fused pair produces the pool output level
         if not (self.offload_enabled and self.plan_ready) or not self.offload_at.get((key, m)):
             return
         # moment 1: the input level of op m is final -> D2H per patch on an idle memory stream

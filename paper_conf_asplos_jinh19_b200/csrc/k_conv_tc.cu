@@ -1119,7 +1119,18 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
     const int cpad = La.Cpad;
     const int cpadc = std::min(cpad, 64);
     const int ncols_out = mode == 0 ? g.L.cout : g.L.cin;
-    const int BN = std::min(256, round_up16(ncols_out));
+    // N tile: up to 256 output channels; small layers (few 128-pixel M tiles, e.g. 2x2 / 4x4 CIFAR tails)
+    // take narrower N tiles so that M tiles x N tiles still covers the SMs
+    int BN = std::min(256, round_up16(ncols_out));
+    {
+        long mt = 0;
+        for (int q = p0; q < p1; ++q) {
+            const int i = q / Lout.nw(), j = q % Lout.nw();
+            mt += ((long)La.N * out_ext_h(i) * out_ext_w(j) + 127) / 128;
+        }
+        while (BN > 64 && BN % 32 == 0 && mt * ((ncols_out + BN - 1) / BN) < num_sms() && !getenv("SPLITCNN_WIDE_N"))
+            BN /= 2;
+    }
     const int nco = (ncols_out + BN - 1) / BN;
     const int N = La.N;
     for (int g0 = p0; g0 < p1; g0 += TC_MAXP) {

@@ -133,7 +133,8 @@ def run_ours(args):
                               omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype)
     else:
         net = SplitNet(c["layers"], c["tail"], c["N"], c.get("C", 3), c["H"], c["W"], split=c["split"], mode=c["mode"],
-                       omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype, static_pool=args.static_pool)
+                       omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype, static_pool=args.static_pool,
+                       input_grad=args.config == "C1")
     net.input_grad = args.config == "C1"      # C1 = one layer's fwd + dgrad + wgrad
     params, x_host, gen = make_inputs(c, net.tdtype, "cuda")
     net.set_params([(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params])
@@ -265,25 +266,17 @@ def run_ours(args):
     h2d = xh.numel() * xh.element_size() + dyh.numel() * dyh.element_size()
     d2h = gh.numel() * gh.element_size()
     ke = max(1, min(args.steps, 10))
-    if graph is None:
-        pipe = HostPipeline(net, x, dy.numel())
-        for _ in range(2):
-            pipe.submit(xh, dyh, gh)
-        pipe.synchronize()
+    pipe = HostPipeline(net, x, dy.numel(), graphs=graph is not None)
+    for _ in range(3):
+        pipe.submit(xh, dyh, gh)
+    pipe.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     barrier()
     e0.record(stream)
     for _ in range(ke):
-        if graph is None:
-            pipe.submit(xh, dyh, gh)
-        else:       # graph-captured step: its input / output buffers are fixed, copies on the same stream
-            x.copy_(xh, non_blocking=True)
-            dy.copy_(dyh, non_blocking=True)
-            step()
-            gh.copy_(net.grad_flat, non_blocking=True)
-    if graph is None:
-        pipe.d2h.synchronize()
-        stream.wait_stream(pipe.d2h)
+        pipe.submit(xh, dyh, gh)
+    pipe.d2h.synchronize()
+    stream.wait_stream(pipe.d2h)
     e1.record(stream)
     barrier()
     ms_e2e = e0.elapsed_time(e1) / ke

@@ -34,7 +34,7 @@ class SplitNet:
                  split=(2, 2), mode: str = "even", omega: float = 0.2, seed: int = 0,
                  dtype: int = sc.BF16, device="cuda", patch_range=None, force_simt: bool = False,
                  grad_buffer: torch.Tensor | None = None, input_relu: bool = False, fuse_pool: bool = True,
-                 static_pool: bool = False):
+                 static_pool: bool = False, input_grad: bool = False):
         self.region_layers, self.tail_layers = region, tail
         self.N, self.C, self.H, self.W = N, C, H, W
         self.split, self.mode, self.omega, self.seed = split, mode, omega, seed
@@ -44,7 +44,7 @@ class SplitNet:
         self.fuse_pool = fuse_pool and dtype == sc.BF16 and not force_simt
         self.step_index = 0
         self.static_pool = static_pool   # HMMS static memory plan: one arena, first-fit offsets
-        self.input_grad = False  # step(): also compute dX of the first layer (C1's single-layer pass)
+        self.input_grad = input_grad  # step(): also compute dX of the first layer (C1's single-layer pass)
         self.timers = None       # list -> every library call is bracketed by CUDA events (bench.py)
         self._label = ""
         self.region = self._make_region_plan(0)

@@ -18,8 +18,9 @@ import torch
 
 
 class HostPipeline:
-    def __init__(self, net, x_like: torch.Tensor | None = None, dy_numel: int | None = None):
+    def __init__(self, net, x_like: torch.Tensor | None = None, dy_numel: int | None = None, graphs: bool = False):
         self.net = net
+        self.graphs = [None, None] if graphs else None   # one CUDA graph per buffer parity (fixed pointers)
         dev = net.device
         self.compute = torch.cuda.current_stream(dev)
         self.h2d = torch.cuda.Stream(dev)
@@ -47,7 +48,12 @@ class HostPipeline:
         if self.used[b]:
             self.compute.wait_event(self.g_free[b])       # this gradient buffer's D2H has finished
         self.net.bind_grads(self.g[b])
-        self.net.step(self.x[b], self.dy[b], self.compute)
+        if self.graphs is not None:
+            if self.graphs[b] is None:
+                self.graphs[b] = self._capture(b)
+            self.graphs[b].replay()
+        else:
+            self.net.step(self.x[b], self.dy[b], self.compute)
         self.in_free[b].record(self.compute)
         self.g_ready[b].record(self.compute)
         if grads_host is not None:
@@ -60,6 +66,18 @@ class HostPipeline:
         self.used[b] = True
         self.i += 1
         return self.g[b]
+
+    def _capture(self, b):
+        """Capture one step on buffers (x[b], dy[b], g[b]) as a CUDA graph (a static plan: even split)."""
+        side = torch.cuda.Stream(self.net.device)
+        side.wait_stream(self.compute)
+        with torch.cuda.stream(side):
+            self.net.step(self.x[b], self.dy[b])           # warm-up outside the capture
+        self.compute.wait_stream(side)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            self.net.step(self.x[b], self.dy[b])
+        return g
 
     def synchronize(self):
         self.compute.synchronize()

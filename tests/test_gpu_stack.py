@@ -307,3 +307,31 @@ def test_host_pipeline_bitwise(sc):
     pipe.synchronize()
     for r, o in zip(ref, outs):
         assert torch.equal(r, o)
+
+
+def test_host_pipeline_graphs_bitwise(sc):
+    """HostPipeline with one CUDA graph per buffer parity: per-step host gradients equal the eager loop."""
+    from paper_conf_asplos_jinh19_b200.net import SplitNet
+    from paper_conf_asplos_jinh19_b200.pipeline import HostPipeline
+    c = synth.vgg_config("C2", N=4)
+    g = synth.rng(2)
+    params = [p for p in synth.layer_params(g, c["layers"] + c["tail"]) if p is not None]
+    tp = [(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params]
+    a = SplitNet(c["layers"], c["tail"], 4, 3, 32, 32, split=c["split"])
+    b = SplitNet(c["layers"], c["tail"], 4, 3, 32, 32, split=c["split"], static_pool=True)
+    a.set_params(tp)
+    b.set_params(tp)
+    xs = [torch.from_numpy(synth.uniform(g, (4, 3, 32, 32))).to(torch.bfloat16).pin_memory() for _ in range(4)]
+    dys = [torch.randn(a.output_numel(), generator=torch.Generator().manual_seed(i)).to(torch.bfloat16).pin_memory()
+           for i in range(4)]
+    ref = []
+    for xh, dyh in zip(xs, dys):
+        a.step(xh.cuda(), dyh.cuda())
+        ref.append(a.grad_flat.cpu())
+    pipe = HostPipeline(b, xs[0].cuda(), a.output_numel(), graphs=True)
+    outs = [torch.empty(b.grad_flat.shape, dtype=torch.float32).pin_memory() for _ in range(4)]
+    for xh, dyh, o in zip(xs, dys, outs):
+        pipe.submit(xh, dyh, o)
+    pipe.synchronize()
+    for r, o in zip(ref, outs):
+        assert torch.equal(r, o)

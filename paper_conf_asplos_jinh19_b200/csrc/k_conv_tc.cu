@@ -1671,7 +1671,10 @@ __global__ void __launch_bounds__(192, 1) wgrad_tc_kernel(const __grid_constant_
             int stage = 0;
             uint32_t ph = 0;
             int ql = 0;
-            const uint32_t tx = 2u * (uint32_t)p.rows_box * 128u + (uint32_t)nblk * p.rows_box * p.cbox * 2u;
+            // the upper 64-channel dY block is skipped when it is all out of bounds (Cout <= 64): its
+            // shared memory stays zero from the clear above, so its accumulator rows add nothing
+            const int nh = co_blk * 128 + 64 < p.Cout ? 2 : 1;
+            const uint32_t tx = (uint32_t)nh * p.rows_box * 128u + (uint32_t)nblk * p.rows_box * p.cbox * 2u;
             for (int b = b0; b < b1; ++b) {
                 while (b >= p.box_prefix[ql + 1]) ++ql;
                 int idx = b - p.box_prefix[ql];
@@ -1683,7 +1686,7 @@ __global__ void __launch_bounds__(192, 1) wgrad_tc_kernel(const __grid_constant_
                 tc::mbar_arrive_expect_tx(&full[stage], tx);
                 uint8_t *a = sA + (size_t)stage * a_stage;
                 uint8_t *bb = sB + (size_t)stage * b_stage_al;
-                for (int h = 0; h < 2; ++h)
+                for (int h = 0; h < nh; ++h)
                     tc::tma_load_4d(a + h * WG_ROWS * 128, &p.mapDY[ql], &full[stage], co_blk * 128 + h * 64, ow0, oh0, n0);
                 for (int k = 0; k < nblk; ++k) {
                     const int blk = blk0 + k;

@@ -109,7 +109,7 @@ def run_ours(args):
     if args.gpus != world:
         world = max(world, 1)
     torch.cuda.set_device(local)
-    if world > 1:
+    if world > 1 or args.force_dist:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     c = workload(args.config)
     if args.dtype is None:
@@ -123,7 +123,7 @@ def run_ours(args):
         cls = ResBNSplitNet if args.bn else ResSplitNet
         net = cls(c["layers"], c["blocks"], c["N"], 3, c["H"], c["W"], split=c["split"], dtype=dtype)
         use_offload = False
-    elif world > 1:
+    elif world > 1 or args.force_dist:
         from paper_conf_asplos_jinh19_b200.dist import DistSplitNet
         net = DistSplitNet(c, world, rank, dtype)
         use_offload = False
@@ -342,7 +342,7 @@ def run_ours(args):
         line["cpu_baseline"] = cpu_baseline(args.config, budget_tiles=args.cpu_tiles)
     if rank == 0:
         print(json.dumps(line), flush=True)
-    if world > 1:
+    if dist.is_initialized():
         dist.destroy_process_group()
 
 
@@ -457,6 +457,8 @@ def main():
     ap.add_argument("--static-pool", dest="static_pool", action="store_true", default=True,
                     help="HMMS static memory plan: all activations / gradients in one first-fit arena (f3; default)")
     ap.add_argument("--no-static-pool", dest="static_pool", action="store_false")
+    ap.add_argument("--force-dist", action="store_true",
+                    help="run the multi-GPU executor (DistSplitNet, NCCL) even at one rank (exercises the N>1 path)")
     ap.add_argument("--bn", action="store_true", help="C3 with whole-tensor BN after every conv (R11, f2)")
     ap.add_argument("--offload", dest="offload", action="store_true", default=None)
     ap.add_argument("--no-offload", dest="offload", action="store_false")

@@ -101,6 +101,7 @@ def reverse(sends, recvs):
 class DistSplitNet:
     def __init__(self, c: dict, world: int, rank: int, dtype: int = sc.BF16, device="cuda"):
         self.world, self.rank, self.dtype = world, rank, dtype
+        self.device = torch.device(device)
         N, H, W = c["N"], c["H"], c["W"]
         self.N = N
         nb = N // world

@@ -88,6 +88,8 @@ def make_inputs(c, dtype_t, device, world=1, rank=0):
     g = synth.rng(c["seed"])
     if c.get("resnet"):
         params = synth.resnet_params(g, c["layers"], c["blocks"])
+        if c.get("full"):
+            params += synth.resnet_params(g, *synth.resnet18_tail_blocks())
     else:
         params = [p for p in synth.layer_params(g, c["layers"] + c["tail"]) if p is not None]
     gen = torch.Generator(device="cpu").manual_seed(c["seed"])
@@ -112,6 +114,8 @@ def run_ours(args):
     if world > 1 or args.force_dist:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     c = workload(args.config)
+    if getattr(args, "full", False) and c.get("resnet"):
+        c["full"] = True
     if args.dtype is None:
         args.dtype = c.get("dtype", "bf16")
     dtype = sc.BF16 if args.dtype == "bf16" else sc.FP32
@@ -120,8 +124,15 @@ def run_ours(args):
         from paper_conf_asplos_jinh19_b200.resnet import ResBNSplitNet, ResSplitNet
         if world > 1:
             raise SystemExit("C3 runs on one GPU (the ResNet stack is not patch-sharded here)")
-        cls = ResBNSplitNet if args.bn else ResSplitNet
-        net = cls(c["layers"], c["blocks"], c["N"], 3, c["H"], c["W"], split=c["split"], dtype=dtype)
+        if args.full:          # the whole trunk: split region -> unsplit layer3/4 -> global average pool (f2)
+            import synth
+            from paper_conf_asplos_jinh19_b200.resnet import ResNet18Net
+            tc, tb = synth.resnet18_tail_blocks()
+            net = ResNet18Net(c["layers"], c["blocks"], tc, tb, c["N"], 3, c["H"], c["W"], split=c["split"],
+                              bn=args.bn, dtype=dtype)
+        else:
+            cls = ResBNSplitNet if args.bn else ResSplitNet
+            net = cls(c["layers"], c["blocks"], c["N"], 3, c["H"], c["W"], split=c["split"], dtype=dtype)
         use_offload = False
     elif world > 1 or args.force_dist:
         from paper_conf_asplos_jinh19_b200.dist import DistSplitNet
@@ -304,7 +315,8 @@ def run_ours(args):
         "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True,
         "scaling": "strong" if world > 1 else "weak", "vs_baseline": None,
         "dtype": args.dtype, "data": "synthetic (seeded PCG64 / torch.Generator; random-init weights)",
-        "config": {"workload": f"{args.config}: {c['desc']}" + (" + whole-tensor BN" if args.bn else ""),
+        "config": {"workload": f"{args.config}: {c['desc']}" + (" + unsplit layer3/4 + GAP (full trunk)" if c.get("full") else "")
+                               + (" + whole-tensor BN" if args.bn else ""),
                    "global_batch": global_batch,
                    "image": [c["H"], c["W"]], "split": list(c["split"]), "split_mode": c["mode"],
                    "split_convs": sum(1 for l in c["layers"] if l["op"] == "conv"),
@@ -339,7 +351,7 @@ def run_ours(args):
                                  "tflops" if ":conv" in k else "gbs": round(v[1] / (v[0] / 1e3) / (1e12 if ":conv" in k else 1e9), 1)}
                              for k, v in per_layer.items()}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline(args.config, budget_tiles=args.cpu_tiles)
+        line["cpu_baseline"] = cpu_baseline(args.config, budget_tiles=args.cpu_tiles, full=bool(c.get("full")))
     if rank == 0:
         print(json.dumps(line), flush=True)
     if dist.is_initialized():
@@ -347,7 +359,7 @@ def run_ours(args):
 
 
 # --------------------------------------------------------------------------- oracle timing
-def oracle_sample_time(config: str, tiles: int):
+def oracle_sample_time(config: str, tiles: int, full: bool = False):
     """Time the ORACLE (as it stands) on a bounded sample of one step and scale to images/s.
 
     Sample: 1 image; for every layer-op of the step (conv fwd / dgrad / wgrad, pool fwd / bwd) the
@@ -363,6 +375,11 @@ def oracle_sample_time(config: str, tiles: int):
     c = workload(config, N=1)
     g = synth.rng(c["seed"])
     layers = c["layers"] + c["tail"]
+    if full and c.get("resnet"):                  # + the unsplit layer3/4 (their downsamples via blocks)
+        tc, tb = synth.resnet18_tail_blocks()
+        off = len(layers)
+        layers = layers + tc
+        c = dict(c, blocks=list(c["blocks"]) + [dict(a=b["a"] + off, ds=b["ds"]) for b in tb])
     params = synth.layer_params(g, layers)
     ops, h = [], c["H"]
     for m, (l, prm) in enumerate(zip(layers, params)):
@@ -406,9 +423,9 @@ def oracle_sample_time(config: str, tiles: int):
     return total, f"1 image, {tiles} of 64 output tiles per layer-op (fwd+dgrad+wgrad / pool fwd+bwd), scaled by output pixels"
 
 
-def cpu_baseline(config: str, budget_tiles: int = 4):
+def cpu_baseline(config: str, budget_tiles: int = 4, full: bool = False):
     import os as _os
-    t_img, sample = oracle_sample_time(config, budget_tiles)
+    t_img, sample = oracle_sample_time(config, budget_tiles, full)
     cores = len(_os.sched_getaffinity(0))
     return {"value": round(1.0 / t_img, 5), "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample,
             "seconds_per_image_est": round(t_img, 2)}
@@ -459,6 +476,7 @@ def main():
     ap.add_argument("--no-static-pool", dest="static_pool", action="store_false")
     ap.add_argument("--force-dist", action="store_true",
                     help="run the multi-GPU executor (DistSplitNet, NCCL) even at one rank (exercises the N>1 path)")
+    ap.add_argument("--full", action="store_true", help="C3: the whole ResNet-18 trunk (split region + tail + GAP)")
     ap.add_argument("--bn", action="store_true", help="C3 with whole-tensor BN after every conv (R11, f2)")
     ap.add_argument("--offload", dest="offload", action="store_true", default=None)
     ap.add_argument("--no-offload", dest="offload", action="store_false")

@@ -265,6 +265,16 @@ SPLITCNN_API splitcnn_status_t splitcnn_add(splitcnn_plan_t plan, int32_t level,
                                 const void *a, const void *b, void *y, const void *mask, uint32_t flags,
                                 int32_t p0, int32_t p1, splitcnn_stream_t stream);
 
+/* ------------------------------------------------------------------ global average pool */
+/* ResNet head (f2): y[n][c] = mean of x[n, c] over the level's logical H x W (every pixel of every
+ * patch; a 1x1-split tail level is plain NHWC).  y: [N][Cpad] in the level dtype (pad channels 0).
+ * Backward: dx = dy[n][c] / (H W) at every pixel of every patch (every element written).  Fixed-order
+ * fp32 sums: bitwise reproducible.  Errors: null pointers, misalignment. */
+SPLITCNN_API splitcnn_status_t splitcnn_gap_fwd(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                    const void *x, void *y, splitcnn_stream_t stream);
+SPLITCNN_API splitcnn_status_t splitcnn_gap_bwd(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                    const void *dy, void *dx, splitcnn_stream_t stream);
+
 /* ------------------------------------------------------------------ batch normalisation */
 /* Whole-tensor BN on a split level.  BN is not a window operator, so
  * Split-CNN keeps it unsplit: its statistics are those of the LOGICAL tensor over all patches,

@@ -224,6 +224,16 @@ def _resplit(Y, like):
     return [[Y[:, :, hs[i]:hs[i + 1], ws[j]:ws[j + 1]] for j in range(len(like[0]))] for i in range(len(like))]
 
 
+def global_avg_pool(Y):
+    """ResNet head: mean over the spatial dims of a full NCHW tensor -> [N][C]."""
+    return np.asarray(Y).mean(axis=(2, 3))
+
+
+def global_avg_pool_bwd(G, H, W):
+    """Adjoint of global_avg_pool: G[n][c] / (H W) at every pixel."""
+    return np.repeat(np.repeat((np.asarray(G) / (H * W))[:, :, None, None], H, axis=2), W, axis=3)
+
+
 def relu_mask(dXp, Mp):
     """ReLU backward: keep the gradient where the ReLU output is > 0."""
     return [[np.where(Mp[i][j] > 0, dXp[i][j], 0.0) for j in range(len(row))]

@@ -318,6 +318,29 @@ extern "C" splitcnn_status_t splitcnn_add(splitcnn_plan_t plan, int32_t level, s
     return check_launch("add");
 }
 
+// ------------------------------------------------------------------ global average pool
+extern "C" splitcnn_status_t splitcnn_gap_fwd(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                              const void *x, void *y, splitcnn_stream_t stream) {
+    if (!plan || level < 0 || level >= (int)plan->levels.size()) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad level");
+    TRY(check_dtype(dtype));
+    if (!x || !y) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    NEED_ALIGNED(x, "x");
+    NEED_ALIGNED(y, "y");
+    launch_gap(dtype, true, plan->levels[level], x, y, (cudaStream_t)stream);
+    return check_launch("gap_fwd");
+}
+
+extern "C" splitcnn_status_t splitcnn_gap_bwd(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                              const void *dy, void *dx, splitcnn_stream_t stream) {
+    if (!plan || level < 0 || level >= (int)plan->levels.size()) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad level");
+    TRY(check_dtype(dtype));
+    if (!dy || !dx) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    NEED_ALIGNED(dy, "dy");
+    NEED_ALIGNED(dx, "dx");
+    launch_gap(dtype, false, plan->levels[level], dy, dx, (cudaStream_t)stream);
+    return check_launch("gap_bwd");
+}
+
 // ------------------------------------------------------------------ batch normalisation
 namespace {
 splitcnn_status_t bn_span(splitcnn_plan_t plan, int level, splitcnn_dtype_t dtype, int &p0, int &p1, int64_t &o0,

@@ -430,6 +430,78 @@ void launch_add(splitcnn_dtype_t dt, const void *a, const void *b, void *y, cons
     else launch_add_t<float>(a, b, y, m, relu, n, st);
 }
 
+// ============================================================ global average pool (ResNet head, f2)
+// Forward: y[n][c] = mean over every pixel of image n in every patch of the level (the logical H x W).
+// One block per (image, 256-channel slab); thread = 8 channels x a pixel stride; fixed-order reduction.
+template <typename T>
+__global__ void __launch_bounds__(256) gap_fwd_kernel(LevelDesc L, const T *__restrict__ x, T *__restrict__ y) {
+    __shared__ float red[256][8];
+    const int n = blockIdx.x, G = L.Cpad / 8;
+    const int gs = min(32, G - blockIdx.y * 32);            // channel groups in this slab
+    const int cg = blockIdx.y * 32 + (int)(threadIdx.x % gs), lanes = 256 / gs, pl = threadIdx.x / gs;
+    float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    if (pl < lanes) {
+        for (int q = 0; q < L.nh * L.nw; ++q) {
+            const PatchGeo g = patch_geo(L, q);
+            const int64_t base = g.off + (int64_t)n * g.hp * g.wp * L.Cpad;
+            for (int px = pl; px < g.hp * g.wp; px += lanes) {
+                float v[8];
+                load8(x + base + (int64_t)px * L.Cpad + cg * 8, v);
+#pragma unroll
+                for (int e = 0; e < 8; ++e) acc[e] += v[e];
+            }
+        }
+    }
+#pragma unroll
+    for (int e = 0; e < 8; ++e) red[threadIdx.x][e] = acc[e];
+    __syncthreads();
+    if ((int)threadIdx.x < gs) {
+        float s8[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        for (int l = 0; l < lanes; ++l)
+#pragma unroll
+            for (int e = 0; e < 8; ++e) s8[e] += red[l * gs + threadIdx.x][e];
+        const float inv = 1.f / (float)(L.H * L.W);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) s8[e] *= inv;
+        store8(y + (int64_t)n * L.Cpad + cg * 8, s8);
+    }
+}
+
+// Backward: dx[n][h][w][c] = dy[n][c] / (H W) at every pixel of every patch.
+template <typename T>
+__global__ void __launch_bounds__(256) gap_bwd_kernel(LevelDesc L, const T *__restrict__ dy, T *__restrict__ dx, int p0) {
+    const PatchGeo g = patch_geo(L, p0 + blockIdx.y);
+    const int G = L.Cpad / 8;
+    const uint32_t units = (uint32_t)L.N * g.hp * g.wp * G;
+    const float inv = 1.f / (float)(L.H * L.W);
+    const FastDiv fg = make_fastdiv((uint32_t)G), fp = make_fastdiv((uint32_t)(g.hp * g.wp));
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < units; u += gridDim.x * blockDim.x) {
+        uint32_t cg, px;
+        const uint32_t r = fdivmod(u, fg, cg);
+        const uint32_t n = fdivmod(r, fp, px);
+        float v[8];
+        load8(dy + (int64_t)n * L.Cpad + cg * 8, v);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) v[e] *= inv;
+        store8(dx + g.off + (int64_t)r * L.Cpad + cg * 8, v);
+    }
+}
+
+void launch_gap(splitcnn_dtype_t dt, bool fwd, const Level &L, const void *a, void *b, cudaStream_t st) {
+    const LevelDesc d = make_level_desc(L);
+    if (fwd) {
+        dim3 grid((unsigned)L.N, (unsigned)((L.Cpad / 8 + 31) / 32));
+        if (dt == SPLITCNN_BF16) gap_fwd_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>(d, (const __nv_bfloat16 *)a, (__nv_bfloat16 *)b);
+        else gap_fwd_kernel<float><<<grid, 256, 0, st>>>(d, (const float *)a, (float *)b);
+    } else {
+        npatch_launch = L.npatch();
+        dim3 grid(grid_x_for(max_patch_units(L, 0, L.npatch(), L.Cpad / 8)), L.npatch());
+        if (dt == SPLITCNN_BF16) gap_bwd_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>(d, (const __nv_bfloat16 *)a, (__nv_bfloat16 *)b, 0);
+        else gap_bwd_kernel<float><<<grid, 256, 0, st>>>(d, (const float *)a, (float *)b, 0);
+    }
+    count_launch();
+}
+
 void launch_pool_fwd(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, void *y,
                      uint8_t *a, int relu_bit, int p0, int p1, cudaStream_t st) {
     if (dt == SPLITCNN_BF16) launch_pool_fwd_t<__nv_bfloat16>(Li, Lo, g, x, y, a, relu_bit, p0, p1, st);

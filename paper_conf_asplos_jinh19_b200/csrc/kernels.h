@@ -13,6 +13,7 @@ void launch_pool_fwd(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, cons
                      uint8_t *a, int relu_bit, int p0, int p1, cudaStream_t st);
 void launch_pool_bwd(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy,
                      const uint8_t *a, void *dx, int relu_bit, int p0, int p1, cudaStream_t st);
+void launch_gap(splitcnn_dtype_t dt, bool fwd, const Level &L, const void *a, void *b, cudaStream_t st);
 void launch_add(splitcnn_dtype_t dt, const void *a, const void *b, void *y, const void *m, int relu, int64_t n,
                 cudaStream_t st);
 

@@ -151,6 +151,11 @@ class ResSplitNet(SplitNet):
             self._ds_params[k][0].copy_(pack_weight(W, p.levels[0]["Cpad"], self.tdtype))
             self._ds_params[k][1].copy_(torch.as_tensor(b, dtype=torch.float32))
 
+    def _conv_keys(self):
+        """Conv keys in synth.resnet_params order: chain convs, then downsamples."""
+        return [("r", m) for m, l in enumerate(self.region_layers) if l["op"] == "conv"] + \
+               [("ds", k) for k in sorted(self.ds_plans)]
+
     def grad_oihw(self, key) -> torch.Tensor:
         """Weight gradient of conv `key` in OIHW (the stem's s2d gradient mapped back to 7x7)."""
         dW = self.grads[key][0]
@@ -555,3 +560,91 @@ class ResBNSplitNet(ResSplitNet):
                 g = out
             m -= 1
         return g
+
+
+class ResNet18Net:
+    """The whole ResNet-18 trunk: the split region (stem .. layer2, split per the
+    config) -> merge at the join (Eq. 7) -> the unsplit tail (layer3, layer4: the same block executor
+    on a 1x1 split) -> global average pool.  BN-free by default, `bn=True` puts whole-tensor BN after
+    every conv.  forward(x NCHW) -> [N][C] pooled features; backward(dY [N][C]).  No FC head (the
+    benchmark drives backward with a synthetic dY)."""
+
+    def __init__(self, region_chain, region_blocks, tail_chain, tail_blocks, N, C, H, W, split=(2, 2), bn=False,
+                 dtype: int = sc.BF16, device="cuda"):
+        cls = ResBNSplitNet if bn else ResSplitNet
+        self.net_r = cls(region_chain, region_blocks, N, C, H, W, split=split, dtype=dtype, device=device)
+        L = self.net_r.region.levels[-1]
+        self.net_t = cls(tail_chain, tail_blocks, N, L["C"], L["H"], L["W"], split=(1, 1), dtype=dtype, device=device)
+        self.dtype, self.tdtype, self.device = dtype, self.net_r.tdtype, self.net_r.device
+        self.N = N
+        Lt = self.net_t.region.levels[-1]
+        self.C_out = Lt["C"]
+        self.pooled = torch.zeros(N * Lt["Cpad"], dtype=self.tdtype, device=self.device)
+        self.g_out = torch.zeros(Lt["total_elems"], dtype=self.tdtype, device=self.device)
+        self.step_index = 0
+        self.input_grad = False
+        n_r, n_t = self.net_r.grad_numel(), self.net_t.grad_numel()
+        self.bind_grads(torch.zeros(n_r + n_t, dtype=torch.float32, device=self.device))
+
+    def bind_grads(self, flat):
+        n_r = self.net_r.grad_numel()
+        self.grad_flat = flat
+        self.net_r.bind_grads(flat[:n_r])
+        self.net_t.bind_grads(flat[n_r:])
+
+    @property
+    def timers(self):
+        return self.net_r.timers
+
+    @timers.setter
+    def timers(self, v):
+        self.net_r.timers = v
+        self.net_t.timers = v
+
+    def set_params(self, params):
+        params = list(params)
+        n_r = sum(1 for l in self.net_r.region_layers if l["op"] == "conv") + len(self.net_r.ds_plans)
+        self.net_r.set_params(params[:n_r])
+        self.net_t.set_params(params[n_r:])
+
+    def set_bn_params(self, bn_params):
+        if not hasattr(self.net_r, "_bn_keys"):
+            return                               # BN-free trunk
+        bn_params = list(bn_params)
+        n_r = len(self.net_r._bn_keys())
+        self.net_r.set_bn_params(bn_params[:n_r])
+        self.net_t.set_bn_params(bn_params[n_r:])
+
+    def output_numel(self) -> int:
+        return self.pooled.numel()
+
+    def forward(self, x, stream=None):
+        y = self.net_r.forward(x, stream)                          # merged NHWC join tensor
+        z = self.net_t.forward(y, stream, sc.NHWC)                 # merged NHWC tail output
+        T = self.net_t.region
+        self.net_t._label = "gap"
+        self.net_t._call("gap", z.numel() * z.element_size(), sc.splitcnn_gap_fwd, T.handle, T.nlayers, self.dtype, z,
+                         self.pooled, stream)
+        return self.pooled
+
+    def backward(self, dy, stream=None, need_input_grad: bool = False):
+        T = self.net_t.region
+        self.net_t._label = "gap"
+        self.net_t._call("gap", self.g_out.numel() * self.g_out.element_size(), sc.splitcnn_gap_bwd, T.handle,
+                         T.nlayers, self.dtype, dy, self.g_out, stream)
+        g = self.net_t.backward(self.g_out, stream, need_input_grad=True)    # tail level 0 = merged NHWC
+        return self.net_r.backward(g, stream, need_input_grad)
+
+    def step(self, x, dy, stream=None):
+        self.forward(x, stream)
+        self.backward(dy, stream, self.input_grad)
+        self.step_index += 1
+
+    def conv_flops(self) -> int:
+        return self.net_r.conv_flops() + self.net_t.conv_flops()
+
+    def grad_of(self, i):
+        """OIHW weight gradient of conv i in resnet_params order (region chain, region ds, tail chain, tail ds)."""
+        keys = [(self.net_r, k) for k in self.net_r._conv_keys()] + [(self.net_t, k) for k in self.net_t._conv_keys()]
+        net, key = keys[i]
+        return net.grad_oihw(key), net.grads[key][1]

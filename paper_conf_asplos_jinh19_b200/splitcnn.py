@@ -36,6 +36,7 @@ EXPORTED = [
     "splitcnn_split", "splitcnn_merge",
     "splitcnn_conv_fwd", "splitcnn_conv_bwd_data", "splitcnn_conv_bwd_filter",
     "splitcnn_pool_fwd", "splitcnn_pool_bwd", "splitcnn_conv_pool_fwd", "splitcnn_conv_pool_supported", "splitcnn_add",
+    "splitcnn_gap_fwd", "splitcnn_gap_bwd",
     "splitcnn_bn_workspace_size", "splitcnn_bn_stats", "splitcnn_bn_fwd", "splitcnn_bn_bwd_sums", "splitcnn_bn_bwd",
     "splitcnn_offload", "splitcnn_prefetch", "splitcnn_patch_bytes",
     "splitcnn_offload_plan", "splitcnn_prefetch_plan", "splitcnn_memplan",
@@ -91,6 +92,8 @@ _sig("splitcnn_conv_bwd_filter", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _
 _sig("splitcnn_pool_fwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
 _sig("splitcnn_pool_bwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
 _sig("splitcnn_conv_pool_fwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
+_sig("splitcnn_gap_fwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp])
+_sig("splitcnn_gap_bwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp])
 _sig("splitcnn_bn_workspace_size", [_vp, _i32, ctypes.POINTER(_sz)])
 _sig("splitcnn_bn_stats", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _sz, _i32, _i32, _vp])
 _sig("splitcnn_bn_fwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _f64, _vp, _vp, _f32, _vp, _vp, _u32, _i32, _i32, _vp])
@@ -279,6 +282,14 @@ def splitcnn_pool_bwd(plan, layer, dtype, dy, argmax, dx, flags=0, p0=0, p1=-1, 
 def splitcnn_add(plan, level, dtype, a, b, y, mask=None, flags=0, p0=0, p1=-1, stream=None):
     _check(_lib.splitcnn_add(plan, level, dtype, _ptr(a), _ptr(b), _ptr(y), _ptr(mask), flags, p0, p1,
                              _stream(stream)))
+
+
+def splitcnn_gap_fwd(plan, level, dtype, x, y, stream=None):
+    _check(_lib.splitcnn_gap_fwd(plan, level, dtype, _ptr(x), _ptr(y), _stream(stream)))
+
+
+def splitcnn_gap_bwd(plan, level, dtype, dy, dx, stream=None):
+    _check(_lib.splitcnn_gap_bwd(plan, level, dtype, _ptr(dy), _ptr(dx), _stream(stream)))
 
 
 def splitcnn_bn_workspace_size(plan, level) -> int:

@@ -69,6 +69,21 @@ def resnet18_blocks(w1: int = 64, w2: int = 128):
     return L, blocks
 
 
+def resnet18_tail_blocks(cin: int = 128, w3: int = 256, w4: int = 512):
+    """The unsplit ResNet-18 tail (layer3, layer4; each first block stride 2 with a 1x1 downsample) in
+    the same (chain, blocks) form as resnet18_blocks; the global average pool follows it."""
+    L, blocks, c = [], [], cin
+    for stage, w in ((3, w3), (4, w4)):
+        for b in range(2):
+            s = 2 if b == 0 else 1
+            ds = conv(c, w, k=1, s=s, p=0, relu=False, name=f"layer{stage}_{b}_ds") if (s != 1 or c != w) else None
+            blocks.append(dict(a=len(L), ds=ds))
+            L.append(conv(c, w, s=s, name=f"layer{stage}_{b}_a"))
+            L.append(conv(w, w, relu=False, name=f"layer{stage}_{b}_b"))
+            c = w
+    return L, blocks
+
+
 def split_region(layers, depth_convs: int, include_next_pool: bool):
     """First ``depth_convs`` convolutions (plus interleaved pools, plus the pool right
     after the last split conv when ``include_next_pool``) -> (region, tail)."""

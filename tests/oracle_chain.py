@@ -99,7 +99,7 @@ def _out(layers, L, dim):
     return L
 
 
-def run_resnet(chain, blocks, N, C, H, W, Oh, Ow, params, X, G, round_bf16=False):
+def run_resnet(chain, blocks, N, C, H, W, Oh, Ow, params, X, G, round_bf16=False, return_input_grad=False):
     """Oracle composition of the BN-free ResNet split stack (synth.resnet18_blocks): the main
     chain with a residual join after every block's second conv, the 1x1 downsample on its own
     one-layer plan sharing the block's output partition.  G is the gradient of the merged output.
@@ -186,6 +186,8 @@ def run_resnet(chain, blocks, N, C, H, W, Oh, Ow, params, X, G, round_bf16=False
     dWs = [grads[m][0] for m in sorted(grads)] + [gds[k][0] for k in sorted(gds)]
     dbs = [grads[m][1] for m in sorted(grads)] + [gds[k][1] for k in sorted(gds)]
     assert len(dWs) == nconv + len(ds)
+    if return_input_grad:
+        return out, dWs, dbs, O.merge(g)
     return out, dWs, dbs
 
 
@@ -283,3 +285,26 @@ def run_resnet_bn(chain, blocks, N, C, H, W, Oh, Ow, params, bn, X, G, round_bf1
         m -= 1
     keys = [("r", m) for m in conv_ms] + [("ds", k) for k in sorted(ds)]
     return out, [grads[k] for k in keys], [bgrads[k][0] for k in keys], [bgrads[k][1] for k in keys]
+
+
+def run_resnet18_full(rc, rb, tc, tb, N, C, H, W, Oh, Ow, params, X, G, round_bf16=False):
+    """Oracle of the whole trunk: split region (stem .. layer2) -> merge -> unsplit tail (layer3,
+    layer4; 1x1 split) -> global average pool; G is the gradient of the pooled [N][C] output.
+    params in synth.resnet_params order for the region, then for the tail.
+    Returns (pooled [N][C], dWs, dbs) in that order."""
+    n_r = sum(1 for l in rc if l["op"] == "conv") + sum(1 for b in rb if b["ds"] is not None)
+    p_r, p_t = params[:n_r], params[n_r:]
+    rp = OP.plan(rc, N, C, H, W, Oh, Ow)
+    Lr = rp.layers[-1]
+    zero = np.zeros((N, rc[-1]["cout"], Lr.H_out, Lr.W_out))
+    out_r, _, _ = run_resnet(rc, rb, N, C, H, W, Oh, Ow, p_r, X, zero, round_bf16)
+    tp = OP.plan(tc, N, rc[-1]["cout"], Lr.H_out, Lr.W_out, [0, _out(tc, Lr.H_out, 0)], [0, _out(tc, Lr.W_out, 1)])
+    Lt = tp.layers[-1]
+    G_t = O.global_avg_pool_bwd(G, Lt.H_out, Lt.W_out)
+    if round_bf16:
+        G_t = synth.to_bf16_f32(G_t.astype(np.float32)).astype(np.float64)
+    out_t, dW_t, db_t, g_in = run_resnet(tc, tb, N, rc[-1]["cout"], Lr.H_out, Lr.W_out, [0, Lt.H_out], [0, Lt.W_out],
+                                         p_t, out_r, G_t, round_bf16, return_input_grad=True)
+    pooled = O.global_avg_pool(out_t)
+    _, dW_r, db_r = run_resnet(rc, rb, N, C, H, W, Oh, Ow, p_r, X, g_in, round_bf16)
+    return pooled, dW_r + dW_t, db_r + db_t

@@ -248,11 +248,11 @@ def test_split_merge_identity_pin8():
 
 
 # --------------------------------------------------------------------------- ResNet split stack
-def _torch_resnet(chain, blocks, X, params):
+def _torch_resnet(chain, blocks, X, params, x_tensor=None):
     """Unsplit BN-free ResNet stack in torch fp64 (library routines), for the 1x1-split pin."""
     import torch
     import torch.nn.functional as F
-    x = torch.tensor(X, requires_grad=True)
+    x = torch.tensor(X, requires_grad=True) if x_tensor is None else x_tensor
     ps = [(torch.tensor(W, requires_grad=True), torch.tensor(b, requires_grad=True)) for W, b in params]
     nconv = sum(1 for l in chain if l["op"] == "conv")
     cidx = {m: i for i, m in enumerate(m for m, l in enumerate(chain) if l["op"] == "conv")}
@@ -396,3 +396,30 @@ def test_batch_norm_split_invariant():
     P1, _, _ = O.batch_norm(O.split(X, [0, 9], [0, 7]), gm, bt, relu=True)
     P2, _, _ = O.batch_norm(O.split(X, [0, 2, 9], [0, 4, 5, 7]), gm, bt, relu=True)
     assert np.array_equal(O.merge(P1), O.merge(P2))
+
+
+def test_resnet18_full_trunk_1x1_split_equals_unsplit_torch():
+    """pin-1 for the whole trunk oracle (split region -> merge -> unsplit tail -> global average pool):
+    with a 1x1 region split it is the unsplit BN-free ResNet-18 trunk; pooled output and every weight /
+    bias gradient vs torch fp64 autograd."""
+    import torch
+    from tests import oracle_chain
+    rc, rb = synth.resnet18_blocks(8, 16)
+    tc, tb = synth.resnet18_tail_blocks(16, 16, 32)
+    g = synth.rng(12)
+    N, H = 2, 64
+    X = synth.uniform(g, (N, 3, H, H)).astype(np.float64)
+    p_r = [(W.astype(np.float64), b.astype(np.float64)) for W, b in synth.resnet_params(g, rc, rb)]
+    p_t = [(W.astype(np.float64), b.astype(np.float64)) for W, b in synth.resnet_params(g, tc, tb)]
+    Yr, x, ps_r = _torch_resnet(rc, rb, X, p_r)
+    # the tail on the region output, then the global average pool
+    Yt, _, ps_t = _torch_resnet(tc, tb, None, p_t, x_tensor=Yr)
+    pooled = Yt.mean(dim=(2, 3))
+    G = synth.normal(g, tuple(pooled.shape)).astype(np.float64)
+    (pooled * torch.tensor(G)).sum().backward()
+    out, dWs, dbs = oracle_chain.run_resnet18_full(rc, rb, tc, tb, N, 3, H, H, [0, Yr.shape[2]], [0, Yr.shape[3]],
+                                                   p_r + p_t, X, G)
+    assert np.abs(out - pooled.detach().numpy()).max() < 1e-12
+    for (Wt, bt), dW, db in zip(ps_r + ps_t, dWs, dbs):
+        assert np.abs(dW - Wt.grad.numpy()).max() < 1e-10 * max(1.0, np.abs(dW).max())
+        assert np.abs(db - bt.grad.numpy()).max() < 1e-10 * max(1.0, np.abs(db).max())

@@ -112,6 +112,30 @@ __global__ void __launch_bounds__(BN_THREADS) bn_apply_kernel(const T *x, const 
                                                               const float *__restrict__ gamma,
                                                               const float *__restrict__ beta, T *y,
                                                               int64_t n8, int G, int C) {
+    if (blockDim.x % G == 0) {
+        // the grid stride is a multiple of G: this thread always sees the same 8 channels -> per-channel
+        // scale / shift once, no 64-bit modulo per unit
+        const int cg = threadIdx.x % G;
+        float sc_[8], sh[8];
+#pragma unroll
+        for (int e = 0; e < 8; ++e) {
+            const int c = cg * 8 + e;
+            sc_[e] = c < C ? gamma[c] * mi[C + c] : 0.f;
+            sh[e] = c < C ? beta[c] - mi[c] * sc_[e] : 0.f;
+        }
+        for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n8; u += (int64_t)gridDim.x * blockDim.x) {
+            float v[8];
+            load8(x + u * 8, v);
+#pragma unroll
+            for (int e = 0; e < 8; ++e) {
+                float o = fmaf(v[e], sc_[e], sh[e]);
+                if (RELU) o = fmaxf(o, 0.f);
+                v[e] = o;
+            }
+            store8(y + u * 8, v);
+        }
+        return;
+    }
     for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n8; u += (int64_t)gridDim.x * blockDim.x) {
         const int cg = (int)(u % G);
         float v[8];
@@ -138,6 +162,34 @@ __global__ void __launch_bounds__(BN_THREADS) bn_bwd_kernel(const T *dy, const T
                                                             const float *__restrict__ gamma,
                                                             const float *__restrict__ t, float invM, T *dx,
                                                             int64_t n8, int G, int C) {
+    if (blockDim.x % G == 0) {      // fixed channels per thread (see bn_apply_kernel)
+        const int cg = threadIdx.x % G;
+        float k1[8], mean[8], inv[8], t0[8], t1[8];
+#pragma unroll
+        for (int e = 0; e < 8; ++e) {
+            const int c = min(cg * 8 + e, C - 1);
+            const bool ok = cg * 8 + e < C;
+            inv[e] = mi[C + c];
+            mean[e] = mi[c];
+            k1[e] = ok ? gamma[c] * inv[e] : 0.f;
+            t0[e] = t[c] * invM;
+            t1[e] = t[C + c] * invM;
+        }
+        for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n8; u += (int64_t)gridDim.x * blockDim.x) {
+            float g[8], v[8], m[8];
+            load8(dy + u * 8, g);
+            load8(x + u * 8, v);
+            if (y) load8(y + u * 8, m);
+#pragma unroll
+            for (int e = 0; e < 8; ++e) {
+                const float ge = (!y || m[e] > 0.f) ? g[e] : 0.f;
+                const float xh = (v[e] - mean[e]) * inv[e];
+                g[e] = k1[e] * (ge - t0[e] - xh * t1[e]);
+            }
+            store8(dx + u * 8, g);
+        }
+        return;
+    }
     for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n8; u += (int64_t)gridDim.x * blockDim.x) {
         const int cg = (int)(u % G);
         float g[8], v[8], m[8];

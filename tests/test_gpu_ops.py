@@ -345,3 +345,49 @@ def test_conv_pool_fused_matches_unfused_and_oracle(sc, case):
     got = unpack_level(_host(yf), lv2)
     err = max(normwise(got[i][j], P[i][j]) for i in range(nh) for j in range(nw))
     assert err <= TOL[dtype], err
+
+
+# --------------------------------------------------------------------------- residual add, global average pool
+@pytest.mark.parametrize("dtype_name", ["bf16", "fp32"])
+def test_add_and_gap_parity(sc, dtype_name):
+    """splitcnn_add (y = relu(a + b); masked gradient sum) on a patch range of uneven patches, and
+    splitcnn_gap_fwd/_bwd (global average pool over the logical H x W) against the oracle definitions."""
+    from paper_conf_asplos_jinh19_b200.plan import SplitPlan
+    dtype = sc.BF16 if dtype_name == "bf16" else sc.FP32
+    td = _td(sc, dtype)
+    N, C, H, W = 3, 24, 9, 11
+    pl = SplitPlan([synth.conv(C, C, 1, 1, 0)], N, C, H, W, [0, 4, 9], [0, 3, 7, 11])
+    lv = pl.levels[0]
+    g = synth.rng(31)
+    A, B, M = (_round(synth.normal(g, (N, C, H, W)), dtype, sc) for _ in range(3))
+    a, b, m = (_dev(sc, pack_level(T, lv), dtype) for T in (A, B, M))
+    y = torch.full_like(a, 7.0)
+    sc.splitcnn_add(pl.handle, 0, dtype, a, b, y, None, sc.FLAG_RELU)
+    ref = O.residual_add(O.split(A, [0, 4, 9], [0, 3, 7, 11]), O.split(B, [0, 4, 9], [0, 3, 7, 11]), relu=True)
+    got = unpack_level(_host(y), lv)
+    tol = TOL[dtype]
+    assert max(normwise(got[i][j], ref[i][j]) for i in range(2) for j in range(3)) <= tol
+    # masked gradient sum on patches [1, 4) only; the rest of y keeps its previous values
+    y2 = y.clone()
+    sc.splitcnn_add(pl.handle, 0, dtype, a, b, y2, m, 0, 1, 4)
+    refm = O.relu_mask(O.residual_add(O.split(A, [0, 4, 9], [0, 3, 7, 11]), O.split(B, [0, 4, 9], [0, 3, 7, 11])),
+                       O.split(M, [0, 4, 9], [0, 3, 7, 11]))
+    got2 = unpack_level(_host(y2), lv)
+    for q in range(6):
+        i, j = divmod(q, 3)
+        exp = refm[i][j] if 1 <= q < 4 else got[i][j]
+        assert normwise(got2[i][j], exp) <= tol, q
+    # global average pool over all patches
+    pooled = torch.full((N * lv["Cpad"],), 7.0, dtype=td, device="cuda")
+    sc.splitcnn_gap_fwd(pl.handle, 0, dtype, a, pooled)
+    gp = _host(pooled).reshape(N, lv["Cpad"])
+    assert normwise(gp[:, :C], O.global_avg_pool(A)) <= tol
+    assert np.all(gp[:, C:] == 0)
+    Gp = _round(synth.normal(g, (N, C)), dtype, sc)
+    gpad = np.zeros((N, lv["Cpad"]))
+    gpad[:, :C] = Gp
+    dx = torch.full_like(a, 7.0)
+    sc.splitcnn_gap_bwd(pl.handle, 0, dtype, torch.from_numpy(gpad.reshape(-1).astype(np.float32)).to("cuda", td), dx)
+    dref = O.split(O.global_avg_pool_bwd(Gp, H, W), [0, 4, 9], [0, 3, 7, 11])
+    gd = unpack_level(_host(dx), lv)
+    assert max(normwise(gd[i][j], dref[i][j]) for i in range(2) for j in range(3)) <= tol

@@ -4,6 +4,7 @@
 //   max-pool forward / backward per patch (Eq. 6 with Op = max-pool)
 // One thread moves 8 channels (16 B in bf16) of one pixel; grid.y enumerates patches.
 #include <algorithm>
+#include <type_traits>
 #include <cstdlib>
 
 #include "common.cuh"
@@ -348,11 +349,113 @@ __global__ void __launch_bounds__(256) pool_bwd_k3s2_kernel(LevelDesc Li, LevelD
     }
 }
 
+// ------------------------------------------------------------ 2x2 / stride-2 bf16 fast paths (VGG pools)
+// Windows tile the patch exactly (k = s = 2, no padding, hp = 2 ho): no bounds checks, and the 8 channels
+// of a unit are handled as 4 bf16x2 words with packed compares / selects -- the generic kernels spend
+// ~440 instructions per unit (ncu), these a fraction of it.  Same results bit for bit: strict '>' in
+// row-major window order (first maximum), ReLU bit = [max > 0] exactly as the float compare.
+__device__ __forceinline__ uint32_t bf2_gt(uint32_t a, uint32_t b) {
+    return __hgt2_mask(*reinterpret_cast<const __nv_bfloat162 *>(&a), *reinterpret_cast<const __nv_bfloat162 *>(&b));
+}
+__device__ __forceinline__ uint32_t bf2_pos_byte(uint32_t w, int half) {   // [element > 0] of one bf16
+    const uint32_t h = (w >> (16 * half)) & 0xFFFFu;
+    return ((h & 0x8000u) == 0u && (h & 0x7FFFu) != 0u && (h & 0x7FFFu) <= 0x7F80u) ? 0x80u : 0u;
+}
+
+__global__ void __launch_bounds__(256) pool2x2_fwd_bf16_kernel(LevelDesc Li, LevelDesc Lo, const __nv_bfloat16 *__restrict__ X,
+                                                               __nv_bfloat16 *__restrict__ Y, uint8_t *__restrict__ A,
+                                                               int p0, int relu_bit) {
+    const int q = p0 + blockIdx.y;
+    const PatchGeo gi = patch_geo(Li, q), go = patch_geo(Lo, q);
+    const int G = Li.Cpad / 8;
+    const uint32_t units = (uint32_t)Lo.N * go.hp * go.wp * G;
+    const Dec3 d = make_dec3(G, go.wp, go.hp);
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < units; u += gridDim.x * blockDim.x) {
+        int cg, ow, oh, n;
+        dec3(u, d, cg, ow, oh, n);
+        const __nv_bfloat16 *x0 = X + gi.off + (((int64_t)n * gi.hp + 2 * oh) * gi.wp + 2 * ow) * Li.Cpad + cg * 8;
+        const int64_t rs = (int64_t)gi.wp * Li.Cpad;
+        uint4 v[4];
+        v[0] = __ldg(reinterpret_cast<const uint4 *>(x0));
+        v[1] = __ldg(reinterpret_cast<const uint4 *>(x0 + Li.Cpad));
+        v[2] = __ldg(reinterpret_cast<const uint4 *>(x0 + rs));
+        v[3] = __ldg(reinterpret_cast<const uint4 *>(x0 + rs + Li.Cpad));
+        uint32_t best[4], arg[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const uint32_t *w0 = reinterpret_cast<const uint32_t *>(&v[0]);
+            best[j] = w0[j];
+            arg[j] = 0;
+#pragma unroll
+            for (int t = 1; t < 4; ++t) {
+                const uint32_t w = reinterpret_cast<const uint32_t *>(&v[t])[j];
+                const uint32_t m = bf2_gt(w, best[j]);
+                best[j] = (w & m) | (best[j] & ~m);
+                arg[j] = ((uint32_t)(t * 0x00010001u) & m) | (arg[j] & ~m);
+            }
+        }
+        const int64_t o = go.off + (((int64_t)n * go.hp + oh) * go.wp + ow) * Lo.Cpad + cg * 8;
+        *reinterpret_cast<uint4 *>(Y + o) = make_uint4(best[0], best[1], best[2], best[3]);
+        uint32_t lo = 0, hi = 0;
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const int k = 2 * j + h;
+                uint32_t b = (arg[j] >> (16 * h)) & 0x3u;
+                if (relu_bit) b |= bf2_pos_byte(best[j], h);
+                if (k < 4) lo |= b << (8 * k); else hi |= b << (8 * (k - 4));
+            }
+        *reinterpret_cast<uint2 *>(A + o) = make_uint2(lo, hi);
+    }
+}
+
+__global__ void __launch_bounds__(256) pool2x2_bwd_bf16_kernel(LevelDesc Li, LevelDesc Lo, const __nv_bfloat16 *__restrict__ dY,
+                                                               const uint8_t *__restrict__ A, __nv_bfloat16 *__restrict__ dX,
+                                                               int p0, int relu_bit) {
+    const int q = p0 + blockIdx.y;
+    const PatchGeo gi = patch_geo(Li, q), go = patch_geo(Lo, q);
+    const int G = Li.Cpad / 8;
+    const uint32_t units = (uint32_t)Lo.N * go.hp * go.wp * G;
+    const Dec3 d = make_dec3(G, go.wp, go.hp);
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < units; u += gridDim.x * blockDim.x) {
+        int cg, ow, oh, n;
+        dec3(u, d, cg, ow, oh, n);
+        const int64_t o = go.off + (((int64_t)n * go.hp + oh) * go.wp + ow) * Lo.Cpad + cg * 8;
+        const uint2 a2 = __ldg(reinterpret_cast<const uint2 *>(A + o));
+        const uint4 g = __ldg(reinterpret_cast<const uint4 *>(dY + o));
+        __nv_bfloat16 *x0 = dX + gi.off + (((int64_t)n * gi.hp + 2 * oh) * gi.wp + 2 * ow) * Li.Cpad + cg * 8;
+        const int64_t rs = (int64_t)gi.wp * Li.Cpad;
+        // hit byte k <=> argmax byte == t (| 0x80 when the ReLU bit gates it)
+        const uint32_t keep = relu_bit ? 0xFFFFFFFFu : 0x7F7F7F7Fu;
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+            const uint32_t tgt = (uint32_t)(t | (relu_bit ? 0x80 : 0)) * 0x01010101u;
+            const uint32_t e_lo = __vcmpeq4(a2.x & keep, tgt), e_hi = __vcmpeq4(a2.y & keep, tgt);
+            const uint4 r = make_uint4(g.x & __byte_perm(e_lo, 0, 0x1100), g.y & __byte_perm(e_lo, 0, 0x3322),
+                                       g.z & __byte_perm(e_hi, 0, 0x1100), g.w & __byte_perm(e_hi, 0, 0x3322));
+            *reinterpret_cast<uint4 *>(x0 + (t >> 1) * rs + (t & 1) * Li.Cpad) = r;
+        }
+    }
+}
+
 template <typename T>
 void launch_pool_fwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, void *y, uint8_t *a,
                        int relu_bit, int p0, int p1, cudaStream_t st) {
     npatch_launch = p1 - p0;
     dim3 grid(grid_x_for(max_patch_units(Lo, p0, p1, Lo.Cpad / 8)), p1 - p0);
+    bool exact = std::is_same<T, __nv_bfloat16>::value && g.L.kh == 2 && g.L.kw == 2 && g.L.sh == 2 && g.L.sw == 2 &&
+                 !getenv("SPLITCNN_POOL_GENERIC");
+    for (size_t i = 0; exact && i < g.pad_h.size(); ++i) exact = g.pad_h[i] == 0;
+    for (size_t i = 0; exact && i < g.pad_w.size(); ++i) exact = g.pad_w[i] == 0;
+    for (int i = 0; exact && i < Li.nh(); ++i) exact = Li.ph(i) == 2 * Lo.ph(i);
+    for (int j = 0; exact && j < Li.nw(); ++j) exact = Li.pw(j) == 2 * Lo.pw(j);
+    if (exact) {
+        pool2x2_fwd_bf16_kernel<<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), (const __nv_bfloat16 *)x,
+                                                      (__nv_bfloat16 *)y, a, p0, relu_bit);
+        count_launch();
+        return;
+    }
     { pool_fwd_kernel<T><<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
                                              (const T *)x, (T *)y, a, p0, relu_bit); count_launch(); }
 }
@@ -364,6 +467,14 @@ void launch_pool_bwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, con
     for (size_t i = 0; exact && i < g.pad_w.size(); ++i) exact = g.pad_w[i] == 0;
     for (int i = 0; exact && i < Li.nh(); ++i) exact = Li.ph(i) == Lo.ph(i) * g.L.sh;
     for (int j = 0; exact && j < Li.nw(); ++j) exact = Li.pw(j) == Lo.pw(j) * g.L.sw;
+    if (exact && std::is_same<T, __nv_bfloat16>::value && g.L.kh == 2 && g.L.kw == 2 && !getenv("SPLITCNN_POOL_GENERIC")) {
+        npatch_launch = p1 - p0;
+        dim3 grid(grid_x_for(max_patch_units(Lo, p0, p1, Lo.Cpad / 8)), p1 - p0);
+        pool2x2_bwd_bf16_kernel<<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), (const __nv_bfloat16 *)dy,
+                                                      a, (__nv_bfloat16 *)dx, p0, relu_bit);
+        count_launch();
+        return;
+    }
     if (exact) {
         npatch_launch = p1 - p0;
         dim3 grid(grid_x_for(max_patch_units(Lo, p0, p1, Lo.Cpad / 8)), p1 - p0);

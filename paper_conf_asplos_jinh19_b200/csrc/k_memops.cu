@@ -410,6 +410,67 @@ __global__ void __launch_bounds__(256) pool2x2_fwd_bf16_kernel(LevelDesc Li, Lev
     }
 }
 
+// 3x3 / stride-2 bf16 forward (ResNet's max-pool, pads per patch): 9 window positions in row-major
+// order with per-position bounds (skipped = -inf), packed bf16x2 compares; bit-identical to the generic
+// kernel (first maximum, strict '>'; the first in-bounds position initialises the maximum).
+__global__ void __launch_bounds__(256) pool3x3s2_fwd_bf16_kernel(LevelDesc Li, LevelDesc Lo, LayerDesc ly,
+                                                                 const __nv_bfloat16 *__restrict__ X,
+                                                                 __nv_bfloat16 *__restrict__ Y, uint8_t *__restrict__ A,
+                                                                 int p0, int relu_bit) {
+    const int q = p0 + blockIdx.y;
+    const PatchGeo gi = patch_geo(Li, q), go = patch_geo(Lo, q);
+    const int pt = ly.pad_h[2 * gi.i], pl = ly.pad_w[2 * gi.j];
+    const int G = Li.Cpad / 8;
+    const uint32_t units = (uint32_t)Lo.N * go.hp * go.wp * G;
+    const Dec3 d = make_dec3(G, go.wp, go.hp);
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < units; u += gridDim.x * blockDim.x) {
+        int cg, ow, oh, n;
+        dec3(u, d, cg, ow, oh, n);
+        const int h0 = 2 * oh - pt, w0 = 2 * ow - pl;
+        uint4 v[9];
+        uint32_t inb = 0;
+#pragma unroll
+        for (int t = 0; t < 9; ++t) {
+            const int h = h0 + t / 3, w = w0 + t % 3;
+            if (h >= 0 && h < gi.hp && w >= 0 && w < gi.wp) {
+                inb |= 1u << t;
+                v[t] = __ldg(reinterpret_cast<const uint4 *>(X + gi.off + (((int64_t)n * gi.hp + h) * gi.wp + w) * Li.Cpad + cg * 8));
+            }
+        }
+        uint32_t best[4] = {0, 0, 0, 0}, arg[4] = {0, 0, 0, 0};
+        bool first = true;
+#pragma unroll
+        for (int t = 0; t < 9; ++t) {
+            if (!(inb & (1u << t))) continue;
+            const uint32_t *w = reinterpret_cast<const uint32_t *>(&v[t]);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const uint32_t m = first ? 0xFFFFFFFFu : bf2_gt(w[j], best[j]);
+                best[j] = (w[j] & m) | (best[j] & ~m);
+                arg[j] = ((uint32_t)(t * 0x00010001u) & m) | (arg[j] & ~m);
+            }
+            first = false;
+        }
+        const int64_t o = go.off + (((int64_t)n * go.hp + oh) * go.wp + ow) * Lo.Cpad + cg * 8;
+        if (first) {   // no in-bounds position: impossible for a valid plan (pads < k); -inf
+            const uint32_t ninf = 0xFF80FF80u;
+            best[0] = best[1] = best[2] = best[3] = ninf;
+        }
+        *reinterpret_cast<uint4 *>(Y + o) = make_uint4(best[0], best[1], best[2], best[3]);
+        uint32_t lo = 0, hi = 0;
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const int k = 2 * j + h;
+                uint32_t b = (arg[j] >> (16 * h)) & 0xFu;
+                if (relu_bit) b |= bf2_pos_byte(best[j], h);
+                if (k < 4) lo |= b << (8 * k); else hi |= b << (8 * (k - 4));
+            }
+        *reinterpret_cast<uint2 *>(A + o) = make_uint2(lo, hi);
+    }
+}
+
 __global__ void __launch_bounds__(256) pool2x2_bwd_bf16_kernel(LevelDesc Li, LevelDesc Lo, const __nv_bfloat16 *__restrict__ dY,
                                                                const uint8_t *__restrict__ A, __nv_bfloat16 *__restrict__ dX,
                                                                int p0, int relu_bit) {
@@ -450,6 +511,13 @@ void launch_pool_fwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, con
     for (size_t i = 0; exact && i < g.pad_w.size(); ++i) exact = g.pad_w[i] == 0;
     for (int i = 0; exact && i < Li.nh(); ++i) exact = Li.ph(i) == 2 * Lo.ph(i);
     for (int j = 0; exact && j < Li.nw(); ++j) exact = Li.pw(j) == 2 * Lo.pw(j);
+    if (std::is_same<T, __nv_bfloat16>::value && g.L.kh == 3 && g.L.kw == 3 && g.L.sh == 2 && g.L.sw == 2 &&
+        !getenv("SPLITCNN_POOL_GENERIC")) {
+        pool3x3s2_fwd_bf16_kernel<<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
+                                                        (const __nv_bfloat16 *)x, (__nv_bfloat16 *)y, a, p0, relu_bit);
+        count_launch();
+        return;
+    }
     if (exact) {
         pool2x2_fwd_bf16_kernel<<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), (const __nv_bfloat16 *)x,
                                                       (__nv_bfloat16 *)y, a, p0, relu_bit);

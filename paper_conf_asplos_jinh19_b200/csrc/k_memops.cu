@@ -323,6 +323,7 @@ __global__ void __launch_bounds__(256) pool_bwd_k3s2_kernel(LevelDesc Li, LevelD
                 load8(dY + o, g[t]);
             }
         }
+        const uint32_t keep = relu_bit ? 0xFFFFFFFFu : 0x7F7F7F7Fu;
 #pragma unroll
         for (int py = 0; py < 2; ++py)
 #pragma unroll
@@ -337,10 +338,12 @@ __global__ void __launch_bounds__(256) pool_bwd_k3s2_kernel(LevelDesc Li, LevelD
                     const int dh = t >> 1, dw = t & 1;
                     if (!in[t] || (dh && !py) || (dw && !px)) continue;   // window (a+dh, b+dw) covers the pixel?
                     const int idx = (1 + py - 2 * dh) * 3 + (1 + px - 2 * dw);
+                    // hit bytes by one packed compare per 4 argmax bytes (| 0x80 when the ReLU bit gates)
+                    const uint32_t tgt = (uint32_t)(idx | (relu_bit ? 0x80 : 0)) * 0x01010101u;
+                    const uint32_t e_lo = __vcmpeq4(am[t].x & keep, tgt), e_hi = __vcmpeq4(am[t].y & keep, tgt);
 #pragma unroll
                     for (int k = 0; k < 8; ++k) {
-                        const uint32_t bt = ((k < 4 ? am[t].x : am[t].y) >> (8 * (k & 3))) & 0xffu;
-                        const bool hit = (int)(bt & 0x7fu) == idx && (!relu_bit || (bt & 0x80u));
+                        const bool hit = ((k < 4 ? e_lo : e_hi) >> (8 * (k & 3))) & 1u;
                         acc[k] += hit ? g[t][k] : 0.f;
                     }
                 }

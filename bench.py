@@ -141,7 +141,7 @@ def run_ours(args):
     elif use_offload:
         from paper_conf_asplos_jinh19_b200.offload import OffloadSplitNet
         net = OffloadSplitNet(c["layers"], c["tail"], c["N"], 3, c["H"], c["W"], split=c["split"], mode=c["mode"],
-                              omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype)
+                              omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype, static_pool=args.static_pool)
     else:
         net = SplitNet(c["layers"], c["tail"], c["N"], c.get("C", 3), c["H"], c["W"], split=c["split"], mode=c["mode"],
                        omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype, static_pool=args.static_pool,

@@ -193,6 +193,8 @@ class SplitNet:
 
     def _tso_bytes(self, name):
         kind, key, m = name
+        if kind in ("aF", "aB"):                           # the two halves of an offloaded level
+            kind = "a"
         plan = self.region if key == "r" else self.tail
         es = 2 if self.dtype == sc.BF16 else 4
         if kind == "am":
@@ -201,11 +203,8 @@ class SplitNet:
             return 0                                       # a fused pair's conv output is never stored
         return plan.level_elems(m) * es
 
-    def _alloc_static(self):
-        """Place every activation, argmax and gradient TSO of the step in ONE device arena with the
-        library's first-fit static planner (splitcnn_memplan, P:287): each lives only from the op
-        that first touches it to the op that last does, so backward gradients reuse the space of
-        activations whose last use has passed."""
+    def _tso_lifetimes(self):
+        """(schedule, TSO names in first-use order, first use, last use) of one step."""
         sched = self._tso_schedule()
         names, first, last = [], {}, {}
         for t, (_, ts) in enumerate(sched):
@@ -214,6 +213,15 @@ class SplitNet:
                     first[n] = t
                     names.append(n)
                 last[n] = t
+        return sched, names, first, last
+
+    def _alloc_static(self, lifetimes=None):
+        """Place every activation, argmax and gradient TSO of the step in ONE device arena with the
+        library's first-fit static planner (splitcnn_memplan, P:287): each lives only from the op
+        that first touches it to the op that last does, so backward gradients reuse the space of
+        activations whose last use has passed.  `lifetimes` (names, first, last) overrides the plain
+        schedule scan (the offload executor splits offloaded levels into two TSOs)."""
+        names, first, last = lifetimes if lifetimes is not None else self._tso_lifetimes()[1:]
         nbytes = [self._tso_bytes(n) for n in names]
         offs, pool = sc.splitcnn_memplan(nbytes, [first[n] for n in names], [last[n] for n in names], 1024)
         self.arena = torch.empty(max(pool, 1024), dtype=torch.uint8, device=self.device)
@@ -225,7 +233,8 @@ class SplitNet:
             v = self.arena[o:o + b]
             views[n] = v if n[0] == "am" else v.view(td)
         empty = torch.zeros(0, dtype=td, device=self.device)
-        self.act_r = [views.get(("a", "r", m), empty) for m in range(self.region.nlayers + 1)]
+        self.static_views = views
+        self.act_r = [views.get(("a", "r", m), views.get(("aF", "r", m), empty)) for m in range(self.region.nlayers + 1)]
         self.act_t = ([views.get(("a", "t", m), empty) for m in range(self.tail.nlayers + 1)] if self.tail else [])
         self.argmax = {(n[1], n[2]): v for n, v in views.items() if n[0] == "am"}
         self.gbuf = {(n[1], n[2]): v for n, v in views.items() if n[0] == "g"}

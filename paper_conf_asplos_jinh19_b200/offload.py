@@ -79,6 +79,10 @@ class OffloadSplitNet(SplitNet):
         """Profiling stage: mean of `reps` timed executions per op; then Algorithm 1."""
         saved = self.offload_enabled
         self.offload_enabled = False
+        if self.static_pool and getattr(self, "_bwd_view", None) is not None:
+            torch.cuda.synchronize()
+            self._fwd_view = self._bwd_view = None
+            self._alloc_static()                        # back to the plain plan while profiling
         self.timers = []
         for _ in range(reps):
             self.forward(x)
@@ -133,15 +137,56 @@ class OffloadSplitNet(SplitNet):
         self._pending = []
         self._inflight = {}
         self._rr = 0
+        if self.static_pool:
+            self._alloc_static_offload()
         return self.stats
+
+    def _alloc_static_offload(self):
+        """HMMS static planning WITH the offload schedule (memory is held 'only for the minimum
+        duration required mandated both by the reference counter and the previously computed offloading
+        and prefetching scheme'): an offloaded level becomes two TSOs -- its forward life (producer op
+        .. the Algorithm-1 sync op that ends its D2H) and its backward life (the op whose prefetch
+        starts its H2D .. its last backward use) -- so the arena reuses its space in between."""
+        torch.cuda.synchronize()
+        sched, names, first, last = self._tso_lifetimes()
+        idx = {op: t for t, (op, _) in enumerate(sched)}
+        fname = lambda k, m: f"{k}{m}+pool" if (k, m) in self.fused else f"{k}{m}"
+        pending, freed_at = [], {}
+        for k, m in self._fwd_ops():                       # replay the forward hooks' bookkeeping
+            if self.offload_at.get((k, m)):
+                pending.append(m)
+            if self.sync_at.get((k, m)) and pending:
+                for lvl in pending:
+                    freed_at[lvl] = idx[fname(k, m)]
+                pending = []
+        pre_at = {lvl: idx[f"{k}{m}'"] for (k, m), lvls in self.prefetch_at.items() for lvl in lvls}
+        names2, first2, last2 = [], {}, {}
+        for n in names:
+            lvl = n[2]
+            if n[0] == "a" and n[1] == "r" and lvl in freed_at and lvl in pre_at:
+                nf, nb = ("aF", "r", lvl), ("aB", "r", lvl)
+                names2 += [nf, nb]
+                first2[nf], last2[nf] = first[n], max(first[n], freed_at[lvl])
+                first2[nb], last2[nb] = pre_at[lvl], last[n]
+            else:
+                names2.append(n)
+                first2[n], last2[n] = first[n], last[n]
+        self._alloc_static((names2, first2, last2))
+        self._fwd_view = {m: self.act_r[m] for m in range(len(self.act_r))}
+        self._bwd_view = {n[2]: v for n, v in self.static_views.items() if n[0] == "aB"}
 
     # ------------------------------------------------------------------ hooks
     def _ensure(self, m):
+        if self.act_r[m] is None and getattr(self, "_fwd_view", None) is not None:
+            self.act_r[m] = self._fwd_view[m]             # static arena: the level's (forward) view
+            return
         if self.act_r[m] is None:
             self.act_r[m] = torch.empty(self.level_bytes[m] // (2 if self.dtype == sc.BF16 else 4),
                                         dtype=self.tdtype, device=self.device)
 
     def forward(self, x, stream=None, x_layout: int = sc.NCHW):
+        if getattr(self, "_bwd_view", None) and not self.offload_enabled:
+            raise RuntimeError("the offload-aware static plan needs offload_enabled (re-run profile_and_plan)")
         self._ensure(0)
         if not (self.offload_enabled and self.plan_ready):
             for m in range(len(self.act_r)):
@@ -183,7 +228,8 @@ class OffloadSplitNet(SplitNet):
             cur = torch.cuda.current_stream()
             for lvl, done, mem in self._pending:
                 cur.wait_event(done)
-                self.act_r[lvl].record_stream(mem)
+                if getattr(self, "_fwd_view", None) is None:
+                    self.act_r[lvl].record_stream(mem)
                 self.act_r[lvl] = None
             self._pending = []
 
@@ -192,7 +238,9 @@ class OffloadSplitNet(SplitNet):
             return
         cur = torch.cuda.current_stream()
         for lvl in self.prefetch_at.get((key, m), []):
-            # moment 3: allocate and start H2D per patch
+            # moment 3: allocate (static arena: the level's backward view) and start H2D per patch
+            if getattr(self, "_bwd_view", None) is not None and lvl in self._bwd_view:
+                self.act_r[lvl] = self._bwd_view[lvl]
             self._ensure(lvl)
             ready = torch.cuda.Event()
             ready.record()
@@ -205,7 +253,8 @@ class OffloadSplitNet(SplitNet):
                                      self.act_r[lvl], ready if q == 0 else None, mem, None)
             done = torch.cuda.Event()
             done.record(mem)
-            self.act_r[lvl].record_stream(mem)
+            if getattr(self, "_fwd_view", None) is None:
+                self.act_r[lvl].record_stream(mem)
             self._inflight[lvl] = done
         if key == "r" and m in self._inflight:
             # moment 4: the compute stream waits right before the first backward use

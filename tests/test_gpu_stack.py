@@ -150,8 +150,9 @@ def test_dist_executor_world1_matches_single(sc):
     assert not bad, f"gradients differ: {bad}"
 
 
+@pytest.mark.parametrize("static", [False, True])
 @pytest.mark.parametrize("bw", [1e15, 2e9])
-def test_offload_prefetch_executor_bitwise(sc, bw):
+def test_offload_prefetch_executor_bitwise(sc, bw, static):
     """Offload/prefetch driven by Algorithm 1 must not change a single bit of the
     step's results; with an unbounded link every candidate is offloaded, with a slow one only what
     the ratio cap allows.  Device memory of freed levels is returned to the allocator."""
@@ -165,12 +166,15 @@ def test_offload_prefetch_executor_bitwise(sc, bw):
     x = torch.from_numpy(synth.uniform(g, (2, 3, H, H))).to("cuda", torch.bfloat16)
     kw = dict(split=c["split"], mode=c["mode"], omega=c["omega"], seed=c["seed"])
     plain = SplitNet(c["layers"], c["tail"], 2, 3, H, H, **kw)
-    off = OffloadSplitNet(c["layers"], c["tail"], 2, 3, H, H, **kw)
+    off = OffloadSplitNet(c["layers"], c["tail"], 2, 3, H, H, static_pool=static, **kw)
     plain.set_params(tp)
     off.set_params(tp)
     dy = torch.randn(plain.output_numel(), generator=torch.Generator().manual_seed(1)).to("cuda", torch.bfloat16)
+    pool0 = getattr(off, "pool_bytes", None)
     stats = off.profile_and_plan(x, dy, reps=2, bw=bw)
     assert stats["offloaded_bytes"] <= stats["cap_bytes"] + 1
+    if static:   # offloaded levels give their arena space back between the sync op and the prefetch
+        assert off.pool_bytes <= pool0
     if bw > 1e12:
         assert stats["offloaded_bytes"] == stats["candidate_bytes"] > 0
     for step in range(2):

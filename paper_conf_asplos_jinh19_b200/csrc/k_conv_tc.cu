@@ -86,8 +86,6 @@ struct TcConvParams {
     int uni;                      // every patch has the same tile grid: O(1) decode by fast division
     FastDiv fd_tpp, fd_mtpp, fd_nco, fd_nwb, fd_nhb;
     int ysh;                      // log2(ychunk)
-    int dstore;                   // two-group epilogue: 16-byte global stores straight from registers (no
-                                  // staging tile / TMA store; frees shared-memory bandwidth at small N)
     // fused 2x2 / stride-2 max-pool epilogue (POOL): pooled values + argmax bytes of level layer+2
     __nv_bfloat16 *pool_y;
     uint8_t *pool_a;
@@ -673,41 +671,6 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 aph ^= 1;
                 continue;
             }
-            if (p.dstore) {
-                // each thread owns one tile row = one output pixel: its channels are contiguous in HBM
-                const int wi = row % p.BW, hi = (row / p.BW) % p.BH, ni = row / (p.BW * p.BH);
-                const int n = n0 + ni, oh = oh0 + hi, ow = ow0 + wi;
-                const bool ok = valid && row < p.rows_box && n < p.N && oh < p.out_h[ql] && ow < p.out_w[ql];
-                const int64_t base = p.out_off[ql] + (((int64_t)n * p.out_h[ql] + oh) * p.out_w[ql] + ow) * p.Cpo + co0;
-                tc::mbar_wait(&tfull[g], aph);
-                tc::tc_fence_after();
-                const uint32_t tacc = tmem_base + (uint32_t)(g * p.BN) + ((uint32_t)(quad * 32) << 16);
-                for (int cc = 0; cc < ncols; cc += 32) {
-                    uint32_t r2[2][16];
-                    tc::tmem_ld16_nw(tacc + cc, r2[0]);
-                    tc::tmem_ld16_nw(tacc + cc + 16, r2[1]);
-                    uint4 m4[4];
-#pragma unroll
-                    for (int u = 0; u < 4; ++u)
-                        m4[u] = (MASK && ok) ? __ldg(reinterpret_cast<const uint4 *>(p.relu_src + base + cc + 8 * u))
-                                             : make_uint4(0, 0, 0, 0);
-                    tc::tmem_wait_ld();
-                    if (ok) {
-#pragma unroll
-                        for (int u = 0; u < 4; ++u)
-                            *reinterpret_cast<uint4 *>(p.y + base + cc + 8 * u) =
-                                epi8_full<BIAS, RELU, MASK>(r2[u >> 1] + 8 * (u & 1), sbias + co0 + cc + 8 * u, m4[u]);
-                    }
-                }
-                tc::tc_fence_before();
-                __syncwarp();
-                if (lane == 0) {
-                    if (CTA2) tc::mbar_arrive_remote(tempty_l);
-                    else tc::mbar_arrive(&tempty[g]);
-                }
-                aph ^= 1;
-                continue;
-            }
             if (gtid == 0) tc::bulk_wait_read0();      // this group's previous store has read the staging
             tc::named_bar_sync(1 + g, 128);
             if (MASK && valid) {
@@ -1243,9 +1206,6 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         if (P.bres && P.bres_bytes + 2u * P.ybuf_bytes + 2u * P.a_stage > 206u * 1024u) P.ybufs = 1;
         P.egroups = (P.ybufs == 2 && !getenv("SPLITCNN_ONE_EPI")) ? 2 : 1;
         if (ph && P.direct) return fail(SPLITCNN_ERR_UNSUPPORTED, "phase dgrad needs a TMA-store output");
-        // direct stores: whole 32-column groups of real channels, no phase view (plain patch strides)
-        P.dstore = (getenv("SPLITCNN_DSTORE") && !pool && !ph && !P.direct && P.egroups == 2 && BN % 32 == 0 &&
-                    ncols_out % BN == 0 && ncols_out == Lout.Cpad) ? 1 : 0;
         const uint32_t staging = P.ybufs * P.ybuf_bytes;
         P.stages = std::min<int>(8, (int)((210u * 1024u - staging - P.bres_bytes) / stage_bytes));
         P.bres_off = (uint32_t)P.stages * stage_bytes;

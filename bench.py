@@ -438,11 +438,12 @@ def run_reference(args):
     if rank != 0:
         return
     c = workload(args.config)
+    tiles = 4      # 4 of 64 output tiles of every layer-op per step (~2 s of oracle work): a stable estimate
     for _ in range(args.warmup):
-        oracle_sample_time(args.config, 1)
+        oracle_sample_time(args.config, tiles)
     vals, t0 = [], time.perf_counter()
     for _ in range(args.steps):
-        t_img, sample = oracle_sample_time(args.config, 1)
+        t_img, sample = oracle_sample_time(args.config, tiles)
         vals.append(t_img * c["N"])
     ms_step = 1e3 * statistics.mean(vals)
     value = c["N"] / (ms_step / 1e3)

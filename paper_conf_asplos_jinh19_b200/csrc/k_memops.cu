@@ -49,6 +49,18 @@ __global__ void __launch_bounds__(256) split_kernel(LevelDesc L, const T *__rest
                 v[k] = (cc < L.C) ? to_f(x[(((int64_t)n * C4 + (cc >> 2)) * H2 + 2 * hg + ((cc >> 1) & 1)) * W2 + 2 * wg + (cc & 1)])
                                   : 0.f;
             }
+        } else if (NCHW && std::is_same<T, __nv_bfloat16>::value) {
+            // bf16 NCHW: raw 16-bit gathers from up to 8 channel planes packed into one 16-byte store
+            const uint16_t *src = reinterpret_cast<const uint16_t *>(x) + (((int64_t)n * L.C + c0) * L.H + hg) * L.W + wg;
+            const int64_t cs = (int64_t)L.H * L.W;
+            const int nc = min(8, L.C - c0);
+            uint32_t w4[4] = {0u, 0u, 0u, 0u};
+#pragma unroll
+            for (int k = 0; k < 8; ++k)
+                if (k < nc) w4[k >> 1] |= (uint32_t)__ldg(src + k * cs) << (16 * (k & 1));
+            *reinterpret_cast<uint4 *>(P + g.off + (((int64_t)n * g.hp + h) * g.wp + w) * L.Cpad + c0) =
+                make_uint4(w4[0], w4[1], w4[2], w4[3]);
+            continue;
         } else if (NCHW) {
 #pragma unroll
             for (int k = 0; k < 8; ++k)

@@ -219,7 +219,11 @@ SPLITCNN_API splitcnn_status_t splitcnn_conv_pool_supported(splitcnn_plan_t plan
 /* Data gradient (adjoint of Eq. 6 within each patch):
  *   dX_p[n,h,w,ci] = sum over co, r, c with oh = (h + pt - r)/sh integral and in range
  *                    of dY_p[n,oh,ow,co] W[co,r,c,ci],   then * [relu_src > 0] if relu_src.
- * dy: level layer+1; dx, relu_src (nullable): level `layer`.  ws: splitcnn_workspace_size(op=1). */
+ * dy: level layer+1; dx, relu_src (nullable): level `layer`.  ws: splitcnn_workspace_size(op=1).
+ * BF16 runs on tcgen05: stride 1 as the forward kernel with 180-degree-rotated weights, stride 2 by
+ * output phase (S*S stride-1 correlations with tap subsets written through strided dX views; phases
+ * no tap reaches, k < s, are zero-filled).  The bias / column-sum work of conv_bwd_filter may run on a
+ * library side stream that is joined back before the call's work completes in `stream` order. */
 SPLITCNN_API splitcnn_status_t splitcnn_conv_bwd_data(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
                                          const void *dy, const void *w, void *dx, const void *relu_src,
                                          void *ws, size_t ws_bytes, uint32_t flags,
@@ -229,7 +233,9 @@ SPLITCNN_API splitcnn_status_t splitcnn_conv_bwd_data(splitcnn_plan_t plan, int3
  *   dW[co,r,c,ci] = beta * dW + sum_p sum_{n,oh,ow} dY_p[n,oh,ow,co] X~_p[n, oh*sh-pt+r, ow*sw-pl+c, ci]
  *   db[co]        = beta * db + sum_p sum_{n,oh,ow} dY_p[n,oh,ow,co]          (db nullable)
  * beta is 0 (overwrite) or 1 (accumulate).  The summation order is fixed (deterministic
- * run to run).  ws: splitcnn_workspace_size(op=2); ERR_INVALID_VALUE if too small. */
+ * run to run).  ws: splitcnn_workspace_size(op=2); ERR_INVALID_VALUE if too small.  With db, the dY
+ * column sums run concurrently on a library-owned side stream (event fork after the work already in
+ * `stream`, joined back into `stream` before return): stream semantics and graph capture are kept. */
 SPLITCNN_API splitcnn_status_t splitcnn_conv_bwd_filter(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
                                            const void *x, const void *dy, float *dw, float *db,
                                            float beta, void *ws, size_t ws_bytes, uint32_t flags,

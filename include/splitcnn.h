@@ -222,8 +222,7 @@ SPLITCNN_API splitcnn_status_t splitcnn_conv_pool_supported(splitcnn_plan_t plan
  * dy: level layer+1; dx, relu_src (nullable): level `layer`.  ws: splitcnn_workspace_size(op=1).
  * BF16 runs on tcgen05: stride 1 as the forward kernel with 180-degree-rotated weights, stride 2 by
  * output phase (S*S stride-1 correlations with tap subsets written through strided dX views; phases
- * no tap reaches, k < s, are zero-filled).  The bias / column-sum work of conv_bwd_filter may run on a
- * library side stream that is joined back before the call's work completes in `stream` order. */
+ * no tap reaches, k < s, are zero-filled). */
 SPLITCNN_API splitcnn_status_t splitcnn_conv_bwd_data(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
                                          const void *dy, const void *w, void *dx, const void *relu_src,
                                          void *ws, size_t ws_bytes, uint32_t flags,

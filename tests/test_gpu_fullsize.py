@@ -1,0 +1,114 @@
+"""Parity at BASELINE.json's full size, in the launch configuration bench.py times:
+C5's conv1_2 -> pool1 (N=256, 64 channels, 224x224, 8x8 split) through the same calls the executor
+makes (conv_pool_fwd, bwd_data with the ReLU mask, bwd_filter with db).  Image n of the batch is the
+seeded base image times an exact bf16 scale s_n (and dY image n the base gradient times t_n), so
+  * forward / data gradient are checked on sampled (image, patch) pairs against the oracle one by one;
+  * the weight gradient, a sum over all 256 images and 64 patches, equals (sum_n s_n t_n) * dW(base)
+    by linearity, and the oracle computes dW(base) over all 64 patches of one image."""
+import numpy as np
+import pytest
+
+import synth
+from oracle import ops as O
+from oracle import plan as OP
+from tests.helpers import normwise
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+N, C, H = 256, 64, 224
+
+
+@pytest.fixture(scope="module")
+def sc():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import __graft_entry__
+    __graft_entry__.build()
+    from paper_conf_asplos_jinh19_b200 import splitcnn
+    return splitcnn
+
+
+def _scales(n, off, every=2):
+    """Exact bf16 scales: powers of two, negative on every `every`-th image (distinct per image group)."""
+    return np.array([(-1.0 if (i + off) % every == every - 1 else 1.0) * 2.0 ** (((i + off) // 2) % 3 - 1)
+                     for i in range(n)])
+
+
+def _fill_level(lv, base_chw, scales, device="cuda"):
+    """Level buffer (bf16) of N scaled copies of one CHW image, patch-major NHWC (layout glue)."""
+    Cp, W = lv["Cpad"], lv["W"]
+    buf = torch.zeros(lv["total_elems"], dtype=torch.bfloat16, device=device)
+    s = torch.from_numpy(scales.astype(np.float32)).to(device)
+    bh, bw = lv["bh"], lv["bw"]
+    for i in range(lv["n_h"]):
+        hp = bh[i + 1] - bh[i]
+        for j in range(lv["n_w"]):
+            wp = bw[j + 1] - bw[j]
+            off = N * Cp * (bh[i] * W + hp * bw[j])
+            blk = torch.zeros((hp, wp, Cp), dtype=torch.float32, device=device)
+            blk[..., :base_chw.shape[0]] = torch.from_numpy(
+                np.ascontiguousarray(base_chw[:, bh[i]:bh[i + 1], bw[j]:bw[j + 1]].transpose(1, 2, 0))).to(device)
+            buf[off:off + N * hp * wp * Cp] = (s[:, None, None, None] * blk[None]).reshape(-1).to(torch.bfloat16)
+    return buf
+
+
+def _patch(buf, lv, i, j, n):
+    Cp, W = lv["Cpad"], lv["W"]
+    bh, bw = lv["bh"], lv["bw"]
+    hp, wp = bh[i + 1] - bh[i], bw[j + 1] - bw[j]
+    off = N * Cp * (bh[i] * W + hp * bw[j]) + n * hp * wp * Cp
+    return buf[off:off + hp * wp * Cp].float().cpu().numpy().reshape(hp, wp, Cp).transpose(2, 0, 1)[None].astype(np.float64)
+
+
+def test_c5_conv1_2_full_size(sc):
+    from paper_conf_asplos_jinh19_b200.net import pack_weight
+    from paper_conf_asplos_jinh19_b200.plan import SplitPlan
+    layers = [synth.conv(C, C, name="conv1_2"), synth.maxpool(C, name="pool1")]
+    Ob = sc.splitcnn_boundaries_even(112, 8)
+    pl = SplitPlan(layers, N, C, H, H, Ob, Ob)
+    assert sc.splitcnn_conv_pool_supported(pl.handle, 0, sc.BF16)
+    lv0, lv1, lv2 = pl.levels
+    ref = OP.plan(layers, 1, C, H, H, Ob, Ob)
+    g = synth.rng(44)
+    base = synth.to_bf16_f32(synth.uniform(g, (C, H, H))).astype(np.float64)
+    Wt = synth.to_bf16_f32(synth.kaiming(g, C, C, 3, 3)).astype(np.float64)
+    b = synth.uniform(g, (C,), -0.1, 0.1).astype(np.float64)
+    gbase = synth.to_bf16_f32(synth.normal(g, (C, H, H))).astype(np.float64)
+    s, t = _scales(N, 0), _scales(N, 1, every=4)     # sum(t) and sum(s t) far from 0 (no cancellation)
+    x = _fill_level(lv0, base, s)
+    dy = _fill_level(lv1, gbase, t)
+    w = pack_weight(torch.from_numpy(Wt), lv0["Cpad"], torch.bfloat16).cuda().contiguous()
+    bias = torch.from_numpy(b.astype(np.float32)).cuda()
+    yp = torch.empty(lv2["total_elems"], dtype=torch.bfloat16, device="cuda")
+    am = torch.empty(lv2["total_elems"], dtype=torch.uint8, device="cuda")
+    sc.splitcnn_conv_pool_fwd(pl.handle, 0, sc.BF16, x, w, bias, yp, am)
+    ws_b = max(pl.workspace_size(0, sc.BF16, 1), pl.workspace_size(0, sc.BF16, 2))
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    dx = torch.empty_like(x)
+    sc.splitcnn_conv_bwd_data(pl.handle, 0, sc.BF16, dy, w, dx, x, ws, ws_b)
+    dw = torch.zeros((C, 3, 3, lv0["Cpad"]), dtype=torch.float32, device="cuda")
+    db = torch.zeros(C, dtype=torch.float32, device="cuda")
+    sc.splitcnn_conv_bwd_filter(pl.handle, 0, sc.BF16, x, dy, dw, db, 0.0, ws, ws_b)
+    torch.cuda.synchronize()
+    lp0, lp1 = ref.layers
+    for n, i, j in ((0, 0, 0), (137, 3, 5), (255, 7, 7), (64, 7, 0)):
+        X = base[:, lp0.Ih[i]:lp0.Ih[i + 1], lp0.Iw[j]:lp0.Iw[j + 1]][None] * s[n]
+        Y = O.conv_fwd_patch(X, Wt, b, 1, 1, lp0.pads_h[i], lp0.pads_w[j], relu=True)
+        Yb = synth.to_bf16_f32(Y.astype(np.float32)).astype(np.float64)   # the GPU pools the bf16 conv outputs
+        P, A = O.pool_fwd_patch(Yb, 2, 2, 2, 2, lp1.pads_h[i], lp1.pads_w[j])
+        got = _patch(yp, lv2, i, j, n)[:, :C]
+        assert normwise(got, P) <= 2e-2, (n, i, j)
+        Ag = _patch(am, lv2, i, j, n)[:, :C].astype(np.int64) & 0x7F
+        assert np.mean(Ag != A) < 1e-2, (n, i, j)           # equal up to bf16 near-ties (R9, R13)
+        G = gbase[:, lp0.Ih[i]:lp0.Ih[i + 1], lp0.Iw[j]:lp0.Iw[j + 1]][None] * t[n]
+        dX = O.conv_bwd_data_patch(G, Wt, X.shape[2], X.shape[3], 1, 1, lp0.pads_h[i], lp0.pads_w[j], mask=X)
+        assert normwise(_patch(dx, lv0, i, j, n)[:, :C], dX) <= 2e-2, (n, i, j)
+    # weight / bias gradient over all 256 images and 64 patches, by linearity in the per-image scales
+    Xp = O.split(base[None], lp0.Ih, lp0.Iw)
+    Gp = O.split(gbase[None], lp0.Ih, lp0.Iw)
+    dW1, db1 = O.conv_bwd_filter(Xp, Gp, lp0)
+    st, tt = float(np.sum(s * t)), float(np.sum(t))
+    dWg = dw[..., :C].permute(0, 3, 1, 2).double().cpu().numpy()
+    assert normwise(dWg, st * dW1) <= 2e-2
+    assert normwise(db.double().cpu().numpy(), tt * db1) <= 2e-2

@@ -112,3 +112,49 @@ def test_c5_conv1_2_full_size(sc):
     dWg = dw[..., :C].permute(0, 3, 1, 2).double().cpu().numpy()
     assert normwise(dWg, st * dW1) <= 2e-2
     assert normwise(db.double().cpu().numpy(), tt * db1) <= 2e-2
+
+
+@pytest.mark.parametrize("name,Cin,Cout,Hin,nsplit", [("conv3_2", 256, 256, 56, 8), ("conv4_2", 512, 512, 28, 1)])
+def test_c5_deep_layers_full_size(sc, name, Cin, Cout, Hin, nsplit):
+    """C5's conv3_2 (split region: 7x7 patches, 2-CTA halo kernels) and conv4_2 (unsplit tail) at N=256:
+    conv_fwd (+bias+ReLU), bwd_data (ReLU mask), bwd_filter (+db) as the executor calls them."""
+    from paper_conf_asplos_jinh19_b200.net import pack_weight
+    from paper_conf_asplos_jinh19_b200.plan import SplitPlan
+    l = synth.conv(Cin, Cout, name=name)
+    Ob = sc.splitcnn_boundaries_even(Hin, nsplit)
+    pl = SplitPlan([l], N, Cin, Hin, Hin, Ob, Ob)
+    lv0, lv1 = pl.levels
+    lp = OP.plan([l], 1, Cin, Hin, Hin, Ob, Ob).layers[0]
+    g = synth.rng(45 + Cin)
+    base = synth.to_bf16_f32(synth.uniform(g, (Cin, Hin, Hin))).astype(np.float64)
+    Wt = synth.to_bf16_f32(synth.kaiming(g, Cout, Cin, 3, 3)).astype(np.float64)
+    b = synth.uniform(g, (Cout,), -0.1, 0.1).astype(np.float64)
+    gbase = synth.to_bf16_f32(synth.normal(g, (Cout, Hin, Hin))).astype(np.float64)
+    s, t = _scales(N, 0), _scales(N, 1, every=4)
+
+    x = _fill_level(lv0, base, s)
+    dy = _fill_level(lv1, gbase, t)
+    w = pack_weight(torch.from_numpy(Wt), lv0["Cpad"], torch.bfloat16).cuda().contiguous()
+    bias = torch.from_numpy(b.astype(np.float32)).cuda()
+    y = torch.empty(lv1["total_elems"], dtype=torch.bfloat16, device="cuda")
+    sc.splitcnn_conv_fwd(pl.handle, 0, sc.BF16, x, w, bias, y, sc.FLAG_RELU)
+    ws_b = max(pl.workspace_size(0, sc.BF16, 1), pl.workspace_size(0, sc.BF16, 2))
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    dx = torch.empty_like(x)
+    sc.splitcnn_conv_bwd_data(pl.handle, 0, sc.BF16, dy, w, dx, x, ws, ws_b)
+    dw = torch.zeros((Cout, 3, 3, lv0["Cpad"]), dtype=torch.float32, device="cuda")
+    db = torch.zeros(Cout, dtype=torch.float32, device="cuda")
+    sc.splitcnn_conv_bwd_filter(pl.handle, 0, sc.BF16, x, dy, dw, db, 0.0, ws, ws_b)
+    torch.cuda.synchronize()
+    last = nsplit - 1
+    for n, i, j in ((3, 0, 0), (200, last, last), (129, last // 2, 0)):
+        X = base[:, lp.Ih[i]:lp.Ih[i + 1], lp.Iw[j]:lp.Iw[j + 1]][None] * s[n]
+        Y = O.conv_fwd_patch(X, Wt, b, 1, 1, lp.pads_h[i], lp.pads_w[j], relu=True)
+        assert normwise(_patch(y, lv1, i, j, n)[:, :Cout], Y) <= 2e-2, (n, i, j)
+        G = gbase[:, lp.Oh[i]:lp.Oh[i + 1], lp.Ow[j]:lp.Ow[j + 1]][None] * t[n]
+        dX = O.conv_bwd_data_patch(G, Wt, X.shape[2], X.shape[3], 1, 1, lp.pads_h[i], lp.pads_w[j], mask=X)
+        assert normwise(_patch(dx, lv0, i, j, n)[:, :Cin], dX) <= 2e-2, (n, i, j)
+    dW1, db1 = O.conv_bwd_filter(O.split(base[None], lp.Ih, lp.Iw), O.split(gbase[None], lp.Oh, lp.Ow), lp)
+    dWg = dw[..., :Cin].permute(0, 3, 1, 2).double().cpu().numpy()
+    assert normwise(dWg, float(np.sum(s * t)) * dW1) <= 2e-2
+    assert normwise(db.double().cpu().numpy(), float(np.sum(t)) * db1) <= 2e-2

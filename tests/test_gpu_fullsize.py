@@ -158,3 +158,72 @@ def test_c5_deep_layers_full_size(sc, name, Cin, Cout, Hin, nsplit):
     dWg = dw[..., :Cin].permute(0, 3, 1, 2).double().cpu().numpy()
     assert normwise(dWg, float(np.sum(s * t)) * dW1) <= 2e-2
     assert normwise(db.double().cpu().numpy(), float(np.sum(t)) * db1) <= 2e-2
+
+
+def test_c3_stride2_and_stem_full_size(sc):
+    """C3 at N=256: layer2_0_a (3x3 s2, 64->128, 56->28, 2x2 split; phase-decomposed tcgen05 dgrad) and
+    the stem (7x7 s2 on 3 channels run as the space-to-depth 4x4 s1 conv: NCHW_S2D split + conv), same
+    sampled-pair / linearity checks against the oracle's own 7x7 s2 / 3x3 s2 definitions."""
+    from paper_conf_asplos_jinh19_b200.net import pack_weight
+    from paper_conf_asplos_jinh19_b200.plan import SplitPlan
+    from paper_conf_asplos_jinh19_b200.resnet import s2d_stem_grad, s2d_stem_layer, s2d_stem_weight
+    g = synth.rng(46)
+    s, t = _scales(N, 0), _scales(N, 1, every=4)
+    # ---- layer2_0_a: 3x3 s2 p1, 64 -> 128
+    l = synth.conv(64, 128, s=2, name="layer2_0_a")
+    Ob = sc.splitcnn_boundaries_even(28, 2)
+    pl = SplitPlan([l], N, 64, 56, 56, Ob, Ob)
+    lv0, lv1 = pl.levels
+    lp = OP.plan([l], 1, 64, 56, 56, Ob, Ob).layers[0]
+    base = synth.to_bf16_f32(synth.uniform(g, (64, 56, 56))).astype(np.float64)
+    Wt = synth.to_bf16_f32(synth.kaiming(g, 128, 64, 3, 3)).astype(np.float64)
+    gbase = synth.to_bf16_f32(synth.normal(g, (128, 28, 28))).astype(np.float64)
+    x, dy = _fill_level(lv0, base, s), _fill_level(lv1, gbase, t)
+    w = pack_weight(torch.from_numpy(Wt), lv0["Cpad"], torch.bfloat16).cuda().contiguous()
+    y = torch.empty(lv1["total_elems"], dtype=torch.bfloat16, device="cuda")
+    sc.splitcnn_conv_fwd(pl.handle, 0, sc.BF16, x, w, None, y, sc.FLAG_RELU)
+    ws_b = max(pl.workspace_size(0, sc.BF16, 1), pl.workspace_size(0, sc.BF16, 2))
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    dx = torch.empty_like(x)
+    sc.splitcnn_conv_bwd_data(pl.handle, 0, sc.BF16, dy, w, dx, x, ws, ws_b)
+    dw = torch.zeros((128, 3, 3, lv0["Cpad"]), dtype=torch.float32, device="cuda")
+    sc.splitcnn_conv_bwd_filter(pl.handle, 0, sc.BF16, x, dy, dw, None, 0.0, ws, ws_b)
+    torch.cuda.synchronize()
+    for n, i, j in ((5, 0, 1), (250, 1, 1)):
+        X = base[:, lp.Ih[i]:lp.Ih[i + 1], lp.Iw[j]:lp.Iw[j + 1]][None] * s[n]
+        Y = O.conv_fwd_patch(X, Wt, None, 2, 2, lp.pads_h[i], lp.pads_w[j], relu=True)
+        assert normwise(_patch(y, lv1, i, j, n)[:, :128], Y) <= 2e-2, (n, i, j)
+        G = gbase[:, lp.Oh[i]:lp.Oh[i + 1], lp.Ow[j]:lp.Ow[j + 1]][None] * t[n]
+        dX = O.conv_bwd_data_patch(G, Wt, X.shape[2], X.shape[3], 2, 2, lp.pads_h[i], lp.pads_w[j], mask=X)
+        assert normwise(_patch(dx, lv0, i, j, n)[:, :64], dX) <= 2e-2, (n, i, j)
+    dW1, _ = O.conv_bwd_filter(O.split(base[None], lp.Ih, lp.Iw), O.split(gbase[None], lp.Oh, lp.Ow), lp)
+    assert normwise(dw[..., :64].permute(0, 3, 1, 2).double().cpu().numpy(), float(np.sum(s * t)) * dW1) <= 2e-2
+    # ---- the stem: 7x7 s2 p3 on 3 channels through the space-to-depth split and 4x4 s1 conv
+    l7 = synth.conv(3, 64, k=7, s=2, p=3, name="conv1")
+    Ob = sc.splitcnn_boundaries_even(112, 2)
+    ls = s2d_stem_layer(l7)
+    pls = SplitPlan([ls], N, 12, 112, 112, Ob, Ob)
+    lvs0, lvs1 = pls.levels
+    lp7 = OP.plan([l7], 1, 3, H, H, Ob, Ob).layers[0]
+    img = synth.to_bf16_f32(synth.uniform(g, (3, H, H))).astype(np.float64)
+    W7 = synth.to_bf16_f32(synth.kaiming(g, 64, 3, 7, 7)).astype(np.float64)
+    gst = synth.to_bf16_f32(synth.normal(g, (64, 112, 112))).astype(np.float64)
+    xf = (torch.from_numpy(s.astype(np.float32))[:, None, None, None] * torch.from_numpy(img.astype(np.float32))[None]
+          ).to("cuda", torch.bfloat16).contiguous()
+    xs = torch.empty(lvs0["total_elems"], dtype=torch.bfloat16, device="cuda")
+    sc.splitcnn_split(pls.handle, 0, sc.BF16, xf, sc.NCHW_S2D, xs)
+    ws7 = pack_weight(s2d_stem_weight(torch.from_numpy(W7)), lvs0["Cpad"], torch.bfloat16).cuda().contiguous()
+    ys = torch.empty(lvs1["total_elems"], dtype=torch.bfloat16, device="cuda")
+    sc.splitcnn_conv_fwd(pls.handle, 0, sc.BF16, xs, ws7, None, ys, sc.FLAG_RELU)
+    dys = _fill_level(lvs1, gst, t)
+    wsb = max(pls.workspace_size(0, sc.BF16, 2), 16)
+    wss = torch.empty(wsb, dtype=torch.uint8, device="cuda")
+    dws = torch.zeros((64, 4, 4, lvs0["Cpad"]), dtype=torch.float32, device="cuda")
+    sc.splitcnn_conv_bwd_filter(pls.handle, 0, sc.BF16, xs, dys, dws, None, 0.0, wss, wsb)
+    torch.cuda.synchronize()
+    for n, i, j in ((1, 0, 0), (254, 1, 0)):
+        X = img[:, lp7.Ih[i]:lp7.Ih[i + 1], lp7.Iw[j]:lp7.Iw[j + 1]][None] * s[n]
+        Y = O.conv_fwd_patch(X, W7, None, 2, 2, lp7.pads_h[i], lp7.pads_w[j], relu=True)
+        assert normwise(_patch(ys, lvs1, i, j, n)[:, :64], Y) <= 2e-2, (n, i, j)
+    dW7, _ = O.conv_bwd_filter(O.split(img[None], lp7.Ih, lp7.Iw), O.split(gst[None], lp7.Oh, lp7.Ow), lp7)
+    assert normwise(s2d_stem_grad(dws, 3).double().cpu().numpy(), float(np.sum(s * t)) * dW7) <= 2e-2

@@ -227,3 +227,45 @@ def test_c3_stride2_and_stem_full_size(sc):
         assert normwise(_patch(ys, lvs1, i, j, n)[:, :64], Y) <= 2e-2, (n, i, j)
     dW7, _ = O.conv_bwd_filter(O.split(img[None], lp7.Ih, lp7.Iw), O.split(gst[None], lp7.Oh, lp7.Ow), lp7)
     assert normwise(s2d_stem_grad(dws, 3).double().cpu().numpy(), float(np.sum(s * t)) * dW7) <= 2e-2
+
+
+def test_c5_split_merge_pool_full_size(sc):
+    """Bit-exact HBM ops at full size: the C5 input split / merge round trip (N=256, 3x224x224, 8x8,
+    NCHW), and the standalone 2x2 pool (pool2 geometry: N=256, 128 channels, 112x112, 8x8) forward
+    values + argmax and backward on sampled (image, patch) pairs against the oracle."""
+    from paper_conf_asplos_jinh19_b200.plan import SplitPlan
+    Ob = sc.splitcnn_boundaries_even(224, 8)
+    pl = SplitPlan([synth.conv(3, 64)], N, 3, H, H, Ob, Ob)
+    gen = torch.Generator(device="cpu").manual_seed(47)
+    x = (torch.rand((N, 3, H, H), generator=gen) * 2 - 1).to("cuda", torch.bfloat16)
+    p = torch.empty(pl.levels[0]["total_elems"], dtype=torch.bfloat16, device="cuda")
+    sc.splitcnn_split(pl.handle, 0, sc.BF16, x, sc.NCHW, p)
+    back = torch.empty_like(x)
+    sc.splitcnn_merge(pl.handle, 0, sc.BF16, p, back, sc.NCHW)
+    torch.cuda.synchronize()
+    assert torch.equal(back, x)
+    # 2x2 pool at pool2's geometry
+    lpool = synth.maxpool(128)
+    Op = sc.splitcnn_boundaries_even(56, 8)
+    pp = SplitPlan([lpool], N, 128, 112, 112, Op, Op)
+    lv0, lv1 = pp.levels
+    lref = OP.plan([lpool], 1, 128, 112, 112, Op, Op).layers[0]
+    g = synth.rng(48)
+    base = synth.to_bf16_f32(synth.normal(g, (128, 112, 112))).astype(np.float64)
+    gb = synth.to_bf16_f32(synth.normal(g, (128, 56, 56))).astype(np.float64)
+    s, t = _scales(N, 0), _scales(N, 1, every=4)
+    xin, dy = _fill_level(lv0, base, s), _fill_level(lv1, gb, t)
+    y = torch.empty(lv1["total_elems"], dtype=torch.bfloat16, device="cuda")
+    a = torch.empty(lv1["total_elems"], dtype=torch.uint8, device="cuda")
+    sc.splitcnn_pool_fwd(pp.handle, 0, sc.BF16, xin, y, a, 0)
+    dx = torch.empty_like(xin)
+    sc.splitcnn_pool_bwd(pp.handle, 0, sc.BF16, dy, a, dx, 0)
+    torch.cuda.synchronize()
+    for n, i, j in ((0, 0, 0), (255, 7, 7), (77, 2, 5)):
+        X = base[:, lref.Ih[i]:lref.Ih[i + 1], lref.Iw[j]:lref.Iw[j + 1]][None] * s[n]
+        Y, A = O.pool_fwd_patch(X, 2, 2, 2, 2, lref.pads_h[i], lref.pads_w[j])
+        assert np.array_equal(_patch(y, lv1, i, j, n)[:, :128], Y), (n, i, j)
+        assert np.array_equal(_patch(a, lv1, i, j, n)[:, :128].astype(np.int64) & 0x7F, A), (n, i, j)
+        G = gb[:, lref.Oh[i]:lref.Oh[i + 1], lref.Ow[j]:lref.Ow[j + 1]][None] * t[n]
+        dX = O.pool_bwd_patch(G, A, X.shape[2], X.shape[3], 2, 2, 2, 2, lref.pads_h[i], lref.pads_w[j])
+        assert np.array_equal(_patch(dx, lv0, i, j, n)[:, :128], dX), (n, i, j)

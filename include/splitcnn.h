@@ -181,6 +181,13 @@ SPLITCNN_API splitcnn_status_t splitcnn_split(splitcnn_plan_t plan, int32_t leve
                                  int32_t p0, int32_t p1, splitcnn_stream_t stream);
 
 /* Eq. 7: concatenate the level's patch buffers into the full tensor y. */
+/* Space-to-depth(2) split of an NCHW tensor with x_channels channels and 2H x 2W pixels into a level
+ * of C >= 4 * x_channels channels: level channel 4c + 2ph + pw of (h, w) = x[n, c, 2h + ph, 2w + pw],
+ * channels >= 4 * x_channels are zero (so a stride-2 stem can run as a stride-1 conv on a level padded
+ * to a tensor-core-friendly channel count).  Errors: x_channels < 1 or 4 * x_channels > C. */
+SPLITCNN_API splitcnn_status_t splitcnn_split_s2d(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                      const void *x, int32_t x_channels, void *patches,
+                                      int32_t p0, int32_t p1, splitcnn_stream_t stream);
 SPLITCNN_API splitcnn_status_t splitcnn_merge(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
                                  const void *patches, void *y, int32_t y_layout,
                                  int32_t p0, int32_t p1, splitcnn_stream_t stream);

@@ -128,6 +128,22 @@ extern "C" splitcnn_status_t splitcnn_split(splitcnn_plan_t plan, int32_t level,
     return check_launch("split");
 }
 
+extern "C" splitcnn_status_t splitcnn_split_s2d(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                                const void *x, int32_t x_channels, void *patches, int32_t p0,
+                                                int32_t p1, splitcnn_stream_t stream) {
+    if (!plan || level < 0 || level >= (int)plan->levels.size()) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad level");
+    TRY(check_dtype(dtype));
+    if (!x || !patches) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    if (x_channels < 1 || 4 * x_channels > plan->levels[level].C)
+        return fail(SPLITCNN_ERR_INVALID_VALUE, "split_s2d: need 1 <= x_channels and 4 * x_channels <= level C");
+    NEED_ALIGNED(x, "x");
+    NEED_ALIGNED(patches, "patches");
+    TRY(check_range(plan, level, p0, p1));
+    if (p1 == p0) return SPLITCNN_OK;
+    launch_split(dtype, plan->levels[level], x, SPLITCNN_NCHW_S2D, patches, p0, p1, (cudaStream_t)stream, x_channels);
+    return check_launch("split_s2d");
+}
+
 extern "C" splitcnn_status_t splitcnn_merge(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
                                             const void *patches, void *y, int32_t y_layout, int32_t p0, int32_t p1,
                                             splitcnn_stream_t stream) {

@@ -30,24 +30,45 @@ __device__ __forceinline__ void dec3(uint32_t u, const Dec3 &d, int &x0, int &x1
     x3 = (int)u;
 }
 template <typename T, bool NCHW, bool S2D = false>
-__global__ void __launch_bounds__(256) split_kernel(LevelDesc L, const T *__restrict__ x, T *__restrict__ P, int p0) {
+__global__ void __launch_bounds__(256) split_kernel(LevelDesc L, const T *__restrict__ x, T *__restrict__ P, int p0,
+                                                    int xc = 0) {
     const PatchGeo g = patch_geo(L, p0 + blockIdx.y);
     const int G = L.Cpad / 8;
     const uint32_t units = (uint32_t)L.N * g.hp * g.wp * G;
-    const Dec3 d = NCHW ? make_dec3(g.wp, g.hp, G) : make_dec3(G, g.wp, g.hp);
+    // NCHW: pixel-fastest (coalesced reads of each channel plane).  NHWC, and the space-to-depth split
+    // (whose level may be much wider than its input, e.g. 12 real of 64 channels): channel-fastest, so a
+    // warp writes whole 16-byte-group rows of consecutive pixels (coalesced stores)
+    constexpr bool PIXEL_FAST = NCHW && !S2D;
+    const Dec3 d = PIXEL_FAST ? make_dec3(g.wp, g.hp, G) : make_dec3(G, g.wp, g.hp);
     for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < units; u += gridDim.x * blockDim.x) {
         int n, h, w, cg;
-        if (NCHW) dec3(u, d, w, h, cg, n);   // pixel-fastest: coalesced reads of each channel plane
-        else dec3(u, d, cg, w, h, n);        // channel-fastest: coalesced 16 B reads and writes
+        if (PIXEL_FAST) dec3(u, d, w, h, cg, n);
+        else dec3(u, d, cg, w, h, n);
         const int hg = g.h0 + h, wg = g.w0 + w, c0 = cg * 8;
         float v[8];
-        if (S2D) {   // level channel 4c + 2ph + pw of (hg, wg) = x[n, c, 2hg + ph, 2wg + pw]
-            const int C4 = L.C >> 2, H2 = 2 * L.H, W2 = 2 * L.W;
+        if (S2D && std::is_same<T, __nv_bfloat16>::value) {   // raw 16-bit gathers; all-zero groups skip loads
+            const int H2 = 2 * L.H, W2 = 2 * L.W, cmax = min(L.C, 4 * xc);
+            uint32_t w4[4] = {0u, 0u, 0u, 0u};
+            if (c0 < cmax) {
+                const uint16_t *xb = reinterpret_cast<const uint16_t *>(x);
+#pragma unroll
+                for (int k = 0; k < 8; ++k) {
+                    const int cc = c0 + k;
+                    if (cc < cmax)
+                        w4[k >> 1] |= (uint32_t)__ldg(xb + (((int64_t)n * xc + (cc >> 2)) * H2 + 2 * hg + ((cc >> 1) & 1)) * W2 +
+                                                      2 * wg + (cc & 1)) << (16 * (k & 1));
+                }
+            }
+            *reinterpret_cast<uint4 *>(P + g.off + (((int64_t)n * g.hp + h) * g.wp + w) * L.Cpad + c0) =
+                make_uint4(w4[0], w4[1], w4[2], w4[3]);
+            continue;
+        } else if (S2D) {   // level channel 4c + 2ph + pw of (hg, wg) = x[n, c, 2hg + ph, 2wg + pw]  (c < xc; else 0)
+            const int C4 = xc, H2 = 2 * L.H, W2 = 2 * L.W, cmax = min(L.C, 4 * xc);
 #pragma unroll
             for (int k = 0; k < 8; ++k) {
                 const int cc = c0 + k;
-                v[k] = (cc < L.C) ? to_f(x[(((int64_t)n * C4 + (cc >> 2)) * H2 + 2 * hg + ((cc >> 1) & 1)) * W2 + 2 * wg + (cc & 1)])
-                                  : 0.f;
+                v[k] = (cc < cmax) ? to_f(x[(((int64_t)n * C4 + (cc >> 2)) * H2 + 2 * hg + ((cc >> 1) & 1)) * W2 + 2 * wg + (cc & 1)])
+                                   : 0.f;
             }
         } else if (NCHW && std::is_same<T, __nv_bfloat16>::value) {
             // bf16 NCHW: raw 16-bit gathers from up to 8 channel planes packed into one 16-byte store
@@ -128,12 +149,12 @@ static int64_t max_patch_units(const Level &L, int p0, int p1, int per_pixel) {
 }
 
 template <typename T>
-void launch_split_t(const Level &L, const void *x, int layout, void *P, int p0, int p1, cudaStream_t st) {
+void launch_split_t(const Level &L, const void *x, int layout, void *P, int p0, int p1, cudaStream_t st, int xc) {
     npatch_launch = p1 - p0;
     dim3 grid(grid_x_for(max_patch_units(L, p0, p1, L.Cpad / 8)), p1 - p0);
     LevelDesc d = make_level_desc(L);
     if (layout == SPLITCNN_NCHW_S2D)
-        { split_kernel<T, true, true><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0); count_launch(); }
+        { split_kernel<T, true, true><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0, xc > 0 ? xc : L.C / 4); count_launch(); }
     else if (layout == SPLITCNN_NCHW)
         { split_kernel<T, true><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0); count_launch(); }
     else
@@ -151,9 +172,10 @@ void launch_merge_t(const Level &L, const void *P, void *y, int layout, int p0, 
         { merge_kernel<T, false><<<grid, 256, 0, st>>>(d, (const T *)P, (T *)y, p0); count_launch(); }
 }
 
-void launch_split(splitcnn_dtype_t dt, const Level &L, const void *x, int layout, void *P, int p0, int p1, cudaStream_t st) {
-    if (dt == SPLITCNN_BF16) launch_split_t<__nv_bfloat16>(L, x, layout, P, p0, p1, st);
-    else launch_split_t<float>(L, x, layout, P, p0, p1, st);
+void launch_split(splitcnn_dtype_t dt, const Level &L, const void *x, int layout, void *P, int p0, int p1, cudaStream_t st,
+                  int xc) {
+    if (dt == SPLITCNN_BF16) launch_split_t<__nv_bfloat16>(L, x, layout, P, p0, p1, st, xc);
+    else launch_split_t<float>(L, x, layout, P, p0, p1, st, xc);
 }
 void launch_merge(splitcnn_dtype_t dt, const Level &L, const void *P, void *y, int layout, int p0, int p1, cudaStream_t st) {
     if (dt == SPLITCNN_BF16) launch_merge_t<__nv_bfloat16>(L, P, y, layout, p0, p1, st);

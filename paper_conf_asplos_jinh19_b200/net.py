@@ -285,8 +285,11 @@ class SplitNet:
         self.timers.append((kind, e0, e1, work, self._label))
 
     def _conv_work(self, plan, m, l):
+        """Algorithmic FLOPs of one pass (a re-expressed layer, e.g. the space-to-depth stem, carries the
+        MACs per output of the layer it implements in "macs_per_out")."""
         lo = plan.levels[m + 1]
-        return 2.0 * lo["N"] * l["cout"] * lo["H"] * lo["W"] * l["cin"] * l["kh"] * l["kw"]
+        macs = l.get("macs_per_out", l["cin"] * l["kh"] * l["kw"])
+        return 2.0 * lo["N"] * l["cout"] * lo["H"] * lo["W"] * macs
 
     def _bytes(self, plan, m):
         es = 2 if self.dtype == sc.BF16 else 4
@@ -422,7 +425,7 @@ class SplitNet:
                 if l["op"] != "conv":
                     continue
                 lo = plan.levels[m + 1]
-                f = 2 * lo["N"] * l["cout"] * lo["H"] * lo["W"] * l["cin"] * l["kh"] * l["kw"]
+                f = 2 * lo["N"] * l["cout"] * lo["H"] * lo["W"] * l.get("macs_per_out", l["cin"] * l["kh"] * l["kw"])
                 total += f * (2 if first and not self.input_grad else 3)
                 first = False
         return total

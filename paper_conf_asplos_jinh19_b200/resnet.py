@@ -17,6 +17,8 @@ BN (R11) is not part of the split stack.
 """
 from __future__ import annotations
 
+import os
+
 import torch
 
 from . import splitcnn as sc
@@ -24,12 +26,16 @@ from .net import SplitNet, pack_weight
 from .plan import SplitPlan
 
 
-def s2d_stem_layer(l: dict) -> dict:
+def s2d_stem_layer(l: dict, cin_pad: int = 0) -> dict:
     """The 7x7 s2 p3 stem on C channels as the equivalent 4x4 s1 conv on the space-to-depth(2) input
     (4C channels, H/2 x W/2): out[t] = sum_{q, phi} Xs2d[t + q - 2][phi] * W[2q + phi - 1] (tap -1 is
-    zero), i.e. begin pad 2, end pad 1 -- and under R2 the same patch-local pads (2, k - s - p_b = 1)."""
-    return dict(op="conv", kh=4, kw=4, sh=1, sw=1, ph_b=2, ph_e=1, pw_b=2, pw_e=1, cin=4 * l["cin"],
-                cout=l["cout"], relu=l.get("relu", True), name=l.get("name", "conv1"))
+    zero), i.e. begin pad 2, end pad 1 -- and under R2 the same patch-local pads (2, k - s - p_b = 1).
+    cin_pad > 4C declares zero channels up to cin_pad (64: the level takes the 64-channel halo /
+    2-CTA tensor-core kernels instead of the 16-channel per-tap path).  "macs_per_out" keeps the
+    algorithmic work of the 7x7 layer for the roofline accounting."""
+    return dict(op="conv", kh=4, kw=4, sh=1, sw=1, ph_b=2, ph_e=1, pw_b=2, pw_e=1, cin=max(4 * l["cin"], cin_pad),
+                cout=l["cout"], relu=l.get("relu", True), name=l.get("name", "conv1"),
+                macs_per_out=l["cin"] * l["kh"] * l["kw"])
 
 
 def s2d_stem_weight(W: torch.Tensor) -> torch.Tensor:
@@ -75,8 +81,9 @@ class ResSplitNet(SplitNet):
         self.s2d = ok if s2d_stem is None else (s2d_stem and ok)
         self.stem_cin = st["cin"]
         if self.s2d:
-            chain = [s2d_stem_layer(st)] + list(chain[1:])
-            C, H, W = 4 * C, H // 2, W // 2
+            stem = s2d_stem_layer(st, 0 if os.environ.get("SPLITCNN_S2D_NARROW") else 64)
+            chain = [stem] + list(chain[1:])
+            C, H, W = stem["cin"], H // 2, W // 2
         super().__init__(chain, [], N, C, H, W, split=split, mode="even", dtype=dtype, device=device,
                          force_simt=force_simt, fuse_pool=False, **kw)
 
@@ -177,9 +184,11 @@ class ResSplitNet(SplitNet):
         acts = self.act_r
         self._label = "input"
         if self.s2d:
-            x_layout = sc.NCHW_S2D
-        self._call("split", 2 * self._bytes(self.region, 0)[0], sc.splitcnn_split, R, 0, dt, x, x_layout, acts[0],
-                   p0, p1, stream)
+            self._call("split", 2 * self._bytes(self.region, 0)[0], sc.splitcnn_split_s2d, R, 0, dt, x, self.stem_cin,
+                       acts[0], p0, p1, stream)
+        else:
+            self._call("split", 2 * self._bytes(self.region, 0)[0], sc.splitcnn_split, R, 0, dt, x, x_layout, acts[0],
+                       p0, p1, stream)
         m = 0
         L = self.region_layers
         while m < len(L):
@@ -425,8 +434,12 @@ class ResBNSplitNet(ResSplitNet):
         R, dt, fl = self.region.handle, self.dtype, self.flags_extra
         acts, L = self.act_r, self.region_layers
         self._label = "input"
-        self._call("split", 2 * self._bytes(self.region, 0)[0], sc.splitcnn_split, R, 0, dt, x,
-                   sc.NCHW_S2D if self.s2d else x_layout, acts[0], p0, p1, stream)
+        if self.s2d:
+            self._call("split", 2 * self._bytes(self.region, 0)[0], sc.splitcnn_split_s2d, R, 0, dt, x, self.stem_cin,
+                       acts[0], p0, p1, stream)
+        else:
+            self._call("split", 2 * self._bytes(self.region, 0)[0], sc.splitcnn_split, R, 0, dt, x, x_layout, acts[0],
+                       p0, p1, stream)
 
         def conv(m, relu):
             W, _ = self.params[("r", m)]

@@ -339,3 +339,46 @@ def test_host_pipeline_graphs_bitwise(sc):
     pipe.synchronize()
     for r, o in zip(ref, outs):
         assert torch.equal(r, o)
+
+
+def test_per_op_autograd_modules(sc):
+    """SplitConv2d / SplitMaxPool2d (torch.autograd on patch buffers): conv(+ReLU) -> pool -> conv on a
+    split plan, fp32, against the oracle composition (output and both weight gradients, 1e-4)."""
+    from oracle import ops as O
+    from oracle import plan as OP
+    from paper_conf_asplos_jinh19_b200.autograd import SplitConv2d, SplitMaxPool2d
+    from paper_conf_asplos_jinh19_b200.net import pack_weight
+    from paper_conf_asplos_jinh19_b200.plan import SplitPlan
+    from tests.helpers import pack_level
+    layers = [synth.conv(8, 16, name="a"), synth.maxpool(16), synth.conv(16, 16, relu=False, name="b")]
+    Oh, Ow = [0, 7, 18], [0, 10, 18]            # ragged 2x2 split of the 18x18 output
+    pl = SplitPlan(layers, 2, 8, 36, 36, Oh, Ow)
+    ref = OP.plan(layers, 2, 8, 36, 36, Oh, Ow)
+    g = synth.rng(21)
+    X = synth.uniform(g, (2, 8, 36, 36)).astype(np.float64)
+    (Wa, ba), _, (Wb, bb) = synth.layer_params(g, layers)
+    c1, p1, c2 = SplitConv2d(pl, 0, sc.FP32), SplitMaxPool2d(pl, 1, sc.FP32), SplitConv2d(pl, 2, sc.FP32, relu=False)
+    with torch.no_grad():
+        c1.weight.copy_(pack_weight(torch.from_numpy(Wa).cuda(), pl.levels[0]["Cpad"], torch.float32))
+        c1.bias.copy_(torch.from_numpy(ba))
+        c2.weight.copy_(pack_weight(torch.from_numpy(Wb).cuda(), pl.levels[2]["Cpad"], torch.float32))
+        c2.bias.copy_(torch.from_numpy(bb))
+    x = torch.from_numpy(pack_level(X, pl.levels[0]).astype(np.float32)).cuda()
+    y = c2(p1(c1(x)))
+    G = synth.normal(g, (2, 16, 18, 18)).astype(np.float64)
+    y.backward(torch.from_numpy(pack_level(G, pl.levels[3]).astype(np.float32)).cuda())
+    torch.cuda.synchronize()
+    l0, l1, l2 = ref.layers
+    A1 = O.conv_fwd(O.split(X, l0.Ih, l0.Iw), Wa.astype(np.float64), ba.astype(np.float64), l0, True)
+    P1, am = O.pool_fwd(A1, l1)
+    Y = O.conv_fwd(P1, Wb.astype(np.float64), bb.astype(np.float64), l2, False)
+    Gp = O.split(G, l2.Oh, l2.Ow)
+    dWb, _ = O.conv_bwd_filter(P1, Gp, l2)
+    gP = O.conv_bwd_data(Gp, Wb.astype(np.float64), l2)
+    gA = O.relu_mask(O.pool_bwd(gP, am, l1), A1)
+    dWa, _ = O.conv_bwd_filter(O.split(X, l0.Ih, l0.Iw), gA, l0)
+    from tests.helpers import unpack_level, w_lib_to_oihw
+    got = unpack_level(y.detach().cpu().numpy(), pl.levels[3])
+    assert max(normwise(got[i][j], Y[i][j]) for i in range(2) for j in range(2)) <= 1e-4
+    assert normwise(w_lib_to_oihw(c2.weight.grad.cpu().numpy(), 16), dWb) <= 1e-4
+    assert normwise(w_lib_to_oihw(c1.weight.grad.cpu().numpy(), 8), dWa) <= 1e-4

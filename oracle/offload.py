@@ -1,6 +1,9 @@
 """Algorithm 1 (offload planning) and its reverse prefetch pass.
-TEST INFRASTRUCTURE ONLY.  PARITY UNPINNED: the paper prints no worked example, so this
-is pinned only by invariants (tests/test_abi_host.py): every offloaded TSO is synchronised
+TEST INFRASTRUCTURE ONLY.  The paper prints no worked example.  Pinned (pin-12,
+tests/test_offload_sim.py) by a discrete-event timeline of one FIFO copy link that knows nothing
+about balances: every non-final sync finds its offloads finished (the no-stall claim)
+and every prefetch not given op 0 arrives before its use; plus hand traces of both passes.
+Also checked by invariants (tests/test_abi_host.py): every offloaded TSO is synchronised
 (ended) no earlier than the op that started it and at the latest at the last op; the balance
 is reset at every sync; offloaded bytes never exceed the theoretical limit (R15);
 every prefetch starts no later than the op that needs it.

@@ -114,10 +114,19 @@ def test_c5_conv1_2_full_size(sc):
     assert normwise(db.double().cpu().numpy(), tt * db1) <= 2e-2
 
 
-@pytest.mark.parametrize("name,Cin,Cout,Hin,nsplit", [("conv3_2", 256, 256, 56, 8), ("conv4_2", 512, 512, 28, 1)])
+@pytest.mark.parametrize("name,Cin,Cout,Hin,nsplit", [
+    ("conv1_1", 3, 64, 224, 8),      # 8-channel padded input: halo8 forward, narrow wgrad
+    ("conv2_1", 64, 128, 112, 8),    # 64 -> 128 channels, 14x14 patches
+    ("conv3_1", 128, 256, 56, 8),    # 128 -> 256 channels, 7x7 patches
+    ("conv3_2", 256, 256, 56, 8),
+    ("conv4_2", 512, 512, 28, 1),
+    ("conv5_2", 512, 512, 14, 1),    # the smallest tail layer (few tiles per SM)
+])
 def test_c5_deep_layers_full_size(sc, name, Cin, Cout, Hin, nsplit):
-    """C5's conv3_2 (split region: 7x7 patches, 2-CTA halo kernels) and conv4_2 (unsplit tail) at N=256:
-    conv_fwd (+bias+ReLU), bwd_data (ReLU mask), bwd_filter (+db) as the executor calls them."""
+    """C5's split-region layers (conv1_1 on the 3->8 padded input, conv2_1, conv3_1, conv3_2 with 2-CTA
+    halo kernels) and unsplit tail layers (conv4_2, conv5_2) at N=256: conv_fwd (+bias+ReLU), bwd_data
+    (ReLU mask), bwd_filter (+db) as the executor calls them (the executor skips conv1_1's bwd_data;
+    it is checked anyway)."""
     from paper_conf_asplos_jinh19_b200.net import pack_weight
     from paper_conf_asplos_jinh19_b200.plan import SplitPlan
     l = synth.conv(Cin, Cout, name=name)

@@ -301,7 +301,40 @@ __global__ void __launch_bounds__(256) colsum_kernel(const T *__restrict__ base,
     }
 }
 
-// returns the number of partial rows written
+// Shared-memory-free variant (channel groups G = Cpad/8 with 32 % G == 0 or G % 32 == 0): it runs on
+// the side stream concurrently with the wgrad GEMM, whose CTAs leave no shared memory free on their
+// SM, so the colsum blocks must need none to co-reside.  Each warp reduces its pixel lanes with
+// shuffles (fixed xor order) and writes its own partial row: RB = G >= 32 ? 256/G : 8 rows per block.
+template <typename T>
+__global__ void __launch_bounds__(256) colsum_warp_kernel(const T *__restrict__ base, int64_t P, int Cpad, int Cout,
+                                                          int64_t R, float *__restrict__ part) {
+    const int G = Cpad / 8;
+    const int lanes = 256 / G;
+    const int cg = threadIdx.x % G, pl = threadIdx.x / G;
+    float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    const int64_t r0 = blockIdx.x * R, r1 = min(P, r0 + R);
+    for (int64_t r = r0 + pl; r < r1; r += lanes) {
+        float v[8];
+        load8(base + r * Cpad + cg * 8, v);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) acc[e] += v[e];
+    }
+    int row;
+    if (G < 32) {
+        for (int o = G; o < 32; o <<= 1)
+#pragma unroll
+            for (int e = 0; e < 8; ++e) acc[e] += __shfl_xor_sync(0xffffffffu, acc[e], o);
+        if ((threadIdx.x & 31) >= G) return;
+        row = blockIdx.x * 8 + (threadIdx.x >> 5);
+    } else {
+        row = blockIdx.x * lanes + pl;
+    }
+#pragma unroll
+    for (int e = 0; e < 8; ++e)
+        if (cg * 8 + e < Cout) part[(int64_t)row * Cout + cg * 8 + e] = acc[e];
+}
+
+// returns the number of partial rows written (at most 8 * 4 * 148: splitcnn_workspace_size's db region)
 int launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, float *part, int cout, int p0, int p1,
                        cudaStream_t st) {
     auto off = [&](int q) -> int64_t {
@@ -313,6 +346,18 @@ int launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, flo
     const int Z = 4 * 148;
     const int64_t R = (P + Z - 1) / Z;
     const int Zr = (int)((P + R - 1) / R);
+    const int G = Lo.Cpad / 8;
+    // 64-channel dY (G = 8, the 224x224 layers) keeps the shared-memory kernel: there the 8x partial rows
+    // cost more in the reduction than co-residency saves (profiles/r1_ab_colsum_warp.txt)
+    if (G >= 16 && G <= 64 && (32 % G == 0 || G % 32 == 0)) {
+        const int RB = G >= 32 ? 256 / G : 8;
+        if (dt == SPLITCNN_BF16)
+            colsum_warp_kernel<__nv_bfloat16><<<Zr, 256, 0, st>>>((const __nv_bfloat16 *)dy + e0, P, Lo.Cpad, cout, R, part);
+        else
+            colsum_warp_kernel<float><<<Zr, 256, 0, st>>>((const float *)dy + e0, P, Lo.Cpad, cout, R, part);
+        count_launch();
+        return Zr * RB;
+    }
     if (dt == SPLITCNN_BF16)
         colsum_kernel<__nv_bfloat16><<<Zr, 256, 0, st>>>((const __nv_bfloat16 *)dy + e0, P, Lo.Cpad, cout, R, part);
     else
@@ -384,7 +429,7 @@ size_t wgrad_simt_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g)
     const int cpp = wgrad_simt_chunks_per_patch(Li, Lo, g, np);
     const int64_t Z = (int64_t)np * cpp;
     const int64_t ncols = (int64_t)g.L.kh * g.L.kw * Li.Cpad;
-    return (size_t)(Z * g.L.cout * ncols + 4 * 148 * g.L.cout) * sizeof(float);
+    return (size_t)(Z * g.L.cout * ncols + 8 * 4 * 148 * g.L.cout) * sizeof(float);   // + db partial rows
 }
 
 void launch_conv_wgrad_simt(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *x,

@@ -10,6 +10,7 @@
 //   WGRAD : M = Cout, N = kh*kw*Cin_pad, K = pixels of one chunk of one patch (split-K);
 //           partials -> workspace -> fixed-order reduction (deterministic)
 #include <algorithm>
+#include <cstdlib>
 #include <type_traits>
 
 #include "common.cuh"
@@ -334,7 +335,21 @@ __global__ void __launch_bounds__(256) colsum_warp_kernel(const T *__restrict__ 
         if (cg * 8 + e < Cout) part[(int64_t)row * Cout + cg * 8 + e] = acc[e];
 }
 
-// returns the number of partial rows written (at most 8 * 4 * 148: splitcnn_workspace_size's db region)
+// part[b][:] = sum of rows [b*chunk, (b+1)*chunk) of rows[Z][n], in row order (deterministic)
+__global__ void __launch_bounds__(256) rows_sum_kernel(const float *__restrict__ rows, int Z, int n, int chunk,
+                                                       float *__restrict__ part) {
+    const int col = blockIdx.x * 256 + threadIdx.x;
+    if (col >= n) return;
+    const int z0 = blockIdx.y * chunk, z1 = min(Z, z0 + chunk);
+    float s = 0.f;
+#pragma unroll 8
+    for (int z = z0; z < z1; ++z) s += __ldg(rows + (int64_t)z * n + col);
+    part[(int64_t)blockIdx.y * n + col] = s;
+}
+
+// returns the number of partial rows left in part[0..) (at most 4 * 148); the db workspace region holds
+// 9 * 4 * 148 rows: the warp variant writes its (up to 8 per block) rows after the first 4 * 148 and
+// folds them into part[0..) in fixed-size chunks, so the final reduction sees at most 4 * 148 rows
 int launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, float *part, int cout, int p0, int p1,
                        cudaStream_t st) {
     auto off = [&](int q) -> int64_t {
@@ -347,16 +362,25 @@ int launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, flo
     const int64_t R = (P + Z - 1) / Z;
     const int Zr = (int)((P + R - 1) / R);
     const int G = Lo.Cpad / 8;
-    // 64-channel dY (G = 8, the 224x224 layers) keeps the shared-memory kernel: there the 8x partial rows
-    // cost more in the reduction than co-residency saves (profiles/r1_ab_colsum_warp.txt)
-    if (G >= 16 && G <= 64 && (32 % G == 0 || G % 32 == 0)) {
+    // when the warp variant pays (same-box A/Bs, profiles/r1_ab_colsum_fold.txt): a dY of >= 32 MB (below
+    // that -- C2's 32x32 layers -- the extra fold launch costs more than co-residency saves), except the
+    // 64-channel 224x224 layers (>= 1 GB at G = 8), where the shared-memory kernel measured faster
+    const int64_t dy_bytes = P * Lo.Cpad * (int64_t)(dt == SPLITCNN_BF16 ? 2 : 4);
+    const bool warp_ok = G <= 64 && (32 % G == 0 || G % 32 == 0) && dy_bytes >= (32ll << 20) &&
+                         (G >= 16 || dy_bytes < (1ll << 30));
+    if (warp_ok && !getenv("SPLITCNN_COLSUM_SMEM")) {
         const int RB = G >= 32 ? 256 / G : 8;
+        float *rows = part + (int64_t)Z * cout;
         if (dt == SPLITCNN_BF16)
-            colsum_warp_kernel<__nv_bfloat16><<<Zr, 256, 0, st>>>((const __nv_bfloat16 *)dy + e0, P, Lo.Cpad, cout, R, part);
+            colsum_warp_kernel<__nv_bfloat16><<<Zr, 256, 0, st>>>((const __nv_bfloat16 *)dy + e0, P, Lo.Cpad, cout, R, rows);
         else
-            colsum_warp_kernel<float><<<Zr, 256, 0, st>>>((const float *)dy + e0, P, Lo.Cpad, cout, R, part);
+            colsum_warp_kernel<float><<<Zr, 256, 0, st>>>((const float *)dy + e0, P, Lo.Cpad, cout, R, rows);
         count_launch();
-        return Zr * RB;
+        const int nrows = Zr * RB, chunk = 2 * RB;
+        const int nch = (nrows + chunk - 1) / chunk;
+        rows_sum_kernel<<<dim3((unsigned)((cout + 255) / 256), (unsigned)nch), 256, 0, st>>>(rows, nrows, cout, chunk, part);
+        count_launch();
+        return nch;
     }
     if (dt == SPLITCNN_BF16)
         colsum_kernel<__nv_bfloat16><<<Zr, 256, 0, st>>>((const __nv_bfloat16 *)dy + e0, P, Lo.Cpad, cout, R, part);
@@ -429,7 +453,7 @@ size_t wgrad_simt_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g)
     const int cpp = wgrad_simt_chunks_per_patch(Li, Lo, g, np);
     const int64_t Z = (int64_t)np * cpp;
     const int64_t ncols = (int64_t)g.L.kh * g.L.kw * Li.Cpad;
-    return (size_t)(Z * g.L.cout * ncols + 8 * 4 * 148 * g.L.cout) * sizeof(float);   // + db partial rows
+    return (size_t)(Z * g.L.cout * ncols + 9 * 4 * 148 * g.L.cout) * sizeof(float);   // + db partial rows
 }
 
 void launch_conv_wgrad_simt(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *x,

@@ -2223,7 +2223,7 @@ size_t wgrad_tc_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g) {
     const int64_t zmax = ngroups * wgrad_zbound(path, Li, g);
     const int64_t nW = (int64_t)g.L.cout * g.L.kh * g.L.kw * Li.Cpad;
     // + a separate region for the db column-sum partials (computed concurrently, see launch_conv_wgrad_tc)
-    const size_t dbp = (((size_t)8 * 4 * 148 * g.L.cout * sizeof(float)) + 255) & ~(size_t)255;   // <= 8 rows per colsum block
+    const size_t dbp = (((size_t)9 * 4 * 148 * g.L.cout * sizeof(float)) + 255) & ~(size_t)255;   // colsum rows + folded rows
     return (((size_t)zmax * nW * sizeof(float) + 255) & ~(size_t)255) + dbp + 256;
 }
 

@@ -13,7 +13,7 @@ for f in sorted(glob.glob("profiles/r1_bench_*.json")):
     rows.append((os.path.basename(f), d.get("config", {}).get("workload", "")[:110], d.get("value"), d.get("ms_per_step"),
                  (d.get("e2e") or {}).get("value"), rf.get("achieved"), rf.get("frac"), hb.get("achieved_gbs"),
                  mem.get("peak_allocated_gb"), (d.get("clocks") or {}).get("sm_mhz")))
-print("| file | workload | img/s | ms/step | e2e img/s | conv TFLOP/s | frac of 1365 | pool/split/merge GB/s | peak GB | SM MHz |")
+print("| file | workload | img/s | ms/step | e2e img/s | conv TFLOP/s | frac of peak | pool/split/merge GB/s | peak GB | SM MHz |")
 print("|---|---|---|---|---|---|---|---|---|---|")
 for r in rows:
     print("| " + " | ".join("" if v is None else (f"{v:.4g}" if isinstance(v, float) else str(v)) for v in r) + " |")

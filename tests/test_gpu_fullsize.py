@@ -278,3 +278,36 @@ def test_c5_split_merge_pool_full_size(sc):
         G = gb[:, lref.Oh[i]:lref.Oh[i + 1], lref.Ow[j]:lref.Ow[j + 1]][None] * t[n]
         dX = O.pool_bwd_patch(G, A, X.shape[2], X.shape[3], 2, 2, 2, 2, lref.pads_h[i], lref.pads_w[j])
         assert np.array_equal(_patch(dx, lv0, i, j, n)[:, :128], dX), (n, i, j)
+
+
+@pytest.mark.parametrize("dtype_name,N_,C_,H_", [
+    ("fp32", 64, 64, 64),     # 67 MB fp32 dY: warp colsum (8 channel groups) + row fold
+    ("bf16", 32, 256, 56),    # 51 MB bf16 dY, 32 channel groups: warp colsum, one row per pixel lane
+    ("bf16", 8, 64, 56),      # 3.2 MB: below the 32 MB cut, shared-memory colsum
+])
+def test_db_column_sums_both_kernels(sc, dtype_name, N_, C_, H_):
+    """a5's bias gradient db[co] = sum over n, h, w of dY (P:153 adjoint) through
+    splitcnn_conv_bwd_filter, at sizes that select each colsum kernel; beta = 1 accumulates.  The
+    expected value is that sum taken in fp64 on the host over the same (rounded) dY."""
+    from paper_conf_asplos_jinh19_b200.plan import SplitPlan
+    dtype = sc.BF16 if dtype_name == "bf16" else sc.FP32
+    tdt = torch.bfloat16 if dtype == sc.BF16 else torch.float32
+    l = synth.conv(C_, C_, name="db")
+    Ob = sc.splitcnn_boundaries_even(H_, 2)
+    pl = SplitPlan([l], N_, C_, H_, H_, Ob, Ob)
+    lv0, lv1 = pl.levels
+    g = torch.Generator().manual_seed(77 + C_)
+    x = torch.randn(lv0["total_elems"], generator=g).to(tdt).cuda()
+    dyh = (torch.randn(lv1["total_elems"], generator=g) + 0.25).to(tdt)
+    dy = dyh.cuda()
+    ws_b = pl.workspace_size(0, dtype, 2)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    dw = torch.zeros((C_, 3, 3, lv0["Cpad"]), dtype=torch.float32, device="cuda")
+    db = torch.full((C_,), 5.0, dtype=torch.float32, device="cuda")
+    sc.splitcnn_conv_bwd_filter(pl.handle, 0, dtype, x, dy, dw, db, 0.0, ws, ws_b)
+    torch.cuda.synchronize()
+    ref = dyh.double().numpy().reshape(-1, lv1["Cpad"])[:, :C_].sum(axis=0)
+    assert normwise(db.double().cpu().numpy(), ref) <= 1e-5
+    sc.splitcnn_conv_bwd_filter(pl.handle, 0, dtype, x, dy, dw, db, 1.0, ws, ws_b)
+    torch.cuda.synchronize()
+    assert normwise(db.double().cpu().numpy(), 2 * ref) <= 1e-5

@@ -271,7 +271,10 @@ SPLITCNN_API splitcnn_status_t splitcnn_pool_bwd(splitcnn_plan_t plan, int32_t l
  *   mask == NULL: y = a + b, then max(., 0) with FLAG_RELU            (forward join)
  *   mask != NULL: y = (a + b) * [mask > 0]                          (backward: sum of a fork's
  *                 two gradient contributions times the ReLU mask of the block output mask)
- * Arithmetic in fp32, one rounding to the storage type.  Errors: null a/b/y, misalignment,
+ *   b == NULL (mask required): y = a * [mask > 0]                   (ReLU backward alone, e.g. the
+ *                 output gradient of a stack whose last op is a conv with a fused ReLU)
+ * Arithmetic in fp32, one rounding to the storage type.  Errors: null a/y, null b without a mask,
+ * misalignment,
  * FLAG_RELU together with a mask. */
 SPLITCNN_API splitcnn_status_t splitcnn_add(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
                                 const void *a, const void *b, void *y, const void *mask, uint32_t flags,

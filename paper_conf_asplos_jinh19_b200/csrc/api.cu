@@ -316,7 +316,7 @@ extern "C" splitcnn_status_t splitcnn_add(splitcnn_plan_t plan, int32_t level, s
                                           int32_t p1, splitcnn_stream_t stream) {
     if (!plan || level < 0 || level >= (int)plan->levels.size()) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad level");
     TRY(check_dtype(dtype));
-    if (!a || !b || !y) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    if (!a || !y || (!b && !mask)) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
     if (mask && (flags & SPLITCNN_FLAG_RELU)) return fail(SPLITCNN_ERR_INVALID_VALUE, "FLAG_RELU with a mask");
     NEED_ALIGNED(a, "a");
     NEED_ALIGNED(b, "b");

@@ -358,6 +358,7 @@ int launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, flo
     };
     const int64_t e0 = off(p0), e1 = off(p1);
     const int64_t P = (e1 - e0) / Lo.Cpad;
+    if (P <= 0) return 0;          // empty patch range: no partials (the reduce then applies beta alone)
     const int Z = 4 * 148;
     const int64_t R = (P + Z - 1) / Z;
     const int Zr = (int)((P + R - 1) / R);
@@ -468,9 +469,11 @@ void launch_conv_wgrad_simt(splitcnn_dtype_t dt, const Level &Li, const Level &L
     a.Li = make_level_desc(Li); a.Lo = make_level_desc(Lo); a.ly = make_layer_desc(g);
     a.x = dy; a.w = x; a.y = part; a.Cout = g.L.cout; a.p0 = p0; a.cpp = cpp;
     dim3 grid((g.L.cout + BM - 1) / BM, (ncols + BN - 1) / BN, Z);
-    if (dt == SPLITCNN_BF16) conv_simt_kernel<__nv_bfloat16, MODE_WGRAD><<<grid, NT, 0, st>>>(a);
-    else conv_simt_kernel<float, MODE_WGRAD><<<grid, NT, 0, st>>>(a);
-    count_launch();
+    if (Z > 0) {                   // empty patch range: dW = beta * dW (the reduce below, Z = 0)
+        if (dt == SPLITCNN_BF16) conv_simt_kernel<__nv_bfloat16, MODE_WGRAD><<<grid, NT, 0, st>>>(a);
+        else conv_simt_kernel<float, MODE_WGRAD><<<grid, NT, 0, st>>>(a);
+        count_launch();
+    }
     const int64_t n = (int64_t)g.L.cout * ncols;
     launch_reduce(part, Z, n, dw, beta, st);
     if (db) {

@@ -609,12 +609,12 @@ void launch_pool_bwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, con
 //                                    contributions of a fork and applies its ReLU mask once)
 // One thread = 8 elements (16 B of bf16); y may alias a or b (each element is read, then written,
 // by the same thread).  fp32 sum, one rounding to T.
-template <typename T, bool RELU, bool MASK>
+template <typename T, bool RELU, bool MASK, bool HASB = true>
 __global__ void __launch_bounds__(256) add_kernel(const T *a, const T *b, T *y, const T *__restrict__ m, int64_t n8) {
     for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n8; u += (int64_t)gridDim.x * blockDim.x) {
-        float va[8], vb[8], vm[8];
+        float va[8], vb[8] = {0, 0, 0, 0, 0, 0, 0, 0}, vm[8];
         load8(a + u * 8, va);
-        load8(b + u * 8, vb);
+        if (HASB) load8(b + u * 8, vb);
         if (MASK) load8(m + u * 8, vm);
 #pragma unroll
         for (int k = 0; k < 8; ++k) {
@@ -631,7 +631,9 @@ template <typename T>
 void launch_add_t(const void *a, const void *b, void *y, const void *m, int relu, int64_t n, cudaStream_t st) {
     const int64_t n8 = n / 8;
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n8 + 255) / 256, 148 * 8));
-    if (m)
+    if (m && !b)   // ReLU backward alone: y = a * [m > 0]
+        add_kernel<T, false, true, false><<<grid, 256, 0, st>>>((const T *)a, nullptr, (T *)y, (const T *)m, n8);
+    else if (m)
         add_kernel<T, false, true><<<grid, 256, 0, st>>>((const T *)a, (const T *)b, (T *)y, (const T *)m, n8);
     else if (relu)
         add_kernel<T, true, false><<<grid, 256, 0, st>>>((const T *)a, (const T *)b, (T *)y, nullptr, n8);

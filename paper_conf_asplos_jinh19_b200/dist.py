@@ -114,7 +114,7 @@ class DistSplitNet:
         del probe
         self.region_net = SplitNet(c["layers"], [], N, 3, H, W, split=c["split"], mode=c["mode"],
                                    omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype, device=device,
-                                   patch_range=self.owners[rank])
+                                   patch_range=self.owners[rank], mask_output_grad=False)
         L = self.region_net.region.levels[-1]
         self.C_join, self.H_join, self.W_join = L["C"], L["H"], L["W"]
         tail = c["tail"]

@@ -34,7 +34,7 @@ class SplitNet:
                  split=(2, 2), mode: str = "even", omega: float = 0.2, seed: int = 0,
                  dtype: int = sc.BF16, device="cuda", patch_range=None, force_simt: bool = False,
                  grad_buffer: torch.Tensor | None = None, input_relu: bool = False, fuse_pool: bool = True,
-                 static_pool: bool = False, input_grad: bool = False):
+                 static_pool: bool = False, input_grad: bool = False, mask_output_grad: bool = True):
         self.region_layers, self.tail_layers = region, tail
         self.N, self.C, self.H, self.W = N, C, H, W
         self.split, self.mode, self.omega, self.seed = split, mode, omega, seed
@@ -45,6 +45,9 @@ class SplitNet:
         self.step_index = 0
         self.static_pool = static_pool   # HMMS static memory plan: one arena, first-fit offsets
         self.input_grad = input_grad  # step(): also compute dX of the first layer (C1's single-layer pass)
+        # dY is the gradient of the stack output; False when the caller already applied the output's ReLU
+        # mask (a region whose gradient comes back from a tail that masks its input, dist.py)
+        self.mask_output_grad = mask_output_grad
         self.timers = None       # list -> every library call is bracketed by CUDA events (bench.py)
         self._label = ""
         self.region = self._make_region_plan(0)
@@ -174,12 +177,15 @@ class SplitNet:
                 else:
                     ops.append((f"{key}{m}", [("a", key, m), ("a", key, m + 1), ("am", key, m)]))
         out_key = ("a", "t", len(self.tail_layers)) if self.tail else ("a", "r", len(self.region_layers))
+        if self._top_masked():
+            tk = "t" if self.tail else "r"
+            ops.append(("topmask'", [out_key, ("g", tk, len(self.tail_layers if self.tail else self.region_layers))]))
         for key, layers in (("t", self.tail_layers), ("r", self.region_layers)):
             if key == "t" and not self.tail:
                 continue
             for m in range(len(layers) - 1, -1, -1):
                 top = m == len(layers) - 1 and (key == "t" or not self.tail)
-                gin = [] if top else [("g", key, m + 1)]          # the step's dY is the caller's
+                gin = [] if top and not self._top_masked() else [("g", key, m + 1)]   # else dY is the caller's
                 last = key == "r" and m == 0 and not self.input_grad
                 gout = [] if last else [("g", key, m)]
                 if layers[m]["op"] == "conv":
@@ -307,6 +313,12 @@ class SplitNet:
             return self.tail_layers[m - 1]["op"] == "conv" and self.tail_layers[m - 1].get("relu", True)
         return self._masked("r", len(self.region_layers))
 
+    def _top_masked(self) -> bool:
+        """The stack ends in a conv with a fused ReLU: dY (the gradient of the stack OUTPUT) reaches the
+        conv's pre-activation only where the output is > 0, one ReLU-backward call."""
+        layers = self.tail_layers if self.tail else self.region_layers
+        return self.mask_output_grad and bool(layers) and layers[-1]["op"] == "conv" and layers[-1].get("relu", True)
+
     # ------------------------------------------------------------------ passes
     def forward(self, x: torch.Tensor, stream=None, x_layout: int = sc.NCHW):
         """x: full tensor (dtype) on the device, NCHW or NHWC.  Returns the output level buffer."""
@@ -369,6 +381,14 @@ class SplitNet:
         """dy: gradient w.r.t. the output level buffer (same layout).  Fills self.grads."""
         p0, p1 = self.patch_range
         g = dy
+        if self._top_masked():
+            key, plan, acts, q0, q1 = (("t", self.tail, self.act_t, 0, 1) if self.tail else
+                                       ("r", self.region, self.act_r, p0, p1))
+            gm = self._gout(key, plan.nlayers, g)
+            es = 2 if self.dtype == sc.BF16 else 4
+            self._call("relu_bwd", 3 * es * dy.numel(), sc.splitcnn_add, plan.handle, plan.nlayers, self.dtype, dy, None,
+                       gm, acts[-1], 0, q0, q1, stream)
+            g = gm
         if self.tail:
             g = self._run_bwd("t", self.tail, self.tail_layers, self.act_t, g, 0, 1, stream, True)
             gi = self._gout("r", self.region.nlayers, g)

@@ -189,3 +189,37 @@ def layer_params(g: np.random.Generator, layers, dtype=np.float32):
         else:
             out.append(None)
     return out
+
+
+# --------------------------------------------------------------------------- exact-arithmetic draws
+# "Dyadic" inputs for the bf16 whole-stack checks: every value is a small multiple of 1/4 and every
+# weight a small integer on a few taps, so every sum the forward / data-gradient passes form is an
+# integer multiple of 1/4 far below 2^24 units -- EXACT in fp32 and in fp64, in any order.  Both sides
+# then round the same exact value to bf16 (RNE), so the activation and gradient levels, every ReLU mask
+# and every pool argmax are the same on both sides, and a whole deep stack can be compared in bf16
+# without near-tie decisions (a decision flip would otherwise re-route a whole gradient element).
+def dyadic(g: np.random.Generator, shape, lim: int = 8, dtype=np.float32):
+    """Integers in [-lim, lim] divided by 4 (exact in bf16)."""
+    return (g.integers(-lim, lim + 1, size=shape) / 4.0).astype(dtype)
+
+
+def sparse_int_weight(g: np.random.Generator, cout, cin, kh, kw, taps: int = 3, dtype=np.float32):
+    """OIHW weight with `taps` nonzero entries per output channel at random (ci, r, c), values in
+    {-2, -1, 1, 2}."""
+    W = np.zeros((cout, cin * kh * kw), dtype=np.float64)
+    for co in range(cout):
+        pos = g.choice(cin * kh * kw, size=min(taps, cin * kh * kw), replace=False)
+        W[co, pos] = g.choice(np.array([-2.0, -1.0, 1.0, 2.0]), size=len(pos))
+    return W.reshape(cout, cin, kh, kw).astype(dtype)
+
+
+def exact_layer_params(g: np.random.Generator, layers, taps: int = 3, dtype=np.float32):
+    """layer_params with dyadic values: sparse integer W, bias in {-2..2}/4; None for pools."""
+    out = []
+    for l in layers:
+        if l["op"] == "conv":
+            out.append((sparse_int_weight(g, l["cout"], l["cin"], l["kh"], l["kw"], taps, dtype),
+                        dyadic(g, (l["cout"],), 2, dtype)))
+        else:
+            out.append(None)
+    return out

@@ -68,6 +68,12 @@ def run(region, tail, N, C, H, W, Oh, Ow, params, X, G, round_bf16=False):
                 g = _rnd(g, round_bf16)
         return g, grads
 
+    def top_mask(layers, acts, g):
+        """loss = <Y, G> with Y the stack OUTPUT: when the last op is a conv with a
+        fused ReLU, G reaches the conv's pre-activation only where Y > 0."""
+        l = layers[-1]
+        return O.relu_mask(g, acts[-1]) if l["op"] == "conv" and l.get("relu", True) else g
+
     pools = {}
     acts_r, args_r = fwd("r", rp, region, _rnd(O.split(X, rp.layers[0].Ih, rp.layers[0].Iw), round_bf16))
     out = O.merge(acts_r[-1])
@@ -77,10 +83,10 @@ def run(region, tail, N, C, H, W, Oh, Ow, params, X, G, round_bf16=False):
         acts_t, args_t = fwd("t", tp, tail, [[out]])
         pools.update({("t", m): (acts_t[m], a) for m, a in args_t.items()})
         out = O.merge(acts_t[-1])
-        g, grads_t = bwd("t", tp, tail, acts_t, args_t, [[G]], region_out_masked, True)
+        g, grads_t = bwd("t", tp, tail, acts_t, args_t, top_mask(tail, acts_t, [[G]]), region_out_masked, True)
         g = O.split(O.merge(g), Lr.Oh, Lr.Ow)
     else:
-        g, grads_t = O.split(G, Lr.Oh, Lr.Ow), {}
+        g, grads_t = top_mask(region, acts_r, O.split(G, Lr.Oh, Lr.Ow)), {}
     _, grads_r = bwd("r", rp, region, acts_r, args_r, g, False, False)
     dWs, dbs = [], []
     for key, layers, grads in (("r", region, grads_r), ("t", tail, grads_t)):

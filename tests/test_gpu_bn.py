@@ -83,14 +83,19 @@ def test_bn_ops_parity(sc, dtype_name, C):
     assert max(normwise(dXg[i][j], dXr[i][j]) for i in range(3) for j in range(2)) <= tol
 
 
-def _run_stack(sc, dtype, N=2, H=64, seed=6):
+def _run_stack(sc, dtype, N=2, H=64, seed=6, exact=False):
     from paper_conf_asplos_jinh19_b200.resnet import ResBNSplitNet
     chain, blocks = synth.resnet18_blocks(64, 128)
     net = ResBNSplitNet(chain, blocks, N, 3, H, H, split=(2, 2), dtype=dtype)
     g = synth.rng(seed)
     bf = dtype == sc.BF16
-    X = synth.uniform(g, (N, 3, H, H))
-    params = synth.resnet_params(g, chain, blocks)
+    if exact:
+        X = synth.dyadic(g, (N, 3, H, H))
+        params = [p for p in synth.exact_layer_params(g, chain) if p is not None]
+        params += synth.exact_layer_params(g, [b["ds"] for b in blocks if b["ds"] is not None])
+    else:
+        X = synth.uniform(g, (N, 3, H, H))
+        params = synth.resnet_params(g, chain, blocks)
     bn = synth.bn_params(g, [W.shape[0] for W, _ in params])
     if bf:
         X = synth.to_bf16_f32(X)
@@ -98,7 +103,7 @@ def _run_stack(sc, dtype, N=2, H=64, seed=6):
     net.set_params([(torch.from_numpy(Wt), torch.from_numpy(b)) for Wt, b in params])
     net.set_bn_params(bn)
     L = net.region.levels[-1]
-    G = synth.normal(g, (N, L["C"], L["H"], L["W"]))
+    G = (synth.dyadic if exact else synth.normal)(g, (N, L["C"], L["H"], L["W"]))
     if bf:
         G = synth.to_bf16_f32(G)
     x = torch.from_numpy(X).to("cuda", net.tdtype)
@@ -129,12 +134,11 @@ def test_resnet_bn_stack_fp32(sc):
 
 
 def test_resnet_bn_stack_bf16(sc):
-    """bf16 (tensor cores, s2d stem): the forward output within the per-op bound 2e-2.  The bf16
-    whole-stack BN backward is only checked to be finite: at this size (layer2 reduces over 128
-    pixels) a single ReLU-kink / max-pool near-tie decision that rounds the other way moves dgamma /
-    dbeta of a channel by a large fraction of their norm (measured up to 0.25 normwise,
-    deterministic), and BN backward's mean subtraction amplifies it; every BN op is held to 2e-2 in
-    bf16 (test_bn_ops_parity) and the whole stack to 1e-4 in fp32 (above)."""
-    errs = _run_stack(sc, sc.BF16)
-    assert errs["out"] <= 2e-2, errs
-    assert all(np.isfinite(v) for v in errs.values()), errs
+    """bf16 (tensor cores, s2d stem) whole BN stack, forward and backward: output, every dW, dgamma,
+    dbeta within the R13 bf16 bar 2e-2.  Dyadic conv inputs / weights keep every conv sum exact; the
+    BN normalisation (1/sqrt(var + eps)) is not, so its outputs can still round differently on the two
+    sides -- measured 0.7e-3 (output) / 1.4e-3 (dW) / 7.0e-3 (dgamma, dbeta) at this size,
+    profiles/r2_diag_bf16.txt.  (With Kaiming draws one ReLU-kink / pool near-tie decision moves a
+    channel's dgamma by up to 0.25 normwise.)"""
+    errs = _run_stack(sc, sc.BF16, exact=True)
+    assert max(errs.values()) <= 2e-2, errs

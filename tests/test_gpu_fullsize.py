@@ -1,10 +1,11 @@
 """Parity at BASELINE.json's full size, in the launch configuration bench.py times:
 C5's conv1_2 -> pool1 (N=256, 64 channels, 224x224, 8x8 split) through the same calls the executor
-makes (conv_pool_fwd, bwd_data with the ReLU mask, bwd_filter with db).  Image n of the batch is the
-seeded base image times an exact bf16 scale s_n (and dY image n the base gradient times t_n), so
+makes (conv_pool_fwd, bwd_data with the ReLU mask, bwd_filter with db).  Image n of the batch is
+S[n,0] B0 + S[n,1] B1 -- the seeded base image split into its two checkerboard pixel classes, with a
+distinct pair of exact scales per image (all 256 images differ; _Batch), and dY likewise, so
   * forward / data gradient are checked on sampled (image, patch) pairs against the oracle one by one;
-  * the weight gradient, a sum over all 256 images and 64 patches, equals (sum_n s_n t_n) * dW(base)
-    by linearity, and the oracle computes dW(base) over all 64 patches of one image."""
+  * the weight gradient, a sum over all 256 images and 64 patches, is bilinear in (X, dY), so it equals
+    sum_{k,l} (sum_n S_x[n,k] S_g[n,l]) dW(Bx_k, Bg_l): four single-image oracle weight gradients."""
 import numpy as np
 import pytest
 
@@ -29,27 +30,67 @@ def sc():
     return splitcnn
 
 
-def _scales(n, off, every=2):
-    """Exact bf16 scales: powers of two, negative on every `every`-th image (distinct per image group)."""
-    return np.array([(-1.0 if (i + off) % every == every - 1 else 1.0) * 2.0 ** (((i + off) // 2) % 3 - 1)
-                     for i in range(n)])
+_TABLE = np.array([m * 2.0 ** -e for e in range(4) for m in (1.0, 1.25, 1.5, 1.75)])   # 16 scales, 3-bit mantissas
 
 
-def _fill_level(lv, base_chw, scales, device="cuda"):
-    """Level buffer (bf16) of N scaled copies of one CHW image, patch-major NHWC (layout glue)."""
+def _round5(a):
+    """Keep 5 significant bits (a seeded draw rounded to bf16, low 3 mantissa bits cleared), so a 5-bit
+    value times a 3-bit scale is exact in bf16."""
+    u = synth.to_bf16_f32(np.asarray(a, dtype=np.float32)).view(np.uint32) & np.uint32(0xFFF8FFFF)
+    return u.view(np.float32).astype(np.float64)
+
+
+class _Batch:
+    """N DISTINCT images: image n = S[n,0] * B0 + S[n,1] * B1 with B0 / B1 the base image on the two
+    checkerboard pixel classes (disjoint supports, so every image is exact in bf16) and (S[n,0], S[n,1])
+    = two base-16 digits of n through _TABLE -- no two of the 256 images are equal, so an image-offset
+    bug is visible.  swap=True reverses the digits (the dY batch)."""
+
+    def __init__(self, base, swap=False):
+        b = _round5(base)
+        h, w = b.shape[1:]
+        m = ((np.arange(h)[:, None] + np.arange(w)[None, :]) % 2 == 0)[None]
+        self.B = [b * m, b * ~m]
+        n = np.arange(N)
+        d0, d1 = (n // 16, n % 16) if swap else (n % 16, n // 16)
+        self.S = np.stack([_TABLE[d0], _TABLE[d1]], 1)
+
+    def img(self, n):
+        return self.S[n, 0] * self.B[0] + self.S[n, 1] * self.B[1]
+
+    def patch(self, n, hs, ws):
+        return self.img(n)[:, hs[0]:hs[1], ws[0]:ws[1]][None]
+
+
+def _bilinear(xb, gb, fn):
+    """sum_n fn(X_n, G_n) for fn bilinear: sum over (k, l) of (sum_n S_x[n,k] S_g[n,l]) fn(Bx_k, Bg_l)."""
+    out = None
+    for k in range(2):
+        for l in range(2):
+            c = float(np.sum(xb.S[:, k] * gb.S[:, l]))
+            v = c * fn(xb.B[k][None], gb.B[l][None])
+            out = v if out is None else out + v
+    return out
+
+
+def _fill_level(lv, batch, device="cuda"):
+    """Level buffer (bf16) of the batch's N images, patch-major NHWC (layout glue)."""
     Cp, W = lv["Cpad"], lv["W"]
     buf = torch.zeros(lv["total_elems"], dtype=torch.bfloat16, device=device)
-    s = torch.from_numpy(scales.astype(np.float32)).to(device)
+    S = torch.from_numpy(batch.S.astype(np.float32)).to(device)
     bh, bw = lv["bh"], lv["bw"]
+    C = batch.B[0].shape[0]
     for i in range(lv["n_h"]):
         hp = bh[i + 1] - bh[i]
         for j in range(lv["n_w"]):
             wp = bw[j + 1] - bw[j]
             off = N * Cp * (bh[i] * W + hp * bw[j])
-            blk = torch.zeros((hp, wp, Cp), dtype=torch.float32, device=device)
-            blk[..., :base_chw.shape[0]] = torch.from_numpy(
-                np.ascontiguousarray(base_chw[:, bh[i]:bh[i + 1], bw[j]:bw[j + 1]].transpose(1, 2, 0))).to(device)
-            buf[off:off + N * hp * wp * Cp] = (s[:, None, None, None] * blk[None]).reshape(-1).to(torch.bfloat16)
+            blk = torch.zeros((2, hp, wp, Cp), dtype=torch.float32, device=device)
+            for k in range(2):
+                blk[k, ..., :C] = torch.from_numpy(np.ascontiguousarray(
+                    batch.B[k][:, bh[i]:bh[i + 1], bw[j]:bw[j + 1]].transpose(1, 2, 0))).to(device)
+            imgs = S[:, 0, None, None, None] * blk[0][None] + S[:, 1, None, None, None] * blk[1][None]
+            buf[off:off + N * hp * wp * Cp] = imgs.reshape(-1).to(torch.bfloat16)
     return buf
 
 
@@ -75,9 +116,9 @@ def test_c5_conv1_2_full_size(sc):
     Wt = synth.to_bf16_f32(synth.kaiming(g, C, C, 3, 3)).astype(np.float64)
     b = synth.uniform(g, (C,), -0.1, 0.1).astype(np.float64)
     gbase = synth.to_bf16_f32(synth.normal(g, (C, H, H))).astype(np.float64)
-    s, t = _scales(N, 0), _scales(N, 1, every=4)     # sum(t) and sum(s t) far from 0 (no cancellation)
-    x = _fill_level(lv0, base, s)
-    dy = _fill_level(lv1, gbase, t)
+    xb, gbt = _Batch(base), _Batch(gbase, swap=True)   # positive scales: sum S_x S_g far from 0
+    x = _fill_level(lv0, xb)
+    dy = _fill_level(lv1, gbt)
     w = pack_weight(torch.from_numpy(Wt), lv0["Cpad"], torch.bfloat16).cuda().contiguous()
     bias = torch.from_numpy(b.astype(np.float32)).cuda()
     yp = torch.empty(lv2["total_elems"], dtype=torch.bfloat16, device="cuda")
@@ -93,7 +134,7 @@ def test_c5_conv1_2_full_size(sc):
     torch.cuda.synchronize()
     lp0, lp1 = ref.layers
     for n, i, j in ((0, 0, 0), (137, 3, 5), (255, 7, 7), (64, 7, 0)):
-        X = base[:, lp0.Ih[i]:lp0.Ih[i + 1], lp0.Iw[j]:lp0.Iw[j + 1]][None] * s[n]
+        X = xb.patch(n, lp0.Ih[i:i + 2], lp0.Iw[j:j + 2])
         Y = O.conv_fwd_patch(X, Wt, b, 1, 1, lp0.pads_h[i], lp0.pads_w[j], relu=True)
         Yb = synth.to_bf16_f32(Y.astype(np.float32)).astype(np.float64)   # the GPU pools the bf16 conv outputs
         P, A = O.pool_fwd_patch(Yb, 2, 2, 2, 2, lp1.pads_h[i], lp1.pads_w[j])
@@ -101,17 +142,18 @@ def test_c5_conv1_2_full_size(sc):
         assert normwise(got, P) <= 2e-2, (n, i, j)
         Ag = _patch(am, lv2, i, j, n)[:, :C].astype(np.int64) & 0x7F
         assert np.mean(Ag != A) < 1e-2, (n, i, j)           # equal up to bf16 near-ties (R9, R13)
-        G = gbase[:, lp0.Ih[i]:lp0.Ih[i + 1], lp0.Iw[j]:lp0.Iw[j + 1]][None] * t[n]
+        G = gbt.patch(n, lp0.Ih[i:i + 2], lp0.Iw[j:j + 2])
         dX = O.conv_bwd_data_patch(G, Wt, X.shape[2], X.shape[3], 1, 1, lp0.pads_h[i], lp0.pads_w[j], mask=X)
         assert normwise(_patch(dx, lv0, i, j, n)[:, :C], dX) <= 2e-2, (n, i, j)
     # weight / bias gradient over all 256 images and 64 patches, by linearity in the per-image scales
-    Xp = O.split(base[None], lp0.Ih, lp0.Iw)
-    Gp = O.split(gbase[None], lp0.Ih, lp0.Iw)
-    dW1, db1 = O.conv_bwd_filter(Xp, Gp, lp0)
-    st, tt = float(np.sum(s * t)), float(np.sum(t))
+    dW_ref = _bilinear(xb, gbt, lambda X1, G1: O.conv_bwd_filter(O.split(X1, lp0.Ih, lp0.Iw),
+                                                                 O.split(G1, lp0.Ih, lp0.Iw), lp0)[0])
+    db_ref = sum(float(np.sum(gbt.S[:, l])) * O.conv_bwd_filter(O.split(xb.B[0][None], lp0.Ih, lp0.Iw),
+                                                               O.split(gbt.B[l][None], lp0.Ih, lp0.Iw), lp0)[1]
+                 for l in range(2))
     dWg = dw[..., :C].permute(0, 3, 1, 2).double().cpu().numpy()
-    assert normwise(dWg, st * dW1) <= 2e-2
-    assert normwise(db.double().cpu().numpy(), tt * db1) <= 2e-2
+    assert normwise(dWg, dW_ref) <= 2e-2
+    assert normwise(db.double().cpu().numpy(), db_ref) <= 2e-2
 
 
 @pytest.mark.parametrize("name,Cin,Cout,Hin,nsplit", [
@@ -139,10 +181,9 @@ def test_c5_deep_layers_full_size(sc, name, Cin, Cout, Hin, nsplit):
     Wt = synth.to_bf16_f32(synth.kaiming(g, Cout, Cin, 3, 3)).astype(np.float64)
     b = synth.uniform(g, (Cout,), -0.1, 0.1).astype(np.float64)
     gbase = synth.to_bf16_f32(synth.normal(g, (Cout, Hin, Hin))).astype(np.float64)
-    s, t = _scales(N, 0), _scales(N, 1, every=4)
-
-    x = _fill_level(lv0, base, s)
-    dy = _fill_level(lv1, gbase, t)
+    xb, gbt = _Batch(base), _Batch(gbase, swap=True)
+    x = _fill_level(lv0, xb)
+    dy = _fill_level(lv1, gbt)
     w = pack_weight(torch.from_numpy(Wt), lv0["Cpad"], torch.bfloat16).cuda().contiguous()
     bias = torch.from_numpy(b.astype(np.float32)).cuda()
     y = torch.empty(lv1["total_elems"], dtype=torch.bfloat16, device="cuda")
@@ -157,16 +198,18 @@ def test_c5_deep_layers_full_size(sc, name, Cin, Cout, Hin, nsplit):
     torch.cuda.synchronize()
     last = nsplit - 1
     for n, i, j in ((3, 0, 0), (200, last, last), (129, last // 2, 0)):
-        X = base[:, lp.Ih[i]:lp.Ih[i + 1], lp.Iw[j]:lp.Iw[j + 1]][None] * s[n]
+        X = xb.patch(n, lp.Ih[i:i + 2], lp.Iw[j:j + 2])
         Y = O.conv_fwd_patch(X, Wt, b, 1, 1, lp.pads_h[i], lp.pads_w[j], relu=True)
         assert normwise(_patch(y, lv1, i, j, n)[:, :Cout], Y) <= 2e-2, (n, i, j)
-        G = gbase[:, lp.Oh[i]:lp.Oh[i + 1], lp.Ow[j]:lp.Ow[j + 1]][None] * t[n]
+        G = gbt.patch(n, lp.Oh[i:i + 2], lp.Ow[j:j + 2])
         dX = O.conv_bwd_data_patch(G, Wt, X.shape[2], X.shape[3], 1, 1, lp.pads_h[i], lp.pads_w[j], mask=X)
         assert normwise(_patch(dx, lv0, i, j, n)[:, :Cin], dX) <= 2e-2, (n, i, j)
-    dW1, db1 = O.conv_bwd_filter(O.split(base[None], lp.Ih, lp.Iw), O.split(gbase[None], lp.Oh, lp.Ow), lp)
+    wg = lambda X1, G1: O.conv_bwd_filter(O.split(X1, lp.Ih, lp.Iw), O.split(G1, lp.Oh, lp.Ow), lp)
+    dW_ref = _bilinear(xb, gbt, lambda X1, G1: wg(X1, G1)[0])
+    db_ref = sum(float(np.sum(gbt.S[:, l])) * wg(xb.B[0][None], gbt.B[l][None])[1] for l in range(2))
     dWg = dw[..., :Cin].permute(0, 3, 1, 2).double().cpu().numpy()
-    assert normwise(dWg, float(np.sum(s * t)) * dW1) <= 2e-2
-    assert normwise(db.double().cpu().numpy(), float(np.sum(t)) * db1) <= 2e-2
+    assert normwise(dWg, dW_ref) <= 2e-2
+    assert normwise(db.double().cpu().numpy(), db_ref) <= 2e-2
 
 
 def test_c3_stride2_and_stem_full_size(sc):
@@ -177,7 +220,6 @@ def test_c3_stride2_and_stem_full_size(sc):
     from paper_conf_asplos_jinh19_b200.plan import SplitPlan
     from paper_conf_asplos_jinh19_b200.resnet import s2d_stem_grad, s2d_stem_layer, s2d_stem_weight
     g = synth.rng(46)
-    s, t = _scales(N, 0), _scales(N, 1, every=4)
     # ---- layer2_0_a: 3x3 s2 p1, 64 -> 128
     l = synth.conv(64, 128, s=2, name="layer2_0_a")
     Ob = sc.splitcnn_boundaries_even(28, 2)
@@ -187,7 +229,8 @@ def test_c3_stride2_and_stem_full_size(sc):
     base = synth.to_bf16_f32(synth.uniform(g, (64, 56, 56))).astype(np.float64)
     Wt = synth.to_bf16_f32(synth.kaiming(g, 128, 64, 3, 3)).astype(np.float64)
     gbase = synth.to_bf16_f32(synth.normal(g, (128, 28, 28))).astype(np.float64)
-    x, dy = _fill_level(lv0, base, s), _fill_level(lv1, gbase, t)
+    xb, gbt = _Batch(base), _Batch(gbase, swap=True)
+    x, dy = _fill_level(lv0, xb), _fill_level(lv1, gbt)
     w = pack_weight(torch.from_numpy(Wt), lv0["Cpad"], torch.bfloat16).cuda().contiguous()
     y = torch.empty(lv1["total_elems"], dtype=torch.bfloat16, device="cuda")
     sc.splitcnn_conv_fwd(pl.handle, 0, sc.BF16, x, w, None, y, sc.FLAG_RELU)
@@ -199,14 +242,15 @@ def test_c3_stride2_and_stem_full_size(sc):
     sc.splitcnn_conv_bwd_filter(pl.handle, 0, sc.BF16, x, dy, dw, None, 0.0, ws, ws_b)
     torch.cuda.synchronize()
     for n, i, j in ((5, 0, 1), (250, 1, 1)):
-        X = base[:, lp.Ih[i]:lp.Ih[i + 1], lp.Iw[j]:lp.Iw[j + 1]][None] * s[n]
+        X = xb.patch(n, lp.Ih[i:i + 2], lp.Iw[j:j + 2])
         Y = O.conv_fwd_patch(X, Wt, None, 2, 2, lp.pads_h[i], lp.pads_w[j], relu=True)
         assert normwise(_patch(y, lv1, i, j, n)[:, :128], Y) <= 2e-2, (n, i, j)
-        G = gbase[:, lp.Oh[i]:lp.Oh[i + 1], lp.Ow[j]:lp.Ow[j + 1]][None] * t[n]
+        G = gbt.patch(n, lp.Oh[i:i + 2], lp.Ow[j:j + 2])
         dX = O.conv_bwd_data_patch(G, Wt, X.shape[2], X.shape[3], 2, 2, lp.pads_h[i], lp.pads_w[j], mask=X)
         assert normwise(_patch(dx, lv0, i, j, n)[:, :64], dX) <= 2e-2, (n, i, j)
-    dW1, _ = O.conv_bwd_filter(O.split(base[None], lp.Ih, lp.Iw), O.split(gbase[None], lp.Oh, lp.Ow), lp)
-    assert normwise(dw[..., :64].permute(0, 3, 1, 2).double().cpu().numpy(), float(np.sum(s * t)) * dW1) <= 2e-2
+    dW_ref = _bilinear(xb, gbt, lambda X1, G1: O.conv_bwd_filter(O.split(X1, lp.Ih, lp.Iw),
+                                                                 O.split(G1, lp.Oh, lp.Ow), lp)[0])
+    assert normwise(dw[..., :64].permute(0, 3, 1, 2).double().cpu().numpy(), dW_ref) <= 2e-2
     # ---- the stem: 7x7 s2 p3 on 3 channels through the space-to-depth split and 4x4 s1 conv
     l7 = synth.conv(3, 64, k=7, s=2, p=3, name="conv1")
     Ob = sc.splitcnn_boundaries_even(112, 2)
@@ -217,25 +261,28 @@ def test_c3_stride2_and_stem_full_size(sc):
     img = synth.to_bf16_f32(synth.uniform(g, (3, H, H))).astype(np.float64)
     W7 = synth.to_bf16_f32(synth.kaiming(g, 64, 3, 7, 7)).astype(np.float64)
     gst = synth.to_bf16_f32(synth.normal(g, (64, 112, 112))).astype(np.float64)
-    xf = (torch.from_numpy(s.astype(np.float32))[:, None, None, None] * torch.from_numpy(img.astype(np.float32))[None]
-          ).to("cuda", torch.bfloat16).contiguous()
+    ib, gsb = _Batch(img), _Batch(gst, swap=True)
+    Sd = torch.from_numpy(ib.S.astype(np.float32)).cuda()
+    Bd = [torch.from_numpy(B.astype(np.float32)).cuda() for B in ib.B]
+    xf = (Sd[:, 0, None, None, None] * Bd[0][None] + Sd[:, 1, None, None, None] * Bd[1][None]).to(torch.bfloat16)
     xs = torch.empty(lvs0["total_elems"], dtype=torch.bfloat16, device="cuda")
     sc.splitcnn_split(pls.handle, 0, sc.BF16, xf, sc.NCHW_S2D, xs)
     ws7 = pack_weight(s2d_stem_weight(torch.from_numpy(W7)), lvs0["Cpad"], torch.bfloat16).cuda().contiguous()
     ys = torch.empty(lvs1["total_elems"], dtype=torch.bfloat16, device="cuda")
     sc.splitcnn_conv_fwd(pls.handle, 0, sc.BF16, xs, ws7, None, ys, sc.FLAG_RELU)
-    dys = _fill_level(lvs1, gst, t)
+    dys = _fill_level(lvs1, gsb)
     wsb = max(pls.workspace_size(0, sc.BF16, 2), 16)
     wss = torch.empty(wsb, dtype=torch.uint8, device="cuda")
     dws = torch.zeros((64, 4, 4, lvs0["Cpad"]), dtype=torch.float32, device="cuda")
     sc.splitcnn_conv_bwd_filter(pls.handle, 0, sc.BF16, xs, dys, dws, None, 0.0, wss, wsb)
     torch.cuda.synchronize()
     for n, i, j in ((1, 0, 0), (254, 1, 0)):
-        X = img[:, lp7.Ih[i]:lp7.Ih[i + 1], lp7.Iw[j]:lp7.Iw[j + 1]][None] * s[n]
+        X = ib.patch(n, lp7.Ih[i:i + 2], lp7.Iw[j:j + 2])
         Y = O.conv_fwd_patch(X, W7, None, 2, 2, lp7.pads_h[i], lp7.pads_w[j], relu=True)
         assert normwise(_patch(ys, lvs1, i, j, n)[:, :64], Y) <= 2e-2, (n, i, j)
-    dW7, _ = O.conv_bwd_filter(O.split(img[None], lp7.Ih, lp7.Iw), O.split(gst[None], lp7.Oh, lp7.Ow), lp7)
-    assert normwise(s2d_stem_grad(dws, 3).double().cpu().numpy(), float(np.sum(s * t)) * dW7) <= 2e-2
+    dW7 = _bilinear(ib, gsb, lambda X1, G1: O.conv_bwd_filter(O.split(X1, lp7.Ih, lp7.Iw),
+                                                              O.split(G1, lp7.Oh, lp7.Ow), lp7)[0])
+    assert normwise(s2d_stem_grad(dws, 3).double().cpu().numpy(), dW7) <= 2e-2
 
 
 def test_c5_split_merge_pool_full_size(sc):
@@ -262,8 +309,8 @@ def test_c5_split_merge_pool_full_size(sc):
     g = synth.rng(48)
     base = synth.to_bf16_f32(synth.normal(g, (128, 112, 112))).astype(np.float64)
     gb = synth.to_bf16_f32(synth.normal(g, (128, 56, 56))).astype(np.float64)
-    s, t = _scales(N, 0), _scales(N, 1, every=4)
-    xin, dy = _fill_level(lv0, base, s), _fill_level(lv1, gb, t)
+    xb, gbt = _Batch(base), _Batch(gb, swap=True)
+    xin, dy = _fill_level(lv0, xb), _fill_level(lv1, gbt)
     y = torch.empty(lv1["total_elems"], dtype=torch.bfloat16, device="cuda")
     a = torch.empty(lv1["total_elems"], dtype=torch.uint8, device="cuda")
     sc.splitcnn_pool_fwd(pp.handle, 0, sc.BF16, xin, y, a, 0)
@@ -271,11 +318,11 @@ def test_c5_split_merge_pool_full_size(sc):
     sc.splitcnn_pool_bwd(pp.handle, 0, sc.BF16, dy, a, dx, 0)
     torch.cuda.synchronize()
     for n, i, j in ((0, 0, 0), (255, 7, 7), (77, 2, 5)):
-        X = base[:, lref.Ih[i]:lref.Ih[i + 1], lref.Iw[j]:lref.Iw[j + 1]][None] * s[n]
+        X = xb.patch(n, lref.Ih[i:i + 2], lref.Iw[j:j + 2])
         Y, A = O.pool_fwd_patch(X, 2, 2, 2, 2, lref.pads_h[i], lref.pads_w[j])
         assert np.array_equal(_patch(y, lv1, i, j, n)[:, :128], Y), (n, i, j)
         assert np.array_equal(_patch(a, lv1, i, j, n)[:, :128].astype(np.int64) & 0x7F, A), (n, i, j)
-        G = gb[:, lref.Oh[i]:lref.Oh[i + 1], lref.Ow[j]:lref.Ow[j + 1]][None] * t[n]
+        G = gbt.patch(n, lref.Oh[i:i + 2], lref.Ow[j:j + 2])
         dX = O.pool_bwd_patch(G, A, X.shape[2], X.shape[3], 2, 2, 2, 2, lref.pads_h[i], lref.pads_w[j])
         assert np.array_equal(_patch(dx, lv0, i, j, n)[:, :128], dX), (n, i, j)
 

@@ -391,3 +391,27 @@ def test_add_and_gap_parity(sc, dtype_name):
     dref = O.split(O.global_avg_pool_bwd(Gp, H, W), [0, 4, 9], [0, 3, 7, 11])
     gd = unpack_level(_host(dx), lv)
     assert max(normwise(gd[i][j], dref[i][j]) for i in range(2) for j in range(3)) <= tol
+
+
+@pytest.mark.parametrize("dtype_name,cin,cout", [("bf16", 64, 64), ("bf16", 8, 64), ("fp32", 16, 16), ("bf16", 16, 16)])
+def test_bwd_filter_empty_patch_range(sc, dtype_name, cin, cout):
+    """An empty patch range (p0 == p1, e.g. a rank with no patches) contributes nothing: bwd_filter with
+    beta 0 writes dW = db = 0, with beta 1 leaves them unchanged (both the tcgen05 and the FFMA path,
+    db requested).  Regression: the db column-sum launch divided by zero on an empty range."""
+    from paper_conf_asplos_jinh19_b200.plan import SplitPlan
+    dtype = sc.BF16 if dtype_name == "bf16" else sc.FP32
+    l = synth.conv(cin, cout)
+    Ob = sc.splitcnn_boundaries_even(16, 2)
+    pl = SplitPlan([l], 2, cin, 16, 16, Ob, Ob)
+    lv0, lv1 = pl.levels
+    x = torch.randn(lv0["total_elems"], dtype=torch.float32, device="cuda").to(_td(sc, dtype))
+    dy = torch.randn(lv1["total_elems"], dtype=torch.float32, device="cuda").to(_td(sc, dtype))
+    ws_b = max(pl.workspace_size(0, dtype, 2), 16)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    for beta in (1.0, 0.0):
+        dw = torch.full((cout, 3, 3, lv0["Cpad"]), 3.0, dtype=torch.float32, device="cuda")
+        db = torch.full((cout,), 5.0, dtype=torch.float32, device="cuda")
+        for p in (0, 2, 4):
+            sc.splitcnn_conv_bwd_filter(pl.handle, 0, dtype, x, dy, dw, db, beta, ws, ws_b, 0, p, p)
+        torch.cuda.synchronize()
+        assert torch.equal(dw, torch.full_like(dw, 3.0 * beta)) and torch.equal(db, torch.full_like(db, 5.0 * beta))

@@ -22,7 +22,7 @@ def sc():
     return splitcnn
 
 
-def _run(sc, dtype, N=2, H=64, widths=(64, 128), split=(2, 2), seed=2, s2d=None):
+def _run(sc, dtype, N=2, H=64, widths=(64, 128), split=(2, 2), seed=2, s2d=None, exact=False):
     from paper_conf_asplos_jinh19_b200.resnet import ResSplitNet
     chain, blocks = synth.resnet18_blocks(*widths)
     net = ResSplitNet(chain, blocks, N, 3, H, H, split=split, dtype=dtype, s2d_stem=s2d)
@@ -30,14 +30,19 @@ def _run(sc, dtype, N=2, H=64, widths=(64, 128), split=(2, 2), seed=2, s2d=None)
         assert net.s2d == s2d
     g = synth.rng(seed)
     bf = dtype == sc.BF16
-    X = synth.uniform(g, (N, 3, H, H))
-    params = synth.resnet_params(g, chain, blocks)
+    if exact:   # dyadic draws: every fwd / dgrad sum exact in fp32 and fp64 (see test_gpu_stack)
+        X = synth.dyadic(g, (N, 3, H, H))
+        params = [p for p in synth.exact_layer_params(g, chain) if p is not None]
+        params += [p for p in synth.exact_layer_params(g, [b["ds"] for b in blocks if b["ds"] is not None])]
+    else:
+        X = synth.uniform(g, (N, 3, H, H))
+        params = synth.resnet_params(g, chain, blocks)
     if bf:
         X = synth.to_bf16_f32(X)
         params = [(synth.to_bf16_f32(Wt), b) for Wt, b in params]
     net.set_params([(torch.from_numpy(Wt), torch.from_numpy(b)) for Wt, b in params])
     L = net.region.levels[-1]
-    G = synth.normal(g, (N, L["C"], L["H"], L["W"]))
+    G = (synth.dyadic if exact else synth.normal)(g, (N, L["C"], L["H"], L["W"]))
     if bf:
         G = synth.to_bf16_f32(G)
     x = torch.from_numpy(X).to("cuda", net.tdtype)
@@ -66,25 +71,25 @@ def test_resnet_stack_fp32(sc):
     assert max(errs.values()) <= 1e-4, errs
 
 
-def test_resnet_stack_bf16(sc):
-    """bf16 tensor-core path, whole stack: the forward output within the per-op bf16 bound 2e-2.
-    The backward through ten bf16-stored gradient levels is not one op: a conv output that rounds
-    to the other side of a ReLU kink (or a 3x3 max-pool near-tie, R9) on one side routes a whole
-    gradient element differently.  At this size layer2's weight gradients reduce over only
-    K = 2 * 8 * 8 = 128 pixels, so one such flip moves a dW entry by ~1/sqrt(K) of its norm and the
-    whole-stack bf16 gradients carry 2-8e-2 normwise (measured on B200; deterministic).  They are
-    held to 1e-1 here as a regression bound, while every op is held to 2e-2 on its own
-    (test_gpu_ops) and the whole stack to 1e-4 in fp32 (above)."""
+def test_resnet_stack_bf16_forward(sc):
+    """bf16 tensor-core path, Kaiming draws: the forward output within the bf16 bar 2e-2.  (The
+    backward of such a draw is not comparable at 2e-2: a conv output that rounds to the other side of
+    a ReLU kink, or a 3x3 max-pool near-tie (R9), re-routes a whole gradient element; the backward is
+    checked on dyadic draws below.)"""
     errs = _run(sc, sc.BF16)
     assert errs["out"] <= 2e-2, errs
-    assert max(errs.values()) <= 1e-1, errs
 
 
-def test_resnet_stack_bf16_strided_stem(sc):
-    """The same stack with the stem run as the plain 7x7 s2 conv (no space-to-depth): same bounds."""
-    errs = _run(sc, sc.BF16, s2d=False)
-    assert errs["out"] <= 2e-2, errs
-    assert max(errs.values()) <= 1e-1, errs
+@pytest.mark.parametrize("s2d", [True, False])
+@pytest.mark.parametrize("N,H,seed", [(2, 64, 200), (1, 112, 201), (1, 56, 202)])
+def test_resnet_stack_bf16_whole_backward(sc, s2d, N, H, seed):
+    """bf16 whole ResNet split stack (s2d or plain 7x7 s2 stem, 3x3 s2 p1 pool, residual joins, 1x1 s2
+    downsample; H=56 gives ragged patches), forward and backward, every dW / db within the R13 bf16 bar
+    2e-2.  Dyadic draws make every fwd / dgrad sum exact, so both sides take the same decisions; the
+    output must agree exactly."""
+    errs = _run(sc, sc.BF16, N=N, H=H, seed=seed, s2d=s2d, exact=True)
+    assert errs["out"] == 0.0, errs
+    assert max(errs.values()) <= 2e-2, errs
 
 
 def test_s2d_stem_conv_matches_oracle_per_op(sc):
@@ -141,10 +146,10 @@ def test_resnet_stack_ragged_bf16(sc):
 @pytest.mark.parametrize("dtype_name", ["fp32", "bf16"])
 def test_resnet18_full_trunk(sc, dtype_name):
     """Whole trunk (f2): split region -> merge -> unsplit layer3/4 -> global average pool, against
-    tests/oracle_chain.run_resnet18_full.  fp32 end to end (pooled output, all 20 dW / db) at 1e-4; bf16
-    pooled output at 2e-2.  bf16 gradients only finite: at this size layer4 reduces over 2 x 2 x 2 = 8
-    pixels, so one bf16 ReLU-kink / pool near-tie decision moves a dW by a large fraction of its norm
-    (measured up to 0.34); every op is held to 2e-2 on its own in test_gpu_ops."""
+    tests/oracle_chain.run_resnet18_full.  fp32 end to end (pooled output, all 20 dW / db) at 1e-4
+    (Kaiming draws); bf16 end to end at the R13 bar 2e-2 on dyadic draws (every fwd / dgrad sum exact,
+    so both sides take the same ReLU / pool decisions; layer4 reduces over only 2 x 2 x 2 = 8 pixels,
+    where one flipped decision of a Kaiming draw moves a dW by up to 0.34 of its norm)."""
     from paper_conf_asplos_jinh19_b200.resnet import ResNet18Net
     dtype = sc.FP32 if dtype_name == "fp32" else sc.BF16
     bf = dtype == sc.BF16
@@ -153,13 +158,21 @@ def test_resnet18_full_trunk(sc, dtype_name):
     N, H = 2, 64
     net = ResNet18Net(rc, rb, tc, tb, N, 3, H, H, split=(2, 2), dtype=dtype)
     g = synth.rng(13)
-    X = synth.uniform(g, (N, 3, H, H))
-    params = synth.resnet_params(g, rc, rb) + synth.resnet_params(g, tc, tb)
+    if bf:
+        X = synth.dyadic(g, (N, 3, H, H))
+        params = []
+        for ch, bl in ((rc, rb), (tc, tb)):
+            params += [p for p in synth.exact_layer_params(g, ch) if p is not None]
+            params += synth.exact_layer_params(g, [b["ds"] for b in bl if b["ds"] is not None])
+        G = synth.dyadic(g, (N, 512))
+    else:
+        X = synth.uniform(g, (N, 3, H, H))
+        params = synth.resnet_params(g, rc, rb) + synth.resnet_params(g, tc, tb)
+        G = synth.normal(g, (N, 512))
     if bf:
         X = synth.to_bf16_f32(X)
         params = [(synth.to_bf16_f32(Wt), b) for Wt, b in params]
     net.set_params([(torch.from_numpy(Wt), torch.from_numpy(b)) for Wt, b in params])
-    G = synth.normal(g, (N, 512))
     if bf:
         G = synth.to_bf16_f32(G)
     pooled = net.forward(torch.from_numpy(X).to("cuda", net.tdtype))
@@ -174,8 +187,4 @@ def test_resnet18_full_trunk(sc, dtype_name):
         dW, db = net.grad_of(i)
         errs[f"dW{i}"] = normwise(dW.double().cpu().numpy(), dWs[i])
         errs[f"db{i}"] = normwise(db.double().cpu().numpy(), dbs[i])
-    if bf:
-        assert errs["out"] <= 2e-2, errs
-        assert all(np.isfinite(v) for v in errs.values()), errs
-    else:
-        assert max(errs.values()) <= 1e-4, errs
+    assert max(errs.values()) <= (2e-2 if bf else 1e-4), errs

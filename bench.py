@@ -109,9 +109,18 @@ def run_ours(args):
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if args.gpus != world:
-        world = max(world, 1)
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}: launch N ranks (bench.py self-launches "
+                         f"them when WORLD_SIZE is unset)")
+    if torch.cuda.device_count() < world or local >= torch.cuda.device_count():
+        raise SystemExit(f"{world} ranks but only {torch.cuda.device_count()} visible GPUs")
     torch.cuda.set_device(local)
     if world > 1 or args.force_dist:
+        if "RANK" not in os.environ:            # --force-dist at one rank without a launcher
+            import socket
+            so = socket.socket()
+            so.bind(("127.0.0.1", 0))
+            os.environ.update(RANK="0", WORLD_SIZE="1", MASTER_ADDR="127.0.0.1", MASTER_PORT=str(so.getsockname()[1]))
+            so.close()
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     c = workload(args.config)
     if getattr(args, "full", False) and c.get("resnet"):
@@ -152,9 +161,14 @@ def run_ours(args):
     if getattr(net, "set_bn_params", None) is not None:
         import synth
         net.set_bn_params(synth.bn_params(synth.rng(c["seed"] + 100), [W.shape[0] for W, _ in params]))
-    x = x_host.cuda()
     out_numel = net.output_numel()
-    dy = torch.randn(out_numel, generator=gen).to(net.tdtype).cuda()
+    dy_all = torch.randn(out_numel * world, generator=gen).to(net.tdtype)
+    dy_host = dy_all[rank * out_numel:(rank + 1) * out_numel]           # this rank's batch shard of dY
+    if world > 1:            # a rank reads only the input rows of its own patch rows (as its loader would)
+        h0, h1 = net.input_rows()
+        x_host = x_host[:, :, h0:h1].contiguous()
+    x = x_host.cuda()
+    dy = dy_host.cuda()
     stream = torch.cuda.current_stream()
 
     def step():
@@ -273,7 +287,8 @@ def run_ours(args):
     from paper_conf_asplos_jinh19_b200.pipeline import HostPipeline
     xh = x_host.pin_memory()
     dyh = dy.cpu().pin_memory()
-    gh = torch.empty(net.grad_flat.shape, dtype=net.grad_flat.dtype, pin_memory=True)
+    g_lo, g_hi = net.grad_slice() if hasattr(net, "grad_slice") else (0, net.grad_flat.numel())
+    gh = torch.empty(g_hi - g_lo, dtype=net.grad_flat.dtype, pin_memory=True)
     h2d = xh.numel() * xh.element_size() + dyh.numel() * dyh.element_size()
     d2h = gh.numel() * gh.element_size()
     ke = max(1, min(args.steps, 10))
@@ -313,7 +328,7 @@ def run_ours(args):
     line = {
         "metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True,
-        "scaling": "strong" if world > 1 else "weak", "vs_baseline": None,
+        "scaling": "strong", "vs_baseline": None,          # the global batch is fixed as N grows
         "dtype": args.dtype, "data": "synthetic (seeded PCG64 / torch.Generator; random-init weights)",
         "config": {"workload": f"{args.config}: {c['desc']}" + (" + unsplit layer3/4 + GAP (full trunk)" if c.get("full") else "")
                                + (" + whole-tensor BN" if args.bn else ""),
@@ -484,6 +499,19 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
+    if args.impl == "ours" and args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        # one process per GPU: re-launch this command under torch.distributed.run (127.0.0.1 rendezvous)
+        import socket
+        import torch
+        if torch.cuda.device_count() < args.gpus:
+            raise SystemExit(f"--gpus {args.gpus} but only {torch.cuda.device_count()} visible GPUs")
+        s = socket.socket()
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+        s.close()
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+        raise SystemExit(subprocess.call(cmd))
     if args.impl == "reference":
         run_reference(args)
     else:

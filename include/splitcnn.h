@@ -188,6 +188,14 @@ SPLITCNN_API splitcnn_status_t splitcnn_split(splitcnn_plan_t plan, int32_t leve
 SPLITCNN_API splitcnn_status_t splitcnn_split_s2d(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
                                       const void *x, int32_t x_channels, void *patches,
                                       int32_t p0, int32_t p1, splitcnn_stream_t stream);
+/* Eq. 4 from a ROW WINDOW of the input: x holds only rows [row0, row1) of the level's logical tensor
+ * (NCHW as [N][C][row1 - row0][W], or NHWC as [N][row1 - row0][W][C]) -- e.g. the rows of the patch
+ * rows a rank owns under patch-row sharding, so a rank copies only its own input rows to
+ * the device.  Same output as splitcnn_split on the full tensor.  Errors: layout not NCHW / NHWC, an
+ * empty or out-of-range window, a patch of [p0, p1) with rows outside the window. */
+SPLITCNN_API splitcnn_status_t splitcnn_split_rows(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                      const void *x, int32_t x_layout, int32_t row0, int32_t row1,
+                                      void *patches, int32_t p0, int32_t p1, splitcnn_stream_t stream);
 SPLITCNN_API splitcnn_status_t splitcnn_merge(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
                                  const void *patches, void *y, int32_t y_layout,
                                  int32_t p0, int32_t p1, splitcnn_stream_t stream);

@@ -128,6 +128,27 @@ extern "C" splitcnn_status_t splitcnn_split(splitcnn_plan_t plan, int32_t level,
     return check_launch("split");
 }
 
+extern "C" splitcnn_status_t splitcnn_split_rows(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
+                                                 const void *x, int32_t x_layout, int32_t row0, int32_t row1,
+                                                 void *patches, int32_t p0, int32_t p1, splitcnn_stream_t stream) {
+    if (!plan || level < 0 || level >= (int)plan->levels.size()) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad level");
+    TRY(check_dtype(dtype));
+    if (!x || !patches) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    if (x_layout != SPLITCNN_NCHW && x_layout != SPLITCNN_NHWC)
+        return fail(SPLITCNN_ERR_INVALID_VALUE, "split_rows: layout must be NCHW or NHWC");
+    NEED_ALIGNED(x, "x");
+    NEED_ALIGNED(patches, "patches");
+    TRY(check_range(plan, level, p0, p1));
+    const Level &L = plan->levels[level];
+    if (row0 < 0 || row1 > L.H || row0 >= row1) return fail(SPLITCNN_ERR_INVALID_VALUE, "split_rows: bad row window");
+    if (p1 == p0) return SPLITCNN_OK;
+    const int i0 = p0 / L.nw(), i1 = (p1 - 1) / L.nw();
+    if (L.bh[i0] < row0 || L.bh[i1 + 1] > row1)
+        return fail(SPLITCNN_ERR_INVALID_VALUE, "split_rows: a patch of [p0, p1) reads rows outside [row0, row1)");
+    launch_split(dtype, L, x, x_layout, patches, p0, p1, (cudaStream_t)stream, 0, row0, row1 - row0);
+    return check_launch("split_rows");
+}
+
 extern "C" splitcnn_status_t splitcnn_split_s2d(splitcnn_plan_t plan, int32_t level, splitcnn_dtype_t dtype,
                                                 const void *x, int32_t x_channels, void *patches, int32_t p0,
                                                 int32_t p1, splitcnn_stream_t stream) {

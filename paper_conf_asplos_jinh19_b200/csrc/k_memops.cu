@@ -31,7 +31,9 @@ __device__ __forceinline__ void dec3(uint32_t u, const Dec3 &d, int &x0, int &x1
 }
 template <typename T, bool NCHW, bool S2D = false>
 __global__ void __launch_bounds__(256) split_kernel(LevelDesc L, const T *__restrict__ x, T *__restrict__ P, int p0,
-                                                    int xc = 0) {
+                                                    int xc = 0, int row0 = 0, int xH = 0) {
+    // x holds rows [row0, row0 + xH) of the logical tensor (a rank's own rows); xH == 0: all L.H rows
+    if (xH == 0) xH = L.H;
     const PatchGeo g = patch_geo(L, p0 + blockIdx.y);
     const int G = L.Cpad / 8;
     const uint32_t units = (uint32_t)L.N * g.hp * g.wp * G;
@@ -72,8 +74,8 @@ __global__ void __launch_bounds__(256) split_kernel(LevelDesc L, const T *__rest
             }
         } else if (NCHW && std::is_same<T, __nv_bfloat16>::value) {
             // bf16 NCHW: raw 16-bit gathers from up to 8 channel planes packed into one 16-byte store
-            const uint16_t *src = reinterpret_cast<const uint16_t *>(x) + (((int64_t)n * L.C + c0) * L.H + hg) * L.W + wg;
-            const int64_t cs = (int64_t)L.H * L.W;
+            const uint16_t *src = reinterpret_cast<const uint16_t *>(x) + (((int64_t)n * L.C + c0) * xH + hg - row0) * L.W + wg;
+            const int64_t cs = (int64_t)xH * L.W;
             const int nc = min(8, L.C - c0);
             uint32_t w4[4] = {0u, 0u, 0u, 0u};
 #pragma unroll
@@ -85,9 +87,9 @@ __global__ void __launch_bounds__(256) split_kernel(LevelDesc L, const T *__rest
         } else if (NCHW) {
 #pragma unroll
             for (int k = 0; k < 8; ++k)
-                v[k] = (c0 + k < L.C) ? to_f(x[(((int64_t)n * L.C + c0 + k) * L.H + hg) * L.W + wg]) : 0.f;
+                v[k] = (c0 + k < L.C) ? to_f(x[(((int64_t)n * L.C + c0 + k) * xH + hg - row0) * L.W + wg]) : 0.f;
         } else {
-            const T *src = x + (((int64_t)n * L.H + hg) * L.W + wg) * L.C + c0;
+            const T *src = x + (((int64_t)n * xH + hg - row0) * L.W + wg) * L.C + c0;
             if ((L.C & 7) == 0) {
                 load8(src, v);
             } else {
@@ -149,16 +151,17 @@ static int64_t max_patch_units(const Level &L, int p0, int p1, int per_pixel) {
 }
 
 template <typename T>
-void launch_split_t(const Level &L, const void *x, int layout, void *P, int p0, int p1, cudaStream_t st, int xc) {
+void launch_split_t(const Level &L, const void *x, int layout, void *P, int p0, int p1, cudaStream_t st, int xc,
+                    int row0, int xH) {
     npatch_launch = p1 - p0;
     dim3 grid(grid_x_for(max_patch_units(L, p0, p1, L.Cpad / 8)), p1 - p0);
     LevelDesc d = make_level_desc(L);
     if (layout == SPLITCNN_NCHW_S2D)
         { split_kernel<T, true, true><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0, xc > 0 ? xc : L.C / 4); count_launch(); }
     else if (layout == SPLITCNN_NCHW)
-        { split_kernel<T, true><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0); count_launch(); }
+        { split_kernel<T, true><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0, 0, row0, xH); count_launch(); }
     else
-        { split_kernel<T, false><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0); count_launch(); }
+        { split_kernel<T, false><<<grid, 256, 0, st>>>(d, (const T *)x, (T *)P, p0, 0, row0, xH); count_launch(); }
 }
 
 template <typename T>
@@ -173,9 +176,9 @@ void launch_merge_t(const Level &L, const void *P, void *y, int layout, int p0, 
 }
 
 void launch_split(splitcnn_dtype_t dt, const Level &L, const void *x, int layout, void *P, int p0, int p1, cudaStream_t st,
-                  int xc) {
-    if (dt == SPLITCNN_BF16) launch_split_t<__nv_bfloat16>(L, x, layout, P, p0, p1, st, xc);
-    else launch_split_t<float>(L, x, layout, P, p0, p1, st, xc);
+                  int xc, int row0, int xH) {
+    if (dt == SPLITCNN_BF16) launch_split_t<__nv_bfloat16>(L, x, layout, P, p0, p1, st, xc, row0, xH);
+    else launch_split_t<float>(L, x, layout, P, p0, p1, st, xc, row0, xH);
 }
 void launch_merge(splitcnn_dtype_t dt, const Level &L, const void *P, void *y, int layout, int p0, int p1, cudaStream_t st) {
     if (dt == SPLITCNN_BF16) launch_merge_t<__nv_bfloat16>(L, P, y, layout, p0, p1, st);

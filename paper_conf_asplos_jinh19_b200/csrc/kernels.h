@@ -8,7 +8,7 @@ namespace splitcnn {
 
 // k_memops.cu
 void launch_split(splitcnn_dtype_t dt, const Level &L, const void *x, int layout, void *P, int p0, int p1, cudaStream_t st,
-                  int xc = 0);
+                  int xc = 0, int row0 = 0, int xH = 0);
 void launch_merge(splitcnn_dtype_t dt, const Level &L, const void *P, void *y, int layout, int p0, int p1, cudaStream_t st);
 void launch_pool_fwd(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, void *y,
                      uint8_t *a, int relu_bit, int p0, int p1, cudaStream_t st);

@@ -2,10 +2,13 @@
 
 Patches of a chained split region never communicate, so the region is sharded by contiguous
 PATCH ROWS: rank r owns patch range [p0, p1) and runs every region layer on it for the whole batch
-(weights replicated).  The unsplit tail runs BATCH-parallel, so at the join the region output is
-re-sharded (patch-sharded -> batch-sharded) and its gradient is sent back in backward.  The only
-reduction is the weight/bias-gradient sum (one NCCL all_reduce over one flat fp32 buffer,
-the wgrad allreduce of SURVEY 8(a) a10 / P:409-415).
+(weights replicated), reading only its own input rows (splitcnn_split_rows).  The unsplit tail runs
+BATCH-parallel, so at the join the region output is re-sharded (patch-sharded -> batch-sharded) and
+its gradient is sent back in backward.  The only reduction is the weight/bias-gradient sum (the wgrad
+allreduce of SURVEY 8(a) a10 / P:409-415), BUCKETED per layer and started as soon as a bucket's
+weight gradients are enqueued, so it runs on NCCL's stream while the rest of the backward computes:
+the step costs max(T_backward, 2|G|/alpha B) rather than their sum (the paper's pipelined model,
+P:413-415).
 
 Join exchange without packing copies: in a patch buffer `[N][Hp][Wp][C]` the images of one batch
 shard are a CONTIGUOUS slice, and on the receiving side the same slice is a whole patch buffer of a
@@ -97,9 +100,68 @@ def reverse(sends, recvs):
     return rsends, rrecvs
 
 
+# ------------------------------------------------------------------ bucketed, overlapped wgrad allreduce
+class GradBuckets:
+    """The flat fp32 gradient buffer cut into buckets of consecutive layers in BACKWARD completion order
+    (layers are laid out in forward order, so a bucket is one contiguous slice).  mark_ready(key) is
+    called right after a layer's weight-gradient call is enqueued; when every layer of a bucket is
+    ready, the bucket's all_reduce(SUM) is issued asynchronously (NCCL orders it after the enqueued
+    work of the current stream and runs it on its own stream, overlapping the remaining backward).
+    wait() makes the current stream wait for every issued bucket; the summed gradient is then in place.
+
+    segments: [(key, offset, numel)] in the order the backward finishes them."""
+
+    def __init__(self, flat: torch.Tensor, segments, bucket_bytes: int = 8 << 20, group=None):
+        self.flat, self.group = flat, group
+        self.buckets = []          # [lo, hi, keys]
+        self.of = {}
+        cur = None
+        for key, off, n in segments:
+            if cur is not None and off + n == cur[0] and (cur[1] - cur[0]) * flat.element_size() < bucket_bytes:
+                cur[0] = off
+                cur[2].append(key)
+            else:
+                cur = [off, off + n, [key]]
+                self.buckets.append(cur)
+            self.of[key] = len(self.buckets) - 1
+        self.pending = [len(b[2]) for b in self.buckets]
+        self.works = []
+
+    def rebind(self, flat: torch.Tensor):
+        self.flat = flat
+
+    def mark_ready(self, key):
+        b = self.of[key]
+        self.pending[b] -= 1
+        if self.pending[b] == 0:
+            lo, hi, _ = self.buckets[b]
+            self.works.append(dist.all_reduce(self.flat[lo:hi], op=dist.ReduceOp.SUM, group=self.group, async_op=True))
+
+    def wait(self):
+        assert all(p == 0 for p in self.pending), "a bucket was never completed"
+        for w in self.works:
+            w.wait()
+        self.works = []
+        self.pending = [len(b[2]) for b in self.buckets]
+
+
+def grad_segments(net, prefix: str, base: int = 0):
+    """[(key, offset, numel)] of a SplitNet's (dW, db) slices in the flat buffer, in backward order."""
+    segs = []
+    off = base
+    for key, layers, plan in (("r", net.region_layers, net.region), ("t", net.tail_layers, net.tail)):
+        for m, l in enumerate(layers):
+            if l["op"] == "conv":
+                n = l["cout"] * l["kh"] * l["kw"] * plan.levels[m]["Cpad"] + l["cout"]
+                segs.append(((prefix + key, m), off, n))
+                off += n
+    return segs[::-1]
+
+
 # ------------------------------------------------------------------ the distributed executor
 class DistSplitNet:
-    def __init__(self, c: dict, world: int, rank: int, dtype: int = sc.BF16, device="cuda"):
+    def __init__(self, c: dict, world: int, rank: int, dtype: int = sc.BF16, device="cuda",
+                 bucket_bytes: int = 8 << 20):
         self.world, self.rank, self.dtype = world, rank, dtype
         self.device = torch.device(device)
         N, H, W = c["N"], c["H"], c["W"]
@@ -122,6 +184,7 @@ class DistSplitNet:
         self.tail_net = SplitNet(tail, [], nb, L["C"], L["H"], L["W"], split=(1, 1), dtype=dtype, device=device,
                                  input_relu=last["op"] == "conv" and last.get("relu", True))
         self.tdtype = self.region_net.tdtype
+        self.bucket_bytes = bucket_bytes
         n_rg, n_tl = self.region_net.grad_numel(), self.tail_net.grad_numel()
         self.bind_grads(torch.zeros(n_rg + n_tl, dtype=torch.float32, device=device))
         self._set_join_plan(0)
@@ -137,11 +200,28 @@ class DistSplitNet:
         self.tail_net.timers = v
 
     def bind_grads(self, flat: torch.Tensor):
-        """All region + tail weight / bias gradients as views of one flat fp32 buffer (one allreduce)."""
+        """All region + tail weight / bias gradients as views of one flat fp32 buffer, cut into allreduce
+        buckets (tail layers finish first in backward, then the region's)."""
         n_rg = self.region_net.grad_numel()
         self.grad_flat = flat
         self.region_net.bind_grads(flat[:n_rg])
         self.tail_net.bind_grads(flat[n_rg:])
+        if getattr(self, "buckets", None) is None:
+            segs = grad_segments(self.tail_net, "t", n_rg) + grad_segments(self.region_net, "r", 0)
+            self.buckets = GradBuckets(flat, segs, self.bucket_bytes)
+            self.tail_net.wgrad_hook = lambda key, m: self.buckets.mark_ready(("t" + key, m))
+            self.region_net.wgrad_hook = lambda key, m: self.buckets.mark_ready(("r" + key, m))
+        self.buckets.rebind(flat)
+
+    def input_rows(self):
+        """Rows [h0, h1) of the input this rank reads (its patch rows at level 0)."""
+        return self.region_net.input_rows()
+
+    def grad_slice(self):
+        """[lo, hi) of the flat gradient this rank reads back to the host (1/world of it; every rank
+        holds the whole sum after the allreduce, so the host gets all of it once across ranks)."""
+        n = self.grad_flat.numel()
+        return (n * self.rank) // self.world, (n * (self.rank + 1)) // self.world
 
     def _set_join_plan(self, step: int):
         rn = self.region_net
@@ -170,6 +250,8 @@ class DistSplitNet:
         return self.tail_net.output_numel()
 
     def step(self, x, dy, stream=None):
+        """x: the full input or only this rank's input_rows() window ([N][C][h1-h0][W]); dy: the gradient
+        of this rank's batch shard of the tail output."""
         rn, tn = self.region_net, self.tail_net
         if rn.mode == "random":
             rn.replan(self.step_index)
@@ -189,6 +271,7 @@ class DistSplitNet:
         g_region = rn.grad[0]
         exchange(self.staging, g_region, rs, rr, self.rank)
         rn.backward(g_region, stream)
-        # the wgrad allreduce (sum over ranks of the per-rank partial sums)
-        dist.all_reduce(self.grad_flat, op=dist.ReduceOp.SUM)
+        # the wgrad allreduce (sum over ranks of the per-rank partial sums): the buckets were issued as
+        # their layers' weight gradients were enqueued; the step ends when the last one has landed
+        self.buckets.wait()
         self.step_index += 1

@@ -49,6 +49,7 @@ class SplitNet:
         # mask (a region whose gradient comes back from a tail that masks its input, dist.py)
         self.mask_output_grad = mask_output_grad
         self.timers = None       # list -> every library call is bracketed by CUDA events (bench.py)
+        self.wgrad_hook = None   # callable(key, m) after each layer's weight-gradient call is enqueued
         self._label = ""
         self.region = self._make_region_plan(0)
         self.patch_range = patch_range or (0, self.region.npatch)
@@ -320,12 +321,24 @@ class SplitNet:
         return self.mask_output_grad and bool(layers) and layers[-1]["op"] == "conv" and layers[-1].get("relu", True)
 
     # ------------------------------------------------------------------ passes
+    def input_rows(self):
+        """Input rows [h0, h1) the patch range reads (all rows for the whole grid)."""
+        lv = self.region.levels[0]
+        p0, p1 = self.patch_range
+        return lv["bh"][p0 // lv["n_w"]], lv["bh"][(p1 - 1) // lv["n_w"] + 1]
+
     def forward(self, x: torch.Tensor, stream=None, x_layout: int = sc.NCHW):
-        """x: full tensor (dtype) on the device, NCHW or NHWC.  Returns the output level buffer."""
+        """x: full tensor (dtype) on the device, NCHW or NHWC -- or only the input_rows() window of it
+        (NCHW [N][C][h1-h0][W]: a rank's own rows under patch-row sharding).  Returns the output level."""
         p0, p1 = self.patch_range
         R, dt, fl = self.region.handle, self.dtype, self.flags_extra
         b_in = 2 * self._bytes(self.region, 0)[0]
-        self._call("split", b_in, sc.splitcnn_split, R, 0, dt, x, x_layout, self.act_r[0], p0, p1, stream)
+        h0, h1 = self.input_rows()
+        if x.dim() == 4 and x_layout == sc.NCHW and x.shape[2] == h1 - h0 and h1 - h0 != self.H:
+            self._call("split", b_in * (h1 - h0) // self.H, sc.splitcnn_split_rows, R, 0, dt, x, x_layout, h0, h1,
+                       self.act_r[0], p0, p1, stream)
+        else:
+            self._call("split", b_in, sc.splitcnn_split, R, 0, dt, x, x_layout, self.act_r[0], p0, p1, stream)
         self._run_fwd("r", self.region, self.region_layers, self.act_r, p0, p1, stream)
         if self.tail:
             b_j = 2 * self._bytes(self.region, self.region.nlayers - 1)[1]
@@ -415,6 +428,8 @@ class SplitNet:
                                relu_src, self.ws, self.ws_bytes, self.flags_extra, p0, p1, stream)
                 self._call("conv_wgrad", work, sc.splitcnn_conv_bwd_filter, plan.handle, m, self.dtype, acts[m], g, dW,
                            db, 0.0, self.ws, self.ws_bytes, self.flags_extra, p0, p1, stream)
+                if self.wgrad_hook is not None:      # e.g. dist.GradBuckets: start this layer's allreduce
+                    self.wgrad_hook(key, m)
             else:
                 flags = sc.FLAG_POOL_RELU_MASK if self._masked(key, m) else 0
                 bi, bo = self._bytes(plan, m)

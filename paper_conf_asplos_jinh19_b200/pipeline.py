@@ -57,9 +57,11 @@ class HostPipeline:
         self.in_free[b].record(self.compute)
         self.g_ready[b].record(self.compute)
         if grads_host is not None:
+            # a sharded executor reads back only its slice of the (allreduced) gradient
+            lo, hi = self.net.grad_slice() if hasattr(self.net, "grad_slice") else (0, self.g[b].numel())
             with torch.cuda.stream(self.d2h):
                 self.d2h.wait_event(self.g_ready[b])
-                grads_host.copy_(self.g[b], non_blocking=True)
+                grads_host.copy_(self.g[b][lo:hi], non_blocking=True)
                 self.g_free[b].record(self.d2h)
         else:
             self.g_free[b].record(self.compute)

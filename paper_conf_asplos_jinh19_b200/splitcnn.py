@@ -33,7 +33,7 @@ EXPORTED = [
     "splitcnn_boundaries_even", "splitcnn_boundaries_random",
     "splitcnn_plan_create", "splitcnn_plan_destroy", "splitcnn_plan_num_layers", "splitcnn_plan_level",
     "splitcnn_plan_layer", "splitcnn_workspace_size",
-    "splitcnn_split", "splitcnn_split_s2d", "splitcnn_merge",
+    "splitcnn_split", "splitcnn_split_s2d", "splitcnn_split_rows", "splitcnn_merge",
     "splitcnn_conv_fwd", "splitcnn_conv_bwd_data", "splitcnn_conv_bwd_filter",
     "splitcnn_pool_fwd", "splitcnn_pool_bwd", "splitcnn_conv_pool_fwd", "splitcnn_conv_pool_supported", "splitcnn_add",
     "splitcnn_gap_fwd", "splitcnn_gap_bwd",
@@ -86,6 +86,7 @@ _sig("splitcnn_plan_layer", [_vp, _i32, ctypes.POINTER(LayerGeom)])
 _sig("splitcnn_workspace_size", [_vp, _i32, ctypes.c_int, _i32, ctypes.POINTER(_sz)])
 _sig("splitcnn_split", [_vp, _i32, ctypes.c_int, _vp, _i32, _vp, _i32, _i32, _vp])
 _sig("splitcnn_split_s2d", [_vp, _i32, ctypes.c_int, _vp, _i32, _vp, _i32, _i32, _vp])
+_sig("splitcnn_split_rows", [_vp, _i32, ctypes.c_int, _vp, _i32, _i32, _i32, _vp, _i32, _i32, _vp])
 _sig("splitcnn_merge", [_vp, _i32, ctypes.c_int, _vp, _vp, _i32, _i32, _i32, _vp])
 _sig("splitcnn_conv_fwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
 _sig("splitcnn_conv_bwd_data", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _vp, _sz, _u32, _i32, _i32, _vp])
@@ -251,6 +252,11 @@ def splitcnn_split(plan, level, dtype, x, x_layout, patches, p0=0, p1=-1, stream
 
 def splitcnn_merge(plan, level, dtype, patches, y, y_layout, p0=0, p1=-1, stream=None):
     _check(_lib.splitcnn_merge(plan, level, dtype, _ptr(patches), _ptr(y), y_layout, p0, p1, _stream(stream)))
+
+
+def splitcnn_split_rows(plan, level, dtype, x, x_layout, row0, row1, patches, p0=0, p1=-1, stream=None):
+    _check(_lib.splitcnn_split_rows(plan, level, dtype, _ptr(x), x_layout, row0, row1, _ptr(patches), p0, p1,
+                                    _stream(stream)))
 
 
 def splitcnn_split_s2d(plan, level, dtype, x, x_channels, patches, p0=0, p1=-1, stream=None):

@@ -1,6 +1,8 @@
-"""Multi-process CPU test (gloo, world_size 2) of the patch-parallel join exchange of dist.py:
-patch-sharded region output -> batch-sharded tail input (forward) and back (backward), as plain
-tensor views with no packing.  Runs on CPU: the plan is host code and the exchange is plumbing."""
+"""Multi-process CPU tests (gloo, world_size 2 and 4) of the communication of one patch-parallel step
+(dist.py): the join exchange (patch-sharded region output -> batch-sharded tail input, and its
+gradient back) as plain tensor views with no packing, and the bucketed wgrad allreduce (GradBuckets:
+buckets issued asynchronously as layers finish in backward order) whose result must be the oracle's
+O10 sum of the per-rank partial gradients.  Runs on CPU: the plan is host code, the exchange plumbing."""
 import os
 import socket
 
@@ -62,22 +64,53 @@ def _worker(rank, world, port, q):
         for qq, (off, per) in enumerate(D.patch_geometry(lf)):
             if p0 <= qq < p1:
                 ok_bwd &= bool(np.array_equal(greg[off:off + N * per].numpy(), ref[off:off + N * per]))
-        q.put((rank, ok_fwd, ok_bwd))
+        # bucketed wgrad allreduce: per-rank partial gradients (dyadic, so any summation order is exact),
+        # layers completed in backward order, buckets issued asynchronously as they fill
+        from oracle import ops as OO
+        sizes = [1728 + 8, 36864 + 64, 73728 + 128, 147456 + 128, 4608 + 512, 9 + 1]   # (dW + db) per layer
+        offs = np.cumsum([0] + sizes)
+        segs = [((("r", m)), int(offs[m]), sizes[m]) for m in range(len(sizes))][::-1]
+        parts = [synth.dyadic(synth.rng(100 + r), (int(offs[-1]),)).astype(np.float64) for r in range(world)]
+        flat = torch.from_numpy(parts[rank].copy())
+        B = D.GradBuckets(flat, segs, bucket_bytes=300_000)
+        cover = sorted((lo, hi) for lo, hi, _ in B.buckets)
+        ok_buckets = (cover[0][0] == 0 and cover[-1][1] == offs[-1] and len(B.buckets) < len(sizes)
+                      and all(a[1] == b[0] for a, b in zip(cover, cover[1:])))
+        for step in range(2):          # twice: the pending counters re-arm after wait()
+            flat.copy_(torch.from_numpy(parts[rank]))
+            for key, _, _ in segs:
+                B.mark_ready(key)
+            B.wait()
+            ok_buckets &= bool(np.array_equal(flat.numpy(), OO.allreduce_sum(parts)))
+        q.put((rank, ok_fwd, ok_bwd, ok_buckets))
     finally:
         dist.destroy_process_group()
 
 
-def test_join_exchange_gloo_world2():
+@pytest.mark.parametrize("world", [2, 4])
+def test_step_communication_gloo(world):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
     for p in procs:
         p.start()
     for p in procs:
         p.join(timeout=180)
-    res = sorted(q.get(timeout=5) for _ in range(2))
-    assert res == [(0, True, True), (1, True, True)], res
+    res = sorted(q.get(timeout=5) for _ in range(world))
+    assert res == [(r, True, True, True) for r in range(world)], res
+
+
+def test_grad_buckets_layout():
+    """Buckets are contiguous slices of consecutive layers in backward order, merged up to the byte cap."""
+    from paper_conf_asplos_jinh19_b200 import dist as D
+    flat = torch.zeros(100, dtype=torch.float32)
+    segs = [(("t", 3), 90, 10), (("t", 1), 60, 30), (("r", 2), 20, 40), (("r", 0), 0, 20)][::1]
+    B = D.GradBuckets(flat, segs, bucket_bytes=4 * 35)
+    assert [(lo, hi, keys) for lo, hi, keys in B.buckets] == [(60, 100, [("t", 3), ("t", 1)]),
+                                                              (20, 60, [("r", 2)]), (0, 20, [("r", 0)])]
+    B = D.GradBuckets(flat, segs, bucket_bytes=1 << 20)
+    assert len(B.buckets) == 1 and B.buckets[0][:2] == [0, 100]
 
 
 def test_patch_and_batch_ranges():

@@ -415,3 +415,34 @@ def test_bwd_filter_empty_patch_range(sc, dtype_name, cin, cout):
             sc.splitcnn_conv_bwd_filter(pl.handle, 0, dtype, x, dy, dw, db, beta, ws, ws_b, 0, p, p)
         torch.cuda.synchronize()
         assert torch.equal(dw, torch.full_like(dw, 3.0 * beta)) and torch.equal(db, torch.full_like(db, 5.0 * beta))
+
+
+@pytest.mark.parametrize("layout", ["NCHW", "NHWC"])
+def test_split_rows_matches_full_split(sc, layout):
+    """splitcnn_split_rows (a rank's own input rows under patch-row sharding) writes bit-exactly the
+    patches splitcnn_split writes from the full tensor, for every contiguous block of patch rows of a
+    ragged 4x3 split; patches outside [p0, p1) are untouched; a window missing a needed row is refused."""
+    from paper_conf_asplos_jinh19_b200.plan import SplitPlan
+    L = sc.NCHW if layout == "NCHW" else sc.NHWC
+    l = synth.conv(5, 8)
+    N, H, W = 3, 29, 22
+    Oh, Ow = [0, 5, 13, 20, 29], [0, 7, 15, 22]
+    pl = SplitPlan([l], N, 5, H, W, Oh, Ow)
+    lv = pl.levels[0]
+    x = torch.randn((N, 5, H, W), dtype=torch.float32, device="cuda").to(torch.bfloat16)
+    xl = x if L == sc.NCHW else x.permute(0, 2, 3, 1).contiguous()
+    ref = torch.empty(lv["total_elems"], dtype=torch.bfloat16, device="cuda")
+    sc.splitcnn_split(pl.handle, 0, sc.BF16, xl, L, ref)
+    bh, nw = lv["bh"], lv["n_w"]
+    for r0 in range(4):
+        for r1 in range(r0 + 1, 5):
+            h0, h1 = bh[r0], bh[r1]
+            xr = (xl[:, :, h0:h1] if L == sc.NCHW else xl[:, h0:h1]).contiguous()
+            got = torch.full_like(ref, 7.0)
+            sc.splitcnn_split_rows(pl.handle, 0, sc.BF16, xr, L, h0, h1, got, r0 * nw, r1 * nw)
+            lo = N * lv["Cpad"] * bh[r0] * W
+            hi = N * lv["Cpad"] * bh[r1] * W
+            assert torch.equal(got[lo:hi], ref[lo:hi]), (r0, r1)
+            assert bool((got[:lo] == 7).all()) and bool((got[hi:] == 7).all())
+    with pytest.raises(Exception):
+        sc.splitcnn_split_rows(pl.handle, 0, sc.BF16, xl[:, :, 1:13].contiguous(), L, 1, 13, ref, 0, 2 * nw)

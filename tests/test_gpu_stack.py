@@ -166,10 +166,13 @@ def test_dist_executor_world1_matches_single(sc):
     single.step(x, dy)
     dnet.step(x, dy)
     torch.cuda.synchronize()
+    assert len(dnet.buckets.buckets) > 1            # the allreduce went out in several overlapped buckets
+    assert dnet.input_rows() == (0, 224) and dnet.grad_slice() == (0, dnet.grad_flat.numel())
     bad = {k: float((v[0] - dnet.grads[k][0]).abs().max()) for k, v in single.grads.items()
            if not (torch.equal(v[0], dnet.grads[k][0]) and torch.equal(v[1], dnet.grads[k][1]))}
     assert torch.equal(single.act_t[-1], dnet.tail_net.act_r[-1]), "forward outputs differ"
     assert not bad, f"gradients differ: {bad}"
+    dist.destroy_process_group()
 
 
 @pytest.mark.parametrize("static", [False, True])

@@ -74,10 +74,17 @@ typedef enum {
     SPLITCNN_ERR_OOM = 5
 } splitcnn_status_t;
 
-/* Storage / compute precision of activations and weights.
- *  BF16: bf16 storage, fp32 accumulation (tcgen05 tensor cores where the shape allows).
- *  FP32: fp32 storage, fp32-accurate arithmetic (FFMA).  Accumulation is fp32. */
-typedef enum { SPLITCNN_BF16 = 0, SPLITCNN_FP32 = 1 } splitcnn_dtype_t;
+/* Storage / compute precision of activations and weights.  Accumulation is fp32.
+ *  BF16: bf16 storage, tcgen05 kind::f16 where the shape allows.
+ *  TF32: fp32 storage; forward / stride-1 data gradient as ONE tcgen05 kind::tf32 pass (operands read as
+ *        TF32); weight gradient by bf16 operand splitting (v = v1 + v2, products of i + j <= 1) on the
+ *        bf16 tensor-core kernels.  Error ~1e-3..1e-4 normwise (R13: held to 2e-3).
+ *  FP32: fp32 storage, fp32-accurate (R13: 1e-4): forward (conv_fwd_ws with a workspace) and stride-1
+ *        data gradient as 3xTF32 (v = hi + lo; lo*W_hi + hi*W_lo + hi*W_hi, three kind::tf32 passes),
+ *        weight gradient by 3-way bf16 splitting (products of i + j <= 2); FFMA on the CUDA cores where
+ *        the tensor-core path does not take the shape (and for conv_fwd without a workspace).
+ *  All three share the element layout of their storage type; every non-conv op treats TF32 as FP32. */
+typedef enum { SPLITCNN_BF16 = 0, SPLITCNN_FP32 = 1, SPLITCNN_TF32 = 2 } splitcnn_dtype_t;
 
 typedef enum { SPLITCNN_OP_CONV = 0, SPLITCNN_OP_MAXPOOL = 1 } splitcnn_op_t;
 
@@ -209,6 +216,14 @@ SPLITCNN_API splitcnn_status_t splitcnn_merge(splitcnn_plan_t plan, int32_t leve
 SPLITCNN_API splitcnn_status_t splitcnn_conv_fwd(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
                                     const void *x, const void *w, const float *bias, void *y,
                                     uint32_t flags, int32_t p0, int32_t p1, splitcnn_stream_t stream);
+
+/* The same with a caller workspace (size: splitcnn_workspace_size, op 0): with SPLITCNN_FP32 the forward
+ * then runs as 3xTF32 on the tensor cores (the hi / lo operand halves live in ws); without one (or with
+ * BF16 / TF32, which need none) it is splitcnn_conv_fwd. */
+SPLITCNN_API splitcnn_status_t splitcnn_conv_fwd_ws(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                       const void *x, const void *w, const float *bias, void *y,
+                                       uint32_t flags, void *ws, size_t ws_bytes, int32_t p0, int32_t p1,
+                                       splitcnn_stream_t stream);
 
 /* Fused forward of a conv (+bias, ReLU) `layer` and the 2x2 / stride-2 / unpadded max-pool
  * `layer + 1` that follows it (ReLU in place): the tcgen05 epilogue pools the

@@ -58,7 +58,7 @@ namespace {
 bool aligned16(const void *p) { return ((uintptr_t)p & 15u) == 0; }
 
 splitcnn_status_t check_dtype(splitcnn_dtype_t dt) {
-    if (dt != SPLITCNN_BF16 && dt != SPLITCNN_FP32) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad dtype");
+    if (dt != SPLITCNN_BF16 && dt != SPLITCNN_FP32 && dt != SPLITCNN_TF32) return fail(SPLITCNN_ERR_INVALID_VALUE, "bad dtype");
     return SPLITCNN_OK;
 }
 
@@ -98,12 +98,16 @@ extern "C" splitcnn_status_t splitcnn_workspace_size(splitcnn_plan_t plan, int32
     const Level &Li = plan->levels[layer], &Lo = plan->levels[layer + 1];
     const LayerGeom &g = plan->layers[layer];
     size_t b = 0;
-    if (op == 1) {
-        if (conv_tc_supported(1, dtype, Li, Lo, g)) b = conv_tc_ws_bytes(1, Li, Lo, g);
+    const bool f32 = dtype != SPLITCNN_BF16;
+    if (op == 0) {
+        if (f32 && conv_tc_supported(0, dtype, Li, Lo, g)) b = f32tc_ws_bytes(0, dtype, Li, Lo, g);
+    } else if (op == 1) {
+        if (conv_tc_supported(1, dtype, Li, Lo, g)) b = f32 ? f32tc_ws_bytes(1, dtype, Li, Lo, g) : conv_tc_ws_bytes(1, Li, Lo, g);
     } else if (op == 2) {
         b = wgrad_simt_ws_bytes(Li, Lo, g);
-        if (conv_tc_supported(2, dtype, Li, Lo, g)) b = std::max(b, conv_tc_ws_bytes(2, Li, Lo, g));
-    } else if (op != 0) {
+        if (conv_tc_supported(2, SPLITCNN_BF16, Li, Lo, g))
+            b = std::max(b, f32 ? f32tc_ws_bytes(2, dtype, Li, Lo, g) : conv_tc_ws_bytes(2, Li, Lo, g));
+    } else {
         return fail(SPLITCNN_ERR_INVALID_VALUE, "workspace_size: op must be 0, 1 or 2");
     }
     *bytes = b;
@@ -180,26 +184,38 @@ extern "C" splitcnn_status_t splitcnn_merge(splitcnn_plan_t plan, int32_t level,
     return check_launch("merge");
 }
 
-extern "C" splitcnn_status_t splitcnn_conv_fwd(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype, const void *x,
-                                               const void *w, const float *bias, void *y, uint32_t flags, int32_t p0,
-                                               int32_t p1, splitcnn_stream_t stream) {
+extern "C" splitcnn_status_t splitcnn_conv_fwd_ws(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                                  const void *x, const void *w, const float *bias, void *y,
+                                                  uint32_t flags, void *ws, size_t ws_bytes, int32_t p0, int32_t p1,
+                                                  splitcnn_stream_t stream) {
     TRY(check_layer(plan, layer, SPLITCNN_OP_CONV));
     TRY(check_dtype(dtype));
     if (!x || !w || !y) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
     NEED_ALIGNED(x, "x");
     NEED_ALIGNED(w, "w");
     NEED_ALIGNED(y, "y");
+    NEED_ALIGNED(ws, "ws");
     TRY(check_range(plan, layer, p0, p1));
     if (p1 == p0) return SPLITCNN_OK;
     const Level &Li = plan->levels[layer], &Lo = plan->levels[layer + 1];
     const LayerGeom &g = plan->layers[layer];
     const int relu = (flags & SPLITCNN_FLAG_RELU) ? 1 : 0;
-    if (!(flags & SPLITCNN_FLAG_FORCE_SIMT) && conv_tc_supported(0, dtype, Li, Lo, g)) {
+    const bool tc = !(flags & SPLITCNN_FLAG_FORCE_SIMT) && conv_tc_supported(0, dtype, Li, Lo, g);
+    if (tc && dtype == SPLITCNN_BF16) {
         TRY(launch_conv_fwd_tc(Li, Lo, g, x, w, bias, y, relu, p0, p1, (cudaStream_t)stream));
+    } else if (tc && (dtype == SPLITCNN_TF32 || (ws && ws_bytes >= f32tc_ws_bytes(0, dtype, Li, Lo, g)))) {
+        // TF32: one kind::tf32 pass; FP32 with a workspace: 3xTF32 (without one: FFMA below)
+        TRY(launch_conv_fwd_f32tc(dtype, Li, Lo, g, x, w, bias, y, relu, p0, p1, ws, (cudaStream_t)stream));
     } else {
         launch_conv_fwd_simt(dtype, Li, Lo, g, x, w, bias, y, relu, p0, p1, (cudaStream_t)stream);
     }
     return check_launch("conv_fwd");
+}
+
+extern "C" splitcnn_status_t splitcnn_conv_fwd(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype, const void *x,
+                                               const void *w, const float *bias, void *y, uint32_t flags, int32_t p0,
+                                               int32_t p1, splitcnn_stream_t stream) {
+    return splitcnn_conv_fwd_ws(plan, layer, dtype, x, w, bias, y, flags, nullptr, 0, p0, p1, stream);
 }
 
 // conv `layer` (+bias, ReLU) followed by a 2x2 / stride-2 / unpadded max-pool `layer + 1` whose
@@ -264,9 +280,11 @@ extern "C" splitcnn_status_t splitcnn_conv_bwd_data(splitcnn_plan_t plan, int32_
     const Level &Li = plan->levels[layer], &Lo = plan->levels[layer + 1];
     const LayerGeom &g = plan->layers[layer];
     if (!(flags & SPLITCNN_FLAG_FORCE_SIMT) && conv_tc_supported(1, dtype, Li, Lo, g)) {
-        const size_t need = conv_tc_ws_bytes(1, Li, Lo, g);
+        const bool f32 = dtype != SPLITCNN_BF16;
+        const size_t need = f32 ? f32tc_ws_bytes(1, dtype, Li, Lo, g) : conv_tc_ws_bytes(1, Li, Lo, g);
         if (ws_bytes < need || (need && !ws)) return fail(SPLITCNN_ERR_INVALID_VALUE, "conv_bwd_data: workspace too small");
-        TRY(launch_conv_dgrad_tc(Li, Lo, g, dy, w, dx, relu_src, ws, p0, p1, (cudaStream_t)stream));
+        if (f32) TRY(launch_conv_dgrad_f32tc(dtype, Li, Lo, g, dy, w, dx, relu_src, p0, p1, ws, (cudaStream_t)stream));
+        else TRY(launch_conv_dgrad_tc(Li, Lo, g, dy, w, dx, relu_src, ws, p0, p1, (cudaStream_t)stream));
     } else {
         launch_conv_dgrad_simt(dtype, Li, Lo, g, dy, w, dx, relu_src, p0, p1, (cudaStream_t)stream);
     }
@@ -288,10 +306,15 @@ extern "C" splitcnn_status_t splitcnn_conv_bwd_filter(splitcnn_plan_t plan, int3
     TRY(check_range(plan, layer, p0, p1));
     const Level &Li = plan->levels[layer], &Lo = plan->levels[layer + 1];
     const LayerGeom &g = plan->layers[layer];
-    const bool tc = !(flags & SPLITCNN_FLAG_FORCE_SIMT) && conv_tc_supported(2, dtype, Li, Lo, g);
-    const size_t need = tc ? conv_tc_ws_bytes(2, Li, Lo, g) : wgrad_simt_ws_bytes(Li, Lo, g);
+    // fp32 storage: bf16 operand splitting onto the bf16 tensor-core kernels where they take the shape
+    const bool f32 = dtype != SPLITCNN_BF16;
+    const bool tc = !(flags & SPLITCNN_FLAG_FORCE_SIMT) && conv_tc_supported(2, SPLITCNN_BF16, Li, Lo, g);
+    const size_t need = !tc ? wgrad_simt_ws_bytes(Li, Lo, g) : f32 ? f32tc_ws_bytes(2, dtype, Li, Lo, g)
+                                                                   : conv_tc_ws_bytes(2, Li, Lo, g);
     if (ws_bytes < need || !ws) return fail(SPLITCNN_ERR_INVALID_VALUE, "conv_bwd_filter: workspace too small");
-    if (tc) {
+    if (tc && f32) {
+        TRY(launch_conv_wgrad_f32tc(dtype, Li, Lo, g, x, dy, dw, db, beta, ws, p0, p1, (cudaStream_t)stream));
+    } else if (tc) {
         TRY(launch_conv_wgrad_tc(Li, Lo, g, x, dy, dw, db, beta, ws, p0, p1, (cudaStream_t)stream));
     } else {
         launch_conv_wgrad_simt(dtype, Li, Lo, g, x, dy, dw, db, beta, ws, p0, p1, (cudaStream_t)stream);

@@ -369,7 +369,7 @@ int launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, flo
     const int64_t dy_bytes = P * Lo.Cpad * (int64_t)(dt == SPLITCNN_BF16 ? 2 : 4);
     const bool warp_ok = G <= 64 && (32 % G == 0 || G % 32 == 0) && dy_bytes >= (32ll << 20) &&
                          (G >= 16 || dy_bytes < (1ll << 30));
-    if (warp_ok && !getenv("SPLITCNN_COLSUM_SMEM")) {
+    if (warp_ok) {
         const int RB = G >= 32 ? 256 / G : 8;
         float *rows = part + (int64_t)Z * cout;
         if (dt == SPLITCNN_BF16)

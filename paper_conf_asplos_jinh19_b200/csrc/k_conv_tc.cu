@@ -69,15 +69,14 @@ struct TcConvParams {
     __nv_bfloat16 *y;
     const __nv_bfloat16 *relu_src;
     int relu;
+    int accum;        // TF32 direct epilogue: y = acc + y (3xTF32 passes), bias / ReLU / mask after the sum
     int tpp;          // tiles per patch when uniform (O(1) decode), else 0
     int direct;       // 1: per-thread global stores (odd channel pads); 0: smem-staged TMA store
     int ychunk;       // channels per output box (64, 32, 16 or 8)
     uint32_t y_mask;  // swizzle mask of the staging tile (7 / 3 / 1 / 0)
     uint32_t stage_off, bar_off;  // smem layout
     int ybufs;                    // staging buffers (2: the TMA store of tile t overlaps tile t+1)
-    int dbg;                      // experiments only (SPLITCNN_DBG): 1 no TMA store, 2 no MMA, 4 no loads, 8 no TMEM->smem
     int egroups;                  // 2: two independent 4-warp epilogue groups, one per TMEM accumulator
-    unsigned long long *trace;    // debug (SPLITCNN_TRACE): per-tile clock64 events of CTA 0
     int cta2;                     // 2-CTA MMA (cluster of 2, M = 256): each CTA owns one 128-row M box and N/2 of B
     int BNh;                      // rows of B per CTA (BN / 2 in 2-CTA mode, else BN)
     int total_m, total_pairs, m_tpp;
@@ -308,10 +307,9 @@ __device__ __forceinline__ void pool32(const uint32_t *w, int bw, bool writer, _
     reinterpret_cast<uint4 *>(ap)[1] = make_uint4(ab[4], ab[5], ab[6], ab[7]);
 }
 
-#define TC_TRACE(i, e) \
-    do { if (p.trace && blockIdx.x == 0 && (i) < 256) p.trace[(i) * 8 + (e)] = clock64(); } while (0)
-
-template <bool BIAS, bool RELU, bool MASK, bool CTA2, bool POOL = false>
+// TF32: fp32 operands (kind::tf32 MMAs on the same byte-addressed tiles: an fp32 channel is two bf16
+// "channels" of the byte layout) and fp32 outputs through the direct epilogue (host: P.direct = 1)
+template <bool BIAS, bool RELU, bool MASK, bool CTA2, bool POOL = false, bool TF32 = false>
 __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_constant__ TcConvParams p) {
     extern __shared__ uint8_t smem_raw[];
     uint8_t *smem = smem_raw + ((1024u - (tc::smem_u32(smem_raw) & 1023u)) & 1023u);   // keeps the shared space
@@ -359,11 +357,6 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
     else __syncthreads();
     tc::tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
-    if (p.trace && threadIdx.x == 0 && blockIdx.x < 1000) {
-        unsigned long long g;
-        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g));
-        p.trace[2048 + 2 * blockIdx.x] = g;
-    }
     const int total = CTA2 ? p.total_pairs : p.tile_prefix[p.npatch];
     const int tfirst = CTA2 ? (int)tc::cluster_id_x() : (int)blockIdx.x;
     const int tstep = CTA2 ? (int)tc::nclusters_x() : (int)gridDim.x;
@@ -410,16 +403,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 const int wbase = wb * p.BW * p.s - p.pl[ql];
                 const int hbase = hb * p.BH * p.s - p.pt[ql];
                 const int n0 = nb * p.BNn, co0 = cb * p.BN;
-                if (p.dbg & 16) continue;
                 for (int ks = 0; ks < p.ksteps; ++ks) {
-                    if (p.dbg & 64) tc::mbar_wait(&empty[stage], ph ^ 1);
-                    else tc::mbar_wait_sleep(&empty[stage], ph ^ 1);
-                    if (ks == 0) TC_TRACE(it, 6);
-                    if (p.dbg & 4) {
-                        tc::mbar_arrive(&full[stage]);
-                        if (++stage == S) { stage = 0; ph ^= 1; }
-                        continue;
-                    }
+                    tc::mbar_wait(&empty[stage], ph ^ 1);
                     uint8_t *a = sA + (size_t)stage * p.a_stage;
                     uint8_t *b = sB + (size_t)stage * b_stage;
                     if (CTA2) {
@@ -482,14 +467,13 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     }
                     if (++stage == S) { stage = 0; ph ^= 1; }
                 }
-                TC_TRACE(it, 7);
             }
         }
     } else if (warp == 1) {
         {
             // ================= MMA issuer: the whole warp runs the loop converged; elect.sync issues.
             // In 2-CTA mode only the leader issues (M = 256 over the pair); the peer's warp 1 idles.
-            const uint32_t idesc = tc::idesc_bf16(CTA2 ? 256 : 128, p.BN);
+            const uint32_t idesc = tc::idesc_k<TF32>(CTA2 ? 256 : 128, p.BN);
             // halo8: per tap pair, the descriptor relative to the stage base (start address field 0)
             uint64_t h8_adesc[8], h8_bdesc[8];
             const int h8_npairs = p.halo8 ? (KT + 1) / 2 : 0;
@@ -520,22 +504,14 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             if (p.bres && leader) tc::mbar_wait(wbar, 0);
             int it = 0;
             for (int t = leader ? tfirst : total; t < total; t += tstep, ++it) {
-                if (p.dbg & 64) tc::mbar_wait(&tempty[acc], aph ^ 1);
-                else tc::mbar_wait_sleep(&tempty[acc], aph ^ 1);
-                if (lane == 0) TC_TRACE(it, 0);
+                tc::mbar_wait(&tempty[acc], aph ^ 1);
                 tc::tc_fence_after();
                 const uint32_t d = tmem_base + (uint32_t)(acc * p.BN);
                 for (int ks = 0; ks < p.ksteps; ++ks) {
-                    if (!(p.dbg & 16)) tc::mbar_wait(&full[stage], ph);
-                    if (ks == 0 && lane == 0) TC_TRACE(it, 1);
+                    tc::mbar_wait(&full[stage], ph);
                     tc::tc_fence_after();
                     const uint32_t a_base = tc::smem_u32(sA + (size_t)stage * p.a_stage);
                     const uint32_t b_base = tc::smem_u32(sB + (size_t)stage * b_stage);
-                    if (p.dbg & 2) {
-                        tc::mma_commit_ws(&empty[stage]);
-                        if (++stage == S) { stage = 0; ph ^= 1; }
-                        continue;
-                    }
                     if (p.halo8) {
                         // no-swizzle K-major A: a core matrix is 8 consecutive pixels x 16 B (8 channels);
                         // M groups (output rows) are Wp pixels apart (SBO = Wp*16 B); each MMA covers the
@@ -546,7 +522,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
 #pragma unroll
                         for (int pr = 0; pr < 8; ++pr) {
                             if (pr < h8_npairs)
-                                tc::mma_bf16_ws(d, h8_adesc[pr] + abase, h8_bdesc[pr] + bbase, idesc, (ks | pr) != 0);
+                                tc::mma_k_ws<TF32>(d, h8_adesc[pr] + abase, h8_bdesc[pr] + bbase, idesc, (ks | pr) != 0);
                         }
                         tc::mma_commit_ws(&empty[stage]);
                         if (++stage == S) { stage = 0; ph ^= 1; }
@@ -580,8 +556,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                                                    : tc::smem_desc(b_base, 16, 1024, 2);
                         const uint32_t bstep = (uint32_t)p.BN * 8u;   // BN*128 B >> 4
                         for (int c = 0; c < p.kw; ++c)
-                            tc::mma_bf16_x4_ws(d, a0 + (uint64_t)(8 * c), b0 + (uint64_t)(bstep * c), idesc, (ks | c) != 0);
-                        if (!(p.dbg & 32)) tc::mma_commit_ws(&empty[stage]);
+                            tc::mma_k_x4_ws<TF32>(d, a0 + (uint64_t)(8 * c), b0 + (uint64_t)(bstep * c), idesc, (ks | c) != 0);
+                        tc::mma_commit_ws(&empty[stage]);
                         if (++stage == S) { stage = 0; ph ^= 1; }
                         continue;
                     }
@@ -589,13 +565,12 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     const uint64_t b0 = tc::smem_desc(b_base, 16, 1024, 2);
 #pragma unroll
                     for (int j = 0; j < 4; ++j)
-                        tc::mma_bf16_ws(d, a0 + (uint64_t)g_aoff[j], b0 + (uint64_t)(2 * j), idesc, (ks | j) != 0);
+                        tc::mma_k_ws<TF32>(d, a0 + (uint64_t)g_aoff[j], b0 + (uint64_t)(2 * j), idesc, (ks | j) != 0);
                     tc::mma_commit_ws(&empty[stage]);
                     if (++stage == S) { stage = 0; ph ^= 1; }
                 }
                 if (CTA2) tc::mma2_commit_mc_ws(&tfull[acc]);
                 else tc::mma_commit_ws(&tfull[acc]);
-                if (lane == 0) TC_TRACE(it, 2);
                 acc ^= 1;
                 if (acc == 0) aph ^= 1;
             }
@@ -625,7 +600,6 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             if (POOL) {
                 // pooled outputs straight from registers: no staging tile, no store of the conv output
                 tc::mbar_wait(&tfull[g], aph);
-                if (gtid == 0) TC_TRACE(it, 3);
                 tc::tc_fence_after();
                 const uint32_t tacc = tmem_base + (uint32_t)(g * p.BN) + ((uint32_t)(quad * 32) << 16);
                 const int wi = row & (p.BW - 1), hi = (row / p.BW) % p.BH, ni = row / (p.BW * p.BH);
@@ -667,7 +641,6 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     if (CTA2) tc::mbar_arrive_remote(tempty_l);
                     else tc::mbar_arrive(&tempty[g]);
                 }
-                if (gtid == 0) TC_TRACE(it, 4);
                 aph ^= 1;
                 continue;
             }
@@ -683,11 +656,10 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 yph ^= 1;
             }
             tc::mbar_wait(&tfull[g], aph);
-            if (gtid == 0) TC_TRACE(it, 3);
             tc::tc_fence_after();
             const uint32_t tacc = tmem_base + (uint32_t)(g * p.BN) + ((uint32_t)(quad * 32) << 16);
             // fast path: whole 32-column groups of real channels inside one staging chunk (ychunk >= 32)
-            const bool fast = (ncols & 31) == 0 && co0 + ncols <= p.Cout && p.ychunk >= 32 && !(p.dbg & 8);
+            const bool fast = (ncols & 31) == 0 && co0 + ncols <= p.Cout && p.ychunk >= 32;
             if (fast) {
                 const uint32_t rbase = (uint32_t)row * rowB;
                 const uint32_t rsw = ((rbase >> 7) & p.y_mask) << 4;
@@ -706,7 +678,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     }
                 }
             }
-            for (int cc = 0; cc < ((p.dbg & 8) || fast ? 0 : ncols); cc += 32) {
+            for (int cc = 0; cc < (fast ? 0 : ncols); cc += 32) {
                 uint32_t r[2][16];
                 tc::tmem_ld16_nw(tacc + cc, r[0]);
                 if (cc + 16 < ncols) tc::tmem_ld16_nw(tacc + cc + 16, r[1]);
@@ -728,15 +700,13 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 if (CTA2) tc::mbar_arrive_remote(tempty_l);
                 else tc::mbar_arrive(&tempty[g]);
             }
-            if (gtid == 0) TC_TRACE(it, 4);
             tc::fence_proxy_async_smem();
             tc::named_bar_sync(1 + g, 128);
-            if (gtid == 0 && valid && !(p.dbg & 1)) {
+            if (gtid == 0 && valid) {
                 for (int k = 0; k < nchunks; ++k)
                     tc::tma_store_4d(&p.mapY[ql], sYb + k * chunk_bytes, co0 + k * p.ychunk, ow0, oh0, n0);
                 tc::bulk_commit();
             }
-            if (gtid == 0) TC_TRACE(it, 5);
             aph ^= 1;
         }
         if (gtid == 0) tc::bulk_wait0();
@@ -833,7 +803,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             }
             tc::fence_proxy_async_smem();
             tc::named_bar_sync(1, 256);
-            if (etid == 0 && valid && !(p.dbg & 1)) {
+            if (etid == 0 && valid) {
                 for (int k = 0; k < nchunks; ++k)
                     tc::tma_store_4d(&p.mapY[ql], sYb + k * chunk_bytes, co0 + k * p.ychunk, ow0, oh0, n0);
                 tc::bulk_commit();
@@ -872,6 +842,9 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             tc::mbar_wait(&tfull[acc], aph);
             tc::tc_fence_after();
             const uint32_t tacc = tmem_base + (uint32_t)(acc * p.BN) + ((uint32_t)(quad * 32) << 16);
+            using OT = typename std::conditional<TF32, float, __nv_bfloat16>::type;
+            OT *yo = reinterpret_cast<OT *>(p.y);
+            const OT *ro = reinterpret_cast<const OT *>(p.relu_src);
             for (int cc = 0; cc < p.BN; cc += 16) {
                 float v[16];
                 tc::tmem_ld16(tacc + cc, v);
@@ -880,10 +853,19 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 for (int g = 0; g < 2; ++g) {
                     const int co = co0 + cc + 8 * g;
                     if (co >= p.Cpo) break;
-                    float o[8];
+                    float o[8], yold[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+                    if (TF32 && p.accum) {
+                        const float *yf = reinterpret_cast<const float *>(yo) + base + co;
+                        const float4 a = *reinterpret_cast<const float4 *>(yf);
+                        yold[0] = a.x; yold[1] = a.y; yold[2] = a.z; yold[3] = a.w;
+                        if (co + 8 <= p.Cpo) {
+                            const float4 b = *reinterpret_cast<const float4 *>(yf + 4);
+                            yold[4] = b.x; yold[5] = b.y; yold[6] = b.z; yold[7] = b.w;
+                        }
+                    }
 #pragma unroll
                     for (int e = 0; e < 8; ++e) {
-                        float x = v[8 * g + e];
+                        float x = v[8 * g + e] + yold[e];
                         if (co + e < p.Cout) {
                             if (p.bias) x += __ldg(p.bias + co + e);
                             if (p.relu) x = fmaxf(x, 0.f);
@@ -892,13 +874,24 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                         }
                         o[e] = x;
                     }
-                    if (p.relu_src) {
+                    if (TF32 && co + 8 > p.Cpo) {   // fp32 levels pad channels to 4: a 4-channel tail group
+                        float *yf = reinterpret_cast<float *>(yo) + base + co;
+                        float4 r = make_float4(o[0], o[1], o[2], o[3]);
+                        if (ro) {
+                            const float4 m = *reinterpret_cast<const float4 *>(reinterpret_cast<const float *>(ro) + base + co);
+                            r.x = m.x > 0.f ? r.x : 0.f; r.y = m.y > 0.f ? r.y : 0.f;
+                            r.z = m.z > 0.f ? r.z : 0.f; r.w = m.w > 0.f ? r.w : 0.f;
+                        }
+                        *reinterpret_cast<float4 *>(yf) = r;
+                        continue;
+                    }
+                    if (ro) {
                         float m[8];
-                        load8(p.relu_src + base + co, m);
+                        load8(ro + base + co, m);
 #pragma unroll
                         for (int e = 0; e < 8; ++e) o[e] = (m[e] > 0.f) ? o[e] : 0.f;
                     }
-                    store8(p.y + base + co, o);
+                    store8(yo + base + co, o);
                 }
             }
             tc::tc_fence_before();
@@ -908,14 +901,6 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             if (acc == 0) aph ^= 1;
         }
         }
-    }
-    if (p.trace && threadIdx.x == 64 && blockIdx.x < 1000) {
-        unsigned long long g;
-        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g));
-        uint32_t smid;
-        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-        p.trace[2048 + 2 * blockIdx.x + 1] = g;
-        p.trace[3072 + blockIdx.x] = smid;
     }
     tc::tc_fence_before();
     if (CTA2) tc::cluster_sync_all();   // the peer's MMAs write this CTA's TMEM until the leader is done
@@ -928,7 +913,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
 }
 
 // dgrad weights: W'[ci][r'][c'][co] = W[co][kh-1-r'][kw-1-c'][ci], zero for co >= Cout
-__global__ void flip_weights_kernel(const __nv_bfloat16 *__restrict__ W, __nv_bfloat16 *__restrict__ Wt, int Cout,
+template <typename T>
+__global__ void flip_weights_kernel(const T *__restrict__ W, T *__restrict__ Wt, int Cout,
                                     int Cpad_in, int Cin, int kh, int kw, int Cpad_out, int r0h, int r0w, int step,
                                     int nth, int ntw) {
     // Wt[ci][j][l][co] = W[co][r0h + step*(nth-1-j)][r0w + step*(ntw-1-l)][ci]   (stride-1 dgrad: r0 = 0,
@@ -942,7 +928,7 @@ __global__ void flip_weights_kernel(const __nv_bfloat16 *__restrict__ W, __nv_bf
         const int r = (int)(t % nth);
         const int ci = (int)(t / nth);
         const int rr = r0h + step * (nth - 1 - r), cc = r0w + step * (ntw - 1 - c);
-        Wt[i] = co < Cout ? W[(((int64_t)co * kh + rr) * kw + cc) * Cpad_in + ci] : __float2bfloat16(0.f);
+        Wt[i] = co < Cout ? W[(((int64_t)co * kh + rr) * kw + cc) * Cpad_in + ci] : from_f<T>(0.f);
     }
 }
 
@@ -1070,16 +1056,22 @@ struct PoolFuse {
     const Level *Lp = nullptr;
 };
 
+// prec 0: bf16 operands and outputs; 1: TF32 -- fp32 operands through kind::tf32 (the byte layout of an fp32
+// level is that of a bf16 level with twice the channels), fp32 outputs by the direct epilogue; accum: add
+// into y (TF32 only)
 splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const LayerGeom &g, const void *a_ptr,
                             const void *w_ptr, int w_rows, const float *bias, void *y, const void *relu_src, int relu,
-                            int p0, int p1, cudaStream_t st, const PoolFuse *pool = nullptr, const Phase *ph = nullptr) {
+                            int p0, int p1, cudaStream_t st, const PoolFuse *pool = nullptr, const Phase *ph = nullptr,
+                            int prec = 0, int accum = 0) {
+    const bool tf32 = prec == 1;
+    const int es = tf32 ? 4 : 2;          // bytes per element of the operand / output levels
     auto encode = get_encode();
     if (!encode) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
     const int kh = ph ? ph->kh : g.L.kh, kw = ph ? ph->kw : g.L.kw, s = mode == 0 ? g.L.sh : 1;
     const int PS = ph ? ph->S : 1, prh = ph ? ph->rh : 0, prw = ph ? ph->rw : 0;
     auto out_ext_h = [&](int i) { return (Lout.ph(i) - prh + PS - 1) / PS; };
     auto out_ext_w = [&](int j) { return (Lout.pw(j) - prw + PS - 1) / PS; };
-    const int cpad = La.Cpad;
+    const int cpad = La.Cpad * es / 2;    // channels of the byte layout in 2-byte units
     const int cpadc = std::min(cpad, 64);
     const int ncols_out = mode == 0 ? g.L.cout : g.L.cin;
     // N tile: up to 256 output channels; small layers (few 128-pixel M tiles, e.g. 2x2 / 4x4 CIFAR tails)
@@ -1091,7 +1083,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             const int i = q / Lout.nw(), j = q % Lout.nw();
             mt += ((long)La.N * out_ext_h(i) * out_ext_w(j) + 127) / 128;
         }
-        while (BN > 64 && BN % 32 == 0 && mt * ((ncols_out + BN - 1) / BN) < num_sms() && !getenv("SPLITCNN_WIDE_N"))
+        while (BN > 64 && BN % 32 == 0 && mt * ((ncols_out + BN - 1) / BN) < num_sms())
             BN /= 2;
     }
     const int nco = (ncols_out + BN - 1) / BN;
@@ -1107,8 +1099,8 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         // halo mode for narrow outputs (per-tap TMA boxes cannot keep the MMA fed there)
         // (BN = 256 too: the A box of a kernel row then serves kw taps, -29% of the L2->SM traffic that
         // bounds these layers; same-process A/B: conv3_2 fwd 0.94 -> 0.73 ms, conv4_2 0.88 -> 0.70 ms)
-        const int halo = (s == 1 && cpad % 64 == 0 && BN <= 256 && kw >= 2 && kw <= 4 && !getenv("SPLITCNN_NO_HALO")) ? 1 : 0;
-        const int halo8 = (mode == 0 && cpad == 8 && s == 1 && kw <= 8 && kh * kw <= 16 && !getenv("SPLITCNN_NO_HALO")) ? 1 : 0;
+        const int halo = (s == 1 && cpad % 64 == 0 && BN <= 256 && kw >= 2 && kw <= 4) ? 1 : 0;
+        const int halo8 = (mode == 0 && cpad == 8 && s == 1 && kw <= 8 && kh * kw <= 16) ? 1 : 0;
         TileShape ts = pool ? choose_tile_pool(ext, N) : choose_tile(ext, N, s, a3d ? 32 : 128);
         if (halo8) {  // 8 output columns x BH output rows, one image per tile
             long best = -1;
@@ -1140,7 +1132,6 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.a3d = a3d;
         P.halo = halo;
         P.halo8 = halo8;
-        P.dbg = getenv("SPLITCNN_DBG") ? atoi(getenv("SPLITCNN_DBG")) : 0;
         P.egroups = 1;
         P.Wp = 8 + kw - 1;
         if (cpad >= 64) {
@@ -1166,7 +1157,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             const bool tma_out = (ych0 == 8 || ych0 == 16 || ych0 == 32 || ych0 == 64) && Lout.Cpad % ych0 == 0;
             long mb = 0;
             for (auto &e : ext) mb += (long)P.nnb * ((e.first + ts.BH - 1) / ts.BH) * ((e.second + ts.BW - 1) / ts.BW);
-            P.cta2 = (cpad % 64 == 0 && !halo8 && !a3d && BN % 32 == 0 && tma_out && mb >= 2 && !getenv("SPLITCNN_NO_CTA2")) ? 1 : 0;
+            P.cta2 = (!tf32 && cpad % 64 == 0 && !halo8 && !a3d && BN % 32 == 0 && tma_out && mb >= 2) ? 1 : 0;
         }
         P.BNh = P.cta2 ? BN / 2 : BN;
         if (P.cta2) P.b_tx_bytes = (uint32_t)P.BNh * 128u;
@@ -1175,7 +1166,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             P.a_tx_bytes = (uint32_t)P.Wp * (ts.BH + kh - 1) * 16u;
             P.a_stage = (P.a_tx_bytes + 1023u) & ~1023u;
             P.b_tx_bytes = (uint32_t)((kh * kw * 8 + 63) / 64) * BN * 128u;
-            if (nco == 1 && !getenv("SPLITCNN_NO_BRES")) {   // the whole filter stays in smem (one load per CTA)
+            if (nco == 1) {   // the whole filter stays in smem (one load per CTA)
                 P.bres = 1;
                 P.bres_bytes = P.b_tx_bytes;
                 P.b_tx_bytes = 0;
@@ -1188,7 +1179,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             // weights resident when they fit next to the staging tile and >= 2 A stages
             const uint32_t wbytes = (uint32_t)(cpad / 64) * kh * kw * P.BNh * 128u;
             const uint32_t stg = (uint32_t)((BN + 63) / 64) * 128u * 128u;   // one staging buffer
-            if (nco == 1 && wbytes + stg + 2u * P.a_stage <= 206u * 1024u && !getenv("SPLITCNN_NO_BRES")) {
+            if (nco == 1 && wbytes + stg + 2u * P.a_stage <= 206u * 1024u) {
                 P.bres = 1;
                 P.bres_bytes = wbytes;
                 P.b_tx_bytes = 0;
@@ -1197,14 +1188,14 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         const uint32_t stage_bytes = P.a_stage + P.b_tx_bytes;
         // output staging for the TMA-store epilogue: channel box of min(64, Cpo), swizzle to match
         const int ych = std::min(64, Lout.Cpad);
-        P.direct = !((ych == 8 || ych == 16 || ych == 32 || ych == 64) && Lout.Cpad % ych == 0);
+        P.direct = tf32 || !((ych == 8 || ych == 16 || ych == 32 || ych == 64) && Lout.Cpad % ych == 0);
         P.ychunk = ych;
         P.y_mask = ych == 64 ? 7u : ych == 32 ? 3u : ych == 16 ? 1u : 0u;
         const uint32_t ybuf = P.direct ? 0u : (uint32_t)((BN + ych - 1) / ych) * 128u * (uint32_t)ych * 2u;
         P.ybuf_bytes = (ybuf + 1023u) & ~1023u;
         P.ybufs = (!P.direct && P.ybuf_bytes <= 32u * 1024u) ? 2 : 1;
         if (P.bres && P.bres_bytes + 2u * P.ybuf_bytes + 2u * P.a_stage > 206u * 1024u) P.ybufs = 1;
-        P.egroups = (P.ybufs == 2 && !getenv("SPLITCNN_ONE_EPI")) ? 2 : 1;
+        P.egroups = (P.ybufs == 2) ? 2 : 1;
         if (ph && P.direct) return fail(SPLITCNN_ERR_UNSUPPORTED, "phase dgrad needs a TMA-store output");
         const uint32_t staging = P.ybufs * P.ybuf_bytes;
         P.stages = std::min<int>(8, (int)((210u * 1024u - staging - P.bres_bytes) / stage_bytes));
@@ -1218,6 +1209,8 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.y = (__nv_bfloat16 *)y;
         P.relu_src = (const __nv_bfloat16 *)relu_src;
         P.relu = relu;
+        P.accum = accum;
+        if (pool && tf32) return fail(SPLITCNN_ERR_UNSUPPORTED, "conv_pool_fwd: bf16 only");
         if (pool) {
             if (halo8 || P.direct || P.Cout != P.Cpo || P.Cout % 16 || (ts.BW & (ts.BW - 1)) || ts.BW > 16 || ts.BH % 2)
                 return fail(SPLITCNN_ERR_UNSUPPORTED, "conv_pool_fwd: geometry not fusable");
@@ -1243,7 +1236,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             mboxes += P.nnb * P.nhb[ql] * P.nwb[ql];
             // A map over the patch buffer: dims (C, W, H, N), TMA zero fill = patch padding
             const int hp = La.ph(i), wp = La.pw(j);
-            void *base = (char *)a_ptr + La.offset(i, j) * 2;
+            void *base = (char *)a_ptr + La.offset(i, j) * es;
             cuuint64_t dims[4] = {(cuuint64_t)cpad, (cuuint64_t)wp, (cuuint64_t)hp, (cuuint64_t)N};
             cuuint64_t strides[3] = {(cuuint64_t)cpad * 2, (cuuint64_t)wp * cpad * 2, (cuuint64_t)hp * wp * cpad * 2};
             cuuint32_t box[4] = {(cuuint32_t)cpadc, (cuuint32_t)(ts.BW * s), (cuuint32_t)(ts.BH * s), (cuuint32_t)ts.BNn};
@@ -1333,17 +1326,11 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         }
         if (tiles == 0) continue;
         const size_t smem = 1024 + (size_t)P.bar_off + 512 + (bias ? 4 * (size_t)g.L.cout : 0) + 64;
-        static unsigned long long *trace_buf = nullptr;
-        if (getenv("SPLITCNN_TRACE")) {
-            if (!trace_buf) cudaMalloc(&trace_buf, 4096 * sizeof(unsigned long long));
-            cudaMemsetAsync(trace_buf, 0, 4096 * sizeof(unsigned long long), st);
-            P.trace = trace_buf;
-        }
         const int grid = P.cta2 ? 2 * std::min(P.total_pairs, num_sms() / 2) : std::min(tiles, num_sms());
         const int mode_bits = (bias ? 4 : 0) | (relu ? 2 : 0) | (relu_src ? 1 : 0);
         auto launch = [&](auto kern) {
-            static bool set[16] = {false};
-            const int key = mode_bits + (P.cta2 ? 8 : 0);
+            static bool set[32] = {false};
+            const int key = mode_bits + (P.cta2 ? 8 : 0) + (tf32 ? 16 : 0);
             if (!set[key]) {
                 cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
                 set[key] = true;
@@ -1399,6 +1386,17 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
                 case 18: launch_pool(conv_tc_kernel<false, true, false, true, true>); break;
                 default: launch_pool(conv_tc_kernel<true, true, false, true, true>); break;
             }
+        } else if (tf32) {
+            switch (mode_bits) {
+                case 0: launch(conv_tc_kernel<false, false, false, false, false, true>); break;
+                case 1: launch(conv_tc_kernel<false, false, true, false, false, true>); break;
+                case 2: launch(conv_tc_kernel<false, true, false, false, false, true>); break;
+                case 3: launch(conv_tc_kernel<false, true, true, false, false, true>); break;
+                case 4: launch(conv_tc_kernel<true, false, false, false, false, true>); break;
+                case 5: launch(conv_tc_kernel<true, false, true, false, false, true>); break;
+                case 6: launch(conv_tc_kernel<true, true, false, false, false, true>); break;
+                default: launch(conv_tc_kernel<true, true, true, false, false, true>); break;
+            }
         } else if (P.cta2) {
             switch (mode_bits) {
                 case 0: launch(conv_tc_kernel<false, false, false, true>); break;
@@ -1427,34 +1425,6 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("conv_tc_kernel: ") + cudaGetErrorString(e));
         }
-        if (P.trace) {   // debug: per-tile event times of CTA 0 relative to its first event
-            static unsigned long long h[4096];
-            cudaStreamSynchronize(st);
-            cudaMemcpy(h, P.trace, sizeof(h), cudaMemcpyDeviceToHost);
-            {
-                unsigned long long s0 = ~0ull, e1 = 0, smax = 0, emin = ~0ull;
-                for (int b = 0; b < std::min(grid, 1000); ++b) {
-                    const unsigned long long e = h[2048 + 2 * b + 1];
-                    s0 = std::min(s0, h[2048 + 2 * b]); smax = std::max(smax, h[2048 + 2 * b]);
-                    e1 = std::max(e1, e); emin = std::min(emin, e);
-                }
-                fprintf(stderr, "trace CTA (block smid end_us):");
-                for (int b = 0; b < std::min(grid, 1000); ++b)
-                    fprintf(stderr, " %d:%d:%.0f", b, (int)h[3072 + b], (h[2048 + 2 * b + 1] - s0) / 1e3);
-                fprintf(stderr, "\n");
-                fprintf(stderr, "trace CTAs: first start 0, last start %.1f us, first end %.1f us, last end %.1f us\n",
-                        (smax - s0) / 1e3, (emin - s0) / 1e3, (e1 - s0) / 1e3);
-            }
-            unsigned long long t0 = h[6];
-            fprintf(stderr, "trace tiles=%d grid=%d ksteps=%d BN=%d cta2=%d  [tile: prod_empty prod_done | mma_tempty mma_full mma_commit | epi_tfull epi_tempty epi_store]\n",
-                    tiles, grid, P.ksteps, P.BN, P.cta2);
-            for (int i = 0; i < 256; ++i) {
-                if (i == 12) i = 230;
-                const unsigned long long *r = h + i * 8;
-                auto d = [&](int e) { return r[e] ? (long long)(r[e] - t0) : -1LL; };
-                fprintf(stderr, "  %3d: %8lld %8lld | %8lld %8lld %8lld | %8lld %8lld %8lld\n", i, d(6), d(7), d(0), d(1), d(2), d(3), d(4), d(5));
-            }
-        }
     }
     return SPLITCNN_OK;
 }
@@ -1462,6 +1432,14 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
 }  // namespace
 
 bool conv_tc_supported(int mode, splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g) {
+    if (dt == SPLITCNN_TF32 || dt == SPLITCNN_FP32) {
+        // fp32 storage on kind::tf32 (SPLITCNN_FP32: three passes hi*hi + hi*lo + lo*hi, api.cu): forward and
+        // stride-1 data gradient; the byte layout has 2 Cpad two-byte channels
+        if (g.L.sh != g.L.sw || Li.npatch() > 1024) return false;
+        if (mode == 0) return a_channels_ok(2 * Li.Cpad) && g.L.sh <= 2;
+        if (mode == 1) return a_channels_ok(2 * Lo.Cpad) && g.L.sh == 1;
+        return false;   // weight gradient: operand splitting onto the bf16 kernels (api.cu)
+    }
     if (dt != SPLITCNN_BF16) return false;
     if (g.L.sh != g.L.sw) return false;
     if (Li.npatch() > 1024) return false;
@@ -1486,15 +1464,18 @@ bool conv_tc_supported(int mode, splitcnn_dtype_t dt, const Level &Li, const Lev
     return false;
 }
 
-size_t conv_tc_ws_bytes(int mode, const Level &Li, const Level &Lo, const LayerGeom &g) {
+size_t conv_tc_ws_bytes(int mode, const Level &Li, const Level &Lo, const LayerGeom &g, splitcnn_dtype_t dt) {
     if (mode == 2) return wgrad_tc_ws_bytes(Li, Lo, g);
-    if (mode == 1) return (size_t)g.L.cin * g.L.kh * g.L.kw * Lo.Cpad * 2 + 256 + (size_t)g.L.sh * g.L.sw * 1024;
+    const size_t es = dt == SPLITCNN_BF16 ? 2 : 4;
+    if (mode == 1) return (size_t)g.L.cin * g.L.kh * g.L.kw * Lo.Cpad * es + 256 + (size_t)g.L.sh * g.L.sw * 1024;
     return 0;
 }
 
 splitcnn_status_t launch_conv_fwd_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *w,
-                                     const float *bias, void *y, int relu, int p0, int p1, cudaStream_t st) {
-    return launch_tc(0, Li, Lo, g, x, w, g.L.cout, bias, y, nullptr, relu, p0, p1, st);
+                                     const float *bias, void *y, int relu, int p0, int p1, cudaStream_t st,
+                                     splitcnn_dtype_t dt, int accum) {
+    return launch_tc(0, Li, Lo, g, x, w, g.L.cout, bias, y, nullptr, relu, p0, p1, st, nullptr, nullptr,
+                     dt == SPLITCNN_BF16 ? 0 : 1, accum);
 }
 
 splitcnn_status_t launch_conv_pool_fwd_tc(const Level &Li, const Level &Lo, const Level &Lp, const LayerGeom &g,
@@ -1504,19 +1485,29 @@ splitcnn_status_t launch_conv_pool_fwd_tc(const Level &Li, const Level &Lo, cons
     pf.y = y_pool;
     pf.a = argmax;
     pf.Lp = &Lp;
-    return launch_tc(0, Li, Lo, g, x, w, g.L.cout, bias, nullptr, nullptr, 1, p0, p1, st, &pf);
+    return launch_tc(0, Li, Lo, g, x, w, g.L.cout, bias, nullptr, nullptr, 1, p0, p1, st, &pf, nullptr, 0, 0);
+}
+
+template <typename T>
+static void flip_weights(const void *w, void *wt, const LayerGeom &g, int cpad_in, int cpad_out, int r0h, int r0w,
+                         int step, int nth, int ntw, cudaStream_t st) {
+    const int64_t n = (int64_t)g.L.cin * nth * ntw * cpad_out;
+    flip_weights_kernel<T><<<(unsigned)std::min<int64_t>((n + 255) / 256, 2048), 256, 0, st>>>(
+        (const T *)w, (T *)wt, g.L.cout, cpad_in, g.L.cin, g.L.kh, g.L.kw, cpad_out, r0h, r0w, step, nth, ntw);
+    count_launch();
 }
 
 splitcnn_status_t launch_conv_dgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy, const void *w,
-                                       void *dx, const void *relu_src, void *ws, int p0, int p1, cudaStream_t st) {
+                                       void *dx, const void *relu_src, void *ws, int p0, int p1, cudaStream_t st,
+                                       splitcnn_dtype_t dt, int accum) {
     const int S = g.L.sh, kh = g.L.kh, kw = g.L.kw;
     if (S == 1) {
-        const int64_t n = (int64_t)g.L.cin * kh * kw * Lo.Cpad;
-        flip_weights_kernel<<<(unsigned)std::min<int64_t>((n + 255) / 256, 2048), 256, 0, st>>>(
-            (const __nv_bfloat16 *)w, (__nv_bfloat16 *)ws, g.L.cout, Li.Cpad, g.L.cin, kh, kw, Lo.Cpad, 0, 0, 1, kh, kw);
-        count_launch();
-        return launch_tc(1, Lo, Li, g, dy, ws, g.L.cin, nullptr, dx, relu_src, 0, p0, p1, st);
+        if (dt == SPLITCNN_BF16) flip_weights<__nv_bfloat16>(w, ws, g, Li.Cpad, Lo.Cpad, 0, 0, 1, kh, kw, st);
+        else flip_weights<float>(w, ws, g, Li.Cpad, Lo.Cpad, 0, 0, 1, kh, kw, st);
+        return launch_tc(1, Lo, Li, g, dy, ws, g.L.cin, nullptr, dx, relu_src, 0, p0, p1, st, nullptr, nullptr,
+                         dt == SPLITCNN_BF16 ? 0 : 1, accum);
     }
+    if (dt != SPLITCNN_BF16) return fail(SPLITCNN_ERR_UNSUPPORTED, "tf32 strided data gradient");
     // stride S: S*S output phases, each a stride-1 correlation with the taps r = (rho + p_b) (mod S)
     // (every patch of a plan shares its begin pad under R2, checked in conv_tc_supported)
     const int pbh = g.pad_h[0], pbw = g.pad_w[0];
@@ -1534,10 +1525,7 @@ splitcnn_status_t launch_conv_dgrad_tc(const Level &Li, const Level &Lo, const L
             }
             const int ch = (rh + pbh - r0h) / S, cw = (rw + pbw - r0w) / S;
             const int64_t n = (int64_t)g.L.cin * nth * ntw * Lo.Cpad;
-            flip_weights_kernel<<<(unsigned)std::min<int64_t>((n + 255) / 256, 2048), 256, 0, st>>>(
-                (const __nv_bfloat16 *)w, (__nv_bfloat16 *)wsp, g.L.cout, Li.Cpad, g.L.cin, kh, kw, Lo.Cpad, r0h, r0w, S,
-                nth, ntw);
-            count_launch();
+            flip_weights<__nv_bfloat16>(w, wsp, g, Li.Cpad, Lo.Cpad, r0h, r0w, S, nth, ntw, st);
             Phase ph{S, rh, rw, nth, ntw, nth - 1 - ch, ntw - 1 - cw};
             const splitcnn_status_t r = launch_tc(1, Lo, Li, g, dy, wsp, g.L.cin, nullptr, dx, relu_src, 0, p0, p1, st,
                                                   nullptr, &ph);
@@ -2107,8 +2095,7 @@ WgradCfg wgrad_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, int p0,
     int Z = std::max(1, (2 * num_sms() + c.ntiles - 1) / c.ntiles);
     Z = std::min(Z, std::max(1, c.total_boxes / 4));  // >= 4 boxes per split
     Z = std::min(Z, 128);
-    if (!getenv("SPLITCNN_ZMAX"))
-        Z = choose_splits(c.total_boxes, c.ntiles, 2.0 * 128 * c.bpt_pad * c.cbox * c.ts.BW * c.ts.BH * c.ts.BNn,
+    Z = choose_splits(c.total_boxes, c.ntiles, 2.0 * 128 * c.bpt_pad * c.cbox * c.ts.BW * c.ts.BH * c.ts.BNn,
                           (double)g.L.cout * KT * Li.Cpad, Z);
     c.boxes_per_split = (c.total_boxes + Z - 1) / Z;
     c.nsplit = (c.total_boxes + c.boxes_per_split - 1) / c.boxes_per_split;
@@ -2149,8 +2136,7 @@ WgHaloCfg wgrad_halo_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, i
     int Z = std::max(1, (2 * num_sms() + c.ntiles - 1) / c.ntiles);
     Z = std::min(Z, std::max(1, c.total_boxes / 4));
     Z = std::min(Z, 128);
-    if (!getenv("SPLITCNN_ZMAX"))
-        Z = choose_splits(c.total_boxes, c.ntiles, 2.0 * 128 * g.L.kw * 64 * c.BH * c.BNn * 8,
+    Z = choose_splits(c.total_boxes, c.ntiles, 2.0 * 128 * g.L.kw * 64 * c.BH * c.BNn * 8,
                           (double)g.L.cout * g.L.kh * g.L.kw * Li.Cpad, Z);
     c.boxes_per_split = (c.total_boxes + Z - 1) / Z;
     c.nsplit = (c.total_boxes + c.boxes_per_split - 1) / c.boxes_per_split;
@@ -2196,7 +2182,7 @@ static bool wgrad_tc_ok(const Level &Li, const Level &Lo, const LayerGeom &g) {
 
 // which weight-gradient kernel takes a layer: 2 narrow (8-channel input), 1 halo, 0 generic
 static int wgrad_path(const Level &Li, const Level &Lo, const LayerGeom &g) {
-    if (wgrad_narrow_ok(Li, Lo, g) && !getenv("SPLITCNN_NO_NARROW_WGRAD")) return 2;
+    if (wgrad_narrow_ok(Li, Lo, g)) return 2;
     if (wgrad_halo_ok(Li, Lo, g)) return 1;
     return 0;
 }
@@ -2365,7 +2351,7 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
             P.boxes_per_split = c.boxes_per_split; P.nsplit = c.nsplit;
             P.Cout = g.L.cout; P.Cpi = Li.Cpad;
             // 2-CTA pairs of 128-channel output blocks when the channels pair up
-            const bool cta2 = g.L.cout % 256 == 0 && !getenv("SPLITCNN_NO_CTA2");
+            const bool cta2 = g.L.cout % 256 == 0;
             if (cta2) P.ntiles = c.ntiles / 2;
             const int Wp = 8 + g.L.kw - 1;
             const uint32_t a_stage = (g.L.cout <= 64 ? 1u : 2u) * c.BH * c.BNn * 8u * 128u;
@@ -2540,6 +2526,152 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
         cudaStreamWaitEvent(st, ss->join, 0);     // join: db is complete in the caller's stream order
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("db column sums: ") + cudaGetErrorString(e));
+    }
+    return SPLITCNN_OK;
+}
+
+
+// ============================================================ fp32 storage on the tensor cores
+// SPLITCNN_TF32: one kind::tf32 pass (operands truncated to TF32 by the MMA, fp32 accumulate).
+// SPLITCNN_FP32 (fp32-accurate): 3xTF32 -- each operand v = hi + lo with hi = v with the low 13 mantissa
+// bits cleared (exactly a TF32 value) and lo = v - hi (exact in fp32); y = lo*W_hi + hi*W_lo + hi*W_hi
+// as three kind::tf32 passes accumulated in fp32 by the direct epilogue (small terms first; bias, ReLU
+// and the dgrad mask after the last pass).  The dropped lo*lo term and lo's own TF32 truncation are
+// ~2^-22 of the product.
+// Weight gradients: bf16 operand splitting on the bf16 wgrad kernels -- v = v1 + v2 (+ v3), v_k bf16
+// (v1 = bf16(v), v2 = bf16(v - v1), v3 = bf16(v - v1 - v2)); every bf16 x bf16 product is exact in fp32,
+// and the pair products summed are those of i + j <= 1 (TF32, 3 products, ~2^-16 of each product) or
+// i + j <= 2 (FP32, 6 products, ~2^-24).  db = sum of dY in fp32.
+
+__global__ void tf32_hilo_kernel(const float4 *__restrict__ x, float4 *__restrict__ hi, float4 *__restrict__ lo, int64_t n4) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n4; i += (int64_t)gridDim.x * blockDim.x) {
+        const float4 v = x[i];
+        float4 h;
+        h.x = __uint_as_float(__float_as_uint(v.x) & 0xFFFFE000u);
+        h.y = __uint_as_float(__float_as_uint(v.y) & 0xFFFFE000u);
+        h.z = __uint_as_float(__float_as_uint(v.z) & 0xFFFFE000u);
+        h.w = __uint_as_float(__float_as_uint(v.w) & 0xFFFFE000u);
+        hi[i] = h;
+        lo[i] = make_float4(v.x - h.x, v.y - h.y, v.z - h.z, v.w - h.w);
+    }
+}
+
+__global__ void bf16_terms_kernel(const float4 *__restrict__ x, __nv_bfloat16 *__restrict__ t, int64_t n4, int64_t stride,
+                                  int nterms) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n4; i += (int64_t)gridDim.x * blockDim.x) {
+        float r[4];
+        const float4 v = x[i];
+        r[0] = v.x; r[1] = v.y; r[2] = v.z; r[3] = v.w;
+        for (int k = 0; k < nterms; ++k) {
+            __nv_bfloat16 b[4];
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+                b[e] = __float2bfloat16_rn(r[e]);
+                r[e] -= __bfloat162float(b[e]);      // exact: the bf16 value is the leading part of r
+            }
+            *reinterpret_cast<uint2 *>(t + k * stride + 4 * i) = *reinterpret_cast<const uint2 *>(b);
+        }
+    }
+}
+
+static size_t al256(size_t b) { return (b + 255) & ~(size_t)255; }
+#define F32TC_TRY(x)                              \
+    do {                                          \
+        const splitcnn_status_t r_ = (x);         \
+        if (r_ != SPLITCNN_OK) return r_;         \
+    } while (0)
+
+static void hilo(const float *x, float *hi, float *lo, int64_t n, cudaStream_t st) {
+    if (n <= 0) return;
+    const int64_t n4 = n / 4;       // levels and weights hold multiples of 8 elements
+    tf32_hilo_kernel<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((n4 + 255) / 256, 148 * 16)), 256, 0, st>>>(
+        (const float4 *)x, (float4 *)hi, (float4 *)lo, n4);
+    count_launch();
+}
+
+static void bf16_terms(const float *x, __nv_bfloat16 *t, int64_t n, int64_t stride, int nterms, cudaStream_t st) {
+    if (n <= 0) return;
+    const int64_t n4 = n / 4;
+    bf16_terms_kernel<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((n4 + 255) / 256, 148 * 16)), 256, 0, st>>>(
+        (const float4 *)x, t, n4, stride, nterms);
+    count_launch();
+}
+
+static int64_t lvl_off(const Level &L, int q) { return q >= L.npatch() ? L.total() : L.offset(q / L.nw(), q % L.nw()); }
+
+size_t f32tc_ws_bytes(int op, splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g) {
+    const size_t wf = (size_t)g.L.cout * g.L.kh * g.L.kw * Li.Cpad * 4;              // forward weights, fp32
+    const size_t wb = (size_t)g.L.cin * g.L.kh * g.L.kw * Lo.Cpad * 4;               // flipped (dgrad) weights
+    if (op == 0) return dt == SPLITCNN_FP32 ? 2 * al256((size_t)Li.total() * 4) + 2 * al256(wf) : 0;
+    if (op == 1) {
+        const size_t flip = al256(conv_tc_ws_bytes(1, Li, Lo, g, dt));
+        return dt == SPLITCNN_FP32 ? flip + 2 * al256((size_t)Lo.total() * 4) + 2 * al256(wb) : flip;
+    }
+    const int nt = dt == SPLITCNN_TF32 ? 2 : 3;
+    return nt * al256((size_t)Li.total() * 2) + nt * al256((size_t)Lo.total() * 2) + al256(wgrad_tc_ws_bytes(Li, Lo, g)) +
+           al256((size_t)9 * 4 * 148 * g.L.cout * sizeof(float));
+}
+
+splitcnn_status_t launch_conv_fwd_f32tc(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g,
+                                        const void *x, const void *w, const float *bias, void *y, int relu, int p0, int p1,
+                                        void *ws, cudaStream_t st) {
+    if (dt == SPLITCNN_TF32) return launch_conv_fwd_tc(Li, Lo, g, x, w, bias, y, relu, p0, p1, st, SPLITCNN_TF32, 0);
+    const int64_t nw = (int64_t)g.L.cout * g.L.kh * g.L.kw * Li.Cpad;
+    char *p = (char *)ws;
+    float *xhi = (float *)p; p += al256((size_t)Li.total() * 4);
+    float *xlo = (float *)p; p += al256((size_t)Li.total() * 4);
+    float *whi = (float *)p; p += al256((size_t)nw * 4);
+    float *wlo = (float *)p;
+    const int64_t o0 = lvl_off(Li, p0), o1 = lvl_off(Li, p1);
+    hilo((const float *)x + o0, xhi + o0, xlo + o0, o1 - o0, st);
+    hilo((const float *)w, whi, wlo, nw, st);
+    F32TC_TRY(launch_conv_fwd_tc(Li, Lo, g, xlo, whi, nullptr, y, 0, p0, p1, st, SPLITCNN_TF32, 0));
+    F32TC_TRY(launch_conv_fwd_tc(Li, Lo, g, xhi, wlo, nullptr, y, 0, p0, p1, st, SPLITCNN_TF32, 1));
+    return launch_conv_fwd_tc(Li, Lo, g, xhi, whi, bias, y, relu, p0, p1, st, SPLITCNN_TF32, 1);
+}
+
+splitcnn_status_t launch_conv_dgrad_f32tc(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g,
+                                          const void *dy, const void *w, void *dx, const void *relu_src, int p0, int p1,
+                                          void *ws, cudaStream_t st) {
+    if (dt == SPLITCNN_TF32) return launch_conv_dgrad_tc(Li, Lo, g, dy, w, dx, relu_src, ws, p0, p1, st, SPLITCNN_TF32, 0);
+    const int kh = g.L.kh, kw = g.L.kw;
+    const int64_t nw = (int64_t)g.L.cin * kh * kw * Lo.Cpad;
+    char *p = (char *)ws;
+    float *wt = (float *)p; p += al256(conv_tc_ws_bytes(1, Li, Lo, g, dt));
+    float *ghi = (float *)p; p += al256((size_t)Lo.total() * 4);
+    float *glo = (float *)p; p += al256((size_t)Lo.total() * 4);
+    float *whi = (float *)p; p += al256((size_t)nw * 4);
+    float *wlo = (float *)p;
+    flip_weights<float>(w, wt, g, Li.Cpad, Lo.Cpad, 0, 0, 1, kh, kw, st);
+    const int64_t o0 = lvl_off(Lo, p0), o1 = lvl_off(Lo, p1);
+    hilo((const float *)dy + o0, ghi + o0, glo + o0, o1 - o0, st);
+    hilo(wt, whi, wlo, nw, st);
+    F32TC_TRY(launch_tc(1, Lo, Li, g, glo, whi, g.L.cin, nullptr, dx, nullptr, 0, p0, p1, st, nullptr, nullptr, 1, 0));
+    F32TC_TRY(launch_tc(1, Lo, Li, g, ghi, wlo, g.L.cin, nullptr, dx, nullptr, 0, p0, p1, st, nullptr, nullptr, 1, 1));
+    return launch_tc(1, Lo, Li, g, ghi, whi, g.L.cin, nullptr, dx, relu_src, 0, p0, p1, st, nullptr, nullptr, 1, 1);
+}
+
+splitcnn_status_t launch_conv_wgrad_f32tc(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g,
+                                          const void *x, const void *dy, float *dw, float *db, float beta, void *ws,
+                                          int p0, int p1, cudaStream_t st) {
+    const int nt = dt == SPLITCNN_TF32 ? 2 : 3;
+    char *p = (char *)ws;
+    const int64_t sx = (int64_t)(al256((size_t)Li.total() * 2) / 2), sg = (int64_t)(al256((size_t)Lo.total() * 2) / 2);
+    __nv_bfloat16 *xt = (__nv_bfloat16 *)p; p += nt * sx * 2;
+    __nv_bfloat16 *gt = (__nv_bfloat16 *)p; p += nt * sg * 2;
+    void *wgws = p; p += al256(wgrad_tc_ws_bytes(Li, Lo, g));
+    float *partdb = (float *)p;
+    const int64_t xo0 = lvl_off(Li, p0), xo1 = lvl_off(Li, p1), go0 = lvl_off(Lo, p0), go1 = lvl_off(Lo, p1);
+    bf16_terms((const float *)x + xo0, xt + xo0, xo1 - xo0, sx, nt, st);
+    bf16_terms((const float *)dy + go0, gt + go0, go1 - go0, sg, nt, st);
+    static const int prs[6][2] = {{0, 0}, {0, 1}, {1, 0}, {0, 2}, {1, 1}, {2, 0}};
+    const int npr = nt == 2 ? 3 : 6;
+    for (int k = 0; k < npr; ++k)
+        F32TC_TRY(launch_conv_wgrad_tc(Li, Lo, g, xt + prs[k][0] * sx, gt + prs[k][1] * sg, dw, nullptr, k == 0 ? beta : 1.f,
+                                 wgws, p0, p1, st));
+    if (db) {
+        const int Zd = launch_db_partials(SPLITCNN_FP32, Lo, dy, partdb, g.L.cout, p0, p1, st);
+        launch_reduce(partdb, Zd, g.L.cout, db, beta, st);
     }
     return SPLITCNN_OK;
 }

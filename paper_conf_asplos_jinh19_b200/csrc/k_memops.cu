@@ -545,14 +545,12 @@ void launch_pool_fwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, con
                        int relu_bit, int p0, int p1, cudaStream_t st) {
     npatch_launch = p1 - p0;
     dim3 grid(grid_x_for(max_patch_units(Lo, p0, p1, Lo.Cpad / 8)), p1 - p0);
-    bool exact = std::is_same<T, __nv_bfloat16>::value && g.L.kh == 2 && g.L.kw == 2 && g.L.sh == 2 && g.L.sw == 2 &&
-                 !getenv("SPLITCNN_POOL_GENERIC");
+    bool exact = std::is_same<T, __nv_bfloat16>::value && g.L.kh == 2 && g.L.kw == 2 && g.L.sh == 2 && g.L.sw == 2;
     for (size_t i = 0; exact && i < g.pad_h.size(); ++i) exact = g.pad_h[i] == 0;
     for (size_t i = 0; exact && i < g.pad_w.size(); ++i) exact = g.pad_w[i] == 0;
     for (int i = 0; exact && i < Li.nh(); ++i) exact = Li.ph(i) == 2 * Lo.ph(i);
     for (int j = 0; exact && j < Li.nw(); ++j) exact = Li.pw(j) == 2 * Lo.pw(j);
-    if (std::is_same<T, __nv_bfloat16>::value && g.L.kh == 3 && g.L.kw == 3 && g.L.sh == 2 && g.L.sw == 2 &&
-        !getenv("SPLITCNN_POOL_GENERIC")) {
+    if (std::is_same<T, __nv_bfloat16>::value && g.L.kh == 3 && g.L.kw == 3 && g.L.sh == 2 && g.L.sw == 2) {
         pool3x3s2_fwd_bf16_kernel<<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
                                                         (const __nv_bfloat16 *)x, (__nv_bfloat16 *)y, a, p0, relu_bit);
         count_launch();
@@ -575,7 +573,7 @@ void launch_pool_bwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, con
     for (size_t i = 0; exact && i < g.pad_w.size(); ++i) exact = g.pad_w[i] == 0;
     for (int i = 0; exact && i < Li.nh(); ++i) exact = Li.ph(i) == Lo.ph(i) * g.L.sh;
     for (int j = 0; exact && j < Li.nw(); ++j) exact = Li.pw(j) == Lo.pw(j) * g.L.sw;
-    if (exact && std::is_same<T, __nv_bfloat16>::value && g.L.kh == 2 && g.L.kw == 2 && !getenv("SPLITCNN_POOL_GENERIC")) {
+    if (exact && std::is_same<T, __nv_bfloat16>::value && g.L.kh == 2 && g.L.kw == 2) {
         npatch_launch = p1 - p0;
         dim3 grid(grid_x_for(max_patch_units(Lo, p0, p1, Lo.Cpad / 8)), p1 - p0);
         pool2x2_bwd_bf16_kernel<<<grid, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), (const __nv_bfloat16 *)dy,
@@ -593,7 +591,7 @@ void launch_pool_bwd_t(const Level &Li, const Level &Lo, const LayerGeom &g, con
     }
     npatch_launch = p1 - p0;
     dim3 grid(grid_x_for(max_patch_units(Li, p0, p1, Li.Cpad / 8)), p1 - p0);
-    if (g.L.kh == 3 && g.L.kw == 3 && g.L.sh == 2 && g.L.sw == 2 && !getenv("SPLITCNN_POOL_GATHER")) {
+    if (g.L.kh == 3 && g.L.kw == 3 && g.L.sh == 2 && g.L.sw == 2) {
         dim3 g4((unsigned)std::max(1, (int)grid.x / 4 + 1), p1 - p0);
         pool_bwd_k3s2_kernel<T><<<g4, 256, 0, st>>>(make_level_desc(Li), make_level_desc(Lo), make_layer_desc(g),
                                                     (const T *)dy, a, (T *)dx, p0, relu_bit);

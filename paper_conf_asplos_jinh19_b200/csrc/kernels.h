@@ -40,15 +40,28 @@ size_t wgrad_simt_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g)
 
 // k_conv_tc.cu (tcgen05); return false when the shape is not supported by the tensor-core path
 bool conv_tc_supported(int mode, splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g);
-size_t conv_tc_ws_bytes(int mode, const Level &Li, const Level &Lo, const LayerGeom &g);
+size_t conv_tc_ws_bytes(int mode, const Level &Li, const Level &Lo, const LayerGeom &g, splitcnn_dtype_t dt = SPLITCNN_BF16);
 splitcnn_status_t launch_conv_fwd_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *w,
-                                     const float *bias, void *y, int relu, int p0, int p1, cudaStream_t st);
+                                     const float *bias, void *y, int relu, int p0, int p1, cudaStream_t st,
+                                     splitcnn_dtype_t dt = SPLITCNN_BF16, int accum = 0);
 splitcnn_status_t launch_conv_pool_fwd_tc(const Level &Li, const Level &Lo, const Level &Lp, const LayerGeom &g,
                                           const void *x, const void *w, const float *bias, void *y_pool, uint8_t *argmax,
                                           int p0, int p1, cudaStream_t st);
 splitcnn_status_t launch_conv_dgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy, const void *w,
-                                       void *dx, const void *relu_src, void *ws, int p0, int p1, cudaStream_t st);
+                                       void *dx, const void *relu_src, void *ws, int p0, int p1, cudaStream_t st,
+                                       splitcnn_dtype_t dt = SPLITCNN_BF16, int accum = 0);
 splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *dy,
                                        float *dw, float *db, float beta, void *ws, int p0, int p1, cudaStream_t st);
+// fp32 storage on the tensor cores (TF32 one pass / FP32 3xTF32; wgrad by bf16 operand splitting)
+size_t f32tc_ws_bytes(int op, splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g);
+splitcnn_status_t launch_conv_fwd_f32tc(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g,
+                                        const void *x, const void *w, const float *bias, void *y, int relu, int p0, int p1,
+                                        void *ws, cudaStream_t st);
+splitcnn_status_t launch_conv_dgrad_f32tc(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g,
+                                          const void *dy, const void *w, void *dx, const void *relu_src, int p0, int p1,
+                                          void *ws, cudaStream_t st);
+splitcnn_status_t launch_conv_wgrad_f32tc(splitcnn_dtype_t dt, const Level &Li, const Level &Lo, const LayerGeom &g,
+                                          const void *x, const void *dy, float *dw, float *db, float beta, void *ws,
+                                          int p0, int p1, cudaStream_t st);
 
 }  // namespace splitcnn

@@ -182,6 +182,20 @@ __device__ __forceinline__ void mma_commit_ws(uint64_t *bar) {
         "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(smem_u32(bar))
         : "memory");
 }
+// kind::f16 (bf16) or kind::tf32 MMAs with the same operand descriptors (32 bytes of K per MMA)
+template <bool TF32>
+__device__ __forceinline__ void mma_k_ws(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc, uint32_t accum) {
+    if constexpr (TF32)
+        asm volatile(
+            "{\n\t.reg .pred p, e;\n\t"
+            "setp.ne.b32 p, %4, 0;\n\t"
+            "elect.sync _|e, 0xffffffff;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+            "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accum)
+            : "memory");
+    else
+        mma_bf16_ws(d_tmem, adesc, bdesc, idesc, accum);
+}
 // 2-CTA (M = 256) MMA, issued by the leader CTA of the pair, converged warp + elect.sync
 __device__ __forceinline__ void mma2_bf16_ws(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc, uint32_t accum) {
     asm volatile(
@@ -208,6 +222,24 @@ __device__ __forceinline__ void mma_bf16_x4_ws(uint32_t d_tmem, uint64_t adesc, 
         "@e tcgen05.mma.cta_group::1.kind::f16 [%0], a3, b3, %3, 1;\n\t}" ::"r"(d_tmem),
         "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accum)
         : "memory");
+}
+template <bool TF32>
+__device__ __forceinline__ void mma_k_x4_ws(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc, uint32_t accum) {
+    if constexpr (TF32)
+        asm volatile(
+            "{\n\t.reg .pred p, e;\n\t.reg .b64 a1, a2, a3, b1, b2, b3;\n\t"
+            "setp.ne.b32 p, %4, 0;\n\t"
+            "add.s64 a1, %1, 2;\n\tadd.s64 a2, %1, 4;\n\tadd.s64 a3, %1, 6;\n\t"
+            "add.s64 b1, %2, 2;\n\tadd.s64 b2, %2, 4;\n\tadd.s64 b3, %2, 6;\n\t"
+            "elect.sync _|e, 0xffffffff;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::tf32 [%0], a1, b1, %3, 1;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::tf32 [%0], a2, b2, %3, 1;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::tf32 [%0], a3, b3, %3, 1;\n\t}" ::"r"(d_tmem),
+            "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accum)
+            : "memory");
+    else
+        mma_bf16_x4_ws(d_tmem, adesc, bdesc, idesc, accum);
 }
 __device__ __forceinline__ void mma2_bf16_x4_ws(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc, uint32_t accum) {
     asm volatile(
@@ -291,6 +323,19 @@ __host__ __device__ constexpr uint32_t idesc_bf16(int M, int N, int a_mn = 0, in
     return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)a_mn << 15) | ((uint32_t)b_mn << 16) |
            ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
 }
+
+// Instruction descriptor, kind::tf32: D fp32, A/B tf32 (fp32 storage, the MMA reads the top 19 bits),
+// A/B major, N>>3, M>>4.  A K = 8 slice is 32 bytes -- the same bytes as a bf16 K = 16 slice, so smem
+// tiles / descriptors of the bf16 kernels carry tf32 operands unchanged (2 bf16 "channels" per fp32).
+__host__ __device__ constexpr uint32_t idesc_tf32(int M, int N, int a_mn = 0, int b_mn = 0) {
+    return (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)a_mn << 15) | ((uint32_t)b_mn << 16) |
+           ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+template <bool TF32>
+__host__ __device__ constexpr uint32_t idesc_k(int M, int N, int a_mn = 0, int b_mn = 0) {
+    return TF32 ? idesc_tf32(M, N, a_mn, b_mn) : idesc_bf16(M, N, a_mn, b_mn);
+}
+
 
 }  // namespace tc
 }  // namespace splitcnn

@@ -13,7 +13,7 @@ import torch
 from . import splitcnn as sc
 from .plan import SplitPlan
 
-TORCH_DTYPE = {sc.BF16: torch.bfloat16, sc.FP32: torch.float32}
+TORCH_DTYPE = {sc.BF16: torch.bfloat16, sc.FP32: torch.float32, sc.TF32: torch.float32}
 
 
 def pack_weight(W_oihw: torch.Tensor, cpad_in: int, dtype) -> torch.Tensor:
@@ -141,7 +141,8 @@ class SplitNet:
                 continue
             for m, l in enumerate(plan.layers):
                 if l["op"] == "conv":
-                    ws = max(ws, plan.workspace_size(m, self.dtype, 1), plan.workspace_size(m, self.dtype, 2))
+                    ws = max(ws, plan.workspace_size(m, self.dtype, 0), plan.workspace_size(m, self.dtype, 1),
+                             plan.workspace_size(m, self.dtype, 2))
         self.ws = torch.zeros(max(ws, 16) // 4 + 4, dtype=torch.float32, device=dev)
         self.ws_bytes = self.ws.numel() * 4
         self.params = {}
@@ -380,8 +381,8 @@ class SplitNet:
             if l["op"] == "conv":
                 W, b = self.params[(key, m)]
                 flags = (sc.FLAG_RELU if l.get("relu", True) else 0) | self.flags_extra
-                self._call("conv_fwd", self._conv_work(plan, m, l), sc.splitcnn_conv_fwd, plan.handle, m, self.dtype,
-                           acts[m], W, b, acts[m + 1], flags, p0, p1, stream)
+                self._call("conv_fwd", self._conv_work(plan, m, l), sc.splitcnn_conv_fwd_ws, plan.handle, m, self.dtype,
+                           acts[m], W, b, acts[m + 1], flags, self.ws, self.ws_bytes, p0, p1, stream)
             else:
                 flags = sc.FLAG_POOL_RELU_MASK if self._masked(key, m) else 0
                 bi, bo = self._bytes(plan, m)

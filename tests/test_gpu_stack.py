@@ -21,7 +21,7 @@ def sc():
     return splitcnn
 
 
-def _run(sc, cfg_name, N, dtype, H=None, step=0, force_simt=False, exact=False, seed=None):
+def _run(sc, cfg_name, N, dtype, H=None, step=0, force_simt=False, exact=False, seed=None, taps=3):
     """exact=True draws synth.dyadic inputs / sparse integer weights (every fwd / dgrad sum exact in
     fp32 and fp64), so the bf16 levels, masks and argmaxes agree and the whole backward is comparable."""
     from paper_conf_asplos_jinh19_b200.net import SplitNet
@@ -33,7 +33,7 @@ def _run(sc, cfg_name, N, dtype, H=None, step=0, force_simt=False, exact=False, 
     bf = dtype == sc.BF16
     if exact:
         X = synth.dyadic(g, (N, 3, H, H))
-        params = synth.exact_layer_params(g, c["layers"] + c["tail"])
+        params = synth.exact_layer_params(g, c["layers"] + c["tail"], taps=taps)
     else:
         X = synth.uniform(g, (N, 3, H, H))
         params = synth.layer_params(g, c["layers"] + c["tail"])
@@ -94,7 +94,7 @@ def _run(sc, cfg_name, N, dtype, H=None, step=0, force_simt=False, exact=False, 
                     # max (values next to the ReLU kink round to 0 on one side and to a tiny positive
                     # value on the other)
                     tie = abs(v1 - v2) <= 2 ** -6 * max(abs(v1), abs(v2)) + 2 ** -8 * scale
-                    assert bf and tie, (key, m, v1, v2, scale)
+                    assert (bf or dtype == sc.TF32) and tie, (key, m, v1, v2, scale)
     errs["argmax_flip_frac"] = flips / max(total, 1)
     return errs
 
@@ -129,6 +129,18 @@ def test_stack_bf16_whole_backward(sc, cfg, N, H, seed):
     assert errs["out"] == 0.0, errs
     assert errs["argmax_flip_frac"] == 0.0, errs
     assert max(errs.values()) <= 2e-2, errs
+
+
+def test_c2_stack_tf32(sc):
+    """TF32 (kind::tf32 forward / data gradient, bf16-split weight gradient) through the whole C2 stack.
+    Kaiming draws: the output within the TF32 bar 2e-3 (R13).  Dyadic draws with one +-1/+-2 tap per
+    output channel keep every level an integer multiple of 1/4 below 2^11 units -- exact in TF32 -- so
+    forward and backward agree with the oracle exactly up to fp32 summation order (every dW / db <= 2e-3)."""
+    errs = _run(sc, "C2", 2, sc.TF32)
+    assert errs["out"] <= 2e-3 and errs["argmax_flip_frac"] < 1e-2, errs
+    errs = _run(sc, "C2", 2, sc.TF32, exact=True, seed=105, taps=1)
+    assert errs["out"] == 0.0 and errs["argmax_flip_frac"] == 0.0, errs
+    assert max(errs.values()) <= 2e-3, errs
 
 
 def test_c4_stochastic_stack_small(sc):

@@ -99,6 +99,12 @@ def make_inputs(c, dtype_t, device, world=1, rank=0):
 
 
 # --------------------------------------------------------------------------- ours
+def _nets(net):
+    """The SplitNet executors inside an executor (the dist executor holds a region and a tail net)."""
+    return [n for n in (getattr(net, "region_net", None), getattr(net, "tail_net", None), getattr(net, "net_r", None),
+                        getattr(net, "net_t", None)) if n is not None] or [net]
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
@@ -253,11 +259,18 @@ def run_ours(args):
     clk = clocks.stop()
     launches = (launches_per_step * args.steps) if graph else sc.splitcnn_kernel_launches() - launches0
     ms = sum(a.elapsed_time(b) for a, b in evs) if flush_l2 else t0.elapsed_time(t1)
-    # per-kind breakdown (roofline) from an eager pass with CUDA events around every library call
+    # per-kind breakdown (roofline) from an eager pass with CUDA events around every library call; the
+    # weight gradients run on the main stream here, so every kernel is timed alone (not while it shares the
+    # GPU with its layer's concurrent data gradient)
+    conc = [(n, n.concurrent_wgrad) for n in _nets(net)]
+    for n, _ in conc:
+        n.concurrent_wgrad = False
     net.timers = []
     for _ in range(args.steps):
         net.step(x, dy)
     barrier()
+    for n, v in conc:
+        n.concurrent_wgrad = v
     if world > 1:
         tt = torch.tensor([ms], device="cuda")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)

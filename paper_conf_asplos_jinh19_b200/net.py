@@ -34,7 +34,8 @@ class SplitNet:
                  split=(2, 2), mode: str = "even", omega: float = 0.2, seed: int = 0,
                  dtype: int = sc.BF16, device="cuda", patch_range=None, force_simt: bool = False,
                  grad_buffer: torch.Tensor | None = None, input_relu: bool = False, fuse_pool: bool = True,
-                 static_pool: bool = False, input_grad: bool = False, mask_output_grad: bool = True):
+                 static_pool: bool = False, input_grad: bool = False, mask_output_grad: bool = True,
+                 concurrent_wgrad: bool = True):
         self.region_layers, self.tail_layers = region, tail
         self.N, self.C, self.H, self.W = N, C, H, W
         self.split, self.mode, self.omega, self.seed = split, mode, omega, seed
@@ -48,6 +49,9 @@ class SplitNet:
         # dY is the gradient of the stack output; False when the caller already applied the output's ReLU
         # mask (a region whose gradient comes back from a tail that masks its input, dist.py)
         self.mask_output_grad = mask_output_grad
+        # a layer's weight gradient and its data gradient both read only dY: the weight gradient runs on a
+        # side stream (its own workspace) concurrently with the data gradient, joined before the next layer
+        self.concurrent_wgrad = concurrent_wgrad
         self.timers = None       # list -> every library call is bracketed by CUDA events (bench.py)
         self.wgrad_hook = None   # callable(key, m) after each layer's weight-gradient call is enqueued
         self._label = ""
@@ -145,6 +149,8 @@ class SplitNet:
                              plan.workspace_size(m, self.dtype, 2))
         self.ws = torch.zeros(max(ws, 16) // 4 + 4, dtype=torch.float32, device=dev)
         self.ws_bytes = self.ws.numel() * 4
+        self.ws_w = torch.zeros_like(self.ws) if self.concurrent_wgrad else self.ws     # the side stream's
+        self.side = None          # created on first use (a meta-device executor only plans)
         self.params = {}
         for key, layers, plan in (("r", self.region_layers, self.region), ("t", self.tail_layers, self.tail)):
             for m, l in enumerate(layers):
@@ -423,14 +429,33 @@ class SplitNet:
                 W, _ = self.params[(key, m)]
                 dW, db = self.grads[(key, m)]
                 work = self._conv_work(plan, m, l)
+                fork = self.concurrent_wgrad and not last
+                main = stream if stream is not None else torch.cuda.current_stream(self.device)
+                if fork and self.side is None:
+                    self.side = torch.cuda.Stream(self.device)
+                    self.fork_ev = [torch.cuda.Event() for _ in range(64)]
+                    self.join_ev = [torch.cuda.Event() for _ in range(64)]
+                if fork:      # the weight gradient on the side stream, after dY (= g) is ready
+                    ev = self.fork_ev[m % 64]
+                    ev.record(main)
+                    self.side.wait_event(ev)
+                    with torch.cuda.stream(self.side):
+                        self._call("conv_wgrad", work, sc.splitcnn_conv_bwd_filter, plan.handle, m, self.dtype, acts[m],
+                                   g, dW, db, 0.0, self.ws_w, self.ws_bytes, self.flags_extra, p0, p1, self.side)
+                        if self.wgrad_hook is not None:
+                            self.wgrad_hook(key, m)
+                        self.join_ev[m % 64].record(self.side)
                 if not last:
                     relu_src = acts[m] if self._masked(key, m) else None
                     self._call("conv_dgrad", work, sc.splitcnn_conv_bwd_data, plan.handle, m, self.dtype, g, W, out,
                                relu_src, self.ws, self.ws_bytes, self.flags_extra, p0, p1, stream)
-                self._call("conv_wgrad", work, sc.splitcnn_conv_bwd_filter, plan.handle, m, self.dtype, acts[m], g, dW,
-                           db, 0.0, self.ws, self.ws_bytes, self.flags_extra, p0, p1, stream)
-                if self.wgrad_hook is not None:      # e.g. dist.GradBuckets: start this layer's allreduce
-                    self.wgrad_hook(key, m)
+                if fork:      # join: the next layer may overwrite g's buffer
+                    main.wait_event(self.join_ev[m % 64])
+                else:
+                    self._call("conv_wgrad", work, sc.splitcnn_conv_bwd_filter, plan.handle, m, self.dtype, acts[m], g,
+                               dW, db, 0.0, self.ws, self.ws_bytes, self.flags_extra, p0, p1, stream)
+                    if self.wgrad_hook is not None:      # e.g. dist.GradBuckets: start this layer's allreduce
+                        self.wgrad_hook(key, m)
             else:
                 flags = sc.FLAG_POOL_RELU_MASK if self._masked(key, m) else 0
                 bi, bo = self._bytes(plan, m)

@@ -102,7 +102,7 @@ def make_inputs(c, dtype_t, device, world=1, rank=0):
 def _nets(net):
     """The SplitNet executors inside an executor (the dist executor holds a region and a tail net)."""
     return [n for n in (getattr(net, "region_net", None), getattr(net, "tail_net", None), getattr(net, "net_r", None),
-                        getattr(net, "net_t", None)) if n is not None] or [net]
+                        getattr(net, "net_t", None), getattr(net, "net", None)) if n is not None] or [net]
 
 
 def run_ours(args):
@@ -137,9 +137,12 @@ def run_ours(args):
     use_offload = args.offload if args.offload is not None else (args.config == "C4")
     if c.get("resnet"):
         from paper_conf_asplos_jinh19_b200.resnet import ResBNSplitNet, ResSplitNet
-        if world > 1:
-            raise SystemExit("C3 runs on one GPU (the ResNet stack is not patch-sharded here)")
-        if args.full:          # the whole trunk: split region -> unsplit layer3/4 -> global average pool (f2)
+        if world > 1 or args.force_dist:
+            if args.full:
+                raise SystemExit("C3 --full (unsplit tail) runs on one GPU; the split stack shards (DistResNet)")
+            from paper_conf_asplos_jinh19_b200.dist import DistResNet
+            net = DistResNet(c, world, rank, dtype, bn=args.bn)
+        elif args.full:          # the whole trunk: split region -> unsplit layer3/4 -> global average pool (f2)
             import synth
             from paper_conf_asplos_jinh19_b200.resnet import ResNet18Net
             tc, tb = synth.resnet18_tail_blocks()
@@ -168,9 +171,12 @@ def run_ours(args):
         import synth
         net.set_bn_params(synth.bn_params(synth.rng(c["seed"] + 100), [W.shape[0] for W, _ in params]))
     out_numel = net.output_numel()
-    dy_all = torch.randn(out_numel * world, generator=gen).to(net.tdtype)
-    dy_host = dy_all[rank * out_numel:(rank + 1) * out_numel]           # this rank's batch shard of dY
-    if world > 1:            # a rank reads only the input rows of its own patch rows (as its loader would)
+    if c.get("resnet"):      # the ResNet region output stays patch-sharded: every rank reads the whole dY
+        dy_host = torch.randn(out_numel, generator=gen).to(net.tdtype)
+    else:                    # the VGG tail is batch-sharded: this rank's batch shard of dY
+        dy_all = torch.randn(out_numel * world, generator=gen).to(net.tdtype)
+        dy_host = dy_all[rank * out_numel:(rank + 1) * out_numel]
+    if world > 1 and hasattr(net, "input_rows"):   # a rank reads only its own patch rows' input (as its loader would)
         h0, h1 = net.input_rows()
         x_host = x_host[:, :, h0:h1].contiguous()
     x = x_host.cuda()

@@ -74,8 +74,30 @@ def join_messages(level_full: dict, level_shard: dict, owners, rank: int, world:
     return sends, recvs
 
 
+def _host_staged(t: torch.Tensor, group=None) -> bool:
+    """gloo cannot read or write device memory: CUDA tensors are then staged through the host (the
+    multi-process test runs several ranks on one GPU over gloo, since NCCL refuses that)."""
+    return t.is_cuda and dist.get_backend(group) == "gloo"
+
+
+def all_reduce_sum(t: torch.Tensor, group=None, async_op: bool = False):
+    """In-place sum over ranks (NCCL on device memory; gloo through a host copy)."""
+    if _host_staged(t, group):
+        h = t.cpu()
+        dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
+        t.copy_(h)
+        return None
+    return dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group, async_op=async_op)
+
+
 def exchange(src_flat: torch.Tensor, dst_flat: torch.Tensor, sends, recvs, rank: int):
     """Post all sends / receives as tensor views (no packing); self-messages are local copies."""
+    if _host_staged(src_flat):
+        hs, hd = src_flat.cpu(), torch.empty(dst_flat.shape, dtype=dst_flat.dtype)
+        exchange(hs, hd, sends, recvs, rank)
+        for src, q, off, cnt in recvs:
+            dst_flat[off:off + cnt].copy_(hd[off:off + cnt])
+        return
     ops = []
     local = {}
     for dst, q, off, cnt in sends:
@@ -135,7 +157,9 @@ class GradBuckets:
         self.pending[b] -= 1
         if self.pending[b] == 0:
             lo, hi, _ = self.buckets[b]
-            self.works.append(dist.all_reduce(self.flat[lo:hi], op=dist.ReduceOp.SUM, group=self.group, async_op=True))
+            w = all_reduce_sum(self.flat[lo:hi], group=self.group, async_op=True)
+            if w is not None:
+                self.works.append(w)
 
     def wait(self):
         assert all(p == 0 for p in self.pending), "a bucket was never completed"
@@ -275,3 +299,66 @@ class DistSplitNet:
         # their layers' weight gradients were enqueued; the step ends when the last one has landed
         self.buckets.wait()
         self.step_index += 1
+
+
+class DistResNet:
+    """Patch-row sharded ResNet-18 split stack (C3).  Rank r runs every region layer on
+    its own patch rows (ResSplitNet / ResBNSplitNet with patch_range; the 1x1 downsamples share the
+    block's patch grid); the output stays patch-sharded (each rank merges only its rows and reads only
+    their rows of dY).  With BN, every BN's per-channel [2][C] sums are all-reduced before use -- the
+    statistics in forward, (dbeta, dgamma) in backward -- so BN is the unsplit whole-tensor BN (R11)
+    under sharding: 2C floats per BN per pass, the only exchange inside the region besides the
+    weight-gradient sum, which is one allreduce of the conv gradients after the backward (the BN
+    parameter gradients are already global)."""
+
+    def __init__(self, c: dict, world: int, rank: int, dtype: int = sc.BF16, bn: bool = False, device="cuda",
+                 group=None):
+        from .resnet import ResBNSplitNet, ResSplitNet
+        self.world, self.rank, self.dtype, self.group = world, rank, dtype, group
+        nh, nw = c["split"]
+        self.owners = patch_row_ranges(nh, nw, world)
+        kw = dict(split=c["split"], dtype=dtype, device=device, patch_range=self.owners[rank])
+        if bn:
+            kw["bn_reduce"] = lambda t: all_reduce_sum(t, group=group)
+        cls = ResBNSplitNet if bn else ResSplitNet
+        self.net = cls(c["layers"], c["blocks"], c["N"], 3, c["H"], c["W"], **kw)
+        self.n_conv = ResSplitNet.grad_numel(self.net)          # conv (dW, db) part of the flat buffer
+        self.tdtype, self.device = self.net.tdtype, self.net.device
+        self.input_grad = False
+
+    @property
+    def timers(self):
+        return self.net.timers
+
+    @timers.setter
+    def timers(self, v):
+        self.net.timers = v
+
+    @property
+    def grad_flat(self):
+        return self.net.grad_flat
+
+    @property
+    def grads(self):
+        return self.net.grads
+
+    def bind_grads(self, flat):
+        self.net.bind_grads(flat)
+
+    def grad_slice(self):
+        n = self.grad_flat.numel()
+        return (n * self.rank) // self.world, (n * (self.rank + 1)) // self.world
+
+    def set_params(self, params):
+        self.net.set_params(params)
+
+    def set_bn_params(self, bn_params):
+        self.net.set_bn_params(bn_params)
+
+    def output_numel(self) -> int:
+        return self.net.output_numel()
+
+    def step(self, x, dy, stream=None):
+        self.net.forward(x, stream)
+        self.net.backward(dy, stream)
+        all_reduce_sum(self.net.grad_flat[:self.n_conv], group=self.group)

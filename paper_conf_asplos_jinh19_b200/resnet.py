@@ -339,10 +339,14 @@ class ResBNSplitNet(ResSplitNet):
         h = ReLU(BN_a(conv_a(x))),  y = ReLU(BN_b(conv_b(h)) + shortcut(x)),  shortcut = x | BN_ds(ds(x)).
     BN statistics are over the logical tensor (all patches) via splitcnn_bn_stats / _bn_fwd; conv
     outputs z are kept (BN backward needs them), BN(+ReLU) outputs live in separate level buffers.
-    One GPU (no stats allreduce here; under patch sharding the [2][C] sums would be all-reduced)."""
+    Under patch sharding (patch_range, dist.DistResNet) every rank sums its own patches and
+    `bn_reduce(t)` all-reduces the per-channel [2][C] sums before they are used: the statistics after
+    splitcnn_bn_stats, the backward sums (dbeta, dgamma) after splitcnn_bn_bwd_sums -- R11's statistics
+    over the whole logical tensor, from per-rank partial sums."""
 
-    def __init__(self, *a, eps: float = 1e-5, **kw):
+    def __init__(self, *a, eps: float = 1e-5, bn_reduce=None, **kw):
         self.eps = eps
+        self.bn_reduce = bn_reduce          # callable(fp32 tensor): in-place sum over ranks, or None
         super().__init__(*a, **kw)
 
     def _bn_keys(self):
@@ -409,10 +413,12 @@ class ResBNSplitNet(ResSplitNet):
     # ------------------------------------------------------------------ BN helpers
     def _bn_fwd(self, key, z, y, relu, stream):
         P, lv, cnt = self._bn_level(key)
-        p0, p1 = self.patch_range if key[0] == "r" else (0, P.npatch)
+        p0, p1 = self.patch_range        # a downsample plan shares its block's patch grid
         nb = z.numel() * z.element_size()
         self._call("bn", nb, sc.splitcnn_bn_stats, P.handle, lv, self.dtype, z, self.bn_sums[key], self.bn_ws,
                    self.bn_ws_bytes, p0, p1, stream)
+        if self.bn_reduce is not None:
+            self.bn_reduce(self.bn_sums[key])
         self._call("bn", 2 * nb, sc.splitcnn_bn_fwd, P.handle, lv, self.dtype, z, self.bn_sums[key], cnt,
                    self.bn_gamma[key], self.bn_beta[key], self.eps, self.bn_mi[key], y,
                    sc.FLAG_RELU if relu else 0, p0, p1, stream)
@@ -420,11 +426,13 @@ class ResBNSplitNet(ResSplitNet):
     def _bn_bwd(self, key, g, z, y_mask, out, stream):
         """out = dL/dz from g = dL/d(BN output) (y_mask: the BN+ReLU output, or None)."""
         P, lv, cnt = self._bn_level(key)
-        p0, p1 = self.patch_range if key[0] == "r" else (0, P.npatch)
+        p0, p1 = self.patch_range
         nb = z.numel() * z.element_size()
         t = self.bn_grads[key]
         self._call("bn", (3 if y_mask is not None else 2) * nb, sc.splitcnn_bn_bwd_sums, P.handle, lv, self.dtype, g,
                    z, y_mask, self.bn_mi[key], t, self.bn_ws, self.bn_ws_bytes, p0, p1, stream)
+        if self.bn_reduce is not None:
+            self.bn_reduce(t)
         self._call("bn", (4 if y_mask is not None else 3) * nb, sc.splitcnn_bn_bwd, P.handle, lv, self.dtype, g, z,
                    y_mask, self.bn_mi[key], self.bn_gamma[key], t, cnt, out, p0, p1, stream)
 
@@ -459,7 +467,7 @@ class ResBNSplitNet(ResSplitNet):
                     W, _ = self._ds_params[k]
                     self._label = lds["name"]
                     self._call("conv_fwd", self._conv_work(P, 0, lds), sc.splitcnn_conv_fwd, P.handle, 0, dt,
-                               self._inp(m), W, None, self.ds_out[k], fl, 0, P.npatch, stream)
+                               self._inp(m), W, None, self.ds_out[k], fl, p0, p1, stream)
                     self._bn_fwd(("ds", k), self.ds_out[k], self.ds_bn[k], False, stream)
                     s = self.ds_bn[k]
                 else:
@@ -541,9 +549,9 @@ class ResBNSplitNet(ResSplitNet):
                     gs = self._free(gz, gx, gzd)
                     wk = self._conv_work(P, 0, lds)
                     self._call("conv_dgrad", wk, sc.splitcnn_conv_bwd_data, P.handle, 0, dt, gzd, W, gs, None, self.ws,
-                               self.ws_bytes, fl, 0, P.npatch, stream)
+                               self.ws_bytes, fl, p0, p1, stream)
                     self._call("conv_wgrad", wk, sc.splitcnn_conv_bwd_filter, P.handle, 0, dt, self._inp(a), gzd, dW,
-                               None, 0.0, self.ws, self.ws_bytes, fl, 0, P.npatch, stream)
+                               None, 0.0, self.ws, self.ws_bytes, fl, p0, p1, stream)
                 else:
                     gs = gz
                 mask = self._inp(a) if a in self.block_out else None

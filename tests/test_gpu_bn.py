@@ -142,3 +142,35 @@ def test_resnet_bn_stack_bf16(sc):
     channel's dgamma by up to 0.25 normwise.)"""
     errs = _run_stack(sc, sc.BF16, exact=True)
     assert max(errs.values()) <= 2e-2, errs
+
+
+def test_dist_resnet_bn_world1_matches_single(sc):
+    """DistResNet (patch-row sharded ResNet split stack with the BN-sums allreduce, R11) at world size 1
+    reproduces ResBNSplitNet bitwise (the allreduces are identities, the kernels and order the same)."""
+    import os
+    import torch.distributed as dist
+    from paper_conf_asplos_jinh19_b200.dist import DistResNet
+    from paper_conf_asplos_jinh19_b200.resnet import ResBNSplitNet
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    os.environ.setdefault("MASTER_PORT", "29534")
+    if not dist.is_initialized():
+        dist.init_process_group("nccl", rank=0, world_size=1)
+    c = synth.vgg_config("C3", N=2)
+    c["H"] = c["W"] = 64
+    g = synth.rng(6)
+    params = synth.resnet_params(g, c["layers"], c["blocks"])
+    bn = synth.bn_params(g, [W.shape[0] for W, _ in params])
+    tp = [(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params]
+    single = ResBNSplitNet(c["layers"], c["blocks"], 2, 3, 64, 64, split=c["split"])
+    dnet = DistResNet(c, 1, 0, bn=True)
+    for n in (single, dnet):
+        n.set_params(tp)
+        n.set_bn_params(bn)
+    x = torch.from_numpy(synth.uniform(g, (2, 3, 64, 64))).to("cuda", torch.bfloat16)
+    dy = torch.randn(single.output_numel(), generator=torch.Generator().manual_seed(0)).to("cuda", torch.bfloat16)
+    single.step(x, dy)
+    dnet.step(x, dy)
+    torch.cuda.synchronize()
+    assert torch.equal(single.out, dnet.net.out)
+    assert torch.equal(single.grad_flat, dnet.grad_flat)
+    dist.destroy_process_group()

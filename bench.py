@@ -162,8 +162,9 @@ def run_ours(args):
                               omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype, static_pool=args.static_pool)
     else:
         net = SplitNet(c["layers"], c["tail"], c["N"], c.get("C", 3), c["H"], c["W"], split=c["split"], mode=c["mode"],
-                       omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype, static_pool=args.static_pool,
-                       input_grad=args.config == "C1")
+                       omega=c.get("omega", 0.2), seed=c["seed"], dtype=dtype,
+                       static_pool=args.static_pool and args.schedule == "layer", input_grad=args.config == "C1",
+                       schedule=args.schedule, group_rows=args.group_rows)
     net.input_grad = args.config == "C1"      # C1 = one layer's fwd + dgrad + wgrad
     params, x_host, gen = make_inputs(c, net.tdtype, "cuda")
     net.set_params([(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params])
@@ -360,7 +361,8 @@ def run_ours(args):
                    "parallelism": f"patch{world}" if world > 1 else "1gpu",
                    "l2": "inputs/activations >> 126 MB L2 (no flush needed)" if c["H"] >= 224 else
                          "L2 flushed (256 MB write) before every timed step; each step timed by its own events",
-                   "cuda_graph": bool(graph)},
+                   "cuda_graph": bool(graph),
+                   "schedule": args.schedule + (f" ({args.group_rows} patch rows per group)" if args.schedule == "patch" else "")},
         "e2e": {"value": round(global_batch / (ms_e2e / 1e3), 2), "unit": UNIT, "h2d_bytes_per_step": h2d,
                 "d2h_bytes_per_step": d2h},
         "gpu_launches": launches,
@@ -516,6 +518,9 @@ def main():
                     help="run the multi-GPU executor (DistSplitNet, NCCL) even at one rank (exercises the N>1 path)")
     ap.add_argument("--full", action="store_true", help="C3: the whole ResNet-18 trunk (split region + tail + GAP)")
     ap.add_argument("--bn", action="store_true", help="C3 with whole-tensor BN after every conv (R11, f2)")
+    ap.add_argument("--schedule", default="layer", choices=["layer", "patch"],
+                    help="patch: patch-major (depth-first) region schedule, --group-rows patch rows per group")
+    ap.add_argument("--group-rows", type=int, default=1)
     ap.add_argument("--offload", dest="offload", action="store_true", default=None)
     ap.add_argument("--no-offload", dest="offload", action="store_false")
     args = ap.parse_args()

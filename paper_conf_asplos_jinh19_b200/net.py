@@ -35,7 +35,7 @@ class SplitNet:
                  dtype: int = sc.BF16, device="cuda", patch_range=None, force_simt: bool = False,
                  grad_buffer: torch.Tensor | None = None, input_relu: bool = False, fuse_pool: bool = True,
                  static_pool: bool = False, input_grad: bool = False, mask_output_grad: bool = True,
-                 concurrent_wgrad: bool = True):
+                 concurrent_wgrad: bool = True, schedule: str = "layer", group_rows: int = 1):
         self.region_layers, self.tail_layers = region, tail
         self.N, self.C, self.H, self.W = N, C, H, W
         self.split, self.mode, self.omega, self.seed = split, mode, omega, seed
@@ -52,6 +52,12 @@ class SplitNet:
         # a layer's weight gradient and its data gradient both read only dY: the weight gradient runs on a
         # side stream (its own workspace) concurrently with the data gradient, joined before the next layer
         self.concurrent_wgrad = concurrent_wgrad
+        # "layer": every layer over all patches, layer after layer; "patch": patch-major (depth-first,
+        # chained patches never communicate, so any schedule is valid): `group_rows` patch rows
+        # run through the whole split region before the next group, forward and backward
+        if schedule not in ("layer", "patch") or (schedule == "patch" and static_pool):
+            raise ValueError("schedule: 'layer', or 'patch' without static_pool")
+        self.schedule, self.group_rows = schedule, group_rows
         self.timers = None       # list -> every library call is bracketed by CUDA events (bench.py)
         self.wgrad_hook = None   # callable(key, m) after each layer's weight-gradient call is enqueued
         self._label = ""
@@ -121,6 +127,8 @@ class SplitNet:
                     self.fused.add((key, m))
         skip_r = {m + 1 for k, m in self.fused if k == "r"}
         skip_t = {m + 1 for k, m in self.fused if k == "t"}
+        self.ws_bytes = self._ws_size()
+        self.side = None          # created on first use (a meta-device executor only plans)
         if self.static_pool:
             self._alloc_static()      # activations, argmax bytes and gradients: views of one planned arena
         else:
@@ -135,31 +143,59 @@ class SplitNet:
                 for m, l in enumerate(plan.layers):
                     if l["op"] == "maxpool":
                         self.argmax[(key, m)] = torch.zeros(plan.level_elems(m + 1), dtype=torch.uint8, device=dev)
-            maxg = max([self.region.level_elems(m) for m in range(self.region.nlayers + 1)] +
+            region_levels = range(self.region.nlayers + 1)
+            if self.schedule == "patch":
+                # patch-major: the region's gradient levels live one patch group at a time in two compact
+                # ping-pong buffers; the full-size ones are needed only by the tail and the join
+                self.groups = self._patch_groups()
+                gmax = max(self._group_span(m, q0, q1)[1] for m in region_levels for q0, q1 in self.groups)
+                self.ggrad = [torch.zeros(gmax, dtype=td, device=dev), torch.zeros(gmax, dtype=td, device=dev)]
+                region_levels = [self.region.nlayers]
+            maxg = max([self.region.level_elems(m) for m in region_levels] +
                        ([self.tail.level_elems(m) for m in range(self.tail.nlayers + 1)] if self.tail else []))
             self.gbuf = None
             self.grad = [torch.zeros(maxg, dtype=td, device=dev), torch.zeros(maxg, dtype=td, device=dev)]
-        ws = 0
+            self.ws = torch.zeros(self.ws_bytes // 4, dtype=torch.float32, device=dev)
+            self.ws_w = torch.zeros_like(self.ws) if self.concurrent_wgrad else self.ws     # the side stream's
+        self._alloc_params(grad_buffer)
+
+    def _ws_size(self) -> int:
+        """Scratch bytes of the largest conv call (library workspace_size over ops 0..2), 256-aligned."""
+        ws = 16
         for plan in (self.region, self.tail):
             if plan is None:
                 continue
             for m, l in enumerate(plan.layers):
                 if l["op"] == "conv":
-                    ws = max(ws, plan.workspace_size(m, self.dtype, 0), plan.workspace_size(m, self.dtype, 1),
-                             plan.workspace_size(m, self.dtype, 2))
-        self.ws = torch.zeros(max(ws, 16) // 4 + 4, dtype=torch.float32, device=dev)
-        self.ws_bytes = self.ws.numel() * 4
-        self.ws_w = torch.zeros_like(self.ws) if self.concurrent_wgrad else self.ws     # the side stream's
-        self.side = None          # created on first use (a meta-device executor only plans)
-        self.params = {}
+                    ws = max(ws, *(plan.workspace_size(m, self.dtype, op) for op in (0, 1, 2)))
+        return (ws + 255) // 256 * 256
+
+    def _alloc_params(self, grad_buffer=None):
+        """HMMS device PARAMETER pool: every conv's weights [Cout][kh][kw][Cpad] (compute dtype) and
+        bias (fp32), and the flat fp32 weight / bias gradient buffer, as views of ONE contiguous
+        allocation (parameters are small tensors: one pool avoids fragmenting the general pool)."""
+        dev, td = self.device, self.tdtype
+        es = 2 if self.dtype == sc.BF16 else 4
+        al = lambda b: (b + 255) // 256 * 256
+        shapes = []
         for key, layers, plan in (("r", self.region_layers, self.region), ("t", self.tail_layers, self.tail)):
             for m, l in enumerate(layers):
                 if l["op"] == "conv":
-                    cpad = plan.levels[m]["Cpad"]
-                    self.params[(key, m)] = (torch.zeros((l["cout"], l["kh"], l["kw"], cpad), dtype=td, device=dev),
-                                             torch.zeros(l["cout"], dtype=torch.float32, device=dev))
-        self.bind_grads(grad_buffer if grad_buffer is not None else
-                        torch.zeros(self.grad_numel(), dtype=torch.float32, device=dev))
+                    shapes.append(((key, m), (l["cout"], l["kh"], l["kw"], plan.levels[m]["Cpad"]), l["cout"]))
+        nbytes = sum(al(4 * co) + al(es * sh[0] * sh[1] * sh[2] * sh[3]) for _, sh, co in shapes)
+        gbytes = 0 if grad_buffer is not None else al(4 * self.grad_numel())
+        self.param_pool = torch.zeros(nbytes + gbytes, dtype=torch.uint8, device=dev)
+        self.params, off = {}, 0
+        for key, sh, co in shapes:
+            nw = es * sh[0] * sh[1] * sh[2] * sh[3]
+            W = self.param_pool[off:off + nw].view(td).view(sh)
+            off += al(nw)
+            b = self.param_pool[off:off + 4 * co].view(torch.float32)
+            off += al(4 * co)
+            self.params[key] = (W, b)
+        if grad_buffer is None:
+            grad_buffer = self.param_pool[off:off + 4 * self.grad_numel()].view(torch.float32)
+        self.bind_grads(grad_buffer)
 
     # ------------------------------------------------------------------ HMMS static memory plan
     def _tso_schedule(self):
@@ -207,6 +243,8 @@ class SplitNet:
 
     def _tso_bytes(self, name):
         kind, key, m = name
+        if kind == "ws":
+            return self.ws_bytes
         if kind in ("aF", "aB"):                           # the two halves of an offloaded level
             kind = "a"
         plan = self.region if key == "r" else self.tail
@@ -218,9 +256,14 @@ class SplitNet:
         return plan.level_elems(m) * es
 
     def _tso_lifetimes(self):
-        """(schedule, TSO names in first-use order, first use, last use) of one step."""
+        """(schedule, TSO names in first-use order, first use, last use) of one step.  The conv workspaces
+        (the main stream's and the concurrent weight gradient's) are TSOs of the same general pool that
+        live through the whole step (the device general pool also provides the conv workspace)."""
         sched = self._tso_schedule()
         names, first, last = [], {}, {}
+        for w in (("ws", "main", 0), ("ws", "side", 0)) if self.concurrent_wgrad else (("ws", "main", 0),):
+            names.append(w)
+            first[w], last[w] = 0, len(sched) - 1
         for t, (_, ts) in enumerate(sched):
             for n in ts:
                 if n not in first:
@@ -245,9 +288,11 @@ class SplitNet:
         views = {}
         for n, o, b in zip(names, offs, nbytes):
             v = self.arena[o:o + b]
-            views[n] = v if n[0] == "am" else v.view(td)
+            views[n] = v if n[0] == "am" else v.view(torch.float32) if n[0] == "ws" else v.view(td)
         empty = torch.zeros(0, dtype=td, device=self.device)
         self.static_views = views
+        self.ws = views[("ws", "main", 0)]
+        self.ws_w = views.get(("ws", "side", 0), self.ws)
         self.act_r = [views.get(("a", "r", m), views.get(("aF", "r", m), empty)) for m in range(self.region.nlayers + 1)]
         self.act_t = ([views.get(("a", "t", m), empty) for m in range(self.tail.nlayers + 1)] if self.tail else [])
         self.argmax = {(n[1], n[2]): v for n, v in views.items() if n[0] == "am"}
@@ -305,6 +350,20 @@ class SplitNet:
         macs = l.get("macs_per_out", l["cin"] * l["kh"] * l["kw"])
         return 2.0 * lo["N"] * l["cout"] * lo["H"] * lo["W"] * macs
 
+    def _frac(self, plan, m, p0, p1) -> float:
+        """Share of layer m's work (its output level's elements) in patches [p0, p1): the accounting of a
+        call over a patch range (a rank's rows, a patch-major group)."""
+        lv = plan.levels[m + 1]
+        n = lv["n_h"] * lv["n_w"]
+        if p0 == 0 and p1 >= n:
+            return 1.0
+        def off(q):
+            if q >= n:
+                return lv["total_elems"]
+            i, j = divmod(q, lv["n_w"])
+            return lv["N"] * lv["Cpad"] * (lv["bh"][i] * lv["W"] + (lv["bh"][i + 1] - lv["bh"][i]) * lv["bw"][j])
+        return (off(p1) - off(p0)) / lv["total_elems"]
+
     def _bytes(self, plan, m):
         es = 2 if self.dtype == sc.BF16 else 4
         li, lo = plan.levels[m], plan.levels[m + 1]
@@ -327,6 +386,44 @@ class SplitNet:
         layers = self.tail_layers if self.tail else self.region_layers
         return self.mask_output_grad and bool(layers) and layers[-1]["op"] == "conv" and layers[-1].get("relu", True)
 
+    # ------------------------------------------------------------------ patch-major schedule
+    def _patch_groups(self):
+        """Contiguous groups of `group_rows` patch rows inside the patch range: [(p0, p1)]."""
+        lv = self.region.levels[0]
+        nw = lv["n_w"]
+        p0, p1 = self.patch_range
+        r0, r1 = p0 // nw, (p1 - 1) // nw + 1
+        return [(max(p0, r * nw), min(p1, min(r + self.group_rows, r1) * nw)) for r in range(r0, r1, self.group_rows)]
+
+    def _group_span(self, m, q0, q1):
+        """(element offset, element count) of patches [q0, q1) in region level m (patches are contiguous)."""
+        lv = self.region.levels[m]
+        N, Cp, W = lv["N"], lv["Cpad"], lv["W"]
+        def off(q):
+            if q >= lv["n_h"] * lv["n_w"]:
+                return lv["total_elems"]
+            i, j = divmod(q, lv["n_w"])
+            return N * Cp * (lv["bh"][i] * W + (lv["bh"][i + 1] - lv["bh"][i]) * lv["bw"][j])
+        return off(q0), off(q1) - off(q0)
+
+    def _run_bwd_patch_major(self, g, stream, need_input_grad):
+        """Region backward one patch group at a time (its whole layer chain), the group's gradient levels in
+        two compact buffers addressed as if they were full levels (base = buffer - offset of the group's
+        first patch: the library reaches a patch at base + its level offset).  Weight gradients accumulate
+        over the groups (beta = 1 after the first); the allreduce hook fires on the last group."""
+        es = 2 if self.dtype == sc.BF16 else 4
+        out = None
+        for k, (q0, q1) in enumerate(self.groups):
+            state = {"cur": None}
+
+            def outbuf(m, gin, q0=q0, state=state):
+                i = 1 if state["cur"] == 0 else 0
+                state["cur"] = i
+                return self.ggrad[i].data_ptr() - self._group_span(m, q0, q0 + 1)[0] * es
+            out = self._run_bwd("r", self.region, self.region_layers, self.act_r, g, q0, q1, stream, need_input_grad,
+                                beta=0.0 if k == 0 else 1.0, hook=k == len(self.groups) - 1, outbuf=outbuf)
+        return out
+
     # ------------------------------------------------------------------ passes
     def input_rows(self):
         """Input rows [h0, h1) the patch range reads (all rows for the whole grid)."""
@@ -346,7 +443,11 @@ class SplitNet:
                        self.act_r[0], p0, p1, stream)
         else:
             self._call("split", b_in, sc.splitcnn_split, R, 0, dt, x, x_layout, self.act_r[0], p0, p1, stream)
-        self._run_fwd("r", self.region, self.region_layers, self.act_r, p0, p1, stream)
+        if self.schedule == "patch":       # depth-first: each patch group through the whole region
+            for q0, q1 in self.groups:
+                self._run_fwd("r", self.region, self.region_layers, self.act_r, q0, q1, stream)
+        else:
+            self._run_fwd("r", self.region, self.region_layers, self.act_r, p0, p1, stream)
         if self.tail:
             b_j = 2 * self._bytes(self.region, self.region.nlayers - 1)[1]
             self._call("merge", b_j, sc.splitcnn_merge, R, self.region.nlayers, dt, self.act_r[-1], self.act_t[0],
@@ -378,7 +479,7 @@ class SplitNet:
             self.hook_before_fwd(key, m)
             if (key, m) in self.fused:
                 W, b = self.params[(key, m)]
-                self._call("conv_fwd", self._conv_work(plan, m, l), sc.splitcnn_conv_pool_fwd, plan.handle, m,
+                self._call("conv_fwd", self._conv_work(plan, m, l) * self._frac(plan, m, p0, p1), sc.splitcnn_conv_pool_fwd, plan.handle, m,
                            self.dtype, acts[m], W, b, acts[m + 2], self.argmax[(key, m + 1)],
                            sc.FLAG_RELU | sc.FLAG_POOL_RELU_MASK | self.flags_extra, p0, p1, stream)
                 self.hook_after_fwd(key, m)
@@ -387,12 +488,12 @@ class SplitNet:
             if l["op"] == "conv":
                 W, b = self.params[(key, m)]
                 flags = (sc.FLAG_RELU if l.get("relu", True) else 0) | self.flags_extra
-                self._call("conv_fwd", self._conv_work(plan, m, l), sc.splitcnn_conv_fwd_ws, plan.handle, m, self.dtype,
+                self._call("conv_fwd", self._conv_work(plan, m, l) * self._frac(plan, m, p0, p1), sc.splitcnn_conv_fwd_ws, plan.handle, m, self.dtype,
                            acts[m], W, b, acts[m + 1], flags, self.ws, self.ws_bytes, p0, p1, stream)
             else:
                 flags = sc.FLAG_POOL_RELU_MASK if self._masked(key, m) else 0
                 bi, bo = self._bytes(plan, m)
-                work = bi + bo + bo // (2 if self.dtype == sc.BF16 else 4)
+                work = (bi + bo + bo // (2 if self.dtype == sc.BF16 else 4)) * self._frac(plan, m, p0, p1)
                 self._call("pool_fwd", work, sc.splitcnn_pool_fwd, plan.handle, m, self.dtype, acts[m], acts[m + 1],
                            self.argmax[(key, m)], flags, p0, p1, stream)
             self.hook_after_fwd(key, m)
@@ -416,19 +517,24 @@ class SplitNet:
             self._call("split", b_j, sc.splitcnn_split, self.region.handle, self.region.nlayers, self.dtype, g,
                        sc.NHWC, gi, p0, p1, stream)
             g = gi
+        if self.schedule == "patch":
+            return self._run_bwd_patch_major(g, stream, need_input_grad)
         return self._run_bwd("r", self.region, self.region_layers, self.act_r, g, p0, p1, stream, need_input_grad)
 
-    def _run_bwd(self, key, plan, layers, acts, g, p0, p1, stream, need_input_grad):
+    def _run_bwd(self, key, plan, layers, acts, g, p0, p1, stream, need_input_grad, beta=0.0, hook=True, outbuf=None):
         for m in range(len(layers) - 1, -1, -1):
             l = layers[m]
             self._label = l.get("name", f"{key}{m}")
             self.hook_before_bwd(key, m)
             last = (m == 0 and not need_input_grad) and key == "r"
-            out = None if (last and self.gbuf is not None) else self._gout(key, m, g)
+            if last and (self.gbuf is not None or outbuf is not None):
+                out = None
+            else:
+                out = outbuf(m, g) if outbuf is not None else self._gout(key, m, g)
             if l["op"] == "conv":
                 W, _ = self.params[(key, m)]
                 dW, db = self.grads[(key, m)]
-                work = self._conv_work(plan, m, l)
+                work = self._conv_work(plan, m, l) * self._frac(plan, m, p0, p1)
                 fork = self.concurrent_wgrad and not last
                 main = stream if stream is not None else torch.cuda.current_stream(self.device)
                 if fork and self.side is None:
@@ -441,8 +547,8 @@ class SplitNet:
                     self.side.wait_event(ev)
                     with torch.cuda.stream(self.side):
                         self._call("conv_wgrad", work, sc.splitcnn_conv_bwd_filter, plan.handle, m, self.dtype, acts[m],
-                                   g, dW, db, 0.0, self.ws_w, self.ws_bytes, self.flags_extra, p0, p1, self.side)
-                        if self.wgrad_hook is not None:
+                                   g, dW, db, beta, self.ws_w, self.ws_bytes, self.flags_extra, p0, p1, self.side)
+                        if self.wgrad_hook is not None and hook:
                             self.wgrad_hook(key, m)
                         self.join_ev[m % 64].record(self.side)
                 if not last:
@@ -453,13 +559,13 @@ class SplitNet:
                     main.wait_event(self.join_ev[m % 64])
                 else:
                     self._call("conv_wgrad", work, sc.splitcnn_conv_bwd_filter, plan.handle, m, self.dtype, acts[m], g,
-                               dW, db, 0.0, self.ws, self.ws_bytes, self.flags_extra, p0, p1, stream)
-                    if self.wgrad_hook is not None:      # e.g. dist.GradBuckets: start this layer's allreduce
+                               dW, db, beta, self.ws, self.ws_bytes, self.flags_extra, p0, p1, stream)
+                    if self.wgrad_hook is not None and hook:      # e.g. dist.GradBuckets: start this layer's allreduce
                         self.wgrad_hook(key, m)
             else:
                 flags = sc.FLAG_POOL_RELU_MASK if self._masked(key, m) else 0
                 bi, bo = self._bytes(plan, m)
-                work = bi + bo + bo // (2 if self.dtype == sc.BF16 else 4)
+                work = (bi + bo + bo // (2 if self.dtype == sc.BF16 else 4)) * self._frac(plan, m, p0, p1)
                 self._call("pool_bwd", work, sc.splitcnn_pool_bwd, plan.handle, m, self.dtype, g,
                            self.argmax[(key, m)], out, flags, p0, p1, stream)
             if not last:

@@ -130,9 +130,7 @@ class OffloadSplitNet(SplitNet):
                           offloaded_levels=[m for (k, m), v in self.offload_at.items() if v],
                           offloaded_bytes=sum(c for c, o in zip(cand, off) if o),
                           candidate_bytes=sum(cand), cap_bytes=sum(op_t) * bw)
-        for m in self.stats["offloaded_levels"]:
-            if m not in self.host:
-                self.host[m] = torch.empty(self.level_bytes[m], dtype=torch.uint8, pin_memory=True)
+        self._alloc_host_pool()
         self.plan_ready = True
         self._pending = []
         self._inflight = {}
@@ -140,6 +138,26 @@ class OffloadSplitNet(SplitNet):
         if self.static_pool:
             self._alloc_static_offload()
         return self.stats
+
+    def _alloc_host_pool(self):
+        """HMMS host general-purpose pool: ONE pinned allocation holds every offloaded level,
+        placed by the same first-fit planner over the host TSOs' lives -- from the forward op whose D2H
+        starts it to the backward op that first reads the prefetched level (serialized step order)."""
+        lvls = self.stats["offloaded_levels"]
+        if not lvls:
+            self.host, self.host_pool_bytes = {}, 0
+            return
+        fops, bops = self._fwd_ops(), self._bwd_ops()
+        fidx = {op: t for t, op in enumerate(fops)}
+        bidx = {op: len(fops) + u for u, op in enumerate(bops)}
+        first = [fidx[("r", m)] for m in lvls]
+        last = [bidx[("r", m)] for m in lvls]
+        sizes = [self.level_bytes[m] for m in lvls]
+        offs, pool = sc.splitcnn_memplan(sizes, first, last, 4096)
+        if getattr(self, "host_pool_bytes", -1) != pool:
+            self.host_pool = torch.empty(max(pool, 4096), dtype=torch.uint8, pin_memory=True)
+            self.host_pool_bytes = pool
+        self.host = {m: self.host_pool[o:o + b] for m, o, b in zip(lvls, offs, sizes)}
 
     def _alloc_static_offload(self):
         """HMMS static planning WITH the offload schedule (memory is held 'only for the minimum

@@ -239,13 +239,19 @@ def test_static_pool_plan_of_a_step(sc, cfg):
             first.setdefault(n, t)
             names.append(n) if n not in names else None
             last[n] = t
+    # the conv workspaces (main stream, concurrent weight gradient) live in the same general pool for the
+    # whole step
+    for i, w in enumerate((("ws", "main", 0), ("ws", "side", 0))):
+        names.insert(i, w)
+        first[w], last[w] = 0, len(sched) - 1
+    assert (names, first, last) == tuple(net._tso_lifetimes()[1:])
     nb = [net._tso_bytes(n) for n in names]
     off, pool = sc.splitcnn_memplan(nb, [first[n] for n in names], [last[n] for n in names], 1024)
     assert pool == net.pool_bytes
     check_plan(nb, [first[n] for n in names], [last[n] for n in names], off, pool, 1024)
     acts = sum(b for n, b in zip(names, nb) if n[0] in ("a", "am"))
     maxg = max(b for n, b in zip(names, nb) if n[0] == "g")
-    assert pool < acts + 2 * maxg
+    assert pool < acts + 2 * maxg + 2 * net.ws_bytes
     # gradient TSOs exist only in the backward part of the op list (op names ending in "'")
     bwd0 = min(t for t, (op, _) in enumerate(sched) if op.endswith("'"))
     for n in names:

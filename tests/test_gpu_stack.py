@@ -422,3 +422,34 @@ def test_per_op_autograd_modules(sc):
     assert max(normwise(got[i][j], Y[i][j]) for i in range(2) for j in range(2)) <= 1e-4
     assert normwise(w_lib_to_oihw(c2.weight.grad.cpu().numpy(), 16), dWb) <= 1e-4
     assert normwise(w_lib_to_oihw(c1.weight.grad.cpu().numpy(), 8), dWa) <= 1e-4
+
+
+@pytest.mark.parametrize("cfg,N,H,rows", [("C5", 4, 224, 1), ("C4", 2, 64, 2), ("C2", 4, 32, 1)])
+def test_patch_major_schedule(sc, cfg, N, H, rows):
+    """Patch-major (depth-first) scheduling (chained patches never communicate, so a group of patch
+    rows can run through the whole split region before the next): every activation level and the output
+    are bitwise those of the layer-major schedule (the same per-patch kernels), the weight gradients --
+    now summed group by group -- agree to fp32 summation order, and the region's gradient levels need
+    only group-sized buffers."""
+    from paper_conf_asplos_jinh19_b200.net import SplitNet
+    c = synth.vgg_config(cfg, N=N)
+    g = synth.rng(c["seed"])
+    params = [p for p in synth.layer_params(g, c["layers"] + c["tail"]) if p is not None]
+    tp = [(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params]
+    kw = dict(split=c["split"], mode=c["mode"], omega=c.get("omega", 0.2), seed=c["seed"])
+    lm = SplitNet(c["layers"], c["tail"], N, 3, H, H, **kw)
+    pm = SplitNet(c["layers"], c["tail"], N, 3, H, H, schedule="patch", group_rows=rows, **kw)
+    assert len(pm.groups) == -(-c["split"][0] // rows)
+    assert pm.ggrad[0].numel() < lm.grad[0].numel()
+    for n in (lm, pm):
+        n.set_params(tp)
+    x = torch.from_numpy(synth.uniform(g, (N, 3, H, H))).to("cuda", torch.bfloat16)
+    dy = torch.randn(lm.output_numel(), generator=torch.Generator().manual_seed(5)).to("cuda", torch.bfloat16)
+    for _ in range(2):
+        lm.step(x, dy)
+        pm.step(x, dy)
+    torch.cuda.synchronize()
+    for a, b in zip(lm.act_r + lm.act_t, pm.act_r + pm.act_t):
+        assert torch.equal(a, b)
+    ref, got = lm.grad_flat.double(), pm.grad_flat.double()
+    assert float((ref - got).abs().max() / ref.abs().max()) <= 1e-5

@@ -141,7 +141,7 @@ def run_ours(args):
             if args.full:
                 raise SystemExit("C3 --full (unsplit tail) runs on one GPU; the split stack shards (DistResNet)")
             from paper_conf_asplos_jinh19_b200.dist import DistResNet
-            net = DistResNet(c, world, rank, dtype, bn=args.bn)
+            net = DistResNet(c, world, rank, dtype, bn=args.bn, stem_pad=args.stem_pad)
         elif args.full:          # the whole trunk: split region -> unsplit layer3/4 -> global average pool (f2)
             import synth
             from paper_conf_asplos_jinh19_b200.resnet import ResNet18Net
@@ -150,7 +150,8 @@ def run_ours(args):
                               bn=args.bn, dtype=dtype)
         else:
             cls = ResBNSplitNet if args.bn else ResSplitNet
-            net = cls(c["layers"], c["blocks"], c["N"], 3, c["H"], c["W"], split=c["split"], dtype=dtype)
+            net = cls(c["layers"], c["blocks"], c["N"], 3, c["H"], c["W"], split=c["split"], dtype=dtype,
+                      stem_pad=args.stem_pad)
         use_offload = False
     elif world > 1 or args.force_dist:
         from paper_conf_asplos_jinh19_b200.dist import DistSplitNet
@@ -521,6 +522,8 @@ def main():
     ap.add_argument("--schedule", default="layer", choices=["layer", "patch"],
                     help="patch: patch-major (depth-first) region schedule, --group-rows patch rows per group")
     ap.add_argument("--group-rows", type=int, default=1)
+    ap.add_argument("--stem-pad", type=int, default=64, choices=[16, 64],
+                    help="C3: channels of the space-to-depth stem level (12 real; 64 = halo/2-CTA kernels)")
     ap.add_argument("--offload", dest="offload", action="store_true", default=None)
     ap.add_argument("--no-offload", dest="offload", action="store_false")
     args = ap.parse_args()

@@ -312,12 +312,12 @@ class DistResNet:
     parameter gradients are already global)."""
 
     def __init__(self, c: dict, world: int, rank: int, dtype: int = sc.BF16, bn: bool = False, device="cuda",
-                 group=None):
+                 group=None, stem_pad: int = 64):
         from .resnet import ResBNSplitNet, ResSplitNet
         self.world, self.rank, self.dtype, self.group = world, rank, dtype, group
         nh, nw = c["split"]
         self.owners = patch_row_ranges(nh, nw, world)
-        kw = dict(split=c["split"], dtype=dtype, device=device, patch_range=self.owners[rank])
+        kw = dict(split=c["split"], dtype=dtype, device=device, patch_range=self.owners[rank], stem_pad=stem_pad)
         if bn:
             kw["bn_reduce"] = lambda t: all_reduce_sum(t, group=group)
         cls = ResBNSplitNet if bn else ResSplitNet

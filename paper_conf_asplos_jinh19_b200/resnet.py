@@ -17,8 +17,6 @@ BN (R11) is not part of the split stack.
 """
 from __future__ import annotations
 
-import os
-
 import torch
 
 from . import splitcnn as sc
@@ -70,7 +68,8 @@ def s2d_stem_grad(dWp: torch.Tensor, cin: int) -> torch.Tensor:
 
 class ResSplitNet(SplitNet):
     def __init__(self, chain: list[dict], blocks: list[dict], N: int, C: int, H: int, W: int, split=(2, 2),
-                 dtype: int = sc.BF16, device="cuda", force_simt: bool = False, s2d_stem: bool | None = None, **kw):
+                 dtype: int = sc.BF16, device="cuda", force_simt: bool = False, s2d_stem: bool | None = None,
+                 stem_pad: int = 64, **kw):
         self.blocks = blocks
         self.block_at = {b["a"]: k for k, b in enumerate(blocks)}
         st = chain[0]
@@ -81,7 +80,9 @@ class ResSplitNet(SplitNet):
         self.s2d = ok if s2d_stem is None else (s2d_stem and ok)
         self.stem_cin = st["cin"]
         if self.s2d:
-            stem = s2d_stem_layer(st, 0 if os.environ.get("SPLITCNN_S2D_NARROW") else 64)
+            # stem_pad 64: the 12 real channels padded to 64 take the halo / 2-CTA kernels (5.3x the MMA
+            # work of the 7x7 layer, counted as the 7x7 work); 16: the per-tap 16-channel path
+            stem = s2d_stem_layer(st, stem_pad)
             chain = [stem] + list(chain[1:])
             C, H, W = stem["cin"], H // 2, W // 2
         super().__init__(chain, [], N, C, H, W, split=split, mode="even", dtype=dtype, device=device,

@@ -41,5 +41,5 @@ r = {}
 r["fwd_ms"] = t(lambda: sc.splitcnn_conv_fwd(pl.handle, 0, sc.BF16, x, w, b, y, sc.FLAG_RELU))
 r["dgrad_ms"] = t(lambda: sc.splitcnn_conv_bwd_data(pl.handle, 0, sc.BF16, y, w, x, x, ws, ws_b))
 r["wgrad_ms"] = t(lambda: sc.splitcnn_conv_bwd_filter(pl.handle, 0, sc.BF16, x, y, dw, None, 0.0, ws, ws_b))
-print(name, cfg, os.environ.get("SPLITCNN_DBG", "0"), {k: round(v, 4) for k, v in r.items()},
+print(name, cfg, {k: round(v, 4) for k, v in r.items()},
       {k.replace("_ms", "_tflops"): round(fl / (v / 1e3) / 1e12, 1) for k, v in r.items()})

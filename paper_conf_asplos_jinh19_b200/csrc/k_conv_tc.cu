@@ -1726,9 +1726,16 @@ struct TcWgHaloParams {
     int npatch, BH, BNn, kh, kw;
     int nco_blk, nchunk, ntiles, boxes_per_split, nsplit;
     int Cout, Cpi, stages;
+    int rpack;    // Cout <= 64: row-pair packing (below)
     uint32_t tmem_cols;
     float *part;  // [nsplit][Cout][kh][kw][Cpi]
 };
+// Row-pair packing (Cout <= 64, where the upper 64 rows of the M = 128 MMA would be padding): the upper dY
+// block is the SAME dY loaded one output row further down, so against the X box of kernel row r those rows
+// accumulate sum_oh dY[oh + 1] X~[oh + r - pt] = the contribution of kernel row r - 1.  A tile then serves
+// kernel rows (r, r - 1): ceil(kh / 2) tiles instead of kh.  The pixel boxes start one output row early
+// (oh0 = hb * BH - 1), so the shifted block also sees output row 0; the extra row of the unshifted block is
+// dY row -1, zero-filled by TMA.
 
 // CTA2: a cluster of 2 runs one tile of 256 output channels (each CTA: its own 128-channel dY block
 // as A) with cta_group::2 MMAs (M = 256); B is split by input channel -- each CTA loads 32 of the
@@ -1744,11 +1751,13 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
     const int rows = p.BNn * p.BH * 8;
     const int Wp = 8 + p.kw - 1;
     const uint32_t a_blk = (uint32_t)rows * 128u;     // one 64-channel dY block
-    // Cout <= 64: the upper dY block is all out of bounds -- not loaded, and not even given space (the
-    // MMA's rows 64..127 read the next stage's bytes; those accumulator rows are never stored)
-    const uint32_t a_stage = (p.Cout <= 64 ? 1u : 2u) * a_blk;
+    // Cout <= 64 without row packing: the upper dY block is all out of bounds -- not loaded, and not even
+    // given space (the MMA's rows 64..127 read the next stage's bytes; those accumulator rows are never stored)
+    const uint32_t a_stage = (p.Cout <= 64 && !p.rpack ? 1u : 2u) * a_blk;
     const uint32_t xrow = CTA2 ? 64u : 128u;            // bytes per X pixel row (32 or 64 channels)
-    const uint32_t b_bytes = (uint32_t)Wp * p.BH * p.BNn * xrow;
+    // row-packed: ONE X box of BH + kh - 1 rows (one image) serves every kernel row (views r * Wp rows on)
+    const int xh = p.rpack ? p.BH + p.kh - 1 : p.BH;
+    const uint32_t b_bytes = (uint32_t)Wp * xh * p.BNn * xrow;
     const uint32_t b_stage = (b_bytes + 1023u) & ~1023u;
     uint8_t *sA = smem;
     uint8_t *sB = smem + (size_t)S * a_stage;
@@ -1781,8 +1790,10 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
     const int item = CTA2 ? (int)(blockIdx.x >> 1) : (int)blockIdx.x;
     const int tile = item % p.ntiles, z = item / p.ntiles;
     const int ch = tile % p.nchunk;
-    const int r = (tile / p.nchunk) % p.kh;
-    const int co_blk = CTA2 ? 2 * (tile / (p.nchunk * p.kh)) + (int)rank : tile / (p.nchunk * p.kh);
+    const int nr = p.rpack ? 1 : p.kh;                              // kernel-row tiles (row-packed: all rows)
+    const int nv = p.rpack ? (p.kh + 1) / 2 : 1;                    // accumulators (kernel-row pairs) per tile
+    const int r = p.rpack ? 0 : (tile / p.nchunk) % p.kh;
+    const int co_blk = CTA2 ? 2 * (tile / (p.nchunk * nr)) + (int)rank : tile / (p.nchunk * nr);
     const int total_boxes = p.box_prefix[p.npatch];
     const int b0 = z * p.boxes_per_split, b1 = min(total_boxes, b0 + p.boxes_per_split);
     const int N = p.kw * 64;
@@ -1791,7 +1802,7 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
         if (lane == 0) {
             int stage = 0, ql = 0;
             uint32_t ph = 0;
-            const bool hi = p.Cout > 64;
+            const bool hi = p.Cout > 64 || p.rpack;
             const uint32_t tx = (hi ? 2u : 1u) * a_blk + b_bytes;
             for (int b = b0; b < b1; ++b) {
                 while (b >= p.box_prefix[ql + 1]) ++ql;
@@ -1799,7 +1810,7 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
                 const int wb = idx % p.nwb[ql];
                 idx /= p.nwb[ql];
                 const int hb = idx % p.nhb[ql], n = (idx / p.nhb[ql]) * p.BNn;
-                const int ow0 = wb * 8, oh0 = hb * p.BH;
+                const int ow0 = wb * 8, oh0 = hb * p.BH - p.rpack;
                 tc::mbar_wait_sleep(&empty[stage], ph ^ 1);
                 uint8_t *a = sA + (size_t)stage * a_stage;
                 if (CTA2) {   // own dY block + own channel half of X; bytes land on the leader's barrier
@@ -1814,9 +1825,10 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
                 }
                 tc::mbar_arrive_expect_tx(&full[stage], tx);
                 tc::tma_load_4d(a, &p.mapDY[ql], &full[stage], co_blk * 128, ow0, oh0, n);
-                if (hi) tc::tma_load_4d(a + a_blk, &p.mapDY[ql], &full[stage], co_blk * 128 + 64, ow0, oh0, n);
+                if (p.rpack) tc::tma_load_4d(a + a_blk, &p.mapDY[ql], &full[stage], 0, ow0, oh0 + 1, n);
+                else if (hi) tc::tma_load_4d(a + a_blk, &p.mapDY[ql], &full[stage], co_blk * 128 + 64, ow0, oh0, n);
                 tc::tma_load_4d(sB + (size_t)stage * b_stage, &p.mapX[ql], &full[stage], ch * 64, ow0 - p.pl[ql],
-                                oh0 - p.pt[ql] + r, n);
+                                oh0 - p.pt[ql] + r, n);   // row-packed: r = 0, the box spans all kh rows
                 if (++stage == S) { stage = 0; ph ^= 1; }
             }
         }
@@ -1843,8 +1855,14 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
                 } else {
                     const uint64_t bd0 = tc::smem_desc(b_base, 128, (uint32_t)Wp * 128u, 2);
                     const uint64_t bstep = (uint64_t)(2 * Wp * 8);   // 2 rows of Wp pixels x 128 B, >> 4
-                    for (int j = 0; j < rows / 16; ++j)
-                        tc::mma_bf16_ws(tmem_base, a0 + (uint64_t)(128 * j), bd0 + bstep * j, idesc, (b != b0 || j) ? 1u : 0u);
+                    // accumulator v (row-packed): X view of kernel row kh-1-2v (its rows 0..63) and kh-2-2v
+                    // (rows 64..127, the shifted dY block) = the box viewed (kh-1-2v)*Wp pixel rows on
+                    for (int v = 0; v < nv; ++v) {
+                        const uint64_t bv = bd0 + (uint64_t)(p.rpack ? (p.kh - 1 - 2 * v) * Wp * 8 : 0);
+                        for (int j = 0; j < rows / 16; ++j)
+                            tc::mma_bf16_ws(tmem_base + (uint32_t)(v * N), a0 + (uint64_t)(128 * j), bv + bstep * j, idesc,
+                                            (b != b0 || j) ? 1u : 0u);
+                    }
                     tc::mma_commit_ws(&empty[stage]);
                 }
                 if (++stage == S) { stage = 0; ph ^= 1; }
@@ -1856,7 +1874,8 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
         }
     } else {
         const int quad = warp & 3;
-        const int co = co_blk * 128 + quad * 32 + lane;
+        // row-packed: accumulator v, rows 0..63 = kernel row kh-1-2v, rows 64..127 = kh-2-2v (same channels)
+        const int co = p.rpack ? (quad & 1) * 32 + lane : co_blk * 128 + quad * 32 + lane;
         const bool any = b1 > b0;
         if (any) {
             tc::mbar_wait(&tfull[0], 0);
@@ -1864,15 +1883,17 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
         }
         const uint32_t tacc = tmem_base + ((uint32_t)(quad * 32) << 16);
         const int KT = p.kh * p.kw;
-        for (int cc = 0; cc < N; cc += 16) {
+        for (int vc = 0; vc < nv * N; vc += 16) {
+            const int cc = vc % N;
+            const int rr = p.rpack ? p.kh - 1 - 2 * (vc / N) - (quad >= 2 ? 1 : 0) : r;
             float v[16];
             if (any) {
-                tc::tmem_ld16(tacc + cc, v);
+                tc::tmem_ld16(tacc + vc, v);
             } else {
 #pragma unroll
                 for (int e = 0; e < 16; ++e) v[e] = 0.f;
             }
-            if (co >= p.Cout) continue;
+            if (co >= p.Cout || rr < 0) continue;
             // D column -> (tap, input channel); CTA2: the first kw*32 columns are the leader's channel half
             int c, ci;
             if (CTA2) {
@@ -1883,7 +1904,7 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
                 c = cc / 64;
                 ci = ch * 64 + (cc % 64);
             }
-            float4 *d4 = reinterpret_cast<float4 *>(p.part + (((int64_t)z * p.Cout + co) * KT + r * p.kw + c) * p.Cpi + ci);
+            float4 *d4 = reinterpret_cast<float4 *>(p.part + (((int64_t)z * p.Cout + co) * KT + rr * p.kw + c) * p.Cpi + ci);
 #pragma unroll
             for (int e = 0; e < 4; ++e) d4[e] = make_float4(v[4 * e], v[4 * e + 1], v[4 * e + 2], v[4 * e + 3]);
         }
@@ -2107,8 +2128,10 @@ WgradCfg wgrad_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, int p0,
 namespace {
 
 struct WgHaloCfg {
-    int BH, BNn, nco_blk, nchunk, ntiles, total_boxes, nsplit, boxes_per_split;
+    int BH, BNn, nco_blk, nchunk, ntiles, total_boxes, nsplit, boxes_per_split, rpack;
 };
+
+int wgrad_rpack(const LayerGeom &g) { return (g.L.cout <= 64 && g.L.kh >= 2) ? 1 : 0; }
 
 bool wgrad_halo_ok(const Level &Li, const Level &Lo, const LayerGeom &g) {
     return g.L.sh == 1 && g.L.sw == 1 && g.L.kw >= 2 && g.L.kw <= 4 && Li.Cpad % 64 == 0 && Lo.Cpad % 64 == 0;
@@ -2118,21 +2141,24 @@ WgHaloCfg wgrad_halo_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, i
     WgHaloCfg c{};
     long best = -1;
     int maxh = 1;
-    for (int q = p0; q < p1; ++q) maxh = std::max(maxh, Lo.ph(q / Lo.nw()));
-    // BH x BNn x 8 pixels per stage (<= 128, a multiple of 16 for the K = 16 MMA steps)
+    c.rpack = wgrad_rpack(g);   // row-pair packing (see TcWgHaloParams)
+    for (int q = p0; q < p1; ++q) maxh = std::max(maxh, Lo.ph(q / Lo.nw()) + c.rpack);
+    // BH x BNn x 8 pixels per stage (<= 128, a multiple of 16 for the K = 16 MMA steps); row-packed boxes
+    // hold one image (its X box is BH + kh - 1 rows tall, so K groups of consecutive images are not Wp apart)
     for (int bh = 1; bh <= std::min(16, maxh); ++bh)
-        for (int bn = 1; bn * bh * 8 <= 128 && bn <= Lo.N; ++bn) {
+        for (int bn = 1; bn * bh * 8 <= 128 && bn <= (c.rpack ? 1 : Lo.N); ++bn) {
             if ((bh * bn) % 2) continue;
             long n = 0;
             for (int q = p0; q < p1; ++q)
-                n += (long)((Lo.N + bn - 1) / bn) * ((Lo.ph(q / Lo.nw()) + bh - 1) / bh) * ((Lo.pw(q % Lo.nw()) + 7) / 8);
+                n += (long)((Lo.N + bn - 1) / bn) * ((Lo.ph(q / Lo.nw()) + c.rpack + bh - 1) / bh) *
+                     ((Lo.pw(q % Lo.nw()) + 7) / 8);
             // cost ~ boxes x (fixed per-box cost + MMA rows): fewer, fuller boxes win
             const long cost = n * (bh * bn * 8 + 256);
             if (best < 0 || cost < best) { best = cost; c.BH = bh; c.BNn = bn; c.total_boxes = (int)n; }
         }
     c.nco_blk = (g.L.cout + 127) / 128;
     c.nchunk = Li.Cpad / 64;
-    c.ntiles = c.nco_blk * g.L.kh * c.nchunk;
+    c.ntiles = c.nco_blk * (c.rpack ? 1 : g.L.kh) * c.nchunk;
     int Z = std::max(1, (2 * num_sms() + c.ntiles - 1) / c.ntiles);
     Z = std::min(Z, std::max(1, c.total_boxes / 4));
     Z = std::min(Z, 128);
@@ -2192,7 +2218,7 @@ static int wgrad_zbound(int path, const Level &Li, const LayerGeom &g) {
     const int nco = (g.L.cout + 127) / 128;
     int ntiles;
     if (path == 2) return std::max(1, std::min(296, (2 * num_sms() + nco - 1) / nco));
-    if (path == 1) ntiles = nco * g.L.kh * (Li.Cpad / 64);
+    if (path == 1) ntiles = nco * (wgrad_rpack(g) ? 1 : g.L.kh) * (Li.Cpad / 64);
     else {
         const int cbox = std::min(Li.Cpad, 64), nblocks = g.L.kh * g.L.kw * (Li.Cpad / cbox);
         const int maxb = std::min(WG_MAXBLK, 256 / cbox);
@@ -2350,15 +2376,17 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
             P.nco_blk = c.nco_blk; P.nchunk = c.nchunk; P.ntiles = c.ntiles;
             P.boxes_per_split = c.boxes_per_split; P.nsplit = c.nsplit;
             P.Cout = g.L.cout; P.Cpi = Li.Cpad;
+            P.rpack = c.rpack;
             // 2-CTA pairs of 128-channel output blocks when the channels pair up
             const bool cta2 = g.L.cout % 256 == 0;
             if (cta2) P.ntiles = c.ntiles / 2;
             const int Wp = 8 + g.L.kw - 1;
-            const uint32_t a_stage = (g.L.cout <= 64 ? 1u : 2u) * c.BH * c.BNn * 8u * 128u;
-            const uint32_t b_stage = ((uint32_t)Wp * c.BH * c.BNn * (cta2 ? 64u : 128u) + 1023u) & ~1023u;
+            const uint32_t a_stage = (g.L.cout <= 64 && !c.rpack ? 1u : 2u) * c.BH * c.BNn * 8u * 128u;
+            const int xh = c.rpack ? c.BH + g.L.kh - 1 : c.BH;
+            const uint32_t b_stage = ((uint32_t)Wp * xh * c.BNn * (cta2 ? 64u : 128u) + 1023u) & ~1023u;
             const uint32_t stage_bytes = a_stage + b_stage;
             P.stages = std::min<int>(8, (int)((200u * 1024u) / stage_bytes));
-            P.tmem_cols = 256;
+            P.tmem_cols = c.rpack ? 512 : 256;
             P.part = part + (int64_t)zoff * nW;
             int boxes = 0;
             for (int q = g0; q < g1; ++q) {
@@ -2366,7 +2394,7 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
                 const int ho = Lo.ph(i), wo = Lo.pw(j), hp = Li.ph(i), wp = Li.pw(j);
                 P.pt[ql] = g.pad_h[2 * i];
                 P.pl[ql] = g.pad_w[2 * j];
-                P.nhb[ql] = (ho + c.BH - 1) / c.BH;
+                P.nhb[ql] = (ho + c.rpack + c.BH - 1) / c.BH;
                 P.nwb[ql] = (wo + 7) / 8;
                 P.box_prefix[ql] = boxes;
                 boxes += ((Lo.N + c.BNn - 1) / c.BNn) * P.nhb[ql] * P.nwb[ql];
@@ -2387,7 +2415,7 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
                     void *base = (char *)x + Li.offset(i, j) * 2;
                     cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)wp, (cuuint64_t)hp, (cuuint64_t)Li.N};
                     cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)wp * C * 2, (cuuint64_t)hp * wp * C * 2};
-                    cuuint32_t box[4] = {cta2 ? 32u : 64u, (cuuint32_t)Wp, (cuuint32_t)c.BH, (cuuint32_t)c.BNn};
+                    cuuint32_t box[4] = {cta2 ? 32u : 64u, (cuuint32_t)Wp, (cuuint32_t)xh, (cuuint32_t)c.BNn};
                     cuuint32_t es[4] = {1, 1, 1, 1};
                     if (encode(&P.mapX[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides, box, es,
                                CU_TENSOR_MAP_INTERLEAVE_NONE, cta2 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B,

@@ -22,6 +22,8 @@
 #include <cstdlib>
 #include <cstring>
 #include <mutex>
+#include <string>
+#include <unordered_map>
 #include <vector>
 
 #include "common.cuh"
@@ -965,6 +967,35 @@ PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
     return fn;
 }
 
+// Tensor-map cache: every conv call builds one map per patch (A, output, mask) plus the weights' map -- ~9k
+// cuTensorMapEncodeTiled calls per C5 step, all repeating from step to step (same buffers, same plan).  A
+// map is a pure function of its encode arguments, so they are the key (per host thread; cleared when large).
+CUresult encode_cached(CUtensorMap *m, CUtensorMapDataType dt, cuuint32_t rank, void *addr, const cuuint64_t *dims,
+                       const cuuint64_t *strides, const cuuint32_t *box, const cuuint32_t *es, CUtensorMapInterleave il,
+                       CUtensorMapSwizzle sw, CUtensorMapL2promotion l2, CUtensorMapFloatOOBfill oob) {
+    static thread_local std::unordered_map<std::string, CUtensorMap> cache;
+    uint64_t k[32];
+    int n = 0;
+    k[n++] = ((uint64_t)dt << 32) | rank;
+    k[n++] = (uint64_t)(uintptr_t)addr;
+    k[n++] = ((uint64_t)il << 48) | ((uint64_t)sw << 32) | ((uint64_t)l2 << 16) | (uint64_t)oob;
+    for (cuuint32_t i = 0; i < rank; ++i) k[n++] = dims[i];
+    for (cuuint32_t i = 0; i + 1 < rank; ++i) k[n++] = strides[i];
+    for (cuuint32_t i = 0; i < rank; ++i) k[n++] = ((uint64_t)box[i] << 32) | es[i];
+    std::string key(reinterpret_cast<const char *>(k), n * sizeof(uint64_t));
+    auto it = cache.find(key);
+    if (it != cache.end()) {
+        *m = it->second;
+        return CUDA_SUCCESS;
+    }
+    const CUresult r = get_encode()(m, dt, rank, addr, dims, strides, box, es, il, sw, l2, oob);
+    if (r == CUDA_SUCCESS) {
+        if (cache.size() >= 8192) cache.clear();
+        cache.emplace(std::move(key), *m);
+    }
+    return r;
+}
+
 int num_sms() {
     static int n = 0;
     if (!n) {
@@ -1065,8 +1096,8 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
                             int prec = 0, int accum = 0) {
     const bool tf32 = prec == 1;
     const int es = tf32 ? 4 : 2;          // bytes per element of the operand / output levels
-    auto encode = get_encode();
-    if (!encode) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+    if (!get_encode()) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+    auto encode = encode_cached;
     const int kh = ph ? ph->kh : g.L.kh, kw = ph ? ph->kw : g.L.kw, s = mode == 0 ? g.L.sh : 1;
     const int PS = ph ? ph->S : 1, prh = ph ? ph->rh : 0, prw = ph ? ph->rw : 0;
     auto out_ext_h = [&](int i) { return (Lout.ph(i) - prh + PS - 1) / PS; };
@@ -2266,8 +2297,8 @@ void launch_reduce(const float *part, int Z, int64_t n, float *out, float beta, 
 
 splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *dy,
                                        float *dw, float *db, float beta, void *ws, int p0, int p1, cudaStream_t st) {
-    auto encode = get_encode();
-    if (!encode) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+    if (!get_encode()) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+    auto encode = encode_cached;
     const int KT = g.L.kh * g.L.kw, s = g.L.sh;
     const int64_t nW = (int64_t)g.L.cout * KT * Li.Cpad;
     float *part = (float *)ws;

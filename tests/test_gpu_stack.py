@@ -453,3 +453,38 @@ def test_patch_major_schedule(sc, cfg, N, H, rows):
         assert torch.equal(a, b)
     ref, got = lm.grad_flat.double(), pm.grad_flat.double()
     assert float((ref - got).abs().max() / ref.abs().max()) <= 1e-5
+
+
+def test_dist_executor_cuda_graph_world1(sc):
+    """The patch-parallel step (join exchange, bucketed NCCL allreduce issued from the concurrent weight-
+    gradient stream) captured in a CUDA graph through HostPipeline(graphs=True) at world size 1: per-step
+    host gradients bitwise equal to the eager HostPipeline (NCCL collectives are graph-capturable)."""
+    import os
+    import torch.distributed as dist
+    from paper_conf_asplos_jinh19_b200.dist import DistSplitNet
+    from paper_conf_asplos_jinh19_b200.pipeline import HostPipeline
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    os.environ.setdefault("MASTER_PORT", "29535")
+    if not dist.is_initialized():
+        dist.init_process_group("nccl", rank=0, world_size=1)
+    c = synth.vgg_config("C2", N=4)
+    g = synth.rng(1)
+    params = [p for p in synth.layer_params(g, c["layers"] + c["tail"]) if p is not None]
+    tp = [(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params]
+    nets = [DistSplitNet(c, 1, 0), DistSplitNet(c, 1, 0)]
+    for n in nets:
+        n.set_params(tp)
+    xs = [torch.from_numpy(synth.uniform(g, (4, 3, 32, 32))).to(torch.bfloat16).pin_memory() for _ in range(3)]
+    dys = [torch.randn(nets[0].output_numel(), generator=torch.Generator().manual_seed(i)).to(torch.bfloat16).pin_memory()
+           for i in range(3)]
+    outs = []
+    for n, graphs in zip(nets, (False, True)):
+        pipe = HostPipeline(n, xs[0].cuda(), n.output_numel(), graphs=graphs)
+        o = [torch.empty(n.grad_flat.shape, dtype=torch.float32).pin_memory() for _ in range(3)]
+        for xh, dyh, oh in zip(xs, dys, o):
+            pipe.submit(xh, dyh, oh)
+        pipe.synchronize()
+        outs.append(o)
+    for a, b in zip(*outs):
+        assert torch.equal(a, b)
+    dist.destroy_process_group()

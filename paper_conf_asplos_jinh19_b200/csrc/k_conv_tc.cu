@@ -57,6 +57,8 @@ struct TcConvParams {
     int kchan;       // Cpad of the A side (K = taps * kchan)
     int a3d;         // 8-channel A: 3-D maps with pixels merged into 128-byte-wide rows (coordinate 8*w)
     int halo;        // stride-1 halo mode: one A box per (channel chunk, kernel row) serves the kw column taps
+    int tall;        // halo, resident weights, one image per tile: ONE A box of BH + kh - 1 rows per channel chunk
+                     // serves every kernel row (view r = r * Wp pixel rows on) -- K step = a channel chunk
     int halo8;       // 8-channel halo mode: ONE merged-row box per tile serves all taps (no-swizzle K-major A)
     int b3d;         // halo: the kw taps' weights arrive as one 3-D box
     int Wp;          // halo: input box width = 8 + kw - 1
@@ -415,7 +417,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                         if (leader) tc::mbar_arrive_expect_tx(&full[stage], 2 * (p.a_tx_bytes + p.b_tx_bytes));
                         const int cor = co0 + (int)rank * p.BNh;
                         if (p.halo) {
-                            const int cc = ks / p.kh, r = ks - cc * p.kh;
+                            const int cc = p.tall ? ks : ks / p.kh, r = p.tall ? 0 : ks - cc * p.kh;
                             tc::tma2_load_4d(a, &p.mapA[ql], fb, cc * 64, wbase, hbase + r, n0);
                             if (!p.bres) {
                                 if (p.b3d) {
@@ -442,7 +444,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                             for (int kb = 0; kb * 64 < KT * 8; ++kb)
                                 tc::tma_load_2d(b + kb * p.BN * 128, &p.mapB, &full[stage], kb * 64, co0);
                     } else if (p.halo) {
-                        const int cc = ks / p.kh, r = ks - cc * p.kh;
+                        const int cc = p.tall ? ks : ks / p.kh, r = p.tall ? 0 : ks - cc * p.kh;
                         tc::tma_load_4d(a, &p.mapA[ql], &full[stage], cc * 64, wbase, hbase + r, n0);
                         if (p.bres) {
                         } else if (p.b3d) {
@@ -530,6 +532,19 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                         if (++stage == S) { stage = 0; ph ^= 1; }
                         continue;
                     }
+                    if (p.halo && CTA2 && p.tall) {   // every kernel row from one box: views r * Wp rows on
+                        const uint32_t bstep = (uint32_t)p.BNh * 8u;
+                        for (int r = 0; r < p.kh; ++r) {
+                            const uint64_t a0 = tc::smem_desc(a_base + (uint32_t)(r * p.Wp) * 128u, 16, (uint32_t)p.Wp * 128u, 2);
+                            const uint64_t b0 = tc::smem_desc(tc::smem_u32(sW) + (uint32_t)((ks * p.kh + r) * p.kw * p.BNh) * 128u,
+                                                              16, 1024, 2);
+                            for (int c = 0; c < p.kw; ++c)
+                                tc::mma2_bf16_x4_ws(d, a0 + (uint64_t)(8 * c), b0 + (uint64_t)(bstep * c), idesc, (ks | r | c) != 0);
+                        }
+                        tc::mma2_commit_mc_ws(&empty[stage]);
+                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        continue;
+                    }
                     if (p.halo && CTA2) {
                         const uint64_t a0 = tc::smem_desc(a_base, 16, (uint32_t)p.Wp * 128u, 2);
                         const uint64_t b0 = p.bres ? tc::smem_desc(tc::smem_u32(sW) + (uint32_t)(ks * p.kw * p.BNh) * 128u, 16, 1024, 2)
@@ -546,6 +561,20 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                         const uint64_t b0 = tc::smem_desc(b_base, 16, 1024, 2);
                         tc::mma2_bf16_x4_ws(d, a0, b0, idesc, ks != 0);
                         tc::mma2_commit_mc_ws(&empty[stage]);
+                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        continue;
+                    }
+                    if (p.halo && p.tall) {   // every kernel row from one box: views r * Wp rows on
+                        const uint32_t bstep = (uint32_t)p.BN * 8u;
+                        for (int r = 0; r < p.kh; ++r) {
+                            const uint64_t a0 = tc::smem_desc(a_base + (uint32_t)(r * p.Wp) * 128u, 16, (uint32_t)p.Wp * 128u, 2);
+                            const uint64_t b0 = tc::smem_desc(tc::smem_u32(sW) + (uint32_t)((ks * p.kh + r) * p.kw * p.BN) * 128u,
+                                                              16, 1024, 2);
+                            for (int c = 0; c < p.kw; ++c)
+                                tc::mma_k_x4_ws<TF32>(d, a0 + (uint64_t)(8 * c), b0 + (uint64_t)(bstep * c), idesc,
+                                                      (ks | r | c) != 0);
+                        }
+                        tc::mma_commit_ws(&empty[stage]);
                         if (++stage == S) { stage = 0; ph ^= 1; }
                         continue;
                     }
@@ -1143,12 +1172,28 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         } else if (halo) {  // 8 output columns per M group; BH x BNn groups (<= 16)
             long best = -1;
             TileShape hs = ts;
-            for (int bh = pool ? 2 : 1; bh <= 16; bh += pool ? 2 : 1)   // fused pool: whole 2x2 windows per tile
-                for (int bn = 1; bh * bn <= 16 && bn <= N; ++bn) {
-                    long t = 0;
-                    for (auto &e : ext) t += (long)((N + bn - 1) / bn) * ((e.first + bh - 1) / bh) * ((e.second + 7) / 8);
-                    if (best < 0 || t < best || (t == best && bh * bn > hs.BH * hs.BNn)) { best = t; hs = {8, bh, bn}; }
-                }
+            // tall boxes (one A box for all kernel rows, P.tall) hold one image per tile: with resident weights
+            // (one N tile), i.e. the narrow-N layers whose shared-memory traffic the per-row boxes dominate
+            // (predicted here as the weights-resident condition below with the largest tall box, BH = 16)
+            const uint32_t wres = (uint32_t)(cpad / 64) * kh * kw * (BN % 32 == 0 ? BN / 2 : BN) * 128u;
+            const uint32_t tall_max = ((uint32_t)(8 + kw - 1) * (16 + kh - 1) * 128u + 1023u) & ~1023u;
+            const bool tall_pre = nco == 1 && wres + (uint32_t)((BN + 63) / 64) * 16384u + 2u * tall_max <= 206u * 1024u;
+            auto search = [&](int bnmax, TileShape &out) {
+                long best = -1;
+                for (int bh = pool ? 2 : 1; bh <= 16; bh += pool ? 2 : 1)   // fused pool: whole 2x2 windows per tile
+                    for (int bn = 1; bh * bn <= 16 && bn <= std::min(N, bnmax); ++bn) {
+                        long t = 0;
+                        for (auto &e : ext) t += (long)((N + bn - 1) / bn) * ((e.first + bh - 1) / bh) * ((e.second + 7) / 8);
+                        if (best < 0 || t < best || (t == best && bh * bn > out.BH * out.BNn)) { best = t; out = {8, bh, bn}; }
+                    }
+                return best;
+            };
+            const long t_any = search(N, hs);
+            TileShape h1 = ts;
+            // one image per tile only where it costs at most 1/4 more tiles (28x28 patches: +14 %; a 4x4 CIFAR
+            // patch would fill a quarter of the rows)
+            if (tall_pre && search(1, h1) * 4 <= t_any * 5) hs = h1;
+            (void)best;
             ts = hs;
         }
         static thread_local TcConvParams P;  // large; avoid the stack
@@ -1210,10 +1255,19 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             // weights resident when they fit next to the staging tile and >= 2 A stages
             const uint32_t wbytes = (uint32_t)(cpad / 64) * kh * kw * P.BNh * 128u;
             const uint32_t stg = (uint32_t)((BN + 63) / 64) * 128u * 128u;   // one staging buffer
+            const uint32_t tall_stage = ((uint32_t)P.Wp * (ts.BH + kh - 1) * 128u + 1023u) & ~1023u;
             if (nco == 1 && wbytes + stg + 2u * P.a_stage <= 206u * 1024u) {
                 P.bres = 1;
                 P.bres_bytes = wbytes;
                 P.b_tx_bytes = 0;
+                // one (BH + kh - 1)-row box per channel chunk instead of kh BH-row boxes: (BH + kh - 1) / (kh BH)
+                // of the TMA shared-memory writes, and the kh*kw*4 MMAs of a chunk in one stage
+                if (ts.BNn == 1 && wbytes + stg + 2u * tall_stage <= 206u * 1024u) {
+                    P.tall = 1;
+                    P.ksteps = cpad / 64;
+                    P.a_tx_bytes = (uint32_t)P.Wp * (ts.BH + kh - 1) * 128u;
+                    P.a_stage = tall_stage;
+                }
             }
         }
         const uint32_t stage_bytes = P.a_stage + P.b_tx_bytes;
@@ -1273,6 +1327,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             cuuint32_t box[4] = {(cuuint32_t)cpadc, (cuuint32_t)(ts.BW * s), (cuuint32_t)(ts.BH * s), (cuuint32_t)ts.BNn};
             cuuint32_t es[4] = {1, (cuuint32_t)s, (cuuint32_t)s, 1};
             if (halo) box[1] = (cuuint32_t)P.Wp;
+            if (P.tall) box[2] = (cuuint32_t)(ts.BH + kh - 1);
             CUresult r;
             if (a3d) {
                 cuuint64_t d3[3] = {(cuuint64_t)wp * 8, (cuuint64_t)hp, (cuuint64_t)N};

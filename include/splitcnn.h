@@ -225,6 +225,15 @@ SPLITCNN_API splitcnn_status_t splitcnn_conv_fwd_ws(splitcnn_plan_t plan, int32_
                                        uint32_t flags, void *ws, size_t ws_bytes, int32_t p0, int32_t p1,
                                        splitcnn_stream_t stream);
 
+/* Forward with the residual join fused (ResNet basic block): y = act(conv(x) + bias + residual), the
+ * residual a level `layer + 1` buffer (same layout as y, must not alias it).  bf16 on the tensor cores: the
+ * epilogue loads the residual tile with the accumulator and rounds once; other shapes / precisions run
+ * conv_fwd_ws then splitcnn_add (the conv output rounded to the storage type first).  ws as conv_fwd_ws. */
+SPLITCNN_API splitcnn_status_t splitcnn_conv_fwd_res(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                        const void *x, const void *w, const float *bias, const void *residual,
+                                        void *y, uint32_t flags, void *ws, size_t ws_bytes, int32_t p0, int32_t p1,
+                                        splitcnn_stream_t stream);
+
 /* Fused forward of a conv (+bias, ReLU) `layer` and the 2x2 / stride-2 / unpadded max-pool
  * `layer + 1` that follows it (ReLU in place): the tcgen05 epilogue pools the
  * bf16-rounded conv outputs of each tile and writes ONLY the pool's output y_pool (level layer+2

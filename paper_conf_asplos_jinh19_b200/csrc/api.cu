@@ -212,6 +212,32 @@ extern "C" splitcnn_status_t splitcnn_conv_fwd_ws(splitcnn_plan_t plan, int32_t 
     return check_launch("conv_fwd");
 }
 
+extern "C" splitcnn_status_t splitcnn_conv_fwd_res(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                                   const void *x, const void *w, const float *bias, const void *residual,
+                                                   void *y, uint32_t flags, void *ws, size_t ws_bytes, int32_t p0,
+                                                   int32_t p1, splitcnn_stream_t stream) {
+    TRY(check_layer(plan, layer, SPLITCNN_OP_CONV));
+    TRY(check_dtype(dtype));
+    if (!x || !w || !y || !residual) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    if (residual == y) return fail(SPLITCNN_ERR_INVALID_VALUE, "conv_fwd_res: residual must not alias y");
+    NEED_ALIGNED(residual, "residual");
+    TRY(check_range(plan, layer, p0, p1));
+    if (p1 == p0) return SPLITCNN_OK;
+    const Level &Li = plan->levels[layer], &Lo = plan->levels[layer + 1];
+    const LayerGeom &g = plan->layers[layer];
+    const int relu = (flags & SPLITCNN_FLAG_RELU) ? 1 : 0;
+    if (dtype == SPLITCNN_BF16 && !(flags & SPLITCNN_FLAG_FORCE_SIMT) && conv_tc_supported(0, dtype, Li, Lo, g)) {
+        const splitcnn_status_t r = launch_conv_fwd_res_tc(Li, Lo, g, x, w, bias, residual, y, relu, p0, p1,
+                                                           (cudaStream_t)stream);
+        if (r == SPLITCNN_OK) return check_launch("conv_fwd_res");
+        if (r != SPLITCNN_ERR_UNSUPPORTED) return r;
+    }
+    // other shapes / precisions: the conv (no activation) into y, then y = act(y + residual)
+    TRY(splitcnn_conv_fwd_ws(plan, layer, dtype, x, w, bias, y, flags & ~SPLITCNN_FLAG_RELU, ws, ws_bytes, p0, p1,
+                             stream));
+    return splitcnn_add(plan, layer + 1, dtype, y, residual, y, nullptr, relu ? SPLITCNN_FLAG_RELU : 0u, p0, p1, stream);
+}
+
 extern "C" splitcnn_status_t splitcnn_conv_fwd(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype, const void *x,
                                                const void *w, const float *bias, void *y, uint32_t flags, int32_t p0,
                                                int32_t p1, splitcnn_stream_t stream) {

@@ -74,6 +74,7 @@ struct TcConvParams {
     const __nv_bfloat16 *relu_src;
     int relu;
     int accum;        // TF32 direct epilogue: y = acc + y (3xTF32 passes), bias / ReLU / mask after the sum
+    int res;          // forward: the relu_src tile is a residual, y = act(acc + bias + residual) (ResNet join)
     int tpp;          // tiles per patch when uniform (O(1) decode), else 0
     int direct;       // 1: per-thread global stores (odd channel pads); 0: smem-staged TMA store
     int ychunk;       // channels per output box (64, 32, 16 or 8)
@@ -163,7 +164,7 @@ constexpr int CONV_THREADS = 64 + 256;  // producer warp, MMA warp, 8 epilogue w
 
 // 8 accumulator columns (all real channels) -> bf16x8: +bias, ReLU, dgrad ReLU mask
 template <bool BIAS, bool RELU, bool MASK>
-__device__ __forceinline__ uint4 epi8_full(const uint32_t *r, const float *sb, uint4 m4) {
+__device__ __forceinline__ uint4 epi8_full(const uint32_t *r, const float *sb, uint4 m4, bool res = false) {
     float o[8];
 #pragma unroll
     for (int e = 0; e < 8; ++e) o[e] = __uint_as_float(r[e]);
@@ -173,11 +174,20 @@ __device__ __forceinline__ uint4 epi8_full(const uint32_t *r, const float *sb, u
         o[0] += b0.x; o[1] += b0.y; o[2] += b0.z; o[3] += b0.w;
         o[4] += b1.x; o[5] += b1.y; o[6] += b1.z; o[7] += b1.w;
     }
+    if (MASK && res) {   // residual join fused into the forward epilogue: the tile holds the shortcut
+        const __nv_bfloat162 *mh = reinterpret_cast<const __nv_bfloat162 *>(&m4);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+            const float2 mf = __bfloat1622float2(mh[e]);
+            o[2 * e] += mf.x;
+            o[2 * e + 1] += mf.y;
+        }
+    }
     if (RELU) {
 #pragma unroll
         for (int e = 0; e < 8; ++e) o[e] = fmaxf(o[e], 0.f);
     }
-    if (MASK) {
+    if (MASK && !res) {
         const __nv_bfloat162 *mh = reinterpret_cast<const __nv_bfloat162 *>(&m4);
 #pragma unroll
         for (int e = 0; e < 4; ++e) {
@@ -195,7 +205,7 @@ __device__ __forceinline__ uint4 epi8_full(const uint32_t *r, const float *sb, u
 
 // 8 accumulator columns -> bf16x8 with the fused epilogue (bias, ReLU, or the dgrad ReLU mask)
 template <bool BIAS, bool RELU, bool MASK>
-__device__ __forceinline__ uint4 epi8(const uint32_t *r, const float *sb, int co, int Cout, uint4 m4) {
+__device__ __forceinline__ uint4 epi8(const uint32_t *r, const float *sb, int co, int Cout, uint4 m4, bool res = false) {
     float o[8];
 #pragma unroll
     for (int e = 0; e < 8; ++e) o[e] = __uint_as_float(r[e]);
@@ -210,11 +220,20 @@ __device__ __forceinline__ uint4 epi8(const uint32_t *r, const float *sb, int co
 #pragma unroll
         for (int e = 0; e < 8; ++e) o[e] = (co + e < Cout) ? (BIAS ? o[e] + sb[co + e] : o[e]) : 0.f;
     }
+    if (MASK && res) {   // residual join (padding channels of the shortcut are zero)
+        const __nv_bfloat162 *mh = reinterpret_cast<const __nv_bfloat162 *>(&m4);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+            const float2 mf = __bfloat1622float2(mh[e]);
+            o[2 * e] += mf.x;
+            o[2 * e + 1] += mf.y;
+        }
+    }
     if (RELU) {
 #pragma unroll
         for (int e = 0; e < 8; ++e) o[e] = fmaxf(o[e], 0.f);
     }
-    if (MASK) {
+    if (MASK && !res) {
         const __nv_bfloat162 *mh = reinterpret_cast<const __nv_bfloat162 *>(&m4);
 #pragma unroll
         for (int e = 0; e < 4; ++e) {
@@ -705,7 +724,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     for (int u = 0; u < 4; ++u) {
                         uint4 *dst = reinterpret_cast<uint4 *>(cbase + ((cb0 + 16u * u) ^ rsw));
                         const uint4 m4 = MASK ? *dst : make_uint4(0, 0, 0, 0);
-                        *dst = epi8_full<BIAS, RELU, MASK>(r2[u >> 1] + 8 * (u & 1), sbias + co0 + cc + 8 * u, m4);
+                        *dst = epi8_full<BIAS, RELU, MASK>(r2[u >> 1] + 8 * (u & 1), sbias + co0 + cc + 8 * u, m4, p.res);
                     }
                 }
             }
@@ -722,7 +741,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     const uint32_t off = tc::swz((uint32_t)row * rowB + (uint32_t)(c8 & (p.ychunk - 1)) * 2u, p.y_mask);
                     uint4 *dst = reinterpret_cast<uint4 *>(sYb + k * chunk_bytes + off);
                     const uint4 m4 = MASK ? *dst : make_uint4(0, 0, 0, 0);
-                    *dst = epi8<BIAS, RELU, MASK>(r[u >> 1] + 8 * (u & 1), sbias, co0 + c8, p.Cout, m4);
+                    *dst = epi8<BIAS, RELU, MASK>(r[u >> 1] + 8 * (u & 1), sbias, co0 + c8, p.Cout, m4, p.res);
                 }
             }
             tc::tc_fence_before();
@@ -823,7 +842,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     const uint32_t off = tc::swz((uint32_t)row * rowB + (uint32_t)(c8 & (p.ychunk - 1)) * 2u, p.y_mask);
                     uint4 *dst = reinterpret_cast<uint4 *>(sYb + k * chunk_bytes + off);
                     const uint4 m4 = MASK ? *dst : make_uint4(0, 0, 0, 0);
-                    *dst = epi8<BIAS, RELU, MASK>(r + 8 * u, sbias, co0 + c8, p.Cout, m4);
+                    *dst = epi8<BIAS, RELU, MASK>(r + 8 * u, sbias, co0 + c8, p.Cout, m4, p.res);
                 }
             }
             tc::tc_fence_before();
@@ -1122,7 +1141,7 @@ struct PoolFuse {
 splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const LayerGeom &g, const void *a_ptr,
                             const void *w_ptr, int w_rows, const float *bias, void *y, const void *relu_src, int relu,
                             int p0, int p1, cudaStream_t st, const PoolFuse *pool = nullptr, const Phase *ph = nullptr,
-                            int prec = 0, int accum = 0) {
+                            int prec = 0, int accum = 0, int res = 0) {
     const bool tf32 = prec == 1;
     const int es = tf32 ? 4 : 2;          // bytes per element of the operand / output levels
     if (!get_encode()) return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
@@ -1295,6 +1314,8 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.relu_src = (const __nv_bfloat16 *)relu_src;
         P.relu = relu;
         P.accum = accum;
+        P.res = res;
+        if (res && (P.direct || pool || mode != 0)) return fail(SPLITCNN_ERR_UNSUPPORTED, "fused residual: TMA-store forward only");
         if (pool && tf32) return fail(SPLITCNN_ERR_UNSUPPORTED, "conv_pool_fwd: bf16 only");
         if (pool) {
             if (halo8 || P.direct || P.Cout != P.Cpo || P.Cout % 16 || (ts.BW & (ts.BW - 1)) || ts.BW > 16 || ts.BH % 2)
@@ -1562,6 +1583,12 @@ splitcnn_status_t launch_conv_fwd_tc(const Level &Li, const Level &Lo, const Lay
                                      splitcnn_dtype_t dt, int accum) {
     return launch_tc(0, Li, Lo, g, x, w, g.L.cout, bias, y, nullptr, relu, p0, p1, st, nullptr, nullptr,
                      dt == SPLITCNN_BF16 ? 0 : 1, accum);
+}
+
+splitcnn_status_t launch_conv_fwd_res_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *w,
+                                         const float *bias, const void *residual, void *y, int relu, int p0, int p1,
+                                         cudaStream_t st) {
+    return launch_tc(0, Li, Lo, g, x, w, g.L.cout, bias, y, residual, relu, p0, p1, st, nullptr, nullptr, 0, 0, 1);
 }
 
 splitcnn_status_t launch_conv_pool_fwd_tc(const Level &Li, const Level &Lo, const Level &Lp, const LayerGeom &g,

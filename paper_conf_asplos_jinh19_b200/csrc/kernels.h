@@ -44,6 +44,9 @@ size_t conv_tc_ws_bytes(int mode, const Level &Li, const Level &Lo, const LayerG
 splitcnn_status_t launch_conv_fwd_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *w,
                                      const float *bias, void *y, int relu, int p0, int p1, cudaStream_t st,
                                      splitcnn_dtype_t dt = SPLITCNN_BF16, int accum = 0);
+splitcnn_status_t launch_conv_fwd_res_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *w,
+                                         const float *bias, const void *residual, void *y, int relu, int p0, int p1,
+                                         cudaStream_t st);
 splitcnn_status_t launch_conv_pool_fwd_tc(const Level &Li, const Level &Lo, const Level &Lp, const LayerGeom &g,
                                           const void *x, const void *w, const float *bias, void *y_pool, uint8_t *argmax,
                                           int p0, int p1, cudaStream_t st);

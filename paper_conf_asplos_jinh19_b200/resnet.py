@@ -198,11 +198,10 @@ class ResSplitNet(SplitNet):
             if m in self.block_at:
                 k = self.block_at[m]
                 la, lb = L[m], L[m + 1]
-                for mm, ll in ((m, la), (m + 1, lb)):
-                    W, b = self.params[("r", mm)]
-                    self._label = ll["name"]
-                    self._call("conv_fwd", self._conv_work(self.region, mm, ll), sc.splitcnn_conv_fwd, R, mm, dt,
-                               acts[mm], W, b, acts[mm + 1], (sc.FLAG_RELU if ll["relu"] else 0) | fl, p0, p1, stream)
+                W, b = self.params[("r", m)]
+                self._label = la["name"]
+                self._call("conv_fwd", self._conv_work(self.region, m, la), sc.splitcnn_conv_fwd, R, m, dt,
+                           acts[m], W, b, acts[m + 1], (sc.FLAG_RELU if la["relu"] else 0) | fl, p0, p1, stream)
                 if k in self.ds_plans:
                     P, lds = self.ds_plans[k], self.blocks[k]["ds"]
                     W, b = self._ds_params[k]
@@ -212,10 +211,12 @@ class ResSplitNet(SplitNet):
                     sc_src = self.ds_out[k]
                 else:
                     sc_src = acts[m]
-                self._label = f"{la['name'][:-2]}_add"
-                nb = self._bytes(self.region, m + 1)[1]
-                self._call("add", 3 * nb, sc.splitcnn_add, R, m + 2, dt, acts[m + 2], sc_src, acts[m + 2], None,
-                           sc.FLAG_RELU, p0, p1, stream)
+                # conv_b with the residual join fused into its epilogue: y = ReLU(conv_b(h) + b + shortcut)
+                W, b = self.params[("r", m + 1)]
+                self._label = lb["name"]
+                self._call("conv_fwd", self._conv_work(self.region, m + 1, lb), sc.splitcnn_conv_fwd_res, R, m + 1, dt,
+                           acts[m + 1], W, b, sc_src, acts[m + 2], sc.FLAG_RELU | fl, self.ws, self.ws_bytes, p0, p1,
+                           stream)
                 m += 2
                 continue
             if l["op"] == "conv":

@@ -34,7 +34,7 @@ EXPORTED = [
     "splitcnn_plan_create", "splitcnn_plan_destroy", "splitcnn_plan_num_layers", "splitcnn_plan_level",
     "splitcnn_plan_layer", "splitcnn_workspace_size",
     "splitcnn_split", "splitcnn_split_s2d", "splitcnn_split_rows", "splitcnn_merge",
-    "splitcnn_conv_fwd", "splitcnn_conv_fwd_ws", "splitcnn_conv_bwd_data", "splitcnn_conv_bwd_filter",
+    "splitcnn_conv_fwd", "splitcnn_conv_fwd_ws", "splitcnn_conv_fwd_res", "splitcnn_conv_bwd_data", "splitcnn_conv_bwd_filter",
     "splitcnn_pool_fwd", "splitcnn_pool_bwd", "splitcnn_conv_pool_fwd", "splitcnn_conv_pool_supported", "splitcnn_add",
     "splitcnn_gap_fwd", "splitcnn_gap_bwd",
     "splitcnn_bn_workspace_size", "splitcnn_bn_stats", "splitcnn_bn_fwd", "splitcnn_bn_bwd_sums", "splitcnn_bn_bwd",
@@ -90,6 +90,7 @@ _sig("splitcnn_split_rows", [_vp, _i32, ctypes.c_int, _vp, _i32, _i32, _i32, _vp
 _sig("splitcnn_merge", [_vp, _i32, ctypes.c_int, _vp, _vp, _i32, _i32, _i32, _vp])
 _sig("splitcnn_conv_fwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
 _sig("splitcnn_conv_fwd_ws", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _u32, _vp, _sz, _i32, _i32, _vp])
+_sig("splitcnn_conv_fwd_res", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _vp, _u32, _vp, _sz, _i32, _i32, _vp])
 _sig("splitcnn_conv_bwd_data", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _vp, _sz, _u32, _i32, _i32, _vp])
 _sig("splitcnn_conv_bwd_filter", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _f32, _vp, _sz, _u32, _i32, _i32, _vp])
 _sig("splitcnn_pool_fwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
@@ -272,6 +273,12 @@ def splitcnn_conv_fwd(plan, layer, dtype, x, w, bias, y, flags=0, p0=0, p1=-1, s
 def splitcnn_conv_fwd_ws(plan, layer, dtype, x, w, bias, y, flags=0, ws=None, ws_bytes=0, p0=0, p1=-1, stream=None):
     _check(_lib.splitcnn_conv_fwd_ws(plan, layer, dtype, _ptr(x), _ptr(w), _f32(bias), _ptr(y), flags, _ptr(ws),
                                      ws_bytes, p0, p1, _stream(stream)))
+
+
+def splitcnn_conv_fwd_res(plan, layer, dtype, x, w, bias, residual, y, flags=0, ws=None, ws_bytes=0, p0=0, p1=-1,
+                          stream=None):
+    _check(_lib.splitcnn_conv_fwd_res(plan, layer, dtype, _ptr(x), _ptr(w), _f32(bias), _ptr(residual), _ptr(y), flags,
+                                      _ptr(ws), ws_bytes, p0, p1, _stream(stream)))
 
 
 def splitcnn_conv_bwd_data(plan, layer, dtype, dy, w, dx, relu_src=None, ws=None, ws_bytes=0, flags=0, p0=0, p1=-1,

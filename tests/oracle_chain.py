@@ -137,7 +137,9 @@ def run_resnet(chain, blocks, N, C, H, W, Oh, Ow, params, X, G, round_bf16=False
             Wa, ba = prm[m]
             Wb, bb = prm[m + 1]
             h = rnd(O.conv_fwd(acts[m], Wa, ba, lp, True))
-            z = rnd(O.conv_fwd(h, Wb, bb, rp.layers[m + 1], False))
+            # the block output y = ReLU(conv_b(h) + s) is the stored level; conv_b's own output is never stored
+            # (the join is fused into its epilogue), so only y is rounded to the storage type (R13)
+            z = O.conv_fwd(h, Wb, bb, rp.layers[m + 1], False)
             if k in ds:
                 dp, (Wd, bd) = ds[k]
                 s = sc_out[k] = rnd(O.conv_fwd(acts[m], Wd, bd, dp, False))

@@ -454,3 +454,36 @@ def test_split_rows_matches_full_split(sc, layout):
             assert bool((got[:lo] == 7).all()) and bool((got[hi:] == 7).all())
     with pytest.raises(Exception):
         sc.splitcnn_split_rows(pl.handle, 0, sc.BF16, xl[:, :, 1:13].contiguous(), L, 1, 13, ref, 0, 2 * nw)
+
+
+@pytest.mark.parametrize("mode", ["tc", "simt", "fp32"])
+@pytest.mark.parametrize("cin,cout,H,nh", [(64, 64, 28, 2), (128, 128, 14, 2), (64, 128, 30, 3)])
+def test_conv_fwd_res_parity(sc, mode, cin, cout, H, nh):
+    """splitcnn_conv_fwd_res (the ResNet join fused into the conv epilogue): y = ReLU(conv(x) + b + s) per
+    patch against the oracle's conv + residual add, bf16 on tcgen05 (one rounding), the conv-then-add path (FORCE_SIMT)
+    and fp32; the residual's patch buffers are those of the output level."""
+    dtype = sc.FP32 if mode == "fp32" else sc.BF16
+    extra = sc.FLAG_FORCE_SIMT if mode == "simt" else 0
+    layers = [synth.conv(cin, cout, 3, 1, 1)]
+    ref, pl = _make(sc, layers, 2, cin, H, H, nh, nh, seed=cin + H)
+    lp = ref.layers[0]
+    lv0, lv1 = pl.levels
+    g = synth.rng(300 + cin)
+    X = _round(synth.uniform(g, (2, cin, H, H)), dtype, sc)
+    Wt = _round(synth.kaiming(g, cout, cin, 3, 3), dtype, sc)
+    b = synth.uniform(g, (cout,), -0.1, 0.1).astype(np.float64)
+    S = _round(synth.uniform(g, (2, cout, H, H)), dtype, sc)
+    x = _dev(sc, pack_level(X, lv0), dtype)
+    s = _dev(sc, pack_level(S, lv1), dtype)
+    w = _dev(sc, w_oihw_to_lib(Wt, lv0["Cpad"]), dtype)
+    bias = torch.from_numpy(b.astype(np.float32)).cuda()
+    y = torch.full((lv1["total_elems"],), 7.0, dtype=_td(sc, dtype), device="cuda")
+    ws_b = max(pl.workspace_size(0, dtype, 0), 16)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    sc.splitcnn_conv_fwd_res(pl.handle, 0, dtype, x, w, bias, s, y, sc.FLAG_RELU | extra, ws, ws_b)
+    Yref = O.residual_add(O.conv_fwd(O.split(X, lp.Ih, lp.Iw), Wt, b, lp), O.split(S, lp.Oh, lp.Ow), relu=True)
+    got = unpack_level(_host(y), lv1, keep_pad=True)
+    assert max(normwise(got[i][j][:, :cout], Yref[i][j]) for i in range(nh) for j in range(nh)) <= TOL[dtype]
+    for row in got:
+        for blk in row:
+            assert np.all(blk[:, cout:] == 0)

@@ -167,6 +167,9 @@ def run_ours(args):
                        static_pool=args.static_pool and args.schedule == "layer", input_grad=args.config == "C1",
                        schedule=args.schedule, group_rows=args.group_rows)
     net.input_grad = args.config == "C1"      # C1 = one layer's fwd + dgrad + wgrad
+    if args.serial_wgrad:                     # weight gradients on the main stream (A/B of the overlap)
+        for n in _nets(net):
+            n.concurrent_wgrad = False
     params, x_host, gen = make_inputs(c, net.tdtype, "cuda")
     net.set_params([(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params])
     if getattr(net, "set_bn_params", None) is not None:
@@ -509,6 +512,8 @@ def main():
     ap.add_argument("--cpu-tiles", type=int, default=12)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--per-layer", action="store_true")
+    ap.add_argument("--serial-wgrad", action="store_true",
+                    help="weight gradients on the main stream instead of concurrently with the data gradients")
     ap.add_argument("--graph", dest="graph", action="store_true", default=None,
                     help="time CUDA-graph replays of the step (default for C1, C2)")
     ap.add_argument("--no-graph", dest="graph", action="store_false")

@@ -23,6 +23,7 @@
 #include <cstring>
 #include <mutex>
 #include <string>
+#include <type_traits>
 #include <unordered_map>
 #include <vector>
 
@@ -82,6 +83,9 @@ struct TcConvParams {
     uint32_t stage_off, bar_off;  // smem layout
     int ybufs;                    // staging buffers (2: the TMA store of tile t overlaps tile t+1)
     int egroups;                  // 2: two independent 4-warp epilogue groups, one per TMEM accumulator
+    int yring;                    // egroups == 2: staging tiles per group (a ring: up to yring - 1 TMA stores in flight)
+    int nacc_g;                   // TMEM accumulators per epilogue group (2 with dual issue)
+    int dual;                     // two MMA-issuing warps (1 and 10) take alternate tiles (short-K tiles)
     int cta2;                     // 2-CTA MMA (cluster of 2, M = 256): each CTA owns one 128-row M box and N/2 of B
     int BNh;                      // rows of B per CTA (BN / 2 in 2-CTA mode, else BN)
     int total_m, total_pairs, m_tpp;
@@ -160,7 +164,8 @@ __device__ __forceinline__ void get_tile(const TcConvParams &p, int t, uint32_t 
 }
 
 
-constexpr int CONV_THREADS = 64 + 256;  // producer warp, MMA warp, 8 epilogue warps (2 per TMEM lane quadrant)
+// producer warp, MMA warp, 8 epilogue warps (2 per TMEM lane quadrant), a second MMA warp (dual issue)
+constexpr int CONV_THREADS = 64 + 256 + 32;
 
 // 8 accumulator columns (all real channels) -> bf16x8: +bias, ReLU, dgrad ReLU mask
 template <bool BIAS, bool RELU, bool MASK>
@@ -344,8 +349,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
     uint64_t *full = (uint64_t *)(smem + p.bar_off);
     uint64_t *empty = full + S;
     uint64_t *tfull = empty + S;
-    uint64_t *tempty = tfull + 2;
-    uint64_t *ybar = tempty + 2;
+    uint64_t *tempty = tfull + 4;
+    uint64_t *ybar = tempty + 4;
     uint64_t *wbar = ybar + 1;
     uint32_t *tmem_slot = (uint32_t *)(wbar + 2);
     uint8_t *sW = smem + p.bres_off;   // resident weights (bres)
@@ -359,7 +364,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             tc::mbar_init(&full[s], 1);
             tc::mbar_init(&empty[s], 1);
         }
-        for (int a = 0; a < 2; ++a) {
+        for (int a = 0; a < 4; ++a) {
             tc::mbar_init(&tfull[a], 1);
             // the leader's accumulator-empty barrier hears both CTAs' epilogues in 2-CTA mode
             tc::mbar_init(&tempty[a], (p.egroups == 2 ? 4 : 8) * (CTA2 ? 2 : 1));
@@ -419,10 +424,23 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             }
             int stage = 0, it = 0;
             uint32_t ph = 0;
+            // dual issue: two stage rings (even / odd stages), iteration it fills ring it & 1, so each MMA
+            // warp waits on its own stages in order (a parity wait must never be two phases ahead)
+            const int S2 = S & ~1;
+            int rs0 = 0, rs1 = 1;            // next stage / phase of ring 0 and ring 1 (registers, no stack)
+            uint32_t rph0 = 0u, rph1 = 0u;
+            // loop-invariant step / ring length: the per-K-step advance costs what `++stage == S` did (the
+            // MMA warp's K-step loop is issue-latency bound for narrow N, every instruction in it shows)
+            const int sstep = p.dual ? 2 : 1, Sx = p.dual ? S2 : S;
+            auto adv = [&]() {
+                stage += sstep;
+                if (stage >= Sx) { stage -= Sx; ph ^= 1; }
+            };
             for (int t = tfirst; t < total; t += tstep, ++it) {
                 int ql, nb, hb, wb, cb;
                 bool valid;
                 get_tile(p, t, rank, ql, nb, hb, wb, cb, valid);
+                if (p.dual) { stage = (it & 1) ? rs1 : rs0; ph = (it & 1) ? rph1 : rph0; }
                 const int wbase = wb * p.BW * p.s - p.pl[ql];
                 const int hbase = hb * p.BH * p.s - p.pt[ql];
                 const int n0 = nb * p.BNn, co0 = cb * p.BN;
@@ -452,7 +470,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                             tc::tma2_load_4d(a, &p.mapA[ql], fb, cc * 64, wbase + c, hbase + r, n0);
                             tc::tma2_load_2d(b, &p.mapB, fb, tap * p.kchan + cc * 64, cor);
                         }
-                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        adv();
                         continue;
                     }
                     tc::mbar_arrive_expect_tx(&full[stage], p.a_tx_bytes + p.b_tx_bytes);
@@ -488,14 +506,25 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                         tc::tma_load_4d(a, &p.mapA[ql], &full[stage], cc * 64, wbase + c, hbase + r, n0);
                         tc::tma_load_2d(b, &p.mapB, &full[stage], tap * p.kchan + cc * 64, co0);
                     }
-                    if (++stage == S) { stage = 0; ph ^= 1; }
+                    adv();
+                }
+                if (p.dual) {
+                    if (it & 1) { rs1 = stage; rph1 = ph; }
+                    else { rs0 = stage; rph0 = ph; }
                 }
             }
         }
-    } else if (warp == 1) {
-        {
+    } else if (warp == 1 || (warp == 10 && p.dual)) {
+        // q (which issuer) is a compile-time constant of each copy of the loop: derived from the warp index
+        // it would make the stage index look thread-varying to the compiler, and every descriptor would take
+        // a broadcast register move per MMA (the issue path of narrow-N tiles is latency-bound)
+        auto mma_run = [&](auto QC) {
             // ================= MMA issuer: the whole warp runs the loop converged; elect.sync issues.
             // In 2-CTA mode only the leader issues (M = 256 over the pair); the peer's warp 1 idles.
+            // Dual issue (p.dual): warps 1 and 10 take alternate tiles, so one warp's per-tile handshake
+            // (accumulator wait, stage wait, commits) overlaps the other's MMAs -- a tcgen05.mma issue does
+            // not run ahead of the tensor pipe by much, so a single issuer leaves it idle for those cycles.
+            constexpr int q = decltype(QC)::value;
             const uint32_t idesc = tc::idesc_k<TF32>(CTA2 ? 256 : 128, p.BN);
             // halo8: per tap pair, the descriptor relative to the stage base (start address field 0)
             uint64_t h8_adesc[8], h8_bdesc[8];
@@ -522,14 +551,28 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 const int chunk = k0 / p.cpadc;
                 g_aoff[j] = (chunk * p.a_chunk_bytes + (uint32_t)((k0 - chunk * p.cpadc) * 2)) >> 4;
             }
-            int stage = 0, acc = 0;
-            uint32_t ph = 0, aph = 0;
+            const int istep = p.dual ? 2 : 1;
+            int stage = p.dual ? q : 0;   // dual: this warp's stage ring (see the producer)
+            uint32_t ph = 0;
+            const int S2 = S & ~1;
+            // loop-invariant step / ring length: the per-K-step advance costs what `++stage == S` did (the
+            // MMA warp's K-step loop is issue-latency bound for narrow N, every instruction in it shows)
+            const int sstep = p.dual ? 2 : 1, Sx = p.dual ? S2 : S;
+            auto adv = [&]() {
+                stage += sstep;
+                if (stage >= Sx) { stage -= Sx; ph ^= 1; }
+            };
             if (p.bres && leader) tc::mbar_wait(wbar, 0);
-            int it = 0;
-            for (int t = leader ? tfirst : total; t < total; t += tstep, ++it) {
-                tc::mbar_wait(&tempty[acc], aph ^ 1);
+            // this warp cycles through two accumulator slots: 0, 1 (one issuer: tile it -> epilogue group
+            // it & 1) or 2q, 2q + 1 (dual: warp q's tiles all go to group q, which alternates its two)
+            const int sbase = p.dual ? 2 * q : 0;
+            int acc = 0;
+            uint32_t aph = 0;
+            for (int t = leader ? tfirst + q * tstep : total; t < total; t += istep * tstep) {
+                const int slot = sbase + acc;
+                tc::mbar_wait(&tempty[slot], aph ^ 1);
                 tc::tc_fence_after();
-                const uint32_t d = tmem_base + (uint32_t)(acc * p.BN);
+                const uint32_t d = tmem_base + (uint32_t)(slot * p.BN);
                 for (int ks = 0; ks < p.ksteps; ++ks) {
                     tc::mbar_wait(&full[stage], ph);
                     tc::tc_fence_after();
@@ -548,7 +591,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                                 tc::mma_k_ws<TF32>(d, h8_adesc[pr] + abase, h8_bdesc[pr] + bbase, idesc, (ks | pr) != 0);
                         }
                         tc::mma_commit_ws(&empty[stage]);
-                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        adv();
                         continue;
                     }
                     if (p.halo && CTA2 && p.tall) {   // every kernel row from one box: views r * Wp rows on
@@ -561,7 +604,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                                 tc::mma2_bf16_x4_ws(d, a0 + (uint64_t)(8 * c), b0 + (uint64_t)(bstep * c), idesc, (ks | r | c) != 0);
                         }
                         tc::mma2_commit_mc_ws(&empty[stage]);
-                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        adv();
                         continue;
                     }
                     if (p.halo && CTA2) {
@@ -572,7 +615,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                         for (int c = 0; c < p.kw; ++c)
                             tc::mma2_bf16_x4_ws(d, a0 + (uint64_t)(8 * c), b0 + (uint64_t)(bstep * c), idesc, (ks | c) != 0);
                         tc::mma2_commit_mc_ws(&empty[stage]);
-                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        adv();
                         continue;
                     }
                     if (CTA2) {
@@ -580,7 +623,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                         const uint64_t b0 = tc::smem_desc(b_base, 16, 1024, 2);
                         tc::mma2_bf16_x4_ws(d, a0, b0, idesc, ks != 0);
                         tc::mma2_commit_mc_ws(&empty[stage]);
-                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        adv();
                         continue;
                     }
                     if (p.halo && p.tall) {   // every kernel row from one box: views r * Wp rows on
@@ -594,7 +637,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                                                       (ks | r | c) != 0);
                         }
                         tc::mma_commit_ws(&empty[stage]);
-                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        adv();
                         continue;
                     }
                     if (p.halo) {
@@ -608,7 +651,7 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                         for (int c = 0; c < p.kw; ++c)
                             tc::mma_k_x4_ws<TF32>(d, a0 + (uint64_t)(8 * c), b0 + (uint64_t)(bstep * c), idesc, (ks | c) != 0);
                         tc::mma_commit_ws(&empty[stage]);
-                        if (++stage == S) { stage = 0; ph ^= 1; }
+                        adv();
                         continue;
                     }
                     const uint64_t a0 = tc::smem_desc(a_base, p.a_lbo, p.a_sbo, p.a_layout);
@@ -617,14 +660,18 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     for (int j = 0; j < 4; ++j)
                         tc::mma_k_ws<TF32>(d, a0 + (uint64_t)g_aoff[j], b0 + (uint64_t)(2 * j), idesc, (ks | j) != 0);
                     tc::mma_commit_ws(&empty[stage]);
-                    if (++stage == S) { stage = 0; ph ^= 1; }
+                    adv();
                 }
-                if (CTA2) tc::mma2_commit_mc_ws(&tfull[acc]);
-                else tc::mma_commit_ws(&tfull[acc]);
+                if (CTA2) tc::mma2_commit_mc_ws(&tfull[slot]);
+                else tc::mma_commit_ws(&tfull[slot]);
                 acc ^= 1;
                 if (acc == 0) aph ^= 1;
             }
-        }
+        };
+        if (warp == 1) mma_run(std::integral_constant<int, 0>{});
+        else mma_run(std::integral_constant<int, 1>{});
+    } else if (warp == 10) {
+        // second MMA warp without dual issue: idle
     } else if (!p.direct && p.egroups == 2) {
         // ================= epilogue, two groups: warps 2..5 take even tiles (accumulator 0, staging 0),
         // warps 6..9 odd tiles (accumulator 1, staging 1), so consecutive tiles' epilogues overlap
@@ -634,12 +681,29 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
         const int gtid = threadIdx.x - 64 - 128 * g;   // 0..127 within the group
         const uint32_t rowB = (uint32_t)p.ychunk * 2u;
         const uint32_t chunk_bytes = 128u * rowB;
-        uint8_t *sYb = sY + (size_t)g * p.ybuf_bytes;
         uint64_t *mbar = g ? wbar + 1 : ybar;
-        uint32_t aph = 0, yph = 0;
-        const uint32_t tempty_l = tc::mapa_shared(&tempty[g], 0);   // the leader's (own in 1-CTA mode)
-        int it = g;
-        for (int t = tfirst + g * tstep; t < total; t += 2 * tstep, it += 2) {
+        uint32_t yph = 0;
+        // ReLU-mask tiles (dgrad) with a staging ring: tile k+1's mask is loaded into its ring buffer as soon
+        // as tile k's store is issued, so the load latency overlaps tile k+1's MMAs instead of following them
+        const bool mpre = MASK && p.yring >= 2;
+        auto mask_load = [&](int tt, uint8_t *buf) {   // gtid 0
+            int ql, nb, hb, wb, cb;
+            bool valid;
+            get_tile(p, tt, rank, ql, nb, hb, wb, cb, valid);
+            if (!valid) return;
+            const int co0 = cb * p.BN, nch = min(p.BN, p.Cpo - co0) / p.ychunk;
+            tc::mbar_arrive_expect_tx(mbar, (uint32_t)nch * p.rows_box * rowB);
+            for (int c = 0; c < nch; ++c)
+                tc::tma_load_4d(buf + c * chunk_bytes, &p.mapR[ql], mbar, co0 + c * p.ychunk, wb * p.BW, hb * p.BH, nb * p.BNn);
+        };
+        if (mpre && gtid == 0 && tfirst + g * tstep < total) mask_load(tfirst + g * tstep, sY + (size_t)(g * p.yring) * p.ybuf_bytes);
+        int it = g, k = 0;
+        for (int t = tfirst + g * tstep; t < total; t += 2 * tstep, it += 2, ++k) {
+            const int slot = g * p.nacc_g + (p.nacc_g == 2 ? (k & 1) : 0);
+            const uint32_t aph = (uint32_t)((p.nacc_g == 2 ? (k >> 1) : k) & 1);
+            const uint32_t tempty_l = tc::mapa_shared(&tempty[slot], 0);   // the leader's (own in 1-CTA mode)
+            // staging ring: tile k of this group fills buffer k % yring
+            uint8_t *sYb = sY + (size_t)(g * p.yring + k % p.yring) * p.ybuf_bytes;
             int ql, nb, hb, wb, cb;
             bool valid;
             get_tile(p, t, rank, ql, nb, hb, wb, cb, valid);
@@ -649,9 +713,9 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             const int nchunks = ncols / p.ychunk;
             if (POOL) {
                 // pooled outputs straight from registers: no staging tile, no store of the conv output
-                tc::mbar_wait(&tfull[g], aph);
+                tc::mbar_wait(&tfull[slot], aph);
                 tc::tc_fence_after();
-                const uint32_t tacc = tmem_base + (uint32_t)(g * p.BN) + ((uint32_t)(quad * 32) << 16);
+                const uint32_t tacc = tmem_base + (uint32_t)(slot * p.BN) + ((uint32_t)(quad * 32) << 16);
                 const int wi = row & (p.BW - 1), hi = (row / p.BW) % p.BH, ni = row / (p.BW * p.BH);
                 const int n = n0 + ni, ph = (oh0 + hi) >> 1, pw = (ow0 + wi) >> 1;
                 const int poh = p.out_h[ql] >> 1, pow_ = p.out_w[ql] >> 1;
@@ -689,25 +753,32 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 __syncwarp();
                 if (lane == 0) {
                     if (CTA2) tc::mbar_arrive_remote(tempty_l);
-                    else tc::mbar_arrive(&tempty[g]);
+                    else tc::mbar_arrive(&tempty[slot]);
                 }
-                aph ^= 1;
                 continue;
             }
-            if (gtid == 0) tc::bulk_wait_read0();      // this group's previous store has read the staging
+            if (gtid == 0) {   // the store that last used this staging buffer (yring - 1 stores back) has read it
+                if (p.yring == 1) tc::bulk_wait_read0();
+                else if (p.yring == 2) tc::bulk_wait_read1();
+                else if (p.yring == 3) tc::bulk_wait_read2();
+                else tc::bulk_wait_read3();
+            }
             tc::named_bar_sync(1 + g, 128);
-            if (MASK && valid) {
+            if (mpre && valid) {
+                tc::mbar_wait(mbar, yph);
+                yph ^= 1;
+            } else if (MASK && valid) {
                 if (gtid == 0) {
                     tc::mbar_arrive_expect_tx(mbar, (uint32_t)nchunks * p.rows_box * rowB);
-                    for (int k = 0; k < nchunks; ++k)
-                        tc::tma_load_4d(sYb + k * chunk_bytes, &p.mapR[ql], mbar, co0 + k * p.ychunk, ow0, oh0, n0);
+                    for (int c = 0; c < nchunks; ++c)
+                        tc::tma_load_4d(sYb + c * chunk_bytes, &p.mapR[ql], mbar, co0 + c * p.ychunk, ow0, oh0, n0);
                 }
                 tc::mbar_wait(mbar, yph);
                 yph ^= 1;
             }
-            tc::mbar_wait(&tfull[g], aph);
+            tc::mbar_wait(&tfull[slot], aph);
             tc::tc_fence_after();
-            const uint32_t tacc = tmem_base + (uint32_t)(g * p.BN) + ((uint32_t)(quad * 32) << 16);
+            const uint32_t tacc = tmem_base + (uint32_t)(slot * p.BN) + ((uint32_t)(quad * 32) << 16);
             // fast path: whole 32-column groups of real channels inside one staging chunk (ychunk >= 32)
             const bool fast = (ncols & 31) == 0 && co0 + ncols <= p.Cout && p.ychunk >= 32;
             if (fast) {
@@ -748,16 +819,23 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             __syncwarp();
             if (lane == 0) {
                 if (CTA2) tc::mbar_arrive_remote(tempty_l);
-                else tc::mbar_arrive(&tempty[g]);
+                else tc::mbar_arrive(&tempty[slot]);
             }
             tc::fence_proxy_async_smem();
             tc::named_bar_sync(1 + g, 128);
-            if (gtid == 0 && valid) {
-                for (int k = 0; k < nchunks; ++k)
-                    tc::tma_store_4d(&p.mapY[ql], sYb + k * chunk_bytes, co0 + k * p.ychunk, ow0, oh0, n0);
+            if (gtid == 0) {   // an empty group keeps the ring's wait counts aligned
+                if (valid)
+                    for (int c = 0; c < nchunks; ++c)
+                        tc::tma_store_4d(&p.mapY[ql], sYb + c * chunk_bytes, co0 + c * p.ychunk, ow0, oh0, n0);
                 tc::bulk_commit();
+                if (mpre && t + 2 * tstep < total) {
+                    // the next tile's buffer was last read by the store yring - 1 tiles before this one
+                    if (p.yring == 2) tc::bulk_wait_read1();
+                    else if (p.yring == 3) tc::bulk_wait_read2();
+                    else tc::bulk_wait_read3();
+                    mask_load(t + 2 * tstep, sY + (size_t)(g * p.yring + (k + 1) % p.yring) * p.ybuf_bytes);
+                }
             }
-            aph ^= 1;
         }
         if (gtid == 0) tc::bulk_wait0();
     } else if (!p.direct) {
@@ -1301,13 +1379,29 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         if (P.bres && P.bres_bytes + 2u * P.ybuf_bytes + 2u * P.a_stage > 206u * 1024u) P.ybufs = 1;
         P.egroups = (P.ybufs == 2) ? 2 : 1;
         if (ph && P.direct) return fail(SPLITCNN_ERR_UNSUPPORTED, "phase dgrad needs a TMA-store output");
-        const uint32_t staging = P.ybufs * P.ybuf_bytes;
+        // two groups: a ring of up to 4 staging tiles each, so that a group refills a tile while the TMA
+        // stores of its last yring - 1 tiles are still reading theirs (one tile per group serialises the
+        // epilogue on the store's shared-memory read, which runs at the HBM write rate: hs_probe.cu)
+        P.yring = 1;
+        if (P.egroups == 2) {
+            const uint32_t min_st = 4;
+            for (int r = 4; r >= 2; --r)
+                if (P.bres_bytes + 2u * (uint32_t)r * P.ybuf_bytes + min_st * stage_bytes <= 210u * 1024u) { P.yring = r; break; }
+        }
+        // dual MMA issue for accumulators of <= 128 columns (4 of them in TMEM): short-K tiles (not the
+        // 8-channel halo forward, whose 5-MMA tiles are store-bound: in the C5 step dual issue costs it 9 %)
+        P.dual = (P.egroups == 2 && BN <= 128 && !tf32 && !halo8) ? 1 : 0;
+        P.nacc_g = P.dual ? 2 : 1;
+        // the fused pool epilogue stores from registers: no staging tiles
+        const uint32_t staging = pool ? 0u : (P.egroups == 2 ? 2u * (uint32_t)P.yring : (uint32_t)P.ybufs) * P.ybuf_bytes;
         P.stages = std::min<int>(8, (int)((210u * 1024u - staging - P.bres_bytes) / stage_bytes));
+        // dual issue splits the stages into two rings: only with >= 2 stages per ring
+        if (P.stages < 4) { P.dual = 0; P.nacc_g = 1; }
         P.bres_off = (uint32_t)P.stages * stage_bytes;
         P.stage_off = P.bres_off + ((P.bres_bytes + 1023u) & ~1023u);
         P.bar_off = P.stage_off + ((staging + 1023u) & ~1023u);
         uint32_t cols = 32;
-        while (cols < 2u * BN) cols <<= 1;
+        while (cols < 2u * (uint32_t)P.nacc_g * BN) cols <<= 1;
         P.tmem_cols = cols;
         P.bias = bias;
         P.y = (__nv_bfloat16 *)y;
@@ -1434,6 +1528,15 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         if (tiles == 0) continue;
         const size_t smem = 1024 + (size_t)P.bar_off + 512 + (bias ? 4 * (size_t)g.L.cout : 0) + 64;
         const int grid = P.cta2 ? 2 * std::min(P.total_pairs, num_sms() / 2) : std::min(tiles, num_sms());
+        // dual issue halves the stage ring a tile sees: only where a CTA has many tiles to overlap
+        const long per_cta = P.cta2 ? ((long)P.total_pairs + grid / 2 - 1) / (grid / 2) : ((long)tiles + grid - 1) / grid;
+        if (P.dual && (per_cta < 8 || P.ksteps > 2)) {
+            P.dual = 0;
+            P.nacc_g = 1;
+            uint32_t c2 = 32;
+            while (c2 < 2u * BN) c2 <<= 1;
+            P.tmem_cols = c2;
+        }
         const int mode_bits = (bias ? 4 : 0) | (relu ? 2 : 0) | (relu_src ? 1 : 0);
         auto launch = [&](auto kern) {
             static bool set[32] = {false};
@@ -1445,7 +1548,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             if (P.cta2) {
                 cudaLaunchConfig_t cfg = {};
                 cfg.gridDim = dim3((unsigned)grid);
-                cfg.blockDim = dim3(CONV_THREADS);
+                cfg.blockDim = dim3(P.dual ? CONV_THREADS : CONV_THREADS - 32);
                 cfg.dynamicSmemBytes = smem;
                 cfg.stream = st;
                 cudaLaunchAttribute at[1];
@@ -1457,7 +1560,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
                 cfg.numAttrs = 1;
                 cudaLaunchKernelEx(&cfg, kern, P);
             } else {
-                kern<<<grid, CONV_THREADS, smem, st>>>(P);
+                kern<<<grid, P.dual ? CONV_THREADS : CONV_THREADS - 32, smem, st>>>(P);
             }
         };
         // kernels holding cta_group::2 instructions must be launched as clusters: separate instantiations
@@ -1472,7 +1575,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
                 if (P.cta2) {
                     cudaLaunchConfig_t cfg = {};
                     cfg.gridDim = dim3((unsigned)grid);
-                    cfg.blockDim = dim3(CONV_THREADS);
+                    cfg.blockDim = dim3(P.dual ? CONV_THREADS : CONV_THREADS - 32);
                     cfg.dynamicSmemBytes = smem;
                     cfg.stream = st;
                     cudaLaunchAttribute at[1];
@@ -1484,7 +1587,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
                     cfg.numAttrs = 1;
                     cudaLaunchKernelEx(&cfg, kern, P);
                 } else {
-                    kern<<<grid, CONV_THREADS, smem, st>>>(P);
+                    kern<<<grid, P.dual ? CONV_THREADS : CONV_THREADS - 32, smem, st>>>(P);
                 }
             };
             switch (key) {

@@ -2455,18 +2455,17 @@ size_t wgrad_tc_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g) {
     return (((size_t)zmax * nW * sizeof(float) + 255) & ~(size_t)255) + dbp + 256;
 }
 
-// Library-owned side stream per device (fork/join through events, so the caller's stream semantics are
-// kept, and CUDA-graph capture records the fork as a parallel branch).
+// Library-owned side stream per device and host thread (fork/join through events, so the caller's stream
+// semantics are kept, and CUDA-graph capture records the fork as a parallel branch; per thread, so two host
+// threads never interleave records of the same fork / join event).
 struct SideStream {
     cudaStream_t s = nullptr;
     cudaEvent_t fork = nullptr, join = nullptr;
 };
 static SideStream &side_stream() {
-    static SideStream ss[16];
-    static std::mutex mu;
+    static thread_local SideStream ss[16];
     int dev = 0;
     cudaGetDevice(&dev);
-    std::lock_guard<std::mutex> lk(mu);
     SideStream &r = ss[dev & 15];
     if (!r.s) {
         cudaStreamCreateWithFlags(&r.s, cudaStreamNonBlocking);
@@ -2501,13 +2500,23 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
         cudaEventRecord(ss->fork, st);
         cudaStreamWaitEvent(ss->s, ss->fork, 0);
     }
+    // every exit joins the side stream back into the caller's (error returns included: an unjoined fork
+    // would invalidate a graph capture and let the db partials race with the next call's workspace)
+    struct Join {
+        SideStream *ss;
+        cudaStream_t st;
+        ~Join() {
+            if (!ss) return;
+            cudaEventRecord(ss->join, ss->s);
+            cudaStreamWaitEvent(st, ss->join, 0);
+        }
+    } join_guard{ss, st};
     bool db_launched = false;
     auto launch_db = [&]() {
         if (!db || db_launched) return;
         db_launched = true;
         const int Zd = launch_db_partials(SPLITCNN_BF16, Lo, dy, part_db, g.L.cout, p0, p1, ss->s);
         launch_reduce(part_db, Zd, g.L.cout, db, beta, ss->s);
-        cudaEventRecord(ss->join, ss->s);
     };
     if (path == 2) {
         static bool narrow_attr = false;
@@ -2766,8 +2775,7 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
     // reproducible, and beta = 1 gives exactly 2x whatever the number of launches
     launch_reduce(part, zoff, nW, dw, beta, st);
     if (db) {
-        launch_db();                              // (no GEMM launch when the range is empty)
-        cudaStreamWaitEvent(st, ss->join, 0);     // join: db is complete in the caller's stream order
+        launch_db();                              // (no GEMM launch when the range is empty; join: join_guard)
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return fail(SPLITCNN_ERR_CUDA, std::string("db column sums: ") + cudaGetErrorString(e));
     }

@@ -61,6 +61,8 @@ struct TcConvParams {
     int tall;        // halo, resident weights, one image per tile: ONE A box of BH + kh - 1 rows per channel chunk
                      // serves every kernel row (view r = r * Wp pixel rows on) -- K step = a channel chunk
     int halo8;       // 8-channel halo mode: ONE merged-row box per tile serves all taps (no-swizzle K-major A)
+    int hn;          // narrow-row halo: 16- / 32-channel input (32 / 64 B SW32 / SW64 rows), one MMA per tap and 16
+                     // channels; a kernel row's taps are one 64-element K box of the weights
     int b3d;         // halo: the kw taps' weights arrive as one 3-D box
     int Wp;          // halo: input box width = 8 + kw - 1
     uint32_t a_stage;  // bytes per A stage (1024-aligned)
@@ -399,6 +401,9 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             if (p.bres && p.halo8) {   // the K = taps x 8 filter in 64-wide boxes, once per CTA
                 tc::mbar_arrive_expect_tx(wbar, p.bres_bytes);
                 for (int kb = 0; kb * 64 < KT * 8; ++kb) tc::tma_load_2d(sW + kb * p.BN * 128, &p.mapB, wbar, kb * 64, 0);
+            } else if (p.bres && p.hn) {   // one 64-element K box per kernel row (its kw taps x Cpad channels)
+                tc::mbar_arrive_expect_tx(wbar, p.bres_bytes);
+                for (int r = 0; r < p.kh; ++r) tc::tma_load_2d(sW + (size_t)r * p.BN * 128, &p.mapB, wbar, r * p.kw * p.kchan, 0);
             } else if (p.bres) {  // every (chunk, kernel row) weight box once, for all tiles of this CTA
                 const int rowB0 = (int)rank * p.BNh;  // 2-CTA: this CTA holds rows [rank*BN/2, +BN/2) of B
                 if (!CTA2) tc::mbar_arrive_expect_tx(wbar, p.bres_bytes);
@@ -484,6 +489,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                         const int cc = p.tall ? ks : ks / p.kh, r = p.tall ? 0 : ks - cc * p.kh;
                         tc::tma_load_4d(a, &p.mapA[ql], &full[stage], cc * 64, wbase, hbase + r, n0);
                         if (p.bres) {
+                        } else if (p.hn) {
+                            tc::tma_load_2d(b, &p.mapB, &full[stage], r * p.kw * p.kchan, co0);
                         } else if (p.b3d) {
                             tc::tma_load_3d(b, &p.mapB, &full[stage], cc * 64, co0, r * p.kw);
                         } else {
@@ -623,6 +630,32 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                         const uint64_t b0 = tc::smem_desc(b_base, 16, 1024, 2);
                         tc::mma2_bf16_x4_ws(d, a0, b0, idesc, ks != 0);
                         tc::mma2_commit_mc_ws(&empty[stage]);
+                        adv();
+                        continue;
+                    }
+                    if (p.hn) {
+                        // narrow rows: tap c of kernel row r is the A box viewed (r * Wp + c) pixel rows on
+                        // (SW32 / SW64, address-based), its K = 16 slices 32 B apart; the weights' slice of tap c
+                        // is 2 * c * Cpad bytes into the kernel row's 128 B K box
+                        const uint32_t rb = 2u * (uint32_t)p.kchan;
+                        const int nrow = p.tall ? p.kh : 1;
+                        for (int rr = 0; rr < nrow; ++rr) {
+                            const int r = p.tall ? rr : ks;
+                            const uint64_t a0 = tc::smem_desc(a_base + (uint32_t)(rr * p.Wp) * rb, 16, (uint32_t)p.Wp * rb, p.a_layout);
+                            const uint64_t b0 = tc::smem_desc(p.bres ? tc::smem_u32(sW) + (uint32_t)(r * p.BN) * 128u : b_base, 16, 1024, 2);
+                            // slice (c, j) sits (c * Cpad / 8 + 2 j) 16-byte units on in BOTH operands: a kernel row
+                            // with kw * Cpad = 64 is exactly the four 32-byte steps of one x4 issue
+                            if (p.kw * p.kchan == 64) {
+                                tc::mma_k_x4_ws<TF32>(d, a0, b0, idesc, (ks | rr) != 0);
+                                continue;
+                            }
+                            for (int c = 0; c < p.kw; ++c)
+                                for (int j = 0; j < p.kchan / 16; ++j)
+                                    tc::mma_k_ws<TF32>(d, a0 + (uint64_t)((c * rb + 32u * j) >> 4),
+                                                       b0 + (uint64_t)((2u * c * p.kchan + 32u * j) >> 4), idesc,
+                                                       (ks | rr | c | j) != 0);
+                        }
+                        tc::mma_commit_ws(&empty[stage]);
                         adv();
                         continue;
                     }
@@ -1256,7 +1289,13 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         // halo mode for narrow outputs (per-tap TMA boxes cannot keep the MMA fed there)
         // (BN = 256 too: the A box of a kernel row then serves kw taps, -29% of the L2->SM traffic that
         // bounds these layers; same-process A/B: conv3_2 fwd 0.94 -> 0.73 ms, conv4_2 0.88 -> 0.70 ms)
-        const int halo = (s == 1 && cpad % 64 == 0 && BN <= 256 && kw >= 2 && kw <= 4) ? 1 : 0;
+        // (also for 4- and 2-wide patches, whose 8-pixel M groups are half / a quarter full: the per-tap
+        // boxes pack whole images but move 3x the operand bytes, and these small layers are bound by the
+        // L2 -> SM operand traffic -- C2 1.18 -> 1.30 ms with per-tap boxes there, scripts/ab_halo_narrow.sh)
+        const int hn = (s == 1 && !tf32 && (cpad == 16 || cpad == 32) && kw >= 2 && kw * cpad <= 64 && mode != 2) ? 1 : 0;
+        const int halo = ((s == 1 && cpad % 64 == 0 && BN <= 256 && kw >= 2 && kw <= 4) || hn) ? 1 : 0;
+        const uint32_t rowb = (uint32_t)std::min(cpad, 64) * 2u;                 // bytes per A pixel row
+        const uint32_t wboxes = hn ? (uint32_t)kh : (uint32_t)(cpad / 64) * kh * kw;   // BN x 128 B weight boxes
         const int halo8 = (mode == 0 && cpad == 8 && s == 1 && kw <= 8 && kh * kw <= 16) ? 1 : 0;
         TileShape ts = pool ? choose_tile_pool(ext, N) : choose_tile(ext, N, s, a3d ? 32 : 128);
         if (halo8) {  // 8 output columns x BH output rows, one image per tile
@@ -1272,8 +1311,8 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             // tall boxes (one A box for all kernel rows, P.tall) hold one image per tile: with resident weights
             // (one N tile), i.e. the narrow-N layers whose shared-memory traffic the per-row boxes dominate
             // (predicted here as the weights-resident condition below with the largest tall box, BH = 16)
-            const uint32_t wres = (uint32_t)(cpad / 64) * kh * kw * (BN % 32 == 0 ? BN / 2 : BN) * 128u;
-            const uint32_t tall_max = ((uint32_t)(8 + kw - 1) * (16 + kh - 1) * 128u + 1023u) & ~1023u;
+            const uint32_t wres = wboxes * (uint32_t)(BN % 32 == 0 && !hn ? BN / 2 : BN) * 128u;
+            const uint32_t tall_max = ((uint32_t)(8 + kw - 1) * (16 + kh - 1) * rowb + 1023u) & ~1023u;
             const bool tall_pre = nco == 1 && wres + (uint32_t)((BN + 63) / 64) * 16384u + 2u * tall_max <= 206u * 1024u;
             auto search = [&](int bnmax, TileShape &out) {
                 long best = -1;
@@ -1305,6 +1344,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.a3d = a3d;
         P.halo = halo;
         P.halo8 = halo8;
+        P.hn = hn;
         P.egroups = 1;
         P.Wp = 8 + kw - 1;
         if (cpad >= 64) {
@@ -1345,14 +1385,14 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
                 P.b_tx_bytes = 0;
             }
         } else if (halo) {
-            P.ksteps = (cpad / 64) * kh;
-            P.a_tx_bytes = (uint32_t)P.Wp * ts.BH * ts.BNn * 128u;
+            P.ksteps = hn ? kh : (cpad / 64) * kh;
+            P.a_tx_bytes = (uint32_t)P.Wp * ts.BH * ts.BNn * rowb;
             P.a_stage = (P.a_tx_bytes + 1023u) & ~1023u;
-            P.b_tx_bytes = (uint32_t)kw * P.BNh * 128u;
+            P.b_tx_bytes = (hn ? 1u : (uint32_t)kw) * P.BNh * 128u;
             // weights resident when they fit next to the staging tile and >= 2 A stages
-            const uint32_t wbytes = (uint32_t)(cpad / 64) * kh * kw * P.BNh * 128u;
+            const uint32_t wbytes = wboxes * P.BNh * 128u;
             const uint32_t stg = (uint32_t)((BN + 63) / 64) * 128u * 128u;   // one staging buffer
-            const uint32_t tall_stage = ((uint32_t)P.Wp * (ts.BH + kh - 1) * 128u + 1023u) & ~1023u;
+            const uint32_t tall_stage = ((uint32_t)P.Wp * (ts.BH + kh - 1) * rowb + 1023u) & ~1023u;
             if (nco == 1 && wbytes + stg + 2u * P.a_stage <= 206u * 1024u) {
                 P.bres = 1;
                 P.bres_bytes = wbytes;
@@ -1361,8 +1401,8 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
                 // of the TMA shared-memory writes, and the kh*kw*4 MMAs of a chunk in one stage
                 if (ts.BNn == 1 && wbytes + stg + 2u * tall_stage <= 206u * 1024u) {
                     P.tall = 1;
-                    P.ksteps = cpad / 64;
-                    P.a_tx_bytes = (uint32_t)P.Wp * (ts.BH + kh - 1) * 128u;
+                    P.ksteps = hn ? 1 : cpad / 64;
+                    P.a_tx_bytes = (uint32_t)P.Wp * (ts.BH + kh - 1) * rowb;
                     P.a_stage = tall_stage;
                 }
             }
@@ -1509,7 +1549,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             cuuint32_t es[2] = {1, 1};
             CUresult r = CUDA_ERROR_INVALID_VALUE;
             P.b3d = 0;
-            if (halo) {  // (ci, co, tap) view of [Cout][taps][Cpad]: one box = the kw taps of a kernel row
+            if (halo && !hn) {  // (ci, co, tap) view of [Cout][taps][Cpad]: one box = the kw taps of a kernel row
                 cuuint64_t d3[3] = {(cuuint64_t)cpad, (cuuint64_t)w_rows, (cuuint64_t)(kh * kw)};
                 cuuint64_t s3[2] = {(cuuint64_t)K * 2, (cuuint64_t)cpad * 2};
                 cuuint32_t b3[3] = {64, (cuuint32_t)P.BNh, (cuuint32_t)kw};

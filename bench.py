@@ -527,8 +527,9 @@ def main():
     ap.add_argument("--schedule", default="layer", choices=["layer", "patch"],
                     help="patch: patch-major (depth-first) region schedule, --group-rows patch rows per group")
     ap.add_argument("--group-rows", type=int, default=1)
-    ap.add_argument("--stem-pad", type=int, default=64, choices=[16, 64],
-                    help="C3: channels of the space-to-depth stem level (12 real; 64 = halo/2-CTA kernels)")
+    ap.add_argument("--stem-pad", type=int, default=16, choices=[16, 64],
+                    help="C3: channels of the space-to-depth stem level (12 real; 16 = narrow-row halo kernels, "
+                         "64 = 64-channel halo / 2-CTA kernels on zero channels)")
     ap.add_argument("--offload", dest="offload", action="store_true", default=None)
     ap.add_argument("--no-offload", dest="offload", action="store_false")
     args = ap.parse_args()

@@ -1983,6 +1983,8 @@ struct TcWgHaloParams {
     int nco_blk, nchunk, ntiles, boxes_per_split, nsplit;
     int Cout, Cpi, stages;
     int rpack;    // Cout <= 64: row-pair packing (below)
+    uint32_t xrow;  // bytes per X pixel row in smem: 128 (64-channel chunks), 64 / 32 (32- / 16-channel levels:
+                    // SW64 / SW32 MN-major, MN block = the level's channels), 64 in 2-CTA mode (channel halves)
     uint32_t tmem_cols;
     float *part;  // [nsplit][Cout][kh][kw][Cpi]
 };
@@ -2010,7 +2012,7 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
     // Cout <= 64 without row packing: the upper dY block is all out of bounds -- not loaded, and not even
     // given space (the MMA's rows 64..127 read the next stage's bytes; those accumulator rows are never stored)
     const uint32_t a_stage = (p.Cout <= 64 && !p.rpack ? 1u : 2u) * a_blk;
-    const uint32_t xrow = CTA2 ? 64u : 128u;            // bytes per X pixel row (32 or 64 channels)
+    const uint32_t xrow = p.xrow;                       // bytes per X pixel row (16, 32 or 64 channels)
     // row-packed: ONE X box of BH + kh - 1 rows (one image) serves every kernel row (views r * Wp rows on)
     const int xh = p.rpack ? p.BH + p.kh - 1 : p.BH;
     const uint32_t b_bytes = (uint32_t)Wp * xh * p.BNn * xrow;
@@ -2052,7 +2054,8 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
     const int co_blk = CTA2 ? 2 * (tile / (p.nchunk * nr)) + (int)rank : tile / (p.nchunk * nr);
     const int total_boxes = p.box_prefix[p.npatch];
     const int b0 = z * p.boxes_per_split, b1 = min(total_boxes, b0 + p.boxes_per_split);
-    const int N = p.kw * 64;
+    const int cw = CTA2 ? 64 : (int)(xrow / 2);                     // channels per tap block of D (both CTAs)
+    const int N = p.kw * cw;
 
     if (warp == 0) {
         if (lane == 0) {
@@ -2109,12 +2112,14 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
                         tc::mma2_bf16_ws(tmem_base, a0 + (uint64_t)(128 * j), bd0 + bstep * j, idesc, (b != b0 || j) ? 1u : 0u);
                     tc::mma2_commit_mc_ws(&empty[stage]);
                 } else {
-                    const uint64_t bd0 = tc::smem_desc(b_base, 128, (uint32_t)Wp * 128u, 2);
-                    const uint64_t bstep = (uint64_t)(2 * Wp * 8);   // 2 rows of Wp pixels x 128 B, >> 4
+                    // (16 / 32-channel levels: SW32 / SW64 MN-major, tap c = c pixel rows of xrow bytes on)
+                    const uint32_t lay = xrow == 128u ? 2u : xrow == 64u ? 4u : 6u;
+                    const uint64_t bd0 = tc::smem_desc(b_base, xrow, (uint32_t)Wp * xrow, lay);
+                    const uint64_t bstep = (uint64_t)(2 * Wp * (xrow >> 4));   // 2 rows of Wp pixels, >> 4
                     // accumulator v (row-packed): X view of kernel row kh-1-2v (its rows 0..63) and kh-2-2v
                     // (rows 64..127, the shifted dY block) = the box viewed (kh-1-2v)*Wp pixel rows on
                     for (int v = 0; v < nv; ++v) {
-                        const uint64_t bv = bd0 + (uint64_t)(p.rpack ? (p.kh - 1 - 2 * v) * Wp * 8 : 0);
+                        const uint64_t bv = bd0 + (uint64_t)(p.rpack ? (p.kh - 1 - 2 * v) * Wp * (int)(xrow >> 4) : 0);
                         for (int j = 0; j < rows / 16; ++j)
                             tc::mma_bf16_ws(tmem_base + (uint32_t)(v * N), a0 + (uint64_t)(128 * j), bv + bstep * j, idesc,
                                             (b != b0 || j) ? 1u : 0u);
@@ -2157,8 +2162,8 @@ __global__ void __launch_bounds__(192, 1) wgrad_halo_kernel(const __grid_constan
                 c = n >> 5;
                 ci = ch * 64 + hb * 32 + (n & 31);
             } else {
-                c = cc / 64;
-                ci = ch * 64 + (cc % 64);
+                c = cc / cw;
+                ci = ch * 64 + (cc % cw);
             }
             float4 *d4 = reinterpret_cast<float4 *>(p.part + (((int64_t)z * p.Cout + co) * KT + rr * p.kw + c) * p.Cpi + ci);
 #pragma unroll
@@ -2390,7 +2395,9 @@ struct WgHaloCfg {
 int wgrad_rpack(const LayerGeom &g) { return (g.L.cout <= 64 && g.L.kh >= 2) ? 1 : 0; }
 
 bool wgrad_halo_ok(const Level &Li, const Level &Lo, const LayerGeom &g) {
-    return g.L.sh == 1 && g.L.sw == 1 && g.L.kw >= 2 && g.L.kw <= 4 && Li.Cpad % 64 == 0 && Lo.Cpad % 64 == 0;
+    // 16- / 32-channel inputs: one MN block of the level's channels per tap, N = kw * Cpad (a multiple of 16)
+    const bool narrow = (Li.Cpad == 16 || Li.Cpad == 32) && (g.L.kw * Li.Cpad) % 16 == 0;
+    return g.L.sh == 1 && g.L.sw == 1 && g.L.kw >= 2 && g.L.kw <= 4 && (Li.Cpad % 64 == 0 || narrow) && Lo.Cpad % 64 == 0;
 }
 
 WgHaloCfg wgrad_halo_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, int p0, int p1) {
@@ -2413,12 +2420,12 @@ WgHaloCfg wgrad_halo_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, i
             if (best < 0 || cost < best) { best = cost; c.BH = bh; c.BNn = bn; c.total_boxes = (int)n; }
         }
     c.nco_blk = (g.L.cout + 127) / 128;
-    c.nchunk = Li.Cpad / 64;
+    c.nchunk = std::max(1, Li.Cpad / 64);
     c.ntiles = c.nco_blk * (c.rpack ? 1 : g.L.kh) * c.nchunk;
     int Z = std::max(1, (2 * num_sms() + c.ntiles - 1) / c.ntiles);
     Z = std::min(Z, std::max(1, c.total_boxes / 4));
     Z = std::min(Z, 128);
-    Z = choose_splits(c.total_boxes, c.ntiles, 2.0 * 128 * g.L.kw * 64 * c.BH * c.BNn * 8,
+    Z = choose_splits(c.total_boxes, c.ntiles, 2.0 * 128 * g.L.kw * std::min(64, Li.Cpad) * c.BH * c.BNn * 8,
                           (double)g.L.cout * g.L.kh * g.L.kw * Li.Cpad, Z);
     c.boxes_per_split = (c.total_boxes + Z - 1) / Z;
     c.nsplit = (c.total_boxes + c.boxes_per_split - 1) / c.boxes_per_split;
@@ -2474,7 +2481,7 @@ static int wgrad_zbound(int path, const Level &Li, const LayerGeom &g) {
     const int nco = (g.L.cout + 127) / 128;
     int ntiles;
     if (path == 2) return std::max(1, std::min(296, (2 * num_sms() + nco - 1) / nco));
-    if (path == 1) ntiles = nco * (wgrad_rpack(g) ? 1 : g.L.kh) * (Li.Cpad / 64);
+    if (path == 1) ntiles = nco * (wgrad_rpack(g) ? 1 : g.L.kh) * std::max(1, Li.Cpad / 64);
     else {
         const int cbox = std::min(Li.Cpad, 64), nblocks = g.L.kh * g.L.kw * (Li.Cpad / cbox);
         const int maxb = std::min(WG_MAXBLK, 256 / cbox);
@@ -2643,12 +2650,13 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
             P.Cout = g.L.cout; P.Cpi = Li.Cpad;
             P.rpack = c.rpack;
             // 2-CTA pairs of 128-channel output blocks when the channels pair up
-            const bool cta2 = g.L.cout % 256 == 0;
+            const bool cta2 = g.L.cout % 256 == 0 && Li.Cpad % 64 == 0;
             if (cta2) P.ntiles = c.ntiles / 2;
             const int Wp = 8 + g.L.kw - 1;
+            P.xrow = cta2 ? 64u : (uint32_t)std::min(Li.Cpad, 64) * 2u;
             const uint32_t a_stage = (g.L.cout <= 64 && !c.rpack ? 1u : 2u) * c.BH * c.BNn * 8u * 128u;
             const int xh = c.rpack ? c.BH + g.L.kh - 1 : c.BH;
-            const uint32_t b_stage = ((uint32_t)Wp * xh * c.BNn * (cta2 ? 64u : 128u) + 1023u) & ~1023u;
+            const uint32_t b_stage = ((uint32_t)Wp * xh * c.BNn * P.xrow + 1023u) & ~1023u;
             const uint32_t stage_bytes = a_stage + b_stage;
             P.stages = std::min<int>(8, (int)((200u * 1024u) / stage_bytes));
             P.tmem_cols = c.rpack ? 512 : 256;
@@ -2680,10 +2688,10 @@ splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const L
                     void *base = (char *)x + Li.offset(i, j) * 2;
                     cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)wp, (cuuint64_t)hp, (cuuint64_t)Li.N};
                     cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)wp * C * 2, (cuuint64_t)hp * wp * C * 2};
-                    cuuint32_t box[4] = {cta2 ? 32u : 64u, (cuuint32_t)Wp, (cuuint32_t)xh, (cuuint32_t)c.BNn};
+                    cuuint32_t box[4] = {P.xrow / 2u, (cuuint32_t)Wp, (cuuint32_t)xh, (cuuint32_t)c.BNn};
                     cuuint32_t es[4] = {1, 1, 1, 1};
                     if (encode(&P.mapX[ql], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides, box, es,
-                               CU_TENSOR_MAP_INTERLEAVE_NONE, cta2 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B,
+                               CU_TENSOR_MAP_INTERLEAVE_NONE, swz_for((int)P.xrow),
                                CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
                         return fail(SPLITCNN_ERR_CUDA, "cuTensorMapEncodeTiled(X halo) failed");
                 }

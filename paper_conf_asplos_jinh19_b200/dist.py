@@ -312,7 +312,7 @@ class DistResNet:
     parameter gradients are already global)."""
 
     def __init__(self, c: dict, world: int, rank: int, dtype: int = sc.BF16, bn: bool = False, device="cuda",
-                 group=None, stem_pad: int = 64):
+                 group=None, stem_pad: int = 16):
         from .resnet import ResBNSplitNet, ResSplitNet
         self.world, self.rank, self.dtype, self.group = world, rank, dtype, group
         nh, nw = c["split"]

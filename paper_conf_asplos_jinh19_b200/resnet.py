@@ -69,7 +69,7 @@ def s2d_stem_grad(dWp: torch.Tensor, cin: int) -> torch.Tensor:
 class ResSplitNet(SplitNet):
     def __init__(self, chain: list[dict], blocks: list[dict], N: int, C: int, H: int, W: int, split=(2, 2),
                  dtype: int = sc.BF16, device="cuda", force_simt: bool = False, s2d_stem: bool | None = None,
-                 stem_pad: int = 64, **kw):
+                 stem_pad: int = 16, **kw):
         self.blocks = blocks
         self.block_at = {b["a"]: k for k, b in enumerate(blocks)}
         st = chain[0]
@@ -80,8 +80,9 @@ class ResSplitNet(SplitNet):
         self.s2d = ok if s2d_stem is None else (s2d_stem and ok)
         self.stem_cin = st["cin"]
         if self.s2d:
-            # stem_pad 64: the 12 real channels padded to 64 take the halo / 2-CTA kernels (5.3x the MMA
-            # work of the 7x7 layer, counted as the 7x7 work); 16: the per-tap 16-channel path
+            # stem_pad 16 (default): the 12 real channels in 16 take the narrow-row halo kernels (forward:
+            # one x4 MMA issue per kernel row; weight gradient: SW32 MN-major X); 64: the 64-channel halo /
+            # 2-CTA kernels on zero channels (5.3x the MMA work of the 7x7 layer, counted as the 7x7 work)
             stem = s2d_stem_layer(st, stem_pad)
             chain = [stem] + list(chain[1:])
             C, H, W = stem["cin"], H // 2, W // 2

@@ -1,7 +1,7 @@
 #!/bin/bash
-O=gpurun_out/ab_hn
+O=gpurun_out/ab_hn22
 mkdir -p $O
-timeout 600 python -m pytest tests/test_gpu_ops.py tests/test_gpu_resnet.py tests/test_gpu_bn.py -q -x > $O/tests.txt 2>&1
+timeout 900 python -m pytest tests/test_gpu_ops.py tests/test_gpu_resnet.py tests/test_gpu_bn.py tests/test_gpu_fullsize.py -q -x > $O/tests.txt 2>&1
 for SP in 16 64; do
 timeout 300 python bench.py --config C3 --steps 10 --warmup 3 --no-cpu-baseline --stem-pad $SP --per-layer > $O/C3_pad$SP.json 2>/dev/null
 done

@@ -227,11 +227,15 @@ def run_ours(args):
                         "cap_gb": round(stats["cap_bytes"] / 1e9, 3),
                         "no_offload_ms_per_step": round(ms_plain, 3),
                         "no_offload_peak_gb": round(peak_plain / 1e9, 2)}
-    use_graph = args.graph if args.graph is not None else (args.config in ("C1", "C2") and world == 1)
+    # default: one CUDA graph per step wherever the plan is static (even split; C4 draws new boundaries
+    # every step) on one process: C1/C2 are launch-bound, C3 gains 5 % (2.97 vs 3.12 ms), C5 is neutral
+    # device-side and gains on the e2e path (profiles/r2_ab_graph.txt)
+    use_graph = args.graph if args.graph is not None else (
+        args.config in ("C1", "C2", "C3", "C5") and world == 1 and not args.force_dist)
     graph = None
     if use_graph:
-        # small configs are launch-bound: capture one whole step (every library call enqueues on the
-        # current stream, the db side stream joins back) and replay it; the plan is static (even split)
+        # capture one whole step (every library call enqueues on the current stream, the db side stream
+        # joins back) and replay it
         side = torch.cuda.Stream()
         side.wait_stream(stream)
         with torch.cuda.stream(side):

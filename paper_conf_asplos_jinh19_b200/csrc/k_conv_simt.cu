@@ -268,6 +268,43 @@ __global__ void __launch_bounds__(256) reduce_partials_kernel(const float *__res
     }
 }
 
+// Few partials (Z <= 8, e.g. the single-split weight gradients of the small-M CIFAR tails): one thread per
+// vector column sums its Z partials in z order, grid-stride -- the 8-warp z split above would leave all but
+// Z warps idle and launch one block per 32 columns.  Bitwise equal to it: both compute
+// ((0 + p_0) + p_1) + ... + beta * out, and a sum started at +0 is never -0, so its + 0 terms change nothing.
+template <int VEC>
+__global__ void __launch_bounds__(256) reduce_few_kernel(const float *__restrict__ part0, int64_t n0,
+                                                         float *__restrict__ out0, int Z0,
+                                                         const float *__restrict__ part1, int64_t n1,
+                                                         float *__restrict__ out1, int Z1, float beta) {
+    using V = typename std::conditional<VEC == 4, float4, float>::type;
+    const int Z = blockIdx.y ? Z1 : Z0;
+    const float *part = blockIdx.y ? part1 : part0;
+    float *out = blockIdx.y ? out1 : out0;
+    const int64_t nv = (blockIdx.y ? n1 : n0) / VEC;
+    for (int64_t col = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; col < nv; col += (int64_t)gridDim.x * blockDim.x) {
+        const V *pv = reinterpret_cast<const V *>(part) + col;
+        V t;
+        float *tf = reinterpret_cast<float *>(&t);
+#pragma unroll
+        for (int e = 0; e < VEC; ++e) tf[e] = 0.f;
+        for (int z = 0; z < Z; ++z) {
+            const V a = __ldg(pv + (int64_t)z * nv);
+            const float *af = reinterpret_cast<const float *>(&a);
+#pragma unroll
+            for (int e = 0; e < VEC; ++e) tf[e] += af[e];
+        }
+        V *ov = reinterpret_cast<V *>(out) + col;
+        if (beta != 0.f) {
+            const V o = *ov;
+            const float *of = reinterpret_cast<const float *>(&o);
+#pragma unroll
+            for (int e = 0; e < VEC; ++e) tf[e] += beta * of[e];
+        }
+        *ov = t;
+    }
+}
+
 // Column sums of the patch-buffer range [p0, p1) viewed as a [P pixels][Cpad] matrix (the patches of
 // a range are contiguous): block b sums rows [b*R, (b+1)*R) with 16-byte loads, reduces its pixel
 // lanes in shared memory in a fixed order and writes part[b][Cout].  Deterministic.
@@ -383,12 +420,17 @@ int launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, flo
         count_launch();
         return nch;
     }
+    // small dY (< 32 MB, the CIFAR-sized levels): at most 64 partial rows of >= 128 pixels each -- one row
+    // per block of a few pixels would leave the (serial-in-z) reduction of ~600 partials as the long pole
+    int64_t Rs = R;
+    if (dy_bytes < (32ll << 20)) Rs = std::max<int64_t>({R, 128, (P + 63) / 64});
+    const int Zs = (int)((P + Rs - 1) / Rs);
     if (dt == SPLITCNN_BF16)
-        colsum_kernel<__nv_bfloat16><<<Zr, 256, 0, st>>>((const __nv_bfloat16 *)dy + e0, P, Lo.Cpad, cout, R, part);
+        colsum_kernel<__nv_bfloat16><<<Zs, 256, 0, st>>>((const __nv_bfloat16 *)dy + e0, P, Lo.Cpad, cout, Rs, part);
     else
-        colsum_kernel<float><<<Zr, 256, 0, st>>>((const float *)dy + e0, P, Lo.Cpad, cout, R, part);
+        colsum_kernel<float><<<Zs, 256, 0, st>>>((const float *)dy + e0, P, Lo.Cpad, cout, Rs, part);
     count_launch();
-    return Zr;
+    return Zs;
 }
 
 void launch_reduce2(const float *part0, int64_t n0, float *out0, int Z0, const float *part1, int64_t n1, float *out1,
@@ -397,6 +439,13 @@ void launch_reduce2(const float *part0, int64_t n0, float *out0, int Z0, const f
     auto al16 = [](const void *q) { return ((uintptr_t)q & 15) == 0; };
     const bool vec = n0 % 4 == 0 && n1 % 4 == 0 && al16(part0) && al16(out0) && (n1 == 0 || (al16(part1) && al16(out1)));
     const int64_t cols = std::max(n0, n1) / (vec ? 4 : 1);
+    if (std::max(Z0, n1 > 0 ? Z1 : 0) <= 8) {
+        dim3 grid((unsigned)std::max<int64_t>(1, std::min<int64_t>((cols + 255) / 256, 148 * 16)), n1 > 0 ? 2 : 1);
+        if (vec) reduce_few_kernel<4><<<grid, 256, 0, st>>>(part0, n0, out0, Z0, part1, n1, out1, Z1, beta);
+        else reduce_few_kernel<1><<<grid, 256, 0, st>>>(part0, n0, out0, Z0, part1, n1, out1, Z1, beta);
+        count_launch();
+        return;
+    }
     dim3 grid((unsigned)((cols + 31) / 32), n1 > 0 ? 2 : 1);
     if (vec) reduce_partials_kernel<4><<<grid, 256, 0, st>>>(part0, n0, out0, Z0, part1, n1, out1, Z1, beta);
     else reduce_partials_kernel<1><<<grid, 256, 0, st>>>(part0, n0, out0, Z0, part1, n1, out1, Z1, beta);

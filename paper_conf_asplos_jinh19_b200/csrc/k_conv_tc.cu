@@ -169,6 +169,30 @@ __device__ __forceinline__ void get_tile(const TcConvParams &p, int t, uint32_t 
 // producer warp, MMA warp, 8 epilogue warps (2 per TMEM lane quadrant), a second MMA warp (dual issue)
 constexpr int CONV_THREADS = 64 + 256 + 32;
 
+// packed epilogue arithmetic (the epilogue warps are issue-latency bound on the narrow-N layers: every
+// instruction per column shows): two fp32 adds per FADD2, ReLU fused into the bf16x2 rounding (F2FP.RELU:
+// round-to-nearest then clamp at 0 == round(max(x, 0)) for every non-NaN x), the dgrad ReLU mask applied
+// to the ROUNDED pair as a bitwise select (bf16(0) = +0, so masking after rounding is bit-identical)
+__device__ __forceinline__ void add2(float &a, float &b, float c, float d) {
+    uint64_t x = ((uint64_t)__float_as_uint(b) << 32) | __float_as_uint(a);
+    const uint64_t y = ((uint64_t)__float_as_uint(d) << 32) | __float_as_uint(c);
+    asm("add.rn.f32x2 %0, %0, %1;" : "+l"(x) : "l"(y));
+    a = __uint_as_float((uint32_t)x);
+    b = __uint_as_float((uint32_t)(x >> 32));
+}
+template <bool RELU>
+__device__ __forceinline__ uint32_t pack_bf16x2(float lo, float hi) {
+    uint32_t r;
+    if (RELU) asm("cvt.rn.relu.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+    else asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+    return r;
+}
+// bf16x2 word m -> 0xFFFF per half where that half is > 0 (NaN / zero / negative: 0)
+__device__ __forceinline__ uint32_t pos_mask2(uint32_t m) {
+    const uint32_t z = 0u;
+    return __hgt2_mask(*reinterpret_cast<const __nv_bfloat162 *>(&m), *reinterpret_cast<const __nv_bfloat162 *>(&z));
+}
+
 // 8 accumulator columns (all real channels) -> bf16x8: +bias, ReLU, dgrad ReLU mask
 template <bool BIAS, bool RELU, bool MASK>
 __device__ __forceinline__ uint4 epi8_full(const uint32_t *r, const float *sb, uint4 m4, bool res = false) {
@@ -178,36 +202,25 @@ __device__ __forceinline__ uint4 epi8_full(const uint32_t *r, const float *sb, u
     if (BIAS) {
         const float4 b0 = *reinterpret_cast<const float4 *>(sb);
         const float4 b1 = *reinterpret_cast<const float4 *>(sb + 4);
-        o[0] += b0.x; o[1] += b0.y; o[2] += b0.z; o[3] += b0.w;
-        o[4] += b1.x; o[5] += b1.y; o[6] += b1.z; o[7] += b1.w;
+        add2(o[0], o[1], b0.x, b0.y); add2(o[2], o[3], b0.z, b0.w);
+        add2(o[4], o[5], b1.x, b1.y); add2(o[6], o[7], b1.z, b1.w);
     }
     if (MASK && res) {   // residual join fused into the forward epilogue: the tile holds the shortcut
         const __nv_bfloat162 *mh = reinterpret_cast<const __nv_bfloat162 *>(&m4);
 #pragma unroll
         for (int e = 0; e < 4; ++e) {
             const float2 mf = __bfloat1622float2(mh[e]);
-            o[2 * e] += mf.x;
-            o[2 * e + 1] += mf.y;
+            add2(o[2 * e], o[2 * e + 1], mf.x, mf.y);
         }
     }
-    if (RELU) {
+    uint32_t w[4];
 #pragma unroll
-        for (int e = 0; e < 8; ++e) o[e] = fmaxf(o[e], 0.f);
-    }
+    for (int e = 0; e < 4; ++e) w[e] = pack_bf16x2<RELU>(o[2 * e], o[2 * e + 1]);
     if (MASK && !res) {
-        const __nv_bfloat162 *mh = reinterpret_cast<const __nv_bfloat162 *>(&m4);
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-            const float2 mf = __bfloat1622float2(mh[e]);
-            o[2 * e] = mf.x > 0.f ? o[2 * e] : 0.f;
-            o[2 * e + 1] = mf.y > 0.f ? o[2 * e + 1] : 0.f;
-        }
+        w[0] &= pos_mask2(m4.x); w[1] &= pos_mask2(m4.y);
+        w[2] &= pos_mask2(m4.z); w[3] &= pos_mask2(m4.w);
     }
-    uint4 pk;
-    __nv_bfloat162 *h2 = reinterpret_cast<__nv_bfloat162 *>(&pk);
-#pragma unroll
-    for (int e = 0; e < 4; ++e) h2[e] = __floats2bfloat162_rn(o[2 * e], o[2 * e + 1]);
-    return pk;
+    return make_uint4(w[0], w[1], w[2], w[3]);
 }
 
 // 8 accumulator columns -> bf16x8 with the fused epilogue (bias, ReLU, or the dgrad ReLU mask)
@@ -220,8 +233,8 @@ __device__ __forceinline__ uint4 epi8(const uint32_t *r, const float *sb, int co
         if (BIAS) {
             const float4 b0 = *reinterpret_cast<const float4 *>(sb + co);
             const float4 b1 = *reinterpret_cast<const float4 *>(sb + co + 4);
-            o[0] += b0.x; o[1] += b0.y; o[2] += b0.z; o[3] += b0.w;
-            o[4] += b1.x; o[5] += b1.y; o[6] += b1.z; o[7] += b1.w;
+            add2(o[0], o[1], b0.x, b0.y); add2(o[2], o[3], b0.z, b0.w);
+            add2(o[4], o[5], b1.x, b1.y); add2(o[6], o[7], b1.z, b1.w);
         }
     } else {
 #pragma unroll
@@ -232,28 +245,17 @@ __device__ __forceinline__ uint4 epi8(const uint32_t *r, const float *sb, int co
 #pragma unroll
         for (int e = 0; e < 4; ++e) {
             const float2 mf = __bfloat1622float2(mh[e]);
-            o[2 * e] += mf.x;
-            o[2 * e + 1] += mf.y;
+            add2(o[2 * e], o[2 * e + 1], mf.x, mf.y);
         }
     }
-    if (RELU) {
+    uint32_t w[4];
 #pragma unroll
-        for (int e = 0; e < 8; ++e) o[e] = fmaxf(o[e], 0.f);
-    }
+    for (int e = 0; e < 4; ++e) w[e] = pack_bf16x2<RELU>(o[2 * e], o[2 * e + 1]);
     if (MASK && !res) {
-        const __nv_bfloat162 *mh = reinterpret_cast<const __nv_bfloat162 *>(&m4);
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-            const float2 mf = __bfloat1622float2(mh[e]);
-            o[2 * e] = mf.x > 0.f ? o[2 * e] : 0.f;
-            o[2 * e + 1] = mf.y > 0.f ? o[2 * e + 1] : 0.f;
-        }
+        w[0] &= pos_mask2(m4.x); w[1] &= pos_mask2(m4.y);
+        w[2] &= pos_mask2(m4.z); w[3] &= pos_mask2(m4.w);
     }
-    uint4 pk;
-    __nv_bfloat162 *h2 = reinterpret_cast<__nv_bfloat162 *>(&pk);
-#pragma unroll
-    for (int e = 0; e < 4; ++e) h2[e] = __floats2bfloat162_rn(o[2 * e], o[2 * e + 1]);
-    return pk;
+    return make_uint4(w[0], w[1], w[2], w[3]);
 }
 
 // Fused 2x2 / stride-2 max-pool of 16 accumulator columns (pool semantics of
@@ -320,18 +322,14 @@ __device__ __forceinline__ void pool32(const uint32_t *w, int bw, bool writer, _
     uint4 *y4 = reinterpret_cast<uint4 *>(yp);
 #pragma unroll
     for (int q = 0; q < 4; ++q) y4[q] = make_uint4(best[4 * q], best[4 * q + 1], best[4 * q + 2], best[4 * q + 3]);
+    // argmax byte per element: window index (bits 0-1, already at bits 0-1 / 16-17 of amask) | [max > 0] << 7,
+    // two elements per word in bytes 0 and 2, then two words' bytes interleaved into four by one PRMT
     uint32_t ab[8];
 #pragma unroll
     for (int q = 0; q < 8; ++q) {
-        uint32_t v = 0;
-#pragma unroll
-        for (int h = 0; h < 2; ++h) {
-            const uint32_t wd = best[2 * q + h], am = amask[2 * q + h];
-            const uint32_t lo = (am & 3u) | ((wd & 0x7FFFu) ? 0x80u : 0u);            // element 2(2q+h)
-            const uint32_t hi = ((am >> 16) & 3u) | ((wd & 0x7FFF0000u) ? 0x80u : 0u); // element 2(2q+h)+1
-            v |= (lo | (hi << 8)) << (16 * h);
-        }
-        ab[q] = v;
+        const uint32_t v0 = amask[2 * q] | (pos_mask2(best[2 * q]) & 0x00800080u);
+        const uint32_t v1 = amask[2 * q + 1] | (pos_mask2(best[2 * q + 1]) & 0x00800080u);
+        ab[q] = __byte_perm(v0, v1, 0x6420);
     }
     reinterpret_cast<uint4 *>(ap)[0] = make_uint4(ab[0], ab[1], ab[2], ab[3]);
     reinterpret_cast<uint4 *>(ap)[1] = make_uint4(ab[4], ab[5], ab[6], ab[7]);
@@ -374,6 +372,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
         tc::mbar_init(ybar, 1);
         tc::mbar_init(wbar, 1);
         tc::mbar_init(wbar + 1, 1);   // group 1's mask barrier
+        uint64_t *mbarR = reinterpret_cast<uint64_t *>(smem + p.bar_off + 256);   // mask ring: 4 slots x 2 groups
+        for (int r = 0; r < 8; ++r) tc::mbar_init(&mbarR[r], 1);
         tc::fence_barrier_init();
     }
     if (BIAS)
@@ -572,11 +572,14 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             if (p.bres && leader) tc::mbar_wait(wbar, 0);
             // this warp cycles through two accumulator slots: 0, 1 (one issuer: tile it -> epilogue group
             // it & 1) or 2q, 2q + 1 (dual: warp q's tiles all go to group q, which alternates its two)
-            const int sbase = p.dual ? 2 * q : 0;
-            int acc = 0;
-            uint32_t aph = 0;
-            for (int t = leader ? tfirst + q * tstep : total; t < total; t += istep * tstep) {
-                const int slot = sbase + acc;
+            // tile ordinal it of this CTA -> epilogue group it & 1, that group's k = it >> 1-th tile -> slot
+            // g * nacc_g + (k & 1) with nacc_g accumulators per group (2: the MMA runs two tiles of a group
+            // ahead of its epilogue; also with one issuer)
+            int it = q;
+            for (int t = leader ? tfirst + q * tstep : total; t < total; t += istep * tstep, it += istep) {
+                const int kg = it >> 1;
+                const int slot = (it & 1) * p.nacc_g + (p.nacc_g == 2 ? (kg & 1) : 0);
+                const uint32_t aph = (uint32_t)((p.nacc_g == 2 ? (kg >> 1) : kg) & 1);
                 tc::mbar_wait(&tempty[slot], aph ^ 1);
                 tc::tc_fence_after();
                 const uint32_t d = tmem_base + (uint32_t)(slot * p.BN);
@@ -697,8 +700,6 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                 }
                 if (CTA2) tc::mma2_commit_mc_ws(&tfull[slot]);
                 else tc::mma_commit_ws(&tfull[slot]);
-                acc ^= 1;
-                if (acc == 0) aph ^= 1;
             }
         };
         if (warp == 1) mma_run(std::integral_constant<int, 0>{});
@@ -714,36 +715,46 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
         const int gtid = threadIdx.x - 64 - 128 * g;   // 0..127 within the group
         const uint32_t rowB = (uint32_t)p.ychunk * 2u;
         const uint32_t chunk_bytes = 128u * rowB;
-        uint64_t *mbar = g ? wbar + 1 : ybar;
-        uint32_t yph = 0;
-        // ReLU-mask tiles (dgrad) with a staging ring: tile k+1's mask is loaded into its ring buffer as soon
-        // as tile k's store is issued, so the load latency overlaps tile k+1's MMAs instead of following them
+        // ReLU-mask / residual tiles (dgrad mask, fused join) through the staging ring: ring slot s has its own
+        // barrier, and the tile that will use slot s is loaded as soon as the TMA store that last read slot s
+        // is done -- yring - 1 group tiles ahead, so the load latency hides behind that many tiles' MMAs
+        // (one tile ahead left the short-K 64-channel layers waiting on every mask: conv1_2 dgrad)
+        uint64_t *mbarR = reinterpret_cast<uint64_t *>(smem + p.bar_off + 256) + 4 * g;
+        uint32_t mph = 0;   // phase bit per ring slot
         const bool mpre = MASK && p.yring >= 2;
-        auto mask_load = [&](int tt, uint8_t *buf) {   // gtid 0
+        auto mask_load = [&](int tt, int slot) {   // gtid 0
             int ql, nb, hb, wb, cb;
             bool valid;
             get_tile(p, tt, rank, ql, nb, hb, wb, cb, valid);
             if (!valid) return;
-            const int co0 = cb * p.BN, nch = min(p.BN, p.Cpo - co0) / p.ychunk;
-            tc::mbar_arrive_expect_tx(mbar, (uint32_t)nch * p.rows_box * rowB);
+            const int co0 = cb * p.BN, nch = min(p.BN, p.Cpo - co0) >> p.ysh;
+            uint8_t *buf = sY + (size_t)(g * p.yring + slot) * p.ybuf_bytes;
+            tc::mbar_arrive_expect_tx(&mbarR[slot], (uint32_t)nch * p.rows_box * rowB);
             for (int c = 0; c < nch; ++c)
-                tc::tma_load_4d(buf + c * chunk_bytes, &p.mapR[ql], mbar, co0 + c * p.ychunk, wb * p.BW, hb * p.BH, nb * p.BNn);
+                tc::tma_load_4d(buf + c * chunk_bytes, &p.mapR[ql], &mbarR[slot], co0 + c * p.ychunk, wb * p.BW, hb * p.BH,
+                                nb * p.BNn);
         };
-        if (mpre && gtid == 0 && tfirst + g * tstep < total) mask_load(tfirst + g * tstep, sY + (size_t)(g * p.yring) * p.ybuf_bytes);
-        int it = g, k = 0;
-        for (int t = tfirst + g * tstep; t < total; t += 2 * tstep, it += 2, ++k) {
+        if (mpre && gtid == 0)
+            for (int j = 0; j < p.yring - 1; ++j) {
+                const int tt = tfirst + (g + 2 * j) * tstep;
+                if (tt < total) mask_load(tt, j);
+            }
+        uint64_t *mbar = g ? wbar + 1 : ybar;   // mask without the ring (yring == 1): loaded per tile
+        uint32_t yph = 0;
+        int it = g, k = 0, ys = 0;   // ys = k % yring (no runtime modulo per tile)
+        for (int t = tfirst + g * tstep; t < total; t += 2 * tstep, it += 2, ++k, ys = (ys + 1 == p.yring) ? 0 : ys + 1) {
             const int slot = g * p.nacc_g + (p.nacc_g == 2 ? (k & 1) : 0);
             const uint32_t aph = (uint32_t)((p.nacc_g == 2 ? (k >> 1) : k) & 1);
             const uint32_t tempty_l = tc::mapa_shared(&tempty[slot], 0);   // the leader's (own in 1-CTA mode)
             // staging ring: tile k of this group fills buffer k % yring
-            uint8_t *sYb = sY + (size_t)(g * p.yring + k % p.yring) * p.ybuf_bytes;
+            uint8_t *sYb = sY + (size_t)(g * p.yring + ys) * p.ybuf_bytes;
             int ql, nb, hb, wb, cb;
             bool valid;
             get_tile(p, t, rank, ql, nb, hb, wb, cb, valid);
             const int co0 = cb * p.BN;
             const int ow0 = wb * p.BW, oh0 = hb * p.BH, n0 = nb * p.BNn;
             const int ncols = min(p.BN, p.Cpo - co0);
-            const int nchunks = ncols / p.ychunk;
+            const int nchunks = ncols >> p.ysh;
             if (POOL) {
                 // pooled outputs straight from registers: no staging tile, no store of the conv output
                 tc::mbar_wait(&tfull[slot], aph);
@@ -798,8 +809,8 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
             }
             tc::named_bar_sync(1 + g, 128);
             if (mpre && valid) {
-                tc::mbar_wait(mbar, yph);
-                yph ^= 1;
+                tc::mbar_wait(&mbarR[ys], (mph >> ys) & 1u);
+                mph ^= 1u << ys;
             } else if (MASK && valid) {
                 if (gtid == 0) {
                     tc::mbar_arrive_expect_tx(mbar, (uint32_t)nchunks * p.rows_box * rowB);
@@ -861,12 +872,14 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
                     for (int c = 0; c < nchunks; ++c)
                         tc::tma_store_4d(&p.mapY[ql], sYb + c * chunk_bytes, co0 + c * p.ychunk, ow0, oh0, n0);
                 tc::bulk_commit();
-                if (mpre && t + 2 * tstep < total) {
-                    // the next tile's buffer was last read by the store yring - 1 tiles before this one
-                    if (p.yring == 2) tc::bulk_wait_read1();
-                    else if (p.yring == 3) tc::bulk_wait_read2();
-                    else tc::bulk_wait_read3();
-                    mask_load(t + 2 * tstep, sY + (size_t)(g * p.yring + (k + 1) % p.yring) * p.ybuf_bytes);
+                if (mpre) {
+                    // tile k + yring - 1 of this group takes the slot of tile k - 1, whose store has read it once
+                    // at most the latest bulk group (this tile's store) is still reading
+                    const int tt = t + 2 * tstep * (p.yring - 1);
+                    if (tt < total) {
+                        tc::bulk_wait_read1();
+                        mask_load(tt, ys == 0 ? p.yring - 1 : ys - 1);
+                    }
                 }
             }
         }
@@ -1079,17 +1092,23 @@ __global__ void flip_weights_kernel(const T *__restrict__ W, T *__restrict__ Wt,
                                     int Cpad_in, int Cin, int kh, int kw, int Cpad_out, int r0h, int r0w, int step,
                                     int nth, int ntw) {
     // Wt[ci][j][l][co] = W[co][r0h + step*(nth-1-j)][r0w + step*(ntw-1-l)][ci]   (stride-1 dgrad: r0 = 0,
-    // step = 1, nt = k -- the 180-degree flip; stride-s phase (rho_h, rho_w): the taps r = r0 (mod s))
-    const int64_t n = (int64_t)Cin * nth * ntw * Cpad_out;
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        const int co = (int)(i % Cpad_out);
-        int64_t t = i / Cpad_out;
-        const int c = (int)(t % ntw);
-        t /= ntw;
-        const int r = (int)(t % nth);
-        const int ci = (int)(t / nth);
-        const int rr = r0h + step * (nth - 1 - r), cc = r0w + step * (ntw - 1 - c);
-        Wt[i] = co < Cout ? W[(((int64_t)co * kh + rr) * kw + cc) * Cpad_in + ci] : from_f<T>(0.f);
+    // step = 1, nt = k -- the 180-degree flip; stride-s phase (rho_h, rho_w): the taps r = r0 (mod s)).
+    // Per tap a (Cout x Cin) -> (Cin x Cpad_out) transpose through a 32 x 32 shared tile: both the reads
+    // (ci contiguous) and the writes (co contiguous) coalesced.  grid (Cin/32, Cpad_out/32, nth*ntw).
+    __shared__ T tile[32][33];
+    const int tap = blockIdx.z, j = tap / ntw, l = tap - j * ntw;
+    const int rr = r0h + step * (nth - 1 - j), cc = r0w + step * (ntw - 1 - l);
+    const int ci0 = blockIdx.x * 32, co0 = blockIdx.y * 32;
+    for (int k = threadIdx.y; k < 32; k += 8) {
+        const int co = co0 + k, ci = ci0 + threadIdx.x;
+        T v = from_f<T>(0.f);
+        if (co < Cout && ci < Cin) v = W[(((int64_t)co * kh + rr) * kw + cc) * Cpad_in + ci];
+        tile[k][threadIdx.x] = v;
+    }
+    __syncthreads();
+    for (int k = threadIdx.y; k < 32; k += 8) {
+        const int ci = ci0 + k, co = co0 + threadIdx.x;
+        if (ci < Cin && co < Cpad_out) Wt[(((int64_t)ci * nth + j) * ntw + l) * Cpad_out + co] = tile[threadIdx.x][k];
     }
 }
 
@@ -1228,6 +1247,11 @@ TileShape choose_tile_pool(const std::vector<std::pair<int, int>> &ext, int N) {
 }
 
 int round_up16(int x) { return (x + 15) / 16 * 16; }
+
+// stages + resident weights + staging ring of the conv kernel (of the 227 KB opt-in shared memory; 220 KB
+// -- a 3-deep mask ring for the 64-channel dgrad -- measured no faster there and 5 % slower on the fused
+// conv1_2 + pool forward, profiles/r2i/ab_epilogue.txt)
+constexpr uint32_t CONV_SMEM_BUDGET = 210u * 1024u;
 
 bool a_channels_ok(int cpad) { return cpad == 8 || cpad == 16 || cpad == 32 || cpad % 64 == 0; }
 
@@ -1426,7 +1450,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         if (P.egroups == 2) {
             const uint32_t min_st = 4;
             for (int r = 4; r >= 2; --r)
-                if (P.bres_bytes + 2u * (uint32_t)r * P.ybuf_bytes + min_st * stage_bytes <= 210u * 1024u) { P.yring = r; break; }
+                if (P.bres_bytes + 2u * (uint32_t)r * P.ybuf_bytes + min_st * stage_bytes <= CONV_SMEM_BUDGET) { P.yring = r; break; }
         }
         // dual MMA issue for accumulators of <= 128 columns (4 of them in TMEM): short-K tiles (not the
         // 8-channel halo forward, whose 5-MMA tiles are store-bound: in the C5 step dual issue costs it 9 %)
@@ -1434,7 +1458,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         P.nacc_g = P.dual ? 2 : 1;
         // the fused pool epilogue stores from registers: no staging tiles
         const uint32_t staging = pool ? 0u : (P.egroups == 2 ? 2u * (uint32_t)P.yring : (uint32_t)P.ybufs) * P.ybuf_bytes;
-        P.stages = std::min<int>(8, (int)((210u * 1024u - staging - P.bres_bytes) / stage_bytes));
+        P.stages = std::min<int>(8, (int)((CONV_SMEM_BUDGET - staging - P.bres_bytes) / stage_bytes));
         // dual issue splits the stages into two rings: only with >= 2 stages per ring
         if (P.stages < 4) { P.dual = 0; P.nacc_g = 1; }
         P.bres_off = (uint32_t)P.stages * stage_bytes;
@@ -1567,6 +1591,7 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         }
         if (tiles == 0) continue;
         const size_t smem = 1024 + (size_t)P.bar_off + 512 + (bias ? 4 * (size_t)g.L.cout : 0) + 64;
+        if (smem > 227u * 1024u) return fail(SPLITCNN_ERR_UNSUPPORTED, "conv: shared-memory plan exceeds 227 KB");
         const int grid = P.cta2 ? 2 * std::min(P.total_pairs, num_sms() / 2) : std::min(tiles, num_sms());
         // dual issue halves the stage ring a tile sees: only where a CTA has many tiles to overlap
         const long per_cta = P.cta2 ? ((long)P.total_pairs + grid / 2 - 1) / (grid / 2) : ((long)tiles + grid - 1) / grid;
@@ -1747,8 +1772,8 @@ splitcnn_status_t launch_conv_pool_fwd_tc(const Level &Li, const Level &Lo, cons
 template <typename T>
 static void flip_weights(const void *w, void *wt, const LayerGeom &g, int cpad_in, int cpad_out, int r0h, int r0w,
                          int step, int nth, int ntw, cudaStream_t st) {
-    const int64_t n = (int64_t)g.L.cin * nth * ntw * cpad_out;
-    flip_weights_kernel<T><<<(unsigned)std::min<int64_t>((n + 255) / 256, 2048), 256, 0, st>>>(
+    const dim3 grid((unsigned)((g.L.cin + 31) / 32), (unsigned)((cpad_out + 31) / 32), (unsigned)(nth * ntw));
+    flip_weights_kernel<T><<<grid, dim3(32, 8), 0, st>>>(
         (const T *)w, (T *)wt, g.L.cout, cpad_in, g.L.cin, g.L.kh, g.L.kw, cpad_out, r0h, r0w, step, nth, ntw);
     count_launch();
 }

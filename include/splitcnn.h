@@ -102,6 +102,9 @@ typedef enum {
 #define SPLITCNN_FLAG_POOL_RELU_MASK 0x2u  /* pool_fwd: record [max > 0] in argmax bit 7;
                                               pool_bwd: multiply dX by that bit (the backward
                                               of the ReLU feeding the pool)          */
+#define SPLITCNN_FLAG_DGRAD_WEIGHTS 0x4u   /* conv_bwd_data: `w` is the prepared buffer written by
+                                              splitcnn_conv_dgrad_weights (no flip inside the call, ws unused);
+                                              ERR_INVALID_VALUE where that buffer's size is 0 */
 #define SPLITCNN_FLAG_FORCE_SIMT 0x100u    /* conv calls: use the CUDA-core kernels even where
                                               the tcgen05 kernel applies (testing)          */
 
@@ -266,6 +269,22 @@ SPLITCNN_API splitcnn_status_t splitcnn_conv_bwd_data(splitcnn_plan_t plan, int3
                                          const void *dy, const void *w, void *dx, const void *relu_src,
                                          void *ws, size_t ws_bytes, uint32_t flags,
                                          int32_t p0, int32_t p1, splitcnn_stream_t stream);
+
+/* Dgrad-ready weights, built once per weight version instead of inside every conv_bwd_data call (e.g. on a
+ * side stream during the forward pass, off the backward's critical path).  Same arithmetic as the flip the
+ * data gradient does in its workspace (the adjoint of Eq. 6): stride 1 the 180-degree-
+ * rotated, Cin<->Cout-transposed filter W'[ci][r'][c'][co] = W[co][kh-1-r'][kw-1-c'][ci] (0 for co >= Cout);
+ * stride S one sub-filter per output phase that a tap reaches, 1 KB-aligned one after another.
+ * _size: bytes of that buffer for (layer, dtype) -- 0 where the data gradient takes none (non-BF16 dtypes,
+ * the CUDA-core path); then conv_bwd_data must not get FLAG_DGRAD_WEIGHTS.
+ * _weights: w = the layer's weights (as conv_bwd_data's `w`), wt: device buffer of >= _size bytes, 256-byte
+ * aligned, owned by the caller and read by later conv_bwd_data calls with FLAG_DGRAD_WEIGHTS (stream-ordered:
+ * the caller orders those calls after this one).  Errors: ERR_UNSUPPORTED if _size is 0, ERR_INVALID_VALUE
+ * for null / misaligned pointers or wt_bytes < _size. */
+SPLITCNN_API splitcnn_status_t splitcnn_conv_dgrad_weights_size(splitcnn_plan_t plan, int32_t layer,
+                                                   splitcnn_dtype_t dtype, size_t *bytes);
+SPLITCNN_API splitcnn_status_t splitcnn_conv_dgrad_weights(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                              const void *w, void *wt, size_t wt_bytes, splitcnn_stream_t stream);
 
 /* Weight gradient summed over the patches [p0, p1) and the batch:
  *   dW[co,r,c,ci] = beta * dW + sum_p sum_{n,oh,ow} dY_p[n,oh,ow,co] X~_p[n, oh*sh-pt+r, ow*sw-pl+c, ci]

@@ -305,7 +305,14 @@ extern "C" splitcnn_status_t splitcnn_conv_bwd_data(splitcnn_plan_t plan, int32_
     if (p1 == p0) return SPLITCNN_OK;
     const Level &Li = plan->levels[layer], &Lo = plan->levels[layer + 1];
     const LayerGeom &g = plan->layers[layer];
-    if (!(flags & SPLITCNN_FLAG_FORCE_SIMT) && conv_tc_supported(1, dtype, Li, Lo, g)) {
+    const bool prepared = (flags & SPLITCNN_FLAG_DGRAD_WEIGHTS) != 0;
+    const bool tc = !(flags & SPLITCNN_FLAG_FORCE_SIMT) && conv_tc_supported(1, dtype, Li, Lo, g);
+    if (prepared && !(tc && dtype == SPLITCNN_BF16))
+        return fail(SPLITCNN_ERR_INVALID_VALUE, "conv_bwd_data: FLAG_DGRAD_WEIGHTS where the data gradient takes none "
+                                                "(splitcnn_conv_dgrad_weights_size = 0)");
+    if (prepared) {   // w = splitcnn_conv_dgrad_weights output: no flip, no workspace
+        TRY(launch_conv_dgrad_tc(Li, Lo, g, dy, w, dx, relu_src, nullptr, p0, p1, (cudaStream_t)stream, SPLITCNN_BF16, 0, true));
+    } else if (tc) {
         const bool f32 = dtype != SPLITCNN_BF16;
         const size_t need = f32 ? f32tc_ws_bytes(1, dtype, Li, Lo, g) : conv_tc_ws_bytes(1, Li, Lo, g);
         if (ws_bytes < need || (need && !ws)) return fail(SPLITCNN_ERR_INVALID_VALUE, "conv_bwd_data: workspace too small");
@@ -315,6 +322,30 @@ extern "C" splitcnn_status_t splitcnn_conv_bwd_data(splitcnn_plan_t plan, int32_
         launch_conv_dgrad_simt(dtype, Li, Lo, g, dy, w, dx, relu_src, p0, p1, (cudaStream_t)stream);
     }
     return check_launch("conv_bwd_data");
+}
+
+extern "C" splitcnn_status_t splitcnn_conv_dgrad_weights_size(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                                             size_t *bytes) {
+    TRY(check_layer(plan, layer, SPLITCNN_OP_CONV));
+    TRY(check_dtype(dtype));
+    if (!bytes) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    const Level &Li = plan->levels[layer], &Lo = plan->levels[layer + 1];
+    const LayerGeom &g = plan->layers[layer];
+    *bytes = (dtype == SPLITCNN_BF16 && conv_tc_supported(1, dtype, Li, Lo, g)) ? conv_tc_ws_bytes(1, Li, Lo, g) : 0;
+    return SPLITCNN_OK;
+}
+
+extern "C" splitcnn_status_t splitcnn_conv_dgrad_weights(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,
+                                                        const void *w, void *wt, size_t wt_bytes, splitcnn_stream_t stream) {
+    size_t need = 0;
+    TRY(splitcnn_conv_dgrad_weights_size(plan, layer, dtype, &need));
+    if (need == 0) return fail(SPLITCNN_ERR_UNSUPPORTED, "conv_dgrad_weights: this layer / dtype takes no prepared weights");
+    if (!w || !wt) return fail(SPLITCNN_ERR_INVALID_VALUE, "null pointer");
+    NEED_ALIGNED(w, "w");
+    NEED_ALIGNED(wt, "wt");
+    if (wt_bytes < need) return fail(SPLITCNN_ERR_INVALID_VALUE, "conv_dgrad_weights: wt too small");
+    prep_dgrad_weights_tc(plan->levels[layer], plan->levels[layer + 1], plan->layers[layer], w, wt, (cudaStream_t)stream, 0);
+    return check_launch("conv_dgrad_weights");
 }
 
 extern "C" splitcnn_status_t splitcnn_conv_bwd_filter(splitcnn_plan_t plan, int32_t layer, splitcnn_dtype_t dtype,

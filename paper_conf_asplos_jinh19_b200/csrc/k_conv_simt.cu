@@ -318,6 +318,7 @@ __global__ void __launch_bounds__(256) colsum_kernel(const T *__restrict__ base,
     float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
     const int64_t r0 = blockIdx.x * R, r1 = min(P, r0 + R);
     if (pl < lanes) {
+#pragma unroll 4
         for (int64_t r = r0 + pl; r < r1; r += lanes) {
             float v[8];
             load8(base + r * Cpad + cg * 8, v);
@@ -420,10 +421,10 @@ int launch_db_partials(splitcnn_dtype_t dt, const Level &Lo, const void *dy, flo
         count_launch();
         return nch;
     }
-    // small dY (< 32 MB, the CIFAR-sized levels): at most 64 partial rows of >= 128 pixels each -- one row
+    // small dY (< 32 MB, the CIFAR-sized levels): at most 128 partial rows of >= 64 pixels each -- one row
     // per block of a few pixels would leave the (serial-in-z) reduction of ~600 partials as the long pole
     int64_t Rs = R;
-    if (dy_bytes < (32ll << 20)) Rs = std::max<int64_t>({R, 128, (P + 63) / 64});
+    if (dy_bytes < (32ll << 20)) Rs = std::max<int64_t>({R, 64, (P + 127) / 128});
     const int Zs = (int)((P + Rs - 1) / Rs);
     if (dt == SPLITCNN_BF16)
         colsum_kernel<__nv_bfloat16><<<Zs, 256, 0, st>>>((const __nv_bfloat16 *)dy + e0, P, Lo.Cpad, cout, Rs, part);

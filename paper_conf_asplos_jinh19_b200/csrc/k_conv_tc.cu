@@ -1093,22 +1093,41 @@ __global__ void flip_weights_kernel(const T *__restrict__ W, T *__restrict__ Wt,
                                     int nth, int ntw) {
     // Wt[ci][j][l][co] = W[co][r0h + step*(nth-1-j)][r0w + step*(ntw-1-l)][ci]   (stride-1 dgrad: r0 = 0,
     // step = 1, nt = k -- the 180-degree flip; stride-s phase (rho_h, rho_w): the taps r = r0 (mod s)).
-    // Per tap a (Cout x Cin) -> (Cin x Cpad_out) transpose through a 32 x 32 shared tile: both the reads
-    // (ci contiguous) and the writes (co contiguous) coalesced.  grid (Cin/32, Cpad_out/32, nth*ntw).
-    __shared__ T tile[32][33];
-    const int tap = blockIdx.z, j = tap / ntw, l = tap - j * ntw;
-    const int rr = r0h + step * (nth - 1 - j), cc = r0w + step * (ntw - 1 - l);
-    const int ci0 = blockIdx.x * 32, co0 = blockIdx.y * 32;
-    for (int k = threadIdx.y; k < 32; k += 8) {
-        const int co = co0 + k, ci = ci0 + threadIdx.x;
-        T v = from_f<T>(0.f);
-        if (co < Cout && ci < Cin) v = W[(((int64_t)co * kh + rr) * kw + cc) * Cpad_in + ci];
-        tile[k][threadIdx.x] = v;
-    }
-    __syncthreads();
-    for (int k = threadIdx.y; k < 32; k += 8) {
-        const int ci = ci0 + k, co = co0 + threadIdx.x;
-        if (ci < Cin && co < Cpad_out) Wt[(((int64_t)ci * nth + j) * ntw + l) * Cpad_out + co] = tile[threadIdx.x][k];
+    // One thread per (8-channel ci group, tap, co), co fastest across lanes: it reads the 8 contiguous ci of
+    // W[co][rr][cc][ci0..+8) (one 16 / 32-byte load) and writes them down 8 Wt rows, each store coalesced
+    // across the warp's consecutive co.  No shared memory: the kernel overlaps whatever else runs.
+    const int ntap = nth * ntw, ng = (Cin + 7) / 8;
+    const int64_t n = (int64_t)ng * ntap * Cpad_out;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const int co = (int)(i % Cpad_out);
+        const int64_t t = i / Cpad_out;
+        const int tap = (int)(t % ntap), cg = (int)(t / ntap);
+        const int j = tap / ntw, l = tap - j * ntw;
+        const int rr = r0h + step * (nth - 1 - j), cc = r0w + step * (ntw - 1 - l);
+        const int ci0 = cg * 8;
+        T v[8];
+#pragma unroll
+        for (int e = 0; e < 8; ++e) v[e] = from_f<T>(0.f);
+        if (co < Cout) {
+            const T *src = W + (((int64_t)co * kh + rr) * kw + cc) * Cpad_in + ci0;
+            if (ci0 + 8 <= Cpad_in) {   // Cpad_in % 8 == 0 and 16-byte aligned rows: vector loads
+                if (sizeof(T) == 2) {
+                    *reinterpret_cast<uint4 *>(v) = __ldg(reinterpret_cast<const uint4 *>(src));
+                } else {
+                    reinterpret_cast<float4 *>(v)[0] = __ldg(reinterpret_cast<const float4 *>(src));
+                    reinterpret_cast<float4 *>(v)[1] = __ldg(reinterpret_cast<const float4 *>(src) + 1);
+                }
+            } else {
+#pragma unroll
+                for (int e = 0; e < 8; ++e)
+                    if (ci0 + e < Cpad_in) v[e] = src[e];
+            }
+        }
+        T *dst = Wt + (((int64_t)ci0 * nth + j) * ntw + l) * Cpad_out + co;
+        const int64_t rs = (int64_t)nth * ntw * Cpad_out;   // Wt row stride (one ci)
+#pragma unroll
+        for (int e = 0; e < 8; ++e)
+            if (ci0 + e < Cin) dst[e * rs] = v[e];
     }
 }
 
@@ -1771,47 +1790,85 @@ splitcnn_status_t launch_conv_pool_fwd_tc(const Level &Li, const Level &Lo, cons
 
 template <typename T>
 static void flip_weights(const void *w, void *wt, const LayerGeom &g, int cpad_in, int cpad_out, int r0h, int r0w,
-                         int step, int nth, int ntw, cudaStream_t st) {
-    const dim3 grid((unsigned)((g.L.cin + 31) / 32), (unsigned)((cpad_out + 31) / 32), (unsigned)(nth * ntw));
-    flip_weights_kernel<T><<<grid, dim3(32, 8), 0, st>>>(
+                         int step, int nth, int ntw, cudaStream_t st, int max_blocks = 148 * 16) {
+    const int64_t n = (int64_t)((g.L.cin + 7) / 8) * nth * ntw * cpad_out;
+    flip_weights_kernel<T><<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, max_blocks)), 256, 0, st>>>(
         (const T *)w, (T *)wt, g.L.cout, cpad_in, g.L.cin, g.L.kh, g.L.kw, cpad_out, r0h, r0w, step, nth, ntw);
     count_launch();
 }
 
+// Stride-S dgrad phase (rh, rw): first tap (r0h, r0w) and tap counts of its sub-filter (0: no tap reaches it)
+struct DgradPhase {
+    int r0h, r0w, nth, ntw;
+};
+static DgradPhase dgrad_phase(const LayerGeom &g, int rh, int rw) {
+    const int S = g.L.sh, pbh = g.pad_h[0], pbw = g.pad_w[0];
+    DgradPhase d;
+    d.r0h = ((rh + pbh) % S + S) % S;
+    d.r0w = ((rw + pbw) % S + S) % S;
+    d.nth = d.r0h < g.L.kh ? (g.L.kh - d.r0h + S - 1) / S : 0;
+    d.ntw = d.r0w < g.L.kw ? (g.L.kw - d.r0w + S - 1) / S : 0;
+    return d;
+}
+
+// The weights the data gradient multiplies with: stride 1 the 180-degree flip, stride S one sub-filter per
+// phase that some tap reaches, 1 KB-aligned one after another (the layout of the dgrad workspace prefix).
+// max_blocks: the in-call flip (on the critical path) takes many blocks; a prepared copy built next to the
+// forward pass takes one per SM, so the persistent conv CTAs still fit beside it (threads, no shared memory)
+void prep_dgrad_weights_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *w, void *wt, cudaStream_t st,
+                           int max_blocks) {
+    const int S = g.L.sh;
+    if (max_blocks <= 0) max_blocks = num_sms();
+    if (S == 1) {
+        flip_weights<__nv_bfloat16>(w, wt, g, Li.Cpad, Lo.Cpad, 0, 0, 1, g.L.kh, g.L.kw, st, max_blocks);
+        return;
+    }
+    char *wsp = (char *)wt;
+    for (int rh = 0; rh < S; ++rh)
+        for (int rw = 0; rw < S; ++rw) {
+            const DgradPhase d = dgrad_phase(g, rh, rw);
+            if (d.nth == 0 || d.ntw == 0) continue;
+            flip_weights<__nv_bfloat16>(w, wsp, g, Li.Cpad, Lo.Cpad, d.r0h, d.r0w, S, d.nth, d.ntw, st, max_blocks);
+            wsp += (((int64_t)g.L.cin * d.nth * d.ntw * Lo.Cpad * 2 + 1023) / 1024) * 1024;
+        }
+}
+
+// prepared: w already holds prep_dgrad_weights_tc's output (BF16) -- no flip in this call
 splitcnn_status_t launch_conv_dgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy, const void *w,
                                        void *dx, const void *relu_src, void *ws, int p0, int p1, cudaStream_t st,
-                                       splitcnn_dtype_t dt, int accum) {
-    const int S = g.L.sh, kh = g.L.kh, kw = g.L.kw;
+                                       splitcnn_dtype_t dt, int accum, bool prepared) {
+    const int S = g.L.sh;
+    if (prepared && dt != SPLITCNN_BF16) return fail(SPLITCNN_ERR_UNSUPPORTED, "prepared dgrad weights: bf16 only");
     if (S == 1) {
-        if (dt == SPLITCNN_BF16) flip_weights<__nv_bfloat16>(w, ws, g, Li.Cpad, Lo.Cpad, 0, 0, 1, kh, kw, st);
-        else flip_weights<float>(w, ws, g, Li.Cpad, Lo.Cpad, 0, 0, 1, kh, kw, st);
-        return launch_tc(1, Lo, Li, g, dy, ws, g.L.cin, nullptr, dx, relu_src, 0, p0, p1, st, nullptr, nullptr,
+        if (!prepared) {
+            if (dt == SPLITCNN_BF16) flip_weights<__nv_bfloat16>(w, ws, g, Li.Cpad, Lo.Cpad, 0, 0, 1, g.L.kh, g.L.kw, st);
+            else flip_weights<float>(w, ws, g, Li.Cpad, Lo.Cpad, 0, 0, 1, g.L.kh, g.L.kw, st);
+        }
+        return launch_tc(1, Lo, Li, g, dy, prepared ? w : ws, g.L.cin, nullptr, dx, relu_src, 0, p0, p1, st, nullptr, nullptr,
                          dt == SPLITCNN_BF16 ? 0 : 1, accum);
     }
     if (dt != SPLITCNN_BF16) return fail(SPLITCNN_ERR_UNSUPPORTED, "tf32 strided data gradient");
     // stride S: S*S output phases, each a stride-1 correlation with the taps r = (rho + p_b) (mod S)
     // (every patch of a plan shares its begin pad under R2, checked in conv_tc_supported)
     const int pbh = g.pad_h[0], pbw = g.pad_w[0];
-    char *wsp = (char *)ws;
+    if (!prepared) prep_dgrad_weights_tc(Li, Lo, g, w, ws, st, 148 * 16);
+    const char *wsp = (const char *)(prepared ? w : ws);
     for (int rh = 0; rh < S; ++rh)
         for (int rw = 0; rw < S; ++rw) {
-            const int r0h = ((rh + pbh) % S + S) % S, r0w = ((rw + pbw) % S + S) % S;
-            const int nth = r0h < kh ? (kh - r0h + S - 1) / S : 0, ntw = r0w < kw ? (kw - r0w + S - 1) / S : 0;
-            if (nth == 0 || ntw == 0) {
-                LevelDesc d = make_level_desc(Li);
+            const DgradPhase d = dgrad_phase(g, rh, rw);
+            if (d.nth == 0 || d.ntw == 0) {
+                LevelDesc ld = make_level_desc(Li);
                 dim3 grid((unsigned)std::max(1, std::min(2048, 148 * 8 / std::max(1, p1 - p0))), (unsigned)(p1 - p0));
-                zero_phase_kernel<<<grid, 256, 0, st>>>((__nv_bfloat16 *)dx, d, S, rh, rw, p0);
+                zero_phase_kernel<<<grid, 256, 0, st>>>((__nv_bfloat16 *)dx, ld, S, rh, rw, p0);
                 count_launch();
                 continue;
             }
-            const int ch = (rh + pbh - r0h) / S, cw = (rw + pbw - r0w) / S;
-            const int64_t n = (int64_t)g.L.cin * nth * ntw * Lo.Cpad;
-            flip_weights<__nv_bfloat16>(w, wsp, g, Li.Cpad, Lo.Cpad, r0h, r0w, S, nth, ntw, st);
-            Phase ph{S, rh, rw, nth, ntw, nth - 1 - ch, ntw - 1 - cw};
+            const int ch = (rh + pbh - d.r0h) / S, cw = (rw + pbw - d.r0w) / S;
+            Phase ph{S, rh, rw, d.nth, d.ntw, d.nth - 1 - ch, d.ntw - 1 - cw};
             const splitcnn_status_t r = launch_tc(1, Lo, Li, g, dy, wsp, g.L.cin, nullptr, dx, relu_src, 0, p0, p1, st,
                                                   nullptr, &ph);
             if (r != SPLITCNN_OK) return r;
-            wsp += ((n * 2 + 1023) / 1024) * 1024;
+            wsp += (((int64_t)g.L.cin * d.nth * d.ntw * Lo.Cpad * 2 + 1023) / 1024) * 1024;
         }
     return SPLITCNN_OK;
 }

@@ -52,7 +52,11 @@ splitcnn_status_t launch_conv_pool_fwd_tc(const Level &Li, const Level &Lo, cons
                                           int p0, int p1, cudaStream_t st);
 splitcnn_status_t launch_conv_dgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *dy, const void *w,
                                        void *dx, const void *relu_src, void *ws, int p0, int p1, cudaStream_t st,
-                                       splitcnn_dtype_t dt = SPLITCNN_BF16, int accum = 0);
+                                       splitcnn_dtype_t dt = SPLITCNN_BF16, int accum = 0, bool prepared = false);
+// the dgrad-ready (flipped / phase) weights launch_conv_dgrad_tc builds in its workspace, into wt (BF16)
+// max_blocks <= 0: one block per SM
+void prep_dgrad_weights_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *w, void *wt, cudaStream_t st,
+                           int max_blocks);
 splitcnn_status_t launch_conv_wgrad_tc(const Level &Li, const Level &Lo, const LayerGeom &g, const void *x, const void *dy,
                                        float *dw, float *db, float beta, void *ws, int p0, int p1, cudaStream_t st);
 // fp32 storage on the tensor cores (TF32 one pass / FP32 3xTF32; wgrad by bf16 operand splitting)

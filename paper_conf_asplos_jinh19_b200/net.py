@@ -35,7 +35,8 @@ class SplitNet:
                  dtype: int = sc.BF16, device="cuda", patch_range=None, force_simt: bool = False,
                  grad_buffer: torch.Tensor | None = None, input_relu: bool = False, fuse_pool: bool = True,
                  static_pool: bool = False, input_grad: bool = False, mask_output_grad: bool = True,
-                 concurrent_wgrad: bool = True, schedule: str = "layer", group_rows: int = 1):
+                 concurrent_wgrad: bool = True, schedule: str = "layer", group_rows: int = 1,
+                 prep_dgrad_weights: bool = False):
         self.region_layers, self.tail_layers = region, tail
         self.N, self.C, self.H, self.W = N, C, H, W
         self.split, self.mode, self.omega, self.seed = split, mode, omega, seed
@@ -52,6 +53,13 @@ class SplitNet:
         # a layer's weight gradient and its data gradient both read only dY: the weight gradient runs on a
         # side stream (its own workspace) concurrently with the data gradient, joined before the next layer
         self.concurrent_wgrad = concurrent_wgrad
+        # prep_dgrad_weights: the data gradients' flipped weights (splitcnn_conv_dgrad_weights) built once per
+        # step on a side stream during the forward pass instead of inside every conv_bwd_data call.  Off by
+        # default: the flips share the SMs with the forward convs and cost more there than the ~5 us each
+        # costs on the backward's path (same-box A/B, C2 0.995 -> 1.03 ms, C5 28.5 -> 28.8 ms:
+        # profiles/r2i/ab_prep_resnet_conc.txt)
+        self.prep_dgrad_weights = prep_dgrad_weights and not force_simt
+        self.prep_stream, self._prep_pending, self._prep_valid = None, False, False
         # "layer": every layer over all patches, layer after layer; "patch": patch-major (depth-first,
         # chained patches never communicate, so any schedule is valid): `group_rows` patch rows
         # run through the whole split region before the next group, forward and backward
@@ -181,18 +189,23 @@ class SplitNet:
         for key, layers, plan in (("r", self.region_layers, self.region), ("t", self.tail_layers, self.tail)):
             for m, l in enumerate(layers):
                 if l["op"] == "conv":
-                    shapes.append(((key, m), (l["cout"], l["kh"], l["kw"], plan.levels[m]["Cpad"]), l["cout"]))
-        nbytes = sum(al(4 * co) + al(es * sh[0] * sh[1] * sh[2] * sh[3]) for _, sh, co in shapes)
+                    wp = (sc.splitcnn_conv_dgrad_weights_size(plan.handle, m, self.dtype)
+                          if self.prep_dgrad_weights and self._has_dgrad(key, m) else 0)
+                    shapes.append(((key, m), (l["cout"], l["kh"], l["kw"], plan.levels[m]["Cpad"]), l["cout"], wp))
+        nbytes = sum(al(4 * co) + al(es * sh[0] * sh[1] * sh[2] * sh[3]) + al(wp) for _, sh, co, wp in shapes)
         gbytes = 0 if grad_buffer is not None else al(4 * self.grad_numel())
         self.param_pool = torch.zeros(nbytes + gbytes, dtype=torch.uint8, device=dev)
-        self.params, off = {}, 0
-        for key, sh, co in shapes:
+        self.params, self.wprep, off = {}, {}, 0
+        for key, sh, co, wp in shapes:
             nw = es * sh[0] * sh[1] * sh[2] * sh[3]
             W = self.param_pool[off:off + nw].view(td).view(sh)
             off += al(nw)
             b = self.param_pool[off:off + 4 * co].view(torch.float32)
             off += al(4 * co)
             self.params[key] = (W, b)
+            if wp:        # the layer's dgrad-ready weights (parameter pool: they live as long as the weights)
+                self.wprep[key] = self.param_pool[off:off + wp]
+                off += al(wp)
         if grad_buffer is None:
             grad_buffer = self.param_pool[off:off + 4 * self.grad_numel()].view(torch.float32)
         self.bind_grads(grad_buffer)
@@ -323,6 +336,7 @@ class SplitNet:
     def set_params(self, params):
         """params: list (region + tail order, convs only) of (W_oihw, b) torch/numpy arrays."""
         it = iter(params)
+        self._prep_valid = False     # new weights: the next forward rebuilds the dgrad-ready copies
         for key, layers, plan in (("r", self.region_layers, self.region), ("t", self.tail_layers, self.tail)):
             for m, l in enumerate(layers):
                 if l["op"] == "conv":
@@ -436,6 +450,7 @@ class SplitNet:
         (NCHW [N][C][h1-h0][W]: a rank's own rows under patch-row sharding).  Returns the output level."""
         p0, p1 = self.patch_range
         R, dt, fl = self.region.handle, self.dtype, self.flags_extra
+        self._prep_dgrad(stream)
         b_in = 2 * self._bytes(self.region, 0)[0]
         h0, h1 = self.input_rows()
         if x.dim() == 4 and x_layout == sc.NCHW and x.shape[2] == h1 - h0 and h1 - h0 != self.H:
@@ -455,6 +470,42 @@ class SplitNet:
             self._run_fwd("t", self.tail, self.tail_layers, self.act_t, 0, 1, stream)
             return self.act_t[-1]
         return self.act_r[-1]
+
+    def _has_dgrad(self, key, m) -> bool:
+        """Whether the backward runs conv (key, m)'s data gradient (not the region's first layer unless the
+        input gradient is asked for)."""
+        return not (key == "r" and m == 0 and not self.input_grad)
+
+    def _prep_dgrad(self, stream):
+        """Fork a side stream off the forward and build every layer's dgrad-ready weights there; the backward
+        waits for it before its first data gradient (a captured step records the fork as a parallel branch)."""
+        if not self.wprep:
+            return
+        main = stream if stream is not None else torch.cuda.current_stream(self.device)
+        if self.prep_stream is None:
+            self.prep_stream = torch.cuda.Stream(self.device)
+            self.prep_fork, self.prep_join = torch.cuda.Event(), torch.cuda.Event()
+        self.prep_fork.record(main)
+        self.prep_stream.wait_event(self.prep_fork)
+        with torch.cuda.stream(self.prep_stream):
+            for (key, m), wt in self.wprep.items():
+                plan = self.region if key == "r" else self.tail
+                W = self.params[(key, m)][0]
+                self._label = (self.region_layers if key == "r" else self.tail_layers)[m].get("name", f"{key}{m}")
+                self._call("dgrad_weights", 2 * W.numel() * W.element_size(), sc.splitcnn_conv_dgrad_weights,
+                           plan.handle, m, self.dtype, W, wt, wt.numel(), self.prep_stream)
+        self.prep_join.record(self.prep_stream)
+        self._prep_pending = self._prep_valid = True
+
+    def _dgrad_w(self, key, m, W, flags, main):
+        """(weights, flags) for conv (key, m)'s data gradient: the prepared copy (+ FLAG_DGRAD_WEIGHTS, after
+        waiting once per backward for the forward's preparation branch) where there is one."""
+        if (key, m) not in self.wprep or not self._prep_valid:
+            return W, flags
+        if self._prep_pending:
+            main.wait_event(self.prep_join)
+            self._prep_pending = False
+        return self.wprep[(key, m)], flags | sc.FLAG_DGRAD_WEIGHTS
 
     # hooks (no-ops here; the offload executor overrides them)
     def hook_before_fwd(self, key, m):
@@ -553,8 +604,9 @@ class SplitNet:
                         self.join_ev[m % 64].record(self.side)
                 if not last:
                     relu_src = acts[m] if self._masked(key, m) else None
-                    self._call("conv_dgrad", work, sc.splitcnn_conv_bwd_data, plan.handle, m, self.dtype, g, W, out,
-                               relu_src, self.ws, self.ws_bytes, self.flags_extra, p0, p1, stream)
+                    wt, fl = self._dgrad_w(key, m, W, self.flags_extra, main)
+                    self._call("conv_dgrad", work, sc.splitcnn_conv_bwd_data, plan.handle, m, self.dtype, g, wt, out,
+                               relu_src, self.ws, self.ws_bytes, fl, p0, p1, stream)
                 if fork:      # join: the next layer may overwrite g's buffer
                     main.wait_event(self.join_ev[m % 64])
                 else:

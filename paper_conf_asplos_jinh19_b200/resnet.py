@@ -121,6 +121,7 @@ class ResSplitNet(SplitNet):
         if ws > self.ws_bytes:
             self.ws = torch.zeros(ws // 4 + 4, dtype=torch.float32, device=dev)
             self.ws_bytes = self.ws.numel() * 4
+            self.ws_w = torch.zeros_like(self.ws) if self.concurrent_wgrad else self.ws
 
     def _ds_layers(self):
         return [(k, self.blocks[k]["ds"], self.ds_plans[k]) for k in sorted(self.ds_plans)]
@@ -184,6 +185,7 @@ class ResSplitNet(SplitNet):
         p0, p1 = self.patch_range
         R, dt, fl = self.region.handle, self.dtype, self.flags_extra
         acts = self.act_r
+        self._prep_dgrad(stream)
         self._label = "input"
         if self.s2d:
             self._call("split", 2 * self._bytes(self.region, 0)[0], sc.splitcnn_split_s2d, R, 0, dt, x, self.stem_cin,
@@ -248,6 +250,37 @@ class ResSplitNet(SplitNet):
         R, dt, fl = self.region.handle, self.dtype, self.flags_extra
         acts, L = self.act_r, self.region_layers
         nl = self.region.nlayers
+        main = stream if stream is not None else torch.cuda.current_stream(self.device)
+        conc = self.concurrent_wgrad
+        nev = [0]
+
+        def wgrad(handle, layer, x_act, gsrc, dW, db, wk):
+            """A weight gradient: concurrently with the data gradients on the side stream (forked after its dY
+            is ready on `main`, own workspace), joined at the end of the block -- or in line."""
+            if not conc:
+                self._call("conv_wgrad", wk, sc.splitcnn_conv_bwd_filter, handle, layer, dt, x_act, gsrc, dW, db, 0.0,
+                           self.ws, self.ws_bytes, fl, p0, p1, stream)
+                return
+            if self.side is None:
+                self.side = torch.cuda.Stream(self.device)
+                self.fork_ev = [torch.cuda.Event() for _ in range(64)]
+                self.join_ev = [torch.cuda.Event() for _ in range(64)]
+            ev = self.fork_ev[nev[0] % 64]
+            nev[0] += 1
+            ev.record(main)
+            self.side.wait_event(ev)
+            with torch.cuda.stream(self.side):
+                self._call("conv_wgrad", wk, sc.splitcnn_conv_bwd_filter, handle, layer, dt, x_act, gsrc, dW, db, 0.0,
+                           self.ws_w, self.ws_bytes, fl, p0, p1, self.side)
+
+        def join():
+            """main waits for the side stream's weight gradients (their dY buffers are reused next)."""
+            if conc and self.side is not None:
+                ev = self.join_ev[nev[0] % 64]
+                nev[0] += 1
+                ev.record(self.side)
+                main.wait_event(ev)
+
         g = self.grad[0]
         self._label = "output"
         self._call("split", 2 * self._bytes(self.region, nl - 1)[1], sc.splitcnn_split, R, nl, dt, dy, sc.NHWC, g,
@@ -267,19 +300,19 @@ class ResSplitNet(SplitNet):
                 dW, db = self.grads[("r", a + 1)]
                 wk = self._conv_work(self.region, a + 1, lb)
                 self._label = lb["name"]
-                self._call("conv_dgrad", wk, sc.splitcnn_conv_bwd_data, R, a + 1, dt, gz, W, gh, acts[a + 1], self.ws,
-                           self.ws_bytes, fl, p0, p1, stream)
-                self._call("conv_wgrad", wk, sc.splitcnn_conv_bwd_filter, R, a + 1, dt, acts[a + 1], gz, dW, db, 0.0,
-                           self.ws, self.ws_bytes, fl, p0, p1, stream)
+                wgrad(R, a + 1, acts[a + 1], gz, dW, db, wk)
+                Wd, fd = self._dgrad_w("r", a + 1, W, fl, main)
+                self._call("conv_dgrad", wk, sc.splitcnn_conv_bwd_data, R, a + 1, dt, gz, Wd, gh, acts[a + 1], self.ws,
+                           self.ws_bytes, fd, p0, p1, stream)
                 gx = self._free(gz, gh)
                 W, _ = self.params[("r", a)]
                 dW, db = self.grads[("r", a)]
                 wk = self._conv_work(self.region, a, la)
                 self._label = la["name"]
-                self._call("conv_dgrad", wk, sc.splitcnn_conv_bwd_data, R, a, dt, gh, W, gx, None, self.ws,
-                           self.ws_bytes, fl, p0, p1, stream)
-                self._call("conv_wgrad", wk, sc.splitcnn_conv_bwd_filter, R, a, dt, acts[a], gh, dW, db, 0.0,
-                           self.ws, self.ws_bytes, fl, p0, p1, stream)
+                wgrad(R, a, acts[a], gh, dW, db, wk)
+                Wd, fd = self._dgrad_w("r", a, W, fl, main)
+                self._call("conv_dgrad", wk, sc.splitcnn_conv_bwd_data, R, a, dt, gh, Wd, gx, None, self.ws,
+                           self.ws_bytes, fd, p0, p1, stream)
                 if k in self.ds_plans:
                     P, lds = self.ds_plans[k], self.blocks[k]["ds"]
                     W, _ = self._ds_params[k]
@@ -287,10 +320,9 @@ class ResSplitNet(SplitNet):
                     gs = self._free(gz, gh, gx)
                     wk = self._conv_work(P, 0, lds)
                     self._label = lds["name"]
+                    wgrad(P.handle, 0, acts[a], gz, dW, db, wk)
                     self._call("conv_dgrad", wk, sc.splitcnn_conv_bwd_data, P.handle, 0, dt, gz, W, gs, None, self.ws,
                                self.ws_bytes, fl, p0, p1, stream)
-                    self._call("conv_wgrad", wk, sc.splitcnn_conv_bwd_filter, P.handle, 0, dt, acts[a], gz, dW, db,
-                               0.0, self.ws, self.ws_bytes, fl, p0, p1, stream)
                 else:
                     gs = gz
                 mask = acts[a] if self._masked("r", a) else None
@@ -298,6 +330,7 @@ class ResSplitNet(SplitNet):
                 nb = self._bytes(self.region, a)[0]
                 self._call("add", (4 if mask is not None else 3) * nb, sc.splitcnn_add, R, a, dt, gx, gs, gx, mask, 0,
                            p0, p1, stream)
+                join()
                 g = gx
                 m = a - 1
                 continue
@@ -310,8 +343,9 @@ class ResSplitNet(SplitNet):
                 dW, db = self.grads[("r", m)]
                 wk = self._conv_work(self.region, m, l)
                 if not last:
-                    self._call("conv_dgrad", wk, sc.splitcnn_conv_bwd_data, R, m, dt, g, W, out,
-                               acts[m] if self._masked("r", m) else None, self.ws, self.ws_bytes, fl, p0, p1, stream)
+                    Wd, fd = self._dgrad_w("r", m, W, fl, main)
+                    self._call("conv_dgrad", wk, sc.splitcnn_conv_bwd_data, R, m, dt, g, Wd, out,
+                               acts[m] if self._masked("r", m) else None, self.ws, self.ws_bytes, fd, p0, p1, stream)
                 self._call("conv_wgrad", wk, sc.splitcnn_conv_bwd_filter, R, m, dt, acts[m], g, dW, db, 0.0, self.ws,
                            self.ws_bytes, fl, p0, p1, stream)
             else:
@@ -322,6 +356,7 @@ class ResSplitNet(SplitNet):
             if not last:
                 g = out
             m -= 1
+        join()
         return g
 
     # ------------------------------------------------------------------ accounting

@@ -25,6 +25,7 @@ OP_CONV, OP_MAXPOOL = 0, 1
 NCHW, NHWC, NCHW_S2D = 0, 1, 2
 FLAG_RELU = 0x1
 FLAG_POOL_RELU_MASK = 0x2
+FLAG_DGRAD_WEIGHTS = 0x4
 FLAG_FORCE_SIMT = 0x100
 MAX_SPLITS = 32
 
@@ -35,6 +36,7 @@ EXPORTED = [
     "splitcnn_plan_layer", "splitcnn_workspace_size",
     "splitcnn_split", "splitcnn_split_s2d", "splitcnn_split_rows", "splitcnn_merge",
     "splitcnn_conv_fwd", "splitcnn_conv_fwd_ws", "splitcnn_conv_fwd_res", "splitcnn_conv_bwd_data", "splitcnn_conv_bwd_filter",
+    "splitcnn_conv_dgrad_weights_size", "splitcnn_conv_dgrad_weights",
     "splitcnn_pool_fwd", "splitcnn_pool_bwd", "splitcnn_conv_pool_fwd", "splitcnn_conv_pool_supported", "splitcnn_add",
     "splitcnn_gap_fwd", "splitcnn_gap_bwd",
     "splitcnn_bn_workspace_size", "splitcnn_bn_stats", "splitcnn_bn_fwd", "splitcnn_bn_bwd_sums", "splitcnn_bn_bwd",
@@ -92,6 +94,8 @@ _sig("splitcnn_conv_fwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _u32, _i
 _sig("splitcnn_conv_fwd_ws", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _u32, _vp, _sz, _i32, _i32, _vp])
 _sig("splitcnn_conv_fwd_res", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _vp, _u32, _vp, _sz, _i32, _i32, _vp])
 _sig("splitcnn_conv_bwd_data", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _vp, _sz, _u32, _i32, _i32, _vp])
+_sig("splitcnn_conv_dgrad_weights_size", [_vp, _i32, ctypes.c_int, ctypes.POINTER(_sz)])
+_sig("splitcnn_conv_dgrad_weights", [_vp, _i32, ctypes.c_int, _vp, _vp, _sz, _vp])
 _sig("splitcnn_conv_bwd_filter", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _vp, _f32, _vp, _sz, _u32, _i32, _i32, _vp])
 _sig("splitcnn_pool_fwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
 _sig("splitcnn_pool_bwd", [_vp, _i32, ctypes.c_int, _vp, _vp, _vp, _u32, _i32, _i32, _vp])
@@ -285,6 +289,16 @@ def splitcnn_conv_bwd_data(plan, layer, dtype, dy, w, dx, relu_src=None, ws=None
                            stream=None):
     _check(_lib.splitcnn_conv_bwd_data(plan, layer, dtype, _ptr(dy), _ptr(w), _ptr(dx), _ptr(relu_src), _ptr(ws),
                                        ws_bytes, flags, p0, p1, _stream(stream)))
+
+
+def splitcnn_conv_dgrad_weights_size(plan, layer, dtype) -> int:
+    b = _sz(0)
+    _check(_lib.splitcnn_conv_dgrad_weights_size(plan, layer, dtype, ctypes.byref(b)))
+    return b.value
+
+
+def splitcnn_conv_dgrad_weights(plan, layer, dtype, w, wt, wt_bytes, stream=None):
+    _check(_lib.splitcnn_conv_dgrad_weights(plan, layer, dtype, _ptr(w), _ptr(wt), wt_bytes, _stream(stream)))
 
 
 def splitcnn_conv_bwd_filter(plan, layer, dtype, x, dy, dw, db=None, beta=0.0, ws=None, ws_bytes=0, flags=0, p0=0,

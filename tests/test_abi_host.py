@@ -132,6 +132,30 @@ def test_errors(sc):
     sc.splitcnn_plan_destroy(p)
 
 
+def test_dgrad_weights_contract(sc):
+    """splitcnn_conv_dgrad_weights_size / _weights host contract: the size is the tcgen05 dgrad's flip
+    workspace for BF16 (stride 1: Cin x kh x kw x Cpad_out bf16, stride 2: one sub-filter per reached phase),
+    0 for the other dtypes, and the build call rejects size 0, null and short buffers before any launch."""
+    layers = [synth.conv(64, 64, name="c1"), synth.conv(64, 128, 3, 2, 1, name="c2"), synth.maxpool(128)]
+    p = sc.splitcnn_plan_create(layers, 2, 64, 32, 32, [0, 4, 8], [0, 4, 8])
+    b1 = sc.splitcnn_conv_dgrad_weights_size(p, 0, sc.BF16)
+    assert b1 >= 64 * 9 * 64 * 2
+    assert b1 == sc.splitcnn_workspace_size(p, 0, sc.BF16, 1)
+    assert sc.splitcnn_conv_dgrad_weights_size(p, 1, sc.BF16) >= 64 * 9 * 128 * 2
+    for dt in (sc.FP32, sc.TF32):
+        assert sc.splitcnn_conv_dgrad_weights_size(p, 0, dt) == 0
+        with pytest.raises(sc.SplitCNNError) as e:
+            sc.splitcnn_conv_dgrad_weights(p, 0, dt, 256, 512, 1 << 20, 0)
+        assert e.value.status == sc.ERR_UNSUPPORTED
+    with pytest.raises(sc.SplitCNNError, match="null"):
+        sc.splitcnn_conv_dgrad_weights(p, 0, sc.BF16, None, 512, b1, 0)
+    with pytest.raises(sc.SplitCNNError, match="too small"):
+        sc.splitcnn_conv_dgrad_weights(p, 0, sc.BF16, 256, 512, b1 - 1, 0)
+    with pytest.raises(sc.SplitCNNError, match="not a convolution"):
+        sc.splitcnn_conv_dgrad_weights_size(p, 2, sc.BF16)
+    sc.splitcnn_plan_destroy(p)
+
+
 # --------------------------------------------------------------------------- Algorithm 1
 def _check_offload_invariants(times, cand, bw, off, sync):
     T = len(times)

@@ -131,6 +131,18 @@ def test_conv_parity(sc, case, mode):
     for row in dXgot:
         for blk in row:
             assert np.all(blk[:, cin:] == 0), "channel padding of dX must be zero"
+    # dgrad-ready weights built once (splitcnn_conv_dgrad_weights) + FLAG_DGRAD_WEIGHTS: bitwise the same dX
+    wt_b = sc.splitcnn_conv_dgrad_weights_size(pl.handle, 0, dtype)
+    if mode == "bf16_tc" and wt_b:
+        wt = torch.empty(wt_b, dtype=torch.uint8, device="cuda")
+        sc.splitcnn_conv_dgrad_weights(pl.handle, 0, dtype, w, wt, wt_b)
+        dx2 = torch.full_like(dx, 5.0)
+        sc.splitcnn_conv_bwd_data(pl.handle, 0, dtype, dy, wt, dx2, mask, None, 0, sc.FLAG_DGRAD_WEIGHTS)
+        assert torch.equal(dx2, dx), "prepared dgrad weights must give the in-call flip's dX bit for bit"
+    elif dtype != sc.BF16:
+        assert wt_b == 0
+        with pytest.raises(sc.SplitCNNError):
+            sc.splitcnn_conv_bwd_data(pl.handle, 0, dtype, dy, w, dx, mask, ws, ws_b, sc.FLAG_DGRAD_WEIGHTS)
 
     dw = torch.full((cout, k, k, lv0["Cpad"]), 3.0, dtype=torch.float32, device="cuda")
     db = torch.full((cout,), 3.0, dtype=torch.float32, device="cuda")

@@ -188,3 +188,29 @@ def test_resnet18_full_trunk(sc, dtype_name):
         errs[f"dW{i}"] = normwise(dW.double().cpu().numpy(), dWs[i])
         errs[f"db{i}"] = normwise(db.double().cpu().numpy(), dbs[i])
     assert max(errs.values()) <= (2e-2 if bf else 1e-4), errs
+
+
+def test_resnet_concurrent_wgrad_bitwise(sc):
+    """The ResNet executor's weight gradients on the side stream (concurrent with the data gradients, joined
+    per block) give bitwise the gradients of the serial backward: the same kernels on the same inputs, only
+    the stream placement differs; two steps, so a join that came too late would show as a stale buffer."""
+    from paper_conf_asplos_jinh19_b200.resnet import ResSplitNet
+    chain, blocks = synth.resnet18_blocks(64, 128)
+    N, H = 4, 64
+    g = synth.rng(7)
+    params = synth.resnet_params(g, chain, blocks)
+    params = [(torch.from_numpy(synth.to_bf16_f32(W)), torch.from_numpy(b)) for W, b in params]
+    x = torch.from_numpy(synth.to_bf16_f32(synth.uniform(g, (N, 3, H, H)))).to("cuda", torch.bfloat16)
+    nets = []
+    for conc in (True, False):
+        net = ResSplitNet(chain, blocks, N, 3, H, H, split=(2, 2), dtype=sc.BF16, concurrent_wgrad=conc)
+        net.set_params(params)
+        nets.append(net)
+    dy = torch.randn(nets[0].output_numel(), generator=torch.Generator().manual_seed(3)).to("cuda", torch.bfloat16)
+    for _ in range(2):
+        for net in nets:
+            net.forward(x)
+            net.backward(dy)
+        torch.cuda.synchronize()
+        assert torch.equal(nets[0].out, nets[1].out)
+        assert torch.equal(nets[0].grad_flat, nets[1].grad_flat)

@@ -281,6 +281,33 @@ def test_static_pool_step_bitwise(sc, cfg, N, H):
         assert torch.equal(plain.grad_flat, stat.grad_flat)
 
 
+@pytest.mark.parametrize("cfg,N,H", [("C2", 8, 32), ("C4", 2, 64)])
+def test_prepared_dgrad_weights_step_bitwise(sc, cfg, N, H):
+    """prep_dgrad_weights (splitcnn_conv_dgrad_weights on a side stream during the forward, FLAG_DGRAD_WEIGHTS
+    in the backward) gives bitwise the outputs and gradients of the default executor (flip inside each
+    conv_bwd_data call), over two steps and after new weights (the copies are rebuilt)."""
+    from paper_conf_asplos_jinh19_b200.net import SplitNet
+    c = synth.vgg_config(cfg, N=N)
+    g = synth.rng(c["seed"] + 5)
+    kw = dict(split=c["split"], mode=c["mode"], omega=c.get("omega", 0.2), seed=c["seed"])
+    plain = SplitNet(c["layers"], c["tail"], N, 3, H, H, **kw)
+    prep = SplitNet(c["layers"], c["tail"], N, 3, H, H, prep_dgrad_weights=True, **kw)
+    assert prep.wprep and not plain.wprep
+    x = torch.from_numpy(synth.uniform(g, (N, 3, H, H))).to("cuda", torch.bfloat16)
+    dy = torch.randn(plain.output_numel(), generator=torch.Generator().manual_seed(4)).to("cuda", torch.bfloat16)
+    for it in range(3):
+        if it != 1:
+            params = [p for p in synth.layer_params(g, c["layers"] + c["tail"]) if p is not None]
+            tp = [(torch.from_numpy(W), torch.from_numpy(b)) for W, b in params]
+            plain.set_params(tp)
+            prep.set_params(tp)
+        plain.step(x, dy)
+        prep.step(x, dy)
+        torch.cuda.synchronize()
+        assert torch.equal(plain.act_t[-1] if plain.tail else plain.act_r[-1], prep.act_t[-1] if prep.tail else prep.act_r[-1])
+        assert torch.equal(plain.grad_flat, prep.grad_flat)
+
+
 def test_autograd_module_matches_executor(sc):
     """SplitStack (torch.nn front end): y, every weight / bias gradient bitwise equal to the executor's
     step; x.grad of a single split conv (C1 shape, fp32) equal to the oracle's data gradient."""

@@ -359,6 +359,10 @@ __global__ void __launch_bounds__(CONV_THREADS, 1) conv_tc_kernel(const __grid_c
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t rank = CTA2 ? tc::cluster_ctarank() : 0u;
     const bool leader = rank == 0;
+    // launched with programmatic stream serialization (PDL): this grid's CTAs are placed while the previous
+    // kernel drains; nothing below touches global memory before the previous grid is complete and visible
+    tc::grid_dep_launch();
+    tc::grid_dep_wait();
     if (warp == 0 && lane == 0) {
         for (int s = 0; s < S; ++s) {
             tc::mbar_init(&full[s], 1);
@@ -1272,6 +1276,8 @@ int round_up16(int x) { return (x + 15) / 16 * 16; }
 // conv1_2 + pool forward, profiles/r2i/ab_epilogue.txt)
 constexpr uint32_t CONV_SMEM_BUDGET = 210u * 1024u;
 
+
+
 bool a_channels_ok(int cpad) { return cpad == 8 || cpad == 16 || cpad == 32 || cpad % 64 == 0; }
 
 // mode 0: forward (A = X at level m, out = level m+1); mode 1: dgrad (A = dY at level m+1, out = level m)
@@ -1309,20 +1315,21 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
     const int ncols_out = mode == 0 ? g.L.cout : g.L.cin;
     // N tile: up to 256 output channels; small layers (few 128-pixel M tiles, e.g. 2x2 / 4x4 CIFAR tails)
     // take narrower N tiles so that M tiles x N tiles still covers the SMs
-    int BN = std::min(256, round_up16(ncols_out));
+    int BN0 = std::min(256, round_up16(ncols_out));
     {
         long mt = 0;
         for (int q = p0; q < p1; ++q) {
             const int i = q / Lout.nw(), j = q % Lout.nw();
             mt += ((long)La.N * out_ext_h(i) * out_ext_w(j) + 127) / 128;
         }
-        while (BN > 64 && BN % 32 == 0 && mt * ((ncols_out + BN - 1) / BN) < num_sms())
-            BN /= 2;
+        while (BN0 > 64 && BN0 % 32 == 0 && mt * ((ncols_out + BN0 - 1) / BN0) < num_sms())
+            BN0 /= 2;
     }
-    const int nco = (ncols_out + BN - 1) / BN;
+    const int nco0 = (ncols_out + BN0 - 1) / BN0;
     const int N = La.N;
     for (int g0 = p0; g0 < p1; g0 += TC_MAXP) {
         const int g1 = std::min(p1, g0 + TC_MAXP);
+        int BN = BN0, nco = nco0;   // this launch's N tile (see the wave rule below)
         std::vector<std::pair<int, int>> ext;
         for (int q = g0; q < g1; ++q) {
             const int i = q / Lout.nw(), j = q % Lout.nw();
@@ -1374,6 +1381,24 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
             if (tall_pre && search(1, h1) * 4 <= t_any * 5) hs = h1;
             (void)best;
             ts = hs;
+        }
+        // Wave quantisation of the 2-CTA pairs (>= 512 output channels, where the tile shape does not depend
+        // on BN): the pair count / 74 clusters leaves a last partial wave -- e.g. C5's unsplit 14x14 conv5
+        // layers: 448 pairs at BN = 256 = 6.05 waves -> 7.  Half-width N tiles (BN = 128, 896 pairs -> 13
+        // waves of half the work) when that finishes >= 5 % earlier.
+        if (halo && !hn && !tf32 && !pool && cpad % 64 == 0 && BN == 256 && ncols_out % 256 == 0 && ncols_out >= 512) {
+            long mb = 0;
+            for (auto &e : ext)
+                mb += (long)((N + ts.BNn - 1) / ts.BNn) * ((e.first + ts.BH - 1) / ts.BH) * ((e.second + ts.BW - 1) / ts.BW);
+            const long ncl = std::max(1, num_sms() / 2);
+            auto cost = [&](int bn) {
+                const long units = ((mb + 1) / 2) * (long)(ncols_out / bn);
+                return ((units + ncl - 1) / ncl) * (long)bn;
+            };
+            if (cost(128) * 100 <= cost(256) * 95) {
+                BN = 128;
+                nco = ncols_out / 128;
+            }
         }
         static thread_local TcConvParams P;  // large; avoid the stack
         std::memset(&P, 0, sizeof(P));
@@ -1629,23 +1654,28 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
                 cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
                 set[key] = true;
             }
+            // programmatic dependent launch (the kernel waits for its predecessor with griddepcontrol.wait
+            // before any global access): the CTAs are placed and set up while the previous kernel drains
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3((unsigned)grid);
+            cfg.blockDim = dim3(P.dual ? CONV_THREADS : CONV_THREADS - 32);
+            cfg.dynamicSmemBytes = smem;
+            cfg.stream = st;
+            cudaLaunchAttribute at[2];
+            int na = 0;
             if (P.cta2) {
-                cudaLaunchConfig_t cfg = {};
-                cfg.gridDim = dim3((unsigned)grid);
-                cfg.blockDim = dim3(P.dual ? CONV_THREADS : CONV_THREADS - 32);
-                cfg.dynamicSmemBytes = smem;
-                cfg.stream = st;
-                cudaLaunchAttribute at[1];
-                at[0].id = cudaLaunchAttributeClusterDimension;
-                at[0].val.clusterDim.x = 2;
-                at[0].val.clusterDim.y = 1;
-                at[0].val.clusterDim.z = 1;
-                cfg.attrs = at;
-                cfg.numAttrs = 1;
-                cudaLaunchKernelEx(&cfg, kern, P);
-            } else {
-                kern<<<grid, P.dual ? CONV_THREADS : CONV_THREADS - 32, smem, st>>>(P);
+                at[na].id = cudaLaunchAttributeClusterDimension;
+                at[na].val.clusterDim.x = 2;
+                at[na].val.clusterDim.y = 1;
+                at[na].val.clusterDim.z = 1;
+                ++na;
             }
+            at[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            at[na].val.programmaticStreamSerializationAllowed = 1;
+            ++na;
+            cfg.attrs = at;
+            cfg.numAttrs = na;
+            cudaLaunchKernelEx(&cfg, kern, P);
         };
         // kernels holding cta_group::2 instructions must be launched as clusters: separate instantiations
         if (pool) {

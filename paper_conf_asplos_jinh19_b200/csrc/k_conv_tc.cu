@@ -2488,7 +2488,7 @@ WgradCfg wgrad_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, int p0,
     c.ntiles = c.nco_blk * c.ntb;
     int Z = std::max(1, (2 * num_sms() + c.ntiles - 1) / c.ntiles);
     Z = std::min(Z, std::max(1, c.total_boxes / 4));  // >= 4 boxes per split
-    Z = std::min(Z, 128);
+    Z = std::min(Z, 296);   // (a single-tile layer takes one split per SM: a cap of 128 left 20 SMs idle)
     Z = choose_splits(c.total_boxes, c.ntiles, 2.0 * 128 * c.bpt_pad * c.cbox * c.ts.BW * c.ts.BH * c.ts.BNn,
                           (double)g.L.cout * KT * Li.Cpad, Z);
     c.boxes_per_split = (c.total_boxes + Z - 1) / Z;
@@ -2536,7 +2536,7 @@ WgHaloCfg wgrad_halo_cfg(const Level &Li, const Level &Lo, const LayerGeom &g, i
     c.ntiles = c.nco_blk * (c.rpack ? 1 : g.L.kh) * c.nchunk;
     int Z = std::max(1, (2 * num_sms() + c.ntiles - 1) / c.ntiles);
     Z = std::min(Z, std::max(1, c.total_boxes / 4));
-    Z = std::min(Z, 128);
+    Z = std::min(Z, 296);   // (the row-packed 64-channel layers are ONE tile: 148 splits, not 128 -- all SMs)
     Z = choose_splits(c.total_boxes, c.ntiles, 2.0 * 128 * g.L.kw * std::min(64, Li.Cpad) * c.BH * c.BNn * 8,
                           (double)g.L.cout * g.L.kh * g.L.kw * Li.Cpad, Z);
     c.boxes_per_split = (c.total_boxes + Z - 1) / Z;
@@ -2599,7 +2599,7 @@ static int wgrad_zbound(int path, const Level &Li, const LayerGeom &g) {
         const int maxb = std::min(WG_MAXBLK, 256 / cbox);
         ntiles = nco * ((nblocks + maxb - 1) / maxb);
     }
-    return std::max(1, std::min(128, (2 * num_sms() + ntiles - 1) / ntiles));
+    return std::max(1, std::min(296, (2 * num_sms() + ntiles - 1) / ntiles));
 }
 
 size_t wgrad_tc_ws_bytes(const Level &Li, const Level &Lo, const LayerGeom &g) {

@@ -1648,11 +1648,16 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         }
         const int mode_bits = (bias ? 4 : 0) | (relu ? 2 : 0) | (relu_src ? 1 : 0);
         auto launch = [&](auto kern) {
-            static bool set[32] = {false};
-            const int key = mode_bits + (P.cta2 ? 8 : 0) + (tf32 ? 16 : 0);
-            if (!set[key]) {
-                cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-                set[key] = true;
+            // the smem opt-in per kernel POINTER (every instantiation has the same function type, so this
+            // generic lambda is one function: a per-mode key would miss kernels that share a mode)
+            static std::vector<const void *> set;
+            static std::mutex mu;
+            {
+                std::lock_guard<std::mutex> lk(mu);
+                if (std::find(set.begin(), set.end(), (const void *)kern) == set.end()) {
+                    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+                    set.push_back((const void *)kern);
+                }
             }
             // programmatic dependent launch (the kernel waits for its predecessor with griddepcontrol.wait
             // before any global access): the CTAs are placed and set up while the previous kernel drains
@@ -1681,10 +1686,12 @@ splitcnn_status_t launch_tc(int mode, const Level &La, const Level &Lout, const 
         if (pool) {
             const int key = 16 + (bias ? 1 : 0) + (P.cta2 ? 2 : 0);
             auto launch_pool = [&](auto kern) {
-                static bool set[4] = {false};
-                if (!set[key - 16]) {
+                static std::vector<const void *> set;
+                static std::mutex mu;
+                std::lock_guard<std::mutex> lk(mu);
+                if (std::find(set.begin(), set.end(), (const void *)kern) == set.end()) {
                     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-                    set[key - 16] = true;
+                    set.push_back((const void *)kern);
                 }
                 if (P.cta2) {
                     cudaLaunchConfig_t cfg = {};

@@ -1890,10 +1890,25 @@ splitcnn_status_t launch_conv_dgrad_tc(const Level &Li, const Level &Lo, const L
     const int pbh = g.pad_h[0], pbw = g.pad_w[0];
     if (!prepared) prep_dgrad_weights_tc(Li, Lo, g, w, ws, st, 148 * 16);
     const char *wsp = (const char *)(prepared ? w : ws);
+    // phases no tap reaches (k < s, e.g. the 1x1 / stride-2 downsample: 3 of 4) are zero: ONE contiguous
+    // memset of the patch range (the reached phases overwrite their pixels) instead of one strided zero
+    // kernel per phase -- 3 x 11.7 us -> ~17 us for C3's downsample data gradient
+    int nzero = 0;
+    for (int rh = 0; rh < S; ++rh)
+        for (int rw = 0; rw < S; ++rw) {
+            const DgradPhase d = dgrad_phase(g, rh, rw);
+            nzero += (d.nth == 0 || d.ntw == 0) ? 1 : 0;
+        }
+    if (nzero > 1) {
+        const int64_t e0 = Li.offset(p0 / Li.nw(), p0 % Li.nw());
+        const int64_t e1 = p1 >= Li.npatch() ? Li.total() : Li.offset(p1 / Li.nw(), p1 % Li.nw());
+        cudaMemsetAsync((__nv_bfloat16 *)dx + e0, 0, (size_t)(e1 - e0) * 2, st);
+    }
     for (int rh = 0; rh < S; ++rh)
         for (int rw = 0; rw < S; ++rw) {
             const DgradPhase d = dgrad_phase(g, rh, rw);
             if (d.nth == 0 || d.ntw == 0) {
+                if (nzero > 1) continue;   // covered by the memset
                 LevelDesc ld = make_level_desc(Li);
                 dim3 grid((unsigned)std::max(1, std::min(2048, 148 * 8 / std::max(1, p1 - p0))), (unsigned)(p1 - p0));
                 zero_phase_kernel<<<grid, 256, 0, st>>>((__nv_bfloat16 *)dx, ld, S, rh, rw, p0);

@@ -519,17 +519,34 @@ __global__ void __launch_bounds__(256, 4) pool3x3s2_fwd_bf16_kernel(LevelDesc Li
         }
         uint32_t best[4] = {0, 0, 0, 0}, arg[4] = {0, 0, 0, 0};
         bool first = true;
+        if (inb == 0x1FFu) {   // the whole window inside the patch (all but the border rows / columns): no checks
+            const uint32_t *w0v = reinterpret_cast<const uint32_t *>(&v[0]);
 #pragma unroll
-        for (int t = 0; t < 9; ++t) {
-            if (!(inb & (1u << t))) continue;
-            const uint32_t *w = reinterpret_cast<const uint32_t *>(&v[t]);
+            for (int j = 0; j < 4; ++j) best[j] = w0v[j];
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                const uint32_t m = first ? 0xFFFFFFFFu : bf2_gt(w[j], best[j]);
-                best[j] = (w[j] & m) | (best[j] & ~m);
-                arg[j] = ((uint32_t)(t * 0x00010001u) & m) | (arg[j] & ~m);
+            for (int t = 1; t < 9; ++t) {
+                const uint32_t *w = reinterpret_cast<const uint32_t *>(&v[t]);
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const uint32_t m = bf2_gt(w[j], best[j]);
+                    best[j] = (w[j] & m) | (best[j] & ~m);
+                    arg[j] = ((uint32_t)(t * 0x00010001u) & m) | (arg[j] & ~m);
+                }
             }
             first = false;
+        } else {
+#pragma unroll
+            for (int t = 0; t < 9; ++t) {
+                if (!(inb & (1u << t))) continue;
+                const uint32_t *w = reinterpret_cast<const uint32_t *>(&v[t]);
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const uint32_t m = first ? 0xFFFFFFFFu : bf2_gt(w[j], best[j]);
+                    best[j] = (w[j] & m) | (best[j] & ~m);
+                    arg[j] = ((uint32_t)(t * 0x00010001u) & m) | (arg[j] & ~m);
+                }
+                first = false;
+            }
         }
         const int64_t o = go.off + (((int64_t)n * go.hp + oh) * go.wp + ow) * Lo.Cpad + cg * 8;
         if (first) {   // no in-bounds position: impossible for a valid plan (pads < k); -inf
@@ -537,17 +554,12 @@ __global__ void __launch_bounds__(256, 4) pool3x3s2_fwd_bf16_kernel(LevelDesc Li
             best[0] = best[1] = best[2] = best[3] = ninf;
         }
         *reinterpret_cast<uint4 *>(Y + o) = make_uint4(best[0], best[1], best[2], best[3]);
-        uint32_t lo = 0, hi = 0;
+        // argmax byte = window index (bits 0-3, already in bytes 0 / 2 of each arg word) | [max > 0] << 7 (the
+        // packed bf16 compare is exactly bf2_pos_byte's test); two words' bytes 0 / 2 interleaved by one PRMT
+        uint32_t bw[4];
 #pragma unroll
-        for (int j = 0; j < 4; ++j)
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                const int k = 2 * j + h;
-                uint32_t b = (arg[j] >> (16 * h)) & 0xFu;
-                if (relu_bit) b |= bf2_pos_byte(best[j], h);
-                if (k < 4) lo |= b << (8 * k); else hi |= b << (8 * (k - 4));
-            }
-        *reinterpret_cast<uint2 *>(A + o) = make_uint2(lo, hi);
+        for (int j = 0; j < 4; ++j) bw[j] = arg[j] | (relu_bit ? (bf2_gt(best[j], 0u) & 0x00800080u) : 0u);
+        *reinterpret_cast<uint2 *>(A + o) = make_uint2(__byte_perm(bw[0], bw[1], 0x6420), __byte_perm(bw[2], bw[3], 0x6420));
     }
 }
 

@@ -437,10 +437,6 @@ __global__ void __launch_bounds__(256, 4) pool_bwd_k3s2_kernel(LevelDesc Li, Lev
 __device__ __forceinline__ uint32_t bf2_gt(uint32_t a, uint32_t b) {
     return __hgt2_mask(*reinterpret_cast<const __nv_bfloat162 *>(&a), *reinterpret_cast<const __nv_bfloat162 *>(&b));
 }
-__device__ __forceinline__ uint32_t bf2_pos_byte(uint32_t w, int half) {   // [element > 0] of one bf16
-    const uint32_t h = (w >> (16 * half)) & 0xFFFFu;
-    return ((h & 0x8000u) == 0u && (h & 0x7FFFu) != 0u && (h & 0x7FFFu) <= 0x7F80u) ? 0x80u : 0u;
-}
 
 __global__ void __launch_bounds__(256) pool2x2_fwd_bf16_kernel(LevelDesc Li, LevelDesc Lo, const __nv_bfloat16 *__restrict__ X,
                                                                __nv_bfloat16 *__restrict__ Y, uint8_t *__restrict__ A,
@@ -476,17 +472,11 @@ __global__ void __launch_bounds__(256) pool2x2_fwd_bf16_kernel(LevelDesc Li, Lev
         }
         const int64_t o = go.off + (((int64_t)n * go.hp + oh) * go.wp + ow) * Lo.Cpad + cg * 8;
         *reinterpret_cast<uint4 *>(Y + o) = make_uint4(best[0], best[1], best[2], best[3]);
-        uint32_t lo = 0, hi = 0;
+        // argmax bytes as in the 3x3 kernel: window index in bytes 0 / 2 of each arg word | [max > 0] << 7, one PRMT
+        uint32_t bw[4];
 #pragma unroll
-        for (int j = 0; j < 4; ++j)
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                const int k = 2 * j + h;
-                uint32_t b = (arg[j] >> (16 * h)) & 0x3u;
-                if (relu_bit) b |= bf2_pos_byte(best[j], h);
-                if (k < 4) lo |= b << (8 * k); else hi |= b << (8 * (k - 4));
-            }
-        *reinterpret_cast<uint2 *>(A + o) = make_uint2(lo, hi);
+        for (int j = 0; j < 4; ++j) bw[j] = arg[j] | (relu_bit ? (bf2_gt(best[j], 0u) & 0x00800080u) : 0u);
+        *reinterpret_cast<uint2 *>(A + o) = make_uint2(__byte_perm(bw[0], bw[1], 0x6420), __byte_perm(bw[2], bw[3], 0x6420));
     }
 }
 
@@ -555,7 +545,7 @@ __global__ void __launch_bounds__(256, 4) pool3x3s2_fwd_bf16_kernel(LevelDesc Li
         }
         *reinterpret_cast<uint4 *>(Y + o) = make_uint4(best[0], best[1], best[2], best[3]);
         // argmax byte = window index (bits 0-3, already in bytes 0 / 2 of each arg word) | [max > 0] << 7 (the
-        // packed bf16 compare is exactly bf2_pos_byte's test); two words' bytes 0 / 2 interleaved by one PRMT
+        // packed bf16 compare with +0: false for NaN, zero and negatives); two words' bytes 0 / 2 by one PRMT
         uint32_t bw[4];
 #pragma unroll
         for (int j = 0; j < 4; ++j) bw[j] = arg[j] | (relu_bit ? (bf2_gt(best[j], 0u) & 0x00800080u) : 0u);

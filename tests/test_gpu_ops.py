@@ -192,6 +192,34 @@ def test_conv_patch_range_sharding(sc):
     torch.testing.assert_close(dwa + dwb, dw, rtol=1e-5, atol=1e-5 * dw.abs().max().item())
 
 
+@pytest.mark.parametrize("k,pad", [(1, 0), (3, 1)])
+def test_strided_dgrad_patch_ranges(sc, k, pad):
+    """Stride-2 data gradient over patch ranges: [0, q) + [q, P) equal one call bit for bit, and a range call
+    writes exactly its own patches (the phases no tap reaches are zeroed by one memset of the range, k < s;
+    the other patches keep a sentinel)."""
+    dtype = sc.BF16
+    layers = [synth.conv(64, 128, k, 2, pad)]
+    ref, pl = _make(sc, layers, 2, 64, 32, 32, 2, 2, seed=11)
+    lv0, lv1 = pl.levels
+    g = synth.rng(11)
+    dy = _dev(sc, pack_level(_round(synth.normal(g, (2, 128, ref.layers[0].H_out, ref.layers[0].W_out)), dtype, sc), lv1),
+              dtype)
+    w = _dev(sc, w_oihw_to_lib(_round(synth.kaiming(g, 128, 64, k, k), dtype, sc), lv0["Cpad"]), dtype)
+    ws_b = pl.workspace_size(0, dtype, 1)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    dx1 = torch.full((lv0["total_elems"],), 7.0, dtype=torch.bfloat16, device="cuda")
+    dx2 = torch.full_like(dx1, 7.0)
+    sc.splitcnn_conv_bwd_data(pl.handle, 0, dtype, dy, w, dx1, None, ws, ws_b)
+    assert not torch.any(dx1 == 7.0), "every dX element is written"
+    sc.splitcnn_conv_bwd_data(pl.handle, 0, dtype, dy, w, dx2, None, ws, ws_b, 0, 0, 1)
+    host = _host(dx2)
+    blocks = unpack_level(host, lv0, keep_pad=True)
+    assert np.all(blocks[0][1] == 7.0) and np.all(blocks[1][0] == 7.0) and np.all(blocks[1][1] == 7.0), \
+        "a range call leaves the other patches alone"
+    sc.splitcnn_conv_bwd_data(pl.handle, 0, dtype, dy, w, dx2, None, ws, ws_b, 0, 1, 4)
+    assert torch.equal(dx1, dx2)
+
+
 # --------------------------------------------------------------------------- split / merge
 @pytest.mark.parametrize("dtype_name", ["bf16", "fp32"])
 def test_split_merge_bit_exact(sc, dtype_name):
